@@ -1,0 +1,145 @@
+"""Pins for the oracle's sigmoid fit, coupling and whole pipeline (CPU, -m "not gpu")."""
+import json
+import os
+
+import numpy as np
+import pytest
+from scipy.optimize import minimize
+
+import datagen
+import oracle
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+# ----------------------------------------------------------------------------- sigmoid (Eq 12-13)
+def _F(ab, v, t):
+    # Eq 13 written as a minimisation of the negative log likelihood, P = 1/(1+exp(Av+B)).
+    z = ab[0] * v + ab[1]
+    logP = -np.logaddexp(0.0, z)       # log 1/(1+e^z)
+    log1mP = z - np.logaddexp(0.0, z)  # log e^z/(1+e^z)
+    return -(t * logP + (1 - t) * log1mP).sum()
+
+
+def _targets(y):
+    Np, Nm = (y > 0).sum(), (y < 0).sum()
+    return np.where(y > 0, (Np + 1.0) / (Np + 2.0), 1.0 / (Nm + 2.0))
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_sigmoid_fit_matches_bfgs_and_zero_gradient(seed):
+    rng = np.random.default_rng(seed)
+    n = 500
+    y = np.where(rng.random(n) < 0.4, 1, -1).astype(np.int32)
+    v = y * rng.gamma(2.0, 0.7, size=n) + rng.normal(0, 0.8, size=n)
+    A, B, it, st = oracle.sigmoid_fit(v, y)
+    assert st == 0
+    t = _targets(y)
+    res = minimize(_F, x0=np.array([0.0, 0.0]), args=(v, t), method="BFGS", options=dict(gtol=1e-11))
+    np.testing.assert_allclose([A, B], res.x, atol=1e-6)
+    # gradient of Eq 13 (L254-L255): sum v (t - P), sum (t - P) vanish at the optimum
+    P = 1.0 / (1.0 + np.exp(A * v + B))
+    assert abs((v * (t - P)).sum()) < 1e-5 and abs((t - P).sum()) < 1e-5
+
+
+def test_sigmoid_constant_decision_values_closed_form():
+    # v = 0 for all instances: only B matters, optimum P = mean(t) => B = log((1 - tbar)/tbar)
+    y = np.array([1] * 30 + [-1] * 70, dtype=np.int32)
+    v = np.zeros(100)
+    A, B, _, st = oracle.sigmoid_fit(v, y)
+    tbar = _targets(y).mean()
+    assert A == 0.0
+    np.testing.assert_allclose(B, np.log((1 - tbar) / tbar), atol=1e-9)
+
+
+# ----------------------------------------------------------------------------- coupling (Eq 14-15)
+def _rmat(k, rng, lo=0.05, hi=0.95):
+    r = np.zeros((k, k))
+    for s in range(k):
+        for t in range(s + 1, k):
+            r[s, t] = rng.uniform(lo, hi)
+            r[t, s] = 1.0 - r[s, t]
+    return r
+
+
+def _Q(r):
+    k = r.shape[0]
+    Q = -r * r.T
+    for s in range(k):
+        Q[s, s] = sum(r[u, s] ** 2 for u in range(k) if u != s)
+    return Q
+
+
+def test_couple_k2_closed_form():
+    for r12 in [0.01, 0.3, 0.5, 0.77, 0.999]:
+        r = np.array([[0.0, r12], [1 - r12, 0.0]])
+        np.testing.assert_allclose(oracle.couple(r), [r12, 1 - r12], atol=1e-14)
+
+
+@pytest.mark.parametrize("k", [3, 5, 10, 26])
+def test_couple_bradley_terry_consistent(k):
+    rng = np.random.default_rng(k)
+    p_star = rng.dirichlet(np.ones(k))
+    r = p_star[:, None] / (p_star[:, None] + p_star[None, :])
+    np.fill_diagonal(r, 0.0)
+    np.testing.assert_allclose(oracle.couple(r), p_star, atol=1e-12)
+
+
+@pytest.mark.parametrize("k", [3, 4, 10, 26])
+def test_couple_eq15_inverse_and_direct_minimisation(k):
+    rng = np.random.default_rng(100 + k)
+    for _ in range(5):
+        r = _rmat(k, rng)
+        p = oracle.couple(r)
+        assert abs(p.sum() - 1.0) < 1e-12 and np.all(p >= 0)
+        Q = _Q(r)
+        qe = np.linalg.solve(Q, np.ones(k))  # Eq 15: p = Q^-1 e / (e^T Q^-1 e)
+        np.testing.assert_allclose(p, qe / qe.sum(), atol=1e-10)
+        # Eq 14 objective as printed (double sum), minimised under sum p = 1
+        def obj(q):
+            return sum((r[t, s] * q[s] - r[s, t] * q[t]) ** 2 for s in range(k) for t in range(k) if t != s)
+        res = minimize(obj, np.full(k, 1.0 / k), method="SLSQP",
+                       constraints=[dict(type="eq", fun=lambda q: q.sum() - 1.0)],
+                       options=dict(ftol=1e-15, maxiter=500))
+        np.testing.assert_allclose(p, res.x, atol=2e-5)
+        assert obj(p) <= obj(res.x) + 1e-12
+
+
+def test_couple_example1_ordering():
+    g = json.load(open(os.path.join(GOLDEN, "example1_coupling.json")))
+    r = np.zeros((3, 3))
+    r[0, 1], r[0, 2], r[1, 2] = g["r12"], g["r13"], g["r23"]
+    r[1, 0], r[2, 0], r[2, 1] = 1 - g["r12"], 1 - g["r13"], 1 - g["r23"]
+    p = oracle.couple(r)
+    printed = np.array(g["printed_p"])
+    # only the ordering of the printed result is reproducible
+    assert list(np.argsort(-p)) == list(np.argsort(-printed))
+    assert np.argmax(p) == 0
+
+
+# ----------------------------------------------------------------------------- pipeline
+def test_pipeline_in_sample_identity_and_sklearn():
+    spec, X, y, Xt, yt = datagen.make_config("blobs")
+    m = oracle.train(X, y, spec.k, spec.C, spec.gamma, 1e-10)
+    assert np.all(m["status"] == 0)
+    # Eq 11 on the training instances == f + y - rho from Eq 3 (two different code paths)
+    dec, prob = oracle.predict(m, X, y, X)
+    for p, (s, t) in enumerate(m["pairs"]):
+        idx, ypm = oracle.pair_members(y, spec.k, s, t)
+        v = m["f"][p] + ypm + m["b"][p]
+        np.testing.assert_allclose(dec[idx, p], v, atol=1e-10)
+    np.testing.assert_allclose(prob.sum(1), 1.0, atol=1e-12)
+    assert np.all(prob >= 0)
+    sk = pytest.importorskip("sklearn.svm")
+    for p, (s, t) in enumerate(m["pairs"]):
+        idx, ypm = oracle.pair_members(y, spec.k, s, t)
+        clf = sk.SVC(C=spec.C, kernel="rbf", gamma=spec.gamma, tol=1e-10, shrinking=False).fit(
+            X[idx].astype(np.float64), ypm)
+        a_sk = np.zeros(len(idx))
+        a_sk[clf.support_] = np.abs(clf.dual_coef_[0])
+        np.testing.assert_allclose(m["alpha"][p], a_sk, atol=1e-6 * spec.C)
+        sign = np.sign(clf.dual_coef_[0][0] * ypm[clf.support_[0]])
+        np.testing.assert_allclose(sign * clf.intercept_[0], m["b"][p], atol=1e-6)
+    # Table-4 pattern (L423-L436): errors of the probabilistic classifier are sane
+    test_err = (prob_t := oracle.predict(m, X, y, Xt, want_dec=False)[1]).argmax(1) != yt
+    assert test_err.mean() < 0.2
