@@ -1,0 +1,60 @@
+// common.cuh -- shared internals of libgmpsvm (CUDA path only; never included by oracle/).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <stdexcept>
+#include <string>
+
+#include "gmpsvm.h"
+
+namespace gmpsvm {
+
+// Error carried through the engine and converted to a status code at the ABI boundary.
+struct Error : std::runtime_error {
+  int code;
+  Error(int c, const std::string& m) : std::runtime_error(m), code(c) {}
+};
+
+[[noreturn]] void throw_cuda(cudaError_t e, const char* what, const char* file, int line);
+
+#define GM_CUDA(call)                                                      \
+  do {                                                                     \
+    cudaError_t e_ = (call);                                               \
+    if (e_ != cudaSuccess) ::gmpsvm::throw_cuda(e_, #call, __FILE__, __LINE__); \
+  } while (0)
+
+#define GM_CHECK_LAUNCH() GM_CUDA(cudaGetLastError())
+
+extern std::atomic<uint64_t> g_launches;  // kernels launched by this library
+
+// Every kernel launch goes through this macro so gmpsvm_launch_count() is exact.
+#define GM_LAUNCH(kernel, grid, block, smem, stream, ...)                  \
+  do {                                                                     \
+    kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);            \
+    ::gmpsvm::g_launches.fetch_add(1, std::memory_order_relaxed);          \
+    GM_CHECK_LAUNCH();                                                     \
+  } while (0)
+
+inline int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+constexpr int kTile = 128;  // GEMM tile edge (rows and columns)
+constexpr int kBK = 16;     // GEMM k-step; feature dimension is padded to a multiple of it
+constexpr double kTau = 1e-12;  // eta floor (reading R3)
+
+// Pair descriptor (device and host): pair p = (s, t), class-sorted layout.
+struct PairDesc {
+  int32_t s, t;        // classes, s < t; s is the +1 side
+  int32_t n_s, n_t;    // class sizes
+  int64_t off_s, off_t;  // first sorted position of class s / t
+  int64_t a_off;       // offset of this pair in the concatenated alpha/f arrays
+  int32_t pid;         // global pair index
+  int32_t pad;
+};
+
+__host__ __device__ inline int pair_index(int s, int t, int k) { return s * k - s * (s + 1) / 2 + (t - s - 1); }
+
+}  // namespace gmpsvm

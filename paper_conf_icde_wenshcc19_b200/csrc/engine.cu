@@ -1,0 +1,677 @@
+// engine.cu -- host orchestration of the hot path (Algorithm 2, and the
+// prediction procedure L259-L273 / L331-L363) on one GPU.  Every arithmetic step runs in the
+// kernels of stage.cu / krow.cu / solver.cu / predict.cu; this file allocates, launches,
+// polls the per-pair stop flags once per outer iteration, and assembles the model.
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "model.h"
+
+namespace gmpsvm {
+
+std::atomic<uint64_t> g_launches{0};
+
+[[noreturn]] void throw_cuda(cudaError_t e, const char* what, const char* file, int line) {
+  std::string msg = std::string("CUDA error ") + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ") at " + file +
+                    ":" + std::to_string(line) + ": " + what;
+  if (e == cudaErrorMemoryAllocation) throw Error(GMPSVM_ENOMEM, msg);
+  throw Error(GMPSVM_ECUDA, msg);
+}
+
+namespace {
+
+constexpr int kMaxK = 64;          // label-rank shared memory bound
+constexpr int kMaxCoupleK = 40;    // coupling shared memory bound
+constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
+constexpr int64_t kPredictChunk = 32768;
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    GM_CUDA(cudaGetDevice(&prev));
+    if (dev != prev) GM_CUDA(cudaSetDevice(dev));
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+std::mutex g_stream_mu;
+cudaStream_t g_streams[64] = {};
+bool g_pool_cfg[64] = {};
+
+cudaStream_t get_stream(const gmpsvm_options& opt) {
+  int dev = opt.device;
+  std::lock_guard<std::mutex> lk(g_stream_mu);
+  if (dev >= 0 && dev < 64 && !g_pool_cfg[dev]) {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    g_pool_cfg[dev] = true;
+  }
+  if (opt.stream) return (cudaStream_t)opt.stream;
+  if (dev < 0 || dev >= 64) throw Error(GMPSVM_EINVAL, "device ordinal out of range");
+  if (!g_streams[dev]) GM_CUDA(cudaStreamCreateWithFlags(&g_streams[dev], cudaStreamNonBlocking));
+  return g_streams[dev];
+}
+
+template <class T>
+struct DevBuf {
+  T* p = nullptr;
+  cudaStream_t st = nullptr;
+  DevBuf() = default;
+  DevBuf(size_t count, cudaStream_t s) : st(s) {
+    if (count) GM_CUDA(cudaMallocAsync((void**)&p, count * sizeof(T), s));
+  }
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  ~DevBuf() {
+    if (p) cudaFreeAsync(p, st);
+  }
+  T* get() const { return p; }
+};
+
+template <class T>
+struct PinnedBuf {
+  T* p = nullptr;
+  explicit PinnedBuf(size_t count) {
+    if (count) GM_CUDA(cudaMallocHost((void**)&p, count * sizeof(T)));
+  }
+  ~PinnedBuf() {
+    if (p) cudaFreeHost(p);
+  }
+};
+
+template <class T>
+T* dev_alloc(size_t count) {
+  T* p = nullptr;
+  if (count) GM_CUDA(cudaMalloc((void**)&p, count * sizeof(T)));
+  return p;
+}
+
+enum { PH_STAGE, PH_KERNEL, PH_SELECT, PH_SUB, PH_FUP, PH_FIN, PH_DEC, PH_COUPLE, PH_D2H, PH_N };
+
+struct PhaseTimer {
+  cudaStream_t st;
+  std::vector<cudaEvent_t> evs[PH_N];
+  explicit PhaseTimer(cudaStream_t s) : st(s) {}
+  void mark(int ph) {
+    cudaEvent_t e;
+    GM_CUDA(cudaEventCreate(&e));
+    GM_CUDA(cudaEventRecord(e, st));
+    evs[ph].push_back(e);
+  }
+  double ms(int ph) {
+    double t = 0.0;
+    for (size_t i = 0; i + 1 < evs[ph].size(); i += 2) {
+      float x = 0.f;
+      GM_CUDA(cudaEventElapsedTime(&x, evs[ph][i], evs[ph][i + 1]));
+      t += x;
+    }
+    return t;
+  }
+  ~PhaseTimer() {
+    for (auto& v : evs)
+      for (auto e : v) cudaEventDestroy(e);
+  }
+};
+
+double host_ms_since(std::chrono::steady_clock::time_point t0) {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+bool finite_pos(double v) { return std::isfinite(v) && v > 0.0; }
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------
+DevModel::~DevModel() {
+  int prev = -1;
+  cudaGetDevice(&prev);
+  if (device >= 0) cudaSetDevice(device);
+  cudaFree(SvT);
+  cudaFree(nsv);
+  cudaFree(coef);
+  cudaFree(items);
+  cudaFree(item_begin);
+  cudaFree(item_end);
+  cudaFree(b);
+  cudaFree(A);
+  cudaFree(B);
+  if (prev >= 0) cudaSetDevice(prev);
+}
+
+std::vector<int64_t> Model::class_off() const {
+  std::vector<int64_t> off(k + 1, 0);
+  for (int c = 0; c < k; ++c) off[c + 1] = off[c] + class_count[c];
+  return off;
+}
+
+std::vector<int64_t> Model::pair_offsets() const {
+  std::vector<int64_t> po(P() + 1, 0);
+  int p = 0;
+  for (int s = 0; s < k; ++s)
+    for (int t = s + 1; t < k; ++t, ++p) po[p + 1] = po[p] + class_count[s] + class_count[t];
+  return po;
+}
+
+int Model::n_trained() const {
+  int c = 0;
+  for (auto t : trained) c += t ? 1 : 0;
+  return c;
+}
+
+gmpsvm_predict_stats& tls_predict_stats() {
+  static thread_local gmpsvm_predict_stats s{};
+  return s;
+}
+
+// Build the device prediction structures from SV rows already on the device.
+// rows: device pointer to rows (stride d); row_of_sv[i] = row of SV i (SV order = sv_pos order).
+static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* rows, const std::vector<int64_t>& row_of_sv,
+                                                 int device, cudaStream_t st) {
+  auto dm = std::make_unique<DevModel>();
+  dm->device = device;
+  const int k = m.k, P = m.P();
+  dm->km1 = k - 1;
+  dm->km1_pad = (int)round_up(k - 1, 4);
+  dm->d_pad = (int)round_up(m.d, kBK);
+  const auto off = m.class_off();
+  const auto po = m.pair_offsets();
+  const int64_t nsv = (int64_t)m.sv_pos.size();
+  // per-class SV ranges (sv_pos ascending => class order)
+  std::vector<int64_t> sv_cls_begin(k + 1, 0);
+  {
+    int64_t i = 0;
+    for (int c = 0; c < k; ++c) {
+      sv_cls_begin[c] = i;
+      while (i < nsv && m.sv_pos[i] < off[c + 1]) ++i;
+    }
+    sv_cls_begin[k] = nsv;
+  }
+  std::vector<int64_t> slot_begin(k + 1, 0);
+  for (int c = 0; c < k; ++c)
+    slot_begin[c + 1] = slot_begin[c] + round_up(sv_cls_begin[c + 1] - sv_cls_begin[c], kTile);
+  dm->nsv_pad = std::max<int64_t>(slot_begin[k], kTile);
+  dm->slot_sv.assign(dm->nsv_pad, -1);
+  std::vector<int64_t> slot_src(dm->nsv_pad, -1);
+  std::vector<float> coef((size_t)dm->nsv_pad * dm->km1_pad, 0.f);
+  std::vector<DecItem> items;
+  std::vector<int32_t> ib(k, 0), ie(k, 0);
+  for (int c = 0; c < k; ++c) {
+    for (int64_t i = sv_cls_begin[c]; i < sv_cls_begin[c + 1]; ++i) {
+      const int64_t slot = slot_begin[c] + (i - sv_cls_begin[c]);
+      dm->slot_sv[slot] = i;
+      slot_src[slot] = row_of_sv[i];
+      const int64_t g = m.sv_pos[i];
+      for (int u = 0; u < k; ++u) {
+        if (u == c) continue;
+        const int s = std::min(c, u), t = std::max(c, u);
+        const int p = pair_index(s, t, k);
+        const int64_t j = (c == s) ? (g - off[s]) : (m.class_count[s] + (g - off[t]));
+        const double a = m.alpha[po[p] + j];
+        const int col = u < c ? u : u - 1;
+        coef[(size_t)slot * dm->km1_pad + col] = (float)((c == s) ? a : -a);
+      }
+    }
+    ib[c] = (int32_t)items.size();
+    const int t0 = (int)(slot_begin[c] / kTile), t1 = (int)(slot_begin[c + 1] / kTile);
+    for (int t = t0; t < t1; t += kItemTiles) items.push_back(DecItem{c, t, std::min(t1, t + kItemTiles), 0});
+    ie[c] = (int32_t)items.size();
+  }
+  if (items.empty()) items.push_back(DecItem{0, 0, 0, 0});  // no SV at all: zero contribution
+  dm->n_items = (int)items.size();
+  dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad);
+  dm->nsv = dev_alloc<float>(dm->nsv_pad);
+  dm->coef = dev_alloc<float>(coef.size());
+  dm->items = dev_alloc<DecItem>(items.size());
+  dm->item_begin = dev_alloc<int32_t>(k);
+  dm->item_end = dev_alloc<int32_t>(k);
+  dm->b = dev_alloc<double>(P);
+  dm->A = dev_alloc<double>(P);
+  dm->B = dev_alloc<double>(P);
+  DevBuf<int64_t> d_src(slot_src.size(), st);
+  GM_CUDA(cudaMemcpyAsync(d_src.get(), slot_src.data(), slot_src.size() * 8, cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->coef, coef.data(), coef.size() * 4, cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->items, items.data(), items.size() * sizeof(DecItem), cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->item_begin, ib.data(), k * 4, cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->item_end, ie.data(), k * 4, cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->b, m.b.data(), P * 8, cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->A, m.A.data(), P * 8, cudaMemcpyHostToDevice, st));
+  GM_CUDA(cudaMemcpyAsync(dm->B, m.B.data(), P * 8, cudaMemcpyHostToDevice, st));
+  launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
+                        nullptr, st);
+  GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
+  return dm;
+}
+
+void ensure_host_sv(const Model& mdl) {
+  Model& m = const_cast<Model&>(mdl);
+  if (m.sv_X_ready) return;
+  const int64_t nsv = (int64_t)m.sv_pos.size();
+  m.sv_X.assign((size_t)nsv * m.d, 0.f);
+  if (nsv > 0) {
+    if (!m.dev) throw Error(GMPSVM_EINVAL, "model has no SV rows on host or device");
+    DeviceGuard dg(m.dev->device);
+    std::vector<float> t((size_t)m.dev->d_pad * m.dev->nsv_pad);
+    GM_CUDA(cudaMemcpy(t.data(), m.dev->SvT, t.size() * 4, cudaMemcpyDeviceToHost));
+    for (int64_t slot = 0; slot < m.dev->nsv_pad; ++slot) {
+      const int64_t i = m.dev->slot_sv[slot];
+      if (i < 0) continue;
+      for (int c = 0; c < m.d; ++c) m.sv_X[(size_t)i * m.d + c] = t[(size_t)c * m.dev->nsv_pad + slot];
+    }
+  }
+  m.sv_X_ready = true;
+}
+
+// ------------------------------------------------------------------------------------------
+int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma, double eps,
+                 const gmpsvm_options& opt, Model** out) {
+  const auto t_start = std::chrono::steady_clock::now();
+  if (!X || !y || !out) throw Error(GMPSVM_EINVAL, "null argument");
+  if (n < 2 || d < 1 || k < 2) throw Error(GMPSVM_EINVAL, "need n >= 2, d >= 1, k >= 2");
+  if (k > kMaxK) throw Error(GMPSVM_ENOTIMPL, "k > 64 classes not supported by this build");
+  if (n >= (int64_t)1 << 31) throw Error(GMPSVM_ENOTIMPL, "n >= 2^31 not supported");
+  if (!finite_pos(C) || !finite_pos(gamma) || !finite_pos(eps)) throw Error(GMPSVM_EINVAL, "C, gamma, eps must be finite and > 0");
+  int B = opt.ws_size ? opt.ws_size : 1024;
+  if (B < 2 || B > 1024 || (B & 1)) throw Error(GMPSVM_EINVAL, "ws_size must be even and in [2, 1024]");
+  int q = opt.q ? opt.q : B / 2;
+  if (q < 2 || q > B) throw Error(GMPSVM_EINVAL, "q must be in [2, ws_size]");
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  const uint64_t launches0 = g_launches.load();
+  PhaseTimer tm(st);
+
+  // ---------------- a1 staging
+  tm.mark(PH_STAGE);
+  DevBuf<float> bufX(opt.inputs_on_device ? 0 : (size_t)n * d, st);
+  DevBuf<int32_t> bufY(opt.inputs_on_device ? 0 : (size_t)n, st);
+  const float* dX = X;
+  const int32_t* dy = y;
+  if (!opt.inputs_on_device) {
+    GM_CUDA(cudaMemcpyAsync(bufX.get(), X, (size_t)n * d * 4, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(bufY.get(), y, (size_t)n * 4, cudaMemcpyHostToDevice, st));
+    dX = bufX.get();
+    dy = bufY.get();
+  }
+  const int nb = (int)ceil_div(n, 1024);
+  DevBuf<int32_t> blk_counts((size_t)nb * (k + 1), st), blk_off((size_t)nb * k, st);
+  DevBuf<int64_t> d_count(k + 1, st), d_off(k + 1, st), d_perm(n, st);
+  launch_class_sort(dy, n, k, blk_counts.get(), blk_off.get(), d_count.get(), d_off.get(), st);
+  std::vector<int64_t> cc(k + 1);
+  GM_CUDA(cudaMemcpyAsync(cc.data(), d_count.get(), (k + 1) * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  if (cc[k] != 0) throw Error(GMPSVM_EINVAL, "labels must be in [0, k)");
+  for (int c = 0; c < k; ++c)
+    if (cc[c] == 0) throw Error(GMPSVM_EINVAL, "every class must have at least one instance");
+  launch_class_rank(dy, n, k, blk_off.get(), d_off.get(), d_perm.get(), st);
+  const int d_pad = (int)round_up(d, kBK);
+  const int64_t n_pad = round_up(n, kTile);
+  DevBuf<float> XT((size_t)d_pad * n_pad, st), norms(n_pad, st);
+  DevBuf<int32_t> bad(1, st);
+  GM_CUDA(cudaMemsetAsync(bad.get(), 0, 4, st));
+  launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
+  int32_t hbad = 0;
+  GM_CUDA(cudaMemcpyAsync(&hbad, bad.get(), 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  if (hbad) throw Error(GMPSVM_EINVAL, "X contains non-finite values");
+  tm.mark(PH_STAGE);
+
+  // ---------------- pairs to train
+  const int P = k * (k - 1) / 2;
+  std::vector<int> pids;
+  if (opt.pair_ids && opt.n_pair_ids > 0) {
+    std::vector<uint8_t> seen(P, 0);
+    for (int i = 0; i < opt.n_pair_ids; ++i) {
+      const int p = opt.pair_ids[i];
+      if (p < 0 || p >= P || seen[p]) throw Error(GMPSVM_EINVAL, "pair_ids out of range or repeated");
+      seen[p] = 1;
+      pids.push_back(p);
+    }
+  } else {
+    for (int p = 0; p < P; ++p) pids.push_back(p);
+  }
+  const int Pl = (int)pids.size();
+  std::vector<int64_t> coff(k + 1, 0);
+  for (int c = 0; c < k; ++c) coff[c + 1] = coff[c] + cc[c];
+  std::vector<int> ps(P), pt(P);
+  for (int s = 0; s < k; ++s)
+    for (int t = s + 1; t < k; ++t) {
+      ps[pair_index(s, t, k)] = s;
+      pt[pair_index(s, t, k)] = t;
+    }
+  std::vector<PairDesc> hp(Pl);
+  int64_t tot = 0, np_max = 0;
+  for (int i = 0; i < Pl; ++i) {
+    const int p = pids[i];
+    PairDesc& x = hp[i];
+    x.s = ps[p];
+    x.t = pt[p];
+    x.n_s = (int32_t)cc[x.s];
+    x.n_t = (int32_t)cc[x.t];
+    x.off_s = coff[x.s];
+    x.off_t = coff[x.t];
+    x.a_off = tot;
+    x.pid = p;
+    x.pad = 0;
+    tot += x.n_s + x.n_t;
+    np_max = std::max<int64_t>(np_max, x.n_s + x.n_t);
+  }
+
+  // ---------------- a2 kernel values: FULL_K regime (the whole class-sorted matrix)
+  const int64_t ldk = round_up(n, 4);
+  const double bytes_K = (double)n * ldk * 4.0;
+  size_t free_b = 0, total_b = 0;
+  GM_CUDA(cudaMemGetInfo(&free_b, &total_b));
+  const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)free_b;
+  if (bytes_K > budget)
+    throw Error(GMPSVM_ENOTIMPL, "kernel matrix (" + std::to_string(bytes_K / 1e9) +
+                                     " GB) exceeds the cache budget; the ROW_CACHE regime is not in this build");
+  DevBuf<float> K((size_t)n * ldk, st);
+  tm.mark(PH_KERNEL);
+  launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
+  tm.mark(PH_KERNEL);
+
+  // ---------------- a4-a6 batched working-set solver, all pairs concurrently
+  const int Bw = B;
+  DevBuf<PairDesc> d_pairs(Pl, st);
+  GM_CUDA(cudaMemcpyAsync(d_pairs.get(), hp.data(), Pl * sizeof(PairDesc), cudaMemcpyHostToDevice, st));
+  DevBuf<double> d_alpha(tot, st), d_f(tot, st), d_v(tot, st), d_dcoef((size_t)Pl * Bw, st), d_gap(Pl, st),
+      d_b(Pl, st), d_A(Pl, st), d_B(Pl, st);
+  DevBuf<uint32_t> d_stamp(tot, st);
+  DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
+      d_outer(Pl, st), d_sig(Pl, st);
+  DevBuf<int64_t> d_inner(Pl, st);
+  DevBuf<float> d_Kws((size_t)Pl * Bw * Bw, st);
+  SolverArgs a{};
+  a.pairs = d_pairs.get();
+  a.K = K.get();
+  a.ldk = ldk;
+  a.alpha = d_alpha.get();
+  a.f = d_f.get();
+  a.v = d_v.get();
+  a.stamp = d_stamp.get();
+  a.ws = d_ws.get();
+  a.ws_n = d_wsn.get();
+  a.ws_tmp = d_wst.get();
+  a.Kws = d_Kws.get();
+  a.dcoef = d_dcoef.get();
+  a.status = d_status.get();
+  a.gap = d_gap.get();
+  a.inner_iters = d_inner.get();
+  a.outer_iters = d_outer.get();
+  a.b = d_b.get();
+  a.A = d_A.get();
+  a.Bs = d_B.get();
+  a.sig_status = d_sig.get();
+  a.B = Bw;
+  a.q = q;
+  a.inner_cap = opt.inner_iter_cap > 0 ? opt.inner_iter_cap : 100 * Bw;
+  a.C = C;
+  a.eps = eps;
+  launch_init_pairs(a, Pl, tot, st);
+  const int64_t max_outer = opt.max_outer_iter > 0 ? opt.max_outer_iter : 1000000;
+  PinnedBuf<int32_t> h_status(Pl);
+  bool cap_hit = false;
+  for (int64_t outer = 0;; ++outer) {
+    tm.mark(PH_SELECT);
+    launch_select_ws(a, Pl, (uint32_t)(outer + 1), outer == 0 ? 1 : 0, st);
+    tm.mark(PH_SELECT);
+    GM_CUDA(cudaMemcpyAsync(h_status.p, d_status.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaStreamSynchronize(st));
+    int active = 0;
+    for (int i = 0; i < Pl; ++i) active += h_status.p[i] == 0;
+    if (active == 0) break;
+    if (outer >= max_outer) {
+      cap_hit = true;
+      break;
+    }
+    tm.mark(PH_SUB);
+    launch_gather_kws(a, Pl, outer == 0 ? 1 : 0, st);
+    launch_local_smo(a, Pl, st);
+    tm.mark(PH_SUB);
+    tm.mark(PH_FUP);
+    launch_f_update(a, Pl, np_max, st);
+    tm.mark(PH_FUP);
+  }
+
+  // ---------------- a7-a9 bias, decision values, sigmoid, SV union
+  tm.mark(PH_FIN);
+  launch_finalize(a, Pl, st);
+  launch_sigmoid_fit(a, Pl, st);
+  DevBuf<uint8_t> d_flags(n, st);
+  GM_CUDA(cudaMemsetAsync(d_flags.get(), 0, n, st));
+  launch_sv_flags(a, Pl, np_max, d_flags.get(), st);
+  std::vector<double> h_alpha(tot), hb(Pl), hA(Pl), hB(Pl);
+  std::vector<int32_t> h_sig(Pl), h_st(Pl), h_outer(Pl);
+  std::vector<int64_t> h_inner(Pl), h_perm(n);
+  std::vector<uint8_t> h_flags(n);
+  GM_CUDA(cudaMemcpyAsync(h_alpha.data(), d_alpha.get(), tot * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(hb.data(), d_b.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(hA.data(), d_A.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(hB.data(), d_B.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_sig.data(), d_sig.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_st.data(), d_status.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_outer.data(), d_outer.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_inner.data(), d_inner.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_perm.data(), d_perm.get(), n * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_flags.data(), d_flags.get(), n, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+
+  auto* mdl = new Model();
+  std::unique_ptr<Model> guard(mdl);
+  mdl->k = k;
+  mdl->d = d;
+  mdl->C = C;
+  mdl->gamma = gamma;
+  mdl->eps = eps;
+  mdl->n = n;
+  mdl->class_count.assign(cc.begin(), cc.begin() + k);
+  mdl->perm = std::move(h_perm);
+  mdl->trained.assign(P, 0);
+  mdl->b.assign(P, 0.0);
+  mdl->A.assign(P, 0.0);
+  mdl->B.assign(P, 0.0);
+  mdl->status.assign(P, 0);
+  const auto po = mdl->pair_offsets();
+  mdl->alpha.assign(po[P], 0.0);
+  int64_t outer_max = 0, outer_sum = 0, inner_sum = 0;
+  for (int i = 0; i < Pl; ++i) {
+    const int p = pids[i];
+    mdl->trained[p] = 1;
+    mdl->b[p] = hb[i];
+    mdl->A[p] = hA[i];
+    mdl->B[p] = hB[i];
+    if (cap_hit && h_st[i] == 0) h_st[i] = 2;
+    mdl->status[p] = (h_st[i] == 1 ? 0 : h_st[i]) | (h_sig[i] << 8);
+    std::memcpy(&mdl->alpha[po[p]], &h_alpha[hp[i].a_off], sizeof(double) * (hp[i].n_s + hp[i].n_t));
+    outer_max = std::max<int64_t>(outer_max, h_outer[i]);
+    outer_sum += h_outer[i];
+    inner_sum += h_inner[i];
+  }
+  for (int64_t g = 0; g < n; ++g)
+    if (h_flags[g]) mdl->sv_pos.push_back(g);
+  std::vector<int64_t> row_of_sv(mdl->sv_pos.size());
+  for (size_t i = 0; i < row_of_sv.size(); ++i) row_of_sv[i] = mdl->perm[mdl->sv_pos[i]];
+  mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st);
+  tm.mark(PH_FIN);
+  GM_CUDA(cudaStreamSynchronize(st));
+
+  gmpsvm_train_stats& s = mdl->stats;
+  s.t_stage_ms = tm.ms(PH_STAGE);
+  s.t_kernel_ms = tm.ms(PH_KERNEL);
+  s.t_select_ms = tm.ms(PH_SELECT);
+  s.t_subproblem_ms = tm.ms(PH_SUB);
+  s.t_fupdate_ms = tm.ms(PH_FUP);
+  s.t_finalize_ms = tm.ms(PH_FIN);
+  s.kernel_values = (double)n * (double)(n + 1) / 2.0;
+  s.kernel_flops = s.kernel_values * (2.0 * d + 3.0);
+  s.krow_launches = 1;
+  s.outer_iters_max = outer_max;
+  s.outer_iters_sum = outer_sum;
+  s.inner_iters_sum = inner_sum;
+  s.n_sv = (int64_t)mdl->sv_pos.size();
+  s.cache_regime = 0;
+  s.n_pairs_trained = Pl;
+  s.launches = (int64_t)(g_launches.load() - launches0);
+  s.t_total_ms = host_ms_since(t_start);
+  *out = guard.release();
+  bool warn = cap_hit;
+  for (int i = 0; i < Pl; ++i) warn = warn || h_sig[i] == 1;
+  return warn ? GMPSVM_WARN_MAXITER : GMPSVM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+static void ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
+  std::lock_guard<std::mutex> lk(mdl.mu);
+  if (mdl.dev && mdl.dev->device == device) return;
+  if (mdl.dev) ensure_host_sv(mdl);
+  const int64_t nsv = (int64_t)mdl.sv_pos.size();
+  DevBuf<float> rows((size_t)std::max<int64_t>(nsv, 1) * mdl.d, st);
+  if (nsv > 0) {
+    if (!mdl.sv_X_ready) throw Error(GMPSVM_EINVAL, "model has no SV rows");
+    GM_CUDA(cudaMemcpyAsync(rows.get(), mdl.sv_X.data(), (size_t)nsv * mdl.d * 4, cudaMemcpyHostToDevice, st));
+  }
+  std::vector<int64_t> row_of_sv(nsv);
+  for (int64_t i = 0; i < nsv; ++i) row_of_sv[i] = i;
+  mdl.dev = build_dev_model(mdl, rows.get(), row_of_sv, device, st);
+}
+
+int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
+                   const gmpsvm_options& opt) {
+  const auto t_start = std::chrono::steady_clock::now();
+  gmpsvm_predict_stats& ps = tls_predict_stats();
+  ps = gmpsvm_predict_stats{};
+  if (m < 0 || (m > 0 && (!Xt || (!prob_out && !dec_out)))) throw Error(GMPSVM_EINVAL, "bad predict arguments");
+  if (mdl.n_trained() != mdl.P()) throw Error(GMPSVM_EINVAL, "model does not contain every pair (merge the parts first)");
+  if (prob_out && mdl.k > kMaxCoupleK) throw Error(GMPSVM_ENOTIMPL, "coupling supports k <= 40");
+  if (m == 0) return GMPSVM_OK;
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  const uint64_t launches0 = g_launches.load();
+  ensure_dev_model(mdl, opt.device, st);
+  const DevModel& dm = *mdl.dev;
+  const int k = mdl.k, d = mdl.d, P = mdl.P();
+  PhaseTimer tm(st);
+  const int64_t mc_max = std::min<int64_t>(m, kPredictChunk);
+  const int64_t mc_pad = round_up(mc_max, kTile);
+  DevBuf<float> xin(opt.inputs_on_device ? 0 : (size_t)mc_max * d, st);
+  DevBuf<float> XtT((size_t)dm.d_pad * mc_pad, st), nt(mc_pad, st);
+  DevBuf<float> part((size_t)dm.n_items * mc_pad * dm.km1_pad, st);
+  DevBuf<double> dec_buf(opt.inputs_on_device ? 0 : (size_t)mc_max * P, st);
+  DevBuf<double> prob_buf((opt.inputs_on_device || !prob_out) ? 0 : (size_t)mc_max * k, st);
+  DevBuf<double> dec_tmp((opt.inputs_on_device && !dec_out) ? (size_t)mc_max * P : 0, st);
+  DevBuf<int32_t> bad(1, st);
+  GM_CUDA(cudaMemsetAsync(bad.get(), 0, 4, st));
+  for (int64_t i0 = 0; i0 < m; i0 += mc_max) {
+    const int64_t mc = std::min(mc_max, m - i0);
+    const int64_t mcp = round_up(mc, kTile);
+    tm.mark(PH_STAGE);
+    const float* src = Xt + i0 * d;
+    if (!opt.inputs_on_device) {
+      GM_CUDA(cudaMemcpyAsync(xin.get(), src, (size_t)mc * d * 4, cudaMemcpyHostToDevice, st));
+      src = xin.get();
+    }
+    launch_stage_features(src, mc, d, nullptr, XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(), st);
+    tm.mark(PH_STAGE);
+    double* dec_d = opt.inputs_on_device ? (dec_out ? dec_out + i0 * P : dec_tmp.get()) : dec_buf.get();
+    tm.mark(PH_DEC);
+    launch_dec_contract(XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef, dm.km1, dm.km1_pad,
+                        dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
+    launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
+    ps.dec_launches += 1;
+    tm.mark(PH_DEC);
+    double* prob_d = nullptr;
+    if (prob_out) {
+      prob_d = opt.inputs_on_device ? prob_out + i0 * k : prob_buf.get();
+      tm.mark(PH_COUPLE);
+      launch_couple(dec_d, mc, k, dm.A, dm.B, prob_d, st);
+      tm.mark(PH_COUPLE);
+    }
+    if (!opt.inputs_on_device) {
+      tm.mark(PH_D2H);
+      if (prob_out)
+        GM_CUDA(cudaMemcpyAsync(prob_out + i0 * k, prob_d, (size_t)mc * k * 8, cudaMemcpyDeviceToHost, st));
+      if (dec_out) GM_CUDA(cudaMemcpyAsync(dec_out + i0 * P, dec_d, (size_t)mc * P * 8, cudaMemcpyDeviceToHost, st));
+      tm.mark(PH_D2H);
+    }
+  }
+  int32_t hbad = 0;
+  GM_CUDA(cudaMemcpyAsync(&hbad, bad.get(), 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  ps.t_stage_ms = tm.ms(PH_STAGE);
+  ps.t_decision_ms = tm.ms(PH_DEC);
+  ps.t_couple_ms = tm.ms(PH_COUPLE);
+  ps.t_d2h_ms = tm.ms(PH_D2H);
+  ps.dec_flops = (double)m * (double)mdl.sv_pos.size() * (2.0 * d + 3.0 + 2.0 * (k - 1));
+  ps.launches = (int64_t)(g_launches.load() - launches0);
+  ps.t_total_ms = host_ms_since(t_start);
+  if (hbad) throw Error(GMPSVM_EINVAL, "Xtest contains non-finite values");
+  return GMPSVM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int32_t d, double gamma, float* K_out,
+                      const gmpsvm_options& opt) {
+  if (n < 0 || m < 0 || d < 1 || !finite_pos(gamma)) throw Error(GMPSVM_EINVAL, "bad rbf_kernel arguments");
+  if (n == 0 || m == 0) return GMPSVM_OK;
+  if (!X || !Y || !K_out) throw Error(GMPSVM_EINVAL, "null argument");
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  const int d_pad = (int)round_up(d, kBK);
+  const int64_t n_pad = round_up(n, kTile), m_pad = round_up(m, kTile);
+  DevBuf<float> bx(opt.inputs_on_device ? 0 : (size_t)n * d, st), by(opt.inputs_on_device ? 0 : (size_t)m * d, st);
+  const float* dX = X;
+  const float* dY = Y;
+  if (!opt.inputs_on_device) {
+    GM_CUDA(cudaMemcpyAsync(bx.get(), X, (size_t)n * d * 4, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(by.get(), Y, (size_t)m * d * 4, cudaMemcpyHostToDevice, st));
+    dX = bx.get();
+    dY = by.get();
+  }
+  // X == Y (same buffer, same size): the symmetric FULL_K launch that training uses (K_ii = 1)
+  const bool sym = (X == Y && n == m);
+  DevBuf<float> XT((size_t)d_pad * n_pad, st), YT(sym ? 0 : (size_t)d_pad * m_pad, st), nx(n_pad, st),
+      ny(sym ? 0 : m_pad, st);
+  launch_stage_features(dX, n, d, nullptr, XT.get(), n_pad, d_pad, n_pad, nx.get(), nullptr, st);
+  if (!sym) launch_stage_features(dY, m, d, nullptr, YT.get(), m_pad, d_pad, m_pad, ny.get(), nullptr, st);
+  DevBuf<float> kb(opt.inputs_on_device ? 0 : (size_t)n * m, st);
+  float* dK = opt.inputs_on_device ? K_out : kb.get();
+  if (sym)
+    launch_krow_full_sym(XT.get(), n_pad, nx.get(), n, d_pad, gamma, dK, m, st);
+  else
+    launch_krow_rect(XT.get(), n_pad, nx.get(), n, YT.get(), m_pad, ny.get(), m, d_pad, gamma, dK, m, st);
+  if (!opt.inputs_on_device) GM_CUDA(cudaMemcpyAsync(K_out, dK, (size_t)n * m * 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  return GMPSVM_OK;
+}
+
+int engine_couple(const double* dec, int64_t m, int32_t k, const double* A, const double* B, double* prob_out,
+                  const gmpsvm_options& opt) {
+  if (m < 0 || k < 2 || !dec || !A || !B || !prob_out) throw Error(GMPSVM_EINVAL, "bad couple arguments");
+  if (k > kMaxCoupleK) throw Error(GMPSVM_ENOTIMPL, "coupling supports k <= 40");
+  if (m == 0) return GMPSVM_OK;
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  const int P = k * (k - 1) / 2;
+  if (opt.inputs_on_device) {
+    launch_couple(dec, m, k, A, B, prob_out, st);
+  } else {
+    DevBuf<double> dd((size_t)m * P, st), dA(P, st), dB(P, st), dp((size_t)m * k, st);
+    GM_CUDA(cudaMemcpyAsync(dd.get(), dec, (size_t)m * P * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(dA.get(), A, P * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(dB.get(), B, P * 8, cudaMemcpyHostToDevice, st));
+    launch_couple(dd.get(), m, k, dA.get(), dB.get(), dp.get(), st);
+    GM_CUDA(cudaMemcpyAsync(prob_out, dp.get(), (size_t)m * k * 8, cudaMemcpyDeviceToHost, st));
+  }
+  GM_CUDA(cudaStreamSynchronize(st));
+  return GMPSVM_OK;
+}
+
+}  // namespace gmpsvm

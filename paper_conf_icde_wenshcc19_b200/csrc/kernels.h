@@ -1,0 +1,72 @@
+// kernels.h -- launchers of the sm_100a kernels (internal to libgmpsvm).
+#pragma once
+
+#include "common.cuh"
+
+namespace gmpsvm {
+
+// ---------------- a1 staging (stage.cu)
+void launch_class_sort(const int32_t* y, int64_t n, int k, int32_t* blk_counts, int32_t* blk_off,
+                       int64_t* class_count, int64_t* class_off, cudaStream_t st);
+void launch_class_rank(const int32_t* y, int64_t n, int k, const int32_t* blk_off, const int64_t* class_off,
+                       int64_t* perm, cudaStream_t st);
+// XT[c][j] = X[src(j)][c] (src = perm[j], or j if perm == NULL; src < 0 = zero padding slot),
+// norms[j] = ||X[src(j)]||^2; *bad (may be NULL) set to 1 if a row is non-finite.
+void launch_stage_features(const float* X, int64_t n, int d, const int64_t* perm, float* XT, int64_t ldx, int d_pad,
+                           int64_t n_pad, float* norms, int32_t* bad, cudaStream_t st);
+void launch_gather_rows(const float* X, int d, const int64_t* idx, int64_t nr, float* dst, cudaStream_t st);
+
+// ---------------- a2 kernel values (krow.cu)
+void launch_krow_full_sym(const float* XT, int64_t ldx, const float* norms, int64_t n, int kdim, double gamma,
+                          float* K, int64_t ldk, cudaStream_t st);
+void launch_krow_rect(const float* AT, int64_t lda, const float* na, int64_t n, const float* BT, int64_t ldb,
+                      const float* nb, int64_t m, int kdim, double gamma, float* K, int64_t ldk, cudaStream_t st);
+
+// ---------------- a4-a9 solver (solver.cu)
+struct SolverArgs {
+  const PairDesc* pairs;
+  const float* K;
+  int64_t ldk;
+  double* alpha;        // [sum n_p]
+  double* f;            // [sum n_p]
+  double* v;            // [sum n_p] in-sample decision values (finalize)
+  uint32_t* stamp;      // [sum n_p] selection stamps
+  int32_t* ws;          // [P][B] working set (pair-local indices), oldest first
+  int32_t* ws_n;        // [P]
+  int32_t* ws_tmp;      // [P][B]
+  float* Kws;           // [P][B][B] gathered K_ws,ws
+  double* dcoef;        // [P][B] delta-alpha * y of the last local solve
+  int32_t* status;      // [P] 0 active, 1 converged, 2 outer cap
+  double* gap;          // [P] global gap at the last selection
+  int64_t* inner_iters; // [P]
+  int32_t* outer_iters; // [P]
+  double* b;            // [P]
+  double* A;            // [P]
+  double* Bs;           // [P] (sigmoid B)
+  int32_t* sig_status;  // [P]
+  int B, q, inner_cap, pad;
+  double C, eps;
+};
+
+void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st);
+void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st);
+void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st);
+void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st);
+void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
+void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
+void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);
+void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st);
+
+// ---------------- a10-a12 prediction (predict.cu)
+struct DecItem {
+  int32_t cls, tile_begin, tile_end, pad;
+};
+void launch_dec_contract(const float* XtT, int64_t ldt, const float* nt, int64_t m, int64_t m_pad, const float* SvT,
+                         int64_t lds, const float* nsv, const float* coef, int km1, int km1_pad, const DecItem* items,
+                         int n_items, int kdim, double gamma, float* part, cudaStream_t st);
+void launch_dec_reduce(const float* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,
+                       const int32_t* item_end, const double* b, double* dec, cudaStream_t st);
+void launch_couple(const double* dec, int64_t m, int k, const double* A, const double* B, double* prob,
+                   cudaStream_t st);
+
+}  // namespace gmpsvm

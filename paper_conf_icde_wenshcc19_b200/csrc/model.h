@@ -1,0 +1,72 @@
+// model.h -- the library-owned model object (opaque gmpsvm_model in the ABI).
+#pragma once
+
+#include <memory>
+#include <mutex>
+#include <vector>
+
+#include "kernels.h"
+
+namespace gmpsvm {
+
+// Device-resident prediction structures (support-vector sharing):
+// the SV union in class-pure 128-column tiles, stored feature-major (SvT[c][slot]),
+// its norms, the LibSVM-style coefficient matrix coef[slot][k-1] (= y * alpha of the SV in
+// each of the k-1 pairs of its class), and the per-class runs of tiles ("items").
+struct DevModel {
+  int device = -1;
+  int d_pad = 0, km1 = 0, km1_pad = 0, n_items = 0;
+  int64_t nsv_pad = 0;
+  float* SvT = nullptr;     // [d_pad][nsv_pad]
+  float* nsv = nullptr;     // [nsv_pad]
+  float* coef = nullptr;    // [nsv_pad][km1_pad]
+  DecItem* items = nullptr; // [n_items]
+  int32_t* item_begin = nullptr;  // [k]
+  int32_t* item_end = nullptr;    // [k]
+  double* b = nullptr;      // [P]
+  double* A = nullptr;      // [P]
+  double* B = nullptr;      // [P]
+  std::vector<int64_t> slot_sv;  // slot -> index into the model's SV list, -1 = padding
+  ~DevModel();
+};
+
+struct Model {
+  int32_t k = 0, d = 0;
+  double C = 0, gamma = 0, eps = 0;
+  int64_t n = 0;
+  std::vector<int64_t> class_count;  // [k]
+  std::vector<int64_t> perm;         // class-sorted position -> original index [n]
+  std::vector<uint8_t> trained;      // [P]
+  std::vector<double> b, A, B;       // [P]
+  std::vector<int32_t> status;       // [P] solver status (0 ok, 2 outer cap) | sigmoid status << 8
+  std::vector<double> alpha;         // [sum_p n_p] pair-local order, all pairs (0 for untrained)
+  std::vector<int64_t> sv_pos;       // class-sorted positions of the SV union, ascending
+  std::vector<float> sv_X;           // [n_sv][d] host copy (materialised lazily from the device)
+  bool sv_X_ready = false;
+  gmpsvm_train_stats stats{};
+  mutable std::mutex mu;
+  mutable std::unique_ptr<DevModel> dev;
+
+  int P() const { return k * (k - 1) / 2; }
+  std::vector<int64_t> class_off() const;
+  std::vector<int64_t> pair_offsets() const;  // [P+1] offsets of each pair into alpha
+  int n_trained() const;
+};
+
+// engine.cu
+int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma, double eps,
+                 const gmpsvm_options& opt, Model** out);
+int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
+                   const gmpsvm_options& opt);
+int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int32_t d, double gamma, float* K_out,
+                      const gmpsvm_options& opt);
+int engine_couple(const double* dec, int64_t m, int32_t k, const double* A, const double* B, double* prob_out,
+                  const gmpsvm_options& opt);
+void ensure_host_sv(const Model& mdl);  // materialise sv_X on the host
+gmpsvm_predict_stats& tls_predict_stats();
+
+}  // namespace gmpsvm
+
+struct gmpsvm_model {
+  std::unique_ptr<gmpsvm::Model> m;
+};

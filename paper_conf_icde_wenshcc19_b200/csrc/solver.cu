@@ -1,0 +1,783 @@
+// solver.cu -- a4..a9: the batched working-set SMO solver of every active pair, run
+// concurrently (one CTA per pair per step; Alg 2), plus the
+// bias, in-sample decision values, Platt fit and SV flags.
+//
+//   select_ws   a4  q/2 smallest f in I_u + q/2 largest f in I_l, newest B-q kept
+//                   (L293-L297, Alg 2 lines 6-7; radix select on order-preserving keys)
+//                   and the global stop test max_{I_l} f - min_{I_u} f < eps (Eq 9-10)
+//   gather_kws  a3  K_ws,ws gathered from the resident kernel matrix (the "GPU buffer", L299-L303)
+//   local_smo   a5  WSS2 SMO restricted to the working set (ImproveSVM, L301-L305, Eq 4-8),
+//                   early stop at local gap < max(eps, 0.1 delta0) (L305, reading R20)
+//   f_update    a6  f_j += sum_ws dalpha_i y_i K_ij over the whole pair (Alg 2 line 11, Eq 8)
+//   finalize    a7  rho (LibSVM rule, reading R7), b = -rho, v_i = f_i + y_i - rho (Eq 3 + 11)
+//   sigmoid_fit a8  Newton + backtracking on Eq 13, 4 step sizes evaluated per pass (L327)
+//   sv_flags    a9  SV union membership over pairs (support-vector sharing, L363)
+#include <cfloat>
+#include <climits>
+
+#include "kernels.h"
+
+namespace gmpsvm {
+
+#define FULLMASK 0xffffffffu
+
+__device__ __forceinline__ uint64_t ord_key(double x) {
+  const uint64_t u = (uint64_t)__double_as_longlong(x);
+  return (u & 0x8000000000000000ull) ? ~u : (u | 0x8000000000000000ull);
+}
+__device__ __forceinline__ double key_double(uint64_t k) {
+  const uint64_t u = (k & 0x8000000000000000ull) ? (k & 0x7fffffffffffffffull) : ~k;
+  return __longlong_as_double((long long)u);
+}
+__device__ __forceinline__ bool in_u(int y, double a, double C) { return (y > 0 && a < C) || (y < 0 && a > 0.0); }
+__device__ __forceinline__ bool in_l(int y, double a, double C) { return (y > 0 && a > 0.0) || (y < 0 && a < C); }
+__device__ __forceinline__ int64_t gpos(const PairDesc& pd, int64_t j) {
+  return j < pd.n_s ? pd.off_s + j : pd.off_t + (j - pd.n_s);
+}
+
+// ------------------------------------------------------------------------------------------
+// block helpers (blockDim.x multiple of 32, <= 1024)
+template <typename T, typename Op>
+__device__ T block_reduce(T v, Op op, T* sm /* >= 32 */) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = op(v, __shfl_xor_sync(FULLMASK, v, o));
+  __syncthreads();
+  if (lane == 0) sm[warp] = v;
+  __syncthreads();
+  T r = sm[0];
+  for (int w = 1; w < nw; ++w) r = op(r, sm[w]);
+  return r;
+}
+
+// exclusive prefix over the block of a flag (block order = thread order); returns rank
+__device__ int block_excl_scan(bool flag, int& total, int* sm /* 33 */) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const unsigned b = __ballot_sync(FULLMASK, flag);
+  const int pre = __popc(b & ((1u << lane) - 1u));
+  __syncthreads();
+  if (lane == 0) sm[warp] = __popc(b);
+  __syncthreads();
+  if (warp == 0) {
+    const int v = lane < nw ? sm[lane] : 0;
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(FULLMASK, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane < nw) sm[lane] = x - v;
+    if (lane == 31) sm[32] = x;
+  }
+  __syncthreads();
+  total = sm[32];
+  return sm[warp] + pre;
+}
+
+// ------------------------------------------------------------------------------------------
+__global__ void init_pairs_kernel(SolverArgs a, const int64_t tot, int P) {
+  // alpha = 0, f = -y (Alg 1 lines 1-2 / Alg 2 line 4), stamps 0
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < tot) {
+    // find pair by binary search over a_off
+    int lo = 0, hi = P - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (a.pairs[mid].a_off <= i) lo = mid;
+      else hi = mid - 1;
+    }
+    const PairDesc pd = a.pairs[lo];
+    const int64_t j = i - pd.a_off;
+    a.alpha[i] = 0.0;
+    a.f[i] = (j < pd.n_s) ? -1.0 : 1.0;
+    a.stamp[i] = 0u;
+  }
+  if (i < P) {
+    a.status[i] = 0;
+    a.ws_n[i] = 0;
+    a.inner_iters[i] = 0;
+    a.outer_iters[i] = 0;
+    a.gap[i] = 0.0;
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// a4: working-set selection
+struct SelSmem {
+  int32_t hist[256];
+  int32_t scan[33];
+  double red[32];
+  int32_t sel_digit, sel_below, take_all, pad;
+};
+
+struct PickCtx {
+  const double* al;
+  const double* fl;
+  uint32_t* st;
+  uint32_t stampv;
+  int n_s, np;
+  double C;
+};
+
+template <bool SIDE_U>
+__device__ __forceinline__ bool pick_cand(const PickCtx& cx, int i, uint64_t& key) {
+  const int y = i < cx.n_s ? 1 : -1;
+  const double a = cx.al[i];
+  const bool ok = SIDE_U ? in_u(y, a, cx.C) : in_l(y, a, cx.C);
+  if (!ok || cx.st[i] == cx.stampv) return false;
+  const double f = cx.fl[i];
+  key = SIDE_U ? ord_key(f) : ord_key(-f);  // ascending key = U: smallest f, L: largest f
+  return true;
+}
+
+// Select the `want` smallest keys among the candidates of one side (ties: lowest index),
+// append them to out[] in index order and stamp them.  Returns the number taken.
+template <bool SIDE_U>
+__device__ int radix_pick(const PickCtx& cx, int want, int32_t* out, SelSmem& sm) {
+  if (want <= 0) return 0;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  uint64_t prefix = 0, pmask = 0;
+  int remaining = want;
+  bool take_all = false;
+  for (int shift = 56; shift >= 0; shift -= 8) {
+    for (int b = tid; b < 256; b += blockDim.x) sm.hist[b] = 0;
+    __syncthreads();
+    for (int base = 0; base < cx.np; base += blockDim.x) {
+      const int i = base + tid;
+      uint64_t key = 0;
+      const bool m = (i < cx.np) && pick_cand<SIDE_U>(cx, i, key) && ((key & pmask) == prefix);
+      const unsigned am = __ballot_sync(FULLMASK, m);
+      if (m) {
+        const int digit = (int)((key >> shift) & 255u);
+        const unsigned peers = __match_any_sync(am, digit);
+        if (lane == __ffs(peers) - 1) atomicAdd(&sm.hist[digit], __popc(peers));
+      }
+    }
+    __syncthreads();
+    if (warp == 0) {
+      int loc[8], s = 0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        loc[q] = sm.hist[lane * 8 + q];
+        s += loc[q];
+      }
+      int incl = s;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(FULLMASK, incl, o);
+        if (lane >= o) incl += y;
+      }
+      const int excl = incl - s;
+      const int total = __shfl_sync(FULLMASK, incl, 31);
+      if (lane == 0) sm.take_all = (shift == 56 && total <= remaining) ? 1 : 0;
+      if (excl < remaining && remaining <= incl) {
+        int below = excl, dg = lane * 8;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          if (below + loc[q] >= remaining) {
+            dg = lane * 8 + q;
+            break;
+          }
+          below += loc[q];
+        }
+        sm.sel_digit = dg;
+        sm.sel_below = below;
+      }
+    }
+    __syncthreads();
+    if (sm.take_all) {
+      take_all = true;
+      break;
+    }
+    remaining -= sm.sel_below;
+    prefix |= (uint64_t)sm.sel_digit << shift;
+    pmask |= (uint64_t)0xffu << shift;
+    __syncthreads();
+  }
+  // collect in index order: all keys < T, then the first `remaining` keys == T
+  const uint64_t T = prefix;
+  int taken = 0, eq_taken = 0;
+  for (int base = 0; base < cx.np; base += blockDim.x) {
+    const int i = base + tid;
+    uint64_t key = 0;
+    const bool c = (i < cx.np) && pick_cand<SIDE_U>(cx, i, key);
+    const bool lt = c && (take_all || key < T);
+    const bool eq = c && !take_all && key == T;
+    int eq_tot = 0, tk_tot = 0;
+    const int eq_rank = block_excl_scan(eq, eq_tot, sm.scan);
+    const bool take = lt || (eq && eq_taken + eq_rank < remaining);
+    const int pos = block_excl_scan(take, tk_tot, sm.scan);
+    if (take) {
+      out[taken + pos] = i;
+      cx.st[i] = cx.stampv;
+    }
+    taken += tk_tot;
+    eq_taken += eq_tot;
+  }
+  __syncthreads();
+  return taken;
+}
+
+__global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t stampv, int first) {
+  __shared__ SelSmem sm;
+  const int lp = blockIdx.x;
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const double* al = a.alpha + pd.a_off;
+  const double* fl = a.f + pd.a_off;
+  const double C = a.C;
+  // global stop test (Eq 9-10 with tolerance eps)
+  double fmin = DBL_MAX, fmax = -DBL_MAX;
+  for (int i = threadIdx.x; i < np; i += blockDim.x) {
+    const int y = i < pd.n_s ? 1 : -1;
+    const double av = al[i], fv = fl[i];
+    if (in_u(y, av, C)) fmin = fmin < fv ? fmin : fv;
+    if (in_l(y, av, C)) fmax = fmax > fv ? fmax : fv;
+  }
+  fmin = block_reduce(fmin, [](double x, double y) { return x < y ? x : y; }, sm.red);
+  fmax = block_reduce(fmax, [](double x, double y) { return x > y ? x : y; }, sm.red);
+  const double gap = fmax - fmin;
+  const bool done = (fmin == DBL_MAX) || (fmax == -DBL_MAX) || !(gap >= a.eps);
+  if (threadIdx.x == 0) {
+    a.gap[lp] = gap;
+    if (done) a.status[lp] = 1;
+    else a.outer_iters[lp] += 1;
+  }
+  if (done) return;
+  const int B = a.B;
+  int32_t* ws = a.ws + (int64_t)lp * B;
+  if (np <= B) {  // the whole pair is the working set
+    if (first) {
+      for (int i = threadIdx.x; i < np; i += blockDim.x) ws[i] = i;
+      if (threadIdx.x == 0) a.ws_n[lp] = np;
+    }
+    return;
+  }
+  int32_t* nxt = a.ws_tmp + (int64_t)lp * B;
+  uint32_t* stp = a.stamp + pd.a_off;
+  const int prev_n = first ? 0 : a.ws_n[lp];
+  const int keep = min(prev_n, B - a.q);
+  for (int e = threadIdx.x; e < keep; e += blockDim.x) {
+    const int idx = ws[prev_n - keep + e];
+    nxt[e] = idx;
+    stp[idx] = stampv;
+  }
+  __syncthreads();
+  PickCtx cx{al, fl, stp, stampv, pd.n_s, np, C};
+  const int need = B - keep;
+  int cnt = keep;
+  cnt += radix_pick<true>(cx, need / 2, nxt + cnt, sm);
+  cnt += radix_pick<false>(cx, B - cnt, nxt + cnt, sm);
+  if (cnt < B) cnt += radix_pick<true>(cx, B - cnt, nxt + cnt, sm);
+  for (int e = threadIdx.x; e < cnt; e += blockDim.x) ws[e] = nxt[e];
+  if (threadIdx.x == 0) a.ws_n[lp] = cnt;
+}
+
+// ------------------------------------------------------------------------------------------
+// a3: K_ws,ws gathered into a dense B x B tile per pair (L2-resident during local_smo)
+constexpr int kGatherRows = 16;
+
+__global__ void __launch_bounds__(256) gather_kws_kernel(SolverArgs a, int first) {
+  const int lp = blockIdx.x;
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  if (np <= a.B && !first) return;  // working set unchanged
+  const int wn = a.ws_n[lp];
+  const int r0 = blockIdx.y * kGatherRows;
+  if (r0 >= wn) return;
+  __shared__ int64_t g[1024];
+  const int32_t* ws = a.ws + (int64_t)lp * a.B;
+  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
+  __syncthreads();
+  const int r1 = min(wn, r0 + kGatherRows);
+  for (int r = r0; r < r1; ++r) {
+    const float* row = a.K + g[r] * a.ldk;
+    float* dst = a.Kws + ((int64_t)lp * a.B + r) * a.B;
+    for (int e = threadIdx.x; e < wn; e += blockDim.x) dst[e] = __ldg(row + g[e]);
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// a5: local SMO on the working set (one CTA per pair, 256 threads, E ws rows per thread)
+struct RedSlot {
+  uint32_t k0, k1;
+  int32_t idx, e;
+  double alpha, f;
+  uint32_t m0, m1;  // running max key (f_max over I_l)
+  uint32_t pad0, pad1;
+};
+
+// lexicographic min of (k0, k1, idx) over the warp; returns the winning lane (lowest on ties)
+__device__ __forceinline__ int warp_argmin(uint32_t& k0, uint32_t& k1, int32_t& idx) {
+  const uint32_t m0 = __reduce_min_sync(FULLMASK, k0);
+  const uint32_t t1 = (k0 == m0) ? k1 : 0xffffffffu;
+  const uint32_t m1 = __reduce_min_sync(FULLMASK, t1);
+  const bool tie = (k0 == m0) && (k1 == m1);
+  const uint32_t t2 = tie ? (uint32_t)idx : 0xffffffffu;
+  const uint32_t m2 = __reduce_min_sync(FULLMASK, t2);
+  const unsigned b = __ballot_sync(FULLMASK, tie && t2 == m2);
+  k0 = m0;
+  k1 = m1;
+  idx = (int32_t)m2;
+  return __ffs(b) - 1;
+}
+__device__ __forceinline__ void warp_max64(uint32_t& h, uint32_t& l) {
+  const uint32_t mh = __reduce_max_sync(FULLMASK, h);
+  const uint32_t tl = (h == mh) ? l : 0u;
+  l = __reduce_max_sync(FULLMASK, tl);
+  h = mh;
+}
+
+// Block argmin of (k0,k1,idx) carrying (e, alpha, f) and a running max key (m0,m1).
+__device__ __forceinline__ RedSlot block_argmin(RedSlot c, RedSlot* slots) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  uint32_t k0 = c.k0, k1 = c.k1, mh = c.m0, ml = c.m1;
+  int32_t idx = c.idx;
+  const int wl = warp_argmin(k0, k1, idx);
+  warp_max64(mh, ml);
+  if (lane == wl) {
+    RedSlot s = c;
+    s.m0 = mh;
+    s.m1 = ml;
+    slots[warp] = s;
+  }
+  __syncthreads();
+  RedSlot r;
+  if (lane < nw) r = slots[lane];
+  else {
+    r.k0 = r.k1 = 0xffffffffu;
+    r.idx = INT_MAX;
+    r.m0 = r.m1 = 0u;
+  }
+  k0 = r.k0;
+  k1 = r.k1;
+  idx = r.idx;
+  mh = r.m0;
+  ml = r.m1;
+  const int w2 = warp_argmin(k0, k1, idx);
+  warp_max64(mh, ml);
+  RedSlot out = slots[w2 < nw ? w2 : 0];
+  out.m0 = mh;
+  out.m1 = ml;
+  if (idx == INT_MAX || k0 == 0xffffffffu && k1 == 0xffffffffu) out.idx = INT_MAX;
+  return out;
+}
+
+template <int E>
+__global__ void __launch_bounds__(256) local_smo_kernel(SolverArgs a) {
+  __shared__ RedSlot slots[2][8];
+  const int lp = blockIdx.x;
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int B = a.B, wn = a.ws_n[lp];
+  const int tid = threadIdx.x;
+  const float* Kw = a.Kws + (int64_t)lp * B * B;
+  const int32_t* ws = a.ws + (int64_t)lp * B;
+  const double C = a.C;
+  int32_t idx[E];
+  int y[E];
+  double al[E], a0[E], fv[E];
+  float kd[E], ku[E];
+  bool valid[E];
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = tid + q * 256;
+    valid[q] = e < wn;
+    idx[q] = valid[q] ? ws[e] : INT_MAX;
+    y[q] = (valid[q] && idx[q] < pd.n_s) ? 1 : -1;
+    al[q] = valid[q] ? a.alpha[pd.a_off + idx[q]] : 0.0;
+    a0[q] = al[q];
+    fv[q] = valid[q] ? a.f[pd.a_off + idx[q]] : 0.0;
+    kd[q] = valid[q] ? Kw[(int64_t)e * B + e] : 1.f;
+  }
+  const int cap = a.inner_cap;
+  int it = 0, par = 0;
+  double delta0 = 0.0;
+  for (;;) {
+    // Step 1 (Eq 4): u = argmin_{I_u} f, ties -> lowest pair-local index
+    RedSlot cu;
+    cu.k0 = cu.k1 = 0xffffffffu;
+    cu.idx = INT_MAX;
+    cu.e = -1;
+    cu.m0 = cu.m1 = 0u;
+    cu.alpha = 0.0;
+    cu.f = 0.0;
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      if (valid[q] && in_u(y[q], al[q], C)) {
+        const uint64_t key = ord_key(fv[q]);
+        const uint32_t h = (uint32_t)(key >> 32), l = (uint32_t)key;
+        if (h < cu.k0 || (h == cu.k0 && (l < cu.k1 || (l == cu.k1 && idx[q] < cu.idx)))) {
+          cu.k0 = h;
+          cu.k1 = l;
+          cu.idx = idx[q];
+          cu.e = tid + q * 256;
+          cu.alpha = al[q];
+          cu.f = fv[q];
+        }
+      }
+    }
+    const RedSlot ru = block_argmin(cu, slots[par]);
+    par ^= 1;
+    if (ru.idx == INT_MAX) break;
+    const int ue = ru.e;
+    const double fu = ru.f, au = ru.alpha;
+    const int yu = ru.idx < pd.n_s ? 1 : -1;
+    const float* Kur = Kw + (int64_t)ue * B;
+#pragma unroll
+    for (int q = 0; q < E; ++q) ku[q] = valid[q] ? Kur[tid + q * 256] : 0.f;
+    const float kuu = Kur[ue];
+    // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_u - f_t)^2 / eta_t ; also f_max over I_l (Eq 10)
+    RedSlot cl;
+    cl.k0 = cl.k1 = 0xffffffffu;
+    cl.idx = INT_MAX;
+    cl.e = -1;
+    cl.m0 = cl.m1 = 0u;
+    cl.alpha = 0.0;
+    cl.f = 0.0;
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      if (valid[q] && in_l(y[q], al[q], C)) {
+        const uint64_t fk = ord_key(fv[q]);
+        const uint32_t h = (uint32_t)(fk >> 32), l = (uint32_t)fk;
+        if (h > cl.m0 || (h == cl.m0 && l > cl.m1)) {
+          cl.m0 = h;
+          cl.m1 = l;
+        }
+        if (fv[q] > fu) {
+          double eta = (double)kuu + (double)kd[q] - 2.0 * (double)ku[q];
+          eta = eta > kTau ? eta : kTau;
+          const double df = fv[q] - fu;
+          const float score = (float)(df * df / eta);
+          const uint32_t sk = ~__float_as_uint(score);
+          if (sk < cl.k0 || (sk == cl.k0 && (0u < cl.k1 || idx[q] < cl.idx))) {
+            cl.k0 = sk;
+            cl.k1 = 0u;
+            cl.idx = idx[q];
+            cl.e = tid + q * 256;
+            cl.alpha = al[q];
+            cl.f = fv[q];
+          }
+        }
+      }
+    }
+    const RedSlot rl = block_argmin(cl, slots[par]);
+    par ^= 1;
+    const double fmax = (rl.m0 == 0u && rl.m1 == 0u) ? -DBL_MAX : key_double(((uint64_t)rl.m0 << 32) | rl.m1);
+    const double gap = fmax - fu;
+    if (it == 0) delta0 = gap;
+    const double tol = a.eps > 0.1 * delta0 ? a.eps : 0.1 * delta0;
+    if (!(gap >= tol) || rl.idx == INT_MAX || it >= cap) break;
+    const int le = rl.e;
+    const double fl = rl.f, alv = rl.alpha;
+    const int yl = rl.idx < pd.n_s ? 1 : -1;
+    const float* Klr = Kw + (int64_t)le * B;
+    // Step 2 (Eq 6-7) with explicit clipping (reading R4): common step s
+    double eta = (double)kuu + (double)Klr[le] - 2.0 * (double)Kur[le];
+    eta = eta > kTau ? eta : kTau;
+    double s = (fl - fu) / eta;
+    const double Uu = yu > 0 ? C - au : au;
+    const double Ll = yl > 0 ? alv : C - alv;
+    bool bu = false, bl = false;
+    if (Uu <= s) {
+      s = Uu;
+      bu = true;
+    }
+    if (Ll <= s) {
+      if (Ll < s) bu = false;
+      s = Ll;
+      bl = true;
+    }
+    double nau = au + yu * s, nal = alv - yl * s;
+    if (bu) nau = yu > 0 ? C : 0.0;
+    if (bl) nal = yl > 0 ? 0.0 : C;
+    // Step 3 (Eq 8) on the working set: f_i += s (K_ui - K_li)
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      const int e = tid + q * 256;
+      if (valid[q]) {
+        const float kl = Klr[e];
+        fv[q] += s * ((double)ku[q] - (double)kl);
+        if (e == ue) al[q] = nau;
+        if (e == le) al[q] = nal;
+      }
+    }
+    ++it;
+  }
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = tid + q * 256;
+    if (valid[q]) {
+      a.alpha[pd.a_off + idx[q]] = al[q];
+      a.dcoef[(int64_t)lp * B + e] = (al[q] - a0[q]) * (double)y[q];
+    }
+  }
+  if (tid == 0) a.inner_iters[lp] += it;
+}
+
+// ------------------------------------------------------------------------------------------
+// a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij for all j in the pair
+constexpr int kFCols = 1024;  // columns per CTA (256 threads x 4)
+
+__global__ void __launch_bounds__(256) f_update_kernel(SolverArgs a) {
+  const int lp = blockIdx.x;
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const int64_t c0 = (int64_t)blockIdx.y * kFCols;
+  if (c0 >= np) return;
+  __shared__ double coef[1024];
+  __shared__ const float* rowp[1024];
+  __shared__ int scan_sm[33];
+  const int B = a.B, wn = a.ws_n[lp];
+  const int32_t* ws = a.ws + (int64_t)lp * B;
+  const double* dc = a.dcoef + (int64_t)lp * B;
+  int nnz = 0;
+  for (int base = 0; base < wn; base += blockDim.x) {
+    const int e = base + threadIdx.x;
+    const double c = (e < wn) ? dc[e] : 0.0;
+    const bool nz = c != 0.0;
+    int tot = 0;
+    const int pos = block_excl_scan(nz, tot, scan_sm);
+    if (nz) {
+      coef[nnz + pos] = c;
+      rowp[nnz + pos] = a.K + gpos(pd, ws[e]) * a.ldk;
+    }
+    nnz += tot;
+  }
+  __syncthreads();
+  if (nnz == 0) return;
+  int64_t gc[4];
+  bool ok[4];
+  double acc[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const int64_t j = c0 + threadIdx.x + q * 256;
+    ok[q] = j < np;
+    gc[q] = ok[q] ? gpos(pd, j) : 0;
+    acc[q] = 0.0;
+  }
+  int r = 0;
+  for (; r + 2 <= nnz; r += 2) {
+    const float* p0 = rowp[r];
+    const float* p1 = rowp[r + 1];
+    const double c0v = coef[r], c1v = coef[r + 1];
+    float v0[4], v1[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      v0[q] = ok[q] ? __ldg(p0 + gc[q]) : 0.f;
+      v1[q] = ok[q] ? __ldg(p1 + gc[q]) : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      acc[q] = fma(c0v, (double)v0[q], acc[q]);
+      acc[q] = fma(c1v, (double)v1[q], acc[q]);
+    }
+  }
+  for (; r < nnz; ++r) {
+    const float* p0 = rowp[r];
+    const double c0v = coef[r];
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      if (ok[q]) acc[q] = fma(c0v, (double)__ldg(p0 + gc[q]), acc[q]);
+  }
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    if (ok[q]) a.f[pd.a_off + c0 + threadIdx.x + q * 256] += acc[q];
+}
+
+// ------------------------------------------------------------------------------------------
+// a7: bias and in-sample decision values
+__global__ void __launch_bounds__(1024) finalize_kernel(SolverArgs a) {
+  __shared__ double red[32];
+  const int lp = blockIdx.x;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const double* al = a.alpha + pd.a_off;
+  const double* fl = a.f + pd.a_off;
+  const double C = a.C;
+  double sum_free = 0.0, n_free = 0.0, ub = DBL_MAX, lb = -DBL_MAX;
+  for (int i = threadIdx.x; i < np; i += blockDim.x) {
+    const int y = i < pd.n_s ? 1 : -1;
+    const double av = al[i], fv = fl[i];
+    if (av > 0.0 && av < C) {
+      sum_free += fv;
+      n_free += 1.0;
+    } else {
+      if (in_u(y, av, C)) ub = ub < fv ? ub : fv;
+      if (in_l(y, av, C)) lb = lb > fv ? lb : fv;
+    }
+  }
+  auto add = [](double x, double y) { return x + y; };
+  sum_free = block_reduce(sum_free, add, red);
+  n_free = block_reduce(n_free, add, red);
+  ub = block_reduce(ub, [](double x, double y) { return x < y ? x : y; }, red);
+  lb = block_reduce(lb, [](double x, double y) { return x > y ? x : y; }, red);
+  const double rho = n_free > 0.0 ? sum_free / n_free : 0.5 * (ub + lb);
+  if (threadIdx.x == 0) a.b[lp] = -rho;
+  for (int i = threadIdx.x; i < np; i += blockDim.x) {
+    const int y = i < pd.n_s ? 1 : -1;
+    a.v[pd.a_off + i] = fl[i] + (double)y - rho;
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// a8: Platt sigmoid fit (Eq 12-13), Newton + backtracking with the constants of ref [15]
+// (reading R12); 4 candidate step sizes evaluated per pass over the data (L327).
+template <int N>
+__device__ void block_sum_n(double (&v)[N], double* sm /* 32*N */) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+#pragma unroll
+  for (int q = 0; q < N; ++q)
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v[q] += __shfl_xor_sync(FULLMASK, v[q], o);
+  __syncthreads();
+  if (lane == 0)
+#pragma unroll
+    for (int q = 0; q < N; ++q) sm[q * 32 + warp] = v[q];
+  __syncthreads();
+#pragma unroll
+  for (int q = 0; q < N; ++q) {
+    double s = 0.0;
+    for (int w = 0; w < nw; ++w) s += sm[q * 32 + w];
+    v[q] = s;
+  }
+}
+
+__device__ __forceinline__ double nll_term(double v, double t, double A, double B) {
+  const double z = v * A + B;
+  return z >= 0.0 ? t * z + log1p(exp(-z)) : (t - 1.0) * z + log1p(exp(z));
+}
+
+__global__ void __launch_bounds__(512) sigmoid_fit_kernel(SolverArgs a) {
+  __shared__ double sm[32 * 5];
+  const int lp = blockIdx.x;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const double* v = a.v + pd.a_off;
+  const double Np = pd.n_s, Nm = pd.n_t;
+  const double hi = (Np + 1.0) / (Np + 2.0), lo = 1.0 / (Nm + 2.0);
+  const int max_iter = 100;
+  const double min_step = 1e-10, sigma = 1e-12, geps = 1e-5;
+  double A = 0.0, B = log((Nm + 1.0) / (Np + 1.0));
+  double F;
+  {
+    double s[1] = {0.0};
+    for (int i = threadIdx.x; i < np; i += blockDim.x) s[0] += nll_term(v[i], i < pd.n_s ? hi : lo, A, B);
+    block_sum_n<1>(s, sm);
+    F = s[0];
+  }
+  int status = 0, it = 0;
+  for (; it < max_iter; ++it) {
+    double h[5] = {0.0, 0.0, 0.0, 0.0, 0.0};  // h11, h22, h21, g1, g2
+    for (int i = threadIdx.x; i < np; i += blockDim.x) {
+      const double vi = v[i], t = i < pd.n_s ? hi : lo;
+      const double z = vi * A + B;
+      double p, q;
+      if (z >= 0.0) {
+        const double e = exp(-z);
+        p = e / (1.0 + e);
+        q = 1.0 / (1.0 + e);
+      } else {
+        const double e = exp(z);
+        p = 1.0 / (1.0 + e);
+        q = e / (1.0 + e);
+      }
+      const double d2 = p * q;
+      h[0] += vi * vi * d2;
+      h[1] += d2;
+      h[2] += vi * d2;
+      const double d1 = t - p;
+      h[3] += vi * d1;
+      h[4] += d1;
+    }
+    block_sum_n<5>(h, sm);
+    const double h11 = h[0] + sigma, h22 = h[1] + sigma, h21 = h[2], g1 = h[3], g2 = h[4];
+    if (fabs(g1) < geps && fabs(g2) < geps) break;
+    const double det = h11 * h22 - h21 * h21;
+    const double dA = -(h22 * g1 - h21 * g2) / det;
+    const double dB = -(-h21 * g1 + h11 * g2) / det;
+    const double gd = g1 * dA + g2 * dB;
+    double step = 1.0;
+    bool found = false;
+    while (step >= min_step && !found) {
+      double fs[4] = {0.0, 0.0, 0.0, 0.0};
+      for (int i = threadIdx.x; i < np; i += blockDim.x) {
+        const double vi = v[i], t = i < pd.n_s ? hi : lo;
+        double st = step;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          fs[c] += nll_term(vi, t, A + st * dA, B + st * dB);
+          st *= 0.5;
+        }
+      }
+      block_sum_n<4>(fs, sm);
+      double st = step;
+      for (int c = 0; c < 4 && st >= min_step; ++c) {
+        if (fs[c] < F + 1e-4 * st * gd) {
+          A += st * dA;
+          B += st * dB;
+          F = fs[c];
+          found = true;
+          break;
+        }
+        st *= 0.5;
+      }
+      step = st;  // if none accepted: continue with the next 4 halvings
+    }
+    if (!found) {
+      status = 2;
+      break;
+    }
+  }
+  if (it >= max_iter) status = 1;
+  if (threadIdx.x == 0) {
+    a.A[lp] = A;
+    a.Bs[lp] = B;
+    a.sig_status[lp] = status;
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// a9: SV union flags over class-sorted positions
+__global__ void sv_flags_kernel(SolverArgs a, uint8_t* flags) {
+  const int lp = blockIdx.x;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const int64_t j = (int64_t)blockIdx.y * blockDim.x + threadIdx.x;
+  if (j < np && a.alpha[pd.a_off + j] > 0.0) flags[gpos(pd, j)] = 1;
+}
+
+// ------------------------------------------------------------------------------------------
+void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st) {
+  const int64_t nthr = tot > P ? tot : P;
+  GM_LAUNCH(init_pairs_kernel, dim3((unsigned)ceil_div(nthr, 256)), dim3(256), 0, st, a, tot, P);
+}
+void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st) {
+  GM_LAUNCH(select_ws_kernel, dim3(P), dim3(1024), 0, st, a, stampv, first);
+}
+void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st) {
+  GM_LAUNCH(gather_kws_kernel, dim3(P, (unsigned)ceil_div(a.B, kGatherRows)), dim3(256), 0, st, a, first);
+}
+void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
+  const int E = (int)ceil_div(a.B, 256);
+  if (E <= 1) GM_LAUNCH(local_smo_kernel<1>, dim3(P), dim3(256), 0, st, a);
+  else if (E == 2) GM_LAUNCH(local_smo_kernel<2>, dim3(P), dim3(256), 0, st, a);
+  else GM_LAUNCH(local_smo_kernel<4>, dim3(P), dim3(256), 0, st, a);
+}
+void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
+  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max, kFCols)), dim3(256), 0, st, a);
+}
+void launch_finalize(const SolverArgs& a, int P, cudaStream_t st) {
+  GM_LAUNCH(finalize_kernel, dim3(P), dim3(1024), 0, st, a);
+}
+void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st) {
+  GM_LAUNCH(sigmoid_fit_kernel, dim3(P), dim3(512), 0, st, a);
+}
+void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st) {
+  GM_LAUNCH(sv_flags_kernel, dim3(P, (unsigned)ceil_div(np_max, 256)), dim3(256), 0, st, a, flags);
+}
+
+}  // namespace gmpsvm

@@ -1,0 +1,157 @@
+// stage.cu -- a1: staging / class grouping (Alg 2 line 3 "getIns", L342).
+//
+// A stable counting sort of the instances by class on the device, so that pair (s,t) is
+// two contiguous class blocks of one class-sorted copy of X (kernel rows shared across
+// pairs, L313-L325).  The sorted copy is stored feature-major (XT[c][j]) and zero-padded
+// to (d_pad x n_pad) for the tile contraction; squared norms are accumulated in FP64.
+#include "kernels.h"
+
+namespace gmpsvm {
+
+// Per-block class histogram of 1024 labels; slot k counts invalid labels.
+__global__ void label_block_count_kernel(const int32_t* __restrict__ y, int64_t n, int k, int32_t* blk_counts) {
+  extern __shared__ int32_t cnt[];
+  for (int c = threadIdx.x; c <= k; c += blockDim.x) cnt[c] = 0;
+  __syncthreads();
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) {
+    const int32_t c = y[i];
+    atomicAdd(&cnt[(c >= 0 && c < k) ? c : k], 1);
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c <= k; c += blockDim.x) blk_counts[(int64_t)blockIdx.x * (k + 1) + c] = cnt[c];
+}
+
+// Exclusive scan of the per-block histograms per class; class sizes and class offsets.
+__global__ void label_scan_kernel(const int32_t* __restrict__ blk_counts, int nb, int k, int32_t* blk_off,
+                                  int64_t* class_count, int64_t* class_off) {
+  for (int c = threadIdx.x; c <= k; c += blockDim.x) {
+    int64_t run = 0;
+    for (int b = 0; b < nb; ++b) {
+      if (c < k) blk_off[(int64_t)b * k + c] = (int32_t)run;
+      run += blk_counts[(int64_t)b * (k + 1) + c];
+    }
+    class_count[c] = run;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int64_t run = 0;
+    for (int c = 0; c < k; ++c) {
+      class_off[c] = run;
+      run += class_count[c];
+    }
+    class_off[k] = run;
+  }
+}
+
+// Stable position of every instance: class_off[c] + (# earlier instances of class c).
+// Labels are validated before this launch.  perm[pos] = original index.
+__global__ void __launch_bounds__(1024) label_rank_kernel(const int32_t* __restrict__ y, int64_t n, int k,
+                                                          const int32_t* __restrict__ blk_off,
+                                                          const int64_t* __restrict__ class_off, int64_t* perm) {
+  extern __shared__ int32_t wcnt[];  // [32][k]
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < 32 * k; i += blockDim.x) wcnt[i] = 0;
+  __syncthreads();
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int c = (i < n) ? y[i] : -1;
+  const unsigned mask = __match_any_sync(0xffffffffu, c);
+  const int rank = __popc(mask & ((1u << lane) - 1u));
+  if (c >= 0 && rank == 0) wcnt[warp * k + c] = __popc(mask);
+  __syncthreads();
+  if (c >= 0) {
+    int before = 0;
+    for (int w = 0; w < warp; ++w) before += wcnt[w * k + c];
+    const int64_t pos = class_off[c] + blk_off[(int64_t)blockIdx.x * k + c] + before + rank;
+    perm[pos] = i;
+  }
+}
+
+// XT[c][j] = X[src(j)][c] for c < d, j < n; zero in the padding.  src(j) = perm ? perm[j] : j.
+__global__ void gather_transpose_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
+                                        float* __restrict__ XT, int64_t ldx, int d_pad, int64_t n_pad) {
+  __shared__ float tile[32][33];
+  const int64_t j0 = (int64_t)blockIdx.x * 32;
+  const int c0 = blockIdx.y * 32;
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  for (int jj = ty; jj < 32; jj += 8) {
+    const int64_t j = j0 + jj;
+    const int c = c0 + tx;
+    float v = 0.f;
+    if (j < n && c < d) {
+      const int64_t src = perm ? perm[j] : j;  // src < 0: padding slot
+      if (src >= 0) v = X[src * d + c];
+    }
+    tile[jj][tx] = v;
+  }
+  __syncthreads();
+  for (int cc = ty; cc < 32; cc += 8) {
+    const int c = c0 + cc;
+    const int64_t j = j0 + tx;
+    if (c < d_pad && j < n_pad) XT[(int64_t)c * ldx + j] = tile[tx][cc];
+  }
+}
+
+// norms[j] = ||X[src(j)]||^2 accumulated in FP64, rounded once to FP32; 0 in the padding.
+// Sets *bad if a row holds a non-finite value (input validation, EINVAL).
+__global__ void row_norms_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
+                                 float* __restrict__ norms, int64_t n_pad, int32_t* bad) {
+  const int64_t j = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (j >= n_pad) return;
+  double s = 0.0;
+  const int64_t src = (j < n) ? (perm ? perm[j] : j) : -1;
+  if (src >= 0) {
+    const float* x = X + src * d;
+    for (int c = lane; c < d; c += 32) {
+      const double v = x[c];
+      s = fma(v, v, s);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) {
+    norms[j] = (float)s;
+    if (bad && !isfinite(s)) atomicExch(bad, 1);
+  }
+}
+
+// Gather rows: dst[r][:] = X[idx[r]][:]  (SV rows of the model, original feature layout)
+__global__ void gather_rows_kernel(const float* __restrict__ X, int d, const int64_t* __restrict__ idx, int64_t nr,
+                                   float* __restrict__ dst) {
+  const int64_t r = blockIdx.x;
+  if (r >= nr) return;
+  const float* s = X + idx[r] * d;
+  float* o = dst + r * d;
+  for (int c = threadIdx.x; c < d; c += blockDim.x) o[c] = s[c];
+}
+
+void launch_class_sort(const int32_t* y, int64_t n, int k, int32_t* blk_counts, int32_t* blk_off,
+                       int64_t* class_count, int64_t* class_off, cudaStream_t st) {
+  const int nb = (int)ceil_div(n, 1024);
+  GM_LAUNCH(label_block_count_kernel, dim3(nb), dim3(1024), (size_t)(k + 1) * sizeof(int32_t), st, y, n, k,
+            blk_counts);
+  GM_LAUNCH(label_scan_kernel, dim3(1), dim3(std::min(1024, k + 1)), 0, st, blk_counts, nb, k, blk_off, class_count,
+            class_off);
+}
+
+void launch_class_rank(const int32_t* y, int64_t n, int k, const int32_t* blk_off, const int64_t* class_off,
+                       int64_t* perm, cudaStream_t st) {
+  const int nb = (int)ceil_div(n, 1024);
+  GM_LAUNCH(label_rank_kernel, dim3(nb), dim3(1024), (size_t)32 * k * sizeof(int32_t), st, y, n, k, blk_off,
+            class_off, perm);
+}
+
+void launch_stage_features(const float* X, int64_t n, int d, const int64_t* perm, float* XT, int64_t ldx, int d_pad,
+                           int64_t n_pad, float* norms, int32_t* bad, cudaStream_t st) {
+  GM_LAUNCH(gather_transpose_kernel, dim3((unsigned)ceil_div(n_pad, 32), (unsigned)ceil_div(d_pad, 32)), dim3(32, 8), 0,
+            st, X, n, d, perm, XT, ldx, d_pad, n_pad);
+  GM_LAUNCH(row_norms_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, norms, n_pad, bad);
+}
+
+void launch_gather_rows(const float* X, int d, const int64_t* idx, int64_t nr, float* dst, cudaStream_t st) {
+  if (nr <= 0) return;
+  GM_LAUNCH(gather_rows_kernel, dim3((unsigned)nr), dim3(128), 0, st, X, d, idx, nr, dst);
+}
+
+}  // namespace gmpsvm
