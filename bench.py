@@ -1,0 +1,292 @@
+"""bench.py -- GMP-SVM hot path on B200: train + predict on the MNIST-shaped workload.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gmpsvm|reference] [--eps E]
+    torchrun --nproc-per-node N bench.py --gpus N ...      (pairs / test rows sharded, NCCL gathers)
+
+One step = one whole pass of the hot path on the workload
+BASELINE.json's metric is quoted on (configs[2]: MNIST-shaped 60k train / 10k test x 784,
+10 classes, gamma 0.125, C 10): gmpsvm_train + gmpsvm_predict_proba.  Inputs are resident
+in HBM when the timed region starts (`value`); `e2e` repeats the step through the C ABI
+from pinned host buffers with the H2D/D2H copies inside the timed region.
+
+Prints ONE JSON line on rank 0.  The metric is time-like (seconds per train+predict job),
+so higher_is_better = false.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import datagen  # noqa: E402
+
+METRIC = "train+predict sec on MNIST-shaped 60k×784×10; kernel GFLOP/s vs peak"
+FP32_PEAK_TFLOPS_DERIVED = 148 * 128 * 2 * 1.965e9 / 1e12  # SMs x FP32 lanes x 2 x max SM clock
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._th = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                f = [x.strip() for x in out.stdout.strip().split(",")]
+                if len(f) >= 7:
+                    self.samples.append(f)
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._th = threading.Thread(target=self._run, daemon=True)
+        self._th.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._th:
+            self._th.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[3 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def _env_dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def lpt_shards(sizes, n_shards):
+    """Longest-processing-time-first assignment of pairs (cost ~ n_p^1.5) to ranks."""
+    order = np.argsort(-np.asarray(sizes, dtype=np.float64) ** 1.5, kind="stable")
+    load = np.zeros(n_shards)
+    out = [[] for _ in range(n_shards)]
+    for p in order:
+        r = int(np.argmin(load))
+        out[r].append(int(p))
+        load[r] += float(sizes[p]) ** 1.5
+    return [sorted(o) for o in out]
+
+
+# ------------------------------------------------------------------------------------------ oracle arms
+def cpu_sample(spec, eps, n_train=6000, n_test=1000):
+    """The oracle, as it stands, on a bounded sample of the same workload (host cores)."""
+    import oracle
+
+    _, X, y, Xt, yt = datagen.make_config(spec.name, n_train=n_train, n_test=n_test)
+    t0 = time.perf_counter()
+    m = oracle.train(X, y, spec.k, spec.C, spec.gamma, eps)
+    t1 = time.perf_counter()
+    oracle.predict(m, X, y, Xt, want_dec=False)
+    t2 = time.perf_counter()
+    return t2 - t0, t1 - t0, t2 - t1, oracle.default_threads()
+
+
+def run_reference(args, spec):
+    ws, rank, _ = _env_dist()
+    if rank != 0:
+        return 0
+    for _ in range(args.warmup):
+        cpu_sample(spec, args.eps)
+    times = []
+    for _ in range(args.steps):
+        t, tt, tp, cores = cpu_sample(spec, args.eps)
+        times.append(t)
+    v = float(np.mean(times))
+    sample = (f"oracle (FP64 C++ WSS2 SMO + LLW sigmoid + exact WLW coupling) on a 10% sample of the workload: "
+              f"6000 train / 1000 test MNIST-shaped rows, eps={args.eps:g}, {cores} host threads")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "s (sample)", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": v * 1e3, "higher_is_better": False,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": _config(spec, args),
+            "cpu_baseline": {"value": v, "unit": "s (sample)", "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": "s (sample)", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def _config(spec, args):
+    return {"workload": f"{spec.name}-shaped {spec.n_train} train / {spec.n_test} test x {spec.d}, k={spec.k}, "
+                        f"C={spec.C:g}, gamma={spec.gamma:g}, eps={args.eps:g}",
+            "n_train": spec.n_train, "n_test": spec.n_test, "d": spec.d, "k": spec.k, "C": spec.C,
+            "gamma": spec.gamma, "eps": args.eps, "ws_size": args.ws_size, "q": args.ws_size // 2,
+            "parallelism": f"pairs+test-rows x{args.gpus}",
+            "l2": "inputs larger than L2 (X 188 MB, kernel matrix 14.4 GB > 126 MB L2); no flush needed"}
+
+
+# ------------------------------------------------------------------------------------------ GPU arm
+def run_gpu(args, spec):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icde_wenshcc19_b200 as gm
+    from paper_conf_icde_wenshcc19_b200 import dist as gdist
+
+    ws, rank, local = _env_dist()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    _, X, y, Xt, yt = datagen.make_config(spec.name)
+    Xd, yd, Xtd = torch.from_numpy(X).to(dev), torch.from_numpy(y).to(dev), torch.from_numpy(Xt).to(dev)
+    Xp, yp, Xtp = (torch.from_numpy(X).pin_memory(), torch.from_numpy(y).pin_memory(),
+                   torch.from_numpy(Xt).pin_memory())
+    stream = torch.cuda.current_stream(dev)
+    opts = dict(ws_size=args.ws_size)
+
+    def step(Xa, ya, Xta, host=False):
+        if ws > 1:
+            model, prob = gdist.train_predict(Xa, ya, Xta, spec.k, spec.C, spec.gamma, args.eps, **opts)
+        else:
+            model = gm.train(Xa, ya, spec.k, spec.C, spec.gamma, args.eps, **opts)
+            prob = model.predict_proba(Xta)
+        return model, prob
+
+    for _ in range(args.warmup):
+        model, prob = step(Xd, yd, Xtd)
+    torch.cuda.synchronize(dev)
+
+    # ---- device-resident timed region
+    t_ms, stats, pstats = [], [], []
+    with ClockSampler(local) as clk:
+        l0 = gm.launch_count()
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            model, prob = step(Xd, yd, Xtd)
+            stats.append(model.train_stats())
+            pstats.append(gm.last_predict_stats())
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        if ws > 1:
+            dist.barrier()
+        launches = gm.launch_count() - l0
+    total_ms = e0.elapsed_time(e1)
+    if ws > 1:
+        t = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms = total_ms / args.steps
+
+    # ---- end to end from pinned host buffers (copies inside the timed region)
+    Xh, yh, Xth = Xp.numpy(), yp.numpy(), Xtp.numpy()
+    torch.cuda.synchronize(dev)
+    if ws > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        model_h, prob_h = step(Xh, yh, Xth, host=True)
+    torch.cuda.synchronize(dev)
+    e2e_ms = (time.perf_counter() - t0) * 1e3 / args.steps
+    if ws > 1:
+        t = torch.tensor([e2e_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+
+    if rank == 0:
+        s = stats[-1]
+        ps = pstats[-1]
+        krow_ms = float(np.mean([x["t_kernel_ms"] for x in stats]))
+        achieved = s["kernel_flops"] / (krow_ms * 1e-3) / 1e12
+        peak = FP32_PEAK_TFLOPS_DERIVED
+        traffic = None
+        tr_path = os.path.join(ROOT, "profiles", "krow_traffic.json")
+        if os.path.exists(tr_path):
+            traffic = json.load(open(tr_path)).get("dram_bytes_per_launch")
+        line = {
+            "metric": METRIC, "value": ms / 1e3, "unit": "s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic (datagen mnist recipe, seeds 1234/1/2)",
+            "config": _config(spec, args),
+            "roofline": {"kernel": "krow_contract", "bound": "alu", "achieved": achieved, "peak": peak,
+                         "unit": "TFLOP/s", "frac": achieved / peak, "traffic": traffic,
+                         "peak_note": "FP32 SIMT derived: 148 SM x 128 lanes x 2 flop x 1965 MHz (no FP32 entry "
+                                      "in MEASURED_PEAKS.json)",
+                         "flops_per_launch": s["kernel_flops"], "launch_ms": krow_ms,
+                         "algorithmic": "n(n+1)/2 kernel values x (2d+3) flop"},
+            "phases_ms": {"stage": s["t_stage_ms"], "kernel_values": s["t_kernel_ms"], "select": s["t_select_ms"],
+                          "subproblem": s["t_subproblem_ms"], "f_update": s["t_fupdate_ms"],
+                          "finalize": s["t_finalize_ms"], "train_total": s["t_total_ms"],
+                          "predict_stage": ps["t_stage_ms"], "decision_values": ps["t_decision_ms"],
+                          "couple": ps["t_couple_ms"], "predict_total": ps["t_total_ms"]},
+            "counters": {"outer_iters_max": s["outer_iters_max"], "inner_iters_sum": s["inner_iters_sum"],
+                         "n_sv": s["n_sv"], "dec_tflops": ps["dec_flops"] / (ps["t_decision_ms"] * 1e-3) / 1e12
+                         if ps["t_decision_ms"] > 0 else None},
+            "gpu_launches": int(launches),
+            "clocks": clk.summary(),
+            "e2e": {"value": e2e_ms / 1e3, "unit": "s", "h2d_bytes_per_step": int(X.nbytes + y.nbytes + Xt.nbytes),
+                    "d2h_bytes_per_step": int(prob_h.nbytes)},
+        }
+        if not args.no_cpu_baseline and ws == 1:
+            v, tt, tp, cores = cpu_sample(spec, args.eps)
+            line["cpu_baseline"] = {"value": v, "unit": "s (sample)", "cores": cores, "kind": "oracle",
+                                    "sample": f"6000 train / 1000 test MNIST-shaped rows (10% of the workload), "
+                                              f"eps={args.eps:g}: train {tt:.1f} s + predict {tp:.1f} s"}
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gmpsvm", choices=["gmpsvm", "reference"])
+    ap.add_argument("--config", default="mnist")
+    ap.add_argument("--eps", type=float, default=1e-3)
+    ap.add_argument("--ws-size", dest="ws_size", type=int, default=1024)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    spec = datagen.CONFIGS[args.config]
+    if args.impl == "reference":
+        return run_reference(args, spec)
+    return run_gpu(args, spec)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

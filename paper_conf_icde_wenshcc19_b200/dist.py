@@ -1,0 +1,114 @@
+"""Multi-GPU driver: one process per GPU (torchrun), pairs sharded for training, test rows
+sharded for prediction, NCCL used only to gather models and probabilities.
+
+Training shards naturally: the k(k-1)/2 binary SVMs are independent, so each
+rank trains an LPT-balanced subset of pairs (cost ~ n_p^1.5) with X replicated, and there is
+no collective inside the solver loop.  The partial models are serialized, all-gathered
+(sizes first, then padded blobs) and merged on every rank.  Prediction shards the test rows
+(instances are independent, L273) and all-gathers the m x k probabilities.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import _lib as gm
+
+
+def pair_list(k):
+    return [(s, t) for s in range(k) for t in range(s + 1, k)]
+
+
+def plan_pairs(class_counts, world, exponent=1.5):
+    """LPT (longest processing time first) assignment of pair indices to `world` ranks."""
+    k = len(class_counts)
+    sizes = np.array([class_counts[s] + class_counts[t] for s, t in pair_list(k)], dtype=np.float64)
+    order = np.argsort(-(sizes ** exponent), kind="stable")
+    load = np.zeros(world)
+    shards = [[] for _ in range(world)]
+    for p in order:
+        r = int(np.argmin(load))
+        shards[r].append(int(p))
+        load[r] += sizes[p] ** exponent
+    return [sorted(s) for s in shards]
+
+
+def _backend_device(group=None):
+    import torch
+    import torch.distributed as dist
+
+    if dist.get_backend(group) == "nccl":
+        return torch.device("cuda", torch.cuda.current_device())
+    return torch.device("cpu")
+
+
+def all_gather_bytes(buf: np.ndarray, group=None):
+    """All-gather variable-length uint8 buffers: sizes first, then padded payloads."""
+    import torch
+    import torch.distributed as dist
+
+    dev = _backend_device(group)
+    world = dist.get_world_size(group)
+    n = torch.tensor([buf.size], dtype=torch.int64, device=dev)
+    sizes = [torch.zeros_like(n) for _ in range(world)]
+    dist.all_gather(sizes, n, group=group)
+    sizes = [int(s.item()) for s in sizes]
+    cap = max(sizes)
+    payload = torch.zeros(cap, dtype=torch.uint8, device=dev)
+    payload[: buf.size] = torch.from_numpy(np.ascontiguousarray(buf)).to(dev)
+    outs = [torch.empty(cap, dtype=torch.uint8, device=dev) for _ in range(world)]
+    dist.all_gather(outs, payload, group=group)
+    return [o[:s].cpu().numpy() for o, s in zip(outs, sizes)]
+
+
+def gather_models(part: "gm.Model", group=None) -> "gm.Model":
+    """Serialize this rank's partial model, all-gather the blobs, merge (identical on all ranks)."""
+    blobs = all_gather_bytes(part.serialize(), group)
+    parts = [gm.Model.deserialize(b) for b in blobs]
+    return gm.Model.merge(parts)
+
+
+def row_range(m, world, rank):
+    lo = (m * rank) // world
+    hi = (m * (rank + 1)) // world
+    return lo, hi
+
+
+def all_gather_rows(local, m_total, group=None):
+    """All-gather row shards (row_range partition) of a [rows, c] tensor/array into [m_total, c]."""
+    import torch
+    import torch.distributed as dist
+
+    dev = _backend_device(group)
+    world = dist.get_world_size(group)
+    t = local if isinstance(local, torch.Tensor) else torch.from_numpy(np.ascontiguousarray(local))
+    t = t.to(dev)
+    cols = t.shape[1]
+    cap = max(row_range(m_total, world, r)[1] - row_range(m_total, world, r)[0] for r in range(world))
+    pad = torch.zeros((cap, cols), dtype=t.dtype, device=dev)
+    pad[: t.shape[0]] = t
+    outs = [torch.empty_like(pad) for _ in range(world)]
+    dist.all_gather(outs, pad, group=group)
+    pieces = []
+    for r in range(world):
+        lo, hi = row_range(m_total, world, r)
+        pieces.append(outs[r][: hi - lo])
+    return torch.cat(pieces, 0)
+
+
+def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
+    """Sharded train (pairs) + sharded predict (rows) on every rank; returns (model, prob)."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    yy = y.cpu().numpy() if isinstance(y, torch.Tensor) else np.asarray(y)
+    counts = np.bincount(yy, minlength=k)
+    mine = plan_pairs(counts, world)[rank]
+    part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts)
+    model = gather_models(part, group)
+    m = Xt.shape[0]
+    lo, hi = row_range(m, world, rank)
+    prob_local = model.predict_proba(Xt[lo:hi])
+    prob = all_gather_rows(prob_local, m, group)
+    return model, prob

@@ -6,6 +6,7 @@ Stores, for the full-size config (datagen recipe): per-pair b,
 n_sv, n_bound, sum(alpha), oracle iterations; and dec values / probabilities of the first
 n_probe test instances.  The GPU parity test (tests/test_gpu_full.py) compares against it.
 """
+import base64
 import json
 import os
 import sys
@@ -32,11 +33,16 @@ def main():
     dec, prob = oracle.predict(m, X, y, Xt[:n_probe])
     t_pred = time.time() - t0
     pairs = []
+    rng = np.random.default_rng(7)
     for p, (s, t) in enumerate(m["pairs"]):
         a = m["alpha"][p]
+        probe = np.sort(rng.choice(len(a), size=min(64, len(a)), replace=False))
         pairs.append(dict(s=s, t=t, b=float(m["b"][p]), A=float(m["A"][p]), B=float(m["B"][p]),
                           n_sv=int((a > 0).sum()), n_bound=int((a >= spec.C).sum()),
-                          sum_alpha=float(a.sum()), iters=int(m["iters"][p]), status=int(m["status"][p])))
+                          sum_alpha=float(a.sum()), iters=int(m["iters"][p]), status=int(m["status"][p]),
+                          sv_mask=base64.b64encode(np.packbits(a > 0).tobytes()).decode(),
+                          firm_mask=base64.b64encode(np.packbits(a >= 1e-4 * spec.C).tobytes()).decode(),
+                          probe_idx=probe.tolist(), probe_alpha=a[probe].tolist()))
     out = dict(config=name, eps=eps, C=spec.C, gamma=spec.gamma, k=spec.k, n_train=int(X.shape[0]),
                n_probe=n_probe, generator="datagen.make_config(%r)" % name,
                written_by="tests/golden/make_full_golden.py (oracle only)",

@@ -104,7 +104,7 @@ def _compare_models(gm_model, ref, X, y, spec_C, eps=EPS, audit=True):
         assert np.abs(a_g - a_o).max() <= 1e-3 * C, (p, np.abs(a_g - a_o).max())
         sv_g, sv_o = a_g > 0, a_o > 0
         diff = sv_g != sv_o
-        tie = (np.minimum(a_g, a_o) < 1e-4 * C) | (np.maximum(a_g, a_o) < 1e-4 * C)
+        tie = np.maximum(a_g, a_o) < 1e-4 * C  # SV in one solution only: its alpha must be tiny
         assert np.all(tie[diff]), (p, np.flatnonzero(diff & ~tie))
         ties += int(diff.sum())
         assert abs(info["b"] - ref["b"][p]) <= 1e-3 * max(1.0, abs(ref["b"][p])), (p, info["b"], ref["b"][p])
@@ -170,7 +170,25 @@ def test_hyperparameter_grid_blobs(gm, C, gamma):
     model = gm.train(X, y, spec.k, C, gamma, EPS)
     _compare_models(model, ref, X, y, C, audit=(C <= 10))
     _, prob_o = oracle.predict(ref, X, y, Xt, want_dec=False)
-    assert np.abs(model.predict_proba(Xt) - prob_o).max() <= 1e-4
+    assert np.abs(model.predict_proba(Xt) - prob_o).max() <= _prob_tol(ref, X, y, Xt)
+
+
+def _prob_tol(ref, X, y, Xt):
+    """1e-4, widened only where FP32 kernel values cannot carry it (R27):
+    |d dec| <= 4 * 2^-24 * max_i sum_j |coef_j| K_ij (representation + rounding of K in FP32), and
+    |d p| <= max|A|/4 * |d dec| per pair probability (dP/d dec = A P (1-P))."""
+    k = ref["k"]
+    worst = 0.0
+    for p, (s, t) in enumerate(ref["pairs"]):
+        idx, ypm = oracle.pair_members(y, k, s, t)
+        a = ref["alpha"][p]
+        sv = a > 0
+        if not sv.any():
+            continue
+        Kt = oracle.rbf_matrix(Xt, X[idx][sv], ref["gamma"])
+        mass = (Kt * a[sv]).sum(1).max()
+        worst = max(worst, abs(ref["A"][p]) / 4 * 4 * 2.0 ** -24 * mass)
+    return 1e-4 + worst
 
 
 @pytest.mark.parametrize("ws,q", [(64, 32), (128, 64), (256, 128), (64, 16)])
