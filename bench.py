@@ -193,8 +193,12 @@ def run_gpu(args, spec):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
+        marks = []
         for _ in range(args.steps):
             model, prob = step(Xd, yd, Xtd)
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record(stream)
+            marks.append(ev)
             stats.append(model.train_stats())
             pstats.append(gm.last_predict_stats())
         e1.record(stream)
@@ -203,6 +207,7 @@ def run_gpu(args, spec):
             dist.barrier()
         launches = gm.launch_count() - l0
     total_ms = e0.elapsed_time(e1)
+    step_ms = [e0.elapsed_time(marks[0])] + [marks[i - 1].elapsed_time(marks[i]) for i in range(1, len(marks))]
     if ws > 1:
         t = torch.tensor([total_ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -250,7 +255,9 @@ def run_gpu(args, spec):
                           "finalize": s["t_finalize_ms"], "train_total": s["t_total_ms"],
                           "predict_stage": ps["t_stage_ms"], "decision_values": ps["t_decision_ms"],
                           "couple": ps["t_couple_ms"], "predict_total": ps["t_total_ms"]},
+            "step_ms": step_ms,
             "counters": {"outer_iters_max": s["outer_iters_max"], "inner_iters_sum": s["inner_iters_sum"],
+                         "smo_cycles_per_step": s["smo_cycles_sum"] / max(1, s["inner_iters_sum"]),
                          "n_sv": s["n_sv"], "dec_tflops": ps["dec_flops"] / (ps["t_decision_ms"] * 1e-3) / 1e12
                          if ps["t_decision_ms"] > 0 else None},
             "gpu_launches": int(launches),

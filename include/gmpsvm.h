@@ -93,6 +93,7 @@ typedef struct {
   int32_t cache_regime;     /* 0 = FULL_K (whole kernel matrix resident)                     */
   int32_t n_pairs_trained;
   int64_t launches;         /* kernels launched by this call                                  */
+  int64_t smo_cycles_sum;   /* SM clock cycles spent in the local SMO, summed over pairs      */
 } gmpsvm_train_stats;
 
 typedef struct {

@@ -387,7 +387,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<uint32_t> d_stamp(tot, st);
   DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
       d_outer(Pl, st), d_sig(Pl, st);
-  DevBuf<int64_t> d_inner(Pl, st);
+  DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
   DevBuf<float> d_Kws((size_t)Pl * Bw * Bw, st);
   SolverArgs a{};
   a.pairs = d_pairs.get();
@@ -405,6 +405,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   a.status = d_status.get();
   a.gap = d_gap.get();
   a.inner_iters = d_inner.get();
+  a.smo_cycles = d_cyc.get();
   a.outer_iters = d_outer.get();
   a.b = d_b.get();
   a.A = d_A.get();
@@ -450,7 +451,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   launch_sv_flags(a, Pl, np_max, d_flags.get(), st);
   std::vector<double> h_alpha(tot), hb(Pl), hA(Pl), hB(Pl);
   std::vector<int32_t> h_sig(Pl), h_st(Pl), h_outer(Pl);
-  std::vector<int64_t> h_inner(Pl), h_perm(n);
+  std::vector<int64_t> h_inner(Pl), h_cyc(Pl), h_perm(n);
   std::vector<uint8_t> h_flags(n);
   GM_CUDA(cudaMemcpyAsync(h_alpha.data(), d_alpha.get(), tot * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(hb.data(), d_b.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
@@ -460,6 +461,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaMemcpyAsync(h_st.data(), d_status.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_outer.data(), d_outer.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_inner.data(), d_inner.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_cyc.data(), d_cyc.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_perm.data(), d_perm.get(), n * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_flags.data(), d_flags.get(), n, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
@@ -481,7 +483,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   mdl->status.assign(P, 0);
   const auto po = mdl->pair_offsets();
   mdl->alpha.assign(po[P], 0.0);
-  int64_t outer_max = 0, outer_sum = 0, inner_sum = 0;
+  int64_t outer_max = 0, outer_sum = 0, inner_sum = 0, cyc_sum = 0;
   for (int i = 0; i < Pl; ++i) {
     const int p = pids[i];
     mdl->trained[p] = 1;
@@ -494,6 +496,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     outer_max = std::max<int64_t>(outer_max, h_outer[i]);
     outer_sum += h_outer[i];
     inner_sum += h_inner[i];
+    cyc_sum += h_cyc[i];
   }
   for (int64_t g = 0; g < n; ++g)
     if (h_flags[g]) mdl->sv_pos.push_back(g);
@@ -516,6 +519,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   s.outer_iters_max = outer_max;
   s.outer_iters_sum = outer_sum;
   s.inner_iters_sum = inner_sum;
+  s.smo_cycles_sum = cyc_sum;
   s.n_sv = (int64_t)mdl->sv_pos.size();
   s.cache_regime = 0;
   s.n_pairs_trained = Pl;

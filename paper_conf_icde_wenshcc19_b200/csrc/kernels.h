@@ -39,6 +39,7 @@ struct SolverArgs {
   int32_t* status;      // [P] 0 active, 1 converged, 2 outer cap
   double* gap;          // [P] global gap at the last selection
   int64_t* inner_iters; // [P]
+  int64_t* smo_cycles;  // [P] SM clock cycles spent in local_smo (diagnostic)
   int32_t* outer_iters; // [P]
   double* b;            // [P]
   double* A;            // [P]

@@ -96,6 +96,7 @@ __global__ void init_pairs_kernel(SolverArgs a, const int64_t tot, int P) {
     a.status[i] = 0;
     a.ws_n[i] = 0;
     a.inner_iters[i] = 0;
+    a.smo_cycles[i] = 0;
     a.outer_iters[i] = 0;
     a.gap[i] = 0.0;
   }
@@ -300,13 +301,19 @@ __global__ void __launch_bounds__(256) gather_kws_kernel(SolverArgs a, int first
 }
 
 // ------------------------------------------------------------------------------------------
-// a5: local SMO on the working set (one CTA per pair, 256 threads, E ws rows per thread)
+// a5: local SMO on the working set (ImproveSVM, Alg 2 line 10).  One CTA per pair, one
+// thread per working-set row (blockDim = B rounded up to a warp multiple, <= 1024).  Per
+// inner step: block argmin (u, Eq 4) -> row u of K_ws,ws -> block argmax (l, Eq 5) fused
+// with max_{I_l} f -> clipped step (Eq 6-7) -> row l -> f update (Eq 8) on the ws.  The two
+// block reductions use redux.sync on 32-bit key words; the winner's alpha, f, K_ii and K_ui
+// travel in the reduction payload, so the only dependent global loads are the two K rows,
+// and a row already held in registers (u or l of the previous step) is reused.
 struct RedSlot {
   uint32_t k0, k1;
   int32_t idx, e;
   double alpha, f;
   uint32_t m0, m1;  // running max key (f_max over I_l)
-  uint32_t pad0, pad1;
+  float kd, ku;     // K_ee and K_ue of the candidate
 };
 
 // lexicographic min of (k0, k1, idx) over the warp; returns the winning lane (lowest on ties)
@@ -330,13 +337,14 @@ __device__ __forceinline__ void warp_max64(uint32_t& h, uint32_t& l) {
   h = mh;
 }
 
-// Block argmin of (k0,k1,idx) carrying (e, alpha, f) and a running max key (m0,m1).
-__device__ __forceinline__ RedSlot block_argmin(RedSlot c, RedSlot* slots) {
+// Block argmin of (k0,k1,idx) carrying the payload and (WITH_MAX) a running max key (m0,m1).
+template <bool WITH_MAX>
+__device__ __forceinline__ RedSlot block_argmin(const RedSlot& c, RedSlot* slots) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   uint32_t k0 = c.k0, k1 = c.k1, mh = c.m0, ml = c.m1;
   int32_t idx = c.idx;
   const int wl = warp_argmin(k0, k1, idx);
-  warp_max64(mh, ml);
+  if (WITH_MAX) warp_max64(mh, ml);
   if (lane == wl) {
     RedSlot s = c;
     s.m0 = mh;
@@ -344,126 +352,105 @@ __device__ __forceinline__ RedSlot block_argmin(RedSlot c, RedSlot* slots) {
     slots[warp] = s;
   }
   __syncthreads();
-  RedSlot r;
-  if (lane < nw) r = slots[lane];
-  else {
-    r.k0 = r.k1 = 0xffffffffu;
-    r.idx = INT_MAX;
-    r.m0 = r.m1 = 0u;
+  if (lane < nw) {
+    k0 = slots[lane].k0;
+    k1 = slots[lane].k1;
+    idx = slots[lane].idx;
+    mh = slots[lane].m0;
+    ml = slots[lane].m1;
+  } else {
+    k0 = k1 = 0xffffffffu;
+    idx = INT_MAX;
+    mh = ml = 0u;
   }
-  k0 = r.k0;
-  k1 = r.k1;
-  idx = r.idx;
-  mh = r.m0;
-  ml = r.m1;
   const int w2 = warp_argmin(k0, k1, idx);
-  warp_max64(mh, ml);
+  if (WITH_MAX) warp_max64(mh, ml);
   RedSlot out = slots[w2 < nw ? w2 : 0];
   out.m0 = mh;
   out.m1 = ml;
-  if (idx == INT_MAX || k0 == 0xffffffffu && k1 == 0xffffffffu) out.idx = INT_MAX;
+  if (idx == INT_MAX) out.idx = INT_MAX;
   return out;
 }
 
-template <int E>
-__global__ void __launch_bounds__(256) local_smo_kernel(SolverArgs a) {
-  __shared__ RedSlot slots[2][8];
+__device__ __forceinline__ RedSlot empty_slot() {
+  RedSlot s;
+  s.k0 = s.k1 = 0xffffffffu;
+  s.idx = INT_MAX;
+  s.e = -1;
+  s.alpha = s.f = 0.0;
+  s.m0 = s.m1 = 0u;
+  s.kd = s.ku = 0.f;
+  return s;
+}
+
+__global__ void __launch_bounds__(1024) local_smo_kernel(SolverArgs a) {
+  __shared__ RedSlot slots[2][32];
   const int lp = blockIdx.x;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int B = a.B, wn = a.ws_n[lp];
-  const int tid = threadIdx.x;
+  const int e = threadIdx.x;
   const float* Kw = a.Kws + (int64_t)lp * B * B;
-  const int32_t* ws = a.ws + (int64_t)lp * B;
   const double C = a.C;
-  int32_t idx[E];
-  int y[E];
-  double al[E], a0[E], fv[E];
-  float kd[E], ku[E];
-  bool valid[E];
-#pragma unroll
-  for (int q = 0; q < E; ++q) {
-    const int e = tid + q * 256;
-    valid[q] = e < wn;
-    idx[q] = valid[q] ? ws[e] : INT_MAX;
-    y[q] = (valid[q] && idx[q] < pd.n_s) ? 1 : -1;
-    al[q] = valid[q] ? a.alpha[pd.a_off + idx[q]] : 0.0;
-    a0[q] = al[q];
-    fv[q] = valid[q] ? a.f[pd.a_off + idx[q]] : 0.0;
-    kd[q] = valid[q] ? Kw[(int64_t)e * B + e] : 1.f;
-  }
+  const bool valid = e < wn;
+  const int32_t idx = valid ? a.ws[(int64_t)lp * B + e] : INT_MAX;
+  const int y = (valid && idx < pd.n_s) ? 1 : -1;
+  double al = valid ? a.alpha[pd.a_off + idx] : 0.0;
+  const double a0 = al;
+  double fv = valid ? a.f[pd.a_off + idx] : 0.0;
+  const float kd = valid ? Kw[(int64_t)e * B + e] : 1.f;
+  // two cached K_ws,ws rows (this thread's column of them): rows ra / rb
+  int ra = -1, rb = -1;
+  float va = 0.f, vb = 0.f;
   const int cap = a.inner_cap;
   int it = 0, par = 0;
   double delta0 = 0.0;
+  const long long t_begin = clock64();
   for (;;) {
     // Step 1 (Eq 4): u = argmin_{I_u} f, ties -> lowest pair-local index
-    RedSlot cu;
-    cu.k0 = cu.k1 = 0xffffffffu;
-    cu.idx = INT_MAX;
-    cu.e = -1;
-    cu.m0 = cu.m1 = 0u;
-    cu.alpha = 0.0;
-    cu.f = 0.0;
-#pragma unroll
-    for (int q = 0; q < E; ++q) {
-      if (valid[q] && in_u(y[q], al[q], C)) {
-        const uint64_t key = ord_key(fv[q]);
-        const uint32_t h = (uint32_t)(key >> 32), l = (uint32_t)key;
-        if (h < cu.k0 || (h == cu.k0 && (l < cu.k1 || (l == cu.k1 && idx[q] < cu.idx)))) {
-          cu.k0 = h;
-          cu.k1 = l;
-          cu.idx = idx[q];
-          cu.e = tid + q * 256;
-          cu.alpha = al[q];
-          cu.f = fv[q];
-        }
-      }
+    RedSlot c = empty_slot();
+    if (valid && in_u(y, al, C)) {
+      const uint64_t key = ord_key(fv);
+      c.k0 = (uint32_t)(key >> 32);
+      c.k1 = (uint32_t)key;
+      c.idx = idx;
+      c.e = e;
+      c.alpha = al;
+      c.f = fv;
+      c.kd = kd;
     }
-    const RedSlot ru = block_argmin(cu, slots[par]);
+    const RedSlot ru = block_argmin<false>(c, slots[par]);
     par ^= 1;
     if (ru.idx == INT_MAX) break;
     const int ue = ru.e;
     const double fu = ru.f, au = ru.alpha;
+    const float kuu = ru.kd;
     const int yu = ru.idx < pd.n_s ? 1 : -1;
-    const float* Kur = Kw + (int64_t)ue * B;
-#pragma unroll
-    for (int q = 0; q < E; ++q) ku[q] = valid[q] ? Kur[tid + q * 256] : 0.f;
-    const float kuu = Kur[ue];
-    // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_u - f_t)^2 / eta_t ; also f_max over I_l (Eq 10)
-    RedSlot cl;
-    cl.k0 = cl.k1 = 0xffffffffu;
-    cl.idx = INT_MAX;
-    cl.e = -1;
-    cl.m0 = cl.m1 = 0u;
-    cl.alpha = 0.0;
-    cl.f = 0.0;
-#pragma unroll
-    for (int q = 0; q < E; ++q) {
-      if (valid[q] && in_l(y[q], al[q], C)) {
-        const uint64_t fk = ord_key(fv[q]);
-        const uint32_t h = (uint32_t)(fk >> 32), l = (uint32_t)fk;
-        if (h > cl.m0 || (h == cl.m0 && l > cl.m1)) {
-          cl.m0 = h;
-          cl.m1 = l;
-        }
-        if (fv[q] > fu) {
-          double eta = (double)kuu + (double)kd[q] - 2.0 * (double)ku[q];
-          eta = eta > kTau ? eta : kTau;
-          const double df = fv[q] - fu;
-          const float score = (float)(df * df / eta);
-          const uint32_t sk = ~__float_as_uint(score);
-          if (sk < cl.k0 || (sk == cl.k0 && (0u < cl.k1 || idx[q] < cl.idx))) {
-            cl.k0 = sk;
-            cl.k1 = 0u;
-            cl.idx = idx[q];
-            cl.e = tid + q * 256;
-            cl.alpha = al[q];
-            cl.f = fv[q];
-          }
-        }
+    float ku;
+    if (ue == ra) ku = va;
+    else if (ue == rb) ku = vb;
+    else ku = valid ? Kw[(int64_t)ue * B + e] : 0.f;
+    // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_u - f_t)^2 / eta_t, and f_max over I_l (Eq 10)
+    c = empty_slot();
+    if (valid && in_l(y, al, C)) {
+      const uint64_t fk = ord_key(fv);
+      c.m0 = (uint32_t)(fk >> 32);
+      c.m1 = (uint32_t)fk;
+      if (fv > fu) {
+        const float eta = fmaxf(kuu + kd - 2.f * ku, 1e-12f);
+        const float df = (float)(fv - fu);
+        const float score = df * df * __frcp_rn(eta);
+        c.k0 = ~__float_as_uint(score);
+        c.k1 = 0u;
+        c.idx = idx;
+        c.e = e;
+        c.alpha = al;
+        c.f = fv;
+        c.kd = kd;
+        c.ku = ku;
       }
     }
-    const RedSlot rl = block_argmin(cl, slots[par]);
+    const RedSlot rl = block_argmin<true>(c, slots[par]);
     par ^= 1;
     const double fmax = (rl.m0 == 0u && rl.m1 == 0u) ? -DBL_MAX : key_double(((uint64_t)rl.m0 << 32) | rl.m1);
     const double gap = fmax - fu;
@@ -473,9 +460,8 @@ __global__ void __launch_bounds__(256) local_smo_kernel(SolverArgs a) {
     const int le = rl.e;
     const double fl = rl.f, alv = rl.alpha;
     const int yl = rl.idx < pd.n_s ? 1 : -1;
-    const float* Klr = Kw + (int64_t)le * B;
-    // Step 2 (Eq 6-7) with explicit clipping (reading R4): common step s
-    double eta = (double)kuu + (double)Klr[le] - 2.0 * (double)Kur[le];
+    // Step 2 (Eq 6-7) with explicit clipping (reading R4): common step s (FP64)
+    double eta = (double)kuu + (double)rl.kd - 2.0 * (double)rl.ku;
     eta = eta > kTau ? eta : kTau;
     double s = (fl - fu) / eta;
     const double Uu = yu > 0 ? C - au : au;
@@ -494,27 +480,27 @@ __global__ void __launch_bounds__(256) local_smo_kernel(SolverArgs a) {
     if (bu) nau = yu > 0 ? C : 0.0;
     if (bl) nal = yl > 0 ? 0.0 : C;
     // Step 3 (Eq 8) on the working set: f_i += s (K_ui - K_li)
-#pragma unroll
-    for (int q = 0; q < E; ++q) {
-      const int e = tid + q * 256;
-      if (valid[q]) {
-        const float kl = Klr[e];
-        fv[q] += s * ((double)ku[q] - (double)kl);
-        if (e == ue) al[q] = nau;
-        if (e == le) al[q] = nal;
-      }
-    }
+    float kl;
+    if (le == ra) kl = va;
+    else if (le == rb) kl = vb;
+    else kl = valid ? Kw[(int64_t)le * B + e] : 0.f;
+    fv += s * ((double)ku - (double)kl);
+    if (e == ue) al = nau;
+    if (e == le) al = nal;
+    ra = ue;
+    va = ku;
+    rb = le;
+    vb = kl;
     ++it;
   }
-#pragma unroll
-  for (int q = 0; q < E; ++q) {
-    const int e = tid + q * 256;
-    if (valid[q]) {
-      a.alpha[pd.a_off + idx[q]] = al[q];
-      a.dcoef[(int64_t)lp * B + e] = (al[q] - a0[q]) * (double)y[q];
-    }
+  if (valid) {
+    a.alpha[pd.a_off + idx] = al;
+    a.dcoef[(int64_t)lp * B + e] = (al - a0) * (double)y;
   }
-  if (tid == 0) a.inner_iters[lp] += it;
+  if (e == 0) {
+    a.inner_iters[lp] += it;
+    a.smo_cycles[lp] += clock64() - t_begin;
+  }
 }
 
 // ------------------------------------------------------------------------------------------
@@ -762,10 +748,8 @@ void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st) {
   GM_LAUNCH(gather_kws_kernel, dim3(P, (unsigned)ceil_div(a.B, kGatherRows)), dim3(256), 0, st, a, first);
 }
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
-  const int E = (int)ceil_div(a.B, 256);
-  if (E <= 1) GM_LAUNCH(local_smo_kernel<1>, dim3(P), dim3(256), 0, st, a);
-  else if (E == 2) GM_LAUNCH(local_smo_kernel<2>, dim3(P), dim3(256), 0, st, a);
-  else GM_LAUNCH(local_smo_kernel<4>, dim3(P), dim3(256), 0, st, a);
+  const int nt = (int)round_up(a.B, 32);  // one thread per working-set row
+  GM_LAUNCH(local_smo_kernel, dim3(P), dim3(nt), 0, st, a);
 }
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
   GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max, kFCols)), dim3(256), 0, st, a);

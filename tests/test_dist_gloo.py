@@ -1,0 +1,105 @@
+"""Multi-process host plumbing of the multi-GPU path on CPU (gloo, world_size 2):
+LPT pair sharding, variable-size model-blob all_gather + merge through libgmpsvm's host
+code, and the test-row shard all_gather.  The NCCL path differs only in the backend."""
+import ctypes as ct
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from blobfmt import make_blob, pair_list
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _problem():
+    rng = np.random.default_rng(0)
+    k, n, d = 4, 60, 5
+    X = rng.normal(size=(n, d)).astype(np.float32)
+    y = (np.arange(n) % k).astype(np.int32)
+    rng.shuffle(y)
+    counts = np.bincount(y, minlength=k)
+    pairs = pair_list(k)
+    P = len(pairs)
+    alphas = {}
+    for p, (s, t) in enumerate(pairs):
+        a = rng.uniform(0, 1, size=counts[s] + counts[t])
+        a[rng.random(len(a)) < 0.5] = 0.0
+        alphas[p] = a
+    b, A, B = rng.normal(size=P), -rng.uniform(1, 2, size=P), rng.normal(size=P)
+    return X, y, k, alphas, b, A, B
+
+
+def _worker(rank, world, port, q):
+    try:
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        import paper_conf_icde_wenshcc19_b200 as gm
+        from paper_conf_icde_wenshcc19_b200 import dist as gdist
+
+        X, y, k, alphas, b, A, B = _problem()
+        shards = gdist.plan_pairs(np.bincount(y, minlength=k), world)
+        mine = {p: alphas[p] for p in shards[rank]}
+        ssz = ct.sizeof(gm._lib.TrainStats)
+        blob, perm, _ = make_blob(X, y, k, 1.0, 0.5, 1e-3, mine, b, A, B, ssz)
+        part = gm.Model.deserialize(blob)
+        merged = gdist.gather_models(part)
+        full_blob, _, sv_pos = make_blob(X, y, k, 1.0, 0.5, 1e-3, alphas, b, A, B, ssz)
+        expect = gm.Model.deserialize(full_blob)
+        ok = merged.n_pairs_trained == len(pair_list(k)) and merged.n_sv == expect.n_sv
+        ok &= bool(np.array_equal(merged.sv_index(), expect.sv_index()))
+        counts = np.bincount(y, minlength=k)
+        for p, (s, t) in enumerate(pair_list(k)):
+            info = merged.pair(s, t, int(counts[s]), int(counts[t]))
+            ok &= bool(np.array_equal(info["alpha"], alphas[p])) and info["b"] == b[p] and info["A"] == A[p]
+        # byte-identical merged blob on every rank
+        blobs = gdist.all_gather_bytes(merged.serialize())
+        ok &= all(np.array_equal(blobs[0], x) for x in blobs)
+        # test-row shards
+        m = 11
+        lo, hi = gdist.row_range(m, world, rank)
+        local = np.arange(lo * 3, hi * 3, dtype=np.float64).reshape(hi - lo, 3)
+        allp = gdist.all_gather_rows(local, m).numpy()
+        ok &= bool(np.array_equal(allp, np.arange(m * 3, dtype=np.float64).reshape(m, 3)))
+        q.put((rank, bool(ok), ""))
+    except Exception as e:  # report instead of hanging the parent
+        q.put((rank, False, repr(e)))
+    finally:
+        if dist.is_initialized():
+            dist.destroy_process_group()
+
+
+def test_plan_pairs_lpt_covers_all_pairs():
+    from paper_conf_icde_wenshcc19_b200 import dist as gdist
+
+    counts = np.array([6000, 6100, 5900, 6050, 5950, 6010, 5990, 6020, 5980, 6000])
+    for world in (1, 2, 4, 8):
+        shards = gdist.plan_pairs(counts, world)
+        flat = sorted(p for s in shards for p in s)
+        assert flat == list(range(45))
+        loads = [sum((counts[a] + counts[b]) ** 1.5 for a, b in (pair_list(10)[p] for p in s)) for s in shards]
+        assert max(loads) / (sum(loads) / world) < 1.2
+
+
+def test_gloo_world2_gather_merge():
+    import __graft_entry__
+
+    __graft_entry__.build()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    assert all(ok for _, ok, _ in res), res
