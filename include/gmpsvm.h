@@ -59,7 +59,8 @@ enum {
 typedef struct {
   int32_t struct_size;      /* sizeof(gmpsvm_options); 0 is accepted as "current"           */
   int32_t ws_size;          /* B: working-set = kernel-buffer rows per pair (L299-L303, L377);
-                               default 1024; clipped to n_p; must be even and >= 2          */
+                               default 192 (K_ws,ws then lives in shared memory; the paper's
+                               1024 is a tuning point); must be even, 2..1024     */
   int32_t q;                /* new violators per outer iteration (L289, L297); default B/2;
                                the newest B-q rows of the previous working set are kept     */
   int32_t device;           /* CUDA device ordinal                                           */
@@ -94,6 +95,10 @@ typedef struct {
   int32_t n_pairs_trained;
   int64_t launches;         /* kernels launched by this call                                  */
   int64_t smo_cycles_sum;   /* SM clock cycles spent in the local SMO, summed over pairs      */
+  double t_solver_ms;       /* a3-a6 as a whole: pairs run on concurrent streams, so select,  */
+                            /* subproblem and f-update overlap (their own fields then stay 0)  */
+  int32_t n_streams;        /* concurrent pair groups (streams) used by the solver             */
+  int32_t pad0;
 } gmpsvm_train_stats;
 
 typedef struct {

@@ -38,7 +38,8 @@ class TrainStats(ct.Structure):
                 ("t_finalize_ms", ct.c_double), ("kernel_flops", ct.c_double), ("kernel_values", ct.c_double),
                 ("krow_launches", ct.c_int64), ("outer_iters_max", ct.c_int64), ("outer_iters_sum", ct.c_int64),
                 ("inner_iters_sum", ct.c_int64), ("n_sv", ct.c_int64), ("cache_regime", ct.c_int32),
-                ("n_pairs_trained", ct.c_int32), ("launches", ct.c_int64), ("smo_cycles_sum", ct.c_int64)]
+                ("n_pairs_trained", ct.c_int32), ("launches", ct.c_int64), ("smo_cycles_sum", ct.c_int64),
+                ("t_solver_ms", ct.c_double), ("n_streams", ct.c_int32), ("pad0", ct.c_int32)]
 
 
 class PredictStats(ct.Structure):

@@ -2,9 +2,14 @@
 // prediction procedure L259-L273 / L331-L363) on one GPU.  Every arithmetic step runs in the
 // kernels of stage.cu / krow.cu / solver.cu / predict.cu; this file allocates, launches,
 // polls the per-pair stop flags once per outer iteration, and assembles the model.
+#include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
+#include <deque>
+#include <thread>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -28,6 +33,10 @@ constexpr int kMaxK = 64;          // label-rank shared memory bound
 constexpr int kMaxCoupleK = 40;    // coupling shared memory bound
 constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
 constexpr int64_t kPredictChunk = 32768;
+constexpr int kMaxStreams = 48;    // concurrent pair groups in the solver
+constexpr int kDefaultStreams = 8; // default pair groups (hardware queues: CUDA_DEVICE_MAX_CONNECTIONS)
+constexpr int kDefaultB = 192;     // working-set rows: K_ws,ws stays in shared memory (B <= 224)
+constexpr int kChunk = 2;          // outer iterations per issued chunk
 
 struct DeviceGuard {
   int prev = -1;
@@ -61,6 +70,34 @@ cudaStream_t get_stream(const gmpsvm_options& opt) {
   return g_streams[dev];
 }
 
+// Per-device pool of non-blocking streams for the concurrent pair groups.
+std::mutex g_pool_mu;
+std::vector<cudaStream_t> g_pools[64];
+const std::vector<cudaStream_t>& stream_pool(int dev) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  auto& v = g_pools[dev];
+  while ((int)v.size() < kMaxStreams) {
+    cudaStream_t s;
+    GM_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    v.push_back(s);
+  }
+  return v;
+}
+
+// Timing-free events created on demand and destroyed with the pool.
+struct EventPool {
+  std::vector<cudaEvent_t> evs;
+  cudaEvent_t get() {
+    cudaEvent_t e;
+    GM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    evs.push_back(e);
+    return e;
+  }
+  ~EventPool() {
+    for (auto e : evs) cudaEventDestroy(e);
+  }
+};
+
 template <class T>
 struct DevBuf {
   T* p = nullptr;
@@ -77,6 +114,65 @@ struct DevBuf {
   T* get() const { return p; }
 };
 
+// Kernel-matrix workspace cache (FULL_K regime): the n^2 x 4 B buffer is the largest
+// allocation of a training run; growing a stream-ordered pool by 14.4 GB costs 0.1-0.5 s, so
+// the buffer is kept per device and reused by later runs.  A buffer is handed out to one run
+// at a time; the next user's stream waits on an event recorded when the previous run ended.
+struct KCacheEntry {
+  float* p = nullptr;
+  size_t bytes = 0;
+  cudaEvent_t done = nullptr;
+  bool busy = false;
+};
+std::mutex g_kcache_mu;
+std::vector<KCacheEntry> g_kcache[64];
+
+struct KWorkspace {
+  int dev;
+  size_t slot = (size_t)-1;
+  cudaStream_t st;
+  float* p = nullptr;
+  KWorkspace(int device, size_t bytes, cudaStream_t s) : dev(device), st(s) {
+    std::lock_guard<std::mutex> lk(g_kcache_mu);
+    auto& v = g_kcache[dev];
+    for (size_t i = 0; i < v.size(); ++i)
+      if (!v[i].busy && v[i].bytes >= bytes) {
+        slot = i;
+        break;
+      }
+    if (slot == (size_t)-1) {
+      for (size_t i = 0; i < v.size(); ++i)  // drop idle buffers that are too small
+        if (!v[i].busy && v[i].p) {
+          GM_CUDA(cudaEventSynchronize(v[i].done));
+          cudaFree(v[i].p);
+          v[i].p = nullptr;
+          v[i].bytes = 0;
+        }
+      KCacheEntry e;
+      GM_CUDA(cudaMalloc((void**)&e.p, bytes));
+      e.bytes = bytes;
+      GM_CUDA(cudaEventCreateWithFlags(&e.done, cudaEventDisableTiming));
+      GM_CUDA(cudaEventRecord(e.done, st));
+      size_t i = 0;
+      for (; i < v.size(); ++i)
+        if (!v[i].busy && !v[i].p) break;
+      if (i == v.size()) v.push_back(e);
+      else v[i] = e;
+      slot = i;
+    }
+    v[slot].busy = true;
+    GM_CUDA(cudaStreamWaitEvent(st, v[slot].done, 0));
+    p = v[slot].p;
+  }
+  ~KWorkspace() {
+    std::lock_guard<std::mutex> lk(g_kcache_mu);
+    auto& e = g_kcache[dev][slot];
+    cudaEventRecord(e.done, st);
+    e.busy = false;
+  }
+  float* get() const { return p; }
+};
+
 template <class T>
 struct PinnedBuf {
   T* p = nullptr;
@@ -89,13 +185,30 @@ struct PinnedBuf {
 };
 
 template <class T>
-T* dev_alloc(size_t count) {
+T* dev_alloc(size_t count, cudaStream_t st) {
   T* p = nullptr;
-  if (count) GM_CUDA(cudaMalloc((void**)&p, count * sizeof(T)));
+  if (count) GM_CUDA(cudaMallocAsync((void**)&p, count * sizeof(T), st));
   return p;
 }
 
-enum { PH_STAGE, PH_KERNEL, PH_SELECT, PH_SUB, PH_FUP, PH_FIN, PH_DEC, PH_COUPLE, PH_D2H, PH_N };
+// Per-thread cached pinned host staging (cudaMallocHost / cudaFreeHost are slow and the
+// latter synchronises the device, so they are not called per training run).
+template <class T>
+T* pinned_scratch(size_t count) {
+  static thread_local void* buf = nullptr;
+  static thread_local size_t cap = 0;
+  const size_t bytes = count * sizeof(T);
+  if (bytes > cap) {
+    if (buf) cudaFreeHost(buf);
+    buf = nullptr;
+    cap = 0;
+    GM_CUDA(cudaMallocHost(&buf, bytes));
+    cap = bytes;
+  }
+  return static_cast<T*>(buf);
+}
+
+enum { PH_STAGE, PH_KERNEL, PH_SELECT, PH_SUB, PH_FUP, PH_FIN, PH_DEC, PH_COUPLE, PH_D2H, PH_SOLVER, PH_N };
 
 struct PhaseTimer {
   cudaStream_t st;
@@ -135,15 +248,22 @@ DevModel::~DevModel() {
   int prev = -1;
   cudaGetDevice(&prev);
   if (device >= 0) cudaSetDevice(device);
-  cudaFree(SvT);
-  cudaFree(nsv);
-  cudaFree(coef);
-  cudaFree(items);
-  cudaFree(item_begin);
-  cudaFree(item_end);
-  cudaFree(b);
-  cudaFree(A);
-  cudaFree(B);
+  gmpsvm_options o;
+  gmpsvm_options_init(&o);
+  o.device = device;
+  cudaStream_t ls = nullptr;
+  try {
+    ls = get_stream(o);
+  } catch (...) {
+  }
+  if (ls && last_use) cudaStreamWaitEvent(ls, last_use, 0);
+  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B};
+  for (void* p : ptrs)
+    if (p) {
+      if (ls) cudaFreeAsync(p, ls);
+      else cudaFree(p);
+    }
+  if (last_use) cudaEventDestroy(last_use);
   if (prev >= 0) cudaSetDevice(prev);
 }
 
@@ -227,15 +347,15 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   }
   if (items.empty()) items.push_back(DecItem{0, 0, 0, 0});  // no SV at all: zero contribution
   dm->n_items = (int)items.size();
-  dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad);
-  dm->nsv = dev_alloc<float>(dm->nsv_pad);
-  dm->coef = dev_alloc<float>(coef.size());
-  dm->items = dev_alloc<DecItem>(items.size());
-  dm->item_begin = dev_alloc<int32_t>(k);
-  dm->item_end = dev_alloc<int32_t>(k);
-  dm->b = dev_alloc<double>(P);
-  dm->A = dev_alloc<double>(P);
-  dm->B = dev_alloc<double>(P);
+  dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad, st);
+  dm->nsv = dev_alloc<float>(dm->nsv_pad, st);
+  dm->coef = dev_alloc<float>(coef.size(), st);
+  dm->items = dev_alloc<DecItem>(items.size(), st);
+  dm->item_begin = dev_alloc<int32_t>(k, st);
+  dm->item_end = dev_alloc<int32_t>(k, st);
+  dm->b = dev_alloc<double>(P, st);
+  dm->A = dev_alloc<double>(P, st);
+  dm->B = dev_alloc<double>(P, st);
   DevBuf<int64_t> d_src(slot_src.size(), st);
   GM_CUDA(cudaMemcpyAsync(d_src.get(), slot_src.data(), slot_src.size() * 8, cudaMemcpyHostToDevice, st));
   GM_CUDA(cudaMemcpyAsync(dm->coef, coef.data(), coef.size() * 4, cudaMemcpyHostToDevice, st));
@@ -247,6 +367,8 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   GM_CUDA(cudaMemcpyAsync(dm->B, m.B.data(), P * 8, cudaMemcpyHostToDevice, st));
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
+  GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
+  GM_CUDA(cudaEventRecord(dm->last_use, st));
   GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
   return dm;
 }
@@ -274,12 +396,23 @@ void ensure_host_sv(const Model& mdl) {
 int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma, double eps,
                  const gmpsvm_options& opt, Model** out) {
   const auto t_start = std::chrono::steady_clock::now();
+  // GMPSVM_HOST_TIMING=1: host-clock checkpoints of the training call on stderr
+  static const bool host_timing = getenv("GMPSVM_HOST_TIMING") != nullptr;
+  auto t_last = t_start;
+  std::string ht_line;
+  auto HT = [&](const char* what) {
+    if (!host_timing) return;
+    const auto now = std::chrono::steady_clock::now();
+    ht_line += std::string(" ") + what + "=" +
+               std::to_string(std::chrono::duration<double, std::milli>(now - t_last).count()).substr(0, 6);
+    t_last = now;
+  };
   if (!X || !y || !out) throw Error(GMPSVM_EINVAL, "null argument");
   if (n < 2 || d < 1 || k < 2) throw Error(GMPSVM_EINVAL, "need n >= 2, d >= 1, k >= 2");
   if (k > kMaxK) throw Error(GMPSVM_ENOTIMPL, "k > 64 classes not supported by this build");
   if (n >= (int64_t)1 << 31) throw Error(GMPSVM_ENOTIMPL, "n >= 2^31 not supported");
   if (!finite_pos(C) || !finite_pos(gamma) || !finite_pos(eps)) throw Error(GMPSVM_EINVAL, "C, gamma, eps must be finite and > 0");
-  int B = opt.ws_size ? opt.ws_size : 1024;
+  int B = opt.ws_size ? opt.ws_size : kDefaultB;
   if (B < 2 || B > 1024 || (B & 1)) throw Error(GMPSVM_EINVAL, "ws_size must be even and in [2, 1024]");
   int q = opt.q ? opt.q : B / 2;
   if (q < 2 || q > B) throw Error(GMPSVM_EINVAL, "q must be in [2, ws_size]");
@@ -289,6 +422,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   PhaseTimer tm(st);
 
   // ---------------- a1 staging
+  HT("stage0");
   tm.mark(PH_STAGE);
   DevBuf<float> bufX(opt.inputs_on_device ? 0 : (size_t)n * d, st);
   DevBuf<int32_t> bufY(opt.inputs_on_device ? 0 : (size_t)n, st);
@@ -322,6 +456,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaStreamSynchronize(st));
   if (hbad) throw Error(GMPSVM_EINVAL, "X contains non-finite values");
   tm.mark(PH_STAGE);
+  HT("stage1");
 
   // ---------------- pairs to train
   const int P = k * (k - 1) / 2;
@@ -346,6 +481,9 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       ps[pair_index(s, t, k)] = s;
       pt[pair_index(s, t, k)] = t;
     }
+  // largest pairs first: they start first and share streams with pairs of similar cost
+  std::stable_sort(pids.begin(), pids.end(),
+                   [&](int x, int y) { return cc[ps[x]] + cc[pt[x]] > cc[ps[y]] + cc[pt[y]]; });
   std::vector<PairDesc> hp(Pl);
   int64_t tot = 0, np_max = 0;
   for (int i = 0; i < Pl; ++i) {
@@ -368,15 +506,18 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   const int64_t ldk = round_up(n, 4);
   const double bytes_K = (double)n * ldk * 4.0;
   size_t free_b = 0, total_b = 0;
+  HT("memgetinfo");
   GM_CUDA(cudaMemGetInfo(&free_b, &total_b));
   const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)free_b;
   if (bytes_K > budget)
     throw Error(GMPSVM_ENOTIMPL, "kernel matrix (" + std::to_string(bytes_K / 1e9) +
                                      " GB) exceeds the cache budget; the ROW_CACHE regime is not in this build");
-  DevBuf<float> K((size_t)n * ldk, st);
+  KWorkspace K(opt.device, (size_t)n * ldk * sizeof(float), st);
+  HT("k_alloc");
   tm.mark(PH_KERNEL);
   launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   tm.mark(PH_KERNEL);
+  HT("krow_launched");
 
   // ---------------- a4-a6 batched working-set solver, all pairs concurrently
   const int Bw = B;
@@ -388,7 +529,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
       d_outer(Pl, st), d_sig(Pl, st);
   DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
-  DevBuf<float> d_Kws((size_t)Pl * Bw * Bw, st);
+  DevBuf<float> d_Kws(local_smo_uses_smem(Bw) ? 0 : (size_t)Pl * Bw * Bw, st);
   SolverArgs a{};
   a.pairs = d_pairs.get();
   a.K = K.get();
@@ -406,6 +547,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   a.gap = d_gap.get();
   a.inner_iters = d_inner.get();
   a.smo_cycles = d_cyc.get();
+  static const bool smo_prof = getenv("GMPSVM_SMO_PHASES") != nullptr;
+  DevBuf<int64_t> d_phase(smo_prof ? (size_t)Pl * 4 : 0, st);
+  if (smo_prof) GM_CUDA(cudaMemsetAsync(d_phase.get(), 0, (size_t)Pl * 4 * 8, st));
+  a.smo_phase = smo_prof ? d_phase.get() : nullptr;
   a.outer_iters = d_outer.get();
   a.b = d_b.get();
   a.A = d_A.get();
@@ -416,34 +561,100 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   a.inner_cap = opt.inner_iter_cap > 0 ? opt.inner_iter_cap : 100 * Bw;
   a.C = C;
   a.eps = eps;
+  HT("solver_alloc");
   launch_init_pairs(a, Pl, tot, st);
   const int64_t max_outer = opt.max_outer_iter > 0 ? opt.max_outer_iter : 1000000;
-  PinnedBuf<int32_t> h_status(Pl);
-  bool cap_hit = false;
-  for (int64_t outer = 0;; ++outer) {
-    tm.mark(PH_SELECT);
-    launch_select_ws(a, Pl, (uint32_t)(outer + 1), outer == 0 ? 1 : 0, st);
-    tm.mark(PH_SELECT);
-    GM_CUDA(cudaMemcpyAsync(h_status.p, d_status.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
-    GM_CUDA(cudaStreamSynchronize(st));
-    int active = 0;
-    for (int i = 0; i < Pl; ++i) active += h_status.p[i] == 0;
-    if (active == 0) break;
-    if (outer >= max_outer) {
-      cap_hit = true;
-      break;
+  // Pairs are independent: groups of pairs run their outer loops on
+  // concurrent streams, so a long local solve of one pair overlaps the selection / f-update
+  // of the others instead of every pair waiting for the slowest one at each outer iteration.
+  // The host keeps two chunks of kChunk outer iterations in flight per group and stops
+  // issuing when the group's stop flags (copied back after each chunk) are all set; kernels
+  // of converged pairs exit at once, so over-issued iterations cost only empty launches.
+  static const int env_streams = getenv("GMPSVM_STREAMS") ? atoi(getenv("GMPSVM_STREAMS")) : 0;
+  const int G = std::max(1, std::min(Pl, env_streams > 0 ? std::min(env_streams, kMaxStreams) : kDefaultStreams));
+  std::vector<int> gb(G + 1);
+  for (int g = 0; g <= G; ++g) gb[g] = (int)((int64_t)g * Pl / G);
+  std::vector<int64_t> g_npmax(G, 0);
+  for (int g = 0; g < G; ++g)
+    for (int i = gb[g]; i < gb[g + 1]; ++i) g_npmax[g] = std::max<int64_t>(g_npmax[g], hp[i].n_s + hp[i].n_t);
+  const std::vector<cudaStream_t>& pool = stream_pool(opt.device);
+  EventPool evp;
+  cudaEvent_t ev_ready = evp.get();
+  GM_CUDA(cudaEventRecord(ev_ready, st));
+  tm.mark(PH_SOLVER);
+  HT("init");
+  for (int g = 0; g < G; ++g) GM_CUDA(cudaStreamWaitEvent(pool[g], ev_ready, 0));
+  struct {
+    int32_t* p;
+  } h_slot{pinned_scratch<int32_t>((size_t)2 * Pl)};  // two status snapshots per pair (alternating chunks)
+  struct Chunk {
+    cudaEvent_t ev;
+    int slot;
+  };
+  std::vector<std::deque<Chunk>> inflight(G);
+  std::vector<int64_t> issued(G, 0);
+  std::vector<int> nchunks(G, 0);
+  std::vector<char> stop(G, 0);
+  auto issue_chunk = [&](int g) {
+    cudaStream_t gs = pool[g];
+    SolverArgs ag = a;
+    ag.pair_base = gb[g];
+    const int gn = gb[g + 1] - gb[g];
+    for (int c = 0; c < kChunk && issued[g] < max_outer + 1; ++c) {
+      const int64_t it = issued[g]++;
+      launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
+      if (it >= max_outer) break;  // the last selection only evaluates the stop test
+      if (!local_smo_uses_smem(Bw)) launch_gather_kws(ag, gn, it == 0 ? 1 : 0, gs);
+      launch_local_smo(ag, gn, gs);
+      launch_f_update(ag, gn, g_npmax[g], gs);
     }
-    tm.mark(PH_SUB);
-    launch_gather_kws(a, Pl, outer == 0 ? 1 : 0, st);
-    launch_local_smo(a, Pl, st);
-    tm.mark(PH_SUB);
-    tm.mark(PH_FUP);
-    launch_f_update(a, Pl, np_max, st);
-    tm.mark(PH_FUP);
+    const int slot = nchunks[g]++ & 1;
+    GM_CUDA(cudaMemcpyAsync(h_slot.p + (size_t)slot * Pl + gb[g], d_status.get() + gb[g], gn * 4,
+                            cudaMemcpyDeviceToHost, gs));
+    cudaEvent_t ev = evp.get();
+    GM_CUDA(cudaEventRecord(ev, gs));
+    inflight[g].push_back(Chunk{ev, slot});
+  };
+  for (int g = 0; g < G; ++g) issue_chunk(g);
+  for (int g = 0; g < G; ++g) issue_chunk(g);
+  int running = G;
+  while (running > 0) {
+    bool progressed = false;
+    for (int g = 0; g < G; ++g) {
+      if (inflight[g].empty()) continue;
+      const Chunk ch = inflight[g].front();
+      const cudaError_t q = cudaEventQuery(ch.ev);
+      if (q == cudaErrorNotReady) continue;
+      GM_CUDA(q);
+      inflight[g].pop_front();
+      progressed = true;
+      if (stop[g]) {
+        if (inflight[g].empty()) --running;
+        continue;
+      }
+      bool all_done = true;
+      for (int i = gb[g]; i < gb[g + 1]; ++i) all_done = all_done && h_slot.p[(size_t)ch.slot * Pl + i] != 0;
+      if (all_done || issued[g] > max_outer) {
+        stop[g] = 1;
+        if (inflight[g].empty()) --running;
+      } else {
+        issue_chunk(g);
+      }
+    }
+    if (!progressed) std::this_thread::yield();
   }
+  for (int g = 0; g < G; ++g) {
+    cudaEvent_t ev = evp.get();
+    GM_CUDA(cudaEventRecord(ev, pool[g]));
+    GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
+  }
+  tm.mark(PH_SOLVER);
+  HT("solver_loop");
+  bool cap_hit = false;
 
   // ---------------- a7-a9 bias, decision values, sigmoid, SV union
   tm.mark(PH_FIN);
+  HT("fin0");
   launch_finalize(a, Pl, st);
   launch_sigmoid_fit(a, Pl, st);
   DevBuf<uint8_t> d_flags(n, st);
@@ -466,6 +677,17 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaMemcpyAsync(h_flags.data(), d_flags.get(), n, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
 
+  if (smo_prof) {
+    std::vector<int64_t> ph((size_t)Pl * 4);
+    GM_CUDA(cudaMemcpy(ph.data(), d_phase.get(), ph.size() * 8, cudaMemcpyDeviceToHost));
+    double tot[4] = {0, 0, 0, 0};
+    for (int i = 0; i < Pl; ++i)
+      for (int q = 0; q < 4; ++q) tot[q] += (double)ph[i * 4 + q];
+    int64_t steps = 0;
+    for (int i = 0; i < Pl; ++i) steps += h_inner[i];
+    fprintf(stderr, "[gmpsvm] local_smo cycles/step: u-reduce %.0f  row-u %.0f  l-reduce %.0f  step+row-l %.0f\n",
+            tot[0] / steps, tot[1] / steps, tot[2] / steps, tot[3] / steps);
+  }
   auto* mdl = new Model();
   std::unique_ptr<Model> guard(mdl);
   mdl->k = k;
@@ -490,7 +712,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     mdl->b[p] = hb[i];
     mdl->A[p] = hA[i];
     mdl->B[p] = hB[i];
-    if (cap_hit && h_st[i] == 0) h_st[i] = 2;
+    if (h_st[i] == 0) {  // still active: the outer-iteration cap stopped it
+      h_st[i] = 2;
+      cap_hit = true;
+    }
     mdl->status[p] = (h_st[i] == 1 ? 0 : h_st[i]) | (h_sig[i] << 8);
     std::memcpy(&mdl->alpha[po[p]], &h_alpha[hp[i].a_off], sizeof(double) * (hp[i].n_s + hp[i].n_t));
     outer_max = std::max<int64_t>(outer_max, h_outer[i]);
@@ -502,8 +727,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     if (h_flags[g]) mdl->sv_pos.push_back(g);
   std::vector<int64_t> row_of_sv(mdl->sv_pos.size());
   for (size_t i = 0; i < row_of_sv.size(); ++i) row_of_sv[i] = mdl->perm[mdl->sv_pos[i]];
+  HT("assembled");
   mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st);
   tm.mark(PH_FIN);
+  HT("devmodel");
   GM_CUDA(cudaStreamSynchronize(st));
 
   gmpsvm_train_stats& s = mdl->stats;
@@ -513,6 +740,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   s.t_subproblem_ms = tm.ms(PH_SUB);
   s.t_fupdate_ms = tm.ms(PH_FUP);
   s.t_finalize_ms = tm.ms(PH_FIN);
+  s.t_solver_ms = tm.ms(PH_SOLVER);
+  s.n_streams = G;
   s.kernel_values = (double)n * (double)(n + 1) / 2.0;
   s.kernel_flops = s.kernel_values * (2.0 * d + 3.0);
   s.krow_launches = 1;
@@ -525,6 +754,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   s.n_pairs_trained = Pl;
   s.launches = (int64_t)(g_launches.load() - launches0);
   s.t_total_ms = host_ms_since(t_start);
+  if (host_timing) fprintf(stderr, "[gmpsvm host ms]%s\n", ht_line.c_str());
   *out = guard.release();
   bool warn = cap_hit;
   for (int i = 0; i < Pl; ++i) warn = warn || h_sig[i] == 1;
@@ -606,6 +836,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
       tm.mark(PH_D2H);
     }
   }
+  GM_CUDA(cudaEventRecord(dm.last_use, st));
   int32_t hbad = 0;
   GM_CUDA(cudaMemcpyAsync(&hbad, bad.get(), 4, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));

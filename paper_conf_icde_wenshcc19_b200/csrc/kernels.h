@@ -40,12 +40,14 @@ struct SolverArgs {
   double* gap;          // [P] global gap at the last selection
   int64_t* inner_iters; // [P]
   int64_t* smo_cycles;  // [P] SM clock cycles spent in local_smo (diagnostic)
+  int64_t* smo_phase;   // [P][4] optional per-phase cycles (GMPSVM_SMO_PHASES=1), else NULL
   int32_t* outer_iters; // [P]
   double* b;            // [P]
   double* A;            // [P]
   double* Bs;           // [P] (sigmoid B)
   int32_t* sig_status;  // [P]
-  int B, q, inner_cap, pad;
+  int B, q, inner_cap;
+  int pair_base;        // first local pair of this launch (grid.x pairs from here)
   double C, eps;
 };
 
@@ -53,6 +55,7 @@ void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st)
 void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st);
 void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st);
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st);
+bool local_smo_uses_smem(int B);  // K_ws,ws gathered in-kernel (no gather_kws launch, no Kws buffer)
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);

@@ -27,6 +27,8 @@ struct DevModel {
   double* A = nullptr;      // [P]
   double* B = nullptr;      // [P]
   std::vector<int64_t> slot_sv;  // slot -> index into the model's SV list, -1 = padding
+  cudaEvent_t last_use = nullptr;  // recorded on the caller's stream after every use
+  // stream-ordered allocation: freed on the library stream after last_use (no device sync)
   ~DevModel();
 };
 

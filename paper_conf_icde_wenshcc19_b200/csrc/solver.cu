@@ -14,6 +14,7 @@
 //   sv_flags    a9  SV union membership over pairs (support-vector sharing, L363)
 #include <cfloat>
 #include <climits>
+#include <cstdlib>
 
 #include "kernels.h"
 
@@ -74,6 +75,29 @@ __device__ int block_excl_scan(bool flag, int& total, int* sm /* 33 */) {
   return sm[warp] + pre;
 }
 
+// exclusive prefix over the warps of a per-warp count (all lanes pass the same value); returns
+// this warp's offset and the block total
+__device__ int block_excl_scan_count(int count, int& total, int* sm /* 33 */) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  __syncthreads();
+  if (lane == 0) sm[warp] = count;
+  __syncthreads();
+  if (warp == 0) {
+    const int v = lane < nw ? sm[lane] : 0;
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(FULLMASK, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane < nw) sm[lane] = x - v;
+    if (lane == 31) sm[32] = x;
+  }
+  __syncthreads();
+  total = sm[32];
+  return sm[warp];
+}
+
 // ------------------------------------------------------------------------------------------
 __global__ void init_pairs_kernel(SolverArgs a, const int64_t tot, int P) {
   // alpha = 0, f = -y (Alg 1 lines 1-2 / Alg 2 line 4), stamps 0
@@ -108,45 +132,71 @@ struct SelSmem {
   int32_t hist[256];
   int32_t scan[33];
   double red[32];
-  int32_t sel_digit, sel_below, take_all, pad;
+  int32_t sel_digit, sel_below, sel_count, take_all;
 };
 
-struct PickCtx {
+// Candidate sources: the global arrays (any n_p) or a shared-memory copy of the keys and
+// I_u / I_l / taken flags (n_p <= kSelSmemMax), both with the same selection semantics.
+struct GlobalSrc {
   const double* al;
   const double* fl;
   uint32_t* st;
   uint32_t stampv;
-  int n_s, np;
+  int n_s;
   double C;
+  template <bool SIDE_U>
+  __device__ __forceinline__ bool cand(int i, uint64_t& key) const {
+    const int y = i < n_s ? 1 : -1;
+    const double a = al[i];
+    const bool ok = SIDE_U ? in_u(y, a, C) : in_l(y, a, C);
+    if (!ok || st[i] == stampv) return false;
+    key = ord_key(fl[i]);
+    if (!SIDE_U) key = ~key;  // ord_key(-f) == ~ord_key(f): largest f first
+    return true;
+  }
+  __device__ __forceinline__ void take(int i) const { st[i] = stampv; }
+};
+struct SmemSrc {
+  const uint64_t* keys;
+  uint8_t* flags;  // bit0 in I_u, bit1 in I_l, bit2 taken / retained
+  template <bool SIDE_U>
+  __device__ __forceinline__ bool cand(int i, uint64_t& key) const {
+    const uint8_t fl = flags[i];
+    if (!(fl & (SIDE_U ? 1 : 2)) || (fl & 4)) return false;
+    key = SIDE_U ? keys[i] : ~keys[i];
+    return true;
+  }
+  __device__ __forceinline__ void take(int i) const { flags[i] |= 4; }
 };
 
-template <bool SIDE_U>
-__device__ __forceinline__ bool pick_cand(const PickCtx& cx, int i, uint64_t& key) {
-  const int y = i < cx.n_s ? 1 : -1;
-  const double a = cx.al[i];
-  const bool ok = SIDE_U ? in_u(y, a, cx.C) : in_l(y, a, cx.C);
-  if (!ok || cx.st[i] == cx.stampv) return false;
-  const double f = cx.fl[i];
-  key = SIDE_U ? ord_key(f) : ord_key(-f);  // ascending key = U: smallest f, L: largest f
-  return true;
-}
-
 // Select the `want` smallest keys among the candidates of one side (ties: lowest index),
-// append them to out[] in index order and stamp them.  Returns the number taken.
-template <bool SIDE_U>
-__device__ int radix_pick(const PickCtx& cx, int want, int32_t* out, SelSmem& sm) {
+// append them to out[] in index order and mark them taken.  Radix select on 8-bit digits
+// from the top; stops as soon as the threshold bucket holds exactly the missing count.
+// kmin / kmax bound the candidates' keys: the bytes above their highest differing bit are
+// common to every candidate and are not scanned.
+template <bool SIDE_U, class Src>
+__device__ int radix_pick(const Src& src, int np, int want, int32_t* out, SelSmem& sm, uint64_t kmin = 0,
+                          uint64_t kmax = ~0ull) {
   if (want <= 0) return 0;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint64_t prefix = 0, pmask = 0;
   int remaining = want;
-  bool take_all = false;
-  for (int shift = 56; shift >= 0; shift -= 8) {
+  bool take_all = false, bucket_all = false;
+  int shift0 = 56;
+  if (kmin <= kmax) {
+    const uint64_t diff = kmin ^ kmax;
+    shift0 = diff ? ((63 - __clzll((long long)diff)) / 8) * 8 : -8;
+    pmask = shift0 >= 56 ? 0ull : ~((1ull << (shift0 + 8)) - 1ull);
+    if (shift0 < 0) pmask = ~0ull;
+    prefix = kmin & pmask;
+  }
+  for (int shift = shift0; shift >= 0; shift -= 8) {
     for (int b = tid; b < 256; b += blockDim.x) sm.hist[b] = 0;
     __syncthreads();
-    for (int base = 0; base < cx.np; base += blockDim.x) {
+    for (int base = 0; base < np; base += blockDim.x) {
       const int i = base + tid;
       uint64_t key = 0;
-      const bool m = (i < cx.np) && pick_cand<SIDE_U>(cx, i, key) && ((key & pmask) == prefix);
+      const bool m = (i < np) && src.template cand<SIDE_U>(i, key) && ((key & pmask) == prefix);
       const unsigned am = __ballot_sync(FULLMASK, m);
       if (m) {
         const int digit = (int)((key >> shift) & 255u);
@@ -170,19 +220,21 @@ __device__ int radix_pick(const PickCtx& cx, int want, int32_t* out, SelSmem& sm
       }
       const int excl = incl - s;
       const int total = __shfl_sync(FULLMASK, incl, 31);
-      if (lane == 0) sm.take_all = (shift == 56 && total <= remaining) ? 1 : 0;
+      if (lane == 0) sm.take_all = (shift == shift0 && total <= remaining) ? 1 : 0;
       if (excl < remaining && remaining <= incl) {
-        int below = excl, dg = lane * 8;
+        int below = excl, dg = lane * 8, cnt = 0;
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
           if (below + loc[q] >= remaining) {
             dg = lane * 8 + q;
+            cnt = loc[q];
             break;
           }
           below += loc[q];
         }
         sm.sel_digit = dg;
         sm.sel_below = below;
+        sm.sel_count = cnt;
       }
     }
     __syncthreads();
@@ -193,51 +245,111 @@ __device__ int radix_pick(const PickCtx& cx, int want, int32_t* out, SelSmem& sm
     remaining -= sm.sel_below;
     prefix |= (uint64_t)sm.sel_digit << shift;
     pmask |= (uint64_t)0xffu << shift;
+    const bool exact = sm.sel_count == remaining;  // the whole bucket is needed
     __syncthreads();
-  }
-  // collect in index order: all keys < T, then the first `remaining` keys == T
-  const uint64_t T = prefix;
-  int taken = 0, eq_taken = 0;
-  for (int base = 0; base < cx.np; base += blockDim.x) {
-    const int i = base + tid;
-    uint64_t key = 0;
-    const bool c = (i < cx.np) && pick_cand<SIDE_U>(cx, i, key);
-    const bool lt = c && (take_all || key < T);
-    const bool eq = c && !take_all && key == T;
-    int eq_tot = 0, tk_tot = 0;
-    const int eq_rank = block_excl_scan(eq, eq_tot, sm.scan);
-    const bool take = lt || (eq && eq_taken + eq_rank < remaining);
-    const int pos = block_excl_scan(take, tk_tot, sm.scan);
-    if (take) {
-      out[taken + pos] = i;
-      cx.st[i] = cx.stampv;
+    if (exact) {
+      bucket_all = true;
+      break;
     }
-    taken += tk_tot;
-    eq_taken += eq_tot;
+  }
+  // Collect in index order: keys below the bucket, then bucket keys (all of them, or the
+  // first `remaining` by index when equal full keys tie).  Each warp owns a contiguous index
+  // range: pass 1 counts per warp, one block scan gives each warp its output offset (and its
+  // rank among tied keys), pass 2 writes.
+  const int nw = blockDim.x >> 5;
+  const int per = (np + nw - 1) / nw;
+  const int lo = min(np, warp * per), hi = min(np, lo + per);
+  auto classify = [&](int i, bool& lt, bool& eq) {
+    uint64_t key = 0;
+    const bool c = (i < hi) && src.template cand<SIDE_U>(i, key);
+    const uint64_t mk = key & pmask;
+    lt = c && (take_all || mk < prefix);
+    eq = c && !take_all && mk == prefix;
+  };
+  int n_lt = 0, n_eq = 0;
+  for (int base = lo; base < hi; base += 32) {
+    bool lt, eq;
+    classify(base + lane, lt, eq);
+    n_lt += __popc(__ballot_sync(FULLMASK, lt));
+    n_eq += __popc(__ballot_sync(FULLMASK, eq));
+  }
+  int eq_tot = 0;
+  int eq_base = 0;
+  if (!bucket_all) {
+    eq_base = block_excl_scan_count(n_eq, eq_tot, sm.scan);
+  }
+  // this warp takes all its lt keys and the eq keys whose global rank is < remaining
+  const int eq_mine = bucket_all ? n_eq : max(0, min(n_eq, remaining - eq_base));
+  int tk_tot = 0;
+  int out_base = block_excl_scan_count(n_lt + eq_mine, tk_tot, sm.scan);
+  int eq_seen = 0;
+  for (int base = lo; base < hi; base += 32) {
+    bool lt, eq;
+    classify(base + lane, lt, eq);
+    const unsigned eb = __ballot_sync(FULLMASK, eq);
+    const int erank = eq_seen + __popc(eb & ((1u << lane) - 1u));
+    const bool take = lt || (eq && erank < eq_mine);
+    const unsigned tb = __ballot_sync(FULLMASK, take);
+    if (take) {
+      const int i = base + lane;
+      out[out_base + __popc(tb & ((1u << lane) - 1u))] = i;
+      src.take(i);
+    }
+    out_base += __popc(tb);
+    eq_seen += __popc(eb);
   }
   __syncthreads();
-  return taken;
+  return tk_tot;
 }
+
+template <class Src>
+__device__ int select_sides(const Src& src, int np, int need, int32_t* out, SelSmem& sm, uint64_t umin = 0,
+                            uint64_t umax = ~0ull, uint64_t lmin = 0, uint64_t lmax = ~0ull) {
+  int cnt = radix_pick<true>(src, np, need / 2, out, sm, umin, umax);
+  cnt += radix_pick<false>(src, np, need - cnt, out + cnt, sm, lmin, lmax);
+  if (cnt < need) cnt += radix_pick<true>(src, np, need - cnt, out + cnt, sm, umin, umax);
+  return cnt;
+}
+
+constexpr int kSelSmemMax = 16384;  // n_p up to which keys + flags are staged in shared memory
 
 __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t stampv, int first) {
   __shared__ SelSmem sm;
-  const int lp = blockIdx.x;
+  extern __shared__ __align__(8) unsigned char sel_dyn[];
+  const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   const double* al = a.alpha + pd.a_off;
   const double* fl = a.f + pd.a_off;
   const double C = a.C;
-  // global stop test (Eq 9-10 with tolerance eps)
-  double fmin = DBL_MAX, fmax = -DBL_MAX;
+  const bool use_smem = np <= kSelSmemMax && np > a.B;
+  uint64_t* keys = reinterpret_cast<uint64_t*>(sel_dyn);
+  uint8_t* flags = sel_dyn + (size_t)kSelSmemMax * 8;
+  // global stop test (Eq 9-10 with tolerance eps); stage keys/flags on the way
+  double fmin = DBL_MAX, fmax = -DBL_MAX, umax = -DBL_MAX, lmin = DBL_MAX;
   for (int i = threadIdx.x; i < np; i += blockDim.x) {
     const int y = i < pd.n_s ? 1 : -1;
     const double av = al[i], fv = fl[i];
-    if (in_u(y, av, C)) fmin = fmin < fv ? fmin : fv;
-    if (in_l(y, av, C)) fmax = fmax > fv ? fmax : fv;
+    const bool u = in_u(y, av, C), l = in_l(y, av, C);
+    if (u) {
+      fmin = fmin < fv ? fmin : fv;
+      umax = umax > fv ? umax : fv;
+    }
+    if (l) {
+      fmax = fmax > fv ? fmax : fv;
+      lmin = lmin < fv ? lmin : fv;
+    }
+    if (use_smem) {
+      keys[i] = ord_key(fv);
+      flags[i] = (u ? 1 : 0) | (l ? 2 : 0);
+    }
   }
   fmin = block_reduce(fmin, [](double x, double y) { return x < y ? x : y; }, sm.red);
   fmax = block_reduce(fmax, [](double x, double y) { return x > y ? x : y; }, sm.red);
+  umax = block_reduce(umax, [](double x, double y) { return x > y ? x : y; }, sm.red);
+  lmin = block_reduce(lmin, [](double x, double y) { return x < y ? x : y; }, sm.red);
+  // key bounds of the two sides: U keys = ord(f) over I_u, L keys = ~ord(f) over I_l
   const double gap = fmax - fmin;
   const bool done = (fmin == DBL_MAX) || (fmax == -DBL_MAX) || !(gap >= a.eps);
   if (threadIdx.x == 0) {
@@ -262,15 +374,19 @@ __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t 
   for (int e = threadIdx.x; e < keep; e += blockDim.x) {
     const int idx = ws[prev_n - keep + e];
     nxt[e] = idx;
-    stp[idx] = stampv;
+    if (use_smem) flags[idx] |= 4;
+    else stp[idx] = stampv;
   }
   __syncthreads();
-  PickCtx cx{al, fl, stp, stampv, pd.n_s, np, C};
-  const int need = B - keep;
   int cnt = keep;
-  cnt += radix_pick<true>(cx, need / 2, nxt + cnt, sm);
-  cnt += radix_pick<false>(cx, B - cnt, nxt + cnt, sm);
-  if (cnt < B) cnt += radix_pick<true>(cx, B - cnt, nxt + cnt, sm);
+  const uint64_t ku0 = ord_key(fmin), ku1 = ord_key(umax), kl0 = ~ord_key(fmax), kl1 = ~ord_key(lmin);
+  if (use_smem) {
+    SmemSrc src{keys, flags};
+    cnt += select_sides(src, np, B - keep, nxt + cnt, sm, ku0, ku1, kl0, kl1);
+  } else {
+    GlobalSrc src{al, fl, stp, stampv, pd.n_s, C};
+    cnt += select_sides(src, np, B - keep, nxt + cnt, sm, ku0, ku1, kl0, kl1);
+  }
   for (int e = threadIdx.x; e < cnt; e += blockDim.x) ws[e] = nxt[e];
   if (threadIdx.x == 0) a.ws_n[lp] = cnt;
 }
@@ -280,7 +396,7 @@ __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t 
 constexpr int kGatherRows = 16;
 
 __global__ void __launch_bounds__(256) gather_kws_kernel(SolverArgs a, int first) {
-  const int lp = blockIdx.x;
+  const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
@@ -383,75 +499,162 @@ __device__ __forceinline__ RedSlot empty_slot() {
   return s;
 }
 
-__global__ void __launch_bounds__(1024) local_smo_kernel(SolverArgs a) {
+__device__ __forceinline__ bool key_less(uint32_t h, uint32_t l, int32_t i, const RedSlot& c) {
+  return h < c.k0 || (h == c.k0 && (l < c.k1 || (l == c.k1 && i < c.idx)));
+}
+
+// E working-set rows per thread (thread t owns rows t, t + nt, ...; nt = blockDim.x).
+// SMEM: K_ws,ws (B <= kSmemMaxB) is gathered straight from the resident kernel matrix into
+// shared memory at kernel start, so the two row reads of every inner step are LDS instead of
+// L2/HBM loads; otherwise rows come from the global K_ws,ws buffer built by gather_kws.
+constexpr int kSmemMaxB = 224;
+
+template <int E, bool SMEM>
+__global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(SolverArgs a) {
   __shared__ RedSlot slots[2][32];
-  const int lp = blockIdx.x;
+  extern __shared__ float kw_smem[];
+  const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int B = a.B, wn = a.ws_n[lp];
-  const int e = threadIdx.x;
-  const float* Kw = a.Kws + (int64_t)lp * B * B;
+  const int nt = blockDim.x;
   const double C = a.C;
-  const bool valid = e < wn;
-  const int32_t idx = valid ? a.ws[(int64_t)lp * B + e] : INT_MAX;
-  const int y = (valid && idx < pd.n_s) ? 1 : -1;
-  double al = valid ? a.alpha[pd.a_off + idx] : 0.0;
-  const double a0 = al;
-  double fv = valid ? a.f[pd.a_off + idx] : 0.0;
-  const float kd = valid ? Kw[(int64_t)e * B + e] : 1.f;
-  // two cached K_ws,ws rows (this thread's column of them): rows ra / rb
+  const float* Kw;
+  if (SMEM) {
+    // gather K[g(ws_r)][g(ws_c)] for r, c < wn into shared memory (row stride B)
+    int32_t* gcol = reinterpret_cast<int32_t*>(kw_smem + (size_t)B * B);
+    for (int e = threadIdx.x; e < wn; e += nt) gcol[e] = (int32_t)gpos(pd, a.ws[(int64_t)lp * B + e]);
+    __syncthreads();
+    for (int r0 = 0; r0 < wn; r0 += 16) {
+      float v[16];
+      const int c = threadIdx.x;
+#pragma unroll
+      for (int rr = 0; rr < 16; ++rr) {
+        const int r = r0 + rr;
+        v[rr] = (r < wn && c < wn) ? __ldg(a.K + (int64_t)gcol[r] * a.ldk + gcol[c]) : 0.f;
+      }
+#pragma unroll
+      for (int rr = 0; rr < 16; ++rr)
+        if (r0 + rr < wn && c < wn) kw_smem[(r0 + rr) * B + c] = v[rr];
+    }
+    __syncthreads();
+    Kw = kw_smem;
+  } else {
+    Kw = a.Kws + (int64_t)lp * B * B;
+  }
+  bool valid[E], iu[E], il[E];
+  int32_t idx[E];
+  int y[E];
+  double al[E], a0[E], fv[E];
+  float kd[E], va[E], vb[E], ku[E];
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = threadIdx.x + q * nt;
+    valid[q] = e < wn;
+    idx[q] = valid[q] ? a.ws[(int64_t)lp * B + e] : INT_MAX;
+    y[q] = (valid[q] && idx[q] < pd.n_s) ? 1 : -1;
+    al[q] = valid[q] ? a.alpha[pd.a_off + idx[q]] : 0.0;
+    a0[q] = al[q];
+    fv[q] = valid[q] ? a.f[pd.a_off + idx[q]] : 0.0;
+    kd[q] = valid[q] ? Kw[(int64_t)e * B + e] : 1.f;
+    iu[q] = valid[q] && in_u(y[q], al[q], C);
+    il[q] = valid[q] && in_l(y[q], al[q], C);
+    va[q] = vb[q] = 0.f;
+  }
+  // two cached K_ws,ws rows (this thread's entries of them): rows ra / rb
   int ra = -1, rb = -1;
-  float va = 0.f, vb = 0.f;
   const int cap = a.inner_cap;
   int it = 0, par = 0;
   double delta0 = 0.0;
   const long long t_begin = clock64();
+  long long ph[4] = {0, 0, 0, 0}, tp = t_begin;
+  const bool prof = a.smo_phase != nullptr;
   for (;;) {
     // Step 1 (Eq 4): u = argmin_{I_u} f, ties -> lowest pair-local index
     RedSlot c = empty_slot();
-    if (valid && in_u(y, al, C)) {
-      const uint64_t key = ord_key(fv);
-      c.k0 = (uint32_t)(key >> 32);
-      c.k1 = (uint32_t)key;
-      c.idx = idx;
-      c.e = e;
-      c.alpha = al;
-      c.f = fv;
-      c.kd = kd;
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      if (iu[q]) {
+        const uint64_t key = ord_key(fv[q]);
+        const uint32_t h = (uint32_t)(key >> 32), l = (uint32_t)key;
+        if (key_less(h, l, idx[q], c)) {
+          c.k0 = h;
+          c.k1 = l;
+          c.idx = idx[q];
+          c.e = threadIdx.x + q * nt;
+          c.alpha = al[q];
+          c.f = fv[q];
+          c.kd = kd[q];
+        }
+      }
     }
     const RedSlot ru = block_argmin<false>(c, slots[par]);
     par ^= 1;
+    if (prof) {
+      const long long t = clock64();
+      ph[0] += t - tp;
+      tp = t;
+    }
     if (ru.idx == INT_MAX) break;
     const int ue = ru.e;
     const double fu = ru.f, au = ru.alpha;
     const float kuu = ru.kd;
     const int yu = ru.idx < pd.n_s ? 1 : -1;
-    float ku;
-    if (ue == ra) ku = va;
-    else if (ue == rb) ku = vb;
-    else ku = valid ? Kw[(int64_t)ue * B + e] : 0.f;
+    if (ue == ra) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) ku[q] = va[q];
+    } else if (ue == rb) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) ku[q] = vb[q];
+    } else {
+      const float* row = Kw + (int64_t)ue * B;
+#pragma unroll
+      for (int q = 0; q < E; ++q) ku[q] = valid[q] ? row[threadIdx.x + q * nt] : 0.f;
+    }
+    if (prof) {
+      float sum = 0.f;
+#pragma unroll
+      for (int q = 0; q < E; ++q) sum += ku[q];
+      if (sum == -1.f) ph[3] += 1;  // force the loads to complete before reading the clock
+      const long long t = clock64();
+      ph[1] += t - tp;
+      tp = t;
+    }
     // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_u - f_t)^2 / eta_t, and f_max over I_l (Eq 10)
     c = empty_slot();
-    if (valid && in_l(y, al, C)) {
-      const uint64_t fk = ord_key(fv);
-      c.m0 = (uint32_t)(fk >> 32);
-      c.m1 = (uint32_t)fk;
-      if (fv > fu) {
-        const float eta = fmaxf(kuu + kd - 2.f * ku, 1e-12f);
-        const float df = (float)(fv - fu);
-        const float score = df * df * __frcp_rn(eta);
-        c.k0 = ~__float_as_uint(score);
-        c.k1 = 0u;
-        c.idx = idx;
-        c.e = e;
-        c.alpha = al;
-        c.f = fv;
-        c.kd = kd;
-        c.ku = ku;
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      if (il[q]) {
+        const uint64_t fk = ord_key(fv[q]);
+        const uint32_t h = (uint32_t)(fk >> 32), l = (uint32_t)fk;
+        if (h > c.m0 || (h == c.m0 && l > c.m1)) {
+          c.m0 = h;
+          c.m1 = l;
+        }
+        if (fv[q] > fu) {
+          const float eta = fmaxf(kuu + kd[q] - 2.f * ku[q], 1e-12f);
+          const float df = (float)(fv[q] - fu);
+          const uint32_t sk = ~__float_as_uint(df * df * __frcp_rn(eta));
+          if (key_less(sk, 0u, idx[q], c)) {
+            c.k0 = sk;
+            c.k1 = 0u;
+            c.idx = idx[q];
+            c.e = threadIdx.x + q * nt;
+            c.alpha = al[q];
+            c.f = fv[q];
+            c.kd = kd[q];
+            c.ku = ku[q];
+          }
+        }
       }
     }
     const RedSlot rl = block_argmin<true>(c, slots[par]);
     par ^= 1;
+    if (prof) {
+      const long long t = clock64();
+      ph[2] += t - tp;
+      tp = t;
+    }
     const double fmax = (rl.m0 == 0u && rl.m1 == 0u) ? -DBL_MAX : key_double(((uint64_t)rl.m0 << 32) | rl.m1);
     const double gap = fmax - fu;
     if (it == 0) delta0 = gap;
@@ -480,42 +683,74 @@ __global__ void __launch_bounds__(1024) local_smo_kernel(SolverArgs a) {
     if (bu) nau = yu > 0 ? C : 0.0;
     if (bl) nal = yl > 0 ? 0.0 : C;
     // Step 3 (Eq 8) on the working set: f_i += s (K_ui - K_li)
-    float kl;
-    if (le == ra) kl = va;
-    else if (le == rb) kl = vb;
-    else kl = valid ? Kw[(int64_t)le * B + e] : 0.f;
-    fv += s * ((double)ku - (double)kl);
-    if (e == ue) al = nau;
-    if (e == le) al = nal;
+    float kl[E];
+    if (le == ra) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) kl[q] = va[q];
+    } else if (le == rb) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) kl[q] = vb[q];
+    } else {
+      const float* row = Kw + (int64_t)le * B;
+#pragma unroll
+      for (int q = 0; q < E; ++q) kl[q] = valid[q] ? row[threadIdx.x + q * nt] : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      const int e = threadIdx.x + q * nt;
+      fv[q] += s * ((double)ku[q] - (double)kl[q]);
+      if (e == ue || e == le) {
+        al[q] = (e == ue) ? nau : nal;
+        iu[q] = in_u(y[q], al[q], C);
+        il[q] = in_l(y[q], al[q], C);
+      }
+      va[q] = ku[q];
+      vb[q] = kl[q];
+    }
     ra = ue;
-    va = ku;
     rb = le;
-    vb = kl;
     ++it;
+    if (prof) {
+      const long long t = clock64();
+      ph[3] += t - tp;
+      tp = t;
+    }
   }
-  if (valid) {
-    a.alpha[pd.a_off + idx] = al;
-    a.dcoef[(int64_t)lp * B + e] = (al - a0) * (double)y;
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = threadIdx.x + q * nt;
+    if (valid[q]) {
+      a.alpha[pd.a_off + idx[q]] = al[q];
+      a.dcoef[(int64_t)lp * B + e] = (al[q] - a0[q]) * (double)y[q];
+    }
   }
-  if (e == 0) {
+  if (threadIdx.x == 0) {
     a.inner_iters[lp] += it;
     a.smo_cycles[lp] += clock64() - t_begin;
+    if (prof)
+      for (int k = 0; k < 4; ++k) a.smo_phase[lp * 4 + k] += ph[k];
   }
 }
 
 // ------------------------------------------------------------------------------------------
-// a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij for all j in the pair
-constexpr int kFCols = 1024;  // columns per CTA (256 threads x 4)
+// a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij for all j in the pair.
+// HBM-bound GEMV over the rows with dalpha != 0: each thread owns kFQ 16-byte column quads of
+// the pair's two class segments (aligned to the kernel matrix rows, ldk % 4 == 0) and streams
+// the rows 2 at a time (kFQ x 2 float4 loads in flight), accumulating in FP64.
+constexpr int kFQ = 2;                       // quads per thread
+constexpr int kFCols = 256 * kFQ * 4;        // columns per CTA
 
 __global__ void __launch_bounds__(256) f_update_kernel(SolverArgs a) {
-  const int lp = blockIdx.x;
+  const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
-  const int np = pd.n_s + pd.n_t;
-  const int64_t c0 = (int64_t)blockIdx.y * kFCols;
-  if (c0 >= np) return;
+  const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;  // quads of class s
+  const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;  // quads of class t
+  const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
+  const int64_t qcta = (int64_t)blockIdx.y * (256 * kFQ);
+  if (qcta >= nq) return;
   __shared__ double coef[1024];
-  __shared__ const float* rowp[1024];
+  __shared__ const float4* rowp[1024];
   __shared__ int scan_sm[33];
   const int B = a.B, wn = a.ws_n[lp];
   const int32_t* ws = a.ws + (int64_t)lp * B;
@@ -529,56 +764,78 @@ __global__ void __launch_bounds__(256) f_update_kernel(SolverArgs a) {
     const int pos = block_excl_scan(nz, tot, scan_sm);
     if (nz) {
       coef[nnz + pos] = c;
-      rowp[nnz + pos] = a.K + gpos(pd, ws[e]) * a.ldk;
+      rowp[nnz + pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, ws[e]) * a.ldk);
     }
     nnz += tot;
   }
   __syncthreads();
   if (nnz == 0) return;
-  int64_t gc[4];
-  bool ok[4];
-  double acc[4];
+  int64_t gq[kFQ];
+  bool okq[kFQ], seg1[kFQ];
+  double acc[kFQ][4];
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const int64_t j = c0 + threadIdx.x + q * 256;
-    ok[q] = j < np;
-    gc[q] = ok[q] ? gpos(pd, j) : 0;
-    acc[q] = 0.0;
+  for (int u = 0; u < kFQ; ++u) {
+    const int64_t qi = qcta + threadIdx.x + u * 256;
+    okq[u] = qi < nq;
+    seg1[u] = qi < nq1;  // a boundary quad shared by adjacent classes is owned once per segment
+    gq[u] = !okq[u] ? 0 : (qi < nq1 ? q1b + qi : q2b + (qi - nq1));
+#pragma unroll
+    for (int c = 0; c < 4; ++c) acc[u][c] = 0.0;
   }
+  // rows 4 at a time: kFQ x 4 independent 16-byte loads in flight per thread (Little's law at
+  // ~1.5 us loaded-DRAM latency needs ~10 MB in flight chip-wide for 6.5 TB/s)
   int r = 0;
-  for (; r + 2 <= nnz; r += 2) {
-    const float* p0 = rowp[r];
-    const float* p1 = rowp[r + 1];
-    const double c0v = coef[r], c1v = coef[r + 1];
-    float v0[4], v1[4];
+  for (; r + 4 <= nnz; r += 4) {
+    float4 v[4][kFQ];
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      v0[q] = ok[q] ? __ldg(p0 + gc[q]) : 0.f;
-      v1[q] = ok[q] ? __ldg(p1 + gc[q]) : 0.f;
-    }
+    for (int rr = 0; rr < 4; ++rr)
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      acc[q] = fma(c0v, (double)v0[q], acc[q]);
-      acc[q] = fma(c1v, (double)v1[q], acc[q]);
+      for (int u = 0; u < kFQ; ++u) v[rr][u] = okq[u] ? __ldg(rowp[r + rr] + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr) {
+      const double cv = coef[r + rr];
+#pragma unroll
+      for (int u = 0; u < kFQ; ++u) {
+        acc[u][0] = fma(cv, (double)v[rr][u].x, acc[u][0]);
+        acc[u][1] = fma(cv, (double)v[rr][u].y, acc[u][1]);
+        acc[u][2] = fma(cv, (double)v[rr][u].z, acc[u][2]);
+        acc[u][3] = fma(cv, (double)v[rr][u].w, acc[u][3]);
+      }
     }
   }
   for (; r < nnz; ++r) {
-    const float* p0 = rowp[r];
+    const float4* p0 = rowp[r];
     const double c0v = coef[r];
 #pragma unroll
-    for (int q = 0; q < 4; ++q)
-      if (ok[q]) acc[q] = fma(c0v, (double)__ldg(p0 + gc[q]), acc[q]);
+    for (int u = 0; u < kFQ; ++u) {
+      const float4 v0 = okq[u] ? __ldg(p0 + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+      acc[u][0] = fma(c0v, (double)v0.x, acc[u][0]);
+      acc[u][1] = fma(c0v, (double)v0.y, acc[u][1]);
+      acc[u][2] = fma(c0v, (double)v0.z, acc[u][2]);
+      acc[u][3] = fma(c0v, (double)v0.w, acc[u][3]);
+    }
   }
+  double* f = a.f + pd.a_off;
 #pragma unroll
-  for (int q = 0; q < 4; ++q)
-    if (ok[q]) a.f[pd.a_off + c0 + threadIdx.x + q * 256] += acc[q];
+  for (int u = 0; u < kFQ; ++u) {
+    if (!okq[u]) continue;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const int64_t g = gq[u] * 4 + c;  // global (class-sorted) column
+      if (seg1[u]) {
+        if (g >= pd.off_s && g < pd.off_s + pd.n_s) f[g - pd.off_s] += acc[u][c];
+      } else if (g >= pd.off_t && g < pd.off_t + pd.n_t) {
+        f[pd.n_s + (g - pd.off_t)] += acc[u][c];
+      }
+    }
+  }
 }
 
 // ------------------------------------------------------------------------------------------
 // a7: bias and in-sample decision values
 __global__ void __launch_bounds__(1024) finalize_kernel(SolverArgs a) {
   __shared__ double red[32];
-  const int lp = blockIdx.x;
+  const int lp = blockIdx.x + a.pair_base;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   const double* al = a.alpha + pd.a_off;
@@ -639,7 +896,7 @@ __device__ __forceinline__ double nll_term(double v, double t, double A, double 
 
 __global__ void __launch_bounds__(512) sigmoid_fit_kernel(SolverArgs a) {
   __shared__ double sm[32 * 5];
-  const int lp = blockIdx.x;
+  const int lp = blockIdx.x + a.pair_base;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   const double* v = a.v + pd.a_off;
@@ -729,7 +986,7 @@ __global__ void __launch_bounds__(512) sigmoid_fit_kernel(SolverArgs a) {
 // ------------------------------------------------------------------------------------------
 // a9: SV union flags over class-sorted positions
 __global__ void sv_flags_kernel(SolverArgs a, uint8_t* flags) {
-  const int lp = blockIdx.x;
+  const int lp = blockIdx.x + a.pair_base;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   const int64_t j = (int64_t)blockIdx.y * blockDim.x + threadIdx.x;
@@ -742,17 +999,43 @@ void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st)
   GM_LAUNCH(init_pairs_kernel, dim3((unsigned)ceil_div(nthr, 256)), dim3(256), 0, st, a, tot, P);
 }
 void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st) {
-  GM_LAUNCH(select_ws_kernel, dim3(P), dim3(1024), 0, st, a, stampv, first);
+  const size_t dyn = (size_t)kSelSmemMax * 9;  // keys (8 B) + flags (1 B)
+  static bool configured = false;
+  if (!configured) {
+    GM_CUDA(cudaFuncSetAttribute(select_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
+    configured = true;
+  }
+  GM_LAUNCH(select_ws_kernel, dim3(P), dim3(1024), dyn, st, a, stampv, first);
 }
 void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st) {
   GM_LAUNCH(gather_kws_kernel, dim3(P, (unsigned)ceil_div(a.B, kGatherRows)), dim3(256), 0, st, a, first);
 }
+bool local_smo_uses_smem(int B) { return B <= kSmemMaxB; }
+
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
-  const int nt = (int)round_up(a.B, 32);  // one thread per working-set row
-  GM_LAUNCH(local_smo_kernel, dim3(P), dim3(nt), 0, st, a);
+  if (local_smo_uses_smem(a.B)) {
+    const size_t dyn = (size_t)a.B * a.B * sizeof(float) + (size_t)a.B * sizeof(int32_t);
+    static size_t configured = 0;
+    if (dyn > configured) {
+      GM_CUDA(cudaFuncSetAttribute(local_smo_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)(kSmemMaxB * kSmemMaxB * 4 + kSmemMaxB * 4)));
+      configured = (size_t)kSmemMaxB * kSmemMaxB * 4 + kSmemMaxB * 4;
+    }
+    GM_LAUNCH((local_smo_kernel<1, true>), dim3(P), dim3((unsigned)round_up(a.B, 32)), dyn, st, a);
+    return;
+  }
+  // E working-set rows per thread; GMPSVM_SMO_E overrides the default (tuning)
+  static const int e_env = getenv("GMPSVM_SMO_E") ? atoi(getenv("GMPSVM_SMO_E")) : 0;
+  int E = e_env > 0 ? e_env : (a.B > 256 ? 2 : 1);
+  if (E != 1 && E != 2 && E != 4) E = 2;
+  const int nt = (int)round_up(ceil_div(a.B, E), 32);
+  if (E == 1) GM_LAUNCH((local_smo_kernel<1, false>), dim3(P), dim3(nt), 0, st, a);
+  else if (E == 2) GM_LAUNCH((local_smo_kernel<2, false>), dim3(P), dim3(nt), 0, st, a);
+  else GM_LAUNCH((local_smo_kernel<4, false>), dim3(P), dim3(nt), 0, st, a);
 }
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
-  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max, kFCols)), dim3(256), 0, st, a);
+  // +8 columns: each class segment may add a partial quad at either end
+  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, kFCols)), dim3(256), 0, st, a);
 }
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st) {
   GM_LAUNCH(finalize_kernel, dim3(P), dim3(1024), 0, st, a);

@@ -20,8 +20,8 @@ pytestmark = pytest.mark.gpu
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "mnist_eps1e-05.json")
 
 
-@pytest.fixture(scope="module")
-def setup():
+@pytest.fixture(scope="module", params=[None, 1024], ids=["bench-config", "ws1024"])
+def setup(request):
     import __graft_entry__
 
     __graft_entry__.build()
@@ -31,7 +31,8 @@ def setup():
     spec, X, y, Xt, yt = datagen.make_config("mnist")
     dev = torch.device("cuda:0")
     Xd, yd = torch.from_numpy(X).to(dev), torch.from_numpy(y).to(dev)
-    model = gm.train(Xd, yd, spec.k, spec.C, spec.gamma, g["eps"], ws_size=1024)
+    opts = {} if request.param is None else {"ws_size": request.param}  # None: bench.py's defaults
+    model = gm.train(Xd, yd, spec.k, spec.C, spec.gamma, g["eps"], **opts)
     return gm, g, spec, X, y, Xt, yt, model
 
 

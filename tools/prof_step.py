@@ -6,6 +6,8 @@ import argparse
 import os
 import sys
 
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
@@ -18,7 +20,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="mnist")
 ap.add_argument("--eps", type=float, default=1e-3)
 ap.add_argument("--reps", type=int, default=1)
-ap.add_argument("--ws-size", type=int, default=1024)
+ap.add_argument("--ws-size", type=int, default=192)
 a = ap.parse_args()
 spec, X, y, Xt, yt = datagen.make_config(a.config)
 dev = torch.device("cuda:0")
