@@ -445,12 +445,21 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   for (int c = 0; c < k; ++c)
     if (cc[c] == 0) throw Error(GMPSVM_EINVAL, "every class must have at least one instance");
   launch_class_rank(dy, n, k, blk_off.get(), d_off.get(), d_perm.get(), st);
-  const int d_pad = (int)round_up(d, kBK);
-  const int64_t n_pad = round_up(n, kTile);
-  DevBuf<float> XT((size_t)d_pad * n_pad, st), norms(n_pad, st);
+  const bool use_tc = krow_use_tc();
+  const int d_pad = use_tc ? krow_tc_d_pad(d) : (int)round_up(d, kBK);
+  const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile);
+  // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split
+  DevBuf<float> XT(use_tc ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad, st);
+  DevBuf<float> Xhi(use_tc ? (size_t)n_pad * d_pad : 0, st), Xlo(use_tc ? (size_t)n_pad * d_pad : 0, st);
   DevBuf<int32_t> bad(1, st);
   GM_CUDA(cudaMemsetAsync(bad.get(), 0, 4, st));
-  launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
+  DevBuf<uint8_t> tc_scratch(use_tc ? krow_tc_scratch_bytes(n, d) : 0, st);
+  if (use_tc) {
+    launch_row_norms(dX, n, d, d_perm.get(), norms.get(), n_pad, bad.get(), st);  // validation (non-finite rows)
+    launch_split_tf32(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st);
+  } else {
+    launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
+  }
   int32_t hbad = 0;
   GM_CUDA(cudaMemcpyAsync(&hbad, bad.get(), 4, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
@@ -514,8 +523,19 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
                                      " GB) exceeds the cache budget; the ROW_CACHE regime is not in this build");
   KWorkspace K(opt.device, (size_t)n * ldk * sizeof(float), st);
   HT("k_alloc");
+  std::vector<int2> tiles;
+  DevBuf<int2> d_tiles;
+  if (use_tc) {
+    tiles = krow_tc_tiles(n);
+    new (&d_tiles) DevBuf<int2>(tiles.size(), st);
+    GM_CUDA(cudaMemcpyAsync(d_tiles.get(), tiles.data(), tiles.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
+  }
   tm.mark(PH_KERNEL);
-  launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
+  if (use_tc)
+    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, K.get(),
+                   ldk, st);
+  else
+    launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   tm.mark(PH_KERNEL);
   HT("krow_launched");
 
@@ -872,6 +892,22 @@ int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int3
   }
   // X == Y (same buffer, same size): the symmetric FULL_K launch that training uses (K_ii = 1)
   const bool sym = (X == Y && n == m);
+  if (sym && krow_use_tc()) {
+    const int dp = krow_tc_d_pad(d);
+    const int64_t np2 = krow_tc_rows_pad(n);
+    DevBuf<float> hi((size_t)np2 * dp, st), lo((size_t)np2 * dp, st), nx2(np2, st);
+    DevBuf<uint8_t> scr(krow_tc_scratch_bytes(n, d), st);
+    launch_split_tf32(dX, n, d, nullptr, hi.get(), lo.get(), nx2.get(), np2, dp, scr.get(), st);
+    const std::vector<int2> tl = krow_tc_tiles(n);
+    DevBuf<int2> dt(tl.size(), st);
+    GM_CUDA(cudaMemcpyAsync(dt.get(), tl.data(), tl.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
+    DevBuf<float> kb2(opt.inputs_on_device ? 0 : (size_t)n * m, st);
+    float* dK2 = opt.inputs_on_device ? K_out : kb2.get();
+    launch_krow_tc(hi.get(), lo.get(), np2, dp, dt.get(), (int)tl.size(), nx2.get(), n, gamma, dK2, m, st);
+    if (!opt.inputs_on_device) GM_CUDA(cudaMemcpyAsync(K_out, dK2, (size_t)n * m * 4, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaStreamSynchronize(st));
+    return GMPSVM_OK;
+  }
   DevBuf<float> XT((size_t)d_pad * n_pad, st), YT(sym ? 0 : (size_t)d_pad * m_pad, st), nx(n_pad, st),
       ny(sym ? 0 : m_pad, st);
   launch_stage_features(dX, n, d, nullptr, XT.get(), n_pad, d_pad, n_pad, nx.get(), nullptr, st);

@@ -1,6 +1,8 @@
 // kernels.h -- launchers of the sm_100a kernels (internal to libgmpsvm).
 #pragma once
 
+#include <vector>
+
 #include "common.cuh"
 
 namespace gmpsvm {
@@ -21,6 +23,21 @@ void launch_krow_full_sym(const float* XT, int64_t ldx, const float* norms, int6
                           float* K, int64_t ldk, cudaStream_t st);
 void launch_krow_rect(const float* AT, int64_t lda, const float* na, int64_t n, const float* BT, int64_t ldb,
                       const float* nb, int64_t m, int kdim, double gamma, float* K, int64_t ldk, cudaStream_t st);
+
+// ---------------- a2 on tcgen05 (krow_tc.cu): 3xTF32 split, TMEM accumulators, TMA staging
+int64_t krow_tc_rows_pad(int64_t n);  // row padding the tile grid needs (multiple of 256)
+int krow_tc_d_pad(int d);             // feature padding (multiple of 32)
+// centre by the column means (mean of the original rows; perm only reorders), split into TF32
+// hi/lo rows and compute the centred squared norms; scratch = krow_tc_scratch_bytes(n, d)
+size_t krow_tc_scratch_bytes(int64_t n, int d);
+void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, float* hi, float* lo, float* norms,
+                       int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
+std::vector<int2> krow_tc_tiles(int64_t n);
+void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
+                    const float* norms, int64_t n, double gamma, float* K, int64_t ldk, cudaStream_t st);
+void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
+                      cudaStream_t st);
+bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel
 
 // ---------------- a4-a9 solver (solver.cu)
 struct SolverArgs {

@@ -1,0 +1,390 @@
+// krow_tc.cu -- a2 on the 5th-generation tensor cores: the kernel-value contraction with a
+// 3xTF32 split (x = hi + lo, hi = x truncated to TF32, lo = x - hi exactly), so that
+//   x.y ~= hi.hi + hi.lo + lo.hi   (the lo.lo term is below FP32 rounding)
+// is accumulated in FP32 in TMEM by tcgen05.mma kind::tf32, operands staged by TMA into
+// 128-byte-swizzled shared memory.  The epilogue (norm combine, clamp, ex2, K_ii = 1,
+// symmetric mirrored store) is the same arithmetic as krow.cu's SIMT kernel.
+//
+// CTA tile 128 x 128, one CTA per tile (bi, bj) of the upper triangle, warp 0 = TMA producer,
+// warp 1 = MMA issuer (+ TMEM allocation), warps 2..5 = epilogue (one TMEM lane quarter each),
+// 3-stage smem ring of 64 KB (A hi/lo and B hi/lo, 128 x 32 FP32 each).  TMEM holds four
+// 128-column FP32 accumulators: hi.hi over each third of the k range, and hi.lo + lo.hi.
+// Entry (r, c) is written, with its mirror (c, r), only by the tile that holds it with r <= c.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <cstdlib>
+#include <mutex>
+#include <vector>
+
+#include "kernels.h"
+
+namespace gmpsvm {
+
+namespace {
+
+constexpr int kTM = 128, kTN = 128, kTK = 32;  // tile rows, columns, k-step (one 128 B swizzle atom)
+constexpr int kTcStages = 3;
+constexpr int kMainAcc = 3;  // hi.hi accumulators (k range split in thirds)
+constexpr int kTcThreads = 192;
+constexpr uint32_t kABytes = kTM * kTK * 4;            // 16 KB
+constexpr uint32_t kBBytes = kTN * kTK * 4;            // 16 KB
+constexpr uint32_t kStageBytes = 2 * kABytes + 2 * kBBytes;  // 64 KB
+constexpr uint32_t kTmemCols = 512;  // 3 x 128 hi.hi (k thirds) + 128 hi.lo + lo.hi
+
+struct TcSmem {
+  // each operand tile 1024-byte aligned (128B swizzle atoms)
+  alignas(1024) uint8_t stage[kTcStages][kStageBytes];
+  alignas(8) uint64_t full[kTcStages];
+  uint64_t empty[kTcStages];
+  uint64_t tmem_full;
+  uint64_t tmem_empty;
+  uint32_t tmem_base;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  const uint32_t a = smem_u32(b);
+  uint32_t done = 0;
+  do {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
+      : "memory");
+}
+// K-major operand, 128-byte swizzle: 8-row groups 1024 B apart (SBO), LBO unused (1), version 1.
+__device__ __forceinline__ uint64_t umma_desc_sw128(const void* p) {
+  const uint64_t addr = smem_u32(p);
+  uint64_t d = 0;
+  d |= (addr >> 4) & 0x3FFFull;        // start address
+  d |= (uint64_t)1 << 16;              // leading byte offset (unused for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;    // stride byte offset
+  d |= (uint64_t)1 << 46;              // descriptor version (sm100)
+  d |= (uint64_t)2 << 61;              // SWIZZLE_128B
+  return d;
+}
+// kind::tf32, A/B TF32 K-major, D F32, M = 128, N = 128
+constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(kTN >> 3) << 17) | ((uint32_t)(kTM >> 4) << 24);
+
+__device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(
+          tmem_d),
+      "l"(a), "l"(b), "r"(kIdesc), "r"(accum));
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),
+        "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]),
+        "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]),
+        "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+      : "r"(taddr));
+}
+
+// Persistent: one CTA per SM walks the tile list (tile = blockIdx.x + i * gridDim.x).  The TMA
+// producer runs ahead across tile boundaries through the smem ring; the epilogue drains the four
+// TMEM accumulators into registers and releases TMEM at once (tmem_empty), so the MMAs of the
+// next tile overlap the exp + stores of the current one.
+__global__ void __launch_bounds__(kTcThreads, 1)
+    krow_tc_kernel(const __grid_constant__ CUtensorMap map_hi, const __grid_constant__ CUtensorMap map_lo,
+                   const int2* __restrict__ tiles, int n_tiles, const float* __restrict__ norms, int64_t n, int nk,
+                   float scale, float* __restrict__ K, int64_t ldk) {
+  extern __shared__ __align__(1024) uint8_t dsmem[];
+  TcSmem& sm = *reinterpret_cast<TcSmem*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < kTcStages; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], 1);
+    }
+    mbar_init(&sm.tmem_full, 1);
+    mbar_init(&sm.tmem_empty, 4);  // one arrive per epilogue warp
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_hi)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_lo)) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&sm.tmem_base)),
+                 "r"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = sm.tmem_base;
+  const int jn = nk < kMainAcc ? nk : kMainAcc;  // hi.hi accumulators in use (short k ranges)
+
+  if (warp == 0) {
+    if (lane == 0) {  // ---- TMA producer (runs ahead across tiles)
+      int g = 0;
+      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+        const int2 tile = tiles[t];
+        const int r0 = tile.x * kTM, c0 = tile.y * kTN;
+        for (int kb = 0; kb < nk; ++kb, ++g) {
+          const int s = g % kTcStages;
+          if (g >= kTcStages) mbar_wait(&sm.empty[s], ((g / kTcStages) + 1) & 1);
+          uint8_t* st = sm.stage[s];
+          mbar_expect_tx(&sm.full[s], kStageBytes);
+          const int kx = kb * kTK;
+          tma_load_2d(st, &map_hi, kx, r0, &sm.full[s]);
+          tma_load_2d(st + kABytes, &map_lo, kx, r0, &sm.full[s]);
+          tma_load_2d(st + 2 * kABytes, &map_hi, kx, c0, &sm.full[s]);
+          tma_load_2d(st + 2 * kABytes + kBBytes, &map_lo, kx, c0, &sm.full[s]);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---- MMA issuer
+      int g = 0, it = 0;
+      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+        if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);  // epilogue drained the previous tile
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        for (int kb = 0; kb < nk; ++kb, ++g) {
+          const int s = g % kTcStages;
+          mbar_wait(&sm.full[s], (g / kTcStages) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          uint8_t* st = sm.stage[s];
+          const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
+          const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
+          // the FP32 accumulation error of the tensor-core adds grows with the number of MMAs into
+          // an accumulator times its magnitude: the hi.hi
+          // products of each k third and the small corrections get accumulators of their own
+          const int j = (kb * jn) / nk;
+          const int kb_first = (j * nk + jn - 1) / jn;
+#pragma unroll
+          for (int kk = 0; kk < kTK / 8; ++kk) {
+            const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 TF32 = 32 bytes along K inside the atom
+            umma_tf32(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
+            umma_tf32(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
+            umma_tf32(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+          }
+          umma_commit(&sm.empty[s]);
+        }
+        umma_commit(&sm.tmem_full);
+      }
+    }
+  } else {  // ---- epilogue: warps 2..5, TMEM lane quarter (warp % 4)
+    const int q = warp & 3;
+    int it = 0;
+    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+      const int2 tile = tiles[t];
+      const int64_t r0 = (int64_t)tile.x * kTM, c0 = (int64_t)tile.y * kTN;
+      const int64_t r = r0 + q * 32 + lane;
+      mbar_wait(&sm.tmem_full, it & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      float dot[kTN];
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) {
+        uint32_t v0[32], v1[32], v2[32], w[32];
+        const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(ch * 32);
+        tmem_ld32(taddr, v0);
+        tmem_ld32(taddr + kTN, v1);
+        tmem_ld32(taddr + 2 * kTN, v2);
+        tmem_ld32(taddr + kMainAcc * kTN, w);
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          float x = __uint_as_float(v0[j]);
+          if (nk > 1) x += __uint_as_float(v1[j]);
+          if (nk > 2) x += __uint_as_float(v2[j]);
+          dot[ch * 32 + j] = x + __uint_as_float(w[j]);
+        }
+      }
+      // TMEM may be overwritten by the next tile's MMAs from here on
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+      const float nr = (r < n) ? norms[r] : 0.f;
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) {
+        const int64_t cb = c0 + ch * 32;
+        float kv[32];
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __ldg(norms + cb + j));
+          float val;
+          asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(val) : "f"(fmaxf(d2, 0.f) * scale));
+          kv[j] = (r == cb + j) ? 1.f : val;
+        }
+        // direct store K[r][c] for r <= c (row segment of 32 contiguous floats)
+        if (r < n) {
+          float* dst = K + r * ldk + cb;
+          const bool full = (cb >= r) && (cb + 31 < n) && ((ldk & 3) == 0);
+          if (full) {
+#pragma unroll
+            for (int j = 0; j < 32; j += 4)
+              *reinterpret_cast<float4*>(dst + j) = make_float4(kv[j], kv[j + 1], kv[j + 2], kv[j + 3]);
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              if (cb + j >= r && cb + j < n) dst[j] = kv[j];
+          }
+        }
+        // mirrored store K[c][r] for r < c (warp-coalesced: lanes hold consecutive rows)
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const int64_t c = cb + j;
+          if (r < c && c < n) K[c * ldk + r] = kv[j];
+        }
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
+  }
+}
+
+// Column means (deterministic two-level FP64 reduction): RBF distances are translation
+// invariant, and centring shrinks the dot products whose tensor-core accumulation error
+// limits the 3xTF32 contraction.
+constexpr int kMeanRows = 1024;
+__global__ void col_partial_kernel(const float* __restrict__ X, int64_t n, int d, double* __restrict__ part) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= d) return;
+  const int64_t r0 = (int64_t)blockIdx.y * kMeanRows;
+  const int64_t r1 = (n < r0 + kMeanRows) ? n : r0 + kMeanRows;
+  double s = 0.0;
+  for (int64_t r = r0; r < r1; ++r) s += X[r * d + c];
+  part[(int64_t)blockIdx.y * d + c] = s;
+}
+__global__ void col_mean_kernel(const double* __restrict__ part, int nchunks, int64_t n, int d, float* __restrict__ mu) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= d) return;
+  double s = 0.0;
+  for (int q = 0; q < nchunks; ++q) s += part[(int64_t)q * d + c];
+  mu[c] = (float)(s / (double)n);
+}
+
+// x' = x - mu (FP32); hi = TF32(x'), lo = TF32(x' - hi) (round to nearest);
+// norms[j] = ||x'_j||^2 accumulated in FP64 (one warp per row); zero padding.
+__global__ void split_tf32_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
+                                  const float* __restrict__ mu, float* __restrict__ hi, float* __restrict__ lo,
+                                  float* __restrict__ norms, int64_t n_pad, int d_pad) {
+  const int64_t j = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (j >= n_pad) return;
+  const int64_t src = (j < n) ? (perm ? perm[j] : j) : -1;
+  double s = 0.0;
+  for (int c = lane; c < d_pad; c += 32) {
+    float x = 0.f;
+    if (src >= 0 && c < d) x = X[src * d + c] - mu[c];
+    // round-to-nearest TF32 for both parts, so the tensor core sees exact TF32 values (it would
+    // otherwise drop the low 13 bits of lo) and the dropped lo.lo / lo-rounding terms are unbiased
+    const float h = __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+    const float r = x - h;
+    hi[j * d_pad + c] = h;
+    lo[j * d_pad + c] = __uint_as_float((__float_as_uint(r) + 0x1000u) & 0xFFFFE000u);
+    s = fma((double)x, (double)x, s);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) norms[j] = (float)s;
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, []() {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+CUtensorMap make_map(const float* base, int64_t rows, int d_pad) {
+  auto enc = get_encode();
+  if (!enc) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  CUtensorMap m;
+  const cuuint64_t dims[2] = {(cuuint64_t)d_pad, (cuuint64_t)rows};
+  const cuuint64_t strides[1] = {(cuuint64_t)d_pad * sizeof(float)};
+  const cuuint32_t box[2] = {(cuuint32_t)kTK, (cuuint32_t)kTM};
+  const cuuint32_t estr[2] = {1, 1};
+  const CUresult r = enc(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
+  return m;
+}
+
+}  // namespace
+
+int64_t krow_tc_rows_pad(int64_t n) { return round_up(n, kTN > kTM ? kTN : kTM); }
+int krow_tc_d_pad(int d) { return (int)round_up(d, kTK); }
+
+size_t krow_tc_scratch_bytes(int64_t n, int d) {
+  return (size_t)ceil_div(n, kMeanRows) * d * sizeof(double) + (size_t)d * sizeof(float);
+}
+
+void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, float* hi, float* lo, float* norms,
+                       int64_t n_pad, int d_pad, void* scratch, cudaStream_t st) {
+  const int nch = (int)ceil_div(n, kMeanRows);
+  double* part = static_cast<double*>(scratch);
+  float* mu = reinterpret_cast<float*>(part + (size_t)nch * d);
+  GM_LAUNCH(col_partial_kernel, dim3((unsigned)ceil_div(d, 128), (unsigned)nch), dim3(128), 0, st, X, n, d, part);
+  GM_LAUNCH(col_mean_kernel, dim3((unsigned)ceil_div(d, 128)), dim3(128), 0, st, part, nch, n, d, mu);
+  GM_LAUNCH(split_tf32_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, hi, lo, norms,
+            n_pad, d_pad);
+}
+
+// Tiles (bi, bj) of 128 x 128 with at least one entry r <= c, in blocked order (16 x 16 tiles)
+// so a wave of CTAs reuses its operand tiles from L2.
+std::vector<int2> krow_tc_tiles(int64_t n) {
+  const int Tr = (int)ceil_div(n, kTM), Tc = (int)ceil_div(n, kTN);
+  std::vector<int2> t;
+  for (int I = 0; I < Tr; I += 16)
+    for (int J = 0; J < Tc; J += 16)
+      for (int bi = I; bi < std::min(Tr, I + 16); ++bi)
+        for (int bj = J; bj < std::min(Tc, J + 16); ++bj)
+          if ((int64_t)(bj + 1) * kTN - 1 >= (int64_t)bi * kTM) t.push_back(make_int2(bi, bj));
+  return t;
+}
+
+void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
+                    const float* norms, int64_t n, double gamma, float* K, int64_t ldk, cudaStream_t st) {
+  const CUtensorMap mhi = make_map(hi, n_pad, d_pad), mlo = make_map(lo, n_pad, d_pad);
+  const size_t smem = sizeof(TcSmem) + 1024;
+  static bool configured = false;
+  if (!configured) {
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    configured = true;
+  }
+  const float scale = (float)(-gamma * 1.4426950408889634);
+  int sms = 148, dev = 0;
+  GM_CUDA(cudaGetDevice(&dev));
+  GM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  const int grid = n_tiles < sms ? n_tiles : sms;
+  GM_LAUNCH(krow_tc_kernel, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, d_pad / kTK,
+            scale, K, ldk);
+}
+
+}  // namespace gmpsvm

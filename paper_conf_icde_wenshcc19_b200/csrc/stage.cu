@@ -4,6 +4,9 @@
 // two contiguous class blocks of one class-sorted copy of X (kernel rows shared across
 // pairs, L313-L325).  The sorted copy is stored feature-major (XT[c][j]) and zero-padded
 // to (d_pad x n_pad) for the tile contraction; squared norms are accumulated in FP64.
+#include <cstdlib>
+#include <string>
+
 #include "kernels.h"
 
 namespace gmpsvm {
@@ -147,6 +150,16 @@ void launch_stage_features(const float* X, int64_t n, int d, const int64_t* perm
   GM_LAUNCH(gather_transpose_kernel, dim3((unsigned)ceil_div(n_pad, 32), (unsigned)ceil_div(d_pad, 32)), dim3(32, 8), 0,
             st, X, n, d, perm, XT, ldx, d_pad, n_pad);
   GM_LAUNCH(row_norms_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, norms, n_pad, bad);
+}
+
+void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
+                      cudaStream_t st) {
+  GM_LAUNCH(row_norms_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, norms, n_pad, bad);
+}
+
+bool krow_use_tc() {
+  static const bool simt = getenv("GMPSVM_KROW") && std::string(getenv("GMPSVM_KROW")) == "simt";
+  return !simt;
 }
 
 void launch_gather_rows(const float* X, int d, const int64_t* idx, int64_t nr, float* dst, cudaStream_t st) {
