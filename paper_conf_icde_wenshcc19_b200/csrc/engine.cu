@@ -35,7 +35,7 @@ constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
 constexpr int64_t kPredictChunk = 32768;
 constexpr int kMaxStreams = 48;    // concurrent pair groups in the solver
 constexpr int kDefaultStreams = 8; // default pair groups (hardware queues: CUDA_DEVICE_MAX_CONNECTIONS)
-constexpr int kDefaultB = 192;     // working-set rows: K_ws,ws stays in shared memory (B <= 224)
+constexpr int kDefaultB = 224;     // working-set rows: K_ws,ws stays in shared memory (B <= 224)
 constexpr int kChunk = 2;          // outer iterations per issued chunk
 
 struct DeviceGuard {
@@ -549,7 +549,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
       d_outer(Pl, st), d_sig(Pl, st);
   DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
-  DevBuf<float> d_Kws(local_smo_uses_smem(Bw) ? 0 : (size_t)Pl * Bw * Bw, st);
+  DevBuf<float> d_Kws((size_t)Pl * Bw * Bw, st);
   SolverArgs a{};
   a.pairs = d_pairs.get();
   a.K = K.get();
@@ -568,9 +568,12 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   a.inner_iters = d_inner.get();
   a.smo_cycles = d_cyc.get();
   static const bool smo_prof = getenv("GMPSVM_SMO_PHASES") != nullptr;
-  DevBuf<int64_t> d_phase(smo_prof ? (size_t)Pl * 4 : 0, st);
-  if (smo_prof) GM_CUDA(cudaMemsetAsync(d_phase.get(), 0, (size_t)Pl * 4 * 8, st));
+  DevBuf<int64_t> d_phase(smo_prof ? (size_t)Pl * 5 : 0, st);
+  if (smo_prof) GM_CUDA(cudaMemsetAsync(d_phase.get(), 0, (size_t)Pl * 5 * 8, st));
   a.smo_phase = smo_prof ? d_phase.get() : nullptr;
+  DevBuf<int64_t> d_sphase(smo_prof ? (size_t)(Pl + 4096) * 5 : 0, st);
+  if (smo_prof) GM_CUDA(cudaMemsetAsync(d_sphase.get(), 0, (size_t)(Pl + 4096) * 5 * 8, st));
+  a.sel_phase = smo_prof ? d_sphase.get() : nullptr;
   a.outer_iters = d_outer.get();
   a.b = d_b.get();
   a.A = d_A.get();
@@ -581,6 +584,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   a.inner_cap = opt.inner_iter_cap > 0 ? opt.inner_iter_cap : 100 * Bw;
   a.C = C;
   a.eps = eps;
+  static const double env_ratio = getenv("GMPSVM_LOCAL_RATIO") ? atof(getenv("GMPSVM_LOCAL_RATIO")) : 0.1;
+  a.local_ratio = env_ratio;
   HT("solver_alloc");
   launch_init_pairs(a, Pl, tot, st);
   const int64_t max_outer = opt.max_outer_iter > 0 ? opt.max_outer_iter : 1000000;
@@ -624,7 +629,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       const int64_t it = issued[g]++;
       launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
       if (it >= max_outer) break;  // the last selection only evaluates the stop test
-      if (!local_smo_uses_smem(Bw)) launch_gather_kws(ag, gn, it == 0 ? 1 : 0, gs);
+      launch_gather_kws(ag, gn, it == 0 ? 1 : 0, gs);
       launch_local_smo(ag, gn, gs);
       launch_f_update(ag, gn, g_npmax[g], gs);
     }
@@ -698,15 +703,33 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaStreamSynchronize(st));
 
   if (smo_prof) {
-    std::vector<int64_t> ph((size_t)Pl * 4);
+    std::vector<int64_t> ph((size_t)Pl * 5);
     GM_CUDA(cudaMemcpy(ph.data(), d_phase.get(), ph.size() * 8, cudaMemcpyDeviceToHost));
-    double tot[4] = {0, 0, 0, 0};
+    double tot[5] = {0, 0, 0, 0, 0};
     for (int i = 0; i < Pl; ++i)
-      for (int q = 0; q < 4; ++q) tot[q] += (double)ph[i * 4 + q];
-    int64_t steps = 0;
-    for (int i = 0; i < Pl; ++i) steps += h_inner[i];
-    fprintf(stderr, "[gmpsvm] local_smo cycles/step: u-reduce %.0f  row-u %.0f  l-reduce %.0f  step+row-l %.0f\n",
-            tot[0] / steps, tot[1] / steps, tot[2] / steps, tot[3] / steps);
+      for (int q = 0; q < 5; ++q) tot[q] += (double)ph[i * 5 + q];
+    int64_t steps = 0, outer = 0;
+    for (int i = 0; i < Pl; ++i) {
+      steps += h_inner[i];
+      outer += h_outer[i];
+    }
+    fprintf(stderr,
+            "[gmpsvm] local_smo cycles/step: u-reduce %.0f  row-u %.0f  l-reduce %.0f  step+row-l %.0f | "
+            "prologue cycles/launch %.0f\n",
+            tot[0] / steps, tot[1] / steps, tot[2] / steps, tot[3] / steps, tot[4] / outer);
+    GM_CUDA(cudaMemcpy(ph.data(), d_sphase.get(), ph.size() * 8, cudaMemcpyDeviceToHost));
+    double sp[5] = {0, 0, 0, 0, 0};
+    for (int i = 0; i < Pl; ++i)
+      for (int q = 0; q < 5; ++q) sp[q] += (double)ph[i * 5 + q];
+    fprintf(stderr, "[gmpsvm] select_ws cycles/launch: staging %.0f  reduce %.0f  retain %.0f  pick %.0f  copy %.0f\n",
+            sp[0] / outer, sp[1] / outer, sp[2] / outer, sp[3] / outer, sp[4] / outer);
+    std::vector<int64_t> fq((size_t)Pl * 5);
+    GM_CUDA(cudaMemcpy(fq.data(), d_sphase.get() + (size_t)4096 * 5, fq.size() * 8, cudaMemcpyDeviceToHost));
+    double fs[5] = {0, 0, 0, 0, 0};
+    for (int i = 0; i < Pl; ++i)
+      for (int q = 0; q < 5; ++q) fs[q] += (double)fq[i * 5 + q];
+    fprintf(stderr, "[gmpsvm] fast select cycles/launch: hist %.0f  scan %.0f  compact %.0f  sort+take %.0f  list %.1f\n",
+            fs[0] / outer, fs[1] / outer, fs[2] / outer, fs[3] / outer, fs[4] / outer);
   }
   auto* mdl = new Model();
   std::unique_ptr<Model> guard(mdl);

@@ -57,7 +57,8 @@ struct SolverArgs {
   double* gap;          // [P] global gap at the last selection
   int64_t* inner_iters; // [P]
   int64_t* smo_cycles;  // [P] SM clock cycles spent in local_smo (diagnostic)
-  int64_t* smo_phase;   // [P][4] optional per-phase cycles (GMPSVM_SMO_PHASES=1), else NULL
+  int64_t* smo_phase;   // [P][5] optional per-phase cycles (GMPSVM_SMO_PHASES=1), else NULL
+  int64_t* sel_phase;   // [P][5] optional select_ws phase cycles (GMPSVM_SMO_PHASES=1), else NULL
   int32_t* outer_iters; // [P]
   double* b;            // [P]
   double* A;            // [P]
@@ -66,6 +67,7 @@ struct SolverArgs {
   int B, q, inner_cap;
   int pair_base;        // first local pair of this launch (grid.x pairs from here)
   double C, eps;
+  double local_ratio;  // local solve stops at gap < max(eps, local_ratio * delta0) (reading R20: 0.1)
 };
 
 void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st);

@@ -132,6 +132,7 @@ struct SelSmem {
   int32_t hist[256];
   int32_t scan[33];
   double red[32];
+  double red4[132];
   int32_t sel_digit, sel_below, sel_count, take_all;
 };
 
@@ -311,13 +312,207 @@ __device__ int select_sides(const Src& src, int np, int need, int32_t* out, SelS
   return cnt;
 }
 
+// Fast path of the selection for shared-memory-staged pairs: one histogram pass (2048 bins,
+// linear in key over each side's [kmin, kmax]) finds the threshold bin of each side, one
+// compaction pass collects the candidates at or below it (typically ~q/2 + a few), and an
+// exact (key, index) bitonic sort of those short lists picks the working set.  Returns -1 (and
+// leaves the flags untouched) when a list would overflow; the caller then runs radix_pick.
+constexpr int kSelBins = 2048;
+constexpr int kSelListCap = 2048;
+
+struct SelLists {
+  int32_t hist[2][kSelBins];
+  uint64_t key[2][kSelListCap];
+  int32_t idx[2][kSelListCap];
+  int32_t cnt[2];
+  int32_t bin[2];
+  int32_t tot[2];
+};
+
+// bins linear in f over each side's range (monotone: f1 <= f2 => bin1 <= bin2)
+struct FBins {
+  double lo, scale;  // bin = (f - lo) * scale (U side) or (lo - f) * scale (L side, lo = max f)
+  __device__ __forceinline__ int up(double f) const { return (int)fmin((f - lo) * scale, (double)(kSelBins - 1)); }
+  __device__ __forceinline__ int down(double f) const { return (int)fmin((lo - f) * scale, (double)(kSelBins - 1)); }
+};
+__device__ __forceinline__ double fbin_scale(double span) { return span > 0.0 ? (kSelBins - 1) / span : 0.0; }
+
+// bitonic sort of (key, idx) pairs, n2 a power of two, ascending
+__device__ void bitonic_pairs(uint64_t* key, int32_t* idx, int n2) {
+  for (int k = 2; k <= n2; k <<= 1)
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+        const int p = i ^ j;
+        if (p > i) {
+          const bool up = (i & k) == 0;
+          const uint64_t ka = key[i], kb = key[p];
+          const int32_t ia = idx[i], ib = idx[p];
+          const bool gt = ka > kb || (ka == kb && ia > ib);
+          if (gt == up) {
+            key[i] = kb;
+            key[p] = ka;
+            idx[i] = ib;
+            idx[p] = ia;
+          }
+        }
+      }
+      __syncthreads();
+    }
+}
+
+__device__ int fast_select_sides(const uint64_t* keys, uint8_t* flags, int np, int need, int32_t* out,
+                                 uint64_t ku0, uint64_t ku1, uint64_t kl0, uint64_t kl1, SelLists& L, SelSmem& sm,
+                                 int64_t* tacc = nullptr) {
+  long long tq = clock64();
+  auto tmark = [&](int k) {
+    if (tacc && threadIdx.x == 0) {
+      const long long t = clock64();
+      atomicAdd((unsigned long long*)&tacc[k], (unsigned long long)(t - tq));
+      tq = t;
+    }
+  };
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const double fu0 = key_double(ku0), fu1 = key_double(ku1);    // U: smallest .. largest f over I_u
+  const double fl1 = key_double(~kl0), fl0 = key_double(~kl1);  // L: largest .. smallest f over I_l
+  const FBins bu_{fu0, fbin_scale(fu1 - fu0)}, bl_{fl1, fbin_scale(fl1 - fl0)};
+  for (int i = tid; i < 2 * kSelBins; i += blockDim.x) (&L.hist[0][0])[i] = 0;
+  if (tid < 2) L.cnt[tid] = 0;
+  __syncthreads();
+  for (int base = 0; base < np; base += blockDim.x) {
+    const int i = base + tid;
+    const uint8_t f = i < np ? flags[i] : 4;
+    const uint64_t k = i < np ? keys[i] : 0;
+    // warp-aggregated histogram updates (clustered f values hit the same bin)
+    const bool cu = (f & 5) == 1, cl = (f & 6) == 2;
+    const double fv = key_double(k);
+    const int b0 = cu ? bu_.up(fv) : -1;
+    const int b1 = cl ? bl_.down(fv) : -1;
+    const unsigned m0 = __match_any_sync(FULLMASK, b0), m1 = __match_any_sync(FULLMASK, b1);
+    if (cu && lane == __ffs(m0) - 1) atomicAdd(&L.hist[0][b0], __popc(m0));
+    if (cl && lane == __ffs(m1) - 1) atomicAdd(&L.hist[1][b1], __popc(m1));
+  }
+  __syncthreads();
+  tmark(0);
+  // warps 0 / 1: threshold bin of the U / L side (cumulative count reaches the wanted number)
+  if (warp < 2) {
+    const int side = warp;
+    int loc = 0;
+    for (int b = lane * 64; b < lane * 64 + 64; ++b) loc += L.hist[side][b];
+    int incl = loc;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(FULLMASK, incl, o);
+      if (lane >= o) incl += y;
+    }
+    const int total = __shfl_sync(FULLMASK, incl, 31);
+    const int totU = __shfl_sync(FULLMASK, incl, 31);  // this warp's own side total
+    (void)totU;
+    if (lane == 0) L.tot[side] = total;
+    // U wants need/2 (or all it has); L wants the rest (estimate; exact counts are handled below)
+    const int want = side == 0 ? min(need / 2, total) : min(need, total);
+    const int excl = incl - loc;
+    if (want == 0) {
+      if (lane == 0) L.bin[side] = -1;
+    } else if (excl < want && want <= incl) {
+      int cum = excl, b = lane * 64;
+      for (; b < lane * 64 + 64; ++b) {
+        cum += L.hist[side][b];
+        if (cum >= want) break;
+      }
+      L.bin[side] = b;
+    }
+  }
+  __syncthreads();
+  tmark(1);
+  const int bu = L.bin[0], bl = L.bin[1];
+  // compaction of the candidates at or below the threshold bins
+  for (int base = 0; base < np; base += blockDim.x) {
+    const int i = base + tid;
+    const uint8_t f = i < np ? flags[i] : 4;
+    const uint64_t k = i < np ? keys[i] : 0;
+    const double fv = key_double(k);
+    const bool tu = (f & 5) == 1 && bu_.up(fv) <= bu;
+    const bool tl = (f & 6) == 2 && bl_.down(fv) <= bl;
+    const unsigned mu = __ballot_sync(FULLMASK, tu), ml = __ballot_sync(FULLMASK, tl);
+    int pu = 0, pl = 0;
+    if (lane == 0) {
+      if (mu) pu = atomicAdd(&L.cnt[0], __popc(mu));
+      if (ml) pl = atomicAdd(&L.cnt[1], __popc(ml));
+    }
+    pu = __shfl_sync(FULLMASK, pu, 0) + __popc(mu & ((1u << lane) - 1u));
+    pl = __shfl_sync(FULLMASK, pl, 0) + __popc(ml & ((1u << lane) - 1u));
+    if (tu && pu < kSelListCap) {
+      L.key[0][pu] = k;
+      L.idx[0][pu] = i;
+    }
+    if (tl && pl < kSelListCap) {
+      L.key[1][pl] = ~k;
+      L.idx[1][pl] = i;
+    }
+  }
+  __syncthreads();
+  tmark(2);
+  const int nu = L.cnt[0], nl = L.cnt[1];
+  if (tacc && threadIdx.x == 0) atomicAdd((unsigned long long*)&tacc[4], (unsigned long long)(nu + nl));
+  if (nu > kSelListCap || nl > kSelListCap) return -1;
+  // U side: exact (key, index) order of the short list, take the first need/2
+  int n2 = 1;
+  while (n2 < nu) n2 <<= 1;
+  for (int i = nu + tid; i < n2; i += blockDim.x) {
+    L.key[0][i] = ~0ull;
+    L.idx[0][i] = INT_MAX;
+  }
+  __syncthreads();
+  bitonic_pairs(L.key[0], L.idx[0], n2);
+  const int take_u = min(need / 2, L.tot[0]);
+  for (int i = tid; i < take_u; i += blockDim.x) {
+    out[i] = L.idx[0][i];
+    flags[L.idx[0][i]] |= 4;
+  }
+  __syncthreads();
+  // L side: drop the ones U took, order, take what is still needed
+  n2 = 1;
+  while (n2 < nl) n2 <<= 1;
+  for (int i = tid; i < n2; i += blockDim.x) {
+    if (i >= nl || (flags[L.idx[1][i]] & 4)) {
+      L.key[1][i] = ~0ull;
+      L.idx[1][i] = INT_MAX;
+    }
+  }
+  __syncthreads();
+  bitonic_pairs(L.key[1], L.idx[1], n2);
+  int valid = 0;
+  for (int i = tid; i < n2; i += blockDim.x) valid += L.idx[1][i] != INT_MAX;
+  valid = block_reduce(valid, [](int x, int y) { return x + y; }, sm.scan);
+  const int need_l = need - take_u;
+  // the list holds every L candidate below the threshold bin; if U took some of them the list
+  // may be short of need_l while more candidates sit in higher bins: radix_pick completes it
+  const int take_l = min(need_l, valid);
+  for (int i = tid; i < take_l; i += blockDim.x) {
+    out[take_u + i] = L.idx[1][i];
+    flags[L.idx[1][i]] |= 4;
+  }
+  __syncthreads();
+  tmark(3);
+  return take_u + take_l;
+}
+
 constexpr int kSelSmemMax = 16384;  // n_p up to which keys + flags are staged in shared memory
 
 __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t stampv, int first) {
   __shared__ SelSmem sm;
   extern __shared__ __align__(8) unsigned char sel_dyn[];
+  const long long t0 = clock64();
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
+  long long tp = t0;
+  auto mark = [&](int k) {
+    if (a.sel_phase && threadIdx.x == 0) {
+      const long long t = clock64();
+      a.sel_phase[lp * 5 + k] += t - tp;
+      tp = t;
+    }
+  };
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   const double* al = a.alpha + pd.a_off;
@@ -345,11 +540,49 @@ __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t 
       flags[i] = (u ? 1 : 0) | (l ? 2 : 0);
     }
   }
-  fmin = block_reduce(fmin, [](double x, double y) { return x < y ? x : y; }, sm.red);
-  fmax = block_reduce(fmax, [](double x, double y) { return x > y ? x : y; }, sm.red);
-  umax = block_reduce(umax, [](double x, double y) { return x > y ? x : y; }, sm.red);
-  lmin = block_reduce(lmin, [](double x, double y) { return x < y ? x : y; }, sm.red);
+  mark(0);
+  {  // the four extremes in one block reduction: warp shuffles, then warp 0 over the warp partials
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      fmin = ::fmin(fmin, __shfl_xor_sync(FULLMASK, fmin, o));
+      fmax = ::fmax(fmax, __shfl_xor_sync(FULLMASK, fmax, o));
+      umax = ::fmax(umax, __shfl_xor_sync(FULLMASK, umax, o));
+      lmin = ::fmin(lmin, __shfl_xor_sync(FULLMASK, lmin, o));
+    }
+    double* red4 = sm.red4;
+    if (lane == 0) {
+      red4[warp] = fmin;
+      red4[32 + warp] = fmax;
+      red4[64 + warp] = umax;
+      red4[96 + warp] = lmin;
+    }
+    __syncthreads();
+    if (warp == 0) {
+      double a0 = lane < nw ? red4[lane] : DBL_MAX, a1 = lane < nw ? red4[32 + lane] : -DBL_MAX;
+      double a2 = lane < nw ? red4[64 + lane] : -DBL_MAX, a3 = lane < nw ? red4[96 + lane] : DBL_MAX;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        a0 = ::fmin(a0, __shfl_xor_sync(FULLMASK, a0, o));
+        a1 = ::fmax(a1, __shfl_xor_sync(FULLMASK, a1, o));
+        a2 = ::fmax(a2, __shfl_xor_sync(FULLMASK, a2, o));
+        a3 = ::fmin(a3, __shfl_xor_sync(FULLMASK, a3, o));
+      }
+      if (lane == 0) {
+        red4[128] = a0;
+        red4[129] = a1;
+        red4[130] = a2;
+        red4[131] = a3;
+      }
+    }
+    __syncthreads();
+    fmin = red4[128];
+    fmax = red4[129];
+    umax = red4[130];
+    lmin = red4[131];
+  }
   // key bounds of the two sides: U keys = ord(f) over I_u, L keys = ~ord(f) over I_l
+  mark(1);
   const double gap = fmax - fmin;
   const bool done = (fmin == DBL_MAX) || (fmax == -DBL_MAX) || !(gap >= a.eps);
   if (threadIdx.x == 0) {
@@ -378,17 +611,32 @@ __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t 
     else stp[idx] = stampv;
   }
   __syncthreads();
+  mark(2);
   int cnt = keep;
   const uint64_t ku0 = ord_key(fmin), ku1 = ord_key(umax), kl0 = ~ord_key(fmax), kl1 = ~ord_key(lmin);
   if (use_smem) {
     SmemSrc src{keys, flags};
-    cnt += select_sides(src, np, B - keep, nxt + cnt, sm, ku0, ku1, kl0, kl1);
+    SelLists& lists = *reinterpret_cast<SelLists*>(sel_dyn + (size_t)kSelSmemMax * 9 + 16);
+    const int need = B - keep;
+    const int got = fast_select_sides(keys, flags, np, need, nxt + cnt, ku0, ku1, kl0, kl1, lists, sm,
+                                      a.sel_phase ? a.sel_phase + (size_t)gridDim.x * 0 + 5 * 64 * 0 + a.pair_base * 0 +
+                                                        (int64_t)5 * (lp + 4096) : nullptr);
+    if (got < 0) {
+      cnt += select_sides(src, np, need, nxt + cnt, sm, ku0, ku1, kl0, kl1);
+    } else {
+      cnt += got;
+      // L side short (its candidates overlapped U's picks): complete from the full arrays
+      if (got < need) cnt += radix_pick<false>(src, np, need - got, nxt + cnt, sm, kl0, kl1);
+      if (cnt - keep < need) cnt += radix_pick<true>(src, np, keep + need - cnt, nxt + cnt, sm, ku0, ku1);
+    }
   } else {
     GlobalSrc src{al, fl, stp, stampv, pd.n_s, C};
     cnt += select_sides(src, np, B - keep, nxt + cnt, sm, ku0, ku1, kl0, kl1);
   }
+  mark(3);
   for (int e = threadIdx.x; e < cnt; e += blockDim.x) ws[e] = nxt[e];
   if (threadIdx.x == 0) a.ws_n[lp] = cnt;
+  mark(4);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -504,15 +752,16 @@ __device__ __forceinline__ bool key_less(uint32_t h, uint32_t l, int32_t i, cons
 }
 
 // E working-set rows per thread (thread t owns rows t, t + nt, ...; nt = blockDim.x).
-// SMEM: K_ws,ws (B <= kSmemMaxB) is gathered straight from the resident kernel matrix into
-// shared memory at kernel start, so the two row reads of every inner step are LDS instead of
-// L2/HBM loads; otherwise rows come from the global K_ws,ws buffer built by gather_kws.
+// SMEM: K_ws,ws (B <= kSmemMaxB, built by gather_kws) is copied into shared memory at kernel
+// start, so the two row reads of every inner step are LDS instead of L2/HBM loads; otherwise
+// rows are read from the global K_ws,ws buffer.
 constexpr int kSmemMaxB = 224;
 
 template <int E, bool SMEM>
 __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(SolverArgs a) {
   __shared__ RedSlot slots[2][32];
   extern __shared__ float kw_smem[];
+  const long long t_entry = clock64();
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
@@ -521,22 +770,11 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
   const double C = a.C;
   const float* Kw;
   if (SMEM) {
-    // gather K[g(ws_r)][g(ws_c)] for r, c < wn into shared memory (row stride B)
-    int32_t* gcol = reinterpret_cast<int32_t*>(kw_smem + (size_t)B * B);
-    for (int e = threadIdx.x; e < wn; e += nt) gcol[e] = (int32_t)gpos(pd, a.ws[(int64_t)lp * B + e]);
-    __syncthreads();
-    for (int r0 = 0; r0 < wn; r0 += 16) {
-      float v[16];
-      const int c = threadIdx.x;
-#pragma unroll
-      for (int rr = 0; rr < 16; ++rr) {
-        const int r = r0 + rr;
-        v[rr] = (r < wn && c < wn) ? __ldg(a.K + (int64_t)gcol[r] * a.ldk + gcol[c]) : 0.f;
-      }
-#pragma unroll
-      for (int rr = 0; rr < 16; ++rr)
-        if (r0 + rr < wn && c < wn) kw_smem[(r0 + rr) * B + c] = v[rr];
-    }
+    // copy this pair's K_ws,ws tile (built by gather_kws, L2-resident) into shared memory
+    const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * B * B);
+    float4* dst = reinterpret_cast<float4*>(kw_smem);
+    const int nv = (B * B) / 4;  // B is even and B*B % 4 == 0
+    for (int i = threadIdx.x; i < nv; i += nt) dst[i] = __ldg(src + i);
     __syncthreads();
     Kw = kw_smem;
   } else {
@@ -567,7 +805,7 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
   int it = 0, par = 0;
   double delta0 = 0.0;
   const long long t_begin = clock64();
-  long long ph[4] = {0, 0, 0, 0}, tp = t_begin;
+  long long ph[5] = {0, 0, 0, 0, 0}, tp = t_begin;
   const bool prof = a.smo_phase != nullptr;
   for (;;) {
     // Step 1 (Eq 4): u = argmin_{I_u} f, ties -> lowest pair-local index
@@ -658,7 +896,7 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
     const double fmax = (rl.m0 == 0u && rl.m1 == 0u) ? -DBL_MAX : key_double(((uint64_t)rl.m0 << 32) | rl.m1);
     const double gap = fmax - fu;
     if (it == 0) delta0 = gap;
-    const double tol = a.eps > 0.1 * delta0 ? a.eps : 0.1 * delta0;
+    const double tol = a.eps > a.local_ratio * delta0 ? a.eps : a.local_ratio * delta0;
     if (!(gap >= tol) || rl.idx == INT_MAX || it >= cap) break;
     const int le = rl.e;
     const double fl = rl.f, alv = rl.alpha;
@@ -728,7 +966,8 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
     a.inner_iters[lp] += it;
     a.smo_cycles[lp] += clock64() - t_begin;
     if (prof)
-      for (int k = 0; k < 4; ++k) a.smo_phase[lp * 4 + k] += ph[k];
+      for (int k = 0; k < 4; ++k) a.smo_phase[lp * 5 + k] += ph[k];
+    if (prof) a.smo_phase[lp * 5 + 4] += t_begin - t_entry;
   }
 }
 
@@ -737,17 +976,18 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
 // HBM-bound GEMV over the rows with dalpha != 0: each thread owns kFQ 16-byte column quads of
 // the pair's two class segments (aligned to the kernel matrix rows, ldk % 4 == 0) and streams
 // the rows 2 at a time (kFQ x 2 float4 loads in flight), accumulating in FP64.
-constexpr int kFQ = 2;                       // quads per thread
-constexpr int kFCols = 256 * kFQ * 4;        // columns per CTA
+constexpr int kFQ = 1;                       // quads per thread
+constexpr int kFThreads = 128;
+constexpr int kFCols = kFThreads * kFQ * 4;  // columns per CTA (512: many CTAs per pair, short latency)
 
-__global__ void __launch_bounds__(256) f_update_kernel(SolverArgs a) {
+__global__ void __launch_bounds__(kFThreads) f_update_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;  // quads of class s
   const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;  // quads of class t
   const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
-  const int64_t qcta = (int64_t)blockIdx.y * (256 * kFQ);
+  const int64_t qcta = (int64_t)blockIdx.y * (kFThreads * kFQ);
   if (qcta >= nq) return;
   __shared__ double coef[1024];
   __shared__ const float4* rowp[1024];
@@ -775,24 +1015,24 @@ __global__ void __launch_bounds__(256) f_update_kernel(SolverArgs a) {
   double acc[kFQ][4];
 #pragma unroll
   for (int u = 0; u < kFQ; ++u) {
-    const int64_t qi = qcta + threadIdx.x + u * 256;
+    const int64_t qi = qcta + threadIdx.x + u * kFThreads;
     okq[u] = qi < nq;
     seg1[u] = qi < nq1;  // a boundary quad shared by adjacent classes is owned once per segment
     gq[u] = !okq[u] ? 0 : (qi < nq1 ? q1b + qi : q2b + (qi - nq1));
 #pragma unroll
     for (int c = 0; c < 4; ++c) acc[u][c] = 0.0;
   }
-  // rows 4 at a time: kFQ x 4 independent 16-byte loads in flight per thread (Little's law at
+  // rows 8 at a time: kFQ x 8 independent 16-byte loads in flight per thread (Little's law at
   // ~1.5 us loaded-DRAM latency needs ~10 MB in flight chip-wide for 6.5 TB/s)
   int r = 0;
-  for (; r + 4 <= nnz; r += 4) {
-    float4 v[4][kFQ];
+  for (; r + 8 <= nnz; r += 8) {
+    float4 v[8][kFQ];
 #pragma unroll
-    for (int rr = 0; rr < 4; ++rr)
+    for (int rr = 0; rr < 8; ++rr)
 #pragma unroll
       for (int u = 0; u < kFQ; ++u) v[rr][u] = okq[u] ? __ldg(rowp[r + rr] + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-    for (int rr = 0; rr < 4; ++rr) {
+    for (int rr = 0; rr < 8; ++rr) {
       const double cv = coef[r + rr];
 #pragma unroll
       for (int u = 0; u < kFQ; ++u) {
@@ -999,7 +1239,7 @@ void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st)
   GM_LAUNCH(init_pairs_kernel, dim3((unsigned)ceil_div(nthr, 256)), dim3(256), 0, st, a, tot, P);
 }
 void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st) {
-  const size_t dyn = (size_t)kSelSmemMax * 9;  // keys (8 B) + flags (1 B)
+  const size_t dyn = (size_t)kSelSmemMax * 9 + 16 + sizeof(SelLists);  // keys (8 B) + flags (1 B) + lists
   static bool configured = false;
   if (!configured) {
     GM_CUDA(cudaFuncSetAttribute(select_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
@@ -1014,7 +1254,7 @@ bool local_smo_uses_smem(int B) { return B <= kSmemMaxB; }
 
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
   if (local_smo_uses_smem(a.B)) {
-    const size_t dyn = (size_t)a.B * a.B * sizeof(float) + (size_t)a.B * sizeof(int32_t);
+    const size_t dyn = (size_t)a.B * a.B * sizeof(float);
     static size_t configured = 0;
     if (dyn > configured) {
       GM_CUDA(cudaFuncSetAttribute(local_smo_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1035,7 +1275,7 @@ void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
 }
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
   // +8 columns: each class segment may add a partial quad at either end
-  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, kFCols)), dim3(256), 0, st, a);
+  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, kFCols)), dim3(kFThreads), 0, st, a);
 }
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st) {
   GM_LAUNCH(finalize_kernel, dim3(P), dim3(1024), 0, st, a);

@@ -20,7 +20,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="mnist")
 ap.add_argument("--eps", type=float, default=1e-3)
 ap.add_argument("--reps", type=int, default=1)
-ap.add_argument("--ws-size", type=int, default=192)
+ap.add_argument("--ws-size", type=int, default=224)
 a = ap.parse_args()
 spec, X, y, Xt, yt = datagen.make_config(a.config)
 dev = torch.device("cuda:0")
