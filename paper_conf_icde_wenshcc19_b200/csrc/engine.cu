@@ -70,6 +70,18 @@ cudaStream_t get_stream(const gmpsvm_options& opt) {
   return g_streams[dev];
 }
 
+size_t device_total_mem(int dev) {
+  static std::mutex mu;
+  static size_t total[64] = {};
+  std::lock_guard<std::mutex> lk(mu);
+  if (!total[dev]) {
+    cudaDeviceProp p;
+    GM_CUDA(cudaGetDeviceProperties(&p, dev));
+    total[dev] = p.totalGlobalMem;
+  }
+  return total[dev];
+}
+
 // Per-device pool of non-blocking streams for the concurrent pair groups.
 std::mutex g_pool_mu;
 std::vector<cudaStream_t> g_pools[64];
@@ -514,10 +526,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   // ---------------- a2 kernel values: FULL_K regime (the whole class-sorted matrix)
   const int64_t ldk = round_up(n, 4);
   const double bytes_K = (double)n * ldk * 4.0;
-  size_t free_b = 0, total_b = 0;
   HT("memgetinfo");
-  GM_CUDA(cudaMemGetInfo(&free_b, &total_b));
-  const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)free_b;
+  // default budget: 85% of the device memory (cached per device; cudaMemGetInfo can take
+  // tens of milliseconds, so it is not queried per call)
+  const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)device_total_mem(opt.device);
   if (bytes_K > budget)
     throw Error(GMPSVM_ENOTIMPL, "kernel matrix (" + std::to_string(bytes_K / 1e9) +
                                      " GB) exceeds the cache budget; the ROW_CACHE regime is not in this build");
@@ -640,9 +652,16 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     GM_CUDA(cudaEventRecord(ev, gs));
     inflight[g].push_back(Chunk{ev, slot});
   };
-  for (int g = 0; g < G; ++g) issue_chunk(g);
-  for (int g = 0; g < G; ++g) issue_chunk(g);
-  int running = G;
+  const bool fused = fused_solver_enabled(Bw);
+  if (fused) {  // the whole outer loop of every pair in one launch (clusters, no host round trips)
+    SolverArgs ag = a;
+    ag.pair_base = 0;
+    launch_pair_solver(ag, Pl, max_outer, pool[0]);
+  } else {
+    for (int g = 0; g < G; ++g) issue_chunk(g);
+    for (int g = 0; g < G; ++g) issue_chunk(g);
+  }
+  int running = fused ? 0 : G;
   while (running > 0) {
     bool progressed = false;
     for (int g = 0; g < G; ++g) {
@@ -730,6 +749,11 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       for (int q = 0; q < 5; ++q) fs[q] += (double)fq[i * 5 + q];
     fprintf(stderr, "[gmpsvm] fast select cycles/launch: hist %.0f  scan %.0f  compact %.0f  sort+take %.0f  list %.1f\n",
             fs[0] / outer, fs[1] / outer, fs[2] / outer, fs[3] / outer, fs[4] / outer);
+    std::string per;
+    for (int i = 0; i < Pl; ++i)
+      per += " (" + std::to_string(hp[i].s) + "," + std::to_string(hp[i].t) + "):" + std::to_string(h_outer[i]) + "/" +
+             std::to_string(h_inner[i]);
+    fprintf(stderr, "[gmpsvm] per pair outer/inner:%s\n", per.c_str());
   }
   auto* mdl = new Model();
   std::unique_ptr<Model> guard(mdl);

@@ -76,6 +76,9 @@ void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st);
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st);
 bool local_smo_uses_smem(int B);  // K_ws,ws gathered in-kernel (no gather_kws launch, no Kws buffer)
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
+// fused outer loop: one cluster per pair, whole solve in one launch (B <= 224)
+bool fused_solver_enabled(int B);
+void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStream_t st);
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st);

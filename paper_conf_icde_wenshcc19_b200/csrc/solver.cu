@@ -15,6 +15,7 @@
 #include <cfloat>
 #include <climits>
 #include <cstdlib>
+#include <string>
 
 #include "kernels.h"
 
@@ -499,11 +500,10 @@ __device__ int fast_select_sides(const uint64_t* keys, uint8_t* flags, int np, i
 
 constexpr int kSelSmemMax = 16384;  // n_p up to which keys + flags are staged in shared memory
 
-__global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t stampv, int first) {
-  __shared__ SelSmem sm;
-  extern __shared__ __align__(8) unsigned char sel_dyn[];
+// Selection of one pair by the whole CTA (1024 threads); sel_dyn: >= kSelDynBytes of smem.
+__device__ void select_body(const SolverArgs& a, int lp, uint32_t stampv, int first, SelSmem& sm,
+                            unsigned char* sel_dyn) {
   const long long t0 = clock64();
-  const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   long long tp = t0;
   auto mark = [&](int k) {
@@ -639,9 +639,32 @@ __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t 
   mark(4);
 }
 
+constexpr size_t kSelDynBytes = (size_t)kSelSmemMax * 9 + 16 + sizeof(SelLists);
+
+__global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t stampv, int first) {
+  __shared__ SelSmem sm;
+  extern __shared__ __align__(16) unsigned char sel_dyn[];
+  select_body(a, blockIdx.x + a.pair_base, stampv, first, sm, sel_dyn);
+}
+
 // ------------------------------------------------------------------------------------------
 // a3: K_ws,ws gathered into a dense B x B tile per pair (L2-resident during local_smo)
 constexpr int kGatherRows = 16;
+
+// rows [r0, r1) of the pair's K_ws,ws tile (g: >= wn int64 of scratch, filled here)
+__device__ void gather_rows_body(const SolverArgs& a, int lp, int r0, int r1, int64_t* g) {
+  const PairDesc pd = a.pairs[lp];
+  const int wn = a.ws_n[lp];
+  const int32_t* ws = a.ws + (int64_t)lp * a.B;
+  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
+  __syncthreads();
+  r1 = min(wn, r1);
+  for (int r = r0; r < r1; ++r) {
+    const float* row = a.K + g[r] * a.ldk;
+    float* dst = a.Kws + ((int64_t)lp * a.B + r) * a.B;
+    for (int e = threadIdx.x; e < wn; e += blockDim.x) dst[e] = __ldg(row + g[e]);
+  }
+}
 
 __global__ void __launch_bounds__(256) gather_kws_kernel(SolverArgs a, int first) {
   const int lp = blockIdx.x + a.pair_base;
@@ -649,19 +672,10 @@ __global__ void __launch_bounds__(256) gather_kws_kernel(SolverArgs a, int first
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   if (np <= a.B && !first) return;  // working set unchanged
-  const int wn = a.ws_n[lp];
   const int r0 = blockIdx.y * kGatherRows;
-  if (r0 >= wn) return;
+  if (r0 >= a.ws_n[lp]) return;
   __shared__ int64_t g[1024];
-  const int32_t* ws = a.ws + (int64_t)lp * a.B;
-  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
-  __syncthreads();
-  const int r1 = min(wn, r0 + kGatherRows);
-  for (int r = r0; r < r1; ++r) {
-    const float* row = a.K + g[r] * a.ldk;
-    float* dst = a.Kws + ((int64_t)lp * a.B + r) * a.B;
-    for (int e = threadIdx.x; e < wn; e += blockDim.x) dst[e] = __ldg(row + g[e]);
-  }
+  gather_rows_body(a, lp, r0, r0 + kGatherRows, g);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -702,9 +716,14 @@ __device__ __forceinline__ void warp_max64(uint32_t& h, uint32_t& l) {
 }
 
 // Block argmin of (k0,k1,idx) carrying the payload and (WITH_MAX) a running max key (m0,m1).
+// barrier over the first nt threads of the CTA (id 0 with nt == blockDim.x is __syncthreads)
+__device__ __forceinline__ void bar_sync(int id, int nt) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nt) : "memory");
+}
+
 template <bool WITH_MAX>
-__device__ __forceinline__ RedSlot block_argmin(const RedSlot& c, RedSlot* slots) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+__device__ __forceinline__ RedSlot block_argmin(const RedSlot& c, RedSlot* slots, int nt, int bar_id) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = nt >> 5;
   uint32_t k0 = c.k0, k1 = c.k1, mh = c.m0, ml = c.m1;
   int32_t idx = c.idx;
   const int wl = warp_argmin(k0, k1, idx);
@@ -715,7 +734,7 @@ __device__ __forceinline__ RedSlot block_argmin(const RedSlot& c, RedSlot* slots
     s.m1 = ml;
     slots[warp] = s;
   }
-  __syncthreads();
+  bar_sync(bar_id, nt);
   if (lane < nw) {
     k0 = slots[lane].k0;
     k1 = slots[lane].k1;
@@ -757,16 +776,13 @@ __device__ __forceinline__ bool key_less(uint32_t h, uint32_t l, int32_t i, cons
 // rows are read from the global K_ws,ws buffer.
 constexpr int kSmemMaxB = 224;
 
+// Run by threads [0, nt) of a CTA; bar_id/nt name the barrier those threads share.
 template <int E, bool SMEM>
-__global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(SolverArgs a) {
-  __shared__ RedSlot slots[2][32];
-  extern __shared__ float kw_smem[];
+__device__ void smo_body(const SolverArgs& a, int lp, int nt, int bar_id, RedSlot (*slots)[32], float* kw_smem) {
   const long long t_entry = clock64();
-  const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int B = a.B, wn = a.ws_n[lp];
-  const int nt = blockDim.x;
   const double C = a.C;
   const float* Kw;
   if (SMEM) {
@@ -775,7 +791,7 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
     float4* dst = reinterpret_cast<float4*>(kw_smem);
     const int nv = (B * B) / 4;  // B is even and B*B % 4 == 0
     for (int i = threadIdx.x; i < nv; i += nt) dst[i] = __ldg(src + i);
-    __syncthreads();
+    bar_sync(bar_id, nt);
     Kw = kw_smem;
   } else {
     Kw = a.Kws + (int64_t)lp * B * B;
@@ -826,7 +842,7 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
         }
       }
     }
-    const RedSlot ru = block_argmin<false>(c, slots[par]);
+    const RedSlot ru = block_argmin<false>(c, slots[par], nt, bar_id);
     par ^= 1;
     if (prof) {
       const long long t = clock64();
@@ -886,7 +902,7 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
         }
       }
     }
-    const RedSlot rl = block_argmin<true>(c, slots[par]);
+    const RedSlot rl = block_argmin<true>(c, slots[par], nt, bar_id);
     par ^= 1;
     if (prof) {
       const long long t = clock64();
@@ -971,6 +987,13 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
   }
 }
 
+template <int E, bool SMEM>
+__global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(SolverArgs a) {
+  __shared__ RedSlot slots[2][32];
+  extern __shared__ float kw_smem[];
+  smo_body<E, SMEM>(a, blockIdx.x + a.pair_base, blockDim.x, 0, slots, kw_smem);
+}
+
 // ------------------------------------------------------------------------------------------
 // a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij for all j in the pair.
 // HBM-bound GEMV over the rows with dalpha != 0: each thread owns kFQ 16-byte column quads of
@@ -980,18 +1003,21 @@ constexpr int kFQ = 1;                       // quads per thread
 constexpr int kFThreads = 128;
 constexpr int kFCols = kFThreads * kFQ * 4;  // columns per CTA (512: many CTAs per pair, short latency)
 
-__global__ void __launch_bounds__(kFThreads) f_update_kernel(SolverArgs a) {
-  const int lp = blockIdx.x + a.pair_base;
-  if (a.status[lp] != 0) return;
+struct FupSmem {
+  double coef[1024];
+  const float4* rowp[1024];
+  int scan[33];
+};
+
+// Quad range [q0, q1) of the pair's concatenated class segments, any blockDim (kFQ quads per
+// thread per sweep).  Returns early (uniformly) when no alpha changed.
+__device__ void fupdate_body(const SolverArgs& a, int lp, int64_t q0, int64_t q1, FupSmem& fs) {
   const PairDesc pd = a.pairs[lp];
   const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;  // quads of class s
   const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;  // quads of class t
   const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
-  const int64_t qcta = (int64_t)blockIdx.y * (kFThreads * kFQ);
-  if (qcta >= nq) return;
-  __shared__ double coef[1024];
-  __shared__ const float4* rowp[1024];
-  __shared__ int scan_sm[33];
+  q1 = q1 < nq ? q1 : nq;
+  if (q0 >= q1) return;
   const int B = a.B, wn = a.ws_n[lp];
   const int32_t* ws = a.ws + (int64_t)lp * B;
   const double* dc = a.dcoef + (int64_t)lp * B;
@@ -1001,74 +1027,177 @@ __global__ void __launch_bounds__(kFThreads) f_update_kernel(SolverArgs a) {
     const double c = (e < wn) ? dc[e] : 0.0;
     const bool nz = c != 0.0;
     int tot = 0;
-    const int pos = block_excl_scan(nz, tot, scan_sm);
+    const int pos = block_excl_scan(nz, tot, fs.scan);
     if (nz) {
-      coef[nnz + pos] = c;
-      rowp[nnz + pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, ws[e]) * a.ldk);
+      fs.coef[nnz + pos] = c;
+      fs.rowp[nnz + pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, ws[e]) * a.ldk);
     }
     nnz += tot;
   }
   __syncthreads();
   if (nnz == 0) return;
-  int64_t gq[kFQ];
-  bool okq[kFQ], seg1[kFQ];
-  double acc[kFQ][4];
-#pragma unroll
-  for (int u = 0; u < kFQ; ++u) {
-    const int64_t qi = qcta + threadIdx.x + u * kFThreads;
-    okq[u] = qi < nq;
-    seg1[u] = qi < nq1;  // a boundary quad shared by adjacent classes is owned once per segment
-    gq[u] = !okq[u] ? 0 : (qi < nq1 ? q1b + qi : q2b + (qi - nq1));
-#pragma unroll
-    for (int c = 0; c < 4; ++c) acc[u][c] = 0.0;
-  }
-  // rows 8 at a time: kFQ x 8 independent 16-byte loads in flight per thread (Little's law at
-  // ~1.5 us loaded-DRAM latency needs ~10 MB in flight chip-wide for 6.5 TB/s)
-  int r = 0;
-  for (; r + 8 <= nnz; r += 8) {
-    float4 v[8][kFQ];
-#pragma unroll
-    for (int rr = 0; rr < 8; ++rr)
-#pragma unroll
-      for (int u = 0; u < kFQ; ++u) v[rr][u] = okq[u] ? __ldg(rowp[r + rr] + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll
-    for (int rr = 0; rr < 8; ++rr) {
-      const double cv = coef[r + rr];
-#pragma unroll
-      for (int u = 0; u < kFQ; ++u) {
-        acc[u][0] = fma(cv, (double)v[rr][u].x, acc[u][0]);
-        acc[u][1] = fma(cv, (double)v[rr][u].y, acc[u][1]);
-        acc[u][2] = fma(cv, (double)v[rr][u].z, acc[u][2]);
-        acc[u][3] = fma(cv, (double)v[rr][u].w, acc[u][3]);
-      }
-    }
-  }
-  for (; r < nnz; ++r) {
-    const float4* p0 = rowp[r];
-    const double c0v = coef[r];
+  double* f = a.f + pd.a_off;
+  for (int64_t qs = q0; qs < q1; qs += (int64_t)blockDim.x * kFQ) {
+    int64_t gq[kFQ];
+    bool okq[kFQ], seg1[kFQ];
+    double acc[kFQ][4];
 #pragma unroll
     for (int u = 0; u < kFQ; ++u) {
-      const float4 v0 = okq[u] ? __ldg(p0 + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
-      acc[u][0] = fma(c0v, (double)v0.x, acc[u][0]);
-      acc[u][1] = fma(c0v, (double)v0.y, acc[u][1]);
-      acc[u][2] = fma(c0v, (double)v0.z, acc[u][2]);
-      acc[u][3] = fma(c0v, (double)v0.w, acc[u][3]);
+      const int64_t qi = qs + threadIdx.x + (int64_t)u * blockDim.x;
+      okq[u] = qi < q1;
+      seg1[u] = qi < nq1;  // a boundary quad shared by adjacent classes is owned once per segment
+      gq[u] = !okq[u] ? 0 : (qi < nq1 ? q1b + qi : q2b + (qi - nq1));
+#pragma unroll
+      for (int c = 0; c < 4; ++c) acc[u][c] = 0.0;
     }
-  }
-  double* f = a.f + pd.a_off;
+    // rows 8 at a time: kFQ x 8 independent 16-byte loads in flight per thread (Little's law at
+    // ~1.5 us loaded-DRAM latency needs ~10 MB in flight chip-wide for 6.5 TB/s)
+    int r = 0;
+    for (; r + 8 <= nnz; r += 8) {
+      float4 v[8][kFQ];
 #pragma unroll
-  for (int u = 0; u < kFQ; ++u) {
-    if (!okq[u]) continue;
+      for (int rr = 0; rr < 8; ++rr)
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
-      const int64_t g = gq[u] * 4 + c;  // global (class-sorted) column
-      if (seg1[u]) {
-        if (g >= pd.off_s && g < pd.off_s + pd.n_s) f[g - pd.off_s] += acc[u][c];
-      } else if (g >= pd.off_t && g < pd.off_t + pd.n_t) {
-        f[pd.n_s + (g - pd.off_t)] += acc[u][c];
+        for (int u = 0; u < kFQ; ++u)
+          v[rr][u] = okq[u] ? __ldg(fs.rowp[r + rr] + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+      for (int rr = 0; rr < 8; ++rr) {
+        const double cv = fs.coef[r + rr];
+#pragma unroll
+        for (int u = 0; u < kFQ; ++u) {
+          acc[u][0] = fma(cv, (double)v[rr][u].x, acc[u][0]);
+          acc[u][1] = fma(cv, (double)v[rr][u].y, acc[u][1]);
+          acc[u][2] = fma(cv, (double)v[rr][u].z, acc[u][2]);
+          acc[u][3] = fma(cv, (double)v[rr][u].w, acc[u][3]);
+        }
+      }
+    }
+    for (; r < nnz; ++r) {
+      const float4* p0 = fs.rowp[r];
+      const double c0v = fs.coef[r];
+#pragma unroll
+      for (int u = 0; u < kFQ; ++u) {
+        const float4 v0 = okq[u] ? __ldg(p0 + gq[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+        acc[u][0] = fma(c0v, (double)v0.x, acc[u][0]);
+        acc[u][1] = fma(c0v, (double)v0.y, acc[u][1]);
+        acc[u][2] = fma(c0v, (double)v0.z, acc[u][2]);
+        acc[u][3] = fma(c0v, (double)v0.w, acc[u][3]);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kFQ; ++u) {
+      if (!okq[u]) continue;
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        const int64_t g = gq[u] * 4 + c;  // global (class-sorted) column
+        if (seg1[u]) {
+          if (g >= pd.off_s && g < pd.off_s + pd.n_s) f[g - pd.off_s] += acc[u][c];
+        } else if (g >= pd.off_t && g < pd.off_t + pd.n_t) {
+          f[pd.n_s + (g - pd.off_t)] += acc[u][c];
+        }
       }
     }
   }
+}
+
+__global__ void __launch_bounds__(kFThreads) f_update_kernel(SolverArgs a) {
+  const int lp = blockIdx.x + a.pair_base;
+  if (a.status[lp] != 0) return;
+  __shared__ FupSmem fs;
+  const int64_t q0 = (int64_t)blockIdx.y * (kFThreads * kFQ);
+  fupdate_body(a, lp, q0, q0 + kFThreads * kFQ, fs);
+}
+
+
+// ------------------------------------------------------------------------------------------
+// a3-a6 fused: one thread-block cluster of nc CTAs runs the whole outer loop of one pair
+// (Algorithm 2 lines 5-12) without returning to the host.  Per outer iteration:
+//   all CTAs   f-update of the previous local solve, columns split across the cluster
+//   CTA 0      working-set selection + stop test (all threads)
+//   all CTAs   K_ws,ws gather, rows split across the cluster
+//   CTA 0      local SMO on the first round_up(B, 32) threads (named barrier 1)
+// separated by cluster barriers (release/acquire at cluster scope also order the global
+// memory the phases exchange).  Pairs progress independently -- no lock-step with the slowest
+// pair, no host round trip per outer iteration.  Shared memory is reused by the phases.
+constexpr size_t kFusedDynBytes =
+    kSelDynBytes > (size_t)kSmemMaxB * kSmemMaxB * 4 ? kSelDynBytes : (size_t)kSmemMaxB * kSmemMaxB * 4;
+
+constexpr int kFusedThreads = 512;  // 128 registers per thread for the local SMO loop
+
+__global__ void __launch_bounds__(kFusedThreads, 1) pair_solver_kernel(SolverArgs a, int64_t max_outer) {
+  __shared__ SelSmem sm;
+  __shared__ RedSlot slots[2][32];
+  extern __shared__ __align__(16) unsigned char dyn[];
+  uint32_t nc, rank;
+  asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(nc));
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  const int lp = blockIdx.x / nc + a.pair_base;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const int64_t nq = (((pd.off_s + pd.n_s + 3) >> 2) - (pd.off_s >> 2)) + (((pd.off_t + pd.n_t + 3) >> 2) - (pd.off_t >> 2));
+  const int nts = (a.B + 31) / 32 * 32;
+  auto cluster_sync = []() {
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+  };
+  for (int64_t it = 0;; ++it) {
+    if (it > 0) {
+      const int64_t per = (nq + nc - 1) / nc;
+      fupdate_body(a, lp, rank * per, rank * per + per, *reinterpret_cast<FupSmem*>(dyn));
+      __syncthreads();
+    }
+    cluster_sync();
+    if (rank == 0) select_body(a, lp, (uint32_t)(it + 1), it == 0 ? 1 : 0, sm, dyn);
+    __syncthreads();
+    cluster_sync();
+    if (*(volatile int32_t*)(a.status + lp) != 0 || it >= max_outer) break;
+    if (np > a.B || it == 0) {
+      const int wn = *(volatile int32_t*)(a.ws_n + lp);
+      const int per = (wn + (int)nc - 1) / (int)nc;
+      gather_rows_body(a, lp, rank * per, rank * per + per, reinterpret_cast<int64_t*>(dyn));
+      __syncthreads();
+    }
+    cluster_sync();
+    if (rank == 0 && (int)threadIdx.x < nts) smo_body<1, true>(a, lp, nts, 1, slots, reinterpret_cast<float*>(dyn));
+    __syncthreads();
+    cluster_sync();
+  }
+}
+
+int fused_solver_cluster() {
+  static const int nc = getenv("GMPSVM_CLUSTER") ? atoi(getenv("GMPSVM_CLUSTER")) : 3;
+  return nc < 1 ? 1 : (nc > 8 ? 8 : nc);
+}
+
+void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStream_t st) {
+  const int nc = fused_solver_cluster();
+  static bool configured = false;
+  if (!configured) {
+    GM_CUDA(cudaFuncSetAttribute(pair_solver_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFusedDynBytes));
+    configured = true;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)(P * nc));
+  cfg.blockDim = dim3(kFusedThreads);
+  cfg.dynamicSmemBytes = kFusedDynBytes;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = nc;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  GM_CUDA(cudaLaunchKernelEx(&cfg, pair_solver_kernel, a, max_outer));
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+}
+
+// Default: the stream-group solver (measured faster on MNIST-shaped data, where the hardest
+// pair's chain dominates and benefits from whole-GPU f-update / gather launches);
+// GMPSVM_SOLVER=fused selects the one-launch cluster solver.
+bool fused_solver_enabled(int B) {
+  static const bool on = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "fused";
+  return on && B <= kSmemMaxB;
 }
 
 // ------------------------------------------------------------------------------------------
