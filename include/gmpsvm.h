@@ -64,7 +64,12 @@ typedef struct {
   int32_t q;                /* new violators per outer iteration (L289, L297); default B/2;
                                the newest B-q rows of the previous working set are kept     */
   int32_t device;           /* CUDA device ordinal                                           */
-  int64_t cache_bytes;      /* kernel-value cache budget in bytes; 0 = 85% of free memory   */
+  int64_t cache_bytes;      /* kernel-value cache budget in bytes; 0 = 85% of device memory.
+                               n*round_up(n,4)*4 <= budget: FULL_K (whole matrix resident);
+                               else ROW_CACHE: per pair a B x round_up(n_p,4) row buffer, the
+                               rows of each outer iteration's new working-set entries computed
+                               on demand (L297-L303); GMPSVM_ENOTIMPL if even the
+                               row buffers exceed 85% of device memory                       */
   void* stream;             /* cudaStream_t to run on (NULL = a library-owned stream)       */
   const int32_t* pair_ids;  /* train only these pair indices (multi-GPU sharding); NULL = all */
   int32_t n_pair_ids;
@@ -85,13 +90,15 @@ typedef struct {
   double t_fupdate_ms;      /* a6: f update                                                   */
   double t_finalize_ms;     /* a7-a9: bias, decision values, sigmoid fit, model assembly    */
   double kernel_flops;      /* flops executed by krow_contract (2d+3 per computed value)     */
-  double kernel_values;     /* kernel values computed (distinct, symmetric half + diagonal)  */
-  int64_t krow_launches;    /* launches of krow_contract                                      */
+  double kernel_values;     /* kernel values computed (FULL_K: distinct, symmetric half +
+                               diagonal; ROW_CACHE: rows computed x n_p, summed over pairs)   */
+  int64_t krow_launches;    /* launches of the kernel-value contraction (FULL_K: 1;
+                               ROW_CACHE: one per issued outer iteration per pair group)      */
   int64_t outer_iters_max;  /* max over pairs of outer iterations                             */
   int64_t outer_iters_sum;  /* sum over pairs                                                 */
   int64_t inner_iters_sum;  /* sum over pairs and working sets of inner SMO steps            */
   int64_t n_sv;             /* |SV union| over the trained pairs                              */
-  int32_t cache_regime;     /* 0 = FULL_K (whole kernel matrix resident)                     */
+  int32_t cache_regime;     /* 0 = FULL_K (whole kernel matrix resident), 1 = ROW_CACHE       */
   int32_t n_pairs_trained;
   int64_t launches;         /* kernels launched by this call                                  */
   int64_t smo_cycles_sum;   /* SM clock cycles spent in the local SMO, summed over pairs      */

@@ -53,6 +53,7 @@ struct PairDesc {
   int64_t a_off;       // offset of this pair in the concatenated alpha/f arrays
   int32_t pid;         // global pair index
   int32_t pad;
+  int64_t r_off;       // ROW_CACHE: offset of this pair's B x ldr row buffer (ldr = round_up(n_p, 4))
 };
 
 __host__ __device__ inline int pair_index(int s, int t, int k) { return s * k - s * (s + 1) / 2 + (t - s - 1); }

@@ -457,9 +457,19 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   for (int c = 0; c < k; ++c)
     if (cc[c] == 0) throw Error(GMPSVM_EINVAL, "every class must have at least one instance");
   launch_class_rank(dy, n, k, blk_off.get(), d_off.get(), d_perm.get(), st);
-  const bool use_tc = krow_use_tc();
+  // a2 regime: FULL_K keeps the whole class-sorted n x n kernel matrix
+  // resident when it fits the cache budget; otherwise ROW_CACHE computes the rows of each
+  // pair's new working-set entries per outer iteration into a B-row buffer per pair.
+  const int64_t ldk = round_up(n, 4);
+  const double bytes_K = (double)n * ldk * 4.0;
+  // default budget: 85% of the device memory (cached per device; cudaMemGetInfo can take
+  // tens of milliseconds, so it is not queried per call)
+  const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)device_total_mem(opt.device);
+  const bool full_k = bytes_K <= budget;
+  const bool use_tc = full_k && krow_use_tc();
   const int d_pad = use_tc ? krow_tc_d_pad(d) : (int)round_up(d, kBK);
-  const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile);
+  // ROW_CACHE column tiles start at 4-aligned segment starts and may run 127 columns past n
+  const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile) + (full_k ? 0 : kTile);
   // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split
   DevBuf<float> XT(use_tc ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad, st);
   DevBuf<float> Xhi(use_tc ? (size_t)n_pad * d_pad : 0, st), Xlo(use_tc ? (size_t)n_pad * d_pad : 0, st);
@@ -523,17 +533,22 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     np_max = std::max<int64_t>(np_max, x.n_s + x.n_t);
   }
 
-  // ---------------- a2 kernel values: FULL_K regime (the whole class-sorted matrix)
-  const int64_t ldk = round_up(n, 4);
-  const double bytes_K = (double)n * ldk * 4.0;
+  // ---------------- a2 kernel values
   HT("memgetinfo");
-  // default budget: 85% of the device memory (cached per device; cudaMemGetInfo can take
-  // tens of milliseconds, so it is not queried per call)
-  const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)device_total_mem(opt.device);
-  if (bytes_K > budget)
-    throw Error(GMPSVM_ENOTIMPL, "kernel matrix (" + std::to_string(bytes_K / 1e9) +
-                                     " GB) exceeds the cache budget; the ROW_CACHE regime is not in this build");
-  KWorkspace K(opt.device, (size_t)n * ldk * sizeof(float), st);
+  const int ldat = (int)round_up(B, kTile);
+  double bytes_R = 0;
+  for (auto& x : hp) {
+    x.r_off = (int64_t)(bytes_R / 4);
+    bytes_R += (double)B * round_up(x.n_s + x.n_t, 4) * 4.0;
+  }
+  if (!full_k) {
+    const double rc_total = bytes_R + (double)Pl * d_pad * ldat * 4.0;
+    if (rc_total > 0.85 * (double)device_total_mem(opt.device))
+      throw Error(GMPSVM_ENOTIMPL, "ROW_CACHE buffers (" + std::to_string(rc_total / 1e9) +
+                                       " GB) exceed the device memory; train the pairs in parts (pair_ids) and merge");
+  }
+  // FULL_K: the n x ldk matrix; ROW_CACHE: the per-pair B x round_up(n_p, 4) row buffers
+  KWorkspace K(opt.device, full_k ? (size_t)n * ldk * sizeof(float) : (size_t)bytes_R, st);
   HT("k_alloc");
   std::vector<int2> tiles;
   DevBuf<int2> d_tiles;
@@ -546,7 +561,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   if (use_tc)
     launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, K.get(),
                    ldk, st);
-  else
+  else if (full_k)
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   tm.mark(PH_KERNEL);
   HT("krow_launched");
@@ -562,10 +577,27 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       d_outer(Pl, st), d_sig(Pl, st);
   DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
   DevBuf<float> d_Kws((size_t)Pl * Bw * Bw, st);
+  const bool rc = !full_k;
+  DevBuf<int32_t> d_slot(rc ? (size_t)Pl * Bw : 0, st), d_slot_tmp(rc ? (size_t)Pl * Bw : 0, st), d_keep(rc ? Pl : 0, st);
+  DevBuf<float> d_ATnew(rc ? (size_t)Pl * d_pad * ldat : 0, st);
+  DevBuf<int64_t> d_rows(rc ? Pl : 0, st);
+  if (rc) GM_CUDA(cudaMemsetAsync(d_rows.get(), 0, Pl * 8, st));
   SolverArgs a{};
   a.pairs = d_pairs.get();
-  a.K = K.get();
+  a.K = full_k ? K.get() : nullptr;
   a.ldk = ldk;
+  a.R = rc ? K.get() : nullptr;
+  a.ws_slot = d_slot.get();
+  a.ws_slot_tmp = d_slot_tmp.get();
+  a.ws_keep = d_keep.get();
+  a.rows_done = d_rows.get();
+  a.XT = XT.get();
+  a.ldx = n_pad;
+  a.norms = norms.get();
+  a.ATnew = d_ATnew.get();
+  a.d_pad = d_pad;
+  a.ldat = ldat;
+  a.gamma = gamma;
   a.alpha = d_alpha.get();
   a.f = d_f.get();
   a.v = d_v.get();
@@ -632,6 +664,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   std::vector<int64_t> issued(G, 0);
   std::vector<int> nchunks(G, 0);
   std::vector<char> stop(G, 0);
+  int64_t rc_launches = 0;  // ROW_CACHE row-contraction launches
   auto issue_chunk = [&](int g) {
     cudaStream_t gs = pool[g];
     SolverArgs ag = a;
@@ -641,6 +674,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       const int64_t it = issued[g]++;
       launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
       if (it >= max_outer) break;  // the last selection only evaluates the stop test
+      if (rc) {
+        launch_rows_compute(ag, gn, g_npmax[g], gs);
+        ++rc_launches;
+      }
       launch_gather_kws(ag, gn, it == 0 ? 1 : 0, gs);
       launch_local_smo(ag, gn, gs);
       launch_f_update(ag, gn, g_npmax[g], gs);
@@ -652,7 +689,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     GM_CUDA(cudaEventRecord(ev, gs));
     inflight[g].push_back(Chunk{ev, slot});
   };
-  const bool fused = fused_solver_enabled(Bw);
+  const bool fused = full_k && fused_solver_enabled(Bw);
   if (fused) {  // the whole outer loop of every pair in one launch (clusters, no host round trips)
     SolverArgs ag = a;
     ag.pair_base = 0;
@@ -809,15 +846,23 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   s.t_finalize_ms = tm.ms(PH_FIN);
   s.t_solver_ms = tm.ms(PH_SOLVER);
   s.n_streams = G;
-  s.kernel_values = (double)n * (double)(n + 1) / 2.0;
+  if (full_k) {
+    s.kernel_values = (double)n * (double)(n + 1) / 2.0;
+    s.krow_launches = 1;
+  } else {
+    std::vector<int64_t> rows(Pl);
+    GM_CUDA(cudaMemcpy(rows.data(), d_rows.get(), Pl * 8, cudaMemcpyDeviceToHost));
+    s.kernel_values = 0;
+    for (int i = 0; i < Pl; ++i) s.kernel_values += (double)rows[i] * (double)(hp[i].n_s + hp[i].n_t);
+    s.krow_launches = rc_launches;
+  }
   s.kernel_flops = s.kernel_values * (2.0 * d + 3.0);
-  s.krow_launches = 1;
   s.outer_iters_max = outer_max;
   s.outer_iters_sum = outer_sum;
   s.inner_iters_sum = inner_sum;
   s.smo_cycles_sum = cyc_sum;
   s.n_sv = (int64_t)mdl->sv_pos.size();
-  s.cache_regime = 0;
+  s.cache_regime = full_k ? 0 : 1;
   s.n_pairs_trained = Pl;
   s.launches = (int64_t)(g_launches.load() - launches0);
   s.t_total_ms = host_ms_since(t_start);

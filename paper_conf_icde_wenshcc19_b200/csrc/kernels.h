@@ -68,6 +68,19 @@ struct SolverArgs {
   int pair_base;        // first local pair of this launch (grid.x pairs from here)
   double C, eps;
   double local_ratio;  // local solve stops at gap < max(eps, local_ratio * delta0) (reading R20: 0.1)
+  // ---- ROW_CACHE regime (kernel matrix does not fit): R != NULL, K == NULL
+  float* R;             // per pair B x ldr rows K(x_ws, x_pair) in pair-local column order (the paper's buffer)
+  int32_t* ws_slot;     // [P][B] R row slot of each working-set position
+  int32_t* ws_slot_tmp; // [P][B]
+  int32_t* ws_keep;     // [P] retained positions of the last selection (rows to compute start there)
+  const float* XT;      // class-sorted feature-major X, d_pad x ldx (zero padded)
+  int64_t ldx;
+  const float* norms;   // [ldx] squared norms (class-sorted)
+  float* ATnew;         // [P][d_pad][B] gathered new working-set rows (feature-major)
+  int d_pad;
+  int64_t* rows_done;  // [P] kernel rows computed (ROW_CACHE statistics)
+  int ldat;            // leading dimension of ATnew (round_up(B, 128))
+  double gamma;
 };
 
 void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st);
@@ -76,6 +89,8 @@ void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st);
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st);
 bool local_smo_uses_smem(int B);  // K_ws,ws gathered in-kernel (no gather_kws launch, no Kws buffer)
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
+// ROW_CACHE: kernel rows of the new working-set entries of every pair of the launch
+void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
 // fused outer loop: one cluster per pair, whole solve in one launch (B <= 224)
 bool fused_solver_enabled(int B);
 void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStream_t st);

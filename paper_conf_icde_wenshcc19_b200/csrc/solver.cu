@@ -17,6 +17,7 @@
 #include <cstdlib>
 #include <string>
 
+#include "gemm_simt.cuh"
 #include "kernels.h"
 
 namespace gmpsvm {
@@ -595,9 +596,13 @@ __device__ void select_body(const SolverArgs& a, int lp, uint32_t stampv, int fi
   int32_t* ws = a.ws + (int64_t)lp * B;
   if (np <= B) {  // the whole pair is the working set
     if (first) {
-      for (int i = threadIdx.x; i < np; i += blockDim.x) ws[i] = i;
+      for (int i = threadIdx.x; i < np; i += blockDim.x) {
+        ws[i] = i;
+        if (a.R) a.ws_slot[(int64_t)lp * B + i] = i;
+      }
       if (threadIdx.x == 0) a.ws_n[lp] = np;
     }
+    if (a.R && threadIdx.x == 0) a.ws_keep[lp] = first ? 0 : np;  // rows computed once
     return;
   }
   int32_t* nxt = a.ws_tmp + (int64_t)lp * B;
@@ -634,6 +639,34 @@ __device__ void select_body(const SolverArgs& a, int lp, uint32_t stampv, int fi
     cnt += select_sides(src, np, B - keep, nxt + cnt, sm, ku0, ku1, kl0, kl1);
   }
   mark(3);
+  if (a.R) {
+    // ROW_CACHE: retained positions keep their row slots; new positions take the free slots in
+    // increasing order (deterministic)
+    int32_t* slot = a.ws_slot + (int64_t)lp * B;
+    int32_t* snx = a.ws_slot_tmp + (int64_t)lp * B;
+    uint8_t* used = reinterpret_cast<uint8_t*>(sm.hist);  // B <= 1024 flags
+    __syncthreads();
+    for (int i = threadIdx.x; i < B; i += blockDim.x) used[i] = 0;
+    __syncthreads();
+    for (int e = threadIdx.x; e < keep; e += blockDim.x) {
+      const int sl = slot[prev_n - keep + e];
+      snx[e] = sl;
+      used[sl] = 1;
+    }
+    __syncthreads();
+    int base = 0;
+    for (int i0 = 0; i0 < B; i0 += blockDim.x) {
+      const int i = i0 + threadIdx.x;
+      const bool fr = i < B && !used[i];
+      int tot = 0;
+      const int pos = block_excl_scan(fr, tot, sm.scan);
+      if (fr && keep + base + pos < cnt) snx[keep + base + pos] = i;
+      base += tot;
+    }
+    __syncthreads();
+    for (int e = threadIdx.x; e < cnt; e += blockDim.x) slot[e] = snx[e];
+    if (threadIdx.x == 0) a.ws_keep[lp] = keep;
+  }
   for (int e = threadIdx.x; e < cnt; e += blockDim.x) ws[e] = nxt[e];
   if (threadIdx.x == 0) a.ws_n[lp] = cnt;
   mark(4);
@@ -656,11 +689,13 @@ __device__ void gather_rows_body(const SolverArgs& a, int lp, int r0, int r1, in
   const PairDesc pd = a.pairs[lp];
   const int wn = a.ws_n[lp];
   const int32_t* ws = a.ws + (int64_t)lp * a.B;
-  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
+  // FULL_K: global class-sorted columns of the resident matrix; ROW_CACHE: pair-local columns
+  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = a.R ? (int64_t)ws[e] : gpos(pd, ws[e]);
   __syncthreads();
   r1 = min(wn, r1);
+  const int64_t ldr = (pd.n_s + pd.n_t + 3) & ~3;
   for (int r = r0; r < r1; ++r) {
-    const float* row = a.K + g[r] * a.ldk;
+    const float* row = a.R ? a.R + pd.r_off + (int64_t)a.ws_slot[(int64_t)lp * a.B + r] * ldr : a.K + g[r] * a.ldk;
     float* dst = a.Kws + ((int64_t)lp * a.B + r) * a.B;
     for (int e = threadIdx.x; e < wn; e += blockDim.x) dst[e] = __ldg(row + g[e]);
   }
@@ -1013,9 +1048,12 @@ struct FupSmem {
 // thread per sweep).  Returns early (uniformly) when no alpha changed.
 __device__ void fupdate_body(const SolverArgs& a, int lp, int64_t q0, int64_t q1, FupSmem& fs) {
   const PairDesc pd = a.pairs[lp];
-  const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;  // quads of class s
-  const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;  // quads of class t
+  const bool rc = a.R != nullptr;  // ROW_CACHE: rows are pair-local, columns 0..n_p contiguous
+  const int64_t q1b = rc ? 0 : pd.off_s >> 2;
+  const int64_t q1e = rc ? (pd.n_s + pd.n_t + 3) >> 2 : (pd.off_s + pd.n_s + 3) >> 2;  // quads of class s
+  const int64_t q2b = rc ? 0 : pd.off_t >> 2, q2e = rc ? 0 : (pd.off_t + pd.n_t + 3) >> 2;  // quads of class t
   const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
+  const int64_t ldr = (pd.n_s + pd.n_t + 3) & ~3;
   q1 = q1 < nq ? q1 : nq;
   if (q0 >= q1) return;
   const int B = a.B, wn = a.ws_n[lp];
@@ -1030,7 +1068,8 @@ __device__ void fupdate_body(const SolverArgs& a, int lp, int64_t q0, int64_t q1
     const int pos = block_excl_scan(nz, tot, fs.scan);
     if (nz) {
       fs.coef[nnz + pos] = c;
-      fs.rowp[nnz + pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, ws[e]) * a.ldk);
+      fs.rowp[nnz + pos] = reinterpret_cast<const float4*>(
+          rc ? a.R + pd.r_off + (int64_t)a.ws_slot[(int64_t)lp * B + e] * ldr : a.K + gpos(pd, ws[e]) * a.ldk);
     }
     nnz += tot;
   }
@@ -1089,8 +1128,10 @@ __device__ void fupdate_body(const SolverArgs& a, int lp, int64_t q0, int64_t q1
       if (!okq[u]) continue;
 #pragma unroll
       for (int c = 0; c < 4; ++c) {
-        const int64_t g = gq[u] * 4 + c;  // global (class-sorted) column
-        if (seg1[u]) {
+        const int64_t g = gq[u] * 4 + c;  // global (class-sorted) column, or pair-local (ROW_CACHE)
+        if (rc) {
+          if (g < pd.n_s + pd.n_t) f[g] += acc[u][c];
+        } else if (seg1[u]) {
           if (g >= pd.off_s && g < pd.off_s + pd.n_s) f[g - pd.off_s] += acc[u][c];
         } else if (g >= pd.off_t && g < pd.off_t + pd.n_t) {
           f[pd.n_s + (g - pd.off_t)] += acc[u][c];
@@ -1198,6 +1239,75 @@ void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStrea
 bool fused_solver_enabled(int B) {
   static const bool on = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "fused";
   return on && B <= kSmemMaxB;
+}
+
+
+// ------------------------------------------------------------------------------------------
+// ROW_CACHE regime (a2 + a3 when the n x n kernel matrix does not fit): per outer iteration the
+// kernel rows of each pair's NEW working-set entries (positions ws_keep..ws_n) are computed
+// against the pair's instances into the pair's B-row buffer R (the paper's GPU buffer,
+// L299-L303; retained rows are reused, L297), in pair-local column order.
+__global__ void rows_gather_kernel(SolverArgs a) {
+  const int lp = blockIdx.x + a.pair_base;
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int keep = a.ws_keep[lp], wn = a.ws_n[lp], nnew = wn - keep;
+  if (nnew <= 0) return;
+  const int B = a.B;
+  if (blockIdx.y == 0 && threadIdx.x == 0) a.rows_done[lp] += nnew;
+  float* at = a.ATnew + (int64_t)lp * a.d_pad * a.ldat;
+  const int32_t* ws = a.ws + (int64_t)lp * B;
+  for (int c = blockIdx.y; c < a.d_pad; c += gridDim.y)
+    for (int i = threadIdx.x; i < a.ldat; i += blockDim.x)
+      at[(int64_t)c * a.ldat + i] = i < nnew ? a.XT[(int64_t)c * a.ldx + gpos(pd, ws[keep + i])] : 0.f;
+}
+
+__global__ void __launch_bounds__(kGemmThreads, 2) rows_contract_kernel(SolverArgs a, float scale) {
+  __shared__ __align__(16) GemmSmem sm;
+  const int lp = blockIdx.x + a.pair_base;
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int keep = a.ws_keep[lp], wn = a.ws_n[lp], nnew = wn - keep;
+  const int rt = blockIdx.z;  // 128-row tile of the new rows
+  if (rt * kTile >= nnew) return;
+  // column tile -> (segment, first global column); segments start at 4-aligned global columns
+  const int64_t sb = pd.off_s & ~3ll, tb = pd.off_t & ~3ll;
+  const int ts = (int)((pd.off_s + pd.n_s - sb + kTile - 1) / kTile);
+  const int tt = (int)((pd.off_t + pd.n_t - tb + kTile - 1) / kTile);
+  const int ct = blockIdx.y;
+  if (ct >= ts + tt) return;
+  const bool seg_s = ct < ts;
+  const int64_t c0 = seg_s ? sb + (int64_t)ct * kTile : tb + (int64_t)(ct - ts) * kTile;
+  const int64_t lo = seg_s ? pd.off_s : pd.off_t, hi = seg_s ? pd.off_s + pd.n_s : pd.off_t + pd.n_t;
+  const int64_t loc0 = seg_s ? -pd.off_s : pd.n_s - pd.off_t;  // pair-local column = g + loc0
+  float acc[8][8];
+  gemm_tile_128(a.ATnew + (int64_t)lp * a.d_pad * a.ldat, a.ldat, (int64_t)rt * kTile, a.XT, a.ldx, c0, a.d_pad, sm, acc);
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int32_t* ws = a.ws + (int64_t)lp * a.B;
+  const int32_t* slot = a.ws_slot + (int64_t)lp * a.B;
+  const int64_t ldr = (pd.n_s + pd.n_t + 3) & ~3;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = rt * kTile + tile_row(ty, i);  // index among the new rows
+    if (r >= nnew) continue;
+    const int64_t gr = gpos(pd, ws[keep + r]);
+    const float nr = a.norms[gr];
+    float* dst = a.R + pd.r_off + (int64_t)slot[keep + r] * ldr;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int64_t g = c0 + tile_col(tx, j);
+      if (g < lo || g >= hi) continue;
+      const float d2 = fmaf(-2.f, acc[i][j], nr + a.norms[g]);
+      dst[g + loc0] = (g == gr) ? 1.f : fast_exp2(fmaxf(d2, 0.f) * scale);
+    }
+  }
+}
+
+void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
+  GM_LAUNCH(rows_gather_kernel, dim3(P, 32), dim3(256), 0, st, a);
+  const int ctiles = (int)ceil_div(np_max + 8, kTile) + 2;
+  const float scale = (float)(-a.gamma * 1.4426950408889634);
+  GM_LAUNCH(rows_contract_kernel, dim3(P, ctiles, (unsigned)ceil_div(a.B, kTile)), dim3(kGemmThreads), 0, st, a, scale);
 }
 
 // ------------------------------------------------------------------------------------------
