@@ -3,6 +3,7 @@
 // model introspection and the serialize / deserialize / merge plumbing used by the
 // multi-GPU driver (pairs sharded across ranks, blobs gathered with NCCL).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -13,6 +14,13 @@ using gmpsvm::Error;
 using gmpsvm::Model;
 
 namespace {
+
+// The solver runs every pair's outer loop as its own branch of one CUDA graph; the runtime
+// executes at most CUDA_DEVICE_MAX_CONNECTIONS (default 8, max 32) branches concurrently.
+// Raise the default to 32 when the library is loaded, before the process creates its CUDA
+// context (an explicit user setting is kept; engine.cu packs the pairs into that many branches).
+__attribute__((constructor)) void gmpsvm_default_connections() { setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0); }
+
 
 thread_local std::string g_err;
 

@@ -185,6 +185,15 @@ struct KWorkspace {
   float* get() const { return p; }
 };
 
+struct GraphGuard {
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  ~GraphGuard() {
+    if (exec) cudaGraphExecDestroy(exec);
+    if (graph) cudaGraphDestroy(graph);
+  }
+};
+
 template <class T>
 struct PinnedBuf {
   T* p = nullptr;
@@ -618,6 +627,20 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<int64_t> d_sphase(smo_prof ? (size_t)(Pl + 4096) * 5 : 0, st);
   if (smo_prof) GM_CUDA(cudaMemsetAsync(d_sphase.get(), 0, (size_t)(Pl + 4096) * 5 * 8, st));
   a.sel_phase = smo_prof ? d_sphase.get() : nullptr;
+  // GMPSVM_TRACE=<pair position>: kernel timeline of that pair (entries sorted largest pair first)
+  static const int trace_pos = getenv("GMPSVM_TRACE") ? atoi(getenv("GMPSVM_TRACE")) : -1;
+  const int trace_cap = 1 << 16;
+  DevBuf<int64_t> d_trace(trace_pos >= 0 ? (size_t)trace_cap * 3 + 2 * (size_t)Pl : 0, st);
+  if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace.get(), 0, ((size_t)trace_cap * 3 + 2 * (size_t)Pl) * 8, st));
+  DevBuf<int32_t> d_trace_n(trace_pos >= 0 ? 1 : 0, st);
+  if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace_n.get(), 0, 4, st));
+  DevBuf<int64_t> d_body(Pl, st);
+  GM_CUDA(cudaMemsetAsync(d_body.get(), 0, Pl * 8, st));
+  a.body_iters = d_body.get();
+  a.trace = d_trace.get();
+  a.trace_n = d_trace_n.get();
+  a.trace_pair = trace_pos;
+  a.trace_cap = trace_cap;
   a.outer_iters = d_outer.get();
   a.b = d_b.get();
   a.A = d_A.get();
@@ -690,15 +713,75 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     inflight[g].push_back(Chunk{ev, slot});
   };
   const bool fused = full_k && fused_solver_enabled(Bw);
+  static const bool streams_mode = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "streams";
+  const bool graph_mode = !fused && !streams_mode;
+  GraphGuard gg;
+  int64_t body_launches = 0;
+  int n_branches = 0;
   if (fused) {  // the whole outer loop of every pair in one launch (clusters, no host round trips)
     SolverArgs ag = a;
     ag.pair_base = 0;
     launch_pair_solver(ag, Pl, max_outer, pool[0]);
+  } else if (graph_mode) {
+    // Device-driven outer loops (default): one CUDA graph holding, per pair, a conditional
+    // WHILE node whose body is that pair's select -> [rows] -> gather -> local SMO -> f-update
+    // chain (the f-update kernel sets the loop condition), followed by one last selection (the
+    // stop test on the final alpha).  The pairs are independent branches of the graph, so no
+    // pair waits for another at a kernel boundary and the host is not involved until the end.
+    // The runtime runs at most CUDA_DEVICE_MAX_CONNECTIONS branches of a graph concurrently (a
+    // branch beyond that waits for another to finish), so the pairs are packed into that many
+    // branches: the largest pairs alone, the smallest two (or more) to a branch in lockstep.
+    const char* conn_env = getenv("CUDA_DEVICE_MAX_CONNECTIONS");
+    const int conn = std::max(1, std::min(32, conn_env ? atoi(conn_env) : 8));
+    const int nbr = std::min(Pl, conn);
+    std::vector<int> bb(nbr + 1, 0);
+    {
+      const int m = Pl / nbr, r = Pl % nbr;  // the last r branches take m + 1 pairs
+      for (int b = 0; b < nbr; ++b) bb[b + 1] = bb[b] + m + (b >= nbr - r ? 1 : 0);
+    }
+    const uint64_t l0 = g_launches.load();
+    GM_CUDA(cudaGraphCreate(&gg.graph, 0));
+    cudaStream_t cs = pool.back();
+    for (int br = 0; br < nbr; ++br) {
+      const int i = bb[br], gn = bb[br + 1] - bb[br];
+      int64_t npi = 0;
+      for (int j = bb[br]; j < bb[br + 1]; ++j) npi = std::max<int64_t>(npi, hp[j].n_s + hp[j].n_t);
+      cudaGraphConditionalHandle h;
+      GM_CUDA(cudaGraphConditionalHandleCreate(&h, gg.graph, 1, cudaGraphCondAssignDefault));
+      cudaGraphNodeParams cp = {};
+      cp.type = cudaGraphNodeTypeConditional;
+      cp.conditional.handle = h;
+      cp.conditional.type = cudaGraphCondTypeWhile;
+      cp.conditional.size = 1;
+      cudaGraphNode_t wnode;
+      GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, nullptr, 0, &cp));
+      SolverArgs ag = a;
+      ag.pair_base = i;
+      const uint64_t b0 = g_launches.load();
+      cudaGraph_t cap;
+      GM_CUDA(cudaStreamBeginCaptureToGraph(cs, cp.conditional.phGraph_out[0], nullptr, nullptr, 0,
+                                            cudaStreamCaptureModeRelaxed));
+      launch_select_ws(ag, gn, 0, -1, cs);
+      if (rc) launch_rows_compute(ag, gn, npi, cs);
+      launch_gather_kws(ag, gn, -1, cs);
+      launch_local_smo(ag, gn, cs);
+      launch_f_update_loop(ag, gn, npi, h, max_outer, cs);
+      GM_CUDA(cudaStreamEndCapture(cs, &cap));
+      body_launches = (int64_t)(g_launches.load() - b0);
+      GM_CUDA(cudaStreamBeginCaptureToGraph(cs, gg.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
+      launch_select_ws(ag, gn, 0, -1, cs);
+      GM_CUDA(cudaStreamEndCapture(cs, &cap));
+    }
+    n_branches = nbr;
+    g_launches.fetch_sub(g_launches.load() - l0);  // captured, not executed: counted after the run
+    GM_CUDA(cudaGraphInstantiate(&gg.exec, gg.graph, 0));
+    HT("graph_build");
+    GM_CUDA(cudaGraphLaunch(gg.exec, pool[0]));
   } else {
     for (int g = 0; g < G; ++g) issue_chunk(g);
     for (int g = 0; g < G; ++g) issue_chunk(g);
   }
-  int running = fused ? 0 : G;
+  int running = (fused || graph_mode) ? 0 : G;
   while (running > 0) {
     bool progressed = false;
     for (int g = 0; g < G; ++g) {
@@ -756,8 +839,57 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaMemcpyAsync(h_cyc.data(), d_cyc.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_perm.data(), d_perm.get(), n * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_flags.data(), d_flags.get(), n, cudaMemcpyDeviceToHost, st));
+  std::vector<int64_t> h_body(Pl);
+  GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
+  if (graph_mode) {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
+    int64_t ex = n_branches;  // one final selection per branch
+    for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_launches;  // counted at each branch's first pair
+    g_launches.fetch_add((uint64_t)ex);
+    if (rc) {
+      rc_launches = 0;
+      for (int i = 0; i < Pl; ++i) rc_launches += h_body[i];
+    }
+  }
 
+  if (trace_pos >= 0 && trace_pos < Pl) {
+    int32_t nt = 0;
+    GM_CUDA(cudaMemcpy(&nt, d_trace_n.get(), 4, cudaMemcpyDeviceToHost));
+    nt = std::min(nt, trace_cap);
+    std::vector<int64_t> tr((size_t)nt * 3);
+    GM_CUDA(cudaMemcpy(tr.data(), d_trace.get(), tr.size() * 8, cudaMemcpyDeviceToHost));
+    std::vector<int> order(nt);
+    for (int i = 0; i < nt; ++i) order[i] = i;
+    std::sort(order.begin(), order.end(), [&](int x, int y) { return tr[3 * x + 1] < tr[3 * y + 1]; });
+    const char* names[6] = {"select", "gather", "smo", "fupdate", "rows_gather", "rows_contract"};
+    double dur[6] = {0}, cnt[6] = {0}, gap_before[6] = {0};
+    for (int j = 0; j < nt; ++j) {
+      const int i = order[j];
+      const int kd = (int)tr[3 * i];
+      dur[kd] += (double)(tr[3 * i + 2] - tr[3 * i + 1]);
+      cnt[kd] += 1;
+      if (j > 0) gap_before[kd] += (double)(tr[3 * i + 1] - tr[3 * order[j - 1] + 2]);
+    }
+    const double span = nt ? (double)(tr[3 * order[nt - 1] + 2] - tr[3 * order[0] + 1]) : 0.0;
+    std::string line;
+    for (int kd = 0; kd < 6; ++kd)
+      if (cnt[kd] > 0)
+        line += std::string(" ") + names[kd] + " n=" + std::to_string((int)cnt[kd]) +
+                " mean_us=" + std::to_string(dur[kd] / cnt[kd] / 1e3).substr(0, 6) +
+                " gap_before_us=" + std::to_string(gap_before[kd] / cnt[kd] / 1e3).substr(0, 6) + ";";
+    std::vector<int64_t> win((size_t)2 * Pl);
+    GM_CUDA(cudaMemcpy(win.data(), d_trace.get() + (size_t)trace_cap * 3, win.size() * 8, cudaMemcpyDeviceToHost));
+    int64_t t_min = INT64_MAX;
+    for (int i = 0; i < Pl; ++i)
+      if (win[2 * i]) t_min = std::min(t_min, win[2 * i]);
+    std::string wl;
+    for (int i = 0; i < Pl; ++i)
+      wl += " " + std::to_string(i) + ":" + std::to_string((win[2 * i] - t_min) / 100000 / 10.0).substr(0, 4) + "-" +
+            std::to_string((win[2 * i + 1] - t_min) / 100000 / 10.0).substr(0, 4);
+    fprintf(stderr, "[gmpsvm trace] pair windows (ms from first start):%s\n", wl.c_str());
+    fprintf(stderr, "[gmpsvm trace] pair (%d,%d) outer %d span %.2f ms:%s\n", hp[trace_pos].s, hp[trace_pos].t,
+            h_outer[trace_pos], span / 1e6, line.c_str());
+  }
   if (smo_prof) {
     std::vector<int64_t> ph((size_t)Pl * 5);
     GM_CUDA(cudaMemcpy(ph.data(), d_phase.get(), ph.size() * 8, cudaMemcpyDeviceToHost));
@@ -845,7 +977,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   s.t_fupdate_ms = tm.ms(PH_FUP);
   s.t_finalize_ms = tm.ms(PH_FIN);
   s.t_solver_ms = tm.ms(PH_SOLVER);
-  s.n_streams = G;
+  s.n_streams = graph_mode ? n_branches : G;
   if (full_k) {
     s.kernel_values = (double)n * (double)(n + 1) / 2.0;
     s.krow_launches = 1;

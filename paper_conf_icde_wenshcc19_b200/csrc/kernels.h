@@ -58,6 +58,10 @@ struct SolverArgs {
   int64_t* inner_iters; // [P]
   int64_t* smo_cycles;  // [P] SM clock cycles spent in local_smo (diagnostic)
   int64_t* smo_phase;   // [P][5] optional per-phase cycles (GMPSVM_SMO_PHASES=1), else NULL
+  int64_t* body_iters;  // [P] executions of the graph loop body (device-driven solver)
+  int64_t* trace;       // optional kernel timeline of one pair (GMPSVM_TRACE=<pair position>): [cap][3]
+  int32_t* trace_n;
+  int32_t trace_pair, trace_cap;
   int64_t* sel_phase;   // [P][5] optional select_ws phase cycles (GMPSVM_SMO_PHASES=1), else NULL
   int32_t* outer_iters; // [P]
   double* b;            // [P]
@@ -90,6 +94,8 @@ void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st);
 bool local_smo_uses_smem(int B);  // K_ws,ws gathered in-kernel (no gather_kws launch, no Kws buffer)
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
 // ROW_CACHE: kernel rows of the new working-set entries of every pair of the launch
+void launch_f_update_loop(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int64_t max_outer,
+                          cudaStream_t st);
 void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
 // fused outer loop: one cluster per pair, whole solve in one launch (B <= 224)
 bool fused_solver_enabled(int B);

@@ -101,6 +101,46 @@ __device__ int block_excl_scan_count(int count, int& total, int* sm /* 33 */) {
 }
 
 // ------------------------------------------------------------------------------------------
+
+// Optional timeline of one pair's solver kernels (GMPSVM_TRACE): thread (0,0,0) of the CTA that
+// serves the traced pair records (kernel id, %globaltimer at entry, at exit).
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+struct TraceScope {
+  int64_t* buf;
+  int32_t* n;
+  int cap, kid;
+  uint64_t t0;
+  __device__ TraceScope(const SolverArgs& a, int lp, int k) : buf(nullptr), kid(k) {
+    if (a.trace && threadIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && a.status[lp] == 0) {
+      // per-pair activity window: first entry, last entry (kernels of active pairs only)
+      int64_t* w = a.trace + 3 * (int64_t)a.trace_cap + 2 * lp;
+      const int64_t now = (int64_t)gtimer();
+      if (w[0] == 0) w[0] = now;
+      w[1] = now;
+    }
+    if (a.trace && lp == a.trace_pair && threadIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0) {
+      buf = a.trace;
+      n = a.trace_n;
+      cap = a.trace_cap;
+      t0 = gtimer();
+    }
+  }
+  __device__ ~TraceScope() {
+    if (buf) {
+      const int s = atomicAdd(n, 1);
+      if (s < cap) {
+        buf[3 * s] = kid;
+        buf[3 * s + 1] = (int64_t)t0;
+        buf[3 * s + 2] = (int64_t)gtimer();
+      }
+    }
+  }
+};
+
 __global__ void init_pairs_kernel(SolverArgs a, const int64_t tot, int P) {
   // alpha = 0, f = -y (Alg 1 lines 1-2 / Alg 2 line 4), stamps 0
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -675,8 +715,14 @@ __device__ void select_body(const SolverArgs& a, int lp, uint32_t stampv, int fi
 constexpr size_t kSelDynBytes = (size_t)kSelSmemMax * 9 + 16 + sizeof(SelLists);
 
 __global__ void __launch_bounds__(1024) select_ws_kernel(SolverArgs a, uint32_t stampv, int first) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 0);
   __shared__ SelSmem sm;
   extern __shared__ __align__(16) unsigned char sel_dyn[];
+  if (stampv == 0) {  // device-driven loop (graph): iteration from the pair's own counter
+    const int32_t oi = a.outer_iters[blockIdx.x + a.pair_base];  // read before select_body increments it
+    first = oi == 0;
+    stampv = (uint32_t)oi + 1u;
+  }
   select_body(a, blockIdx.x + a.pair_base, stampv, first, sm, sel_dyn);
 }
 
@@ -702,10 +748,12 @@ __device__ void gather_rows_body(const SolverArgs& a, int lp, int r0, int r1, in
 }
 
 __global__ void __launch_bounds__(256) gather_kws_kernel(SolverArgs a, int first) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 1);
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
+  if (first < 0) first = a.outer_iters[lp] == 1;  // device-driven loop: after the first selection
   if (np <= a.B && !first) return;  // working set unchanged
   const int r0 = blockIdx.y * kGatherRows;
   if (r0 >= a.ws_n[lp]) return;
@@ -1024,9 +1072,225 @@ __device__ void smo_body(const SolverArgs& a, int lp, int nt, int bar_id, RedSlo
 
 template <int E, bool SMEM>
 __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(SolverArgs a) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 2);
   __shared__ RedSlot slots[2][32];
   extern __shared__ float kw_smem[];
   smo_body<E, SMEM>(a, blockIdx.x + a.pair_base, blockDim.x, 0, slots, kw_smem);
+}
+
+// Single-warp local SMO (B <= kSmemMaxB): the whole working set lives in the registers of one
+// warp (lane owns rows lane, lane + 32, ...), so the two argmin/argmax reductions of every inner
+// step are warp-level (redux.sync + ballot) with no CTA barrier and no shared-memory slots; the
+// winner's f comes from its key, its K_ee from the shared K_ws,ws tile, so only alpha and the
+// row index are shuffled.  All CTA threads copy K_ws,ws into shared memory first; warps 1.. then
+// exit.  Same arithmetic and tie rules as smo_body, so the iterates are identical.
+template <int E>
+__device__ __forceinline__ void smo_warp(const SolverArgs& a, int lp, const float* Kw, long long t_entry) {
+  const int lane = threadIdx.x;
+  const PairDesc pd = a.pairs[lp];
+  const int B = a.B, wn = a.ws_n[lp];
+  const double C = a.C;
+  bool valid[E], iu[E], il[E];
+  int32_t idx[E];
+  int y[E];
+  double al[E], a0[E], fv[E];
+  float kd[E], va[E], vb[E], ku[E];
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = lane + 32 * q;
+    valid[q] = e < wn;
+    idx[q] = valid[q] ? a.ws[(int64_t)lp * B + e] : INT_MAX;
+    y[q] = (valid[q] && idx[q] < pd.n_s) ? 1 : -1;
+    al[q] = valid[q] ? a.alpha[pd.a_off + idx[q]] : 0.0;
+    a0[q] = al[q];
+    fv[q] = valid[q] ? a.f[pd.a_off + idx[q]] : 0.0;
+    kd[q] = valid[q] ? Kw[(int64_t)e * B + e] : 1.f;
+    iu[q] = valid[q] && in_u(y[q], al[q], C);
+    il[q] = valid[q] && in_l(y[q], al[q], C);
+    va[q] = vb[q] = 0.f;
+  }
+  int ra = -1, rb = -1;
+  const int cap = a.inner_cap;
+  int it = 0;
+  double delta0 = 0.0;
+  const long long t_begin = clock64();
+  long long ph[4] = {0, 0, 0, 0}, tp = t_begin;
+  const bool prof = a.smo_phase != nullptr;
+  for (;;) {
+    // Step 1 (Eq 4): u = argmin_{I_u} f, ties -> lowest pair-local index
+    uint32_t h0 = 0xffffffffu, l0 = 0xffffffffu;
+    int32_t bi = INT_MAX;
+    int be = 0;
+    double ba = 0.0;
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      if (iu[q]) {
+        const uint64_t key = ord_key(fv[q]);
+        const uint32_t h = (uint32_t)(key >> 32), l = (uint32_t)key;
+        if (h < h0 || (h == h0 && (l < l0 || (l == l0 && idx[q] < bi)))) {
+          h0 = h;
+          l0 = l;
+          bi = idx[q];
+          be = lane + 32 * q;
+          ba = al[q];
+        }
+      }
+    }
+    const int wu = warp_argmin(h0, l0, bi);
+    if (bi == INT_MAX) break;
+    const int ue = __shfl_sync(FULLMASK, be, wu);
+    const double au = __shfl_sync(FULLMASK, ba, wu);
+    const double fu = key_double(((uint64_t)h0 << 32) | l0);
+    const float kuu = Kw[(int64_t)ue * B + ue];
+    const int yu = bi < pd.n_s ? 1 : -1;
+    if (prof) {
+      const long long t = clock64();
+      ph[0] += t - tp;
+      tp = t;
+    }
+    if (ue == ra) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) ku[q] = va[q];
+    } else if (ue == rb) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) ku[q] = vb[q];
+    } else {
+      const float* row = Kw + (int64_t)ue * B;
+#pragma unroll
+      for (int q = 0; q < E; ++q) ku[q] = valid[q] ? row[lane + 32 * q] : 0.f;
+    }
+    // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_u - f_t)^2 / eta_t, and f_max over I_l (Eq 10)
+    uint32_t m0 = 0u, m1 = 0u;
+    uint32_t g0 = 0xffffffffu, g1 = 0u;
+    int32_t li = INT_MAX;
+    int le_c = 0;
+    double la = 0.0, lf = 0.0;
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      if (il[q]) {
+        const uint64_t fk = ord_key(fv[q]);
+        const uint32_t h = (uint32_t)(fk >> 32), l = (uint32_t)fk;
+        if (h > m0 || (h == m0 && l > m1)) {
+          m0 = h;
+          m1 = l;
+        }
+        if (fv[q] > fu) {
+          const float eta = fmaxf(kuu + kd[q] - 2.f * ku[q], 1e-12f);
+          const float df = (float)(fv[q] - fu);
+          const uint32_t sk = ~__float_as_uint(df * df * __frcp_rn(eta));
+          if (sk < g0 || (sk == g0 && idx[q] < li)) {
+            g0 = sk;
+            li = idx[q];
+            le_c = lane + 32 * q;
+            la = al[q];
+            lf = fv[q];
+          }
+        }
+      }
+    }
+    const int wl = warp_argmin(g0, g1, li);
+    warp_max64(m0, m1);
+    if (prof) {
+      const long long t = clock64();
+      ph[1] += t - tp;
+      tp = t;
+    }
+    const double fmax = (m0 == 0u && m1 == 0u) ? -DBL_MAX : key_double(((uint64_t)m0 << 32) | m1);
+    const double gap = fmax - fu;
+    if (it == 0) delta0 = gap;
+    const double tol = a.eps > a.local_ratio * delta0 ? a.eps : a.local_ratio * delta0;
+    if (!(gap >= tol) || li == INT_MAX || it >= cap) break;
+    const int le = __shfl_sync(FULLMASK, le_c, wl);
+    const double alv = __shfl_sync(FULLMASK, la, wl);
+    const double fl = __shfl_sync(FULLMASK, lf, wl);
+    const float kll = Kw[(int64_t)le * B + le], kul = Kw[(int64_t)ue * B + le];
+    const int yl = li < pd.n_s ? 1 : -1;
+    // Step 2 (Eq 6-7) with explicit clipping (reading R4): common step s (FP64)
+    double eta = (double)kuu + (double)kll - 2.0 * (double)kul;
+    eta = eta > kTau ? eta : kTau;
+    double s = (fl - fu) / eta;
+    const double Uu = yu > 0 ? C - au : au;
+    const double Ll = yl > 0 ? alv : C - alv;
+    bool bu = false, bl = false;
+    if (Uu <= s) {
+      s = Uu;
+      bu = true;
+    }
+    if (Ll <= s) {
+      if (Ll < s) bu = false;
+      s = Ll;
+      bl = true;
+    }
+    double nau = au + yu * s, nal = alv - yl * s;
+    if (bu) nau = yu > 0 ? C : 0.0;
+    if (bl) nal = yl > 0 ? 0.0 : C;
+    // Step 3 (Eq 8) on the working set: f_i += s (K_ui - K_li)
+    float kl[E];
+    if (le == ra) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) kl[q] = va[q];
+    } else if (le == rb) {
+#pragma unroll
+      for (int q = 0; q < E; ++q) kl[q] = vb[q];
+    } else {
+      const float* row = Kw + (int64_t)le * B;
+#pragma unroll
+      for (int q = 0; q < E; ++q) kl[q] = valid[q] ? row[lane + 32 * q] : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      const int e = lane + 32 * q;
+      fv[q] += s * ((double)ku[q] - (double)kl[q]);
+      if (e == ue || e == le) {
+        al[q] = (e == ue) ? nau : nal;
+        iu[q] = in_u(y[q], al[q], C);
+        il[q] = in_l(y[q], al[q], C);
+      }
+      va[q] = ku[q];
+      vb[q] = kl[q];
+    }
+    ra = ue;
+    rb = le;
+    ++it;
+    if (prof) {
+      const long long t = clock64();
+      ph[3] += t - tp;
+      tp = t;
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = lane + 32 * q;
+    if (valid[q]) {
+      a.alpha[pd.a_off + idx[q]] = al[q];
+      a.dcoef[(int64_t)lp * B + e] = (al[q] - a0[q]) * (double)y[q];
+    }
+  }
+  if (lane == 0) {
+    a.inner_iters[lp] += it;
+    a.smo_cycles[lp] += clock64() - t_begin;
+    if (prof) {
+      for (int k = 0; k < 4; ++k) a.smo_phase[lp * 5 + k] += ph[k];
+      a.smo_phase[lp * 5 + 4] += t_begin - t_entry;
+    }
+  }
+}
+
+template <int E>
+__global__ void __launch_bounds__(256) local_smo_warp_kernel(SolverArgs a) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 2);
+  extern __shared__ float kw_smem[];
+  const long long t_entry = clock64();
+  const int lp = blockIdx.x + a.pair_base;
+  if (a.status[lp] != 0) return;
+  const int B = a.B;
+  const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * B * B);
+  float4* dst = reinterpret_cast<float4*>(kw_smem);
+  const int nv = (B * B) / 4;
+  for (int i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
+  __syncthreads();
+  if (threadIdx.x >= 32) return;
+  smo_warp<E>(a, lp, kw_smem, t_entry);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1141,12 +1405,128 @@ __device__ void fupdate_body(const SolverArgs& a, int lp, int64_t q0, int64_t q1
   }
 }
 
-__global__ void __launch_bounds__(kFThreads) f_update_kernel(SolverArgs a) {
+// Row-split f update (the launched kernels): a CTA of kFSWarps warps owns 32 column quads (128
+// columns); warp w streams rows w, w + kFSWarps, ... (8 float4 loads in flight per thread), so
+// a pair's update has ~n_p/128 CTAs x 256 threads of loads in flight instead of one thread
+// walking all rows of its quad; the kFSWarps partial sums are combined in a fixed order
+// (deterministic).  FP64 accumulation as in fupdate_body.
+constexpr int kFSWarps = 8;
+constexpr int kFSThreads = kFSWarps * 32;
+constexpr int kFSCols = 128;
+struct FupSplitSmem {
+  double coef[1024];
+  const float4* rowp[1024];
+  int scan[33];
+  double red[kFSWarps][32][4];
+};
+
+__device__ void fupdate_split(const SolverArgs& a, int lp, int64_t q0, FupSplitSmem& fs) {
+  const PairDesc pd = a.pairs[lp];
+  const bool rc = a.R != nullptr;
+  const int64_t q1b = rc ? 0 : pd.off_s >> 2;
+  const int64_t q1e = rc ? (pd.n_s + pd.n_t + 3) >> 2 : (pd.off_s + pd.n_s + 3) >> 2;
+  const int64_t q2b = rc ? 0 : pd.off_t >> 2, q2e = rc ? 0 : (pd.off_t + pd.n_t + 3) >> 2;
+  const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
+  const int64_t ldr = (pd.n_s + pd.n_t + 3) & ~3;
+  if (q0 >= nq) return;
+  const int B = a.B, wn = a.ws_n[lp];
+  const int32_t* ws = a.ws + (int64_t)lp * B;
+  const double* dc = a.dcoef + (int64_t)lp * B;
+  int nnz = 0;
+  for (int base = 0; base < wn; base += blockDim.x) {
+    const int e = base + threadIdx.x;
+    const double c = (e < wn) ? dc[e] : 0.0;
+    const bool nz = c != 0.0;
+    int tot = 0;
+    const int pos = block_excl_scan(nz, tot, fs.scan);
+    if (nz) {
+      fs.coef[nnz + pos] = c;
+      fs.rowp[nnz + pos] = reinterpret_cast<const float4*>(
+          rc ? a.R + pd.r_off + (int64_t)a.ws_slot[(int64_t)lp * B + e] * ldr : a.K + gpos(pd, ws[e]) * a.ldk);
+    }
+    nnz += tot;
+  }
+  __syncthreads();
+  if (nnz == 0) return;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t qi = q0 + lane;
+  const bool okq = qi < nq;
+  const int64_t gq = !okq ? 0 : (qi < nq1 ? q1b + qi : q2b + (qi - nq1));
+  double acc[4] = {0.0, 0.0, 0.0, 0.0};
+  int r = warp;
+  for (; r + 7 * kFSWarps < nnz; r += 8 * kFSWarps) {
+    float4 v[8];
+#pragma unroll
+    for (int rr = 0; rr < 8; ++rr)
+      v[rr] = okq ? __ldg(fs.rowp[r + rr * kFSWarps] + gq) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int rr = 0; rr < 8; ++rr) {
+      const double cv = fs.coef[r + rr * kFSWarps];
+      acc[0] = fma(cv, (double)v[rr].x, acc[0]);
+      acc[1] = fma(cv, (double)v[rr].y, acc[1]);
+      acc[2] = fma(cv, (double)v[rr].z, acc[2]);
+      acc[3] = fma(cv, (double)v[rr].w, acc[3]);
+    }
+  }
+  for (; r < nnz; r += kFSWarps) {
+    const float4 v0 = okq ? __ldg(fs.rowp[r] + gq) : make_float4(0.f, 0.f, 0.f, 0.f);
+    const double cv = fs.coef[r];
+    acc[0] = fma(cv, (double)v0.x, acc[0]);
+    acc[1] = fma(cv, (double)v0.y, acc[1]);
+    acc[2] = fma(cv, (double)v0.z, acc[2]);
+    acc[3] = fma(cv, (double)v0.w, acc[3]);
+  }
+#pragma unroll
+  for (int c = 0; c < 4; ++c) fs.red[warp][lane][c] = acc[c];
+  __syncthreads();
+  if (threadIdx.x < 128) {
+    const int l = threadIdx.x >> 2, c = threadIdx.x & 3;
+    const int64_t qj = q0 + l;
+    if (qj < nq) {
+      double sum = 0.0;
+#pragma unroll
+      for (int w = 0; w < kFSWarps; ++w) sum += fs.red[w][l][c];
+      const bool seg1 = qj < nq1;  // a boundary quad shared by adjacent classes is owned once per segment
+      const int64_t g = (seg1 ? q1b + qj : q2b + (qj - nq1)) * 4 + c;
+      double* f = a.f + pd.a_off;
+      if (rc) {
+        if (g < pd.n_s + pd.n_t) f[g] += sum;
+      } else if (seg1) {
+        if (g >= pd.off_s && g < pd.off_s + pd.n_s) f[g - pd.off_s] += sum;
+      } else if (g >= pd.off_t && g < pd.off_t + pd.n_t) {
+        f[pd.n_s + (g - pd.off_t)] += sum;
+      }
+    }
+  }
+}
+
+// f update + loop condition of the device-driven (graph) outer loop of one pair: continue while
+// the pair is active and below the outer-iteration cap.
+__global__ void __launch_bounds__(kFSThreads) f_update_loop_kernel(SolverArgs a, cudaGraphConditionalHandle h,
+                                                                   int64_t max_outer) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 3);
+  const int lp = blockIdx.x + a.pair_base;
+  if (blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {
+    // the branch's pairs run in lockstep: continue while any of them is active
+    bool more = false;
+    for (int i = 0; i < (int)gridDim.x; ++i) {
+      const int p = a.pair_base + i;
+      more = more || (a.status[p] == 0 && (int64_t)a.outer_iters[p] < max_outer);
+    }
+    cudaGraphSetConditional(h, more ? 1u : 0u);
+    a.body_iters[a.pair_base] += 1;
+  }
+  if (a.status[lp] != 0) return;
+  __shared__ FupSplitSmem fs;
+  fupdate_split(a, lp, (int64_t)blockIdx.y * 32, fs);
+}
+
+__global__ void __launch_bounds__(kFSThreads) f_update_kernel(SolverArgs a) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 3);
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
-  __shared__ FupSmem fs;
-  const int64_t q0 = (int64_t)blockIdx.y * (kFThreads * kFQ);
-  fupdate_body(a, lp, q0, q0 + kFThreads * kFQ, fs);
+  __shared__ FupSplitSmem fs;
+  fupdate_split(a, lp, (int64_t)blockIdx.y * 32, fs);
 }
 
 
@@ -1248,6 +1628,7 @@ bool fused_solver_enabled(int B) {
 // against the pair's instances into the pair's B-row buffer R (the paper's GPU buffer,
 // L299-L303; retained rows are reused, L297), in pair-local column order.
 __global__ void rows_gather_kernel(SolverArgs a) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 4);
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
@@ -1263,6 +1644,7 @@ __global__ void rows_gather_kernel(SolverArgs a) {
 }
 
 __global__ void __launch_bounds__(kGemmThreads, 2) rows_contract_kernel(SolverArgs a, float scale) {
+  TraceScope ts_(a, blockIdx.x + a.pair_base, 5);
   __shared__ __align__(16) GemmSmem sm;
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
@@ -1492,6 +1874,29 @@ void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st) {
 bool local_smo_uses_smem(int B) { return B <= kSmemMaxB; }
 
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
+  static const bool block_smo = getenv("GMPSVM_SMO") && std::string(getenv("GMPSVM_SMO")) == "block";
+  if (local_smo_uses_smem(a.B) && !block_smo) {
+    const size_t dyn = (size_t)a.B * a.B * sizeof(float);
+    const int E = (int)ceil_div(a.B, 32);
+    static bool configured_w[8] = {};
+    auto go = [&](auto kern) {
+      if (!configured_w[E]) {
+        GM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSmemMaxB * kSmemMaxB * 4)));
+        configured_w[E] = true;
+      }
+      GM_LAUNCH(kern, dim3(P), dim3(256), dyn, st, a);
+    };
+    switch (E) {
+      case 1: go(local_smo_warp_kernel<1>); break;
+      case 2: go(local_smo_warp_kernel<2>); break;
+      case 3: go(local_smo_warp_kernel<3>); break;
+      case 4: go(local_smo_warp_kernel<4>); break;
+      case 5: go(local_smo_warp_kernel<5>); break;
+      case 6: go(local_smo_warp_kernel<6>); break;
+      default: go(local_smo_warp_kernel<7>); break;
+    }
+    return;
+  }
   if (local_smo_uses_smem(a.B)) {
     const size_t dyn = (size_t)a.B * a.B * sizeof(float);
     static size_t configured = 0;
@@ -1514,7 +1919,12 @@ void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
 }
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
   // +8 columns: each class segment may add a partial quad at either end
-  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, kFCols)), dim3(kFThreads), 0, st, a);
+  GM_LAUNCH(f_update_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, kFSCols)), dim3(kFSThreads), 0, st, a);
+}
+void launch_f_update_loop(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int64_t max_outer,
+                          cudaStream_t st) {
+  GM_LAUNCH(f_update_loop_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, kFSCols)), dim3(kFSThreads), 0, st, a, h,
+            max_outer);
 }
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st) {
   GM_LAUNCH(finalize_kernel, dim3(P), dim3(1024), 0, st, a);
