@@ -585,7 +585,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
       d_outer(Pl, st), d_sig(Pl, st);
   DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
-  DevBuf<float> d_Kws((size_t)Pl * Bw * Bw, st);
+  DevBuf<float> d_Kws((size_t)Pl * std::max<size_t>((size_t)Bw * Bw, ws_tile_floats(Bw)), st);
   const bool rc = !full_k;
   DevBuf<int32_t> d_slot(rc ? (size_t)Pl * Bw : 0, st), d_slot_tmp(rc ? (size_t)Pl * Bw : 0, st), d_keep(rc ? Pl : 0, st);
   DevBuf<float> d_ATnew(rc ? (size_t)Pl * d_pad * ldat : 0, st);
@@ -695,6 +695,15 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     const int gn = gb[g + 1] - gb[g];
     for (int c = 0; c < kChunk && issued[g] < max_outer + 1; ++c) {
       const int64_t it = issued[g]++;
+      if (!rc && ws_solve_supported(Bw, g_npmax[g])) {  // selection + gather + local SMO in one CTA per pair
+        if (it >= max_outer) {  // the last selection only evaluates the stop test
+          launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
+          break;
+        }
+        launch_ws_solve(ag, gn, gs);
+        launch_f_update(ag, gn, g_npmax[g], gs);
+        continue;
+      }
       launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
       if (it >= max_outer) break;  // the last selection only evaluates the stop test
       if (rc) {
@@ -761,10 +770,14 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       cudaGraph_t cap;
       GM_CUDA(cudaStreamBeginCaptureToGraph(cs, cp.conditional.phGraph_out[0], nullptr, nullptr, 0,
                                             cudaStreamCaptureModeRelaxed));
-      launch_select_ws(ag, gn, 0, -1, cs);
-      if (rc) launch_rows_compute(ag, gn, npi, cs);
-      launch_gather_kws(ag, gn, -1, cs);
-      launch_local_smo(ag, gn, cs);
+      if (!rc && ws_solve_supported(Bw, npi)) {  // selection + gather + local SMO in one CTA per pair
+        launch_ws_solve(ag, gn, cs);
+      } else {
+        launch_select_ws(ag, gn, 0, -1, cs);
+        if (rc) launch_rows_compute(ag, gn, npi, cs);
+        launch_gather_kws(ag, gn, -1, cs);
+        launch_local_smo(ag, gn, cs);
+      }
       launch_f_update_loop(ag, gn, npi, h, max_outer, cs);
       GM_CUDA(cudaStreamEndCapture(cs, &cap));
       body_launches = (int64_t)(g_launches.load() - b0);
@@ -861,8 +874,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     std::vector<int> order(nt);
     for (int i = 0; i < nt; ++i) order[i] = i;
     std::sort(order.begin(), order.end(), [&](int x, int y) { return tr[3 * x + 1] < tr[3 * y + 1]; });
-    const char* names[6] = {"select", "gather", "smo", "fupdate", "rows_gather", "rows_contract"};
-    double dur[6] = {0}, cnt[6] = {0}, gap_before[6] = {0};
+    const char* names[7] = {"select", "gather", "smo", "fupdate", "rows_gather", "rows_contract", "ws_solve"};
+    double dur[7] = {0}, cnt[7] = {0}, gap_before[7] = {0};
     for (int j = 0; j < nt; ++j) {
       const int i = order[j];
       const int kd = (int)tr[3 * i];
@@ -872,7 +885,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     }
     const double span = nt ? (double)(tr[3 * order[nt - 1] + 2] - tr[3 * order[0] + 1]) : 0.0;
     std::string line;
-    for (int kd = 0; kd < 6; ++kd)
+    for (int kd = 0; kd < 7; ++kd)
       if (cnt[kd] > 0)
         line += std::string(" ") + names[kd] + " n=" + std::to_string((int)cnt[kd]) +
                 " mean_us=" + std::to_string(dur[kd] / cnt[kd] / 1e3).substr(0, 6) +

@@ -100,6 +100,12 @@ void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_
 // fused outer loop: one cluster per pair, whole solve in one launch (B <= 224)
 bool fused_solver_enabled(int B);
 void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStream_t st);
+// a3-a5 default kernels (wsolve.cu): fast selection, multi-CTA K_ws,ws gather into an
+// L2-resident tile, single-warp local SMO (FULL_K regime, B <= 224, n_p <= 16384;
+// GMPSVM_WSOLVE=0 selects the select_ws / gather_kws / local_smo kernels of solver.cu)
+bool ws_solve_supported(int B, int64_t np_max);
+size_t ws_tile_floats(int B);  // per-pair floats of the Kws tile buffer
+void launch_ws_solve(const SolverArgs& a, int P, cudaStream_t st);
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st);

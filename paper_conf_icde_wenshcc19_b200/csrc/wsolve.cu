@@ -1,0 +1,732 @@
+// wsolve.cu -- the default solver kernels of one outer iteration (FULL_K regime, B <= 224,
+// n_p <= 16384), Algorithm 2 lines 6-10 (L293-L305):
+//
+//   ws_select_kernel   a4  one 1024-thread CTA per pair.  Stages every instance's key ord(f) and
+//                          I_u / I_l flags in shared memory together with the global stop test
+//                          (Eq 9-10).  Sort-free selection: the r-th smallest of the warps' four
+//                          smallest per-thread minima is a threshold T with at least r candidates
+//                          <= T; one compaction pass collects the (few) candidates <= T and their
+//                          exact (key, index) ranks are counted -- O(list^2) compares on a list of
+//                          ~r entries.  Same semantics as select_body (reading R19): the newest
+//                          B - q rows retained, q/2 smallest f in I_u, the rest largest f in I_l.
+//                          The working set is written twice: in age order (retention) and sorted
+//                          by pair-local index (everything else), so "lowest position" == "lowest
+//                          index" for the tie rule R5 in the local solver.
+//   ws_gather_kernel   a3  K_ws,ws from the resident class-sorted kernel matrix, rows spread over
+//                          many CTAs (the gather is scattered 4-byte loads: one SM's outstanding
+//                          misses bound it at ~80 us, measured), into an L2-resident tile.
+//   ws_smo_kernel      a5  ONE warp per pair: the tile is bulk-copied (cp.async.bulk) into shared
+//                          memory; lane l owns working-set rows l, l+32, ...  Per inner step
+//                          (Eq 4-8, WSS2, local stop R20): per-lane min/max over its rows,
+//                          redux.sync over the warp -- no CTA barrier, no shared reduction slots.
+#include <cfloat>
+#include <climits>
+#include <cstdlib>
+#include <string>
+
+#include "kernels.h"
+#include "solver_dev.cuh"
+
+namespace gmpsvm {
+
+constexpr int kWT = 1024;        // select threads per CTA
+constexpr int kWMaxNp = 16384;   // pair size up to which keys and flags fit in shared memory
+constexpr int kWMaxB = 224;      // working-set rows (tile in the SMO kernel's shared memory)
+constexpr int kBufW = 16;        // per-warp candidate buffer (per side)
+constexpr int kFlat = 512;       // flattened candidate list capacity (per side)
+constexpr int kWRank = 128;      // threshold samples per side (4 per warp)
+
+__host__ __device__ inline int ws_tile_ld(int B) { return (B + 3) & ~3; }
+
+struct WSelSmall {
+  uint32_t retained[kWMaxNp / 32];
+  double red[2][32];
+  uint64_t sk[2][kWRank];  // the warps' 4 smallest per-thread minima
+  int32_t si[2][kWRank];
+  uint64_t bk[2][32][kBufW];  // per-warp candidates <= threshold
+  int32_t bi[2][32][kBufW];
+  int32_t bcnt[2][32];
+  int32_t boff[2][33];
+  uint64_t fk[2][kFlat];  // flattened candidate lists
+  int32_t fi[2][kFlat];
+  int32_t pick[1024];  // new working set in age order
+  int32_t wpre[kWMaxNp / 32];  // prefix popcounts of the picked-index bitmap
+  uint64_t thr_k[2];
+  int32_t thr_i[2];
+  int32_t overflow;
+  SelSmem sel;  // radix_pick fallback
+};
+
+__device__ __forceinline__ bool kless(uint64_t ka, int32_t ia, uint64_t kb, int32_t ib) {
+  return ka < kb || (ka == kb && ia < ib);
+}
+
+// lexicographic warp min of (key64, idx); all lanes get the winner's (k, i); returns its lane
+__device__ __forceinline__ int warp_min_ki(uint64_t& k, int32_t& i) {
+  const uint32_t h = (uint32_t)(k >> 32), l = (uint32_t)k;
+  const uint32_t m0 = __reduce_min_sync(FULLMASK, h);
+  const uint32_t m1 = __reduce_min_sync(FULLMASK, h == m0 ? l : 0xffffffffu);
+  const bool tie = h == m0 && l == m1;
+  const uint32_t m2 = __reduce_min_sync(FULLMASK, tie ? (uint32_t)i : 0xffffffffu);
+  const unsigned b = __ballot_sync(FULLMASK, tie && (uint32_t)i == m2);
+  k = ((uint64_t)m0 << 32) | m1;
+  i = (int32_t)m2;
+  return __ffs(b) - 1;
+}
+
+// exclusive prefix over the block of one value per thread (block order = thread order)
+__device__ __forceinline__ int block_excl_scan_count_thread(int v, int& total, int* sm /* 33 */) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(FULLMASK, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) sm[warp] = x;
+  __syncthreads();
+  if (warp == 0) {
+    const int w = lane < nw ? sm[lane] : 0;
+    int z = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(FULLMASK, z, o);
+      if (lane >= o) z += y;
+    }
+    if (lane < nw) sm[lane] = z - w;
+    if (lane == 31) sm[32] = z;
+  }
+  __syncthreads();
+  total = sm[32];
+  return sm[warp] + x - v;
+}
+
+// ------------------------------------------------------------------------------------------
+// a4 selection
+__global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a) {
+  const int lp = blockIdx.x + a.pair_base;
+  TraceScope ts_(a, lp, 0);
+  if (a.status[lp] != 0) return;
+  extern __shared__ __align__(16) unsigned char sdyn[];
+  uint64_t* keys = reinterpret_cast<uint64_t*>(sdyn);
+  uint8_t* flags = sdyn + (size_t)kWMaxNp * 8;
+  __shared__ WSelSmall W;
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t, B = a.B;
+  const double C = a.C;
+  const double* al = a.alpha + pd.a_off;
+  const double* fl = a.f + pd.a_off;
+  const int first = a.outer_iters[lp] == 0;
+  int32_t* ws_age = a.ws_tmp + (int64_t)lp * B;  // age order (oldest first)
+  int32_t* ws_idx = a.ws + (int64_t)lp * B;      // sorted by pair-local index
+  long long tq = clock64();
+  auto mark = [&](int k) {  // GMPSVM_SMO_PHASES: selection sub-phase cycles (thread 0)
+    if (a.sel_phase && t == 0) {
+      const long long tc = clock64();
+      a.sel_phase[(int64_t)(lp + 4096) * 5 + k] += tc - tq;
+      tq = tc;
+    }
+  };
+  // retained rows: the newest B - q of the previous working set (reading R19)
+  const int prev_n = first ? 0 : a.ws_n[lp];
+  const int keep = np <= B ? 0 : min(prev_n, B - a.q);
+  for (int w = t; w < (np + 31) / 32; w += kWT) W.retained[w] = 0u;
+  if (t == 0) W.overflow = 0;
+  __syncthreads();
+  for (int e = t; e < keep; e += kWT) {
+    const int idx = ws_age[prev_n - keep + e];
+    W.pick[e] = idx;
+    atomicOr(&W.retained[idx >> 5], 1u << (idx & 31));
+  }
+  __syncthreads();
+  // stage keys / flags, stop test (Eq 9-10), per-thread minima of the candidates of both sides
+  double fmin = DBL_MAX, fmax = -DBL_MAX;
+  uint64_t mk[2] = {~0ull, ~0ull};
+  int32_t mi[2] = {INT_MAX, INT_MAX};
+  for (int base = 0; base < np; base += 4 * kWT) {
+    double av[4], fv[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const int i = base + m * kWT + t;
+      av[m] = i < np ? al[i] : 0.0;
+      fv[m] = i < np ? fl[i] : 0.0;
+    }
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const int i = base + m * kWT + t;
+      if (i < np) {
+        const int y = i < pd.n_s ? 1 : -1;
+        const bool u = in_u(y, av[m], C), l = in_l(y, av[m], C);
+        const bool ret = (W.retained[i >> 5] >> (i & 31)) & 1u;
+        if (u) fmin = fmin < fv[m] ? fmin : fv[m];
+        if (l) fmax = fmax > fv[m] ? fmax : fv[m];
+        const uint64_t key = ord_key(fv[m]);
+        keys[i] = key;
+        flags[i] = (uint8_t)((u ? 1 : 0) | (l ? 2 : 0) | (ret ? 4 : 0));
+        if (u && !ret && key < mk[0]) {  // ascending i: strict < keeps the lowest index
+          mk[0] = key;
+          mi[0] = i;
+        }
+        if (l && !ret && ~key < mk[1]) {
+          mk[1] = ~key;
+          mi[1] = i;
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    fmin = ::fmin(fmin, __shfl_xor_sync(FULLMASK, fmin, o));
+    fmax = ::fmax(fmax, __shfl_xor_sync(FULLMASK, fmax, o));
+  }
+  if (lane == 0) {
+    W.red[0][warp] = fmin;
+    W.red[1][warp] = fmax;
+  }
+  __syncthreads();
+  fmin = W.red[0][lane];
+  fmax = W.red[1][lane];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    fmin = ::fmin(fmin, __shfl_xor_sync(FULLMASK, fmin, o));
+    fmax = ::fmax(fmax, __shfl_xor_sync(FULLMASK, fmax, o));
+  }
+  const double gap = fmax - fmin;
+  const bool done = (fmin == DBL_MAX) || (fmax == -DBL_MAX) || !(gap >= a.eps);
+  if (t == 0) {
+    a.gap[lp] = gap;
+    if (done) a.status[lp] = 1;
+    else a.outer_iters[lp] += 1;
+  }
+  mark(0);
+  if (done) return;
+  if (np <= B) {  // the whole pair is the working set (unchanged after the first iteration)
+    if (first) {
+      for (int e = t; e < np; e += kWT) {
+        ws_idx[e] = e;
+        ws_age[e] = e;
+      }
+      if (t == 0) a.ws_n[lp] = np;
+    }
+    return;
+  }
+  const int need = B - keep, need_u = need / 2;
+  // the four smallest per-thread minima of each warp (both sides), for the thresholds
+#pragma unroll 1
+  for (int j = 0; j < 4; ++j) {
+#pragma unroll
+    for (int s = 0; s < 2; ++s) {
+      uint64_t k = mk[s];
+      int32_t x = mi[s];
+      const int wl = warp_min_ki(k, x);
+      if (lane == 0) {
+        W.sk[s][warp * 4 + j] = k;
+        W.si[s][warp * 4 + j] = x;
+      }
+      if (lane == wl) {
+        mk[s] = ~0ull;
+        mi[s] = INT_MAX;
+      }
+    }
+  }
+  if (t < 2) {
+    W.thr_k[t] = ~0ull;  // fewer samples than the rank: every candidate qualifies
+    W.thr_i[t] = INT_MAX;
+  }
+  __syncthreads();
+  // thresholds by counting ranks: U at rank need_u - 1, L at rank need - 1 (so the L list
+  // still holds need - (U picks) candidates after removing the U picks it shares)
+  if (t < 2 * kWRank) {
+    const int s = t / kWRank, j = t % kWRank;
+    const int r = s == 0 ? need_u : need;
+    const uint64_t k = W.sk[s][j];
+    const int32_t x = W.si[s][j];
+    if (x != INT_MAX && r >= 1 && r <= kWRank) {
+      int rank = 0;
+      for (int q = 0; q < kWRank; ++q) rank += kless(W.sk[s][q], W.si[s][q], k, x) ? 1 : 0;
+      if (rank == r - 1) {
+        W.thr_k[s] = k;
+        W.thr_i[s] = x;
+      }
+    }
+    if (s == 0 && j == 0 && r == 0) {  // nothing wanted from U
+      W.thr_k[0] = 0ull;
+      W.thr_i[0] = -1;
+    }
+  }
+  __syncthreads();
+  mark(1);
+  // compaction of the candidates at or below the thresholds into per-warp buffers
+  {
+    const uint64_t tk0 = W.thr_k[0], tk1 = W.thr_k[1];
+    const int32_t ti0 = W.thr_i[0], ti1 = W.thr_i[1];
+    int c0 = 0, c1 = 0;
+    for (int base = 0; base < np; base += kWT) {
+      const int i = base + t;
+      bool cu = false, cl = false;
+      uint64_t kk = 0;
+      if (i < np) {
+        const uint8_t fg = flags[i];
+        kk = keys[i];
+        cu = (fg & 5) == 1 && !kless(tk0, ti0, kk, i);
+        cl = (fg & 6) == 2 && !kless(tk1, ti1, ~kk, i);
+      }
+      const unsigned bu = __ballot_sync(FULLMASK, cu), bl = __ballot_sync(FULLMASK, cl);
+      const int ou = c0 + __popc(bu & ((1u << lane) - 1u)), ol = c1 + __popc(bl & ((1u << lane) - 1u));
+      if (cu && ou < kBufW) {
+        W.bk[0][warp][ou] = kk;
+        W.bi[0][warp][ou] = i;
+      }
+      if (cl && ol < kBufW) {
+        W.bk[1][warp][ol] = ~kk;
+        W.bi[1][warp][ol] = i;
+      }
+      c0 += __popc(bu);
+      c1 += __popc(bl);
+    }
+    if (lane == 0) {
+      W.bcnt[0][warp] = c0;
+      W.bcnt[1][warp] = c1;
+      if (c0 > kBufW || c1 > kBufW) W.overflow = 1;
+    }
+  }
+  __syncthreads();
+  if (warp < 2) {  // prefix offsets of the per-warp buffers (warp s: side s)
+    const int v = W.bcnt[warp][lane];
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(FULLMASK, x, o);
+      if (lane >= o) x += y;
+    }
+    W.boff[warp][lane] = x - v;
+    if (lane == 31) {
+      W.boff[warp][32] = x;
+      if (x > kFlat) W.overflow = 1;
+    }
+  }
+  __syncthreads();
+  int got = 0;
+  if (!W.overflow) {
+    {  // flatten: thread (warp w, lane j) copies slot j of warp w's U (j < 16) or L (j >= 16) buffer
+      const int s = lane >> 4, j = lane & 15;
+      if (j < W.bcnt[s][warp]) {
+        const int o = W.boff[s][warp] + j;
+        W.fk[s][o] = W.bk[s][warp][j];
+        W.fi[s][o] = W.bi[s][warp][j];
+      }
+    }
+    __syncthreads();
+    const int nu = W.boff[0][32], nl = W.boff[1][32];
+    // U: exact (key, index) rank by counting; the need_u smallest in rank order
+    const int got_u = min(need_u, nu);
+    if (t < nu) {
+      const uint64_t k = W.fk[0][t];
+      const int32_t x = W.fi[0][t];
+      int rank = 0;
+      for (int q = 0; q < nu; ++q) rank += kless(W.fk[0][q], W.fi[0][q], k, x) ? 1 : 0;
+      if (rank < got_u) {
+        W.pick[keep + rank] = x;
+        flags[x] |= 4;
+      }
+    }
+    __syncthreads();
+    // L: rank among the entries U did not take (threads 512.. while U's threads are idle)
+    const int need_l = need - got_u;
+    const int tl = t - 512;
+    bool free_l = false;
+    if (tl >= 0 && tl < nl) {
+      const uint64_t k = W.fk[1][tl];
+      const int32_t x = W.fi[1][tl];
+      free_l = !(flags[x] & 4);
+      if (free_l) {
+        int rank = 0;
+        for (int q = 0; q < nl; ++q) {
+          const int32_t xq = W.fi[1][q];
+          rank += (!(flags[xq] & 4) && kless(W.fk[1][q], xq, k, x)) ? 1 : 0;
+        }
+        if (rank < need_l) W.pick[keep + got_u + rank] = x;
+      }
+    }
+    const int nfree = __syncthreads_count(free_l);
+    got = got_u + min(need_l, nfree);
+    for (int e = keep + got_u + t; e < keep + got; e += kWT) flags[W.pick[e]] |= 4;
+    __syncthreads();
+    // L ran short (every L candidate is in the list): U again, as select_sides does
+    if (got < need) got += radix_pick<true>(SmemSrc{keys, flags}, np, need - got, W.pick + keep + got, W.sel);
+  } else {  // a buffer overflowed (heavily tied or clustered keys): exact radix selection
+    got = select_sides(SmemSrc{keys, flags}, np, need, W.pick + keep, W.sel);
+    if (a.sel_phase && t == 0) a.sel_phase[(int64_t)(lp + 4096) * 5 + 4] += 1;  // fallbacks (diagnostic)
+  }
+  __syncthreads();
+  mark(2);
+  // write the working set: age order, and sorted by index (rank = set bits below it in a
+  // bitmap of the picked indices: per-word prefix popcounts)
+  const int cnt = keep + got;
+  const int nwords = (np + 31) / 32;
+  for (int w = t; w < nwords; w += kWT) W.retained[w] = 0u;
+  __syncthreads();
+  if (t < cnt) atomicOr(&W.retained[W.pick[t] >> 5], 1u << (W.pick[t] & 31));
+  __syncthreads();
+  {  // exclusive prefix of the word popcounts (nwords <= 512: 16 per warp... one per thread)
+    int v = t < nwords ? __popc(W.retained[t]) : 0;
+    int tot = 0;
+    const int pre = block_excl_scan_count_thread(v, tot, W.boff[0]);
+    if (t < nwords) W.wpre[t] = pre;
+  }
+  __syncthreads();
+  if (t < cnt) {
+    const int32_t x = W.pick[t];
+    const int rank = W.wpre[x >> 5] + __popc(W.retained[x >> 5] & ((1u << (x & 31)) - 1u));
+    ws_age[t] = x;
+    ws_idx[rank] = x;
+  }
+  if (t == 0) a.ws_n[lp] = cnt;
+  mark(3);
+}
+
+// ------------------------------------------------------------------------------------------
+// a3: K_ws,ws tile (row stride ws_tile_ld(B)) from the resident kernel matrix
+constexpr int kGR = 8;  // tile rows per CTA
+
+__global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
+  const int lp = blockIdx.x + a.pair_base;
+  TraceScope ts_(a, lp, 1);
+  if (a.status[lp] != 0) return;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  if (np <= a.B && a.outer_iters[lp] != 1) return;  // working set (and tile) unchanged
+  const int wn = a.ws_n[lp];
+  const int r0 = blockIdx.y * kGR;
+  if (r0 >= wn) return;
+  __shared__ int64_t g[kWMaxB];
+  const int32_t* ws = a.ws + (int64_t)lp * a.B;
+  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
+  __syncthreads();
+  const int ld = ws_tile_ld(a.B);
+  float* tile = a.Kws + (int64_t)lp * a.B * ld;
+  const int r1 = min(wn, r0 + kGR);
+  constexpr int M = (kGR * kWMaxB + 255) / 256;  // loads per thread, all in flight
+  float v[M];
+#pragma unroll
+  for (int m = 0; m < M; ++m) {
+    const int q = threadIdx.x + m * 256;
+    const int r = r0 + q / wn, c = q % wn;
+    v[m] = r < r1 ? __ldg(a.K + g[r] * a.ldk + g[c]) : 0.f;
+  }
+#pragma unroll
+  for (int m = 0; m < M; ++m) {
+    const int q = threadIdx.x + m * 256;
+    const int r = r0 + q / wn, c = q % wn;
+    if (r < r1) tile[(int64_t)r * ld + c] = v[m];
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// a5: single-warp local SMO
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+size_t ws_smo_smem(int B) { return (size_t)B * ws_tile_ld(B) * 4 + (size_t)B * 8 + 256; }
+
+__device__ __forceinline__ float lds_f32(uint32_t addr) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ double lds_f64(uint32_t addr) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ void sts_f64(uint32_t addr, double v) {
+  asm volatile("st.shared.f64 [%0], %1;" ::"r"(addr), "d"(v) : "memory");
+}
+
+// in-place pairwise (tree) reductions over a lane's rows; the lower row wins ties
+template <int E>
+__device__ __forceinline__ void tree_min_u64(uint64_t (&k)[E], int (&q)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w)
+      if (k[i + w] < k[i]) {
+        k[i] = k[i + w];
+        q[i] = q[i + w];
+      }
+}
+template <int E>
+__device__ __forceinline__ void tree_max_u32(uint32_t (&k)[E], int (&q)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w)
+      if (k[i + w] > k[i]) {
+        k[i] = k[i + w];
+        q[i] = q[i + w];
+      }
+}
+template <int E>
+__device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w) k[i] = k[i + w] > k[i] ? k[i + w] : k[i];
+}
+
+template <int E>
+__global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
+  const int lp = blockIdx.x + a.pair_base;
+  TraceScope ts_(a, lp, 2);
+  if (a.status[lp] != 0) return;
+  extern __shared__ __align__(16) unsigned char mdyn[];
+  const int lane = threadIdx.x;
+  const PairDesc pd = a.pairs[lp];
+  const int B = a.B, wn = a.ws_n[lp], ld = ws_tile_ld(B);
+  uint32_t kws;  // K_ws,ws tile, row stride ld (opaque: keeps the shared window base out of the loop)
+  asm volatile("mov.u32 %0, %1;" : "=r"(kws) : "r"(smem_addr(mdyn)));
+  const uint32_t als = kws + (uint32_t)B * ld * 4;               // alpha of the working set
+  const uint32_t bar = als + (uint32_t)B * 8;                    // mbarrier of the bulk copy
+  const long long t_entry = clock64();
+  // bulk copy of the tile rows [0, wn) into shared memory
+  const uint32_t bytes = (uint32_t)wn * ld * 4;  // ld % 4 == 0: a multiple of 16
+  if (lane == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+    const char* src = reinterpret_cast<const char*>(a.Kws + (int64_t)lp * B * ld);
+    constexpr uint32_t kChunk = 32768;
+    for (uint32_t o = 0; o < bytes; o += kChunk) {
+      const uint32_t n = bytes - o < kChunk ? bytes - o : kChunk;
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                       kws + o),
+                   "l"(src + o), "r"(n), "r"(bar)
+                   : "memory");
+    }
+  }
+  __syncwarp();
+  // per-row state: lane owns positions lane + 32 q (the working set sorted by index)
+  const double C = a.C, eps = a.eps, ratio = a.local_ratio;
+  const int32_t* ws = a.ws + (int64_t)lp * B;
+  int32_t idx[E];
+  double f[E];
+  uint32_t umask = 0u, lmask = 0u, ypos = 0u, vmask = 0u;
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = lane + 32 * q;
+    const bool valid = e < wn;
+    idx[q] = valid ? ws[e] : INT_MAX;
+    const int y = (valid && idx[q] < pd.n_s) ? 1 : -1;
+    const double al = valid ? a.alpha[pd.a_off + idx[q]] : 0.0;
+    f[q] = valid ? a.f[pd.a_off + idx[q]] : 0.0;
+    if (valid) {
+      sts_f64(als + e * 8, al);
+      vmask |= 1u << q;
+      if (y > 0) ypos |= 1u << q;
+      if (in_u(y, al, C)) umask |= 1u << q;
+      if (in_l(y, al, C)) lmask |= 1u << q;
+    }
+  }
+  const long long t_state = clock64();
+  {
+    uint32_t done = 0;
+    do {
+      asm volatile(
+          "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n selp.u32 %0, 1, 0, p;\n}\n"
+          : "=r"(done)
+          : "r"(bar)
+          : "memory");
+    } while (!done);
+  }
+  float kd[E];
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = lane + 32 * q;
+    kd[q] = e < wn ? lds_f32(kws + (uint32_t)(e * ld + e) * 4) : 1.f;
+  }
+  __syncwarp();
+  const int cap = a.inner_cap;
+  int it = 0;
+  double delta0 = 0.0;
+  const long long t_begin = clock64();
+  const bool prof = a.smo_phase != nullptr;  // GMPSVM_SMO_PHASES: per-phase SM cycles
+  long long ph[4] = {0, 0, 0, 0}, tp = t_begin;
+  auto markp = [&](int k) {
+    if (prof) {
+      const long long tc = clock64();
+      ph[k] += tc - tp;
+      tp = tc;
+    }
+  };
+  for (;;) {
+    // Eq 4: u = argmin_{I_u} f; ties -> lowest position (== lowest pair-local index, R5)
+    uint64_t uk[E];
+    int uq[E];
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      uk[q] = ((umask >> q) & 1u) ? ord_key(f[q]) : ~0ull;
+      uq[q] = q;
+    }
+    tree_min_u64<E>(uk, uq);
+    const uint32_t h = (uint32_t)(uk[0] >> 32), l = (uint32_t)uk[0];
+    const uint32_t pos = uk[0] == ~0ull ? 0xffffffffu : (uint32_t)(lane + 32 * uq[0]);
+    const uint32_t m0 = __reduce_min_sync(FULLMASK, h);
+    const uint32_t m1 = __reduce_min_sync(FULLMASK, h == m0 ? l : 0xffffffffu);
+    const uint32_t ue32 = __reduce_min_sync(FULLMASK, (h == m0 && l == m1) ? pos : 0xffffffffu);
+    if (ue32 == 0xffffffffu) break;  // I_u empty
+    const int ue = (int)ue32;
+    const int uq0 = ue >> 5, ul = ue & 31;
+    const int yu = ((__shfl_sync(FULLMASK, ypos, ul) >> uq0) & 1u) ? 1 : -1;
+    const double fu = key_double(((uint64_t)m0 << 32) | m1);
+    const uint32_t urow = kws + (uint32_t)(ue * ld) * 4;
+    const double au = lds_f64(als + ue * 8);
+    const float kuu = lds_f32(urow + ue * 4);
+    float ku[E];
+#pragma unroll
+    for (int q = 0; q < E; ++q) ku[q] = lds_f32(urow + (lane + 32 * q) * 4);
+    markp(0);
+    // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_t - f_u)^2 / eta_t (FP32, reading R29); the
+    // winner's (f_t - f_u) / eta_t is the unclipped step; Eq 10: f_max over I_l
+    uint32_t sb[E];
+    int sq[E];
+    float st[E];
+    uint64_t lk[E];
+#pragma unroll
+    for (int q = 0; q < E; ++q) {
+      const bool il = (lmask >> q) & 1u;
+      const float eta = fmaxf(fmaf(-2.f, ku[q], kuu + kd[q]), 1e-12f);
+      const float df = (float)(f[q] - fu);
+      float r;
+      asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(eta));
+      st[q] = df * r;
+      sb[q] = (il && f[q] > fu) ? __float_as_uint(df * st[q]) : 0u;  // scores >= 0: bits order as values
+      sq[q] = q;
+      lk[q] = il ? ord_key(f[q]) : 0ull;
+    }
+    tree_max_u32<E>(sb, sq);
+    tree_max_u64<E>(lk);
+    const uint32_t xh = __reduce_max_sync(FULLMASK, (uint32_t)(lk[0] >> 32));
+    const uint32_t xl = __reduce_max_sync(FULLMASK, (uint32_t)(lk[0] >> 32) == xh ? (uint32_t)lk[0] : 0u);
+    const uint32_t smax = __reduce_max_sync(FULLMASK, sb[0]);
+    const uint32_t lpos = (sb[0] != 0u && sb[0] == smax) ? (uint32_t)(lane + 32 * sq[0]) : 0xffffffffu;
+    const uint32_t le32 = __reduce_min_sync(FULLMASK, lpos);
+    markp(1);
+    const double fmax = (xh == 0u && xl == 0u) ? -DBL_MAX : key_double(((uint64_t)xh << 32) | xl);
+    const double gap = fmax - fu;
+    if (it == 0) delta0 = gap;
+    const double tol = eps > ratio * delta0 ? eps : ratio * delta0;
+    if (!(gap >= tol) || le32 == 0xffffffffu || it >= cap) break;
+    const int le = (int)le32;
+    const int ll = le & 31, lq = le >> 5;
+    float stl = st[0];
+#pragma unroll
+    for (int q = 1; q < E; ++q)
+      if (q == lq) stl = st[q];
+    double s = (double)__shfl_sync(FULLMASK, stl, ll);
+    const int yl = ((__shfl_sync(FULLMASK, ypos, ll) >> lq) & 1u) ? 1 : -1;
+    const uint32_t lrow = kws + (uint32_t)(le * ld) * 4;
+    const double alv = lds_f64(als + le * 8);
+    float kl[E];
+#pragma unroll
+    for (int q = 0; q < E; ++q) kl[q] = lds_f32(lrow + (lane + 32 * q) * 4);
+    markp(2);
+    // Eq 6-7 with explicit clipping (reading R4): common step s, bounds assigned exactly
+    const double Uu = yu > 0 ? C - au : au;
+    const double Ll = yl > 0 ? alv : C - alv;
+    bool bnu = false, bnl = false;
+    if (Uu <= s) {
+      s = Uu;
+      bnu = true;
+    }
+    if (Ll <= s) {
+      if (Ll < s) bnu = false;
+      s = Ll;
+      bnl = true;
+    }
+    const double nau = bnu ? (yu > 0 ? C : 0.0) : au + yu * s;
+    const double nal = bnl ? (yl > 0 ? 0.0 : C) : alv - yl * s;
+    // Eq 8 on the working set: f_i += s (K_ui - K_li)
+#pragma unroll
+    for (int q = 0; q < E; ++q) f[q] = fma(s, (double)(ku[q] - kl[q]), f[q]);
+    // membership of u and l after the step (owners update their bits; alpha in shared memory)
+    const uint32_t uin = in_u(yu, nau, C) ? 1u : 0u, uil = in_l(yu, nau, C) ? 1u : 0u;
+    const uint32_t lin = in_u(yl, nal, C) ? 1u : 0u, lil = in_l(yl, nal, C) ? 1u : 0u;
+    if (lane == ul) {
+      umask = (umask & ~(1u << uq0)) | (uin << uq0);
+      lmask = (lmask & ~(1u << uq0)) | (uil << uq0);
+    }
+    if (lane == ll) {
+      umask = (umask & ~(1u << lq)) | (lin << lq);
+      lmask = (lmask & ~(1u << lq)) | (lil << lq);
+    }
+    if (lane == 0) {
+      sts_f64(als + ue * 8, nau);
+      sts_f64(als + le * 8, nal);
+    }
+    __syncwarp();
+    ++it;
+    if (prof && f[0] == -1.2345e300) ph[3] += 1;  // keep the f update ahead of the clock read
+    markp(3);
+  }
+  __syncwarp();
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = lane + 32 * q;
+    if ((vmask >> q) & 1u) {
+      const double al = lds_f64(als + e * 8);
+      const double a0 = a.alpha[pd.a_off + idx[q]];
+      a.dcoef[(int64_t)lp * B + e] = (al - a0) * (((ypos >> q) & 1u) ? 1.0 : -1.0);
+      a.alpha[pd.a_off + idx[q]] = al;
+    }
+  }
+  if (lane == 0) {
+    a.inner_iters[lp] += it;
+    a.smo_cycles[lp] += clock64() - t_begin;
+    if (prof) {
+      for (int k = 0; k < 4; ++k) a.smo_phase[lp * 5 + k] += ph[k];
+      a.smo_phase[lp * 5 + 4] += t_begin - t_entry;
+      a.sel_phase[lp * 5 + 2] += t_state - t_entry;  // prologue split: state loads | tile wait
+      a.sel_phase[lp * 5 + 3] += t_begin - t_state;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+bool ws_solve_supported(int B, int64_t np_max) {
+  static const bool off = getenv("GMPSVM_WSOLVE") && std::string(getenv("GMPSVM_WSOLVE")) == "0";
+  return !off && B >= 2 && B <= kWMaxB && np_max <= kWMaxNp;
+}
+
+size_t ws_tile_floats(int B) { return (size_t)B * ws_tile_ld(B); }
+
+void launch_ws_solve(const SolverArgs& a, int P, cudaStream_t st) {
+  const size_t sel_dyn = (size_t)kWMaxNp * 9;
+  const size_t smo_dyn = ws_smo_smem(a.B);
+  static bool configured = false;
+  if (!configured) {
+    GM_CUDA(cudaFuncSetAttribute(ws_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sel_dyn));
+    const int mx = (int)ws_smo_smem(kWMaxB);
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<5>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    configured = true;
+  }
+  GM_LAUNCH(ws_select_kernel, dim3(P), dim3(kWT), sel_dyn, st, a);
+  GM_LAUNCH(ws_gather_kernel, dim3(P, (unsigned)ceil_div(a.B, kGR)), dim3(256), 0, st, a);
+  switch ((a.B + 31) / 32) {
+    case 1: GM_LAUNCH(ws_smo_kernel<1>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 2: GM_LAUNCH(ws_smo_kernel<2>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 3: GM_LAUNCH(ws_smo_kernel<3>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 4: GM_LAUNCH(ws_smo_kernel<4>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 5: GM_LAUNCH(ws_smo_kernel<5>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 6: GM_LAUNCH(ws_smo_kernel<6>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    default: GM_LAUNCH(ws_smo_kernel<7>, dim3(P), dim3(32), smo_dyn, st, a); break;
+  }
+}
+
+}  // namespace gmpsvm

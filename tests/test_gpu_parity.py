@@ -8,6 +8,8 @@ Tolerances (SURVEY.md §8(c) "Parity contract"):
   KKT audit          exact-K gap of the GPU alpha <= eps + 2 max_i |sum_j a_j y_j (K32_ij - K64_ij)|
 All at eps = 1e-5 (at 1e-3 even LibSVM sits 1.7e-3 C from the optimum).
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -18,6 +20,7 @@ torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
 EPS = 1e-5
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.fixture(scope="module")
@@ -191,7 +194,7 @@ def _prob_tol(ref, X, y, Xt):
     return 1e-4 + worst
 
 
-@pytest.mark.parametrize("ws,q", [(64, 32), (128, 64), (256, 128), (64, 16)])
+@pytest.mark.parametrize("ws,q", [(64, 32), (128, 64), (256, 128), (64, 16), (100, 50), (224, 112), (224, 56)])
 def test_batched_working_set_multi_outer_iterations(gm, ws, q):
     # n_p = 400 > B: exercises the radix selection, retention of the newest B-q rows and
     # many outer iterations (L289-L305); the fixed point must not depend on B, q.
@@ -230,3 +233,27 @@ def test_device_inputs_match_host_inputs(gm):
     p1 = m1.predict_proba(Xt)
     p2 = m2.predict_proba(torch.from_numpy(Xt).cuda()).cpu().numpy()
     np.testing.assert_array_equal(p1, p2)  # deterministic kernels: bitwise identical
+
+
+def test_fused_and_split_solver_paths_agree(gm, tmp_path):
+    """The fused selection + gather + local-SMO kernel (wsolve.cu, default for B <= 224) and the
+    split select_ws / gather_kws / local_smo kernels (GMPSVM_WSOLVE=0) implement the same
+    readings (R19, R20); both must reach the same fixed point (Eq 9) on a multi-pair
+    MNIST-shaped problem with many outer iterations."""
+    import subprocess
+    import sys
+
+    spec, X, y, Xt, yt = datagen.make_config("mnist", n_train=3000, n_test=200)
+    m1 = gm.train(X, y, spec.k, spec.C, spec.gamma, EPS, ws_size=96)
+    assert m1.train_stats()["outer_iters_max"] > 3
+    p1 = m1.predict_proba(Xt)
+    code = (
+        "import sys, json, numpy as np; sys.path.insert(0, %r); import datagen, paper_conf_icde_wenshcc19_b200 as gm;"
+        "spec, X, y, Xt, yt = datagen.make_config('mnist', n_train=3000, n_test=200);"
+        "m = gm.train(X, y, spec.k, spec.C, spec.gamma, %r, ws_size=96);"
+        "np.save(%r, m.predict_proba(Xt))" % (ROOT, EPS, str(tmp_path / "p2.npy"))
+    )
+    env = dict(os.environ, GMPSVM_WSOLVE="0")
+    subprocess.run([sys.executable, "-c", code], check=True, env=env, timeout=600)
+    p2 = np.load(tmp_path / "p2.npy")
+    assert np.abs(p1 - p2).max() <= 1e-4
