@@ -695,13 +695,9 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     const int gn = gb[g + 1] - gb[g];
     for (int c = 0; c < kChunk && issued[g] < max_outer + 1; ++c) {
       const int64_t it = issued[g]++;
-      if (!rc && ws_solve_supported(Bw, g_npmax[g])) {  // selection + gather + local SMO in one CTA per pair
-        if (it >= max_outer) {  // the last selection only evaluates the stop test
-          launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
-          break;
-        }
-        launch_ws_solve(ag, gn, gs);
-        launch_f_update(ag, gn, g_npmax[g], gs);
+      if (!rc && ws_solve_supported(Bw, g_npmax[g])) {  // default kernels (wsolve.cu)
+        launch_ws_iteration(ag, gn, g_npmax[g], 0, 0, max_outer, gs, it > 0);
+        if (it >= max_outer) break;
         continue;
       }
       launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
@@ -726,7 +722,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   const bool graph_mode = !fused && !streams_mode;
   GraphGuard gg;
   int64_t body_launches = 0;
-  int n_branches = 0;
+  std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
+  int n_branches = 0, final_selects = 0;
   if (fused) {  // the whole outer loop of every pair in one launch (clusters, no host round trips)
     SolverArgs ag = a;
     ag.pair_base = 0;
@@ -766,27 +763,36 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, nullptr, 0, &cp));
       SolverArgs ag = a;
       ag.pair_base = i;
+      const bool wsp = !rc && ws_solve_supported(Bw, npi);
       const uint64_t b0 = g_launches.load();
       cudaGraph_t cap;
       GM_CUDA(cudaStreamBeginCaptureToGraph(cs, cp.conditional.phGraph_out[0], nullptr, nullptr, 0,
                                             cudaStreamCaptureModeRelaxed));
-      if (!rc && ws_solve_supported(Bw, npi)) {  // selection + gather + local SMO in one CTA per pair
-        launch_ws_solve(ag, gn, cs);
+      if (wsp) {  // default kernels (wsolve.cu): selection -> gather -> local SMO -> f-update, unrolled:
+                  // the conditional node's re-launch (~10 us) is paid every `unroll` iterations
+        static const int unroll = getenv("GMPSVM_UNROLL") ? std::max(1, atoi(getenv("GMPSVM_UNROLL"))) : 2;
+        for (int u = 0; u < unroll; ++u) launch_ws_iteration(ag, gn, npi, h, u == unroll - 1, max_outer, cs, u > 0);
       } else {
         launch_select_ws(ag, gn, 0, -1, cs);
         if (rc) launch_rows_compute(ag, gn, npi, cs);
         launch_gather_kws(ag, gn, -1, cs);
         launch_local_smo(ag, gn, cs);
+        launch_f_update_loop(ag, gn, npi, h, max_outer, cs);
       }
-      launch_f_update_loop(ag, gn, npi, h, max_outer, cs);
       GM_CUDA(cudaStreamEndCapture(cs, &cap));
       body_launches = (int64_t)(g_launches.load() - b0);
-      GM_CUDA(cudaStreamBeginCaptureToGraph(cs, gg.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
-      launch_select_ws(ag, gn, 0, -1, cs);
-      GM_CUDA(cudaStreamEndCapture(cs, &cap));
+      body_per_pair[i] = body_launches;
+      if (!wsp) {  // the stop test on the final alpha (the default path tests in every f-update)
+        GM_CUDA(cudaStreamBeginCaptureToGraph(cs, gg.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
+        launch_select_ws(ag, gn, 0, -1, cs);
+        GM_CUDA(cudaStreamEndCapture(cs, &cap));
+        ++final_selects;
+      }
     }
-    n_branches = nbr;
+    n_branches = final_selects;
     g_launches.fetch_sub(g_launches.load() - l0);  // captured, not executed: counted after the run
+    GM_CUDA(cudaEventRecord(ev_ready, st));
+    GM_CUDA(cudaStreamWaitEvent(pool[0], ev_ready, 0));
     GM_CUDA(cudaGraphInstantiate(&gg.exec, gg.graph, 0));
     HT("graph_build");
     GM_CUDA(cudaGraphLaunch(gg.exec, pool[0]));
@@ -856,8 +862,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
   if (graph_mode) {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
-    int64_t ex = n_branches;  // one final selection per branch
-    for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_launches;  // counted at each branch's first pair
+    int64_t ex = n_branches;  // one final selection per split-path branch
+    for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_per_pair[i];  // counted at each branch's first pair
     g_launches.fetch_add((uint64_t)ex);
     if (rc) {
       rc_launches = 0;
@@ -961,7 +967,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     mdl->b[p] = hb[i];
     mdl->A[p] = hA[i];
     mdl->B[p] = hB[i];
-    if (h_st[i] == 0) {  // still active: the outer-iteration cap stopped it
+    if (h_st[i] == 0 || h_st[i] == 2) {  // still active / capped in-kernel: the outer-iteration cap stopped it
       h_st[i] = 2;
       cap_hit = true;
     }

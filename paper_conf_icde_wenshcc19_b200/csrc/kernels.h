@@ -39,7 +39,7 @@ void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, flo
                       cudaStream_t st);
 bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel
 
-// ---------------- a4-a9 solver (solver.cu)
+// ---------------- a4-a9 solver (solver.cu, wsolve.cu)
 struct SolverArgs {
   const PairDesc* pairs;
   const float* K;
@@ -86,6 +86,7 @@ struct SolverArgs {
   int ldat;            // leading dimension of ATnew (round_up(B, 128))
   double gamma;
 };
+constexpr int kWsMaxNp = 16384;  // pair size limit of the default path (keys + flags in shared memory)
 
 void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st);
 void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st);
@@ -104,8 +105,12 @@ void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStrea
 // L2-resident tile, single-warp local SMO (FULL_K regime, B <= 224, n_p <= 16384;
 // GMPSVM_WSOLVE=0 selects the select_ws / gather_kws / local_smo kernels of solver.cu)
 bool ws_solve_supported(int B, int64_t np_max);
-size_t ws_tile_floats(int B);  // per-pair floats of the Kws tile buffer
-void launch_ws_solve(const SolverArgs& a, int P, cudaStream_t st);
+size_t ws_tile_floats(int B);  // per-pair floats of the Kws buffer (tile + SMO state)
+// one outer iteration: selection (+ stop test), K_ws,ws gather, single-warp local SMO, f-update
+// (with set_cond it sets the graph loop condition); programmatic dependent launches inside the
+// iteration, and across iterations when chained (the previous iteration is in the same stream)
+void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int set_cond,
+                         int64_t max_outer, cudaStream_t st, bool chained = false);
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st);

@@ -30,7 +30,7 @@
 namespace gmpsvm {
 
 constexpr int kWT = 1024;        // select threads per CTA
-constexpr int kWMaxNp = 16384;   // pair size up to which keys and flags fit in shared memory
+constexpr int kWMaxNp = kWsMaxNp;  // pair size up to which keys and flags fit in shared memory
 constexpr int kWMaxB = 224;      // working-set rows (tile in the SMO kernel's shared memory)
 constexpr int kBufW = 16;        // per-warp candidate buffer (per side)
 constexpr int kFlat = 512;       // flattened candidate list capacity (per side)
@@ -38,8 +38,18 @@ constexpr int kWRank = 128;      // threshold samples per side (4 per warp)
 
 __host__ __device__ inline int ws_tile_ld(int B) { return (B + 3) & ~3; }
 
+// Programmatic dependent launch: each kernel of an outer iteration lets the next one be scheduled
+// at once (its CTAs become resident and wait), and waits for its predecessor's completion and
+// memory before touching shared state -- the launch latency leaves the per-iteration chain.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_enter() {
+  pdl_wait();
+  pdl_trigger();
+}
+
 struct WSelSmall {
-  uint32_t retained[kWMaxNp / 32];
+  uint32_t retained[kWMaxNp / 32];  // retained rows; then the write-out bitmap
   double red[2][32];
   uint64_t sk[2][kWRank];  // the warps' 4 smallest per-thread minima
   int32_t si[2][kWRank];
@@ -102,8 +112,59 @@ __device__ __forceinline__ int block_excl_scan_count_thread(int v, int& total, i
 }
 
 // ------------------------------------------------------------------------------------------
+// Kws buffer of a pair: the K_ws,ws tile (B rows, stride ld) followed by the local solver's
+// state in sorted order: alpha[B] (FP64), f[B] (FP64), index[round_up(B, 4)] (int32).
+__host__ __device__ inline size_t ws_state_off(int B) { return (size_t)B * ws_tile_ld(B); }  // in floats
+__host__ __device__ inline size_t ws_buf_floats(int B) { return ws_state_off(B) + 4 * (size_t)B + ((B + 3) & ~3); }
+
+// exclusive prefix of the popcounts of nwords bitmap words (any blockDim); sm: 33 ints
+__device__ void bitmap_prefix(const uint32_t* bm, int nwords, int32_t* wpre, int* sm) {
+  int carry = 0;
+  for (int base = 0; base < nwords; base += blockDim.x) {
+    const int w = base + threadIdx.x;
+    const int v = w < nwords ? __popc(bm[w]) : 0;
+    int tot = 0;
+    const int pre = block_excl_scan_count_thread(v, tot, sm);
+    if (w < nwords) wpre[w] = carry + pre;
+    carry += tot;
+    __syncthreads();
+  }
+}
+
+// Publishes the new working set of pair lp (pick[0..cnt) in age order, oldest first): a.ws_tmp
+// (age order, for the next retention), a.ws (sorted by pair-local index), a.ws_n, and the SMO
+// state (alpha, f, index in sorted order) behind the pair's tile.  All threads; bm:
+// kWsMaxNp/32 words, wpre: kWsMaxNp/32, sm: 33 ints of shared scratch.
+__device__ void ws_write_out(const SolverArgs& a, int lp, const int32_t* pick, int cnt, uint32_t* bm, int32_t* wpre,
+                             int* sm) {
+  const int t = threadIdx.x;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t, B = a.B, nwords = (np + 31) / 32;
+  for (int w = t; w < nwords; w += blockDim.x) bm[w] = 0u;
+  __syncthreads();
+  for (int e = t; e < cnt; e += blockDim.x) atomicOr(&bm[pick[e] >> 5], 1u << (pick[e] & 31));
+  __syncthreads();
+  bitmap_prefix(bm, nwords, wpre, sm);
+  float* buf = a.Kws + (int64_t)lp * ws_buf_floats(B);
+  double* st_al = reinterpret_cast<double*>(buf + ws_state_off(B));
+  double* st_f = st_al + B;
+  int32_t* st_ix = reinterpret_cast<int32_t*>(st_f + B);
+  for (int e = t; e < cnt; e += blockDim.x) {
+    const int32_t x = pick[e];
+    const int rank = wpre[x >> 5] + __popc(bm[x >> 5] & ((1u << (x & 31)) - 1u));
+    a.ws_tmp[(int64_t)lp * B + e] = x;
+    a.ws[(int64_t)lp * B + rank] = x;
+    st_al[rank] = a.alpha[pd.a_off + x];
+    st_f[rank] = a.f[pd.a_off + x];
+    st_ix[rank] = x;
+  }
+  if (t == 0) a.ws_n[lp] = cnt;
+}
+
+// ------------------------------------------------------------------------------------------
 // a4 selection
-__global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a) {
+__global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t max_outer) {
+  pdl_enter();
   const int lp = blockIdx.x + a.pair_base;
   TraceScope ts_(a, lp, 0);
   if (a.status[lp] != 0) return;
@@ -119,7 +180,6 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a) {
   const double* fl = a.f + pd.a_off;
   const int first = a.outer_iters[lp] == 0;
   int32_t* ws_age = a.ws_tmp + (int64_t)lp * B;  // age order (oldest first)
-  int32_t* ws_idx = a.ws + (int64_t)lp * B;      // sorted by pair-local index
   long long tq = clock64();
   auto mark = [&](int k) {  // GMPSVM_SMO_PHASES: selection sub-phase cycles (thread 0)
     if (a.sel_phase && t == 0) {
@@ -194,21 +254,19 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a) {
   }
   const double gap = fmax - fmin;
   const bool done = (fmin == DBL_MAX) || (fmax == -DBL_MAX) || !(gap >= a.eps);
+  const bool capped = !done && (int64_t)a.outer_iters[lp] >= max_outer;
   if (t == 0) {
     a.gap[lp] = gap;
     if (done) a.status[lp] = 1;
+    else if (capped) a.status[lp] = 2;  // outer-iteration cap (GMPSVM_WARN_MAXITER)
     else a.outer_iters[lp] += 1;
   }
   mark(0);
-  if (done) return;
-  if (np <= B) {  // the whole pair is the working set (unchanged after the first iteration)
-    if (first) {
-      for (int e = t; e < np; e += kWT) {
-        ws_idx[e] = e;
-        ws_age[e] = e;
-      }
-      if (t == 0) a.ws_n[lp] = np;
-    }
+  if (done || capped) return;
+  if (np <= B) {  // the whole pair is the working set (unchanged from here on)
+    for (int e = t; e < np; e += kWT) W.pick[e] = e;
+    __syncthreads();
+    ws_write_out(a, lp, W.pick, np, W.retained, W.wpre, W.boff[0]);
     return;
   }
   const int need = B - keep, need_u = need / 2;
@@ -361,28 +419,8 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a) {
   }
   __syncthreads();
   mark(2);
-  // write the working set: age order, and sorted by index (rank = set bits below it in a
-  // bitmap of the picked indices: per-word prefix popcounts)
   const int cnt = keep + got;
-  const int nwords = (np + 31) / 32;
-  for (int w = t; w < nwords; w += kWT) W.retained[w] = 0u;
-  __syncthreads();
-  if (t < cnt) atomicOr(&W.retained[W.pick[t] >> 5], 1u << (W.pick[t] & 31));
-  __syncthreads();
-  {  // exclusive prefix of the word popcounts (nwords <= 512: 16 per warp... one per thread)
-    int v = t < nwords ? __popc(W.retained[t]) : 0;
-    int tot = 0;
-    const int pre = block_excl_scan_count_thread(v, tot, W.boff[0]);
-    if (t < nwords) W.wpre[t] = pre;
-  }
-  __syncthreads();
-  if (t < cnt) {
-    const int32_t x = W.pick[t];
-    const int rank = W.wpre[x >> 5] + __popc(W.retained[x >> 5] & ((1u << (x & 31)) - 1u));
-    ws_age[t] = x;
-    ws_idx[rank] = x;
-  }
-  if (t == 0) a.ws_n[lp] = cnt;
+  ws_write_out(a, lp, W.pick, cnt, W.retained, W.wpre, W.boff[0]);
   mark(3);
 }
 
@@ -392,6 +430,7 @@ constexpr int kGR = 8;  // tile rows per CTA
 
 __global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
+  pdl_enter();
   TraceScope ts_(a, lp, 1);
   if (a.status[lp] != 0) return;
   const PairDesc pd = a.pairs[lp];
@@ -405,7 +444,7 @@ __global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
   for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
   __syncthreads();
   const int ld = ws_tile_ld(a.B);
-  float* tile = a.Kws + (int64_t)lp * a.B * ld;
+  float* tile = a.Kws + (int64_t)lp * ws_buf_floats(a.B);
   const int r1 = min(wn, r0 + kGR);
   constexpr int M = (kGR * kWMaxB + 255) / 256;  // loads per thread, all in flight
   float v[M];
@@ -428,7 +467,7 @@ __global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
 
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
-size_t ws_smo_smem(int B) { return (size_t)B * ws_tile_ld(B) * 4 + (size_t)B * 8 + 256; }
+size_t ws_smo_smem(int B) { return ws_buf_floats(B) * 4 + (size_t)B * 8 + 256; }
 
 __device__ __forceinline__ float lds_f32(uint32_t addr) {
   float v;
@@ -478,6 +517,7 @@ __device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
 template <int E>
 __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
+  pdl_wait();  // the f-update is released when the local solve ends (below)
   TraceScope ts_(a, lp, 2);
   if (a.status[lp] != 0) return;
   extern __shared__ __align__(16) unsigned char mdyn[];
@@ -486,49 +526,33 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   const int B = a.B, wn = a.ws_n[lp], ld = ws_tile_ld(B);
   uint32_t kws;  // K_ws,ws tile, row stride ld (opaque: keeps the shared window base out of the loop)
   asm volatile("mov.u32 %0, %1;" : "=r"(kws) : "r"(smem_addr(mdyn)));
-  const uint32_t als = kws + (uint32_t)B * ld * 4;               // alpha of the working set
-  const uint32_t bar = als + (uint32_t)B * 8;                    // mbarrier of the bulk copy
+  const uint32_t als = kws + (uint32_t)ws_state_off(B) * 4;     // alpha of the working set (state)
+  const uint32_t fst = als + (uint32_t)B * 8;                     // f (state)
+  const uint32_t ixs = fst + (uint32_t)B * 8;                     // index (state)
+  const uint32_t a0s = ixs + (uint32_t)((B + 3) & ~3) * 4;        // alpha at entry
+  const uint32_t bar = a0s + (uint32_t)B * 8;                     // mbarrier of the bulk copies
   const long long t_entry = clock64();
-  // bulk copy of the tile rows [0, wn) into shared memory
-  const uint32_t bytes = (uint32_t)wn * ld * 4;  // ld % 4 == 0: a multiple of 16
+  // bulk copies: tile rows [0, wn) and the state block (alpha, f, index) written by the selection
+  const uint32_t tbytes = (uint32_t)wn * ld * 4;  // ld % 4 == 0: multiples of 16
+  const uint32_t sbytes = (uint32_t)B * 16 + (uint32_t)((B + 3) & ~3) * 4;
   if (lane == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-    const char* src = reinterpret_cast<const char*>(a.Kws + (int64_t)lp * B * ld);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(tbytes + sbytes) : "memory");
+    const char* src = reinterpret_cast<const char*>(a.Kws + (int64_t)lp * ws_buf_floats(B));
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(als),
+                 "l"(src + ws_state_off(B) * 4), "r"(sbytes), "r"(bar)
+                 : "memory");
     constexpr uint32_t kChunk = 32768;
-    for (uint32_t o = 0; o < bytes; o += kChunk) {
-      const uint32_t n = bytes - o < kChunk ? bytes - o : kChunk;
+    for (uint32_t o = 0; o < tbytes; o += kChunk) {
+      const uint32_t n = tbytes - o < kChunk ? tbytes - o : kChunk;
       asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                        kws + o),
                    "l"(src + o), "r"(n), "r"(bar)
                    : "memory");
     }
   }
-  __syncwarp();
-  // per-row state: lane owns positions lane + 32 q (the working set sorted by index)
   const double C = a.C, eps = a.eps, ratio = a.local_ratio;
-  const int32_t* ws = a.ws + (int64_t)lp * B;
-  int32_t idx[E];
-  double f[E];
-  uint32_t umask = 0u, lmask = 0u, ypos = 0u, vmask = 0u;
-#pragma unroll
-  for (int q = 0; q < E; ++q) {
-    const int e = lane + 32 * q;
-    const bool valid = e < wn;
-    idx[q] = valid ? ws[e] : INT_MAX;
-    const int y = (valid && idx[q] < pd.n_s) ? 1 : -1;
-    const double al = valid ? a.alpha[pd.a_off + idx[q]] : 0.0;
-    f[q] = valid ? a.f[pd.a_off + idx[q]] : 0.0;
-    if (valid) {
-      sts_f64(als + e * 8, al);
-      vmask |= 1u << q;
-      if (y > 0) ypos |= 1u << q;
-      if (in_u(y, al, C)) umask |= 1u << q;
-      if (in_l(y, al, C)) lmask |= 1u << q;
-    }
-  }
-  const long long t_state = clock64();
   {
     uint32_t done = 0;
     do {
@@ -538,6 +562,29 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
           : "r"(bar)
           : "memory");
     } while (!done);
+  }
+  const long long t_state = clock64();
+  // per-row state: lane owns positions lane + 32 q (the working set sorted by index)
+  int32_t idx[E];
+  double f[E];
+  uint32_t umask = 0u, lmask = 0u, ypos = 0u, vmask = 0u;
+#pragma unroll
+  for (int q = 0; q < E; ++q) {
+    const int e = lane + 32 * q;
+    const bool valid = e < wn;
+    int32_t ix = INT_MAX;
+    if (valid) asm volatile("ld.shared.s32 %0, [%1];" : "=r"(ix) : "r"(ixs + e * 4));
+    idx[q] = ix;
+    const int y = (valid && ix < pd.n_s) ? 1 : -1;
+    const double al = valid ? lds_f64(als + e * 8) : 0.0;
+    f[q] = valid ? lds_f64(fst + e * 8) : 0.0;
+    if (valid) {
+      sts_f64(a0s + e * 8, al);
+      vmask |= 1u << q;
+      if (y > 0) ypos |= 1u << q;
+      if (in_u(y, al, C)) umask |= 1u << q;
+      if (in_l(y, al, C)) lmask |= 1u << q;
+    }
   }
   float kd[E];
 #pragma unroll
@@ -670,12 +717,13 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
     markp(3);
   }
   __syncwarp();
+  pdl_trigger();
 #pragma unroll
   for (int q = 0; q < E; ++q) {
     const int e = lane + 32 * q;
     if ((vmask >> q) & 1u) {
       const double al = lds_f64(als + e * 8);
-      const double a0 = a.alpha[pd.a_off + idx[q]];
+      const double a0 = lds_f64(a0s + e * 8);
       a.dcoef[(int64_t)lp * B + e] = (al - a0) * (((ypos >> q) & 1u) ? 1.0 : -1.0);
       a.alpha[pd.a_off + idx[q]] = al;
     }
@@ -693,40 +741,171 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
 }
 
 // ------------------------------------------------------------------------------------------
+// a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij over the pair (Alg 2 line 11,
+// Eq 8).  HBM-bound GEMV over the kernel-matrix rows of the working set: a CTA owns 32 column
+// quads (128 columns) of the pair's two class segments, its 8 warps split the rows (8 float4
+// loads in flight per thread), FP64 accumulation, partial sums combined in a fixed order.  With
+// set_cond, block (0,0) sets the graph loop condition: continue while a pair of the launch is
+// active (the selection of this iteration has set the status).
+constexpr int kFW = 8;         // warps per f-update CTA
+constexpr int kFT = kFW * 32;  // threads
+
+struct WFup {
+  double coef[kWMaxB];
+  const float4* rowp[kWMaxB];
+  double red[kFW][32][4];
+  int scan[33];
+};
+
+__global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraphConditionalHandle h, int set_cond) {
+  pdl_enter();
+  const int lp = blockIdx.x + a.pair_base;
+  TraceScope ts_(a, lp, 3);
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  if (blockIdx.x == 0 && blockIdx.y == 0 && t == 0) {
+    bool more = false;
+    for (int i = 0; i < (int)gridDim.x; ++i) more = more || a.status[a.pair_base + i] == 0;
+    if (set_cond) {
+      cudaGraphSetConditional(h, more ? 1u : 0u);
+      a.body_iters[a.pair_base] += 1;
+    }
+  }
+  if (a.status[lp] != 0) return;
+  __shared__ WFup F;
+  const PairDesc pd = a.pairs[lp];
+  const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;
+  const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;
+  const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
+  const int64_t q0 = (int64_t)blockIdx.y * 32;
+  if (q0 >= nq) return;
+  const int B = a.B, wn = a.ws_n[lp];
+  const int32_t* ws = a.ws + (int64_t)lp * B;
+  const double* dc = a.dcoef + (int64_t)lp * B;
+  int nnz = 0;
+  {
+    const double c = t < wn ? dc[t] : 0.0;
+    const bool nz = c != 0.0;
+    int tot = 0;
+    const int pos = block_excl_scan(nz, tot, F.scan);
+    if (nz) {
+      F.coef[pos] = c;
+      F.rowp[pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, ws[t]) * a.ldk);
+    }
+    nnz = tot;
+  }
+  __syncthreads();
+  if (nnz == 0) return;
+  const int64_t qi = q0 + lane;
+  const bool okq = qi < nq;
+  const int64_t gq = !okq ? 0 : (qi < nq1 ? q1b + qi : q2b + (qi - nq1));
+  double acc[4] = {0.0, 0.0, 0.0, 0.0};
+  int r = warp;
+  for (; r + 7 * kFW < nnz; r += 8 * kFW) {
+    float4 v[8];
+#pragma unroll
+    for (int rr = 0; rr < 8; ++rr) v[rr] = okq ? __ldg(F.rowp[r + rr * kFW] + gq) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int rr = 0; rr < 8; ++rr) {
+      const double cv = F.coef[r + rr * kFW];
+      acc[0] = fma(cv, (double)v[rr].x, acc[0]);
+      acc[1] = fma(cv, (double)v[rr].y, acc[1]);
+      acc[2] = fma(cv, (double)v[rr].z, acc[2]);
+      acc[3] = fma(cv, (double)v[rr].w, acc[3]);
+    }
+  }
+  for (; r < nnz; r += kFW) {
+    const float4 v0 = okq ? __ldg(F.rowp[r] + gq) : make_float4(0.f, 0.f, 0.f, 0.f);
+    const double cv = F.coef[r];
+    acc[0] = fma(cv, (double)v0.x, acc[0]);
+    acc[1] = fma(cv, (double)v0.y, acc[1]);
+    acc[2] = fma(cv, (double)v0.z, acc[2]);
+    acc[3] = fma(cv, (double)v0.w, acc[3]);
+  }
+#pragma unroll
+  for (int c = 0; c < 4; ++c) F.red[warp][lane][c] = acc[c];
+  __syncthreads();
+  if (t < 128) {  // column: component t & 3 of quad t >> 2
+    const int l = t >> 2, c = t & 3;
+    const int64_t qj = q0 + l;
+    if (qj < nq) {
+      const bool seg1 = qj < nq1;  // a boundary quad shared by adjacent classes is owned once per segment
+      const int64_t g = (seg1 ? q1b + qj : q2b + (qj - nq1)) * 4 + c;
+      int64_t j = -1;
+      if (seg1) j = (g >= pd.off_s && g < pd.off_s + pd.n_s) ? g - pd.off_s : -1;
+      else j = (g >= pd.off_t && g < pd.off_t + pd.n_t) ? pd.n_s + (g - pd.off_t) : -1;
+      if (j >= 0) {
+        double sum = 0.0;
+#pragma unroll
+        for (int w = 0; w < kFW; ++w) sum += F.red[w][l][c];
+        a.f[pd.a_off + j] += sum;
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
 bool ws_solve_supported(int B, int64_t np_max) {
   static const bool off = getenv("GMPSVM_WSOLVE") && std::string(getenv("GMPSVM_WSOLVE")) == "0";
   return !off && B >= 2 && B <= kWMaxB && np_max <= kWMaxNp;
 }
 
-size_t ws_tile_floats(int B) { return (size_t)B * ws_tile_ld(B); }
+size_t ws_tile_floats(int B) { return ws_buf_floats(B); }
 
-void launch_ws_solve(const SolverArgs& a, int P, cudaStream_t st) {
-  const size_t sel_dyn = (size_t)kWMaxNp * 9;
-  const size_t smo_dyn = ws_smo_smem(a.B);
+
+
+static bool pdl_enabled() {
+  static const bool on = !(getenv("GMPSVM_PDL") && std::string(getenv("GMPSVM_PDL")) == "0");
+  return on;
+}
+
+template <typename... KArgs, typename... Args>
+static void launch_pdl(void (*kern)(KArgs...), dim3 g, dim3 b, size_t smem, cudaStream_t st, Args... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = g;
+  cfg.blockDim = b;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  GM_CUDA(cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...));
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+}
+
+static void ws_configure() {
   static bool configured = false;
-  if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(ws_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sel_dyn));
-    const int mx = (int)ws_smo_smem(kWMaxB);
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<5>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-    configured = true;
-  }
-  GM_LAUNCH(ws_select_kernel, dim3(P), dim3(kWT), sel_dyn, st, a);
-  GM_LAUNCH(ws_gather_kernel, dim3(P, (unsigned)ceil_div(a.B, kGR)), dim3(256), 0, st, a);
+  if (configured) return;
+  GM_CUDA(cudaFuncSetAttribute(ws_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)((size_t)kWMaxNp * 9)));
+  const int mx = (int)ws_smo_smem(kWMaxB);
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<5>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  configured = true;
+}
+
+void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int set_cond,
+                         int64_t max_outer, cudaStream_t st, bool chained) {
+  ws_configure();
+  const size_t sel_dyn = (size_t)kWMaxNp * 9, smo_dyn = ws_smo_smem(a.B);
+  if (chained) launch_pdl(ws_select_kernel, dim3(P), dim3(kWT), sel_dyn, st, a, max_outer);
+  else GM_LAUNCH(ws_select_kernel, dim3(P), dim3(kWT), sel_dyn, st, a, max_outer);
+  launch_pdl(ws_gather_kernel, dim3(P, (unsigned)ceil_div(a.B, kGR)), dim3(256), 0, st, a);
   switch ((a.B + 31) / 32) {
-    case 1: GM_LAUNCH(ws_smo_kernel<1>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 2: GM_LAUNCH(ws_smo_kernel<2>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 3: GM_LAUNCH(ws_smo_kernel<3>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 4: GM_LAUNCH(ws_smo_kernel<4>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 5: GM_LAUNCH(ws_smo_kernel<5>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 6: GM_LAUNCH(ws_smo_kernel<6>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    default: GM_LAUNCH(ws_smo_kernel<7>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 1: launch_pdl(ws_smo_kernel<1>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 2: launch_pdl(ws_smo_kernel<2>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 3: launch_pdl(ws_smo_kernel<3>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 4: launch_pdl(ws_smo_kernel<4>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 5: launch_pdl(ws_smo_kernel<5>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 6: launch_pdl(ws_smo_kernel<6>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    default: launch_pdl(ws_smo_kernel<7>, dim3(P), dim3(32), smo_dyn, st, a); break;
   }
+  launch_pdl(ws_fupdate_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, 128)), dim3(kFT), 0, st, a, h, set_cond);
 }
 
 }  // namespace gmpsvm
