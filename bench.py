@@ -302,7 +302,7 @@ def main():
     ap.add_argument("--impl", default="gmpsvm", choices=["gmpsvm", "reference"])
     ap.add_argument("--config", default="mnist")
     ap.add_argument("--eps", type=float, default=1e-3)
-    ap.add_argument("--ws-size", dest="ws_size", type=int, default=224)
+    ap.add_argument("--ws-size", dest="ws_size", type=int, default=192)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:

@@ -35,7 +35,7 @@ constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
 constexpr int64_t kPredictChunk = 32768;
 constexpr int kMaxStreams = 48;    // concurrent pair groups in the solver
 constexpr int kDefaultStreams = 8; // default pair groups (hardware queues: CUDA_DEVICE_MAX_CONNECTIONS)
-constexpr int kDefaultB = 224;     // working-set rows: K_ws,ws stays in shared memory (B <= 224)
+constexpr int kDefaultB = 192;     // working-set rows (tuned on MNIST-shaped data; the tile of K_ws,ws stays in shared memory for B <= 224)
 constexpr int kChunk = 2;          // outer iterations per issued chunk
 
 struct DeviceGuard {
@@ -85,15 +85,32 @@ size_t device_total_mem(int dev) {
 // Per-device pool of non-blocking streams for the concurrent pair groups.
 std::mutex g_pool_mu;
 std::vector<cudaStream_t> g_pools[64];
+// The solver's streams have the highest priority: when the kernel-value waves share the GPU with
+// the solver (overlap mode), the block scheduler dispatches solver CTAs first.
 const std::vector<cudaStream_t>& stream_pool(int dev) {
   std::lock_guard<std::mutex> lk(g_pool_mu);
   auto& v = g_pools[dev];
+  int least = 0, greatest = 0;
+  if (v.size() < (size_t)kMaxStreams) GM_CUDA(cudaDeviceGetStreamPriorityRange(&least, &greatest));
   while ((int)v.size() < kMaxStreams) {
     cudaStream_t s;
-    GM_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    GM_CUDA(cudaStreamCreateWithPriority(&s, cudaStreamNonBlocking, greatest));
     v.push_back(s);
   }
   return v;
+}
+
+// Low-priority stream for the kernel-value waves of the overlap mode.
+cudaStream_t krow_stream(int dev) {
+  static std::mutex mu;
+  static cudaStream_t s[64] = {};
+  std::lock_guard<std::mutex> lk(mu);
+  if (!s[dev]) {
+    int least = 0, greatest = 0;
+    GM_CUDA(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+    GM_CUDA(cudaStreamCreateWithPriority(&s[dev], cudaStreamNonBlocking, least));
+  }
+  return s[dev];
 }
 
 // Timing-free events created on demand and destroyed with the pool.
@@ -230,6 +247,25 @@ T* pinned_scratch(size_t count) {
 }
 
 enum { PH_STAGE, PH_KERNEL, PH_SELECT, PH_SUB, PH_FUP, PH_FIN, PH_DEC, PH_COUPLE, PH_D2H, PH_SOLVER, PH_N };
+
+// default solver structure (device-driven graph), i.e. neither GMPSVM_SOLVER=fused nor =streams
+static bool graph_solver_default(int B) {
+  static const bool streams = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "streams";
+  return !fused_solver_enabled(B) && !streams;
+}
+
+// timing events of the overlap mode's kernel-value waves (destroyed with the scope)
+struct TimedEvents {
+  cudaEvent_t a = nullptr, b = nullptr;
+  TimedEvents() {
+    GM_CUDA(cudaEventCreate(&a));
+    GM_CUDA(cudaEventCreate(&b));
+  }
+  ~TimedEvents() {
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+  }
+};
 
 struct PhaseTimer {
   cudaStream_t st;
@@ -497,6 +533,26 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   if (hbad) throw Error(GMPSVM_EINVAL, "X contains non-finite values");
   tm.mark(PH_STAGE);
   HT("stage1");
+  // class means of the staged rows: pairs of the closest classes are expected to need the most
+  // solver work, so they get their kernel values first (overlap mode) and their own branches
+  std::vector<double> cdist;  // squared distance of the class means, per pair index (tc path)
+  if (use_tc) {
+    DevBuf<float> d_mu((size_t)k * d_pad, st);
+    launch_class_means(Xhi.get(), d_pad, d_off.get(), k, d_mu.get(), st);
+    std::vector<float> mu((size_t)k * d_pad);
+    GM_CUDA(cudaMemcpyAsync(mu.data(), d_mu.get(), mu.size() * 4, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaStreamSynchronize(st));
+    cdist.assign((size_t)k * (k - 1) / 2, 0.0);
+    for (int s0 = 0; s0 < k; ++s0)
+      for (int t0 = s0 + 1; t0 < k; ++t0) {
+        double acc = 0.0;
+        for (int f = 0; f < d_pad; ++f) {
+          const double df = (double)mu[(size_t)s0 * d_pad + f] - mu[(size_t)t0 * d_pad + f];
+          acc += df * df;
+        }
+        cdist[pair_index(s0, t0, k)] = acc;
+      }
+  }
 
   // ---------------- pairs to train
   const int P = k * (k - 1) / 2;
@@ -521,9 +577,13 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       ps[pair_index(s, t, k)] = s;
       pt[pair_index(s, t, k)] = t;
     }
-  // largest pairs first: they start first and share streams with pairs of similar cost
-  std::stable_sort(pids.begin(), pids.end(),
-                   [&](int x, int y) { return cc[ps[x]] + cc[pt[x]] > cc[ps[y]] + cc[pt[y]]; });
+  // largest pairs first (closest class means first on the tensor-core path, see above): they
+  // start first and share streams with pairs of similar cost
+  if (!cdist.empty())
+    std::stable_sort(pids.begin(), pids.end(), [&](int x, int y) { return cdist[x] < cdist[y]; });
+  else
+    std::stable_sort(pids.begin(), pids.end(),
+                     [&](int x, int y) { return cc[ps[x]] + cc[pt[x]] > cc[ps[y]] + cc[pt[y]]; });
   std::vector<PairDesc> hp(Pl);
   int64_t tot = 0, np_max = 0;
   for (int i = 0; i < Pl; ++i) {
@@ -561,16 +621,82 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   HT("k_alloc");
   std::vector<int2> tiles;
   DevBuf<int2> d_tiles;
+  // Overlap mode (tensor-core FULL_K path with the device-driven default solver): the kernel
+  // matrix is computed in waves on a low-priority stream, wave w holding the tiles first needed
+  // by the w-th pair (pair order above); each pair's solver branch starts as soon as the waves
+  // covering its class blocks (s,s), (s,t), (t,t) are done, so the solver of the first pairs runs
+  // while the kernel values of the others are still being computed.  Tiles no trained pair needs
+  // (pair subsets, multi-GPU shards) are skipped.
+  // Opt-in (GMPSVM_OVERLAP=1): measured slower on MNIST-shaped data (B200: 62 vs 57 ms train +
+  // predict) -- the waves' tensor/HBM load stretches the solver's latency-bound chain more than
+  // the overlap saves.
+  static const bool overlap_env = getenv("GMPSVM_OVERLAP") && std::string(getenv("GMPSVM_OVERLAP")) == "1";
+  const bool overlap = overlap_env && use_tc && graph_solver_default(B) && ws_solve_supported(B, np_max);
+  cudaStream_t kst = krow_stream(opt.device);
+  TimedEvents kev;
+  cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
+  std::vector<int> wave_off;     // tile range of wave w: [wave_off[w], wave_off[w + 1])
+  std::vector<int> ready_wave;   // per pair position: the wave after which its kernel values are complete
   if (use_tc) {
     tiles = krow_tc_tiles(n);
+    if (overlap) {
+      const int INF = INT_MAX;
+      std::vector<int> minpos(k, INF);  // first position of a pair containing class c
+      std::vector<int> pos((size_t)k * k, INF);
+      for (int i = 0; i < Pl; ++i) {
+        minpos[hp[i].s] = std::min(minpos[hp[i].s], i);
+        minpos[hp[i].t] = std::min(minpos[hp[i].t], i);
+        pos[(size_t)hp[i].s * k + hp[i].t] = i;
+      }
+      auto cls = [&](int64_t r) { return (int)(std::upper_bound(coff.begin(), coff.end(), r) - coff.begin()) - 1; };
+      std::vector<int> tw(tiles.size());
+      std::vector<int> blockmax((size_t)k * k, -1);
+      for (size_t ti = 0; ti < tiles.size(); ++ti) {
+        const int64_t r0 = (int64_t)tiles[ti].x * kKrowTileRows, c0 = (int64_t)tiles[ti].y * kKrowTileRows;
+        const int ra = cls(r0), rb = cls(std::min<int64_t>(n, r0 + kKrowTileRows) - 1);
+        const int ca = cls(c0), cb = cls(std::min<int64_t>(n, c0 + kKrowTileRows) - 1);
+        int w = INF;
+        for (int a0 = ra; a0 <= rb; ++a0)
+          for (int b0 = ca; b0 <= cb; ++b0) {
+            const int lo = std::min(a0, b0), hi = std::max(a0, b0);
+            w = std::min(w, lo == hi ? minpos[lo] : pos[(size_t)lo * k + hi]);
+          }
+        tw[ti] = w;
+        if (w == INF) continue;
+        for (int a0 = ra; a0 <= rb; ++a0)
+          for (int b0 = ca; b0 <= cb; ++b0) {
+            int& m = blockmax[(size_t)std::min(a0, b0) * k + std::max(a0, b0)];
+            m = std::max(m, w);
+          }
+      }
+      std::vector<int> order(tiles.size());
+      for (size_t ti = 0; ti < tiles.size(); ++ti) order[ti] = (int)ti;
+      std::stable_sort(order.begin(), order.end(), [&](int x, int y) { return tw[x] < tw[y]; });
+      std::vector<int2> sorted;
+      sorted.reserve(tiles.size());
+      wave_off.assign(Pl + 1, 0);
+      for (int ti : order) {
+        if (tw[ti] == INF) break;
+        sorted.push_back(tiles[ti]);
+        wave_off[tw[ti] + 1] += 1;
+      }
+      for (int w = 0; w < Pl; ++w) wave_off[w + 1] += wave_off[w];
+      tiles.swap(sorted);
+      ready_wave.assign(Pl, -1);
+      for (int i = 0; i < Pl; ++i) {
+        const int s0 = hp[i].s, t0 = hp[i].t;
+        ready_wave[i] = std::max(std::max(blockmax[(size_t)s0 * k + s0], blockmax[(size_t)s0 * k + t0]),
+                                 blockmax[(size_t)t0 * k + t0]);
+      }
+    }
     new (&d_tiles) DevBuf<int2>(tiles.size(), st);
     GM_CUDA(cudaMemcpyAsync(d_tiles.get(), tiles.data(), tiles.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
   }
   tm.mark(PH_KERNEL);
-  if (use_tc)
+  if (use_tc && !overlap)
     launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, K.get(),
                    ldk, st);
-  else if (full_k)
+  else if (full_k && !use_tc)
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   tm.mark(PH_KERNEL);
   HT("krow_launched");
@@ -745,13 +871,33 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       const int m = Pl / nbr, r = Pl % nbr;  // the last r branches take m + 1 pairs
       for (int b = 0; b < nbr; ++b) bb[b + 1] = bb[b] + m + (b >= nbr - r ? 1 : 0);
     }
+    std::vector<cudaEvent_t> ev_wave(Pl, nullptr);
+    if (overlap) {  // kernel-value waves on the low-priority stream, one event per wave
+      cudaEvent_t ev_staged = evp.get();
+      GM_CUDA(cudaEventRecord(ev_staged, st));
+      GM_CUDA(cudaStreamWaitEvent(kst, ev_staged, 0));
+      GM_CUDA(cudaEventRecord(ev_k0, kst));
+      for (int w = 0; w < Pl; ++w) {
+        const int cnt = wave_off[w + 1] - wave_off[w];
+        if (cnt > 0)
+          launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get() + wave_off[w], cnt, norms.get(), n, gamma,
+                         K.get(), ldk, kst);
+        ev_wave[w] = evp.get();
+        GM_CUDA(cudaEventRecord(ev_wave[w], kst));
+      }
+      GM_CUDA(cudaEventRecord(ev_k1, kst));
+    }
     const uint64_t l0 = g_launches.load();
     GM_CUDA(cudaGraphCreate(&gg.graph, 0));
     cudaStream_t cs = pool.back();
     for (int br = 0; br < nbr; ++br) {
       const int i = bb[br], gn = bb[br + 1] - bb[br];
       int64_t npi = 0;
-      for (int j = bb[br]; j < bb[br + 1]; ++j) npi = std::max<int64_t>(npi, hp[j].n_s + hp[j].n_t);
+      int rw = -1;
+      for (int j = bb[br]; j < bb[br + 1]; ++j) {
+        npi = std::max<int64_t>(npi, hp[j].n_s + hp[j].n_t);
+        if (overlap) rw = std::max(rw, ready_wave[j]);
+      }
       cudaGraphConditionalHandle h;
       GM_CUDA(cudaGraphConditionalHandleCreate(&h, gg.graph, 1, cudaGraphCondAssignDefault));
       cudaGraphNodeParams cp = {};
@@ -759,8 +905,13 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       cp.conditional.handle = h;
       cp.conditional.type = cudaGraphCondTypeWhile;
       cp.conditional.size = 1;
-      cudaGraphNode_t wnode;
-      GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, nullptr, 0, &cp));
+      cudaGraphNode_t wnode, wait_node;
+      if (rw >= 0) {  // the branch starts when the waves covering its pairs' class blocks are done
+        GM_CUDA(cudaGraphAddEventWaitNode(&wait_node, gg.graph, nullptr, 0, ev_wave[rw]));
+        GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, &wait_node, 1, &cp));
+      } else {
+        GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, nullptr, 0, &cp));
+      }
       SolverArgs ag = a;
       ag.pair_base = i;
       const bool wsp = !rc && ws_solve_supported(Bw, npi);
@@ -831,6 +982,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     GM_CUDA(cudaEventRecord(ev, pool[g]));
     GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
   }
+  if (overlap) GM_CUDA(cudaStreamWaitEvent(st, ev_k1, 0));  // every kernel-value wave (K is reused by the next call)
   tm.mark(PH_SOLVER);
   HT("solver_loop");
   bool cap_hit = false;
@@ -990,7 +1142,13 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
 
   gmpsvm_train_stats& s = mdl->stats;
   s.t_stage_ms = tm.ms(PH_STAGE);
-  s.t_kernel_ms = tm.ms(PH_KERNEL);
+  if (overlap) {  // span of the kernel-value waves (they share the GPU with the solver)
+    float x = 0.f;
+    GM_CUDA(cudaEventElapsedTime(&x, ev_k0, ev_k1));
+    s.t_kernel_ms = x;
+  } else {
+    s.t_kernel_ms = tm.ms(PH_KERNEL);
+  }
   s.t_select_ms = tm.ms(PH_SELECT);
   s.t_subproblem_ms = tm.ms(PH_SUB);
   s.t_fupdate_ms = tm.ms(PH_FUP);

@@ -33,6 +33,9 @@ size_t krow_tc_scratch_bytes(int64_t n, int d);
 void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, float* hi, float* lo, float* norms,
                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
 std::vector<int2> krow_tc_tiles(int64_t n);
+constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
+// per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
+void launch_class_means(const float* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
 void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float* K, int64_t ldk, cudaStream_t st);
 void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,

@@ -356,6 +356,30 @@ void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, fl
             n_pad, d_pad);
 }
 
+// Per-class means of the staged (centred, class-sorted) rows, from the TF32 hi part: used only to
+// order the pairs for the overlap of the kernel-value waves with the solver (engine.cu).
+__global__ void class_means_kernel(const float* hi, int d_pad, const int64_t* coff, float* mu) {
+  const int c = blockIdx.y, f = blockIdx.x * 32 + threadIdx.x;
+  const int64_t r0 = coff[c], r1 = coff[c + 1];
+  float s = 0.f;
+  if (f < d_pad)
+    for (int64_t r = r0 + threadIdx.y; r < r1; r += 8) s += hi[r * d_pad + f];
+  __shared__ float red[8][33];
+  red[threadIdx.y][threadIdx.x] = s;
+  __syncthreads();
+  if (threadIdx.y == 0 && f < d_pad) {
+    float t = 0.f;
+#pragma unroll
+    for (int y = 0; y < 8; ++y) t += red[y][threadIdx.x];
+    mu[(int64_t)c * d_pad + f] = r1 > r0 ? t / (float)(r1 - r0) : 0.f;
+  }
+}
+
+void launch_class_means(const float* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st) {
+  GM_LAUNCH(class_means_kernel, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st, hi, d_pad, coff,
+            mu);
+}
+
 // Tiles (bi, bj) of 128 x 128 with at least one entry r <= c, in blocked order (16 x 16 tiles)
 // so a wave of CTAs reuses its operand tiles from L2.
 std::vector<int2> krow_tc_tiles(int64_t n) {

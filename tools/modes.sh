@@ -1,6 +1,3 @@
-python -m pytest tests -m gpu -x -q 2>&1 | tail -3
-python tools/sweep.py "" "ws_size=192" 2>&1 | grep total
-GMPSVM_UNROLL=1 python tools/sweep.py "" 2>&1 | grep total
-GMPSVM_UNROLL=4 python tools/sweep.py "" 2>&1 | grep total
-GMPSVM_SOLVER=streams python tools/sweep.py "" 2>&1 | grep total
-GMPSVM_TRACE=32 python tools/sweep.py "" 2>&1 | grep trace | tail -1
+python tools/sweep.py "" "ws_size=160" "ws_size=176" "ws_size=208" 2>&1 | grep total
+for r in 0.05 0.15 0.2; do echo ratio $r; GMPSVM_LOCAL_RATIO=$r python tools/sweep.py "" 2>&1 | grep total; done
+python bench.py --steps 5 --warmup 3 > gpurun_out/bench2.json 2> gpurun_out/bench2.err; cat gpurun_out/bench2.json
