@@ -314,7 +314,7 @@ DevModel::~DevModel() {
   } catch (...) {
   }
   if (ls && last_use) cudaStreamWaitEvent(ls, last_use, 0);
-  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B};
+  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B, SvHi, SvLo, nsvc, mu};
   for (void* p : ptrs)
     if (p) {
       if (ls) cudaFreeAsync(p, ls);
@@ -424,6 +424,20 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   GM_CUDA(cudaMemcpyAsync(dm->B, m.B.data(), P * 8, cudaMemcpyHostToDevice, st));
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
+  dm->h_items = items;
+  // tensor-core decision values: centre = mean of the SV rows, TF32 hi/lo split of the SV slots
+  static const bool dec_simt = getenv("GMPSVM_DEC") && std::string(getenv("GMPSVM_DEC")) == "simt";
+  dm->tc = !dec_simt && krow_use_tc() && dm->km1_pad <= dec_tc_max_km1();
+  if (dm->tc) {
+    dm->dpt = krow_tc_d_pad(m.d);
+    dm->mu = dev_alloc<float>(m.d, st);
+    dm->SvHi = dev_alloc<float>((size_t)dm->nsv_pad * dm->dpt, st);
+    dm->SvLo = dev_alloc<float>((size_t)dm->nsv_pad * dm->dpt, st);
+    dm->nsvc = dev_alloc<float>(dm->nsv_pad, st);
+    launch_gather_col_mean(rows, m.d, d_src.get(), dm->nsv_pad, nsv, dm->mu, st);
+    launch_split_tf32_mu(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, dm->SvHi, dm->SvLo, dm->nsvc, dm->nsv_pad, dm->dpt,
+                         st);
+  }
   GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
   GM_CUDA(cudaEventRecord(dm->last_use, st));
   GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
@@ -1217,7 +1231,8 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   const int64_t mc_max = std::min<int64_t>(m, kPredictChunk);
   const int64_t mc_pad = round_up(mc_max, kTile);
   DevBuf<float> xin(opt.inputs_on_device ? 0 : (size_t)mc_max * d, st);
-  DevBuf<float> XtT((size_t)dm.d_pad * mc_pad, st), nt(mc_pad, st);
+  DevBuf<float> XtT(dm.tc ? 0 : (size_t)dm.d_pad * mc_pad, st), nt(mc_pad, st);
+  DevBuf<float> Xhi(dm.tc ? (size_t)mc_pad * dm.dpt : 0, st), Xlo(dm.tc ? (size_t)mc_pad * dm.dpt : 0, st);
   DevBuf<float> part((size_t)dm.n_items * mc_pad * dm.km1_pad, st);
   DevBuf<double> dec_buf(opt.inputs_on_device ? 0 : (size_t)mc_max * P, st);
   DevBuf<double> prob_buf((opt.inputs_on_device || !prob_out) ? 0 : (size_t)mc_max * k, st);
@@ -1233,12 +1248,46 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
       GM_CUDA(cudaMemcpyAsync(xin.get(), src, (size_t)mc * d * 4, cudaMemcpyHostToDevice, st));
       src = xin.get();
     }
-    launch_stage_features(src, mc, d, nullptr, XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(), st);
+    DevBuf<int2> d_dtiles;
+    DevBuf<int32_t> d_uoff, d_uitem;
+    int n_units = 0;
+    if (dm.tc) {
+      launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
+      launch_split_tf32_mu(src, mc, d, nullptr, dm.mu, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
+      // work units: (item, test tile), test tiles fastest; unit = the item's SV tiles for that test tile
+      const int ntt = (int)(mcp / kTile);
+      std::vector<int2> dt;
+      std::vector<int32_t> uoff(1, 0), uitem;
+      for (int it = 0; it < dm.n_items; ++it)
+        for (int tt = 0; tt < ntt; ++tt) {
+          for (int sv = dm.h_items[it].tile_begin; sv < dm.h_items[it].tile_end; ++sv) dt.push_back(make_int2(tt, sv));
+          uoff.push_back((int32_t)dt.size());
+          uitem.push_back(it);
+        }
+      n_units = (int)uitem.size();
+      new (&d_dtiles) DevBuf<int2>(std::max<size_t>(dt.size(), 1), st);
+      new (&d_uoff) DevBuf<int32_t>(uoff.size(), st);
+      new (&d_uitem) DevBuf<int32_t>(std::max<size_t>(uitem.size(), 1), st);
+      if (!dt.empty())
+        GM_CUDA(cudaMemcpyAsync(d_dtiles.get(), dt.data(), dt.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
+      GM_CUDA(cudaMemcpyAsync(d_uoff.get(), uoff.data(), uoff.size() * 4, cudaMemcpyHostToDevice, st));
+      if (!uitem.empty())
+        GM_CUDA(cudaMemcpyAsync(d_uitem.get(), uitem.data(), uitem.size() * 4, cudaMemcpyHostToDevice, st));
+    } else {
+      launch_stage_features(src, mc, d, nullptr, XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(), st);
+    }
     tm.mark(PH_STAGE);
     double* dec_d = opt.inputs_on_device ? (dec_out ? dec_out + i0 * P : dec_tmp.get()) : dec_buf.get();
     tm.mark(PH_DEC);
-    launch_dec_contract(XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef, dm.km1, dm.km1_pad,
-                        dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
+    if (dm.tc) {
+      GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
+      if (n_units > 0)
+        launch_dec_tc(Xhi.get(), Xlo.get(), mcp, dm.SvHi, dm.SvLo, dm.nsv_pad, dm.dpt, d_dtiles.get(), d_uoff.get(),
+                      d_uitem.get(), n_units, nt.get(), dm.nsvc, dm.coef, dm.km1, dm.km1_pad, mdl.gamma, part.get(), st);
+    } else {
+      launch_dec_contract(XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef, dm.km1, dm.km1_pad,
+                          dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
+    }
     launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     ps.dec_launches += 1;
     tm.mark(PH_DEC);

@@ -34,6 +34,19 @@ void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, fl
                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
 std::vector<int2> krow_tc_tiles(int64_t n);
 constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
+// split with a given centre mu[d] (prediction: the test rows take the SV centre)
+void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float* hi, float* lo,
+                          float* norms, int64_t n_pad, int d_pad, cudaStream_t st);
+// mu[c] = mean over the rows idx[i] >= 0 (cnt of them) of X[., c]
+void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
+                            cudaStream_t st);
+// a10 on tcgen05 (krow_tc.cu): tiles = (test tile, SV tile) grouped in units [unit_off[u],
+// unit_off[u+1]), unit u writes part[unit_item[u]][row][0..km1_pad) (as launch_dec_contract)
+int dec_tc_max_km1();
+void launch_dec_tc(const float* thi, const float* tlo, int64_t m_pad, const float* shi, const float* slo,
+                   int64_t nsv_pad, int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item,
+                   int n_units, const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma,
+                   float* part, cudaStream_t st);
 // per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
 void launch_class_means(const float* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
 void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,

@@ -31,6 +31,7 @@ constexpr uint32_t kABytes = kTM * kTK * 4;            // 16 KB
 constexpr uint32_t kBBytes = kTN * kTK * 4;            // 16 KB
 constexpr uint32_t kStageBytes = 2 * kABytes + 2 * kBBytes;  // 64 KB
 constexpr uint32_t kTmemCols = 512;  // 3 x 128 hi.hi (k thirds) + 128 hi.lo + lo.hi
+constexpr int kDecMaxKm1 = 32;       // dec_tc: pair columns per SV (k - 1, padded), k <= 33
 
 struct TcSmem {
   // each operand tile 1024-byte aligned (128B swizzle atoms)
@@ -261,6 +262,202 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   }
 }
 
+// ------------------------------------------------------------------------------------------
+// a10 on the tensor cores: decision values dec[x][p] = sum_j coef_{j,p} K(x, sv_j) (+ b_p later)
+// with the same 3xTF32 split / split accumulators as the kernel-value contraction.  A = a 128-row
+// test tile, B = a class-pure 128-SV tile; the epilogue turns the 128 x 128 dot products into
+// kernel values and contracts them with the SV tile's coefficients (each SV of class c feeds the
+// k-1 pairs of c) into per-row FP32 accumulators that live across the SV tiles of a work unit
+// (one test tile x one run of SV tiles of one class); K never leaves the SM.  Persistent CTAs
+// take the units round-robin; unit u covers tiles [unit_off[u], unit_off[u + 1]) of the list.
+template <int KM>
+struct DecTcSmem {
+  alignas(1024) uint8_t stage[kTcStages][kStageBytes];
+  alignas(16) float coefS[2][kTN][KM];
+  alignas(8) uint64_t full[kTcStages];
+  uint64_t empty[kTcStages];
+  uint64_t tmem_full;
+  uint64_t tmem_empty;
+  uint32_t tmem_base;
+};
+
+template <int KM>  // compile-time bound of the pair columns (k - 1 <= KM, KM % 4 == 0)
+__global__ void __launch_bounds__(kTcThreads, 1)
+    dec_tc_kernel(const __grid_constant__ CUtensorMap map_thi, const __grid_constant__ CUtensorMap map_tlo,
+                  const __grid_constant__ CUtensorMap map_shi, const __grid_constant__ CUtensorMap map_slo,
+                  const int2* __restrict__ tiles, const int32_t* __restrict__ unit_off,
+                  const int32_t* __restrict__ unit_item, int n_units, const float* __restrict__ nt,
+                  const float* __restrict__ nsv, const float* __restrict__ coef, int km1, int km1_pad, int nk,
+                  float scale, int64_t m_pad, float* __restrict__ part) {
+  extern __shared__ __align__(1024) uint8_t dsmem[];
+  DecTcSmem<KM>& sm =
+      *reinterpret_cast<DecTcSmem<KM>*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < kTcStages; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], 1);
+    }
+    mbar_init(&sm.tmem_full, 1);
+    mbar_init(&sm.tmem_empty, 4);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&sm.tmem_base)),
+                 "r"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = sm.tmem_base;
+  const int jn = nk < kMainAcc ? nk : kMainAcc;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ---- TMA producer
+      int g = 0;
+      for (int u = blockIdx.x; u < n_units; u += gridDim.x)
+        for (int t = unit_off[u]; t < unit_off[u + 1]; ++t) {
+          const int2 tile = tiles[t];
+          const int r0 = tile.x * kTM, c0 = tile.y * kTN;
+          for (int kb = 0; kb < nk; ++kb, ++g) {
+            const int s = g % kTcStages;
+            if (g >= kTcStages) mbar_wait(&sm.empty[s], ((g / kTcStages) + 1) & 1);
+            uint8_t* st = sm.stage[s];
+            mbar_expect_tx(&sm.full[s], kStageBytes);
+            const int kx = kb * kTK;
+            tma_load_2d(st, &map_thi, kx, r0, &sm.full[s]);
+            tma_load_2d(st + kABytes, &map_tlo, kx, r0, &sm.full[s]);
+            tma_load_2d(st + 2 * kABytes, &map_shi, kx, c0, &sm.full[s]);
+            tma_load_2d(st + 2 * kABytes + kBBytes, &map_slo, kx, c0, &sm.full[s]);
+          }
+        }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---- MMA issuer
+      int g = 0, it = 0;
+      for (int u = blockIdx.x; u < n_units; u += gridDim.x)
+        for (int t = unit_off[u]; t < unit_off[u + 1]; ++t, ++it) {
+          if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          for (int kb = 0; kb < nk; ++kb, ++g) {
+            const int s = g % kTcStages;
+            mbar_wait(&sm.full[s], (g / kTcStages) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            uint8_t* st = sm.stage[s];
+            const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
+            const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
+            const int j = (kb * jn) / nk;
+            const int kb_first = (j * nk + jn - 1) / jn;
+#pragma unroll
+            for (int kk = 0; kk < kTK / 8; ++kk) {
+              const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+              umma_tf32(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
+              umma_tf32(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
+              umma_tf32(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+            }
+            umma_commit(&sm.empty[s]);
+          }
+          umma_commit(&sm.tmem_full);
+        }
+    }
+  } else {  // ---- epilogue: warps 2..5 (TMEM lane quarter warp % 4), thread = one test row
+    const int q = warp & 3, et = threadIdx.x - 64;  // et: 0..127
+    int it = 0;
+    for (int u = blockIdx.x; u < n_units; u += gridDim.x) {
+      float acc[KM];
+#pragma unroll
+      for (int v = 0; v < KM; ++v) acc[v] = 0.f;
+      int64_t r = 0;
+      for (int t = unit_off[u]; t < unit_off[u + 1]; ++t, ++it) {
+        const int2 tile = tiles[t];
+        const int64_t r0 = (int64_t)tile.x * kTM, c0 = (int64_t)tile.y * kTN;
+        r = r0 + q * 32 + lane;
+        // this SV tile's coefficients (double buffer: one barrier per tile)
+        float* cs = &sm.coefS[it & 1][0][0];
+#pragma unroll
+        for (int v = 0; v < KM; ++v) cs[et * KM + v] = v < km1_pad ? coef[(c0 + et) * km1_pad + v] : 0.f;
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        mbar_wait(&sm.tmem_full, it & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        float dot[kTN];
+#pragma unroll
+        for (int ch = 0; ch < kTN / 32; ++ch) {  // one 32-column accumulator slice at a time (registers)
+          const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(ch * 32);
+          uint32_t v[32];
+          tmem_ld32(taddr + kMainAcc * kTN, v);
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj) dot[ch * 32 + jj] = __uint_as_float(v[jj]);
+#pragma unroll
+          for (int a = 0; a < kMainAcc; ++a) {
+            if (a >= nk) break;
+            tmem_ld32(taddr + a * kTN, v);
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+            for (int jj = 0; jj < 32; ++jj) dot[ch * 32 + jj] += __uint_as_float(v[jj]);
+          }
+        }
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+        const float nr = nt[r];
+#pragma unroll
+        for (int j = 0; j < kTN; ++j) {
+          const float d2 = fmaf(-2.f, dot[j], nr + __ldg(nsv + c0 + j));
+          float kv;
+          asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv) : "f"(fmaxf(d2, 0.f) * scale));
+          const float4* cj = reinterpret_cast<const float4*>(cs + j * KM);
+#pragma unroll
+          for (int v4 = 0; v4 < KM / 4; ++v4) {
+            const float4 cv = cj[v4];
+            acc[4 * v4 + 0] = fmaf(kv, cv.x, acc[4 * v4 + 0]);
+            acc[4 * v4 + 1] = fmaf(kv, cv.y, acc[4 * v4 + 1]);
+            acc[4 * v4 + 2] = fmaf(kv, cv.z, acc[4 * v4 + 2]);
+            acc[4 * v4 + 3] = fmaf(kv, cv.w, acc[4 * v4 + 3]);
+          }
+        }
+      }
+      // the unit's partial decision values: part[item][row][col]
+      float* out = part + ((int64_t)unit_item[u] * m_pad + r) * km1_pad;
+#pragma unroll
+      for (int v = 0; v < KM; ++v)
+        if (v < km1_pad) out[v] = v < km1 ? acc[v] : 0.f;
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
+  }
+}
+
+// column means of the rows idx[0..n) of X (idx < 0: skipped): per-chunk FP64 partials, then a
+// fixed-order sum over the chunks (deterministic)
+constexpr int kGatherMeanRows = 256;
+__global__ void gather_col_partial_kernel(const float* __restrict__ X, int d, const int64_t* __restrict__ idx,
+                                          int64_t n, double* __restrict__ part) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= d) return;
+  const int64_t i0 = (int64_t)blockIdx.y * kGatherMeanRows;
+  const int64_t i1 = (n < i0 + kGatherMeanRows) ? n : i0 + kGatherMeanRows;
+  double s = 0.0;
+  for (int64_t i = i0; i < i1; ++i) {
+    const int64_t r = idx[i];
+    if (r >= 0) s += X[r * d + c];
+  }
+  part[(int64_t)blockIdx.y * d + c] = s;
+}
+__global__ void gather_col_mean_kernel(const double* __restrict__ part, int nch, int d, int64_t cnt,
+                                       float* __restrict__ mu) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= d) return;
+  double s = 0.0;
+  for (int q = 0; q < nch; ++q) s += part[(int64_t)q * d + c];
+  mu[c] = (float)(cnt > 0 ? s / (double)cnt : 0.0);
+}
+
 // Column means (deterministic two-level FP64 reduction): RBF distances are translation
 // invariant, and centring shrinks the dot products whose tensor-core accumulation error
 // limits the 3xTF32 contraction.
@@ -409,6 +606,49 @@ void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, 
   const int grid = n_tiles < sms ? n_tiles : sms;
   GM_LAUNCH(krow_tc_kernel, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, d_pad / kTK,
             scale, K, ldk);
+}
+
+void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float* hi, float* lo,
+                          float* norms, int64_t n_pad, int d_pad, cudaStream_t st) {
+  GM_LAUNCH(split_tf32_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, hi, lo, norms,
+            n_pad, d_pad);
+}
+
+void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
+                            cudaStream_t st) {
+  const int nch = (int)ceil_div(n, kGatherMeanRows);
+  double* part = nullptr;
+  GM_CUDA(cudaMallocAsync(&part, (size_t)nch * d * sizeof(double), st));
+  GM_LAUNCH(gather_col_partial_kernel, dim3((unsigned)ceil_div(d, 128), (unsigned)nch), dim3(128), 0, st, X, d, idx, n,
+            part);
+  GM_LAUNCH(gather_col_mean_kernel, dim3((unsigned)ceil_div(d, 128)), dim3(128), 0, st, part, nch, d, cnt, mu);
+  GM_CUDA(cudaFreeAsync(part, st));
+}
+
+int dec_tc_max_km1() { return kDecMaxKm1; }
+
+void launch_dec_tc(const float* thi, const float* tlo, int64_t m_pad, const float* shi, const float* slo,
+                   int64_t nsv_pad, int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item,
+                   int n_units, const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma,
+                   float* part, cudaStream_t st) {
+  const CUtensorMap mthi = make_map(thi, m_pad, d_pad), mtlo = make_map(tlo, m_pad, d_pad);
+  const CUtensorMap mshi = make_map(shi, nsv_pad, d_pad), mslo = make_map(slo, nsv_pad, d_pad);
+  const float scale = (float)(-gamma * 1.4426950408889634);
+  int sms = 148, dev = 0;
+  GM_CUDA(cudaGetDevice(&dev));
+  GM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  const int grid = n_units < sms ? n_units : sms;
+  auto go = [&](auto kern, size_t smem, bool& configured) {
+    if (!configured) {
+      GM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      configured = true;
+    }
+    GM_LAUNCH(kern, dim3(grid), dim3(kTcThreads), smem, st, mthi, mtlo, mshi, mslo, tiles, unit_off, unit_item, n_units,
+              nt, nsv, coef, km1, km1_pad, d_pad / kTK, scale, m_pad, part);
+  };
+  static bool c12 = false, c32 = false;
+  if (km1_pad <= 12) go(dec_tc_kernel<12>, sizeof(DecTcSmem<12>) + 1024, c12);
+  else go(dec_tc_kernel<kDecMaxKm1>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024, c32);
 }
 
 }  // namespace gmpsvm

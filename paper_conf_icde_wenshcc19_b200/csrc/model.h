@@ -26,6 +26,15 @@ struct DevModel {
   double* b = nullptr;      // [P]
   double* A = nullptr;      // [P]
   double* B = nullptr;      // [P]
+  // tensor-core decision values (dec_tc): SV rows centred by mu, TF32 hi/lo split, row-major
+  // [nsv_pad][dpt], their centred squared norms; test rows are split with the same mu
+  bool tc = false;
+  int dpt = 0;
+  float* SvHi = nullptr;
+  float* SvLo = nullptr;
+  float* nsvc = nullptr;    // [nsv_pad]
+  float* mu = nullptr;      // [d]
+  std::vector<DecItem> h_items;  // host copy of the items (work-unit lists of dec_tc)
   std::vector<int64_t> slot_sv;  // slot -> index into the model's SV list, -1 = padding
   cudaEvent_t last_use = nullptr;  // recorded on the caller's stream after every use
   // stream-ordered allocation: freed on the library stream after last_use (no device sync)
