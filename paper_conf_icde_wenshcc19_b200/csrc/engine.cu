@@ -431,12 +431,13 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   if (dm->tc) {
     dm->dpt = krow_tc_d_pad(m.d);
     dm->mu = dev_alloc<float>(m.d, st);
-    dm->SvHi = dev_alloc<float>((size_t)dm->nsv_pad * dm->dpt, st);
-    dm->SvLo = dev_alloc<float>((size_t)dm->nsv_pad * dm->dpt, st);
+    dm->SvHi = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st);
+    dm->SvLo = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st);
     dm->nsvc = dev_alloc<float>(dm->nsv_pad, st);
     launch_gather_col_mean(rows, m.d, d_src.get(), dm->nsv_pad, nsv, dm->mu, st);
-    launch_split_tf32_mu(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, dm->SvHi, dm->SvLo, dm->nsvc, dm->nsv_pad, dm->dpt,
-                         st);
+    dm->sc = krow_split_scale(launch_maxabs(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, st));
+    launch_split_tf32_mu(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, dm->sc, dm->SvHi, dm->SvLo, dm->nsvc, dm->nsv_pad,
+                         dm->dpt, st);
   }
   GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
   GM_CUDA(cudaEventRecord(dm->last_use, st));
@@ -531,13 +532,14 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile) + (full_k ? 0 : kTile);
   // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split
   DevBuf<float> XT(use_tc ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad, st);
-  DevBuf<float> Xhi(use_tc ? (size_t)n_pad * d_pad : 0, st), Xlo(use_tc ? (size_t)n_pad * d_pad : 0, st);
+  DevBuf<float> Xhi(use_tc ? krow_tc_buf_floats(n_pad, d_pad) : 0, st), Xlo(use_tc ? krow_tc_buf_floats(n_pad, d_pad) : 0, st);
+  float ksc = 1.f;  // scale of the split (FP16: exact power of two)
   DevBuf<int32_t> bad(1, st);
   GM_CUDA(cudaMemsetAsync(bad.get(), 0, 4, st));
   DevBuf<uint8_t> tc_scratch(use_tc ? krow_tc_scratch_bytes(n, d) : 0, st);
   if (use_tc) {
     launch_row_norms(dX, n, d, d_perm.get(), norms.get(), n_pad, bad.get(), st);  // validation (non-finite rows)
-    launch_split_tf32(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st);
+    ksc = launch_split_tf32(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st);
   } else {
     launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
   }
@@ -708,7 +710,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   }
   tm.mark(PH_KERNEL);
   if (use_tc && !overlap)
-    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, K.get(),
+    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, ksc, K.get(),
                    ldk, st);
   else if (full_k && !use_tc)
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
@@ -894,7 +896,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       for (int w = 0; w < Pl; ++w) {
         const int cnt = wave_off[w + 1] - wave_off[w];
         if (cnt > 0)
-          launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get() + wave_off[w], cnt, norms.get(), n, gamma,
+          launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get() + wave_off[w], cnt, norms.get(), n, gamma, ksc,
                          K.get(), ldk, kst);
         ev_wave[w] = evp.get();
         GM_CUDA(cudaEventRecord(ev_wave[w], kst));
@@ -1232,7 +1234,9 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   const int64_t mc_pad = round_up(mc_max, kTile);
   DevBuf<float> xin(opt.inputs_on_device ? 0 : (size_t)mc_max * d, st);
   DevBuf<float> XtT(dm.tc ? 0 : (size_t)dm.d_pad * mc_pad, st), nt(mc_pad, st);
-  DevBuf<float> Xhi(dm.tc ? (size_t)mc_pad * dm.dpt : 0, st), Xlo(dm.tc ? (size_t)mc_pad * dm.dpt : 0, st);
+  DevBuf<float> Xhi(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st), Xlo(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st);
+  // the SIMT decision values need the feature-major copy only as the FP16-range fallback
+  DevBuf<float> XtTf(dm.tc ? (size_t)dm.d_pad * mc_pad : 0, st);
   DevBuf<float> part((size_t)dm.n_items * mc_pad * dm.km1_pad, st);
   DevBuf<double> dec_buf(opt.inputs_on_device ? 0 : (size_t)mc_max * P, st);
   DevBuf<double> prob_buf((opt.inputs_on_device || !prob_out) ? 0 : (size_t)mc_max * k, st);
@@ -1251,9 +1255,11 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     DevBuf<int2> d_dtiles;
     DevBuf<int32_t> d_uoff, d_uitem;
     int n_units = 0;
-    if (dm.tc) {
+    // FP16 split: test rows far outside the SVs' range would overflow half precision -> SIMT
+    const bool use_tc = dm.tc && (!krow_split_f16() || launch_maxabs(src, mc, d, nullptr, dm.mu, st) * dm.sc < 60000.f);
+    if (use_tc) {
       launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
-      launch_split_tf32_mu(src, mc, d, nullptr, dm.mu, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
+      launch_split_tf32_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
       // work units: (item, test tile), test tiles fastest; unit = the item's SV tiles for that test tile
       const int ntt = (int)(mcp / kTile);
       std::vector<int2> dt;
@@ -1274,19 +1280,21 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
       if (!uitem.empty())
         GM_CUDA(cudaMemcpyAsync(d_uitem.get(), uitem.data(), uitem.size() * 4, cudaMemcpyHostToDevice, st));
     } else {
-      launch_stage_features(src, mc, d, nullptr, XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(), st);
+      launch_stage_features(src, mc, d, nullptr, dm.tc ? XtTf.get() : XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(),
+                            st);
     }
     tm.mark(PH_STAGE);
     double* dec_d = opt.inputs_on_device ? (dec_out ? dec_out + i0 * P : dec_tmp.get()) : dec_buf.get();
     tm.mark(PH_DEC);
-    if (dm.tc) {
+    if (use_tc) {
       GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
       if (n_units > 0)
         launch_dec_tc(Xhi.get(), Xlo.get(), mcp, dm.SvHi, dm.SvLo, dm.nsv_pad, dm.dpt, d_dtiles.get(), d_uoff.get(),
-                      d_uitem.get(), n_units, nt.get(), dm.nsvc, dm.coef, dm.km1, dm.km1_pad, mdl.gamma, part.get(), st);
+                      d_uitem.get(), n_units, nt.get(), dm.nsvc, dm.coef, dm.km1, dm.km1_pad, mdl.gamma, dm.sc, part.get(),
+                      st);
     } else {
-      launch_dec_contract(XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef, dm.km1, dm.km1_pad,
-                          dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
+      launch_dec_contract(dm.tc ? XtTf.get() : XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef,
+                          dm.km1, dm.km1_pad, dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
     }
     launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     ps.dec_launches += 1;
@@ -1345,15 +1353,15 @@ int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int3
   if (sym && krow_use_tc()) {
     const int dp = krow_tc_d_pad(d);
     const int64_t np2 = krow_tc_rows_pad(n);
-    DevBuf<float> hi((size_t)np2 * dp, st), lo((size_t)np2 * dp, st), nx2(np2, st);
+    DevBuf<float> hi(krow_tc_buf_floats(np2, dp), st), lo(krow_tc_buf_floats(np2, dp), st), nx2(np2, st);
     DevBuf<uint8_t> scr(krow_tc_scratch_bytes(n, d), st);
-    launch_split_tf32(dX, n, d, nullptr, hi.get(), lo.get(), nx2.get(), np2, dp, scr.get(), st);
+    const float ksc = launch_split_tf32(dX, n, d, nullptr, hi.get(), lo.get(), nx2.get(), np2, dp, scr.get(), st);
     const std::vector<int2> tl = krow_tc_tiles(n);
     DevBuf<int2> dt(tl.size(), st);
     GM_CUDA(cudaMemcpyAsync(dt.get(), tl.data(), tl.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
     DevBuf<float> kb2(opt.inputs_on_device ? 0 : (size_t)n * m, st);
     float* dK2 = opt.inputs_on_device ? K_out : kb2.get();
-    launch_krow_tc(hi.get(), lo.get(), np2, dp, dt.get(), (int)tl.size(), nx2.get(), n, gamma, dK2, m, st);
+    launch_krow_tc(hi.get(), lo.get(), np2, dp, dt.get(), (int)tl.size(), nx2.get(), n, gamma, ksc, dK2, m, st);
     if (!opt.inputs_on_device) GM_CUDA(cudaMemcpyAsync(K_out, dK2, (size_t)n * m * 4, cudaMemcpyDeviceToHost, st));
     GM_CUDA(cudaStreamSynchronize(st));
     return GMPSVM_OK;

@@ -24,33 +24,40 @@ void launch_krow_full_sym(const float* XT, int64_t ldx, const float* norms, int6
 void launch_krow_rect(const float* AT, int64_t lda, const float* na, int64_t n, const float* BT, int64_t ldb,
                       const float* nb, int64_t m, int kdim, double gamma, float* K, int64_t ldk, cudaStream_t st);
 
-// ---------------- a2 on tcgen05 (krow_tc.cu): 3xTF32 split, TMEM accumulators, TMA staging
-int64_t krow_tc_rows_pad(int64_t n);  // row padding the tile grid needs (multiple of 256)
-int krow_tc_d_pad(int d);             // feature padding (multiple of 32)
-// centre by the column means (mean of the original rows; perm only reorders), split into TF32
-// hi/lo rows and compute the centred squared norms; scratch = krow_tc_scratch_bytes(n, d)
+// ---------------- a2 on tcgen05 (krow_tc.cu): 2-part split (FP16 default, TF32 with
+// GMPSVM_SPLIT=tf32), TMEM split accumulators, TMA staging.  hi / lo buffers are row-major
+// n_pad x d_pad elements of the split type (krow_tc_buf_floats floats of storage).
+int64_t krow_tc_rows_pad(int64_t n);  // row padding the tile grid needs (multiple of 128)
+bool krow_split_f16();
+int krow_tc_d_pad(int d);             // feature padding in elements (one 128-byte atom: 64 FP16 / 32 TF32)
+size_t krow_tc_buf_floats(int64_t n_pad, int d_pad);
+float krow_split_scale(float maxabs);  // exact power-of-two scale of the FP16 split (1 for TF32)
+// centre by the column means (mean of the original rows; perm only reorders), scale, split into
+// hi/lo rows and compute the squared norms (scaled units); returns the scale
 size_t krow_tc_scratch_bytes(int64_t n, int d);
-void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, float* hi, float* lo, float* norms,
-                       int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
+float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
+                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
+// max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
+float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
 std::vector<int2> krow_tc_tiles(int64_t n);
 constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
-// split with a given centre mu[d] (prediction: the test rows take the SV centre)
-void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float* hi, float* lo,
-                          float* norms, int64_t n_pad, int d_pad, cudaStream_t st);
+// per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
+void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
+// split with a given centre mu[d] and scale sc (prediction: the test rows take the SVs' mu, sc)
+void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
+                          void* lo, float* norms, int64_t n_pad, int d_pad, cudaStream_t st);
 // mu[c] = mean over the rows idx[i] >= 0 (cnt of them) of X[., c]
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
                             cudaStream_t st);
 // a10 on tcgen05 (krow_tc.cu): tiles = (test tile, SV tile) grouped in units [unit_off[u],
 // unit_off[u+1]), unit u writes part[unit_item[u]][row][0..km1_pad) (as launch_dec_contract)
 int dec_tc_max_km1();
-void launch_dec_tc(const float* thi, const float* tlo, int64_t m_pad, const float* shi, const float* slo,
-                   int64_t nsv_pad, int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item,
-                   int n_units, const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma,
+void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* shi, const void* slo, int64_t nsv_pad,
+                   int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item, int n_units,
+                   const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma, float sc,
                    float* part, cudaStream_t st);
-// per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
-void launch_class_means(const float* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
-void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
-                    const float* norms, int64_t n, double gamma, float* K, int64_t ldk, cudaStream_t st);
+void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
+                    const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st);
 void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
                       cudaStream_t st);
 bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel

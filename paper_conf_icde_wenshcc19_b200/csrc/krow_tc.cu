@@ -10,11 +10,22 @@
 // 3-stage smem ring of 64 KB (A hi/lo and B hi/lo, 128 x 32 FP32 each).  TMEM holds four
 // 128-column FP32 accumulators: hi.hi over each third of the k range, and hi.lo + lo.hi.
 // Entry (r, c) is written, with its mirror (c, r), only by the tile that holds it with r <= c.
+//
+// Default split: FP16 instead of TF32 (GMPSVM_SPLIT=tf32 selects TF32).  Both carry an 11-bit
+// significand per part, so hi + lo represents x to ~2^-22 either way, but kind::f16 runs at twice
+// the kind::tf32 rate (K = 16 per MMA in the same cycles as K = 8).  FP16's narrow exponent range
+// is handled by an exact power-of-two scale s (max |x - mu| s <= 2^12, well inside FP16 and away
+// from its subnormals); distances are computed in scaled units and the exp argument is divided
+// by s^2 (exact).
 #include <cuda.h>
+#include <cuda_fp16.h>
 #include <cudaTypedefs.h>
 
+#include <cmath>
 #include <cstdlib>
+#include <cstring>
 #include <mutex>
+#include <string>
 #include <vector>
 
 #include "kernels.h"
@@ -80,14 +91,22 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(const void* p) {
   d |= (uint64_t)2 << 61;              // SWIZZLE_128B
   return d;
 }
-// kind::tf32, A/B TF32 K-major, D F32, M = 128, N = 128
+// kind::tf32 / kind::f16, A/B K-major, D F32, M = 128, N = 128 (a/b format 2 = TF32, 0 = F16)
 constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(kTN >> 3) << 17) | ((uint32_t)(kTM >> 4) << 24);
+constexpr uint32_t kIdescF16 = (1u << 4) | ((uint32_t)(kTN >> 3) << 17) | ((uint32_t)(kTM >> 4) << 24);
 
+template <bool F16>
 __device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
-  asm volatile(
-      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(
-          tmem_d),
-      "l"(a), "l"(b), "r"(kIdesc), "r"(accum));
+  if (F16)
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(
+            tmem_d),
+        "l"(a), "l"(b), "r"(kIdescF16), "r"(accum));
+  else
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(
+            tmem_d),
+        "l"(a), "l"(b), "r"(kIdesc), "r"(accum));
 }
 __device__ __forceinline__ void umma_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
@@ -109,6 +128,7 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
 // producer runs ahead across tile boundaries through the smem ring; the epilogue drains the four
 // TMEM accumulators into registers and releases TMEM at once (tmem_empty), so the MMAs of the
 // next tile overlap the exp + stores of the current one.
+template <bool F16>
 __global__ void __launch_bounds__(kTcThreads, 1)
     krow_tc_kernel(const __grid_constant__ CUtensorMap map_hi, const __grid_constant__ CUtensorMap map_lo,
                    const int2* __restrict__ tiles, int n_tiles, const float* __restrict__ norms, int64_t n, int nk,
@@ -150,7 +170,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           if (g >= kTcStages) mbar_wait(&sm.empty[s], ((g / kTcStages) + 1) & 1);
           uint8_t* st = sm.stage[s];
           mbar_expect_tx(&sm.full[s], kStageBytes);
-          const int kx = kb * kTK;
+          const int kx = kb * (F16 ? 2 * kTK : kTK);
           tma_load_2d(st, &map_hi, kx, r0, &sm.full[s]);
           tma_load_2d(st + kABytes, &map_lo, kx, r0, &sm.full[s]);
           tma_load_2d(st + 2 * kABytes, &map_hi, kx, c0, &sm.full[s]);
@@ -179,9 +199,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 TF32 = 32 bytes along K inside the atom
-            umma_tf32(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
-            umma_tf32(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
-            umma_tf32(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+            umma_tf32<F16>(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
+            umma_tf32<F16>(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
+            umma_tf32<F16>(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
           }
           umma_commit(&sm.empty[s]);
         }
@@ -281,7 +301,7 @@ struct DecTcSmem {
   uint32_t tmem_base;
 };
 
-template <int KM>  // compile-time bound of the pair columns (k - 1 <= KM, KM % 4 == 0)
+template <int KM, bool F16>  // KM: compile-time bound of the pair columns (k - 1 <= KM, KM % 4 == 0)
 __global__ void __launch_bounds__(kTcThreads, 1)
     dec_tc_kernel(const __grid_constant__ CUtensorMap map_thi, const __grid_constant__ CUtensorMap map_tlo,
                   const __grid_constant__ CUtensorMap map_shi, const __grid_constant__ CUtensorMap map_slo,
@@ -325,7 +345,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             if (g >= kTcStages) mbar_wait(&sm.empty[s], ((g / kTcStages) + 1) & 1);
             uint8_t* st = sm.stage[s];
             mbar_expect_tx(&sm.full[s], kStageBytes);
-            const int kx = kb * kTK;
+            const int kx = kb * (F16 ? 2 * kTK : kTK);
             tma_load_2d(st, &map_thi, kx, r0, &sm.full[s]);
             tma_load_2d(st + kABytes, &map_tlo, kx, r0, &sm.full[s]);
             tma_load_2d(st + 2 * kABytes, &map_shi, kx, c0, &sm.full[s]);
@@ -352,9 +372,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
             for (int kk = 0; kk < kTK / 8; ++kk) {
               const uint64_t adv = (uint64_t)(kk * 32) >> 4;
-              umma_tf32(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
-              umma_tf32(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
-              umma_tf32(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+              umma_tf32<F16>(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
+              umma_tf32<F16>(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
+              umma_tf32<F16>(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
             }
             umma_commit(&sm.empty[s]);
           }
@@ -479,10 +499,12 @@ __global__ void col_mean_kernel(const double* __restrict__ part, int nchunks, in
   mu[c] = (float)(s / (double)n);
 }
 
-// x' = x - mu (FP32); hi = TF32(x'), lo = TF32(x' - hi) (round to nearest);
-// norms[j] = ||x'_j||^2 accumulated in FP64 (one warp per row); zero padding.
+// x' = (x - mu) s (FP32; s = 1 for TF32); TF32: hi = TF32(x'), lo = TF32(x' - hi) (round to
+// nearest); FP16: hi = half(x'), lo = half(x' - hi); norms[j] = ||x'_j||^2 accumulated in FP64
+// (one warp per row); zero padding.  hi / lo rows are d_pad elements (4 or 2 bytes).
+template <bool F16>
 __global__ void split_tf32_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
-                                  const float* __restrict__ mu, float* __restrict__ hi, float* __restrict__ lo,
+                                  const float* __restrict__ mu, float sc, void* __restrict__ hi_, void* __restrict__ lo_,
                                   float* __restrict__ norms, int64_t n_pad, int d_pad) {
   const int64_t j = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
@@ -491,18 +513,41 @@ __global__ void split_tf32_kernel(const float* __restrict__ X, int64_t n, int d,
   double s = 0.0;
   for (int c = lane; c < d_pad; c += 32) {
     float x = 0.f;
-    if (src >= 0 && c < d) x = X[src * d + c] - mu[c];
-    // round-to-nearest TF32 for both parts, so the tensor core sees exact TF32 values (it would
-    // otherwise drop the low 13 bits of lo) and the dropped lo.lo / lo-rounding terms are unbiased
-    const float h = __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
-    const float r = x - h;
-    hi[j * d_pad + c] = h;
-    lo[j * d_pad + c] = __uint_as_float((__float_as_uint(r) + 0x1000u) & 0xFFFFE000u);
+    if (src >= 0 && c < d) x = (X[src * d + c] - mu[c]) * sc;
+    if (F16) {
+      const __half h = __float2half_rn(x);
+      const float r = x - __half2float(h);
+      static_cast<__half*>(hi_)[j * d_pad + c] = h;
+      static_cast<__half*>(lo_)[j * d_pad + c] = __float2half_rn(r);
+    } else {
+      // round-to-nearest TF32 for both parts, so the tensor core sees exact TF32 values (it would
+      // otherwise drop the low 13 bits of lo) and the dropped lo.lo / lo-rounding terms are unbiased
+      const float h = __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+      const float r = x - h;
+      static_cast<float*>(hi_)[j * d_pad + c] = h;
+      static_cast<float*>(lo_)[j * d_pad + c] = __uint_as_float((__float_as_uint(r) + 0x1000u) & 0xFFFFE000u);
+    }
     s = fma((double)x, (double)x, s);
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   if (lane == 0) norms[j] = (float)s;
+}
+
+// max over the rows of |x - mu| (non-negative floats order as their bit patterns: atomicMax)
+__global__ void maxabs_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
+                              const float* __restrict__ mu, unsigned* __restrict__ out) {
+  float m = 0.f;
+  const int64_t total = n * d;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = e / d;
+    const int c = (int)(e - j * d);
+    const int64_t src = perm ? perm[j] : j;
+    if (src >= 0) m = fmaxf(m, fabsf(X[src * d + c] - mu[c]));
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(out, __float_as_uint(m));
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -518,17 +563,18 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   return fn;
 }
 
-CUtensorMap make_map(const float* base, int64_t rows, int d_pad) {
+CUtensorMap make_map(const void* base, int64_t rows, int d_pad, bool f16) {
   auto enc = get_encode();
   if (!enc) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled unavailable");
   CUtensorMap m;
+  const size_t eb = f16 ? 2 : 4;
   const cuuint64_t dims[2] = {(cuuint64_t)d_pad, (cuuint64_t)rows};
-  const cuuint64_t strides[1] = {(cuuint64_t)d_pad * sizeof(float)};
-  const cuuint32_t box[2] = {(cuuint32_t)kTK, (cuuint32_t)kTM};
+  const cuuint64_t strides[1] = {(cuuint64_t)d_pad * eb};
+  const cuuint32_t box[2] = {(cuuint32_t)(128 / eb), (cuuint32_t)kTM};  // one 128-byte swizzle atom along K
   const cuuint32_t estr[2] = {1, 1};
-  const CUresult r = enc(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
-                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  const CUresult r = enc(&m, f16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                         const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
   return m;
 }
@@ -536,31 +582,71 @@ CUtensorMap make_map(const float* base, int64_t rows, int d_pad) {
 }  // namespace
 
 int64_t krow_tc_rows_pad(int64_t n) { return round_up(n, kTN > kTM ? kTN : kTM); }
-int krow_tc_d_pad(int d) { return (int)round_up(d, kTK); }
-
-size_t krow_tc_scratch_bytes(int64_t n, int d) {
-  return (size_t)ceil_div(n, kMeanRows) * d * sizeof(double) + (size_t)d * sizeof(float);
+bool krow_split_f16() {
+  static const bool tf32 = getenv("GMPSVM_SPLIT") && std::string(getenv("GMPSVM_SPLIT")) == "tf32";
+  return !tf32;
+}
+int krow_tc_d_pad(int d) { return (int)round_up(d, krow_split_f16() ? 2 * kTK : kTK); }
+size_t krow_tc_buf_floats(int64_t n_pad, int d_pad) {
+  return (size_t)n_pad * d_pad * (krow_split_f16() ? 2 : 4) / 4;
+}
+float krow_split_scale(float maxabs) {  // power of two with maxabs * s <= 2^12 (FP16 split); 1 for TF32
+  if (!krow_split_f16() || !(maxabs > 0.f) || !std::isfinite(maxabs)) return 1.f;
+  int e = 0;
+  std::frexp(4096.0 / (double)maxabs, &e);  // 4096 / maxabs = f * 2^e, f in [0.5, 1)
+  e = std::max(-60, std::min(60, e - 1));
+  return (float)std::ldexp(1.0, e);
 }
 
-void launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, float* hi, float* lo, float* norms,
-                       int64_t n_pad, int d_pad, void* scratch, cudaStream_t st) {
+size_t krow_tc_scratch_bytes(int64_t n, int d) {
+  return (size_t)ceil_div(n, kMeanRows) * d * sizeof(double) + (size_t)d * sizeof(float) + 16;
+}
+
+float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st) {
+  unsigned* dm = nullptr;
+  GM_CUDA(cudaMallocAsync(&dm, sizeof(unsigned), st));
+  GM_CUDA(cudaMemsetAsync(dm, 0, sizeof(unsigned), st));
+  GM_LAUNCH(maxabs_kernel, dim3(592), dim3(256), 0, st, X, n, d, perm, mu, dm);
+  unsigned h = 0;
+  GM_CUDA(cudaMemcpyAsync(&h, dm, sizeof(unsigned), cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaFreeAsync(dm, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  float v;
+  std::memcpy(&v, &h, 4);
+  return v;
+}
+
+void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
+                          void* lo, float* norms, int64_t n_pad, int d_pad, cudaStream_t st) {
+  if (krow_split_f16())
+    GM_LAUNCH(split_tf32_kernel<true>, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, sc, hi,
+              lo, norms, n_pad, d_pad);
+  else
+    GM_LAUNCH(split_tf32_kernel<false>, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, 1.f,
+              hi, lo, norms, n_pad, d_pad);
+}
+
+float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
+                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st) {
   const int nch = (int)ceil_div(n, kMeanRows);
   double* part = static_cast<double*>(scratch);
   float* mu = reinterpret_cast<float*>(part + (size_t)nch * d);
   GM_LAUNCH(col_partial_kernel, dim3((unsigned)ceil_div(d, 128), (unsigned)nch), dim3(128), 0, st, X, n, d, part);
   GM_LAUNCH(col_mean_kernel, dim3((unsigned)ceil_div(d, 128)), dim3(128), 0, st, part, nch, n, d, mu);
-  GM_LAUNCH(split_tf32_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, hi, lo, norms,
-            n_pad, d_pad);
+  const float sc = krow_split_f16() ? krow_split_scale(launch_maxabs(X, n, d, nullptr, mu, st)) : 1.f;
+  launch_split_tf32_mu(X, n, d, perm, mu, sc, hi, lo, norms, n_pad, d_pad, st);
+  return sc;
 }
 
-// Per-class means of the staged (centred, class-sorted) rows, from the TF32 hi part: used only to
-// order the pairs for the overlap of the kernel-value waves with the solver (engine.cu).
-__global__ void class_means_kernel(const float* hi, int d_pad, const int64_t* coff, float* mu) {
+// Per-class means of the staged (centred, class-sorted) rows, from the hi part: used only to
+// order the pairs (engine.cu).
+template <typename T>
+__global__ void class_means_kernel(const T* hi, int d_pad, const int64_t* coff, float* mu) {
   const int c = blockIdx.y, f = blockIdx.x * 32 + threadIdx.x;
   const int64_t r0 = coff[c], r1 = coff[c + 1];
   float s = 0.f;
   if (f < d_pad)
-    for (int64_t r = r0 + threadIdx.y; r < r1; r += 8) s += hi[r * d_pad + f];
+    for (int64_t r = r0 + threadIdx.y; r < r1; r += 8) s += (float)hi[r * d_pad + f];
   __shared__ float red[8][33];
   red[threadIdx.y][threadIdx.x] = s;
   __syncthreads();
@@ -572,9 +658,13 @@ __global__ void class_means_kernel(const float* hi, int d_pad, const int64_t* co
   }
 }
 
-void launch_class_means(const float* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st) {
-  GM_LAUNCH(class_means_kernel, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st, hi, d_pad, coff,
-            mu);
+void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st) {
+  if (krow_split_f16())
+    GM_LAUNCH(class_means_kernel<__half>, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st,
+              static_cast<const __half*>(hi), d_pad, coff, mu);
+  else
+    GM_LAUNCH(class_means_kernel<float>, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st,
+              static_cast<const float*>(hi), d_pad, coff, mu);
 }
 
 // Tiles (bi, bj) of 128 x 128 with at least one entry r <= c, in blocked order (16 x 16 tiles)
@@ -590,28 +680,35 @@ std::vector<int2> krow_tc_tiles(int64_t n) {
   return t;
 }
 
-void launch_krow_tc(const float* hi, const float* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
-                    const float* norms, int64_t n, double gamma, float* K, int64_t ldk, cudaStream_t st) {
-  const CUtensorMap mhi = make_map(hi, n_pad, d_pad), mlo = make_map(lo, n_pad, d_pad);
-  const size_t smem = sizeof(TcSmem) + 1024;
-  static bool configured = false;
-  if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured = true;
-  }
-  const float scale = (float)(-gamma * 1.4426950408889634);
+static int num_sms() {
   int sms = 148, dev = 0;
   GM_CUDA(cudaGetDevice(&dev));
   GM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-  const int grid = n_tiles < sms ? n_tiles : sms;
-  GM_LAUNCH(krow_tc_kernel, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, d_pad / kTK,
-            scale, K, ldk);
+  return sms;
 }
 
-void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float* hi, float* lo,
-                          float* norms, int64_t n_pad, int d_pad, cudaStream_t st) {
-  GM_LAUNCH(split_tf32_kernel, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, hi, lo, norms,
-            n_pad, d_pad);
+void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
+                    const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st) {
+  const bool f16 = krow_split_f16();
+  const CUtensorMap mhi = make_map(hi, n_pad, d_pad, f16), mlo = make_map(lo, n_pad, d_pad, f16);
+  const size_t smem = sizeof(TcSmem) + 1024;
+  static bool configured = false;
+  if (!configured) {
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    configured = true;
+  }
+  // distances are in units scaled by sc: exp(-gamma d2 / sc^2) = exp2(d2 * scale)
+  const float scale = (float)(-gamma * 1.4426950408889634 / ((double)sc * (double)sc));
+  const int sms = num_sms();
+  const int grid = n_tiles < sms ? n_tiles : sms;
+  const int nk = d_pad / (f16 ? 2 * kTK : kTK);
+  if (f16)
+    GM_LAUNCH(krow_tc_kernel<true>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, nk,
+              scale, K, ldk);
+  else
+    GM_LAUNCH(krow_tc_kernel<false>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, nk,
+              scale, K, ldk);
 }
 
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
@@ -627,28 +724,33 @@ void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n
 
 int dec_tc_max_km1() { return kDecMaxKm1; }
 
-void launch_dec_tc(const float* thi, const float* tlo, int64_t m_pad, const float* shi, const float* slo,
-                   int64_t nsv_pad, int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item,
-                   int n_units, const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma,
+void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* shi, const void* slo, int64_t nsv_pad,
+                   int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item, int n_units,
+                   const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma, float sc,
                    float* part, cudaStream_t st) {
-  const CUtensorMap mthi = make_map(thi, m_pad, d_pad), mtlo = make_map(tlo, m_pad, d_pad);
-  const CUtensorMap mshi = make_map(shi, nsv_pad, d_pad), mslo = make_map(slo, nsv_pad, d_pad);
-  const float scale = (float)(-gamma * 1.4426950408889634);
-  int sms = 148, dev = 0;
-  GM_CUDA(cudaGetDevice(&dev));
-  GM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  const bool f16 = krow_split_f16();
+  const CUtensorMap mthi = make_map(thi, m_pad, d_pad, f16), mtlo = make_map(tlo, m_pad, d_pad, f16);
+  const CUtensorMap mshi = make_map(shi, nsv_pad, d_pad, f16), mslo = make_map(slo, nsv_pad, d_pad, f16);
+  const float scale = (float)(-gamma * 1.4426950408889634 / ((double)sc * (double)sc));
+  const int sms = num_sms();
   const int grid = n_units < sms ? n_units : sms;
+  const int nk = d_pad / (f16 ? 2 * kTK : kTK);
   auto go = [&](auto kern, size_t smem, bool& configured) {
     if (!configured) {
       GM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       configured = true;
     }
     GM_LAUNCH(kern, dim3(grid), dim3(kTcThreads), smem, st, mthi, mtlo, mshi, mslo, tiles, unit_off, unit_item, n_units,
-              nt, nsv, coef, km1, km1_pad, d_pad / kTK, scale, m_pad, part);
+              nt, nsv, coef, km1, km1_pad, nk, scale, m_pad, part);
   };
-  static bool c12 = false, c32 = false;
-  if (km1_pad <= 12) go(dec_tc_kernel<12>, sizeof(DecTcSmem<12>) + 1024, c12);
-  else go(dec_tc_kernel<kDecMaxKm1>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024, c32);
+  static bool c[4] = {false, false, false, false};
+  if (km1_pad <= 12) {
+    if (f16) go(dec_tc_kernel<12, true>, sizeof(DecTcSmem<12>) + 1024, c[0]);
+    else go(dec_tc_kernel<12, false>, sizeof(DecTcSmem<12>) + 1024, c[1]);
+  } else {
+    if (f16) go(dec_tc_kernel<kDecMaxKm1, true>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024, c[2]);
+    else go(dec_tc_kernel<kDecMaxKm1, false>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024, c[3]);
+  }
 }
 
 }  // namespace gmpsvm

@@ -34,6 +34,7 @@ struct DevModel {
   float* SvLo = nullptr;
   float* nsvc = nullptr;    // [nsv_pad]
   float* mu = nullptr;      // [d]
+  float sc = 1.f;           // split scale (exact power of two; 1 for TF32)
   std::vector<DecItem> h_items;  // host copy of the items (work-unit lists of dec_tc)
   std::vector<int64_t> slot_sv;  // slot -> index into the model's SV list, -1 = padding
   cudaEvent_t last_use = nullptr;  // recorded on the caller's stream after every use

@@ -1,2 +1,5 @@
+python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+python tools/krow_check.py 2>&1 | tail -3
+GMPSVM_SPLIT=tf32 python tools/krow_check.py 2>&1 | tail -3
 python tools/sweep.py "" 2>&1 | grep total
-python bench.py --steps 5 --warmup 3 > gpurun_out/bench3.json 2> gpurun_out/bench3.err; cat gpurun_out/bench3.json
+python tools/prof_step.py 2>&1 | tail -1
