@@ -242,11 +242,13 @@ def run_gpu(args, spec):
         achieved = s["kernel_flops"] / (krow_ms * 1e-3) / 1e12
         peaks = _peaks()
         bf16 = peaks.get("bf16_tflops", 1590.0)
-        # krow_contract runs on tcgen05 kind::tf32 with a 3xTF32 split (3 MMAs per product for FP32
-        # accuracy): its speed of light is the TF32 dense peak / 3, TF32 = measured bf16 burst x 0.5
-        # (the guide's nominal TF32:BF16 ratio 1.13 : 2.25)
-        tf32 = bf16 * 0.5
-        peak = tf32 / 3.0
+        # krow_contract runs on tcgen05 with a two-part (hi + lo) split and 3 MMAs per FP32-accurate
+        # product (hi*hi + hi*lo + lo*hi): its speed of light is the dense peak of the MMA kind / 3.
+        # Default kind::f16 (FP16 parts) at the measured bf16 burst peak (same dense rate for f16);
+        # GMPSVM_SPLIT=tf32 uses kind::tf32 at bf16 x 0.5 (the guide's nominal 1.13 : 2.25 ratio)
+        split = "tf32" if os.environ.get("GMPSVM_SPLIT", "") == "tf32" else "f16"
+        mma_peak = bf16 * (0.5 if split == "tf32" else 1.0)
+        peak = mma_peak / 3.0
         traffic = None
         tr_path = os.path.join(ROOT, "profiles", "krow_traffic.json")
         if os.path.exists(tr_path):
@@ -256,13 +258,15 @@ def run_gpu(args, spec):
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False, "scaling": "strong",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (datagen mnist recipe, seeds 1234/1/2)",
             "config": _config(spec, args),
-            "roofline": {"kernel": "krow_contract (krow_tc_kernel, tcgen05 3xTF32)", "bound": "tensor",
+            "roofline": {"kernel": f"krow_contract (krow_tc_kernel, tcgen05 kind::{split}, 3-MMA hi/lo split)",
+                         "bound": "tensor",
                          "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                          "traffic": traffic,
-                         "peak_note": (f"TF32 dense = measured bf16 burst {bf16} x 0.5 = {tf32:.1f} TFLOP/s"
-                                       f"{'' if 'bf16_tflops' in peaks else ' (fallback)'}; 3xTF32 needs 3 MMAs per "
-                                       "FP32-accurate product, so peak = TF32/3"),
-                         "frac_of_tf32_peak": achieved / tf32,
+                         "peak_note": (f"kind::{split} dense = measured bf16 burst {bf16}"
+                                       f"{' x 0.5' if split == 'tf32' else ''} = {mma_peak:.1f} TFLOP/s"
+                                       f"{'' if 'bf16_tflops' in peaks else ' (fallback)'}; the hi/lo split needs 3 MMAs "
+                                       "per FP32-accurate product, so peak = that / 3"),
+                         "frac_of_mma_peak": achieved / mma_peak,
                          "frac_of_fp32_simt_peak": achieved / FP32_PEAK_TFLOPS_DERIVED,
                          "flops_per_launch": s["kernel_flops"], "launch_ms": krow_ms,
                          "algorithmic": "n(n+1)/2 kernel values x (2d+3) flop"},

@@ -22,6 +22,7 @@
 #include <cudaTypedefs.h>
 
 #include <cmath>
+#include <cstdint>
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
@@ -44,13 +45,18 @@ constexpr uint32_t kStageBytes = 2 * kABytes + 2 * kBBytes;  // 64 KB
 constexpr uint32_t kTmemCols = 512;  // 3 x 128 hi.hi (k thirds) + 128 hi.lo + lo.hi
 constexpr int kDecMaxKm1 = 32;       // dec_tc: pair columns per SV (k - 1, padded), k <= 33
 
+constexpr int kEpiWarps = 4;
 struct TcSmem {
   // each operand tile 1024-byte aligned (128B swizzle atoms)
   alignas(1024) uint8_t stage[kTcStages][kStageBytes];
+  // epilogue staging for the TMA stores, per epilogue warp: [0] its 32 x 32 block of K (rows r,
+  // columns c, 128-byte swizzled), [1] the mirrored block (rows c, columns r)
+  alignas(1024) float epi[kEpiWarps][2][32 * 32];
   alignas(8) uint64_t full[kTcStages];
   uint64_t empty[kTcStages];
   uint64_t tmem_full;
   uint64_t tmem_empty;
+  uint64_t tmem_empty2;
   uint32_t tmem_base;
 };
 
@@ -80,6 +86,17 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, i
       "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* src, int x, int y) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(smem_u32(src)), "r"(x), "r"(y)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
 // K-major operand, 128-byte swizzle: 8-row groups 1024 B apart (SBO), LBO unused (1), version 1.
 __device__ __forceinline__ uint64_t umma_desc_sw128(const void* p) {
   const uint64_t addr = smem_u32(p);
@@ -131,8 +148,9 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
 template <bool F16>
 __global__ void __launch_bounds__(kTcThreads, 1)
     krow_tc_kernel(const __grid_constant__ CUtensorMap map_hi, const __grid_constant__ CUtensorMap map_lo,
+                   const __grid_constant__ CUtensorMap map_ksw, const __grid_constant__ CUtensorMap map_kns,
                    const int2* __restrict__ tiles, int n_tiles, const float* __restrict__ norms, int64_t n, int nk,
-                   float scale, float* __restrict__ K, int64_t ldk) {
+                   float scale, float* __restrict__ K, int64_t ldk, int tma_store) {
   extern __shared__ __align__(1024) uint8_t dsmem[];
   TcSmem& sm = *reinterpret_cast<TcSmem*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -143,7 +161,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_init(&sm.empty[s], 1);
     }
     mbar_init(&sm.tmem_full, 1);
-    mbar_init(&sm.tmem_empty, 4);  // one arrive per epilogue warp
+    mbar_init(&sm.tmem_empty, 4);   // one arrive per epilogue warp: accumulators 0 and 3 drained
+    mbar_init(&sm.tmem_empty2, 4);  // accumulators 1 and 2 drained
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_hi)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_lo)) : "memory");
@@ -196,6 +215,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           // products of each k third and the small corrections get accumulators of their own
           const int j = (kb * jn) / nk;
           const int kb_first = (j * nk + jn - 1) / jn;
+          // the epilogue releases accumulators 0 + 3 first (the next tile starts with them) and 1 + 2
+          // after: the second half of its drain overlaps this tile's first k third
+          if (it > 0 && j == 1 && kb == kb_first) {
+            mbar_wait(&sm.tmem_empty2, (it - 1) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          }
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 TF32 = 32 bytes along K inside the atom
@@ -215,38 +240,86 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       const int2 tile = tiles[t];
       const int64_t r0 = (int64_t)tile.x * kTM, c0 = (int64_t)tile.y * kTN;
       const int64_t r = r0 + q * 32 + lane;
+      const float nr = (r < n) ? norms[r] : 0.f;
+      float cnv[kTN / 32];  // column norms of the tile (lane holds column c0 + 32 ch + lane), loaded early
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) cnv[ch] = norms[c0 + ch * 32 + lane];  // n_pad >= c0 + 128 (zero padded)
       mbar_wait(&sm.tmem_full, it & 1);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       float dot[kTN];
+      const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
 #pragma unroll
-      for (int ch = 0; ch < kTN / 32; ++ch) {
-        uint32_t v0[32], v1[32], v2[32], w[32];
-        const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(ch * 32);
-        tmem_ld32(taddr, v0);
-        tmem_ld32(taddr + kTN, v1);
-        tmem_ld32(taddr + 2 * kTN, v2);
-        tmem_ld32(taddr + kMainAcc * kTN, w);
+      for (int ch = 0; ch < kTN / 32; ++ch) {  // accumulators 0 (first k third) and 3 (corrections)
+        uint32_t v0[32], w[32];
+        tmem_ld32(trow + (uint32_t)(ch * 32), v0);
+        tmem_ld32(trow + (uint32_t)(ch * 32) + kMainAcc * kTN, w);
         asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 #pragma unroll
-        for (int j = 0; j < 32; ++j) {
-          float x = __uint_as_float(v0[j]);
-          if (nk > 1) x += __uint_as_float(v1[j]);
-          if (nk > 2) x += __uint_as_float(v2[j]);
-          dot[ch * 32 + j] = x + __uint_as_float(w[j]);
+        for (int j = 0; j < 32; ++j) dot[ch * 32 + j] = __uint_as_float(v0[j]) + __uint_as_float(w[j]);
+      }
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+      if (nk > 1) {
+#pragma unroll
+        for (int ch = 0; ch < kTN / 32; ++ch) {  // accumulators 1 and 2 (second and third k thirds)
+          uint32_t v1[32], v2[32];
+          tmem_ld32(trow + (uint32_t)(ch * 32) + kTN, v1);
+          tmem_ld32(trow + (uint32_t)(ch * 32) + 2 * kTN, v2);
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            float x = dot[ch * 32 + j] + __uint_as_float(v1[j]);
+            if (nk > 2) x += __uint_as_float(v2[j]);
+            dot[ch * 32 + j] = x;
+          }
         }
       }
       // TMEM may be overwritten by the next tile's MMAs from here on
       asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
       __syncwarp();
-      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
-      const float nr = (r < n) ? norms[r] : 0.f;
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty2)) : "memory");
+      if (tma_store && tile.x != tile.y) {
+        // off-diagonal tile (every r < c): the 128 x 128 block and its mirror leave through shared
+        // memory as full-line TMA stores (one 32 x 32 block pair per warp and column chunk; rows /
+        // columns >= n are clipped by the tensor maps)
+        float* eb = sm.epi[q][0];
+        float* em = sm.epi[q][1];
+#pragma unroll
+        for (int ch = 0; ch < kTN / 32; ++ch) {
+          const int64_t cb = c0 + ch * 32;
+          const float cn = cnv[ch];
+          float kv[32];
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cn, j));
+            asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv[j]) : "f"(fmaxf(d2, 0.f) * scale));
+          }
+          if (lane == 0) bulk_wait_read0();  // the previous chunk's stores have read the staging
+          __syncwarp();
+#pragma unroll
+          for (int jj = 0; jj < 8; ++jj)  // row `lane`, 16-byte chunk jj at jj ^ (row % 8) (128B swizzle)
+            *reinterpret_cast<float4*>(eb + lane * 32 + ((jj ^ (lane & 7)) << 2)) =
+                make_float4(kv[4 * jj], kv[4 * jj + 1], kv[4 * jj + 2], kv[4 * jj + 3]);
+#pragma unroll
+          for (int j = 0; j < 32; ++j) em[j * 32 + lane] = kv[j];
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) {
+            tma_store_2d(&map_ksw, eb, (int)cb, (int)(r0 + q * 32));
+            tma_store_2d(&map_kns, em, (int)(r0 + q * 32), (int)cb);
+            bulk_commit();
+          }
+        }
+        continue;
+      }
 #pragma unroll
       for (int ch = 0; ch < kTN / 32; ++ch) {
         const int64_t cb = c0 + ch * 32;
         float kv[32];
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
-          const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __ldg(norms + cb + j));
+          const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cnv[ch], j));
           float val;
           asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(val) : "f"(fmaxf(d2, 0.f) * scale));
           kv[j] = (r == cb + j) ? 1.f : val;
@@ -273,6 +346,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
       }
     }
+    if (lane == 0) bulk_wait0();  // every TMA store of this warp complete before the CTA exits
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
@@ -687,10 +761,31 @@ static int num_sms() {
   return sms;
 }
 
+// K (n x n FP32, row stride ldk) as the target of the epilogue's 32 x 32 TMA stores
+CUtensorMap make_kmap(float* K, int64_t n, int64_t ldk, bool swizzle) {
+  auto enc = get_encode();
+  if (!enc) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  CUtensorMap m;
+  const cuuint64_t dims[2] = {(cuuint64_t)n, (cuuint64_t)n};
+  const cuuint64_t strides[1] = {(cuuint64_t)ldk * 4};
+  const cuuint32_t box[2] = {32, 32};
+  const cuuint32_t estr[2] = {1, 1};
+  const CUresult r = enc(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, K, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         swizzle ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                         CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled (K) failed: " + std::to_string((int)r));
+  return m;
+}
+
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st) {
   const bool f16 = krow_split_f16();
   const CUtensorMap mhi = make_map(hi, n_pad, d_pad, f16), mlo = make_map(lo, n_pad, d_pad, f16);
+  // TMA stores need a 16-byte aligned base and row stride; otherwise every tile takes the
+  // per-thread store path
+  static const bool no_tma_env = getenv("GMPSVM_KROW_STORE") && std::string(getenv("GMPSVM_KROW_STORE")) == "st";
+  const int tma = !no_tma_env && (ldk % 4) == 0 && (reinterpret_cast<uintptr_t>(K) & 15) == 0 && n < (int64_t)INT32_MAX;
+  const CUtensorMap mksw = make_kmap(K, tma ? n : 1, tma ? ldk : 4, true), mkns = make_kmap(K, tma ? n : 1, tma ? ldk : 4, false);
   const size_t smem = sizeof(TcSmem) + 1024;
   static bool configured = false;
   if (!configured) {
@@ -704,11 +799,11 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
   const int grid = n_tiles < sms ? n_tiles : sms;
   const int nk = d_pad / (f16 ? 2 * kTK : kTK);
   if (f16)
-    GM_LAUNCH(krow_tc_kernel<true>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, nk,
-              scale, K, ldk);
+    GM_LAUNCH(krow_tc_kernel<true>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles, norms,
+              n, nk, scale, K, ldk, tma);
   else
-    GM_LAUNCH(krow_tc_kernel<false>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, tiles, n_tiles, norms, n, nk,
-              scale, K, ldk);
+    GM_LAUNCH(krow_tc_kernel<false>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles,
+              norms, n, nk, scale, K, ldk, tma);
 }
 
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
