@@ -232,9 +232,11 @@ T* dev_alloc(size_t count, cudaStream_t st) {
 // Per-thread cached pinned host staging (cudaMallocHost / cudaFreeHost are slow and the
 // latter synchronises the device, so they are not called per training run).
 template <class T>
-T* pinned_scratch(size_t count) {
-  static thread_local void* buf = nullptr;
-  static thread_local size_t cap = 0;
+T* pinned_scratch(size_t count, int slot = 0) {
+  static thread_local void* bufs[2] = {nullptr, nullptr};
+  static thread_local size_t caps[2] = {0, 0};
+  void*& buf = bufs[slot];
+  size_t& cap = caps[slot];
   const size_t bytes = count * sizeof(T);
   if (bytes > cap) {
     if (buf) cudaFreeHost(buf);
@@ -351,9 +353,23 @@ gmpsvm_predict_stats& tls_predict_stats() {
 
 // Build the device prediction structures from SV rows already on the device.
 // rows: device pointer to rows (stride d); row_of_sv[i] = row of SV i (SV order = sv_pos order).
+// mu_in / sc_in: a given centre and split scale for the SV rows; nullptr = compute them from the
+// SV rows
 static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* rows, const std::vector<int64_t>& row_of_sv,
-                                                 int device, cudaStream_t st) {
+                                                 int device, cudaStream_t st, const float* mu_in = nullptr,
+                                                 float sc_in = 0.f) {
   auto dm = std::make_unique<DevModel>();
+  static const bool ht = getenv("GMPSVM_HOST_TIMING") != nullptr;
+  auto t_last = std::chrono::steady_clock::now();
+  std::string line;
+  auto HT = [&](const char* what) {
+    if (!ht) return;
+    GM_CUDA(cudaStreamSynchronize(st));
+    const auto now = std::chrono::steady_clock::now();
+    line += std::string(" ") + what + "=" +
+            std::to_string(std::chrono::duration<double, std::milli>(now - t_last).count()).substr(0, 6);
+    t_last = now;
+  };
   dm->device = device;
   const int k = m.k, P = m.P();
   dm->km1 = k - 1;
@@ -404,6 +420,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   }
   if (items.empty()) items.push_back(DecItem{0, 0, 0, 0});  // no SV at all: zero contribution
   dm->n_items = (int)items.size();
+  HT("host_coef");
   dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad, st);
   dm->nsv = dev_alloc<float>(dm->nsv_pad, st);
   dm->coef = dev_alloc<float>(coef.size(), st);
@@ -424,6 +441,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   GM_CUDA(cudaMemcpyAsync(dm->B, m.B.data(), P * 8, cudaMemcpyHostToDevice, st));
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
+  HT("h2d_svt");
   dm->h_items = items;
   // tensor-core decision values: centre = mean of the SV rows, TF32 hi/lo split of the SV slots
   static const bool dec_simt = getenv("GMPSVM_DEC") && std::string(getenv("GMPSVM_DEC")) == "simt";
@@ -434,11 +452,20 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
     dm->SvHi = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st);
     dm->SvLo = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st);
     dm->nsvc = dev_alloc<float>(dm->nsv_pad, st);
-    launch_gather_col_mean(rows, m.d, d_src.get(), dm->nsv_pad, nsv, dm->mu, st);
-    dm->sc = krow_split_scale(launch_maxabs(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, st));
+    if (mu_in) {
+      GM_CUDA(cudaMemcpyAsync(dm->mu, mu_in, (size_t)m.d * 4, cudaMemcpyDeviceToDevice, st));
+      dm->sc = sc_in;
+    } else {
+      launch_gather_col_mean(rows, m.d, d_src.get(), dm->nsv_pad, nsv, dm->mu, st);
+      HT("mean");
+      dm->sc = krow_split_scale(launch_maxabs(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, st));
+      HT("maxabs");
+    }
     launch_split_tf32_mu(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, dm->sc, dm->SvHi, dm->SvLo, dm->nsvc, dm->nsv_pad,
                          dm->dpt, st);
+    HT("split");
   }
+  if (ht) fprintf(stderr, "[gmpsvm devmodel ms]%s\n", line.c_str());
   GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
   GM_CUDA(cudaEventRecord(dm->last_use, st));
   GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
@@ -937,7 +964,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
                                             cudaStreamCaptureModeRelaxed));
       if (wsp) {  // default kernels (wsolve.cu): selection -> gather -> local SMO -> f-update, unrolled:
                   // the conditional node's re-launch (~10 us) is paid every `unroll` iterations
-        static const int unroll = getenv("GMPSVM_UNROLL") ? std::max(1, atoi(getenv("GMPSVM_UNROLL"))) : 2;
+        static const int unroll = getenv("GMPSVM_UNROLL") ? std::max(1, atoi(getenv("GMPSVM_UNROLL"))) : 4;
         for (int u = 0; u < unroll; ++u) launch_ws_iteration(ag, gn, npi, h, u == unroll - 1, max_outer, cs, u > 0);
       } else {
         launch_select_ws(ag, gn, 0, -1, cs);
@@ -1006,16 +1033,28 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   // ---------------- a7-a9 bias, decision values, sigmoid, SV union
   tm.mark(PH_FIN);
   HT("fin0");
+  if (host_timing) {  // synchronised checkpoints: the solver's end, then each finalize step
+    GM_CUDA(cudaStreamSynchronize(st));
+    HT("solver_wait");
+  }
   launch_finalize(a, Pl, st);
   launch_sigmoid_fit(a, Pl, st);
   DevBuf<uint8_t> d_flags(n, st);
   GM_CUDA(cudaMemsetAsync(d_flags.get(), 0, n, st));
   launch_sv_flags(a, Pl, np_max, d_flags.get(), st);
-  std::vector<double> h_alpha(tot), hb(Pl), hA(Pl), hB(Pl);
+  if (host_timing) {
+    GM_CUDA(cudaStreamSynchronize(st));
+    HT("fin_kernels");
+  }
+  std::vector<double> hb(Pl), hA(Pl), hB(Pl);
   std::vector<int32_t> h_sig(Pl), h_st(Pl), h_outer(Pl);
-  std::vector<int64_t> h_inner(Pl), h_cyc(Pl), h_perm(n);
-  std::vector<uint8_t> h_flags(n);
-  GM_CUDA(cudaMemcpyAsync(h_alpha.data(), d_alpha.get(), tot * 8, cudaMemcpyDeviceToHost, st));
+  std::vector<int64_t> h_inner(Pl), h_cyc(Pl);
+  // the large read-backs (alpha, permutation, SV flags) land in pinned memory (async DMA)
+  uint8_t* pin = pinned_scratch<uint8_t>((size_t)tot * 8 + (size_t)n * 8 + (size_t)n + 64, 1);
+  double* h_alpha = reinterpret_cast<double*>(pin);
+  int64_t* h_permp = reinterpret_cast<int64_t*>(pin + (size_t)tot * 8);
+  uint8_t* h_flags = pin + (size_t)tot * 8 + (size_t)n * 8;
+  GM_CUDA(cudaMemcpyAsync(h_alpha, d_alpha.get(), tot * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(hb.data(), d_b.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(hA.data(), d_A.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(hB.data(), d_B.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
@@ -1024,11 +1063,12 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   GM_CUDA(cudaMemcpyAsync(h_outer.data(), d_outer.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_inner.data(), d_inner.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_cyc.data(), d_cyc.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_perm.data(), d_perm.get(), n * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_flags.data(), d_flags.get(), n, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_permp, d_perm.get(), n * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(h_flags, d_flags.get(), n, cudaMemcpyDeviceToHost, st));
   std::vector<int64_t> h_body(Pl);
   GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
+  HT("fin_d2h");
   if (graph_mode) {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
     int64_t ex = n_branches;  // one final selection per split-path branch
     for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_per_pair[i];  // counted at each branch's first pair
@@ -1120,7 +1160,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   mdl->eps = eps;
   mdl->n = n;
   mdl->class_count.assign(cc.begin(), cc.begin() + k);
-  mdl->perm = std::move(h_perm);
+  mdl->perm.assign(h_permp, h_permp + n);
   mdl->trained.assign(P, 0);
   mdl->b.assign(P, 0.0);
   mdl->A.assign(P, 0.0);
@@ -1151,6 +1191,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   std::vector<int64_t> row_of_sv(mdl->sv_pos.size());
   for (size_t i = 0; i < row_of_sv.size(); ++i) row_of_sv[i] = mdl->perm[mdl->sv_pos[i]];
   HT("assembled");
+  // the SV-row centre and scale are recomputed from the SV rows (not the training call's), so a
+  // model merged from partial trainings predicts bitwise like the single-call model
   mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st);
   tm.mark(PH_FIN);
   HT("devmodel");

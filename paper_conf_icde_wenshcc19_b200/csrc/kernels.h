@@ -35,6 +35,7 @@ float krow_split_scale(float maxabs);  // exact power-of-two scale of the FP16 s
 // centre by the column means (mean of the original rows; perm only reorders), scale, split into
 // hi/lo rows and compute the squared norms (scaled units); returns the scale
 size_t krow_tc_scratch_bytes(int64_t n, int d);
+const float* krow_tc_scratch_mu(const void* scratch, int64_t n, int d);
 float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
                         int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)

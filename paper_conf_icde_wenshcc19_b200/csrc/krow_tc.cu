@@ -529,7 +529,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 
 // column means of the rows idx[0..n) of X (idx < 0: skipped): per-chunk FP64 partials, then a
 // fixed-order sum over the chunks (deterministic)
-constexpr int kGatherMeanRows = 256;
+constexpr int kGatherMeanRows = 256;  // rows per partial
+constexpr int kGatherBatch = 32;     // loads in flight per thread
 __global__ void gather_col_partial_kernel(const float* __restrict__ X, int d, const int64_t* __restrict__ idx,
                                           int64_t n, double* __restrict__ part) {
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -537,9 +538,15 @@ __global__ void gather_col_partial_kernel(const float* __restrict__ X, int d, co
   const int64_t i0 = (int64_t)blockIdx.y * kGatherMeanRows;
   const int64_t i1 = (n < i0 + kGatherMeanRows) ? n : i0 + kGatherMeanRows;
   double s = 0.0;
-  for (int64_t i = i0; i < i1; ++i) {
-    const int64_t r = idx[i];
-    if (r >= 0) s += X[r * d + c];
+  for (int64_t b = i0; b < i1; b += kGatherBatch) {
+    float v[kGatherBatch];  // a batch of loads in flight before its (fixed-order) sum
+#pragma unroll
+    for (int j = 0; j < kGatherBatch; ++j) {
+      const int64_t r = b + j < i1 ? idx[b + j] : -1;
+      v[j] = r >= 0 ? X[r * d + c] : 0.f;
+    }
+#pragma unroll
+    for (int j = 0; j < kGatherBatch; ++j) s += v[j];
   }
   part[(int64_t)blockIdx.y * d + c] = s;
 }
@@ -672,6 +679,9 @@ float krow_split_scale(float maxabs) {  // power of two with maxabs * s <= 2^12 
   return (float)std::ldexp(1.0, e);
 }
 
+const float* krow_tc_scratch_mu(const void* scratch, int64_t n, int d) {  // the column means launch_split_tf32 left
+  return reinterpret_cast<const float*>(static_cast<const double*>(scratch) + (size_t)ceil_div(n, kMeanRows) * d);
+}
 size_t krow_tc_scratch_bytes(int64_t n, int d) {
   return (size_t)ceil_div(n, kMeanRows) * d * sizeof(double) + (size_t)d * sizeof(float) + 16;
 }
