@@ -1143,7 +1143,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     double fs[5] = {0, 0, 0, 0, 0};
     for (int i = 0; i < Pl; ++i)
       for (int q = 0; q < 5; ++q) fs[q] += (double)fq[i * 5 + q];
-    fprintf(stderr, "[gmpsvm] fast select cycles/launch: hist %.0f  scan %.0f  compact %.0f  sort+take %.0f  list %.1f\n",
+    fprintf(stderr, "[gmpsvm] fast select cycles/launch: staging %.0f  thresholds %.0f  compact %.0f  ranks %.0f  write-out %.0f (fallbacks x1e6)\n",
             fs[0] / outer, fs[1] / outer, fs[2] / outer, fs[3] / outer, fs[4] / outer);
     std::string per;
     for (int i = 0; i < Pl; ++i)

@@ -35,6 +35,10 @@ constexpr int kWMaxB = 224;      // working-set rows (tile in the SMO kernel's s
 constexpr int kBufW = 16;        // per-warp candidate buffer (per side)
 constexpr int kFlat = 512;       // flattened candidate list capacity (per side)
 constexpr int kWRank = 128;      // threshold samples per side (4 per warp)
+#ifndef GMPSVM_STAGE_UNROLL
+#define GMPSVM_STAGE_UNROLL 4
+#endif
+constexpr int kStageUnroll = GMPSVM_STAGE_UNROLL;  // staging: elements (alpha + f loads) in flight per thread
 
 __host__ __device__ inline int ws_tile_ld(int B) { return (B + 3) & ~3; }
 
@@ -82,6 +86,20 @@ __device__ __forceinline__ int warp_min_ki(uint64_t& k, int32_t& i) {
   k = ((uint64_t)m0 << 32) | m1;
   i = (int32_t)m2;
   return __ffs(b) - 1;
+}
+
+// Threads per list entry for a rank count over n entries by the whole CTA: the largest power of
+// two g <= 32 with n * g <= kWT (g lanes of one warp share an entry and split its comparisons).
+__device__ __forceinline__ int rank_group(int n) {
+  int g = 32;
+  while (g > 1 && n * g > kWT) g >>= 1;
+  return g;
+}
+__device__ __forceinline__ int group_sum(int v, int g) {  // sum over the g-lane group (g | 32)
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1)
+    if (o < g) v += __shfl_xor_sync(FULLMASK, v, o);
+  return v;
 }
 
 // exclusive prefix over the block of one value per thread (block order = thread order)
@@ -204,16 +222,16 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
   double fmin = DBL_MAX, fmax = -DBL_MAX;
   uint64_t mk[2] = {~0ull, ~0ull};
   int32_t mi[2] = {INT_MAX, INT_MAX};
-  for (int base = 0; base < np; base += 4 * kWT) {
-    double av[4], fv[4];
+  for (int base = 0; base < np; base += kStageUnroll * kWT) {
+    double av[kStageUnroll], fv[kStageUnroll];
 #pragma unroll
-    for (int m = 0; m < 4; ++m) {
+    for (int m = 0; m < kStageUnroll; ++m) {
       const int i = base + m * kWT + t;
       av[m] = i < np ? al[i] : 0.0;
       fv[m] = i < np ? fl[i] : 0.0;
     }
 #pragma unroll
-    for (int m = 0; m < 4; ++m) {
+    for (int m = 0; m < kStageUnroll; ++m) {
       const int i = base + m * kWT + t;
       if (i < np) {
         const int y = i < pd.n_s ? 1 : -1;
@@ -294,23 +312,27 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
   }
   __syncthreads();
   // thresholds by counting ranks: U at rank need_u - 1, L at rank need - 1 (so the L list
-  // still holds need - (U picks) candidates after removing the U picks it shares)
-  if (t < 2 * kWRank) {
-    const int s = t / kWRank, j = t % kWRank;
+  // still holds need - (U picks) candidates after removing the U picks it shares); 4 threads per
+  // sample split its comparisons
+  {
+    constexpr int G = kWT / (2 * kWRank);
+    const int e = t / G, sub = t % G;
+    const int s = e / kWRank, j = e % kWRank;
     const int r = s == 0 ? need_u : need;
     const uint64_t k = W.sk[s][j];
     const int32_t x = W.si[s][j];
-    if (x != INT_MAX && r >= 1 && r <= kWRank) {
-      int rank = 0;
-      for (int q = 0; q < kWRank; ++q) rank += kless(W.sk[s][q], W.si[s][q], k, x) ? 1 : 0;
-      if (rank == r - 1) {
+    int rank = 0;
+    for (int q = sub; q < kWRank; q += G) rank += kless(W.sk[s][q], W.si[s][q], k, x) ? 1 : 0;
+    rank = group_sum(rank, G);
+    if (sub == 0) {
+      if (x != INT_MAX && r >= 1 && r <= kWRank && rank == r - 1) {
         W.thr_k[s] = k;
         W.thr_i[s] = x;
       }
-    }
-    if (s == 0 && j == 0 && r == 0) {  // nothing wanted from U
-      W.thr_k[0] = 0ull;
-      W.thr_i[0] = -1;
+      if (s == 0 && j == 0 && r == 0) {  // nothing wanted from U
+        W.thr_k[0] = 0ull;
+        W.thr_i[0] = -1;
+      }
     }
   }
   __syncthreads();
@@ -366,6 +388,7 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
   }
   __syncthreads();
   int got = 0;
+  mark(2);
   if (!W.overflow) {
     {  // flatten: thread (warp w, lane j) copies slot j of warp w's U (j < 16) or L (j >= 16) buffer
       const int s = lane >> 4, j = lane & 15;
@@ -377,35 +400,45 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
     }
     __syncthreads();
     const int nu = W.boff[0][32], nl = W.boff[1][32];
-    // U: exact (key, index) rank by counting; the need_u smallest in rank order
+    // U: exact (key, index) rank by counting (g threads per entry); the need_u smallest in rank order
     const int got_u = min(need_u, nu);
-    if (t < nu) {
-      const uint64_t k = W.fk[0][t];
-      const int32_t x = W.fi[0][t];
+    {
+      const int g = rank_group(nu), e = t / g, sub = t % g;
+      uint64_t k = 0;
+      int32_t x = 0;
       int rank = 0;
-      for (int q = 0; q < nu; ++q) rank += kless(W.fk[0][q], W.fi[0][q], k, x) ? 1 : 0;
-      if (rank < got_u) {
+      if (e < nu) {
+        k = W.fk[0][e];
+        x = W.fi[0][e];
+        for (int q = sub; q < nu; q += g) rank += kless(W.fk[0][q], W.fi[0][q], k, x) ? 1 : 0;
+      }
+      rank = group_sum(rank, g);
+      if (e < nu && sub == 0 && rank < got_u) {
         W.pick[keep + rank] = x;
         flags[x] |= 4;
       }
     }
     __syncthreads();
-    // L: rank among the entries U did not take (threads 512.. while U's threads are idle)
+    // L: rank among the entries U did not take
     const int need_l = need - got_u;
-    const int tl = t - 512;
     bool free_l = false;
-    if (tl >= 0 && tl < nl) {
-      const uint64_t k = W.fk[1][tl];
-      const int32_t x = W.fi[1][tl];
-      free_l = !(flags[x] & 4);
-      if (free_l) {
-        int rank = 0;
-        for (int q = 0; q < nl; ++q) {
-          const int32_t xq = W.fi[1][q];
-          rank += (!(flags[xq] & 4) && kless(W.fk[1][q], xq, k, x)) ? 1 : 0;
-        }
-        if (rank < need_l) W.pick[keep + got_u + rank] = x;
+    {
+      const int g = rank_group(nl), e = t / g, sub = t % g;
+      int rank = 0;
+      int32_t x = 0;
+      if (e < nl) {
+        const uint64_t k = W.fk[1][e];
+        x = W.fi[1][e];
+        free_l = !(flags[x] & 4);
+        if (free_l)
+          for (int q = sub; q < nl; q += g) {
+            const int32_t xq = W.fi[1][q];
+            rank += (!(flags[xq] & 4) && kless(W.fk[1][q], xq, k, x)) ? 1 : 0;
+          }
       }
+      rank = group_sum(rank, g);
+      free_l = free_l && sub == 0;
+      if (free_l && rank < need_l) W.pick[keep + got_u + rank] = x;
     }
     const int nfree = __syncthreads_count(free_l);
     got = got_u + min(need_l, nfree);
@@ -415,13 +448,13 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
     if (got < need) got += radix_pick<true>(SmemSrc{keys, flags}, np, need - got, W.pick + keep + got, W.sel);
   } else {  // a buffer overflowed (heavily tied or clustered keys): exact radix selection
     got = select_sides(SmemSrc{keys, flags}, np, need, W.pick + keep, W.sel);
-    if (a.sel_phase && t == 0) a.sel_phase[(int64_t)(lp + 4096) * 5 + 4] += 1;  // fallbacks (diagnostic)
+    if (a.sel_phase && t == 0) a.sel_phase[(int64_t)(lp + 4096) * 5 + 4] += 1000000;  // fallbacks (diagnostic)
   }
   __syncthreads();
-  mark(2);
+  mark(3);
   const int cnt = keep + got;
   ws_write_out(a, lp, W.pick, cnt, W.retained, W.wpre, W.boff[0]);
-  mark(3);
+  mark(4);
 }
 
 // ------------------------------------------------------------------------------------------
