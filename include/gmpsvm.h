@@ -59,7 +59,7 @@ enum {
 typedef struct {
   int32_t struct_size;      /* sizeof(gmpsvm_options); 0 is accepted as "current"           */
   int32_t ws_size;          /* B: working-set = kernel-buffer rows per pair (L299-L303, L377);
-                               default 224 (K_ws,ws then lives in shared memory; the paper's
+                               default 192 (K_ws,ws then lives in shared memory; the paper's
                                1024 is a tuning point); must be even, 2..1024     */
   int32_t q;                /* new violators per outer iteration (L289, L297); default B/2;
                                the newest B-q rows of the previous working set are kept     */
