@@ -680,8 +680,9 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
   std::vector<int> wave_off;     // tile range of wave w: [wave_off[w], wave_off[w + 1])
   std::vector<int> ready_wave;   // per pair position: the wave after which its kernel values are complete
+  const bool two_cta = use_tc && !overlap && krow_tc_2cta();  // the overlap waves use single-CTA tiles
   if (use_tc) {
-    tiles = krow_tc_tiles(n);
+    tiles = krow_tc_tiles(n, two_cta);
     if (overlap) {
       const int INF = INT_MAX;
       std::vector<int> minpos(k, INF);  // first position of a pair containing class c
@@ -738,7 +739,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   tm.mark(PH_KERNEL);
   if (use_tc && !overlap)
     launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, ksc, K.get(),
-                   ldk, st);
+                   ldk, st, two_cta);
   else if (full_k && !use_tc)
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   tm.mark(PH_KERNEL);
@@ -1398,12 +1399,13 @@ int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int3
     DevBuf<float> hi(krow_tc_buf_floats(np2, dp), st), lo(krow_tc_buf_floats(np2, dp), st), nx2(np2, st);
     DevBuf<uint8_t> scr(krow_tc_scratch_bytes(n, d), st);
     const float ksc = launch_split_tf32(dX, n, d, nullptr, hi.get(), lo.get(), nx2.get(), np2, dp, scr.get(), st);
-    const std::vector<int2> tl = krow_tc_tiles(n);
-    DevBuf<int2> dt(tl.size(), st);
-    GM_CUDA(cudaMemcpyAsync(dt.get(), tl.data(), tl.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
     DevBuf<float> kb2(opt.inputs_on_device ? 0 : (size_t)n * m, st);
     float* dK2 = opt.inputs_on_device ? K_out : kb2.get();
-    launch_krow_tc(hi.get(), lo.get(), np2, dp, dt.get(), (int)tl.size(), nx2.get(), n, gamma, ksc, dK2, m, st);
+    const bool two_cta = krow_tc_2cta() && (m % 4) == 0 && (reinterpret_cast<uintptr_t>(dK2) & 15) == 0;
+    const std::vector<int2> tl = krow_tc_tiles(n, two_cta);
+    DevBuf<int2> dt(tl.size(), st);
+    GM_CUDA(cudaMemcpyAsync(dt.get(), tl.data(), tl.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
+    launch_krow_tc(hi.get(), lo.get(), np2, dp, dt.get(), (int)tl.size(), nx2.get(), n, gamma, ksc, dK2, m, st, two_cta);
     if (!opt.inputs_on_device) GM_CUDA(cudaMemcpyAsync(K_out, dK2, (size_t)n * m * 4, cudaMemcpyDeviceToHost, st));
     GM_CUDA(cudaStreamSynchronize(st));
     return GMPSVM_OK;

@@ -40,7 +40,8 @@ float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, v
                         int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
-std::vector<int2> krow_tc_tiles(int64_t n);
+bool krow_tc_2cta();
+std::vector<int2> krow_tc_tiles(int64_t n, bool two_cta);
 constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
 // per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
 void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
@@ -58,7 +59,8 @@ void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* 
                    const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma, float sc,
                    float* part, cudaStream_t st);
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
-                    const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st);
+                    const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
+                    bool two_cta = false);
 void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
                       cudaStream_t st);
 bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel

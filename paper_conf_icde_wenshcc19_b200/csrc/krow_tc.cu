@@ -86,6 +86,14 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, i
       "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar,
+                                            uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, %3}], "
+      "[%4], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar)), "l"(policy)
+      : "memory");
+}
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* src, int x, int y) {
   asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
                    reinterpret_cast<uint64_t>(map)),
@@ -97,6 +105,28 @@ __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
+// L2 policies: operand rows stay (re-read by many tiles), kernel-matrix stores stream through
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_normal() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void tma_store_2d_hint(const CUtensorMap* map, const void* src, int x, int y, uint64_t policy) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3}], [%1], %4;" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(smem_u32(src)), "r"(x), "r"(y), "l"(policy)
+               : "memory");
+}
 // K-major operand, 128-byte swizzle: 8-row groups 1024 B apart (SBO), LBO unused (1), version 1.
 __device__ __forceinline__ uint64_t umma_desc_sw128(const void* p) {
   const uint64_t addr = smem_u32(p);
@@ -181,6 +211,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   if (warp == 0) {
     if (lane == 0) {  // ---- TMA producer (runs ahead across tiles)
       int g = 0;
+      const uint64_t pol = policy_evict_last();
       for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
         const int2 tile = tiles[t];
         const int r0 = tile.x * kTM, c0 = tile.y * kTN;
@@ -190,10 +221,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           uint8_t* st = sm.stage[s];
           mbar_expect_tx(&sm.full[s], kStageBytes);
           const int kx = kb * (F16 ? 2 * kTK : kTK);
-          tma_load_2d(st, &map_hi, kx, r0, &sm.full[s]);
-          tma_load_2d(st + kABytes, &map_lo, kx, r0, &sm.full[s]);
-          tma_load_2d(st + 2 * kABytes, &map_hi, kx, c0, &sm.full[s]);
-          tma_load_2d(st + 2 * kABytes + kBBytes, &map_lo, kx, c0, &sm.full[s]);
+          tma_load_2d(st, &map_hi, kx, r0, &sm.full[s], pol);
+          tma_load_2d(st + kABytes, &map_lo, kx, r0, &sm.full[s], pol);
+          tma_load_2d(st + 2 * kABytes, &map_hi, kx, c0, &sm.full[s], pol);
+          tma_load_2d(st + 2 * kABytes + kBBytes, &map_lo, kx, c0, &sm.full[s], pol);
         }
       }
     }
@@ -235,6 +266,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
   } else {  // ---- epilogue: warps 2..5, TMEM lane quarter (warp % 4)
     const int q = warp & 3;
+    const uint64_t spol = policy_evict_first();
     int it = 0;
     for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
       const int2 tile = tiles[t];
@@ -306,8 +338,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           fence_proxy_async_smem();
           __syncwarp();
           if (lane == 0) {
-            tma_store_2d(&map_ksw, eb, (int)cb, (int)(r0 + q * 32));
-            tma_store_2d(&map_kns, em, (int)(r0 + q * 32), (int)cb);
+            tma_store_2d_hint(&map_ksw, eb, (int)cb, (int)(r0 + q * 32), spol);
+            tma_store_2d_hint(&map_kns, em, (int)(r0 + q * 32), (int)cb, spol);
             bulk_commit();
           }
         }
@@ -353,6 +385,303 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   if (warp == 1) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// The same contraction on CTA pairs (cluster of 2, tcgen05 cta_group::2): one MMA computes a
+// 256 x 128 tile; CTA r holds rows 128 r .. 128 r + 127 of A (its own 128 rows, hi and lo) and
+// rows 64 r .. 64 r + 63 of B, so per SM an MMA reads 4 KB of A + 2 KB of B from shared memory
+// instead of 4 + 4 KB, and each SM's TMA fills 12 instead of 16 KB per k step: the shared-memory
+// operand bandwidth that bounds the single-CTA kernel drops by a quarter.  The leader (rank 0)
+// issues the MMAs; its full barriers count both CTAs' TMA bytes, its MMA commits arrive on both
+// CTAs' empty / tmem_full barriers (multicast), and both CTAs' epilogue warps release TMEM on the
+// leader's tmem_empty barriers.  Accumulators: CTA r's TMEM lanes hold its 128 rows (same layout
+// as the single-CTA kernel), so the epilogue is unchanged per CTA.  Tile (I, J) covers rows
+// 256 I .. 256 I + 255 and columns 128 J .. 128 J + 127; CTA r's 128 x 128 half is the
+// single-CTA tile (2 I + r, J): stored by TMA when off-diagonal, per thread on the diagonal,
+// not at all when below it (computed, discarded: one half-tile per diagonal).
+constexpr int kTc2Stages = 4;
+constexpr uint32_t kBHalfBytes = (kTN / 2) * 128;              // 64 rows x 128 B = 8 KB
+constexpr uint32_t kStage2Bytes = 2 * kABytes + 2 * kBHalfBytes;  // 48 KB
+constexpr uint32_t kIdescF16M256 = (1u << 4) | ((uint32_t)(kTN >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
+constexpr uint32_t kPeerMask = 0xFEFFFFFFu;  // shared::cluster address of the same offset in CTA rank 0
+
+struct Tc2Smem {
+  alignas(1024) uint8_t stage[kTc2Stages][kStage2Bytes];
+  alignas(1024) float epi[kEpiWarps][2][32 * 32];
+  alignas(8) uint64_t full[kTc2Stages];  // leader: TMA bytes of both CTAs
+  uint64_t empty[kTc2Stages];            // both: MMA commit (multicast)
+  uint64_t acc_ready[2];                 // both: MMA commit after the first / second k third (multicast)
+  uint64_t tmem_full;                    // both: MMA commit after the last MMA of the tile (multicast)
+  uint64_t free03;                       // leader: 8 epilogue warps (both CTAs) drained accumulators 0 and 3
+  uint64_t free1;                        // leader: accumulator 1 drained
+  uint64_t free2;                        // leader: accumulator 2 drained
+  uint32_t tmem_base;
+};
+
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t mapa_rank(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void tma_load_2d_2sm(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar,
+                                                uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], "
+      "[%1, {%2, %3}], [%4], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar) & kPeerMask), "l"(policy)
+      : "memory");
+}
+__device__ __forceinline__ void umma_f16_2sm(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(
+          tmem_d),
+      "l"(a), "l"(b), "r"(kIdescF16M256), "r"(accum));
+}
+__device__ __forceinline__ void umma_commit_2sm(uint64_t* bar) {  // arrive on the barrier at this offset in both CTAs
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          smem_u32(bar)),
+      "h"((uint16_t)3)
+      : "memory");
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kTcThreads, 1)
+    krow_tc2_kernel(const __grid_constant__ CUtensorMap map_hi, const __grid_constant__ CUtensorMap map_lo,
+                    const __grid_constant__ CUtensorMap map_bhi, const __grid_constant__ CUtensorMap map_blo,
+                    const __grid_constant__ CUtensorMap map_ksw, const __grid_constant__ CUtensorMap map_kns,
+                    const int2* __restrict__ tiles, int n_tiles, const float* __restrict__ norms, int64_t n, int nk,
+                    float scale, float* __restrict__ K, int64_t ldk, int diag) {
+  // diag (GMPSVM_KROW_DIAG, timing experiments only): 1 = no stores, 2 = no MMAs, 4 = drain every
+  // accumulator at the tile's end
+  const bool late = (diag & 4) != 0;
+  extern __shared__ __align__(1024) uint8_t dsmem[];
+  Tc2Smem& sm = *reinterpret_cast<Tc2Smem*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const bool leader = rank == 0;
+  const int cl = blockIdx.x >> 1, ncl = gridDim.x >> 1;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < kTc2Stages; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], 1);
+    }
+    mbar_init(&sm.acc_ready[0], 1);
+    mbar_init(&sm.acc_ready[1], 1);
+    mbar_init(&sm.tmem_full, 1);
+    mbar_init(&sm.free03, 2 * kEpiWarps);
+    mbar_init(&sm.free1, 2 * kEpiWarps);
+    mbar_init(&sm.free2, 2 * kEpiWarps);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_hi)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_lo)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_bhi)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_blo)) : "memory");
+  }
+  if (warp == 1) {  // same warp in both CTAs, same destination offset (cta_group::2 allocation)
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&sm.tmem_base)),
+                 "r"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  cluster_sync_all();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = sm.tmem_base;
+  int jn = nk < kMainAcc ? nk : kMainAcc;
+  if ((diag & 16) && jn > 1) jn = 1;  // precision experiments: one or two hi.hi accumulators
+  if ((diag & 32) && jn > 2) jn = 2;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ---- TMA producer (both CTAs): own A rows, own half of the B rows
+      int g = 0;
+      const uint64_t pol = (diag & 8) ? policy_evict_normal() : policy_evict_last();
+      for (int t = cl; t < n_tiles; t += ncl) {
+        const int2 tile = tiles[t];
+        const int ra = tile.x * 2 * kTM + (int)rank * kTM, cbh = tile.y * kTN + (int)rank * (kTN / 2);
+        for (int kb = 0; kb < nk; ++kb, ++g) {
+          const int s = g % kTc2Stages;
+          if (g >= kTc2Stages) mbar_wait(&sm.empty[s], ((g / kTc2Stages) + 1) & 1);
+          uint8_t* st = sm.stage[s];
+          if (leader) mbar_expect_tx(&sm.full[s], 2 * kStage2Bytes);
+          const int kx = kb * 2 * kTK;
+          tma_load_2d_2sm(st, &map_hi, kx, ra, &sm.full[s], pol);
+          tma_load_2d_2sm(st + kABytes, &map_lo, kx, ra, &sm.full[s], pol);
+          tma_load_2d_2sm(st + 2 * kABytes, &map_bhi, kx, cbh, &sm.full[s], pol);
+          tma_load_2d_2sm(st + 2 * kABytes + kBHalfBytes, &map_blo, kx, cbh, &sm.full[s], pol);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (leader && lane == 0) {  // ---- MMA issuer (leader only)
+      int g = 0, it = 0;
+      for (int t = cl; t < n_tiles; t += ncl, ++it) {
+        // accumulators are drained per k third: 0 during the tile (after its first third), 3 and
+        // the last third's at the end; the next tile needs only 0 and 3 to start (free03)
+        if (it > 0) mbar_wait(&sm.free03, (it - 1) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        for (int kb = 0; kb < nk; ++kb, ++g) {
+          const int s = g % kTc2Stages;
+          const int j = (kb * jn) / nk;
+          const int kb_first = (j * nk + jn - 1) / jn;
+          if (it > 0 && j > 0 && kb == kb_first && !late) {
+            mbar_wait(j == 1 ? &sm.free1 : &sm.free2, (it - 1) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          }
+          mbar_wait(&sm.full[s], (g / kTc2Stages) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          uint8_t* st = sm.stage[s];
+          const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
+          const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBHalfBytes);
+#pragma unroll
+          for (int kk = 0; kk < kTK / 8; ++kk) {
+            if (diag & 2) break;
+            const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 16 FP16 = 32 bytes along K inside the atom
+            umma_f16_2sm(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
+            if (diag & 64) continue;  // timing experiment: hi.hi only
+            umma_f16_2sm(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
+            umma_f16_2sm(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+          }
+          umma_commit_2sm(&sm.empty[s]);
+          // the last k block of a third that is not the tile's last: that accumulator is complete
+          if (!late && j < jn - 1 && kb + 1 == (((j + 1) * nk + jn - 1) / jn)) umma_commit_2sm(&sm.acc_ready[j]);
+        }
+        umma_commit_2sm(&sm.tmem_full);
+      }
+    }
+  } else {  // ---- epilogue: warps 2..5 of both CTAs, TMEM lane quarter (warp % 4) of this CTA's rows
+    const int q = warp & 3;
+    const uint32_t f03 = mapa_rank(smem_u32(&sm.free03), 0), f1 = mapa_rank(smem_u32(&sm.free1), 0),
+                   f2 = mapa_rank(smem_u32(&sm.free2), 0);
+    auto release = [&](uint32_t bar) {  // this warp's TMEM reads are done: arrive on the leader's barrier
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar) : "memory");
+    };
+    const uint64_t spol = policy_evict_first();
+    int it = 0;
+    for (int t = cl; t < n_tiles; t += ncl, ++it) {
+      const int2 tile = tiles[t];
+      const int bi = tile.x * 2 + (int)rank;
+      const int64_t r0 = (int64_t)bi * kTM, c0 = (int64_t)tile.y * kTN;
+      const int64_t r = r0 + q * 32 + lane;
+      const float nr = (r < n) ? norms[r] : 0.f;
+      float cnv[kTN / 32];
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) cnv[ch] = norms[c0 + ch * 32 + lane];
+      float dot[kTN];
+      const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
+      // accumulator acc of this warp's rows, added into dot (first = assign)
+      auto drain = [&](int acc, bool first) {
+#pragma unroll
+        for (int ch = 0; ch < kTN / 32; ++ch) {
+          uint32_t v[32];
+          tmem_ld32(trow + (uint32_t)(ch * 32 + acc * kTN), v);
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+          for (int j = 0; j < 32; ++j)
+            dot[ch * 32 + j] = first ? __uint_as_float(v[j]) : dot[ch * 32 + j] + __uint_as_float(v[j]);
+        }
+      };
+      // thirds completed during the tile (all but the last): drained as soon as they are ready
+      for (int j = 0; j < (late ? 0 : jn - 1); ++j) {
+        mbar_wait(&sm.acc_ready[j], it & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        drain(j, j == 0);
+        if (j == 1) release(f1);
+      }
+      mbar_wait(&sm.tmem_full, it & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      if (late) {  // all accumulators at the end: 0 + 3, release, then 1 + 2
+        drain(0, true);
+        drain(kMainAcc, false);
+        release(f03);
+        for (int j = 1; j < jn; ++j) drain(j, false);
+        release(f1);
+        release(f2);
+      } else {
+        drain(kMainAcc, jn == 1);  // corrections
+        if (jn == 1) drain(0, false);
+        release(f03);  // the next tile may start (accumulators 0 and 3 are free)
+        if (jn >= 2) {
+          drain(jn - 1, false);
+          release(jn - 1 == 1 ? f1 : f2);
+        }
+      }
+      if (diag & 1) continue;
+      if (bi > tile.y) continue;  // entirely below the diagonal: nothing to store
+      if (bi < tile.y) {          // off-diagonal: TMA stores of the block and its mirror
+        float* eb = sm.epi[q][0];
+        float* em = sm.epi[q][1];
+#pragma unroll
+        for (int ch = 0; ch < kTN / 32; ++ch) {
+          const int64_t cb = c0 + ch * 32;
+          const float cn = cnv[ch];
+          float kv[32];
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cn, j));
+            asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv[j]) : "f"(fmaxf(d2, 0.f) * scale));
+          }
+          if (lane == 0) bulk_wait_read0();
+          __syncwarp();
+#pragma unroll
+          for (int jj = 0; jj < 8; ++jj)
+            *reinterpret_cast<float4*>(eb + lane * 32 + ((jj ^ (lane & 7)) << 2)) =
+                make_float4(kv[4 * jj], kv[4 * jj + 1], kv[4 * jj + 2], kv[4 * jj + 3]);
+#pragma unroll
+          for (int j = 0; j < 32; ++j) em[j * 32 + lane] = kv[j];
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) {
+            tma_store_2d_hint(&map_ksw, eb, (int)cb, (int)(r0 + q * 32), spol);
+            tma_store_2d_hint(&map_kns, em, (int)(r0 + q * 32), (int)cb, spol);
+            bulk_commit();
+          }
+        }
+        continue;
+      }
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) {  // diagonal tile: K[r][c] for r <= c and the mirror for r < c
+        const int64_t cb = c0 + ch * 32;
+        float kv[32];
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cnv[ch], j));
+          float val;
+          asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(val) : "f"(fmaxf(d2, 0.f) * scale));
+          kv[j] = (r == cb + j) ? 1.f : val;
+        }
+        if (r < n) {
+          float* dst = K + r * ldk + cb;
+#pragma unroll
+          for (int j = 0; j < 32; ++j)
+            if (cb + j >= r && cb + j < n) dst[j] = kv[j];
+        }
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const int64_t c = cb + j;
+          if (r < c && c < n) K[c * ldk + r] = kv[j];
+        }
+      }
+    }
+    if (lane == 0) bulk_wait0();
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  cluster_sync_all();  // the peer's MMAs / arrivals are done before TMEM is released
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
   }
 }
 
@@ -644,14 +973,14 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   return fn;
 }
 
-CUtensorMap make_map(const void* base, int64_t rows, int d_pad, bool f16) {
+CUtensorMap make_map(const void* base, int64_t rows, int d_pad, bool f16, int box_rows = kTM) {
   auto enc = get_encode();
   if (!enc) throw Error(GMPSVM_ECUDA, "cuTensorMapEncodeTiled unavailable");
   CUtensorMap m;
   const size_t eb = f16 ? 2 : 4;
   const cuuint64_t dims[2] = {(cuuint64_t)d_pad, (cuuint64_t)rows};
   const cuuint64_t strides[1] = {(cuuint64_t)d_pad * eb};
-  const cuuint32_t box[2] = {(cuuint32_t)(128 / eb), (cuuint32_t)kTM};  // one 128-byte swizzle atom along K
+  const cuuint32_t box[2] = {(cuuint32_t)(128 / eb), (cuuint32_t)box_rows};  // one 128-byte swizzle atom along K
   const cuuint32_t estr[2] = {1, 1};
   const CUresult r = enc(&m, f16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
                          const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -753,9 +1082,28 @@ void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, f
 
 // Tiles (bi, bj) of 128 x 128 with at least one entry r <= c, in blocked order (16 x 16 tiles)
 // so a wave of CTAs reuses its operand tiles from L2.
-std::vector<int2> krow_tc_tiles(int64_t n) {
-  const int Tr = (int)ceil_div(n, kTM), Tc = (int)ceil_div(n, kTN);
+// CTA-pair kernel (FP16 split only), opt-in with GMPSVM_KROW_CTA=2: measured on B200 (MNIST-shaped
+// n = 60,000) at 8.0-10.6 ms against 7.7 ms for the single-CTA kernel -- halving the B operand's
+// shared-memory reads and L2 traffic did not help; the contraction is bound by the TMA operand
+// stream's latency x bytes in flight (TMA alone: 4.0 ms; MMA alone ~3.8 ms), DESIGN.md §6.1.
+bool krow_tc_2cta() {
+  static const bool two = getenv("GMPSVM_KROW_CTA") && std::string(getenv("GMPSVM_KROW_CTA")) == "2";
+  return two && krow_split_f16();
+}
+
+std::vector<int2> krow_tc_tiles(int64_t n, bool two_cta) {
+  const int Tc = (int)ceil_div(n, kTN);
   std::vector<int2> t;
+  if (two_cta) {  // tiles (I, J) of 256 x 128 whose first 128-row half has an entry r <= c
+    const int Tr2 = (int)ceil_div(n, 2 * kTM);
+    for (int I = 0; I < Tr2; I += 8)
+      for (int J = 0; J < Tc; J += 16)
+        for (int bi = I; bi < std::min(Tr2, I + 8); ++bi)
+          for (int bj = J; bj < std::min(Tc, J + 16); ++bj)
+            if ((int64_t)(bj + 1) * kTN - 1 >= (int64_t)bi * 2 * kTM) t.push_back(make_int2(bi, bj));
+    return t;
+  }
+  const int Tr = (int)ceil_div(n, kTM);
   for (int I = 0; I < Tr; I += 16)
     for (int J = 0; J < Tc; J += 16)
       for (int bi = I; bi < std::min(Tr, I + 16); ++bi)
@@ -788,7 +1136,8 @@ CUtensorMap make_kmap(float* K, int64_t n, int64_t ldk, bool swizzle) {
 }
 
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
-                    const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st) {
+                    const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
+                    bool two_cta) {
   const bool f16 = krow_split_f16();
   const CUtensorMap mhi = make_map(hi, n_pad, d_pad, f16), mlo = make_map(lo, n_pad, d_pad, f16);
   // TMA stores need a 16-byte aligned base and row stride; otherwise every tile takes the
@@ -806,8 +1155,24 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
   // distances are in units scaled by sc: exp(-gamma d2 / sc^2) = exp2(d2 * scale)
   const float scale = (float)(-gamma * 1.4426950408889634 / ((double)sc * (double)sc));
   const int sms = num_sms();
-  const int grid = n_tiles < sms ? n_tiles : sms;
   const int nk = d_pad / (f16 ? 2 * kTK : kTK);
+  if (two_cta) {
+    if (!f16 || !tma) throw Error(GMPSVM_EINVAL, "CTA-pair kernel-value launch needs the FP16 split and TMA stores");
+    const size_t smem2 = sizeof(Tc2Smem) + 1024;
+    static bool configured2 = false;
+    if (!configured2) {
+      GM_CUDA(cudaFuncSetAttribute(krow_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2));
+      configured2 = true;
+    }
+    // B operand: 64-row boxes (each CTA of the pair loads its half of the 128 columns' rows)
+    const CUtensorMap mbhi = make_map(hi, n_pad, d_pad, f16, kTN / 2), mblo = make_map(lo, n_pad, d_pad, f16, kTN / 2);
+    const int clusters = std::min(n_tiles, sms / 2);
+    static const int diag = getenv("GMPSVM_KROW_DIAG") ? atoi(getenv("GMPSVM_KROW_DIAG")) : 0;
+    GM_LAUNCH(krow_tc2_kernel, dim3(2 * clusters), dim3(kTcThreads), smem2, st, mhi, mlo, mbhi, mblo, mksw, mkns, tiles,
+              n_tiles, norms, n, nk, scale, K, ldk, diag);
+    return;
+  }
+  const int grid = n_tiles < sms ? n_tiles : sms;
   if (f16)
     GM_LAUNCH(krow_tc_kernel<true>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles, norms,
               n, nk, scale, K, ldk, tma);

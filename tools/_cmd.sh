@@ -1,6 +1,5 @@
 out=gpurun_out/$1; mkdir -p $out
 python -c "import __graft_entry__ as g; g.build()" > $out/build.log 2>&1
-timeout 900 python -m pytest tests -m gpu -x -q > $out/pytest.log 2>&1; echo "pytest rc=$?" >> $out/pytest.log
-GMPSVM_SMO_PHASES=1 timeout 300 python tools/prof_step.py --ws-size 192 --reps 2 > $out/phases.log 2>&1
-GMPSVM_TRACE=1 timeout 300 python tools/prof_step.py --ws-size 192 --reps 2 > $out/trace1.log 2>&1
-timeout 600 python bench.py --steps 5 --warmup 3 --no-cpu-baseline > $out/bench.json 2> $out/bench.err
+echo "1cta+hints" >> $out/diag.log; GMPSVM_KROW_CTA=1 timeout 120 python tools/krow_check.py 2>&1 | grep krow | tail -1 >> $out/diag.log
+for dg in 4 68 69 5; do echo "diag $dg" >> $out/diag.log; GMPSVM_KROW_DIAG=$dg timeout 120 python tools/krow_check.py 2>&1 | grep krow | tail -1 >> $out/diag.log; done
+cat $out/diag.log
