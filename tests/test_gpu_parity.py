@@ -66,6 +66,28 @@ def test_rbf_kernel_symmetric_full_k_vs_oracle(gm, n, d, gamma):
     assert _rel_ok(K, oracle.rbf_matrix(X, X, gamma))
 
 
+@pytest.mark.parametrize("n,d,gamma", [(1000, 784, 0.125), (513, 16, 0.5), (300, 8, 0.5)])
+def test_rbf_kernel_cta_pair_variant(gm, tmp_path, n, d, gamma):
+    """The opt-in CTA-pair (cta_group::2) kernel-value launch (GMPSVM_KROW_CTA=2, read once per
+    process, hence the subprocess): same tolerance, exact symmetry and K_ii = 1."""
+    import os
+    import subprocess
+    import sys
+
+    if d == 784:
+        _, X, _, _, _ = datagen.make_config("mnist", n_train=n, n_test=1)
+    else:
+        X = np.random.default_rng(n).normal(0, 0.5, size=(n, d)).astype(np.float32)
+    np.save(tmp_path / "x.npy", X)
+    code = (f"import sys, numpy as np; sys.path.insert(0, {ROOT!r}); import paper_conf_icde_wenshcc19_b200 as gm; "
+            f"X = np.load({str(tmp_path / 'x.npy')!r}); np.save({str(tmp_path / 'k.npy')!r}, gm.rbf_kernel(X, X, {gamma}))")
+    subprocess.run([sys.executable, "-c", code], check=True, env=dict(os.environ, GMPSVM_KROW_CTA="2"), timeout=300)
+    K = np.load(tmp_path / "k.npy")
+    assert np.all(np.diag(K) == 1.0)
+    np.testing.assert_array_equal(K, K.T)
+    assert _rel_ok(K, oracle.rbf_matrix(X, X, gamma))
+
+
 def test_rbf_kernel_device_pointers(gm):
     X = np.random.default_rng(0).normal(size=(200, 30)).astype(np.float32)
     Xd = torch.from_numpy(X).cuda()
