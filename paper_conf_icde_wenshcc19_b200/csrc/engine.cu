@@ -755,7 +755,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
       d_outer(Pl, st), d_sig(Pl, st);
   DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
-  DevBuf<float> d_Kws((size_t)Pl * std::max<size_t>((size_t)Bw * Bw, ws_tile_floats(Bw)), st);
+  DevBuf<float> d_Kws((size_t)Pl * kws_pair_stride(Bw), st);
   const bool rc = !full_k;
   DevBuf<int32_t> d_slot(rc ? (size_t)Pl * Bw : 0, st), d_slot_tmp(rc ? (size_t)Pl * Bw : 0, st), d_keep(rc ? Pl : 0, st);
   DevBuf<float> d_ATnew(rc ? (size_t)Pl * d_pad * ldat : 0, st);

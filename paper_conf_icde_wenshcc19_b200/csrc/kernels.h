@@ -132,6 +132,13 @@ void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStrea
 // GMPSVM_WSOLVE=0 selects the select_ws / gather_kws / local_smo kernels of solver.cu)
 bool ws_solve_supported(int B, int64_t np_max);
 size_t ws_tile_floats(int B);  // per-pair floats of the Kws buffer (tile + SMO state)
+// Per-pair stride (floats) of the Kws buffer, the same for both solver paths: one graph may run
+// wsolve.cu pairs (tile with row stride round_up(B, 4) + alpha/f/index state) next to solver.cu
+// pairs (B x B tile), so every pair's slot must use this stride.
+__host__ __device__ inline size_t kws_pair_stride(int B) {
+  const size_t ld = (size_t)((B + 3) & ~3);
+  return (size_t)B * ld + 4 * (size_t)B + ld;
+}
 // one outer iteration: selection (+ stop test), K_ws,ws gather, single-warp local SMO, f-update
 // (with set_cond it sets the graph loop condition); programmatic dependent launches inside the
 // iteration, and across iterations when chained (the previous iteration is in the same stream)

@@ -439,7 +439,7 @@ __device__ void gather_rows_body(const SolverArgs& a, int lp, int r0, int r1, in
   const int64_t ldr = (pd.n_s + pd.n_t + 3) & ~3;
   for (int r = r0; r < r1; ++r) {
     const float* row = a.R ? a.R + pd.r_off + (int64_t)a.ws_slot[(int64_t)lp * a.B + r] * ldr : a.K + g[r] * a.ldk;
-    float* dst = a.Kws + ((int64_t)lp * a.B + r) * a.B;
+    float* dst = a.Kws + (int64_t)lp * kws_pair_stride(a.B) + (int64_t)r * a.B;
     for (int e = threadIdx.x; e < wn; e += blockDim.x) dst[e] = __ldg(row + g[e]);
   }
 }
@@ -567,14 +567,14 @@ __device__ void smo_body(const SolverArgs& a, int lp, int nt, int bar_id, RedSlo
   const float* Kw;
   if (SMEM) {
     // copy this pair's K_ws,ws tile (built by gather_kws, L2-resident) into shared memory
-    const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * B * B);
+    const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * kws_pair_stride(B));
     float4* dst = reinterpret_cast<float4*>(kw_smem);
     const int nv = (B * B) / 4;  // B is even and B*B % 4 == 0
     for (int i = threadIdx.x; i < nv; i += nt) dst[i] = __ldg(src + i);
     bar_sync(bar_id, nt);
     Kw = kw_smem;
   } else {
-    Kw = a.Kws + (int64_t)lp * B * B;
+    Kw = a.Kws + (int64_t)lp * kws_pair_stride(B);
   }
   bool valid[E], iu[E], il[E];
   int32_t idx[E];
@@ -981,7 +981,7 @@ __global__ void __launch_bounds__(256) local_smo_warp_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
   if (a.status[lp] != 0) return;
   const int B = a.B;
-  const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * B * B);
+  const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * kws_pair_stride(B));
   float4* dst = reinterpret_cast<float4*>(kw_smem);
   const int nv = (B * B) / 4;
   for (int i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);

@@ -19,6 +19,7 @@
 //                          memory; lane l owns working-set rows l, l+32, ...  Per inner step
 //                          (Eq 4-8, WSS2, local stop R20): per-lane min/max over its rows,
 //                          redux.sync over the warp -- no CTA barrier, no shared reduction slots.
+#include <algorithm>
 #include <cfloat>
 #include <climits>
 #include <cstdlib>
@@ -133,7 +134,7 @@ __device__ __forceinline__ int block_excl_scan_count_thread(int v, int& total, i
 // Kws buffer of a pair: the K_ws,ws tile (B rows, stride ld) followed by the local solver's
 // state in sorted order: alpha[B] (FP64), f[B] (FP64), index[round_up(B, 4)] (int32).
 __host__ __device__ inline size_t ws_state_off(int B) { return (size_t)B * ws_tile_ld(B); }  // in floats
-__host__ __device__ inline size_t ws_buf_floats(int B) { return ws_state_off(B) + 4 * (size_t)B + ((B + 3) & ~3); }
+__host__ __device__ inline size_t ws_buf_floats(int B) { return kws_pair_stride(B); }  // tile + state
 
 // exclusive prefix of the popcounts of nwords bitmap words (any blockDim); sm: 33 ints
 __device__ void bitmap_prefix(const uint32_t* bm, int nwords, int32_t* wpre, int* sm) {
@@ -879,7 +880,10 @@ __global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraph
 // ------------------------------------------------------------------------------------------
 bool ws_solve_supported(int B, int64_t np_max) {
   static const bool off = getenv("GMPSVM_WSOLVE") && std::string(getenv("GMPSVM_WSOLVE")) == "0";
-  return !off && B >= 2 && B <= kWMaxB && np_max <= kWMaxNp;
+  // GMPSVM_WS_MAXNP lowers the pair-size limit (tests: one graph mixing both solver paths)
+  static const int64_t lim =
+      getenv("GMPSVM_WS_MAXNP") ? std::min<int64_t>(kWMaxNp, atoll(getenv("GMPSVM_WS_MAXNP"))) : kWMaxNp;
+  return !off && B >= 2 && B <= kWMaxB && np_max <= lim;
 }
 
 size_t ws_tile_floats(int B) { return ws_buf_floats(B); }

@@ -279,3 +279,30 @@ def test_fused_and_split_solver_paths_agree(gm, tmp_path):
     subprocess.run([sys.executable, "-c", code], check=True, env=env, timeout=600)
     p2 = np.load(tmp_path / "p2.npy")
     assert np.abs(p1 - p2).max() <= 1e-4
+
+
+def test_mixed_solver_paths_in_one_graph(gm, tmp_path):
+    """Pairs above the wsolve.cu size limit run the solver.cu kernels in the same device-driven
+    graph as the others (covtype-shaped data: one 17k-instance pair next to small ones).  The
+    limit is lowered (GMPSVM_WS_MAXNP, read once per process: subprocess) so a small problem
+    mixes both paths; both must share the per-pair K_ws,ws slot stride (regression: mixed
+    strides overlapped slots and corrupted the working-set state) and reach the oracle's fixed
+    point (Eq 9)."""
+    import subprocess
+    import sys
+
+    spec, X, y, Xt, yt = datagen.make_config("mnist", n_train=2000, n_test=200)
+    ref = oracle.train(X, y, spec.k, spec.C, spec.gamma, EPS)
+    _, prob_o = oracle.predict(ref, X, y, Xt, want_dec=False)
+    sizes = sorted(int((y == s).sum() + (y == t).sum()) for s, t in oracle.pair_list(spec.k))
+    limit = sizes[len(sizes) // 2]  # about half of the pairs on each path
+    code = (
+        "import sys, numpy as np; sys.path.insert(0, %r); import datagen, paper_conf_icde_wenshcc19_b200 as gm;"
+        "spec, X, y, Xt, yt = datagen.make_config('mnist', n_train=2000, n_test=200);"
+        "m = gm.train(X, y, spec.k, spec.C, spec.gamma, %r, ws_size=96);"
+        "np.save(%r, m.predict_proba(Xt))" % (ROOT, EPS, str(tmp_path / "p.npy"))
+    )
+    env = dict(os.environ, GMPSVM_WS_MAXNP=str(limit))
+    subprocess.run([sys.executable, "-c", code], check=True, env=env, timeout=600)
+    p = np.load(tmp_path / "p.npy")
+    assert np.abs(p - prob_o).max() <= 1e-4
