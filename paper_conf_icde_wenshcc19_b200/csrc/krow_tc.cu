@@ -21,6 +21,7 @@
 #include <cuda_fp16.h>
 #include <cudaTypedefs.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdint>
 #include <cstdlib>
@@ -1172,7 +1173,10 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
               n_tiles, norms, n, nk, scale, K, ldk, diag);
     return;
   }
-  const int grid = n_tiles < sms ? n_tiles : sms;
+  // GMPSVM_KROW_RESERVE: SMs left free (the overlap mode's solver chains run beside the waves)
+  static const int reserve = getenv("GMPSVM_KROW_RESERVE") ? std::max(0, atoi(getenv("GMPSVM_KROW_RESERVE"))) : 0;
+  const int cap = std::max(1, sms - reserve);
+  const int grid = n_tiles < cap ? n_tiles : cap;
   if (f16)
     GM_LAUNCH(krow_tc_kernel<true>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles, norms,
               n, nk, scale, K, ldk, tma);

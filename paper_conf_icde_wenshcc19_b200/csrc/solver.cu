@@ -1503,6 +1503,7 @@ __global__ void __launch_bounds__(512) sigmoid_fit_kernel(SolverArgs a) {
     const double gd = g1 * dA + g2 * dB;
     double step = 1.0;
     bool found = false;
+    int ncand = 1;  // the full Newton step first (accepted in most iterations), then 4 halvings per pass
     while (step >= min_step && !found) {
       double fs[4] = {0.0, 0.0, 0.0, 0.0};
       for (int i = threadIdx.x; i < np; i += blockDim.x) {
@@ -1510,13 +1511,13 @@ __global__ void __launch_bounds__(512) sigmoid_fit_kernel(SolverArgs a) {
         double st = step;
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
-          fs[c] += nll_term(vi, t, A + st * dA, B + st * dB);
+          if (c < ncand) fs[c] += nll_term(vi, t, A + st * dA, B + st * dB);
           st *= 0.5;
         }
       }
       block_sum_n<4>(fs, sm);
       double st = step;
-      for (int c = 0; c < 4 && st >= min_step; ++c) {
+      for (int c = 0; c < ncand && st >= min_step; ++c) {
         if (fs[c] < F + 1e-4 * st * gd) {
           A += st * dA;
           B += st * dB;
@@ -1526,7 +1527,8 @@ __global__ void __launch_bounds__(512) sigmoid_fit_kernel(SolverArgs a) {
         }
         st *= 0.5;
       }
-      step = st;  // if none accepted: continue with the next 4 halvings
+      step = st;  // if none accepted: continue with the next halvings
+      ncand = 4;
     }
     if (!found) {
       status = 2;
