@@ -98,6 +98,7 @@ std::vector<uint8_t> serialize(const Model& m) {
   {
     std::lock_guard<std::mutex> lk(m.mu);
     gmpsvm::ensure_host_sv(m);
+    gmpsvm::ensure_host_alpha(m);
   }
   Writer w;
   w.buf.insert(w.buf.end(), kMagic, kMagic + 8);
@@ -174,6 +175,7 @@ Model* merge(const Model* const* parts, int n) {
       throw Error(GMPSVM_EINVAL, "parts were not trained on the same problem");
     std::lock_guard<std::mutex> lk(q.mu);
     gmpsvm::ensure_host_sv(q);
+    gmpsvm::ensure_host_alpha(q);
   }
   auto m = std::make_unique<Model>();
   m->k = f.k;
@@ -306,6 +308,10 @@ int gmpsvm_model_pair(const gmpsvm_model* model, int32_t s, int32_t t, double* b
     if (A) *A = m.A[p];
     if (B) *B = m.B[p];
     if (alpha_out) {
+      {
+        std::lock_guard<std::mutex> lk(m.mu);
+        gmpsvm::ensure_host_alpha(m);
+      }
       const auto po = m.pair_offsets();
       std::copy(m.alpha.begin() + po[p], m.alpha.begin() + po[p + 1], alpha_out);
     }

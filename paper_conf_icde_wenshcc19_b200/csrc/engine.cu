@@ -316,7 +316,7 @@ DevModel::~DevModel() {
   } catch (...) {
   }
   if (ls && last_use) cudaStreamWaitEvent(ls, last_use, 0);
-  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B, SvHi, SvLo, nsvc, mu};
+  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B, SvHi, SvLo, nsvc, mu, alpha_dev};
   for (void* p : ptrs)
     if (p) {
       if (ls) cudaFreeAsync(p, ls);
@@ -355,9 +355,13 @@ gmpsvm_predict_stats& tls_predict_stats() {
 // rows: device pointer to rows (stride d); row_of_sv[i] = row of SV i (SV order = sv_pos order).
 // mu_in / sc_in: a given centre and split scale for the SV rows; nullptr = compute them from the
 // SV rows
+// alpha_hp / alpha_off: the training call's device alpha (solver pair order) and each model
+// pair's offset into it; the coefficients are then built on the device and the DevModel keeps
+// a copy of alpha (Model::alpha stays on the device until asked for).  nullptr: from m.alpha.
 static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* rows, const std::vector<int64_t>& row_of_sv,
                                                  int device, cudaStream_t st, const float* mu_in = nullptr,
-                                                 float sc_in = 0.f) {
+                                                 float sc_in = 0.f, const double* alpha_hp = nullptr,
+                                                 int64_t alpha_tot = 0, const std::vector<int64_t>* alpha_off = nullptr) {
   auto dm = std::make_unique<DevModel>();
   static const bool ht = getenv("GMPSVM_HOST_TIMING") != nullptr;
   auto t_last = std::chrono::steady_clock::now();
@@ -394,7 +398,9 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   dm->nsv_pad = std::max<int64_t>(slot_begin[k], kTile);
   dm->slot_sv.assign(dm->nsv_pad, -1);
   std::vector<int64_t> slot_src(dm->nsv_pad, -1);
-  std::vector<float> coef((size_t)dm->nsv_pad * dm->km1_pad, 0.f);
+  const bool dev_coef = alpha_hp != nullptr;
+  std::vector<float> coef(dev_coef ? 0 : (size_t)dm->nsv_pad * dm->km1_pad, 0.f);
+  std::vector<int64_t> slot_g(dev_coef ? dm->nsv_pad : 0, -1);  // device coef: class-sorted position per slot
   std::vector<DecItem> items;
   std::vector<int32_t> ib(k, 0), ie(k, 0);
   for (int c = 0; c < k; ++c) {
@@ -403,6 +409,10 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
       dm->slot_sv[slot] = i;
       slot_src[slot] = row_of_sv[i];
       const int64_t g = m.sv_pos[i];
+      if (dev_coef) {
+        slot_g[slot] = g;
+        continue;
+      }
       for (int u = 0; u < k; ++u) {
         if (u == c) continue;
         const int s = std::min(c, u), t = std::max(c, u);
@@ -423,7 +433,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   HT("host_coef");
   dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad, st);
   dm->nsv = dev_alloc<float>(dm->nsv_pad, st);
-  dm->coef = dev_alloc<float>(coef.size(), st);
+  dm->coef = dev_alloc<float>((size_t)dm->nsv_pad * dm->km1_pad, st);
   dm->items = dev_alloc<DecItem>(items.size(), st);
   dm->item_begin = dev_alloc<int32_t>(k, st);
   dm->item_end = dev_alloc<int32_t>(k, st);
@@ -432,7 +442,20 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   dm->B = dev_alloc<double>(P, st);
   DevBuf<int64_t> d_src(slot_src.size(), st);
   GM_CUDA(cudaMemcpyAsync(d_src.get(), slot_src.data(), slot_src.size() * 8, cudaMemcpyHostToDevice, st));
-  GM_CUDA(cudaMemcpyAsync(dm->coef, coef.data(), coef.size() * 4, cudaMemcpyHostToDevice, st));
+  if (dev_coef) {
+    dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st);
+    if (alpha_tot) GM_CUDA(cudaMemcpyAsync(dm->alpha_dev, alpha_hp, (size_t)alpha_tot * 8, cudaMemcpyDeviceToDevice, st));
+    dm->alpha_dev_off = *alpha_off;
+    DevBuf<int64_t> d_g(slot_g.size(), st), d_aoff(P, st), d_off(k + 1, st), d_cc(k, st);
+    GM_CUDA(cudaMemcpyAsync(d_g.get(), slot_g.data(), slot_g.size() * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_aoff.get(), alpha_off->data(), (size_t)P * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_off.get(), off.data(), (size_t)(k + 1) * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_cc.get(), m.class_count.data(), (size_t)k * 8, cudaMemcpyHostToDevice, st));
+    launch_build_coef(dm->alpha_dev, d_aoff.get(), d_g.get(), d_off.get(), d_cc.get(), k, dm->nsv_pad, dm->km1_pad,
+                      dm->coef, st);
+  } else {
+    GM_CUDA(cudaMemcpyAsync(dm->coef, coef.data(), coef.size() * 4, cudaMemcpyHostToDevice, st));
+  }
   GM_CUDA(cudaMemcpyAsync(dm->items, items.data(), items.size() * sizeof(DecItem), cudaMemcpyHostToDevice, st));
   GM_CUDA(cudaMemcpyAsync(dm->item_begin, ib.data(), k * 4, cudaMemcpyHostToDevice, st));
   GM_CUDA(cudaMemcpyAsync(dm->item_end, ie.data(), k * 4, cudaMemcpyHostToDevice, st));
@@ -489,6 +512,22 @@ void ensure_host_sv(const Model& mdl) {
     }
   }
   m.sv_X_ready = true;
+}
+
+void ensure_host_alpha(const Model& mdl) {
+  Model& m = const_cast<Model&>(mdl);
+  if (m.alpha_ready) return;
+  const auto po = m.pair_offsets();
+  const int P = m.P();
+  m.alpha.assign(po[P], 0.0);
+  if (!m.dev || !m.dev->alpha_dev) throw Error(GMPSVM_EINVAL, "model alpha is on neither host nor device");
+  DeviceGuard dg(m.dev->device);
+  for (int p = 0; p < P; ++p) {
+    const int64_t o = m.dev->alpha_dev_off[p];
+    if (o >= 0 && po[p + 1] > po[p])
+      GM_CUDA(cudaMemcpy(&m.alpha[po[p]], m.dev->alpha_dev + o, (size_t)(po[p + 1] - po[p]) * 8, cudaMemcpyDeviceToHost));
+  }
+  m.alpha_ready = true;
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1068,11 +1107,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   std::vector<int32_t> h_sig(Pl), h_st(Pl), h_outer(Pl);
   std::vector<int64_t> h_inner(Pl), h_cyc(Pl);
   // the large read-backs (alpha, permutation, SV flags) land in pinned memory (async DMA)
-  uint8_t* pin = pinned_scratch<uint8_t>((size_t)tot * 8 + (size_t)n * 8 + (size_t)n + 64, 1);
-  double* h_alpha = reinterpret_cast<double*>(pin);
-  int64_t* h_permp = reinterpret_cast<int64_t*>(pin + (size_t)tot * 8);
-  uint8_t* h_flags = pin + (size_t)tot * 8 + (size_t)n * 8;
-  GM_CUDA(cudaMemcpyAsync(h_alpha, d_alpha.get(), tot * 8, cudaMemcpyDeviceToHost, st));
+  // alpha stays on the device (the model's host copy is materialised on demand, ensure_host_alpha)
+  uint8_t* pin = pinned_scratch<uint8_t>((size_t)n * 8 + (size_t)n + 64, 1);
+  int64_t* h_permp = reinterpret_cast<int64_t*>(pin);
+  uint8_t* h_flags = pin + (size_t)n * 8;
   GM_CUDA(cudaMemcpyAsync(hb.data(), d_b.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(hA.data(), d_A.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(hB.data(), d_B.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
@@ -1185,7 +1223,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   mdl->B.assign(P, 0.0);
   mdl->status.assign(P, 0);
   const auto po = mdl->pair_offsets();
-  mdl->alpha.assign(po[P], 0.0);
+  mdl->alpha_ready = false;
+  std::vector<int64_t> alpha_off(P, -1);  // model pair -> offset into the solver's device alpha
   int64_t outer_max = 0, outer_sum = 0, inner_sum = 0, cyc_sum = 0;
   for (int i = 0; i < Pl; ++i) {
     const int p = pids[i];
@@ -1198,7 +1237,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
       cap_hit = true;
     }
     mdl->status[p] = (h_st[i] == 1 ? 0 : h_st[i]) | (h_sig[i] << 8);
-    std::memcpy(&mdl->alpha[po[p]], &h_alpha[hp[i].a_off], sizeof(double) * (hp[i].n_s + hp[i].n_t));
+    alpha_off[p] = hp[i].a_off;
     outer_max = std::max<int64_t>(outer_max, h_outer[i]);
     outer_sum += h_outer[i];
     inner_sum += h_inner[i];
@@ -1211,7 +1250,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   HT("assembled");
   // the SV-row centre and scale are recomputed from the SV rows (not the training call's), so a
   // model merged from partial trainings predicts bitwise like the single-call model
-  mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st);
+  mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st, nullptr, 0.f, d_alpha.get(), tot, &alpha_off);
   tm.mark(PH_FIN);
   HT("devmodel");
   GM_CUDA(cudaStreamSynchronize(st));
@@ -1262,7 +1301,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
 static void ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
   std::lock_guard<std::mutex> lk(mdl.mu);
   if (mdl.dev && mdl.dev->device == device) return;
-  if (mdl.dev) ensure_host_sv(mdl);
+  if (mdl.dev) {  // moving to another device: the host copies are the source of the new one
+    ensure_host_sv(mdl);
+    ensure_host_alpha(mdl);
+  }
   const int64_t nsv = (int64_t)mdl.sv_pos.size();
   DevBuf<float> rows((size_t)std::max<int64_t>(nsv, 1) * mdl.d, st);
   if (nsv > 0) {

@@ -41,6 +41,8 @@ float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, v
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
 bool krow_tc_2cta();
+void launch_build_coef(const double* alpha, const int64_t* aoff, const int64_t* slot_g, const int64_t* off,
+                       const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, cudaStream_t st);
 std::vector<int2> krow_tc_tiles(int64_t n, bool two_cta);
 constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
 // per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]

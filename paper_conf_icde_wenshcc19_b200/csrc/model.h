@@ -37,6 +37,11 @@ struct DevModel {
   float sc = 1.f;           // split scale (exact power of two; 1 for TF32)
   std::vector<DecItem> h_items;  // host copy of the items (work-unit lists of dec_tc)
   std::vector<int64_t> slot_sv;  // slot -> index into the model's SV list, -1 = padding
+  // training output kept on the device: alpha of every trained pair in the solver's pair order;
+  // alpha_dev_off[p] = offset of model pair p (-1: untrained).  The host copy Model::alpha is
+  // materialised from it only when asked for (introspection, serialisation, merge).
+  double* alpha_dev = nullptr;
+  std::vector<int64_t> alpha_dev_off;
   cudaEvent_t last_use = nullptr;  // recorded on the caller's stream after every use
   // stream-ordered allocation: freed on the library stream after last_use (no device sync)
   ~DevModel();
@@ -52,6 +57,7 @@ struct Model {
   std::vector<double> b, A, B;       // [P]
   std::vector<int32_t> status;       // [P] solver status (0 ok, 2 outer cap) | sigmoid status << 8
   std::vector<double> alpha;         // [sum_p n_p] pair-local order, all pairs (0 for untrained)
+  bool alpha_ready = true;           // false: alpha still only on the device (ensure_host_alpha)
   std::vector<int64_t> sv_pos;       // class-sorted positions of the SV union, ascending
   std::vector<float> sv_X;           // [n_sv][d] host copy (materialised lazily from the device)
   bool sv_X_ready = false;
@@ -74,7 +80,8 @@ int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int3
                       const gmpsvm_options& opt);
 int engine_couple(const double* dec, int64_t m, int32_t k, const double* A, const double* B, double* prob_out,
                   const gmpsvm_options& opt);
-void ensure_host_sv(const Model& mdl);  // materialise sv_X on the host
+void ensure_host_sv(const Model& mdl);     // materialise sv_X on the host
+void ensure_host_alpha(const Model& mdl);  // materialise alpha on the host
 gmpsvm_predict_stats& tls_predict_stats();
 
 }  // namespace gmpsvm

@@ -167,4 +167,35 @@ void launch_gather_rows(const float* X, int d, const int64_t* idx, int64_t nr, f
   GM_LAUNCH(gather_rows_kernel, dim3((unsigned)nr), dim3(128), 0, st, X, d, idx, nr, dst);
 }
 
+// a9: LibSVM-style coefficients of the SV slots, coef[slot][col] = y * alpha of the SV in each of
+// the k - 1 pairs of its class, read from the training call's device
+// alpha (aoff[p] = offset of pair p's alpha, -1: untrained -> 0).  One thread per slot.
+__global__ void build_coef_kernel(const double* __restrict__ alpha, const int64_t* __restrict__ aoff,
+                                  const int64_t* __restrict__ slot_g, const int64_t* __restrict__ off,
+                                  const int64_t* __restrict__ cc, int k, int64_t nsv_pad, int km1_pad,
+                                  float* __restrict__ coef) {
+  const int64_t slot = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (slot >= nsv_pad) return;
+  float* out = coef + slot * km1_pad;
+  for (int col = 0; col < km1_pad; ++col) out[col] = 0.f;
+  const int64_t g = slot_g[slot];
+  if (g < 0) return;  // padding slot
+  int c = 0;
+  while (c + 1 < k && off[c + 1] <= g) ++c;
+  for (int u = 0; u < k; ++u) {
+    if (u == c) continue;
+    const int s = c < u ? c : u, t = c < u ? u : c;
+    const int p = pair_index(s, t, k);
+    const int64_t j = (c == s) ? (g - off[s]) : (cc[s] + (g - off[t]));
+    const double a = aoff[p] >= 0 ? alpha[aoff[p] + j] : 0.0;
+    out[u < c ? u : u - 1] = (float)((c == s) ? a : -a);
+  }
+}
+
+void launch_build_coef(const double* alpha, const int64_t* aoff, const int64_t* slot_g, const int64_t* off,
+                       const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, cudaStream_t st) {
+  GM_LAUNCH(build_coef_kernel, dim3((unsigned)ceil_div(nsv_pad, 256)), dim3(256), 0, st, alpha, aoff, slot_g, off, cc, k,
+            nsv_pad, km1_pad, coef);
+}
+
 }  // namespace gmpsvm
