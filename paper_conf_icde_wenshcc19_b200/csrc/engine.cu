@@ -737,8 +737,36 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   std::vector<int> wave_off;     // tile range of wave w: [wave_off[w], wave_off[w + 1])
   std::vector<int> ready_wave;   // per pair position: the wave after which its kernel values are complete
   const bool two_cta = use_tc && !overlap && krow_tc_2cta();  // the overlap waves use single-CTA tiles
+  double kv_subset = -1;  // >= 0: kernel values computed for a pair subset (tiles skipped)
   if (use_tc) {
     tiles = krow_tc_tiles(n, two_cta);
+    if (!overlap && !two_cta && Pl < P) {
+      // pair subset (multi-GPU shard, pair_ids): only the tiles overlapping a class block
+      // (s,s), (s,t), (t,t) of a trained pair are computed (PAPER.md L313-L325 sharing, per rank)
+      std::vector<uint8_t> need((size_t)k * k, 0);
+      for (int i = 0; i < Pl; ++i) {
+        need[(size_t)hp[i].s * k + hp[i].s] = need[(size_t)hp[i].t * k + hp[i].t] = 1;
+        need[(size_t)std::min(hp[i].s, hp[i].t) * k + std::max(hp[i].s, hp[i].t)] = 1;
+      }
+      auto cls = [&](int64_t r) { return (int)(std::upper_bound(coff.begin(), coff.end(), r) - coff.begin()) - 1; };
+      std::vector<int2> kept;
+      for (const int2 tl : tiles) {
+        const int64_t r0 = (int64_t)tl.x * kKrowTileRows, c0 = (int64_t)tl.y * kKrowTileRows;
+        const int ra = cls(r0), rb = cls(std::min<int64_t>(n, r0 + kKrowTileRows) - 1);
+        const int ca = cls(c0), cb = cls(std::min<int64_t>(n, c0 + kKrowTileRows) - 1);
+        bool any = false;
+        for (int a0 = ra; a0 <= rb && !any; ++a0)
+          for (int b0 = ca; b0 <= cb && !any; ++b0) any = need[(size_t)std::min(a0, b0) * k + std::max(a0, b0)] != 0;
+        if (any) kept.push_back(tl);
+      }
+      tiles.swap(kept);
+      kv_subset = 0;  // kernel values (r <= c) the kept tiles compute
+      for (const int2 tl : tiles) {
+        const int64_t r0 = (int64_t)tl.x * kKrowTileRows, c0 = (int64_t)tl.y * kKrowTileRows;
+        const int64_t nr = std::min<int64_t>(n, r0 + kKrowTileRows) - r0, nc = std::min<int64_t>(n, c0 + kKrowTileRows) - c0;
+        kv_subset += tl.x == tl.y ? (double)nr * (double)(nr + 1) / 2.0 : (double)nr * (double)nc;
+      }
+    }
     if (overlap) {
       const int INF = INT_MAX;
       std::vector<int> minpos(k, INF);  // first position of a pair containing class c
@@ -1271,7 +1299,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   s.t_solver_ms = tm.ms(PH_SOLVER);
   s.n_streams = graph_mode ? n_branches : G;
   if (full_k) {
-    s.kernel_values = (double)n * (double)(n + 1) / 2.0;
+    s.kernel_values = kv_subset >= 0 ? kv_subset : (double)n * (double)(n + 1) / 2.0;
     s.krow_launches = 1;
   } else {
     std::vector<int64_t> rows(Pl);
