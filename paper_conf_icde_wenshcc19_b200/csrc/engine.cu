@@ -202,12 +202,33 @@ struct KWorkspace {
   float* get() const { return p; }
 };
 
+// Destroying the solver's executable graph (hundreds of nodes) takes ~3 ms of host time and holds
+// the driver while it runs, so a finished graph is not destroyed when its training call returns:
+// it is parked here and destroyed by the next training call right after that call has launched
+// its own solver graph (the GPU then has tens of ms of queued work to hide it behind).
+std::mutex g_parked_mu;
+std::vector<std::pair<cudaGraphExec_t, cudaGraph_t>> g_parked;
+
+void destroy_parked_graphs() {
+  std::vector<std::pair<cudaGraphExec_t, cudaGraph_t>> v;
+  {
+    std::lock_guard<std::mutex> lk(g_parked_mu);
+    v.swap(g_parked);
+  }
+  for (auto& e : v) {
+    if (e.first) cudaGraphExecDestroy(e.first);
+    if (e.second) cudaGraphDestroy(e.second);
+  }
+}
+
 struct GraphGuard {
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
   ~GraphGuard() {
-    if (exec) cudaGraphExecDestroy(exec);
-    if (graph) cudaGraphDestroy(graph);
+    if (exec || graph) {
+      std::lock_guard<std::mutex> lk(g_parked_mu);
+      g_parked.emplace_back(exec, graph);
+    }
   }
 };
 
@@ -1075,6 +1096,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
     GM_CUDA(cudaGraphInstantiate(&gg.exec, gg.graph, 0));
     HT("graph_build");
     GM_CUDA(cudaGraphLaunch(gg.exec, pool[0]));
+    destroy_parked_graphs();  // the previous calls' graphs, while this solver runs
   } else {
     for (int g = 0; g < G; ++g) issue_chunk(g);
     for (int g = 0; g < G; ++g) issue_chunk(g);

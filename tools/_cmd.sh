@@ -1,7 +1,5 @@
-out=gpurun_out/$1; mkdir -p $out
-python -c "import __graft_entry__ as g; g.build()" > $out/build.log 2>&1
-timeout 600 python -m pytest tests/test_gpu_parity.py -x -q > $out/pytest.log 2>&1; echo "rc=$?" >> $out/pytest.log
-echo base >> $out/ov.log; timeout 300 python tools/sweep.py "ws_size=192" >> $out/ov.log 2>&1
-for r in 0 8 16 32; do echo "overlap reserve $r" >> $out/ov.log; GMPSVM_OVERLAP=1 GMPSVM_KROW_RESERVE=$r timeout 300 python tools/sweep.py "ws_size=192" >> $out/ov.log 2>&1; done
-GMPSVM_SMO_PHASES=1 timeout 300 python tools/prof_step.py --ws-size 192 --reps 2 2>&1 | grep -i sigmoid >> $out/ov.log
-tail -2 $out/pytest.log; cat $out/ov.log | cut -c1-190
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+timeout 300 python tools/step_overhead.py 2>&1 | tail -3
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -2
+timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > /tmp/b.json 2>/dev/null; python -c "
+import json;d=json.load(open('/tmp/b.json')); print(d['value'], d['e2e']['value'], d['step_ms'], d['phases_ms'])"
