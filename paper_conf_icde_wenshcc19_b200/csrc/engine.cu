@@ -337,7 +337,7 @@ DevModel::~DevModel() {
   } catch (...) {
   }
   if (ls && last_use) cudaStreamWaitEvent(ls, last_use, 0);
-  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B, SvHi, SvLo, nsvc, mu, alpha_dev};
+  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B, SvHi, SvLo, nsvc, mu, alpha_dev, coef64, nsv64};
   for (void* p : ptrs)
     if (p) {
       if (ls) cudaFreeAsync(p, ls);
@@ -374,6 +374,22 @@ gmpsvm_predict_stats& tls_predict_stats() {
 
 // Build the device prediction structures from SV rows already on the device.
 // rows: device pointer to rows (stride d); row_of_sv[i] = row of SV i (SV order = sv_pos order).
+// pair index -> (s, t), the inverse of pair_index
+static int ps_of(int p, int k) {
+  int s = 0, rem = p;
+  while (rem >= k - 1 - s) rem -= k - 1 - s++;
+  return s;
+}
+static int pt_of(int p, int k) {
+  int s = 0, rem = p;
+  while (rem >= k - 1 - s) rem -= k - 1 - s++;
+  return s + 1 + rem;
+}
+// FP64 decision values when the worst-case probability shift from FP32 kernel values exceeds
+// this (MNIST-shaped C = 10 models sit near 2e-3 and meet 1e-4 on the TF32/FP16-split path;
+// MNIST8M-shaped C = 1000 models are far above it)
+constexpr double kDecF64Cond = 0.02;
+
 // mu_in / sc_in: a given centre and split scale for the SV rows; nullptr = compute them from the
 // SV rows
 // alpha_hp / alpha_off: the training call's device alpha (solver pair order) and each model
@@ -421,6 +437,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   std::vector<int64_t> slot_src(dm->nsv_pad, -1);
   const bool dev_coef = alpha_hp != nullptr;
   std::vector<float> coef(dev_coef ? 0 : (size_t)dm->nsv_pad * dm->km1_pad, 0.f);
+  std::vector<double> coef64(dev_coef ? 0 : (size_t)dm->nsv_pad * dm->km1_pad, 0.0);
   std::vector<int64_t> slot_g(dev_coef ? dm->nsv_pad : 0, -1);  // device coef: class-sorted position per slot
   std::vector<DecItem> items;
   std::vector<int32_t> ib(k, 0), ie(k, 0);
@@ -442,6 +459,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
         const double a = m.alpha[po[p] + j];
         const int col = u < c ? u : u - 1;
         coef[(size_t)slot * dm->km1_pad + col] = (float)((c == s) ? a : -a);
+        coef64[(size_t)slot * dm->km1_pad + col] = (c == s) ? a : -a;
       }
     }
     ib[c] = (int32_t)items.size();
@@ -463,6 +481,27 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   dm->B = dev_alloc<double>(P, st);
   DevBuf<int64_t> d_src(slot_src.size(), st);
   GM_CUDA(cudaMemcpyAsync(d_src.get(), slot_src.data(), slot_src.size() * 8, cudaMemcpyHostToDevice, st));
+  // conditioning of the decision values: sum_j |alpha_pj| per trained pair
+  std::vector<double> abs_sum(P, 0.0);
+  if (dev_coef) {
+    std::vector<int64_t> npv(P, 0);
+    for (int p = 0; p < P; ++p) npv[p] = m.class_count[ps_of(p, k)] + m.class_count[pt_of(p, k)];
+    DevBuf<int64_t> d_ao(P, st), d_np(P, st);
+    DevBuf<double> d_sum(P, st);
+    GM_CUDA(cudaMemcpyAsync(d_ao.get(), alpha_off->data(), (size_t)P * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_np.get(), npv.data(), (size_t)P * 8, cudaMemcpyHostToDevice, st));
+    launch_alpha_abs_sum(alpha_hp, d_ao.get(), d_np.get(), P, d_sum.get(), st);
+    GM_CUDA(cudaMemcpyAsync(abs_sum.data(), d_sum.get(), (size_t)P * 8, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaStreamSynchronize(st));
+  } else {
+    for (int p = 0; p < P; ++p)
+      for (int64_t j = po[p]; j < po[p + 1]; ++j) abs_sum[p] += std::fabs(m.alpha[j]);
+  }
+  for (int p = 0; p < P; ++p) dm->cond = std::max(dm->cond, std::fabs(m.A[p]) / 4.0 * std::ldexp(1.0, -22) * abs_sum[p]);
+  static const char* dec_env = getenv("GMPSVM_DEC");
+  const std::string dec_mode = dec_env ? dec_env : "";
+  dm->f64 = dec_mode == "f64" || (dec_mode.empty() && dm->cond > kDecF64Cond);
+  if (dm->f64) dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
   if (dev_coef) {
     dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st);
     if (alpha_tot) GM_CUDA(cudaMemcpyAsync(dm->alpha_dev, alpha_hp, (size_t)alpha_tot * 8, cudaMemcpyDeviceToDevice, st));
@@ -473,9 +512,10 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
     GM_CUDA(cudaMemcpyAsync(d_off.get(), off.data(), (size_t)(k + 1) * 8, cudaMemcpyHostToDevice, st));
     GM_CUDA(cudaMemcpyAsync(d_cc.get(), m.class_count.data(), (size_t)k * 8, cudaMemcpyHostToDevice, st));
     launch_build_coef(dm->alpha_dev, d_aoff.get(), d_g.get(), d_off.get(), d_cc.get(), k, dm->nsv_pad, dm->km1_pad,
-                      dm->coef, st);
+                      dm->coef, dm->coef64, st);
   } else {
     GM_CUDA(cudaMemcpyAsync(dm->coef, coef.data(), coef.size() * 4, cudaMemcpyHostToDevice, st));
+    if (dm->f64) GM_CUDA(cudaMemcpyAsync(dm->coef64, coef64.data(), coef64.size() * 8, cudaMemcpyHostToDevice, st));
   }
   GM_CUDA(cudaMemcpyAsync(dm->items, items.data(), items.size() * sizeof(DecItem), cudaMemcpyHostToDevice, st));
   GM_CUDA(cudaMemcpyAsync(dm->item_begin, ib.data(), k * 4, cudaMemcpyHostToDevice, st));
@@ -486,6 +526,10 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
   HT("h2d_svt");
+  if (dm->f64) {
+    dm->nsv64 = dev_alloc<double>(dm->nsv_pad, st);
+    launch_col_norms64(dm->SvT, dm->nsv_pad, dm->nsv_pad, dm->d_pad, dm->nsv64, st);
+  }
   dm->h_items = items;
   // tensor-core decision values: centre = mean of the SV rows, TF32 hi/lo split of the SV slots
   static const bool dec_simt = getenv("GMPSVM_DEC") && std::string(getenv("GMPSVM_DEC")) == "simt";
@@ -509,7 +553,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
                          dm->dpt, st);
     HT("split");
   }
-  if (ht) fprintf(stderr, "[gmpsvm devmodel ms]%s\n", line.c_str());
+  if (ht) fprintf(stderr, "[gmpsvm devmodel ms]%s cond=%.3e f64=%d\n", line.c_str(), dm->cond, (int)dm->f64);
   GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
   GM_CUDA(cudaEventRecord(dm->last_use, st));
   GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
@@ -1389,7 +1433,8 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   DevBuf<float> Xhi(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st), Xlo(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st);
   // the SIMT decision values need the feature-major copy only as the FP16-range fallback
   DevBuf<float> XtTf(dm.tc ? (size_t)dm.d_pad * mc_pad : 0, st);
-  DevBuf<float> part((size_t)dm.n_items * mc_pad * dm.km1_pad, st);
+  DevBuf<float> part(dm.f64 ? 0 : (size_t)dm.n_items * mc_pad * dm.km1_pad, st);
+  DevBuf<double> part64(dm.f64 ? (size_t)dm.n_items * mc_pad * dm.km1_pad : 0, st), nt64(dm.f64 ? mc_pad : 0, st);
   DevBuf<double> dec_buf(opt.inputs_on_device ? 0 : (size_t)mc_max * P, st);
   DevBuf<double> prob_buf((opt.inputs_on_device || !prob_out) ? 0 : (size_t)mc_max * k, st);
   DevBuf<double> dec_tmp((opt.inputs_on_device && !dec_out) ? (size_t)mc_max * P : 0, st);
@@ -1408,7 +1453,8 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     DevBuf<int32_t> d_uoff, d_uitem;
     int n_units = 0;
     // FP16 split: test rows far outside the SVs' range would overflow half precision -> SIMT
-    const bool use_tc = dm.tc && (!krow_split_f16() || launch_maxabs(src, mc, d, nullptr, dm.mu, st) * dm.sc < 60000.f);
+    const bool use_tc = !dm.f64 && dm.tc &&
+                        (!krow_split_f16() || launch_maxabs(src, mc, d, nullptr, dm.mu, st) * dm.sc < 60000.f);
     if (use_tc) {
       launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
       launch_split_tf32_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
@@ -1438,7 +1484,14 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     tm.mark(PH_STAGE);
     double* dec_d = opt.inputs_on_device ? (dec_out ? dec_out + i0 * P : dec_tmp.get()) : dec_buf.get();
     tm.mark(PH_DEC);
-    if (use_tc) {
+    if (dm.f64) {  // ill-conditioned model: FP64 decision values
+      float* xt = dm.tc ? XtTf.get() : XtT.get();
+      launch_col_norms64(xt, mcp, mcp, dm.d_pad, nt64.get(), st);
+      GM_CUDA(cudaMemsetAsync(part64.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 8, st));
+      launch_dec_f64(xt, mcp, nt64.get(), mcp, dm.SvT, dm.nsv_pad, dm.nsv64, dm.coef64, dm.km1, dm.km1_pad, dm.items,
+                     dm.n_items, dm.d_pad, mdl.gamma, part64.get(), st);
+      launch_dec_reduce64(part64.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
+    } else if (use_tc) {
       GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
       if (n_units > 0)
         launch_dec_tc(Xhi.get(), Xlo.get(), mcp, dm.SvHi, dm.SvLo, dm.nsv_pad, dm.dpt, d_dtiles.get(), d_uoff.get(),
@@ -1448,7 +1501,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
       launch_dec_contract(dm.tc ? XtTf.get() : XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef,
                           dm.km1, dm.km1_pad, dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
     }
-    launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
+    if (!dm.f64) launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     ps.dec_launches += 1;
     tm.mark(PH_DEC);
     double* prob_d = nullptr;

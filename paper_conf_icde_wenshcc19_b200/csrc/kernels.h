@@ -42,7 +42,10 @@ float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, v
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
 bool krow_tc_2cta();
 void launch_build_coef(const double* alpha, const int64_t* aoff, const int64_t* slot_g, const int64_t* off,
-                       const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, cudaStream_t st);
+                       const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, double* coef64,
+                       cudaStream_t st);
+void launch_alpha_abs_sum(const double* alpha, const int64_t* aoff, const int64_t* np, int P, double* out,
+                          cudaStream_t st);
 std::vector<int2> krow_tc_tiles(int64_t n, bool two_cta);
 constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
 // per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
@@ -157,6 +160,12 @@ struct DecItem {
 void launch_dec_contract(const float* XtT, int64_t ldt, const float* nt, int64_t m, int64_t m_pad, const float* SvT,
                          int64_t lds, const float* nsv, const float* coef, int km1, int km1_pad, const DecItem* items,
                          int n_items, int kdim, double gamma, float* part, cudaStream_t st);
+void launch_col_norms64(const float* XT, int64_t ld, int64_t n, int d_pad, double* out, cudaStream_t st);
+void launch_dec_f64(const float* XtT, int64_t ldt, const double* nt64, int64_t m_pad, const float* SvT, int64_t lds,
+                    const double* nsv64, const double* coef64, int km1, int km1_pad, const DecItem* items, int n_items,
+                    int d_pad, double gamma, double* part, cudaStream_t st);
+void launch_dec_reduce64(const double* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,
+                         const int32_t* item_end, const double* b, double* dec, cudaStream_t st);
 void launch_dec_reduce(const float* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,
                        const int32_t* item_end, const double* b, double* dec, cudaStream_t st);
 void launch_couple(const double* dec, int64_t m, int k, const double* A, const double* B, double* prob,

@@ -41,6 +41,12 @@ struct DevModel {
   // alpha_dev_off[p] = offset of model pair p (-1: untrained).  The host copy Model::alpha is
   // materialised from it only when asked for (introspection, serialisation, merge).
   double* alpha_dev = nullptr;
+  // FP64 decision values for ill-conditioned models: cond = max_p |A_p|/4 *
+  // 2^-22 * sum_j |alpha_pj| (worst-case probability shift from FP32 kernel values)
+  bool f64 = false;
+  double cond = 0.0;
+  double* coef64 = nullptr;  // [nsv_pad][km1_pad]
+  double* nsv64 = nullptr;   // [nsv_pad] FP64 squared norms of the SV rows
   std::vector<int64_t> alpha_dev_off;
   cudaEvent_t last_use = nullptr;  // recorded on the caller's stream after every use
   // stream-ordered allocation: freed on the library stream after last_use (no device sync)

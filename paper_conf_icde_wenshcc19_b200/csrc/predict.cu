@@ -243,6 +243,152 @@ void launch_dec_contract(const float* XtT, int64_t ldt, const float* nt, int64_t
             ldt, nt, m, m_pad, SvT, lds, nsv, coef, km1, km1_pad, items, kdim, scale, part);
 }
 
+// ------------------------------------------------------------------------------------------
+// a10 in FP64 (ill-conditioned models): when sum_j |coef_j| K_ij is so large that
+// FP32 kernel values alone would move probabilities beyond the 1e-4 contract (e.g. C = 1000),
+// the decision values are computed in FP64 end to end -- FP64 norms and dot products of the
+// FP32 inputs, exp in FP64, FP64 coefficient contraction -- the oracle's arithmetic up to
+// summation order.  Same work decomposition as dec_contract (one CTA = a test tile x a class-pure
+// run of SV tiles); FP64 tiles of 64 x 64, thread (ty, tx) owns rows 4 ty.. and columns 4 tx...
+constexpr int kF64Tile = 64, kF64BK = 16;
+
+__global__ void __launch_bounds__(256) dec_f64_kernel(const float* __restrict__ XtT, int64_t ldt,
+                                                      const double* __restrict__ nt64, const float* __restrict__ SvT,
+                                                      int64_t lds, const double* __restrict__ nsv64,
+                                                      const double* __restrict__ coef64, int km1, int km1_pad,
+                                                      const DecItem* __restrict__ items, int kdim, double gamma,
+                                                      int64_t m_pad, double* __restrict__ part) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  double* as = reinterpret_cast<double*>(dsm);        // [kF64BK][64]
+  double* bs = as + kF64BK * kF64Tile;                // [kF64BK][64]
+  double* coefS = bs + kF64BK * kF64Tile;             // [64][km1_pad]
+  double* decS = coefS + kF64Tile * km1_pad;          // [64][km1_pad]
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int64_t r0 = (int64_t)blockIdx.x * kF64Tile;
+  const DecItem it = items[blockIdx.y];
+  for (int i = tid; i < kF64Tile * km1_pad; i += 256) decS[i] = 0.0;
+  double nr[4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) nr[i] = nt64[r0 + ty * 4 + i];
+  const int64_t c_begin = (int64_t)it.tile_begin * kTile, c_end = (int64_t)it.tile_end * kTile;
+  for (int64_t c0 = c_begin; c0 < c_end; c0 += kF64Tile) {
+    double acc[4][4] = {};
+    for (int k0 = 0; k0 < kdim; k0 += kF64BK) {
+      __syncthreads();  // previous chunk / tile done with as, bs, coefS
+      for (int e = tid; e < kF64BK * kF64Tile; e += 256) {
+        const int kk = e / kF64Tile, c = e % kF64Tile;
+        as[e] = (double)XtT[(int64_t)(k0 + kk) * ldt + r0 + c];
+        bs[e] = (double)SvT[(int64_t)(k0 + kk) * lds + c0 + c];
+      }
+      __syncthreads();
+#pragma unroll
+      for (int kk = 0; kk < kF64BK; ++kk) {
+        double a[4], b[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) a[i] = as[kk * kF64Tile + ty * 4 + i];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) b[j] = bs[kk * kF64Tile + tx * 4 + j];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
+      }
+    }
+    for (int e = tid; e < kF64Tile * km1_pad; e += 256) coefS[e] = coef64[c0 * km1_pad + e];
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const double nc = nsv64[c0 + tx * 4 + j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const double d2 = nr[i] + nc - 2.0 * acc[i][j];
+        acc[i][j] = exp(-gamma * (d2 > 0.0 ? d2 : 0.0));  // K in FP64
+      }
+    }
+    for (int u = 0; u < km1; ++u) {
+      double p[4] = {0.0, 0.0, 0.0, 0.0};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const double cv = coefS[(tx * 4 + j) * km1_pad + u];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) p[i] = fma(acc[i][j], cv, p[i]);
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {  // sum over the 16 threads sharing these rows (fixed order)
+        double v = p[i];
+        v += __shfl_xor_sync(0xffffffffu, v, 1);
+        v += __shfl_xor_sync(0xffffffffu, v, 2);
+        v += __shfl_xor_sync(0xffffffffu, v, 4);
+        v += __shfl_xor_sync(0xffffffffu, v, 8);
+        p[i] = v;
+      }
+      if (tx == 0)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) decS[(ty * 4 + i) * km1_pad + u] += p[i];
+    }
+  }
+  __syncthreads();
+  double* out = part + ((int64_t)blockIdx.y * m_pad + r0) * km1_pad;
+  for (int i = tid; i < kF64Tile * km1_pad; i += 256) out[i] = decS[i];
+}
+
+// FP64 squared norms of the columns of a feature-major matrix XT[d_pad][ld] (n columns)
+__global__ void col_norms64_kernel(const float* __restrict__ XT, int64_t ld, int64_t n, int d_pad,
+                                   double* __restrict__ out) {
+  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  double s = 0.0;
+  for (int f = 0; f < d_pad; ++f) {
+    const double x = (double)XT[(int64_t)f * ld + c];
+    s = fma(x, x, s);
+  }
+  out[c] = s;
+}
+
+__global__ void dec_reduce64_kernel(const double* __restrict__ part, int64_t m, int64_t m_pad, int k, int km1_pad,
+                                    const int32_t* __restrict__ item_begin, const int32_t* __restrict__ item_end,
+                                    const double* __restrict__ b, double* __restrict__ dec) {
+  const int P = k * (k - 1) / 2;
+  const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (gid >= m * P) return;
+  const int64_t i = gid / P;
+  const int p = (int)(gid % P);
+  int s = 0, rem = p;
+  while (rem >= k - 1 - s) {
+    rem -= k - 1 - s;
+    ++s;
+  }
+  const int t = s + 1 + rem;
+  double acc = b[p];
+  for (int q = item_begin[s]; q < item_end[s]; ++q) acc += part[((int64_t)q * m_pad + i) * km1_pad + (t - 1)];
+  for (int q = item_begin[t]; q < item_end[t]; ++q) acc += part[((int64_t)q * m_pad + i) * km1_pad + s];
+  dec[gid] = acc;
+}
+
+void launch_col_norms64(const float* XT, int64_t ld, int64_t n, int d_pad, double* out, cudaStream_t st) {
+  GM_LAUNCH(col_norms64_kernel, dim3((unsigned)ceil_div(n, 256)), dim3(256), 0, st, XT, ld, n, d_pad, out);
+}
+
+void launch_dec_f64(const float* XtT, int64_t ldt, const double* nt64, int64_t m_pad, const float* SvT, int64_t lds,
+                    const double* nsv64, const double* coef64, int km1, int km1_pad, const DecItem* items, int n_items,
+                    int d_pad, double gamma, double* part, cudaStream_t st) {
+  const size_t smem = (size_t)(2 * kF64BK * kF64Tile + 2 * kF64Tile * km1_pad) * sizeof(double);
+  static bool configured = false;
+  if (!configured) {
+    GM_CUDA(cudaFuncSetAttribute(dec_f64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(96 * 1024)));
+    configured = true;
+  }
+  GM_LAUNCH(dec_f64_kernel, dim3((unsigned)(m_pad / kF64Tile), (unsigned)n_items), dim3(256), smem, st, XtT, ldt, nt64,
+            SvT, lds, nsv64, coef64, km1, km1_pad, items, d_pad, gamma, m_pad, part);
+}
+
+void launch_dec_reduce64(const double* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,
+                         const int32_t* item_end, const double* b, double* dec, cudaStream_t st) {
+  const int64_t tot = m * (int64_t)(k * (k - 1) / 2);
+  GM_LAUNCH(dec_reduce64_kernel, dim3((unsigned)ceil_div(tot, 256)), dim3(256), 0, st, part, m, m_pad, k, km1_pad,
+            item_begin, item_end, b, dec);
+}
+
 void launch_dec_reduce(const float* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,
                        const int32_t* item_end, const double* b, double* dec, cudaStream_t st) {
   const int64_t tot = m * (int64_t)(k * (k - 1) / 2);

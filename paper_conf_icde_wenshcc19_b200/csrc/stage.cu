@@ -173,11 +173,15 @@ void launch_gather_rows(const float* X, int d, const int64_t* idx, int64_t nr, f
 __global__ void build_coef_kernel(const double* __restrict__ alpha, const int64_t* __restrict__ aoff,
                                   const int64_t* __restrict__ slot_g, const int64_t* __restrict__ off,
                                   const int64_t* __restrict__ cc, int k, int64_t nsv_pad, int km1_pad,
-                                  float* __restrict__ coef) {
+                                  float* __restrict__ coef, double* __restrict__ coef64) {
   const int64_t slot = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (slot >= nsv_pad) return;
   float* out = coef + slot * km1_pad;
-  for (int col = 0; col < km1_pad; ++col) out[col] = 0.f;
+  double* out64 = coef64 ? coef64 + slot * km1_pad : nullptr;
+  for (int col = 0; col < km1_pad; ++col) {
+    out[col] = 0.f;
+    if (out64) out64[col] = 0.0;
+  }
   const int64_t g = slot_g[slot];
   if (g < 0) return;  // padding slot
   int c = 0;
@@ -189,13 +193,38 @@ __global__ void build_coef_kernel(const double* __restrict__ alpha, const int64_
     const int64_t j = (c == s) ? (g - off[s]) : (cc[s] + (g - off[t]));
     const double a = aoff[p] >= 0 ? alpha[aoff[p] + j] : 0.0;
     out[u < c ? u : u - 1] = (float)((c == s) ? a : -a);
+    if (out64) out64[u < c ? u : u - 1] = (c == s) ? a : -a;
   }
 }
 
+// sum_j |alpha_j| per trained pair (conditioning of the decision values)
+__global__ void alpha_abs_sum_kernel(const double* __restrict__ alpha, const int64_t* __restrict__ aoff,
+                                     const int64_t* __restrict__ np, double* __restrict__ out) {
+  const int p = blockIdx.x;
+  __shared__ double red[32];
+  double s = 0.0;
+  if (aoff[p] >= 0)
+    for (int64_t j = threadIdx.x; j < np[p]; j += blockDim.x) s += fabs(alpha[aoff[p] + j]);
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+    out[p] = t;
+  }
+}
+
+void launch_alpha_abs_sum(const double* alpha, const int64_t* aoff, const int64_t* np, int P, double* out,
+                          cudaStream_t st) {
+  GM_LAUNCH(alpha_abs_sum_kernel, dim3((unsigned)P), dim3(256), 0, st, alpha, aoff, np, out);
+}
+
 void launch_build_coef(const double* alpha, const int64_t* aoff, const int64_t* slot_g, const int64_t* off,
-                       const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, cudaStream_t st) {
+                       const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, double* coef64,
+                       cudaStream_t st) {
   GM_LAUNCH(build_coef_kernel, dim3((unsigned)ceil_div(nsv_pad, 256)), dim3(256), 0, st, alpha, aoff, slot_g, off, cc, k,
-            nsv_pad, km1_pad, coef);
+            nsv_pad, km1_pad, coef, coef64);
 }
 
 }  // namespace gmpsvm

@@ -306,3 +306,27 @@ def test_mixed_solver_paths_in_one_graph(gm, tmp_path):
     subprocess.run([sys.executable, "-c", code], check=True, env=env, timeout=600)
     p = np.load(tmp_path / "p.npy")
     assert np.abs(p - prob_o).max() <= 1e-4
+
+
+def test_fp64_decision_path_vs_oracle(gm, tmp_path):
+    """The FP64 decision-value path (taken automatically for ill-conditioned models; forced here
+    with GMPSVM_DEC=f64, read once per process: subprocess) evaluates Eq 11 with FP64 kernel
+    values: against the oracle's FP64 evaluation of the same model it agrees to rounding."""
+    import subprocess
+    import sys
+
+    spec, X, y, Xt, yt = datagen.make_config("mnist", n_train=1500, n_test=300)
+    code = (
+        "import sys, numpy as np; sys.path.insert(0, %r); import datagen, paper_conf_icde_wenshcc19_b200 as gm;"
+        "spec, X, y, Xt, yt = datagen.make_config('mnist', n_train=1500, n_test=300);"
+        "m = gm.train(X, y, spec.k, spec.C, spec.gamma, %r);"
+        "al = [m.pair(s, t, int((y == s).sum()), int((y == t).sum())) for s in range(spec.k) for t in range(s + 1, spec.k)];"
+        "np.savez(%r, dec=m.decision_function(Xt), prob=m.predict_proba(Xt), alpha=np.concatenate([a['alpha'] for a in al]),"
+        " b=[a['b'] for a in al], A=[a['A'] for a in al], B=[a['B'] for a in al])" % (ROOT, EPS, str(tmp_path / "r.npz"))
+    )
+    subprocess.run([sys.executable, "-c", code], check=True, env=dict(os.environ, GMPSVM_DEC="f64"), timeout=600)
+    r = np.load(tmp_path / "r.npz")
+    ref = dict(k=spec.k, gamma=spec.gamma, alpha_flat=r["alpha"], b=r["b"], A=r["A"], B=r["B"])
+    dec_o, prob_o = oracle.predict(ref, X, y, Xt)
+    assert np.abs(r["dec"] - dec_o).max() <= 1e-9 * max(1.0, np.abs(dec_o).max())
+    assert np.abs(r["prob"] - prob_o).max() <= 1e-9
