@@ -161,6 +161,17 @@ GMPSVM_API int gmpsvm_model_serialize(const gmpsvm_model* model, void* buf, size
 GMPSVM_API int gmpsvm_model_deserialize(const void* buf, size_t len, gmpsvm_model** out);
 /* Union of partial models trained on disjoint pair subsets of the same (X, y, C, gamma). */
 GMPSVM_API int gmpsvm_model_merge(const gmpsvm_model* const* parts, int32_t n_parts, gmpsvm_model** out);
+/* The complete model from every pair's solution computed elsewhere -- the multi-GPU path's
+ * gather: each rank trains a pair subset (pair_ids), the ranks all-reduce the disjoint per-pair
+ * alpha / b / A / B (O(sum n_p) doubles over NCCL) and every rank rebuilds the model from its
+ * own replicated X (SV union, coefficients, Alg 2 l.16, L331-L333, L363).  X, y: as in
+ * gmpsvm_train_ex (device pointers if opt->inputs_on_device); alpha: sum_p n_p doubles, pairs
+ * in index order, each in pair-local order (the layout of gmpsvm_model_pair's alpha_out), every
+ * value in [0, C] (else EINVAL); b, A, B: P doubles; status: P int32 or NULL -- host pointers. */
+GMPSVM_API int gmpsvm_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C,
+                                       double gamma, const double* alpha, const double* b, const double* A,
+                                       const double* B, const int32_t* status, const gmpsvm_options* opt,
+                                       gmpsvm_model** out);
 
 /* ---- component entry points (steps of the path, exposed for parity tests and bench) ---- */
 /* a2 alone (K1, L287-L299, RBF L75): K_out[i*m + j] = exp(-gamma ||X_i - Y_j||^2) in FP32 via

@@ -74,6 +74,8 @@ _SIGS = {
     "gmpsvm_model_serialize": (ct.c_int, [_P, _P, _P]),
     "gmpsvm_model_deserialize": (ct.c_int, [_P, ct.c_size_t, _P]),
     "gmpsvm_model_merge": (ct.c_int, [_P, ct.c_int32, _P]),
+    "gmpsvm_model_from_alpha": (ct.c_int, [_P, _P, ct.c_int64, ct.c_int32, ct.c_int32, ct.c_double, ct.c_double, _P, _P,
+                                           _P, _P, _P, _P, _P]),
     "gmpsvm_rbf_kernel": (ct.c_int, [_P, ct.c_int64, _P, ct.c_int64, ct.c_int32, ct.c_double, _P, _P]),
     "gmpsvm_couple": (ct.c_int, [_P, ct.c_int64, ct.c_int32, _P, _P, _P, _P]),
     "gmpsvm_launch_count": (ct.c_uint64, []),
@@ -234,6 +236,14 @@ class Model:
                                             alpha.ctypes.data if alpha is not None else None))
         return dict(b=b.value, A=A.value, B=B.value, alpha=alpha, status=rc)
 
+    def trained_pairs(self):
+        """Indices of the pairs this model holds (all of them unless trained with pair_ids)."""
+        out = []
+        for p, (s, t) in enumerate((s, t) for s in range(self.k) for t in range(s + 1, self.k)):
+            if lib().gmpsvm_model_pair(self._h, s, t, None, None, None, None) >= 0:
+                out.append(p)
+        return out
+
     def sv_index(self):
         idx = np.empty(self.n_sv, dtype=np.int64)
         _check(lib().gmpsvm_model_sv_index(self._h, idx.ctypes.data))
@@ -278,6 +288,26 @@ def train(X, y, k, C, gamma, eps, **opts) -> Model:
     h = ct.c_void_p()
     rc = _check(lib().gmpsvm_train_ex(a.ptr, b.ptr, n, d, int(k), float(C), float(gamma), float(eps), ct.byref(o),
                                       ct.byref(h)))
+    return Model(h.value, rc)
+
+
+def model_from_alpha(X, y, k, C, gamma, alpha, b, A, B, status=None, **opts) -> Model:
+    """gmpsvm_model_from_alpha: the complete model from every pair's (alpha, b, A, B) -- alpha
+    concatenated over pairs in index order, each pair in pair-local order (Model.pair layout)."""
+    a = _Arg(X, np.float32, "X", 2)
+    yy = _Arg(y, np.int32, "y", 1)
+    n, d = a.shape
+    P = int(k) * (int(k) - 1) // 2
+    al = np.ascontiguousarray(alpha, dtype=np.float64)
+    bb, AA, BB = (np.ascontiguousarray(v, dtype=np.float64) for v in (b, A, B))
+    if bb.size != P or AA.size != P or BB.size != P:
+        raise ValueError("b, A, B need k(k-1)/2 entries")
+    st = None if status is None else np.ascontiguousarray(status, dtype=np.int32)
+    o, keep = _options([a, yy], **opts)
+    h = ct.c_void_p()
+    rc = _check(lib().gmpsvm_model_from_alpha(a.ptr, yy.ptr, n, d, int(k), float(C), float(gamma), al.ctypes.data,
+                                              bb.ctypes.data, AA.ctypes.data, BB.ctypes.data,
+                                              st.ctypes.data if st is not None else None, ct.byref(o), ct.byref(h)))
     return Model(h.value, rc)
 
 

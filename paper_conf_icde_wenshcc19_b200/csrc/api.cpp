@@ -380,6 +380,21 @@ int gmpsvm_model_merge(const gmpsvm_model* const* parts, int32_t n_parts, gmpsvm
   });
 }
 
+int gmpsvm_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
+                            const double* alpha, const double* b, const double* A, const double* B,
+                            const int32_t* status, const gmpsvm_options* opt, gmpsvm_model** out) {
+  return guarded([&]() {
+    if (!out) throw Error(GMPSVM_EINVAL, "out is NULL");
+    *out = nullptr;
+    Model* m = nullptr;
+    const int rc = gmpsvm::engine_model_from_alpha(X, y, n, d, k, C, gamma, alpha, b, A, B, status, resolve(opt), &m);
+    auto* h = new gmpsvm_model();
+    h->m.reset(m);
+    *out = h;
+    return rc;
+  });
+}
+
 int gmpsvm_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int32_t d, double gamma, float* K_out,
                       const gmpsvm_options* opt) {
   return guarded([&]() { return gmpsvm::engine_rbf_kernel(X, n, Y, m, d, gamma, K_out, resolve(opt)); });

@@ -1392,6 +1392,86 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
 }
 
 // ------------------------------------------------------------------------------------------
+// The complete model from per-pair solutions computed elsewhere (multi-GPU: each rank trains a
+// pair subset; the ranks all-reduce the disjoint alpha / b / A / B vectors and every rank
+// rebuilds the model from its own replicated X -- only O(sum n_p) doubles cross NVLink instead
+// of serialized SV rows).  alpha: sum_p n_p doubles, pairs in index order, pair-local order (the
+// gmpsvm_model_pair layout); b, A, B: P doubles; status: P int32 or NULL.  Host pointers.
+int engine_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
+                            const double* alpha, const double* b, const double* A, const double* B,
+                            const int32_t* status, const gmpsvm_options& opt, Model** out) {
+  if (!X || !y || !alpha || !b || !A || !B || !out) throw Error(GMPSVM_EINVAL, "null argument");
+  if (n < 2 || d < 1 || k < 2) throw Error(GMPSVM_EINVAL, "need n >= 2, d >= 1, k >= 2");
+  if (k > kMaxK) throw Error(GMPSVM_ENOTIMPL, "k > 64 classes not supported by this build");
+  if (!finite_pos(C) || !finite_pos(gamma)) throw Error(GMPSVM_EINVAL, "C, gamma must be finite and > 0");
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  DevBuf<float> bufX(opt.inputs_on_device ? 0 : (size_t)n * d, st);
+  DevBuf<int32_t> bufY(opt.inputs_on_device ? 0 : (size_t)n, st);
+  const float* dX = X;
+  const int32_t* dy = y;
+  if (!opt.inputs_on_device) {
+    GM_CUDA(cudaMemcpyAsync(bufX.get(), X, (size_t)n * d * 4, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(bufY.get(), y, (size_t)n * 4, cudaMemcpyHostToDevice, st));
+    dX = bufX.get();
+    dy = bufY.get();
+  }
+  // a1: the same stable class sort as training (class-sorted positions <-> original rows)
+  const int nb = (int)ceil_div(n, 1024);
+  DevBuf<int32_t> blk_counts((size_t)nb * (k + 1), st), blk_off((size_t)nb * k, st);
+  DevBuf<int64_t> d_count(k + 1, st), d_off(k + 1, st), d_perm(n, st);
+  launch_class_sort(dy, n, k, blk_counts.get(), blk_off.get(), d_count.get(), d_off.get(), st);
+  std::vector<int64_t> cc(k + 1);
+  GM_CUDA(cudaMemcpyAsync(cc.data(), d_count.get(), (k + 1) * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  if (cc[k] != 0) throw Error(GMPSVM_EINVAL, "labels must be in [0, k)");
+  for (int c = 0; c < k; ++c)
+    if (cc[c] == 0) throw Error(GMPSVM_EINVAL, "every class must have at least one instance");
+  launch_class_rank(dy, n, k, blk_off.get(), d_off.get(), d_perm.get(), st);
+  auto* mdl = new Model();
+  std::unique_ptr<Model> guard(mdl);
+  mdl->k = k;
+  mdl->d = d;
+  mdl->C = C;
+  mdl->gamma = gamma;
+  mdl->n = n;
+  mdl->class_count.assign(cc.begin(), cc.begin() + k);
+  mdl->perm.resize(n);
+  GM_CUDA(cudaMemcpyAsync(mdl->perm.data(), d_perm.get(), (size_t)n * 8, cudaMemcpyDeviceToHost, st));
+  const int P = k * (k - 1) / 2;
+  const auto po = mdl->pair_offsets();
+  mdl->trained.assign(P, 1);
+  mdl->b.assign(b, b + P);
+  mdl->A.assign(A, A + P);
+  mdl->B.assign(B, B + P);
+  mdl->status.assign(P, 0);
+  if (status) mdl->status.assign(status, status + P);
+  mdl->alpha.assign(alpha, alpha + po[P]);
+  for (int64_t j = 0; j < po[P]; ++j)
+    if (!(alpha[j] >= 0.0 && alpha[j] <= C)) throw Error(GMPSVM_EINVAL, "alpha outside [0, C]");
+  // a9: the SV union over the pairs, ascending class-sorted position (Alg 2 l.16, L363)
+  std::vector<int64_t> off(k + 1, 0);
+  for (int c = 0; c < k; ++c) off[c + 1] = off[c] + cc[c];
+  std::vector<uint8_t> is_sv(n, 0);
+  for (int p = 0; p < P; ++p) {
+    const int s = ps_of(p, k), t = pt_of(p, k);
+    for (int64_t j = 0; j < cc[s] + cc[t]; ++j)
+      if (alpha[po[p] + j] > 0.0) is_sv[j < cc[s] ? off[s] + j : off[t] + (j - cc[s])] = 1;
+  }
+  GM_CUDA(cudaStreamSynchronize(st));  // perm on the host
+  for (int64_t g = 0; g < n; ++g)
+    if (is_sv[g]) mdl->sv_pos.push_back(g);
+  std::vector<int64_t> row_of_sv(mdl->sv_pos.size());
+  for (size_t i = 0; i < row_of_sv.size(); ++i) row_of_sv[i] = mdl->perm[mdl->sv_pos[i]];
+  mdl->stats = gmpsvm_train_stats{};
+  mdl->stats.n_sv = (int64_t)mdl->sv_pos.size();
+  mdl->stats.n_pairs_trained = P;
+  mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st);
+  *out = guard.release();
+  return GMPSVM_OK;
+}
+
+// ------------------------------------------------------------------------------------------
 static void ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
   std::lock_guard<std::mutex> lk(mdl.mu);
   if (mdl.dev && mdl.dev->device == device) return;

@@ -3,8 +3,10 @@ sharded for prediction, NCCL used only to gather models and probabilities (SURVE
 
 Training shards naturally: the k(k-1)/2 binary SVMs are independent, so each
 rank trains an LPT-balanced subset of pairs (cost ~ n_p^1.5) with X replicated, and there is
-no collective inside the solver loop.  The partial models are serialized, all-gathered
-(sizes first, then padded blobs) and merged on every rank.  Prediction shards the test rows
+no collective inside the solver loop.  The ranks then combine the disjoint per-pair solutions
+(alpha, b, A, B: O(sum n_p) doubles, one all-reduce over NCCL) and every rank rebuilds the
+complete model from its own replicated X (gmpsvm_model_from_alpha); serializing and merging
+whole partial models (gather_models) remains available.  Prediction shards the test rows
 (instances are independent, L273) and all-gathers the m x k probabilities.
 """
 from __future__ import annotations
@@ -67,6 +69,51 @@ def gather_models(part: "gm.Model", group=None) -> "gm.Model":
     return gm.Model.merge(parts)
 
 
+def pair_layout(counts):
+    """(pair list, offsets of each pair's alpha in the concatenated pair-local layout)."""
+    k = len(counts)
+    pairs = pair_list(k)
+    sizes = [int(counts[s] + counts[t]) for s, t in pairs]
+    return pairs, np.concatenate([[0], np.cumsum(sizes)]).astype(np.int64)
+
+
+def pack_solutions(part: "gm.Model", counts):
+    """This rank's trained pairs as one flat FP64 vector [alpha | b | A | B | status | trained]
+    in the global layout (zeros for pairs other ranks train) -- disjoint across ranks."""
+    pairs, off = pair_layout(counts)
+    P = len(pairs)
+    tot = int(off[-1])
+    v = np.zeros(tot + 5 * P)
+    mine = part.trained_pairs()
+    for p in mine:
+        s, t = pairs[p]
+        info = part.pair(s, t, int(counts[s]), int(counts[t]))
+        v[off[p]:off[p + 1]] = info["alpha"]
+        v[tot + p], v[tot + P + p], v[tot + 2 * P + p] = info["b"], info["A"], info["B"]
+        v[tot + 3 * P + p] = float(info["status"])
+        v[tot + 4 * P + p] = 1.0
+    return v
+
+
+def gather_solutions(part: "gm.Model", X, y, k, C, gamma, group=None, **opts) -> "gm.Model":
+    """All-reduce (sum) of the disjoint per-pair solutions, then the complete model rebuilt from
+    the local X on every rank (identical on all ranks)."""
+    import torch
+    import torch.distributed as dist
+
+    yy = y.cpu().numpy() if isinstance(y, torch.Tensor) else np.asarray(y)
+    counts = np.bincount(yy, minlength=k)
+    v = torch.from_numpy(pack_solutions(part, counts)).to(_backend_device(group))
+    dist.all_reduce(v, op=dist.ReduceOp.SUM, group=group)
+    v = v.cpu().numpy()
+    pairs, off = pair_layout(counts)
+    P, tot = len(pairs), int(off[-1])
+    if not np.all(v[tot + 4 * P:] == 1.0):
+        raise RuntimeError("every pair must be trained by exactly one rank")
+    return gm.model_from_alpha(X, y, k, C, gamma, v[:tot], v[tot:tot + P], v[tot + P:tot + 2 * P],
+                               v[tot + 2 * P:tot + 3 * P], v[tot + 3 * P:tot + 4 * P].astype(np.int32), **opts)
+
+
 def row_range(m, world, rank):
     lo = (m * rank) // world
     hi = (m * (rank + 1)) // world
@@ -106,7 +153,8 @@ def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
     counts = np.bincount(yy, minlength=k)
     mine = plan_pairs(counts, world)[rank]
     part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts)
-    model = gather_models(part, group)
+    dev_opts = {key: opts[key] for key in ("device", "stream") if key in opts}
+    model = gather_solutions(part, X, y, k, C, gamma, group, **dev_opts)
     m = Xt.shape[0]
     lo, hi = row_range(m, world, rank)
     prob_local = model.predict_proba(Xt[lo:hi])

@@ -159,6 +159,47 @@ def test_partial_training_merge_and_serialization_bitwise(gm):
         assert a1["b"] == a2["b"] and a1["A"] == a2["A"]
 
 
+def test_model_from_alpha_and_sharded_gather_bitwise(gm):
+    """The multi-GPU gather path (dist.gather_solutions -> gmpsvm_model_from_alpha): shards of
+    pairs trained separately, their disjoint per-pair solutions summed (gloo, world size 1 here;
+    NCCL across ranks), the complete model rebuilt from X -- predicts bitwise like the full model;
+    a vector that misses a pair or an alpha outside [0, C] is rejected."""
+    import torch.distributed as dist
+
+    from paper_conf_icde_wenshcc19_b200 import dist as gdist
+
+    spec, X, y, Xt, yt = datagen.make_config("letter", n_train=2000, n_test=100)
+    full = gm.train(X, y, spec.k, spec.C, spec.gamma, 1e-3, ws_size=128)
+    counts = np.bincount(y, minlength=spec.k)
+    shards = gdist.plan_pairs(counts, 3)
+    parts = [gm.train(X, y, spec.k, spec.C, spec.gamma, 1e-3, ws_size=128, pair_ids=sh) for sh in shards]
+    v = sum(gdist.pack_solutions(p, counts) for p in parts)
+    pairs, off = gdist.pair_layout(counts)
+    P, tot = len(pairs), int(off[-1])
+    assert np.all(v[tot + 4 * P:] == 1.0)
+    m = gm.model_from_alpha(X, y, spec.k, spec.C, spec.gamma, v[:tot], v[tot:tot + P], v[tot + P:tot + 2 * P],
+                            v[tot + 2 * P:tot + 3 * P])
+    assert m.n_sv == full.n_sv
+    np.testing.assert_array_equal(m.sv_index(), full.sv_index())
+    np.testing.assert_array_equal(m.predict_proba(Xt), full.predict_proba(Xt))
+    np.testing.assert_array_equal(m.decision_function(Xt), full.decision_function(Xt))
+    bad = v[:tot].copy()
+    bad[3] = spec.C * 2
+    with pytest.raises(gm.GmpsvmError):
+        gm.model_from_alpha(X, y, spec.k, spec.C, spec.gamma, bad, v[tot:tot + P], v[tot + P:tot + 2 * P],
+                            v[tot + 2 * P:tot + 3 * P])
+    # the dist driver end to end on a single-process gloo group
+    import os
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29611")
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        model, prob = gdist.train_predict(X, y, Xt, spec.k, spec.C, spec.gamma, 1e-3, ws_size=128)
+        np.testing.assert_array_equal(np.asarray(prob), full.predict_proba(Xt))
+    finally:
+        dist.destroy_process_group()
+
+
 def test_sv_index_matches_alpha(gm):
     spec, X, y, Xt, yt = datagen.make_config("blobs")
     m = gm.train(X, y, 3, spec.C, spec.gamma, 1e-3)
