@@ -210,7 +210,7 @@ def run_gpu(args, spec):
             ev = torch.cuda.Event(enable_timing=True)
             ev.record(stream)
             marks.append(ev)
-            stats.append(model.train_stats())
+            stats.append(getattr(model, "part_stats", None) or model.train_stats())
             pstats.append(gm.last_predict_stats())
         e1.record(stream)
         if len(clk.samples) <= n_warm:  # short timed region: one sample while its last step still runs
@@ -242,7 +242,7 @@ def run_gpu(args, spec):
         model_h, prob_h = step(Xh, yh, Xth, host=True)
     torch.cuda.synchronize(dev)
     e2e_ms = (time.perf_counter() - t0) * 1e3 / args.steps
-    e2e_train = model_h.train_stats() if ws == 1 else {}
+    e2e_train = model_h.train_stats() if ws == 1 else getattr(model_h, "part_stats", {})
     e2e_pred = gm.last_predict_stats()
     if ws > 1:
         t = torch.tensor([e2e_ms], device=dev)

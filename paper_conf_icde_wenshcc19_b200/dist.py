@@ -155,6 +155,7 @@ def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
     part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts)
     dev_opts = {key: opts[key] for key in ("device", "stream") if key in opts}
     model = gather_solutions(part, X, y, k, C, gamma, group, **dev_opts)
+    model.part_stats = part.train_stats()  # this rank's training (the rebuilt model has no solver stats)
     m = Xt.shape[0]
     lo, hi = row_range(m, world, rank)
     prob_local = model.predict_proba(Xt[lo:hi])
