@@ -165,10 +165,13 @@ def run_gpu(args, spec):
     from paper_conf_icde_wenshcc19_b200 import dist as gdist
 
     ws, rank, local = _env_dist()
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # one rank per GPU; GMPSVM_DIST_BACKEND=gloo with more ranks than GPUs is a plumbing check only
+    gpu = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(gpu)
+    dev = torch.device("cuda", gpu)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("GMPSVM_DIST_BACKEND", "nccl")
+        dist.init_process_group(backend, device_id=dev if backend == "nccl" else None)
     _, X, y, Xt, yt = datagen.make_config(spec.name)
     Xd, yd, Xtd = torch.from_numpy(X).to(dev), torch.from_numpy(y).to(dev), torch.from_numpy(Xt).to(dev)
     Xp, yp, Xtp = (torch.from_numpy(X).pin_memory(), torch.from_numpy(y).pin_memory(),
@@ -186,7 +189,7 @@ def run_gpu(args, spec):
 
     # the clock sampler (an nvidia-smi process every 0.2 s) starts during the warm-up, so its
     # start-up cost does not land in the first timed step
-    clk = ClockSampler(local).__enter__()
+    clk = ClockSampler(gpu).__enter__()
     for _ in range(args.warmup):
         model, prob = step(Xd, yd, Xtd)
     torch.cuda.synchronize(dev)
@@ -225,7 +228,7 @@ def run_gpu(args, spec):
     total_ms = e0.elapsed_time(e1)
     step_ms = [e0.elapsed_time(marks[0])] + [marks[i - 1].elapsed_time(marks[i]) for i in range(1, len(marks))]
     if ws > 1:
-        t = torch.tensor([total_ms], device=dev)
+        t = torch.tensor([total_ms], device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     ms = total_ms / args.steps
@@ -245,7 +248,7 @@ def run_gpu(args, spec):
     e2e_train = model_h.train_stats() if ws == 1 else getattr(model_h, "part_stats", {})
     e2e_pred = gm.last_predict_stats()
     if ws > 1:
-        t = torch.tensor([e2e_ms], device=dev)
+        t = torch.tensor([e2e_ms], device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
 
