@@ -35,6 +35,14 @@ METRIC = "train+predict sec on MNIST-shaped 60k×784×10; kernel GFLOP/s vs peak
 FP32_PEAK_TFLOPS_DERIVED = 148 * 128 * 2 * 1.965e9 / 1e12  # SMs x FP32 lanes x 2 x max SM clock
 
 
+def _fp32_peak():
+    """Measured FFMA peak (tools/micro/ffma_peak.cu, profiles/fp32_ffma_peak.json), else derived."""
+    try:
+        return float(json.load(open(os.path.join(ROOT, "profiles", "fp32_ffma_peak.json")))["sustained_tflops"])
+    except Exception:
+        return FP32_PEAK_TFLOPS_DERIVED
+
+
 def _peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -284,7 +292,8 @@ def run_gpu(args, spec):
                                        f"{'' if 'bf16_tflops' in peaks else ' (fallback)'}; the hi/lo split needs 3 MMAs "
                                        "per FP32-accurate product, so peak = that / 3"),
                          "frac_of_mma_peak": achieved / mma_peak,
-                         "frac_of_fp32_simt_peak": achieved / FP32_PEAK_TFLOPS_DERIVED,
+                         "frac_of_fp32_simt_peak": achieved / _fp32_peak(),
+                         "fp32_simt_peak": _fp32_peak(),
                          "flops_per_launch": s["kernel_flops"], "launch_ms": krow_ms,
                          "algorithmic": "n(n+1)/2 kernel values x (2d+3) flop"},
             "phases_ms": {"stage": s["t_stage_ms"], "kernel_values": s["t_kernel_ms"], "select": s["t_select_ms"],
