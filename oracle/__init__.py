@@ -10,6 +10,7 @@ Readings of silent/garbled passages: SURVEY.md §8(c), repeated in DESIGN.md.
 """
 from __future__ import annotations
 
+import contextlib
 import ctypes as ct
 import os
 import subprocess
@@ -65,8 +66,26 @@ def _load():
         lib.oracle_predict.argtypes = [_f32p, _i32p, ct.c_int64, ct.c_int, ct.c_int, ct.c_double, _f64p, _f64p,
                                        _f64p, _f64p, _f32p, ct.c_int64, ct.c_void_p, ct.c_void_p, ct.c_int]
         lib.oracle_predict.restype = ct.c_int
+        lib.oracle_set_kernel.argtypes = [ct.c_int, ct.c_double, ct.c_int]
+        lib.oracle_set_kernel.restype = ct.c_int
         _lib = lib
         return lib
+
+
+KERNELS = {"rbf": 0, "linear": 1, "poly": 2, "sigmoid": 3}
+
+
+@contextlib.contextmanager
+def kernel(kind="rbf", coef0=0.0, degree=3):
+    """Every oracle call inside uses this kernel (LibSVM definitions):
+    rbf exp(-gamma |x-y|^2), linear x.y, poly (gamma x.y + coef0)^degree, sigmoid
+    tanh(gamma x.y + coef0).  Process-wide; restored to rbf on exit."""
+    if _load().oracle_set_kernel(KERNELS[kind], float(coef0), int(degree)) != 0:
+        raise ValueError("bad kernel parameters")
+    try:
+        yield
+    finally:
+        _load().oracle_set_kernel(0, 0.0, 3)
 
 
 def default_threads() -> int:

@@ -55,8 +55,25 @@ void parallel_for(int64_t n, int nthreads, const std::function<void(int64_t)>& f
   for (auto& x : th) x.join();
 }
 
-// Gaussian kernel: K(x_i, x_j) = exp(-gamma ||x_i - x_j||^2), direct differences.
+// Kernel functions: the Gaussian kernel K(x_i, x_j) = exp(-gamma ||x_i - x_j||^2)
+// (direct differences) is the default; oracle_set_kernel selects the other kernels the paper lists
+// (NEXT-4): linear x_i.x_j, polynomial (gamma x_i.x_j + coef0)^degree, sigmoid
+// tanh(gamma x_i.x_j + coef0) -- the LibSVM definitions.  Set before a call, process-wide.
+struct KernelSpec {
+  int type = 0;  // 0 RBF, 1 linear, 2 polynomial, 3 sigmoid
+  double coef0 = 0.0;
+  int degree = 3;
+};
+KernelSpec g_kernel;
+
 inline double rbf(const float* xi, const float* xj, int d, double gamma) {
+  if (g_kernel.type != 0) {
+    double dot = 0.0;
+    for (int c = 0; c < d; ++c) dot += (double)xi[c] * (double)xj[c];
+    if (g_kernel.type == 1) return dot;
+    if (g_kernel.type == 2) return std::pow(gamma * dot + g_kernel.coef0, (double)g_kernel.degree);
+    return std::tanh(gamma * dot + g_kernel.coef0);
+  }
   double s = 0.0;
   for (int c = 0; c < d; ++c) {
     double diff = (double)xi[c] - (double)xj[c];
@@ -412,6 +429,15 @@ int oracle_sigmoid_fit(const double* v, const int32_t* y, int64_t n, double* A, 
 }
 
 int oracle_couple(const double* r, int k, double* p) { return couple(r, k, p); }
+
+// Kernel of every following call (NEXT-4; type 0 = the paper's RBF, the default).
+int oracle_set_kernel(int type, double coef0, int degree) {
+  if (type < 0 || type > 3 || degree < 1) return -1;
+  g_kernel.type = type;
+  g_kernel.coef0 = coef0;
+  g_kernel.degree = degree;
+  return 0;
+}
 
 // ---------------------------------------------------------------------------------------
 // Multi-class training (Algorithm 2; pairs L191-L195).

@@ -160,3 +160,35 @@ def test_smo_matches_sklearn_libsvm():
         f = oracle.exact_f(X, y, a, spec.gamma)
         b = -oracle.rho(a, f, y, spec.C)
         np.testing.assert_allclose(sign * clf.intercept_[0], b, atol=1e-6)
+
+
+# ------------------------------------------------------------------------------------ NEXT-4
+@pytest.mark.parametrize("kind,gamma,coef0,degree", [("linear", 1.0, 0.0, 3), ("poly", 0.5, 1.0, 3),
+                                                     ("poly", 0.3, 0.5, 2), ("sigmoid", 0.05, -0.5, 3)])
+def test_other_kernels_match_closed_forms_and_sklearn(kind, gamma, coef0, degree):
+    """The paper's other kernels (L76-L78, LibSVM definitions): the kernel matrix equals the
+    closed form computed with numpy, and the SMO fixed point (alpha, SV set, intercept) equals
+    scikit-learn's LibSVM with the same kernel at tight tolerance."""
+    sk = pytest.importorskip("sklearn.svm")
+    spec, X, y = _pair("blobs", 0, 1)
+    X64 = X.astype(np.float64)
+    dot = X64 @ X64.T
+    closed = {"linear": dot, "poly": (gamma * dot + coef0) ** degree, "sigmoid": np.tanh(gamma * dot + coef0)}[kind]
+    C = 0.5 if kind == "sigmoid" else spec.C
+    with oracle.kernel(kind, coef0, degree):
+        K = oracle.rbf_matrix(X, X, gamma)
+        np.testing.assert_allclose(K, closed, rtol=1e-12, atol=1e-12)
+        r = oracle.smo(X, y, C, gamma, 1e-10)
+        a = r["alpha"]
+        f = oracle.exact_f(X, y, a, gamma)
+        b = -oracle.rho(a, f, y, C)
+    clf = sk.SVC(C=C, kernel=kind, gamma=gamma, coef0=coef0, degree=degree, tol=1e-10, shrinking=False,
+                 cache_size=200)
+    clf.fit(X64, y)
+    a_sk = np.zeros(len(y))
+    a_sk[clf.support_] = np.abs(clf.dual_coef_[0])
+    np.testing.assert_allclose(a, a_sk, atol=1e-5 * C)
+    sign = np.sign(clf.dual_coef_[0][0] * y[clf.support_[0]])
+    np.testing.assert_allclose(sign * clf.intercept_[0], b, atol=1e-5)
+    # and the default is restored
+    np.testing.assert_allclose(np.diag(oracle.rbf_matrix(X[:5], X[:5], gamma)), 1.0)
