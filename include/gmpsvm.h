@@ -76,8 +76,19 @@ typedef struct {
   int32_t inputs_on_device; /* 1: X/y/Xtest/out are device pointers on `device`             */
   int64_t max_outer_iter;   /* cap on outer (working-set) iterations per pair; 0 = 1,000,000 */
   int32_t inner_iter_cap;   /* cap on inner SMO steps per working set; 0 = 100 * B          */
-  int32_t reserved[7];
+  int32_t kernel;           /* GMPSVM_KERNEL_*: the paper's RBF (L75, default) or one of the
+                               other kernels it lists (L76-L78; LibSVM definitions, gamma the
+                               train call's): training needs the FULL_K regime on the tensor
+                               cores (else GMPSVM_ENOTIMPL); prediction runs in FP64         */
+  double coef0;             /* polynomial / sigmoid offset (LibSVM coef0); default 0         */
+  int32_t degree;           /* polynomial degree; 0 = 3                                      */
+  int32_t reserved[3];
 } gmpsvm_options;
+
+enum { GMPSVM_KERNEL_RBF = 0,      /* exp(-gamma |x - y|^2)                 */
+       GMPSVM_KERNEL_LINEAR = 1,   /* x . y                                 */
+       GMPSVM_KERNEL_POLY = 2,     /* (gamma x . y + coef0)^degree          */
+       GMPSVM_KERNEL_SIGMOID = 3   /* tanh(gamma x . y + coef0)             */ };
 
 /* Per-phase CUDA-event times of the last training run (mirrors the paper's Fig 11
  * breakdown, L483-L497) and counters. */

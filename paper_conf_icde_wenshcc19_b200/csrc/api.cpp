@@ -105,7 +105,7 @@ std::vector<uint8_t> serialize(const Model& m) {
   w.put<int32_t>(GMPSVM_ABI_VERSION);
   w.put<int32_t>(m.k);
   w.put<int32_t>(m.d);
-  w.put<int32_t>(0);
+  w.put<int32_t>(m.kernel);
   w.put<double>(m.C);
   w.put<double>(m.gamma);
   w.put<double>(m.eps);
@@ -122,6 +122,8 @@ std::vector<uint8_t> serialize(const Model& m) {
   w.put_vec(m.sv_pos);
   w.put_vec(m.sv_X);
   w.put(m.stats);
+  w.put<double>(m.coef0);
+  w.put<int32_t>(m.degree);
   return std::move(w.buf);
 }
 
@@ -132,7 +134,8 @@ Model* deserialize(const void* buf, size_t len) {
   if (r.get<int32_t>() != GMPSVM_ABI_VERSION) throw Error(GMPSVM_EFORMAT, "model blob version mismatch");
   m->k = r.get<int32_t>();
   m->d = r.get<int32_t>();
-  r.get<int32_t>();
+  m->kernel = r.get<int32_t>();
+  if (m->kernel < 0 || m->kernel > 3) throw Error(GMPSVM_EFORMAT, "bad kernel type");
   m->C = r.get<double>();
   m->gamma = r.get<double>();
   m->eps = r.get<double>();
@@ -161,6 +164,8 @@ Model* deserialize(const void* buf, size_t len) {
       throw Error(GMPSVM_EFORMAT, "bad SV positions");
   r.get_vec(m->sv_X, (size_t)nsv * m->d);
   m->stats = r.get<gmpsvm_train_stats>();
+  m->coef0 = r.get<double>();
+  m->degree = r.get<int32_t>();
   m->sv_X_ready = true;
   return m.release();
 }
@@ -170,7 +175,8 @@ Model* merge(const Model* const* parts, int n) {
   const Model& f = *parts[0];
   for (int i = 0; i < n; ++i) {
     const Model& q = *parts[i];
-    if (q.k != f.k || q.d != f.d || q.n != f.n || q.C != f.C || q.gamma != f.gamma || q.class_count != f.class_count ||
+    if (q.k != f.k || q.d != f.d || q.n != f.n || q.C != f.C || q.gamma != f.gamma || q.kernel != f.kernel ||
+        q.coef0 != f.coef0 || q.degree != f.degree || q.class_count != f.class_count ||
         q.perm != f.perm)
       throw Error(GMPSVM_EINVAL, "parts were not trained on the same problem");
     std::lock_guard<std::mutex> lk(q.mu);
@@ -183,6 +189,9 @@ Model* merge(const Model* const* parts, int n) {
   m->C = f.C;
   m->gamma = f.gamma;
   m->eps = f.eps;
+  m->kernel = f.kernel;
+  m->coef0 = f.coef0;
+  m->degree = f.degree;
   m->n = f.n;
   m->class_count = f.class_count;
   m->perm = f.perm;

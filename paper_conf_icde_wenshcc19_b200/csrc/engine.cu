@@ -500,7 +500,8 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   for (int p = 0; p < P; ++p) dm->cond = std::max(dm->cond, std::fabs(m.A[p]) / 4.0 * std::ldexp(1.0, -22) * abs_sum[p]);
   static const char* dec_env = getenv("GMPSVM_DEC");
   const std::string dec_mode = dec_env ? dec_env : "";
-  dm->f64 = dec_mode == "f64" || (dec_mode.empty() && dm->cond > kDecF64Cond);
+  // the other kernels (L76-L78) predict through the FP64 path only (its epilogue has them)
+  dm->f64 = m.kernel != 0 || dec_mode == "f64" || (dec_mode.empty() && dm->cond > kDecF64Cond);
   if (dm->f64) dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
   if (dev_coef) {
     dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st);
@@ -615,6 +616,11 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   if (k > kMaxK) throw Error(GMPSVM_ENOTIMPL, "k > 64 classes not supported by this build");
   if (n >= (int64_t)1 << 31) throw Error(GMPSVM_ENOTIMPL, "n >= 2^31 not supported");
   if (!finite_pos(C) || !finite_pos(gamma) || !finite_pos(eps)) throw Error(GMPSVM_EINVAL, "C, gamma, eps must be finite and > 0");
+  const int ktype = opt.kernel;  // GMPSVM_KERNEL_*: the paper's RBF or one of its other kernels (L76-L78)
+  const double kcoef0 = opt.coef0;
+  const int kdegree = opt.degree ? opt.degree : 3;
+  if (ktype < 0 || ktype > 3 || kdegree < 1 || kdegree > 16 || !std::isfinite(kcoef0))
+    throw Error(GMPSVM_EINVAL, "kernel must be 0..3, degree 1..16, coef0 finite");
   int B = opt.ws_size ? opt.ws_size : kDefaultB;
   if (B < 2 || B > 1024 || (B & 1)) throw Error(GMPSVM_EINVAL, "ws_size must be even and in [2, 1024]");
   int q = opt.q ? opt.q : B / 2;
@@ -658,6 +664,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)device_total_mem(opt.device);
   const bool full_k = bytes_K <= budget;
   const bool use_tc = full_k && krow_use_tc();
+  if (ktype != 0 && !(use_tc && krow_split_f16()))
+    throw Error(GMPSVM_ENOTIMPL, "the linear / polynomial / sigmoid kernels need the FULL_K regime on the tensor cores");
   const int d_pad = use_tc ? krow_tc_d_pad(d) : (int)round_up(d, kBK);
   // ROW_CACHE column tiles start at 4-aligned segment starts and may run 127 columns past n
   const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile) + (full_k ? 0 : kTile);
@@ -670,7 +678,8 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   DevBuf<uint8_t> tc_scratch(use_tc ? krow_tc_scratch_bytes(n, d) : 0, st);
   if (use_tc) {
     launch_row_norms(dX, n, d, d_perm.get(), norms.get(), n_pad, bad.get(), st);  // validation (non-finite rows)
-    ksc = launch_split_tf32(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st);
+    ksc = launch_split_tf32(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st,
+                            ktype == 0);
   } else {
     launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
   }
@@ -795,13 +804,13 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   // predict) -- the waves' tensor/HBM load stretches the solver's latency-bound chain more than
   // the overlap saves.
   static const bool overlap_env = getenv("GMPSVM_OVERLAP") && std::string(getenv("GMPSVM_OVERLAP")) == "1";
-  const bool overlap = overlap_env && use_tc && graph_solver_default(B) && ws_solve_supported(B, np_max);
+  const bool overlap = overlap_env && ktype == 0 && use_tc && graph_solver_default(B) && ws_solve_supported(B, np_max);
   cudaStream_t kst = krow_stream(opt.device);
   TimedEvents kev;
   cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
   std::vector<int> wave_off;     // tile range of wave w: [wave_off[w], wave_off[w + 1])
   std::vector<int> ready_wave;   // per pair position: the wave after which its kernel values are complete
-  const bool two_cta = use_tc && !overlap && krow_tc_2cta();  // the overlap waves use single-CTA tiles
+  const bool two_cta = use_tc && !overlap && ktype == 0 && krow_tc_2cta();  // overlap waves: single-CTA tiles
   double kv_subset = -1;  // >= 0: kernel values computed for a pair subset (tiles skipped)
   if (use_tc) {
     tiles = krow_tc_tiles(n, two_cta);
@@ -887,8 +896,11 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   }
   tm.mark(PH_KERNEL);
   if (use_tc && !overlap)
+  {
+    const KrowKernel kk{ktype, (float)gamma, (float)kcoef0, 0.f, kdegree};
     launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, ksc, K.get(),
-                   ldk, st, two_cta);
+                   ldk, st, two_cta, ktype != 0 ? &kk : nullptr);
+  }
   else if (full_k && !use_tc)
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   tm.mark(PH_KERNEL);
@@ -1308,6 +1320,9 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
   mdl->C = C;
   mdl->gamma = gamma;
   mdl->eps = eps;
+  mdl->kernel = ktype;
+  mdl->coef0 = kcoef0;
+  mdl->degree = kdegree;
   mdl->n = n;
   mdl->class_count.assign(cc.begin(), cc.begin() + k);
   mdl->perm.assign(h_permp, h_permp + n);
@@ -1434,6 +1449,11 @@ int engine_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t
   mdl->d = d;
   mdl->C = C;
   mdl->gamma = gamma;
+  mdl->kernel = opt.kernel;
+  mdl->coef0 = opt.coef0;
+  mdl->degree = opt.degree ? opt.degree : 3;
+  if (mdl->kernel < 0 || mdl->kernel > 3 || mdl->degree < 1 || mdl->degree > 16 || !std::isfinite(mdl->coef0))
+    throw Error(GMPSVM_EINVAL, "kernel must be 0..3, degree 1..16, coef0 finite");
   mdl->n = n;
   mdl->class_count.assign(cc.begin(), cc.begin() + k);
   mdl->perm.resize(n);
@@ -1569,7 +1589,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
       launch_col_norms64(xt, mcp, mcp, dm.d_pad, nt64.get(), st);
       GM_CUDA(cudaMemsetAsync(part64.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 8, st));
       launch_dec_f64(xt, mcp, nt64.get(), mcp, dm.SvT, dm.nsv_pad, dm.nsv64, dm.coef64, dm.km1, dm.km1_pad, dm.items,
-                     dm.n_items, dm.d_pad, mdl.gamma, part64.get(), st);
+                     dm.n_items, dm.d_pad, mdl.gamma, part64.get(), st, mdl.kernel, mdl.coef0, mdl.degree);
       launch_dec_reduce64(part64.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     } else if (use_tc) {
       GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
@@ -1618,6 +1638,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
 int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int32_t d, double gamma, float* K_out,
                       const gmpsvm_options& opt) {
   if (n < 0 || m < 0 || d < 1 || !finite_pos(gamma)) throw Error(GMPSVM_EINVAL, "bad rbf_kernel arguments");
+  if (opt.kernel != 0) throw Error(GMPSVM_ENOTIMPL, "gmpsvm_rbf_kernel computes the Gaussian kernel only");
   if (n == 0 || m == 0) return GMPSVM_OK;
   if (!X || !Y || !K_out) throw Error(GMPSVM_EINVAL, "null argument");
   DeviceGuard dg(opt.device);

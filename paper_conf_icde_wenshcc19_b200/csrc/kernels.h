@@ -37,7 +37,13 @@ float krow_split_scale(float maxabs);  // exact power-of-two scale of the FP16 s
 size_t krow_tc_scratch_bytes(int64_t n, int d);
 const float* krow_tc_scratch_mu(const void* scratch, int64_t n, int d);
 float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
-                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st);
+                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st, bool center = true);
+// the paper's other kernels (L76-L78): type 1 linear, 2 polynomial, 3 sigmoid (inv_s2 set by the launch)
+struct KrowKernel {
+  int type;
+  float gamma, coef0, inv_s2;
+  int degree;
+};
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
 bool krow_tc_2cta();
@@ -65,7 +71,7 @@ void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* 
                    float* part, cudaStream_t st);
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
-                    bool two_cta = false);
+                    bool two_cta = false, const KrowKernel* dk = nullptr);
 void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
                       cudaStream_t st);
 bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel
@@ -163,7 +169,8 @@ void launch_dec_contract(const float* XtT, int64_t ldt, const float* nt, int64_t
 void launch_col_norms64(const float* XT, int64_t ld, int64_t n, int d_pad, double* out, cudaStream_t st);
 void launch_dec_f64(const float* XtT, int64_t ldt, const double* nt64, int64_t m_pad, const float* SvT, int64_t lds,
                     const double* nsv64, const double* coef64, int km1, int km1_pad, const DecItem* items, int n_items,
-                    int d_pad, double gamma, double* part, cudaStream_t st);
+                    int d_pad, double gamma, double* part, cudaStream_t st, int ktype = 0, double coef0 = 0.0,
+                    int degree = 3);
 void launch_dec_reduce64(const double* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,
                          const int32_t* item_end, const double* b, double* dec, cudaStream_t st);
 void launch_dec_reduce(const float* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,

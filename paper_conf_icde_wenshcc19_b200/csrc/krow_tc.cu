@@ -172,16 +172,34 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
       : "r"(taddr));
 }
 
+// The paper's other kernels (L76-L78, NEXT-4) on the same contraction: with uncentred rows the
+// tensor cores deliver s^2 x . y; K = x.y, (gamma x.y + coef0)^degree or tanh(gamma x.y + coef0).
+template <int KT>  // 1 linear, 2 polynomial, 3 sigmoid
+__device__ __forceinline__ float dot_kernel_value(float xy, const KrowKernel& kp) {
+  if (KT == 1) return xy;
+  const float z = fmaf(kp.gamma, xy, kp.coef0);
+  if (KT == 3) return tanhf(z);
+  float v = 1.f, b = z;  // z^degree by squaring, degree <= 16: no data-dependent loop in the epilogue
+  int e = kp.degree;
+#pragma unroll
+  for (int i = 0; i < 5; ++i) {
+    if (e & 1) v *= b;
+    b *= b;
+    e >>= 1;
+  }
+  return v;
+}
+
 // Persistent: one CTA per SM walks the tile list (tile = blockIdx.x + i * gridDim.x).  The TMA
 // producer runs ahead across tile boundaries through the smem ring; the epilogue drains the four
 // TMEM accumulators into registers and releases TMEM at once (tmem_empty), so the MMAs of the
 // next tile overlap the exp + stores of the current one.
-template <bool F16>
+template <bool F16, int KT>  // KT: 0 the Gaussian, else a dot-product kernel (kp): 1 linear, 2 poly, 3 sigmoid
 __global__ void __launch_bounds__(kTcThreads, 1)
     krow_tc_kernel(const __grid_constant__ CUtensorMap map_hi, const __grid_constant__ CUtensorMap map_lo,
                    const __grid_constant__ CUtensorMap map_ksw, const __grid_constant__ CUtensorMap map_kns,
                    const int2* __restrict__ tiles, int n_tiles, const float* __restrict__ norms, int64_t n, int nk,
-                   float scale, float* __restrict__ K, int64_t ldk, int tma_store) {
+                   float scale, float* __restrict__ K, int64_t ldk, int tma_store, KrowKernel kp) {
   extern __shared__ __align__(1024) uint8_t dsmem[];
   TcSmem& sm = *reinterpret_cast<TcSmem*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -325,8 +343,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           float kv[32];
 #pragma unroll
           for (int j = 0; j < 32; ++j) {
-            const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cn, j));
-            asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv[j]) : "f"(fmaxf(d2, 0.f) * scale));
+            if (KT != 0) {
+              kv[j] = dot_kernel_value<KT>(dot[ch * 32 + j] * kp.inv_s2, kp);
+            } else {
+              const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cn, j));
+              asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv[j]) : "f"(fmaxf(d2, 0.f) * scale));
+            }
           }
           if (lane == 0) bulk_wait_read0();  // the previous chunk's stores have read the staging
           __syncwarp();
@@ -352,10 +374,14 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         float kv[32];
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
-          const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cnv[ch], j));
-          float val;
-          asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(val) : "f"(fmaxf(d2, 0.f) * scale));
-          kv[j] = (r == cb + j) ? 1.f : val;
+          if (KT != 0) {
+            kv[j] = dot_kernel_value<KT>(dot[ch * 32 + j] * kp.inv_s2, kp);  // K_ii computed (not 1)
+          } else {
+            const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cnv[ch], j));
+            float val;
+            asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(val) : "f"(fmaxf(d2, 0.f) * scale));
+            kv[j] = (r == cb + j) ? 1.f : val;
+          }
         }
         // direct store K[r][c] for r <= c (row segment of 32 contiguous floats)
         if (r < n) {
@@ -1041,12 +1067,16 @@ void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm,
 }
 
 float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
-                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st) {
+                        int64_t n_pad, int d_pad, void* scratch, cudaStream_t st, bool center) {
   const int nch = (int)ceil_div(n, kMeanRows);
   double* part = static_cast<double*>(scratch);
   float* mu = reinterpret_cast<float*>(part + (size_t)nch * d);
-  GM_LAUNCH(col_partial_kernel, dim3((unsigned)ceil_div(d, 128), (unsigned)nch), dim3(128), 0, st, X, n, d, part);
-  GM_LAUNCH(col_mean_kernel, dim3((unsigned)ceil_div(d, 128)), dim3(128), 0, st, part, nch, n, d, mu);
+  if (center) {  // RBF: translation invariant, centring shrinks the dot products
+    GM_LAUNCH(col_partial_kernel, dim3((unsigned)ceil_div(d, 128), (unsigned)nch), dim3(128), 0, st, X, n, d, part);
+    GM_LAUNCH(col_mean_kernel, dim3((unsigned)ceil_div(d, 128)), dim3(128), 0, st, part, nch, n, d, mu);
+  } else {  // dot-product kernels need x . y itself
+    GM_CUDA(cudaMemsetAsync(mu, 0, (size_t)d * sizeof(float), st));
+  }
   const float sc = krow_split_f16() ? krow_split_scale(launch_maxabs(X, n, d, nullptr, mu, st)) : 1.f;
   launch_split_tf32_mu(X, n, d, perm, mu, sc, hi, lo, norms, n_pad, d_pad, st);
   return sc;
@@ -1138,7 +1168,7 @@ CUtensorMap make_kmap(float* K, int64_t n, int64_t ldk, bool swizzle) {
 
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
-                    bool two_cta) {
+                    bool two_cta, const KrowKernel* dk) {
   const bool f16 = krow_split_f16();
   const CUtensorMap mhi = make_map(hi, n_pad, d_pad, f16), mlo = make_map(lo, n_pad, d_pad, f16);
   // TMA stores need a 16-byte aligned base and row stride; otherwise every tile takes the
@@ -1149,8 +1179,11 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
   const size_t smem = sizeof(TcSmem) + 1024;
   static bool configured = false;
   if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<false, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     configured = true;
   }
   // distances are in units scaled by sc: exp(-gamma d2 / sc^2) = exp2(d2 * scale)
@@ -1177,12 +1210,25 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
   static const int reserve = getenv("GMPSVM_KROW_RESERVE") ? std::max(0, atoi(getenv("GMPSVM_KROW_RESERVE"))) : 0;
   const int cap = std::max(1, sms - reserve);
   const int grid = n_tiles < cap ? n_tiles : cap;
-  if (f16)
-    GM_LAUNCH(krow_tc_kernel<true>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles, norms,
-              n, nk, scale, K, ldk, tma);
-  else
-    GM_LAUNCH(krow_tc_kernel<false>, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles,
-              norms, n, nk, scale, K, ldk, tma);
+  KrowKernel kp{};
+  if (dk) {
+    if (!f16 || two_cta) throw Error(GMPSVM_ENOTIMPL, "dot-product kernels need the FP16-split single-CTA launch");
+    kp = *dk;
+    kp.inv_s2 = (float)(1.0 / ((double)sc * (double)sc));
+    auto go = [&](auto kern) {
+      GM_LAUNCH(kern, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles, norms, n, nk, scale,
+                K, ldk, tma, kp);
+    };
+    if (kp.type == 1) go(krow_tc_kernel<true, 1>);
+    else if (kp.type == 2) go(krow_tc_kernel<true, 2>);
+    else go(krow_tc_kernel<true, 3>);
+  } else if (f16) {
+    GM_LAUNCH((krow_tc_kernel<true, 0>), dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles,
+              n_tiles, norms, n, nk, scale, K, ldk, tma, kp);
+  } else {
+    GM_LAUNCH((krow_tc_kernel<false, 0>), dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles,
+              n_tiles, norms, n, nk, scale, K, ldk, tma, kp);
+  }
 }
 
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,

@@ -56,6 +56,9 @@ struct DevModel {
 struct Model {
   int32_t k = 0, d = 0;
   double C = 0, gamma = 0, eps = 0;
+  int32_t kernel = 0;  // GMPSVM_KERNEL_* (0 = RBF)
+  double coef0 = 0;
+  int32_t degree = 3;
   int64_t n = 0;
   std::vector<int64_t> class_count;  // [k]
   std::vector<int64_t> perm;         // class-sorted position -> original index [n]

@@ -257,7 +257,8 @@ __global__ void __launch_bounds__(256) dec_f64_kernel(const float* __restrict__ 
                                                       int64_t lds, const double* __restrict__ nsv64,
                                                       const double* __restrict__ coef64, int km1, int km1_pad,
                                                       const DecItem* __restrict__ items, int kdim, double gamma,
-                                                      int64_t m_pad, double* __restrict__ part) {
+                                                      int64_t m_pad, double* __restrict__ part, int ktype,
+                                                      double coef0, int degree) {
   extern __shared__ __align__(16) unsigned char dsm[];
   double* as = reinterpret_cast<double*>(dsm);        // [kF64BK][64]
   double* bs = as + kF64BK * kF64Tile;                // [kF64BK][64]
@@ -301,8 +302,18 @@ __global__ void __launch_bounds__(256) dec_f64_kernel(const float* __restrict__ 
       const double nc = nsv64[c0 + tx * 4 + j];
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
-        const double d2 = nr[i] + nc - 2.0 * acc[i][j];
-        acc[i][j] = exp(-gamma * (d2 > 0.0 ? d2 : 0.0));  // K in FP64
+        if (ktype == 0) {
+          const double d2 = nr[i] + nc - 2.0 * acc[i][j];
+          acc[i][j] = exp(-gamma * (d2 > 0.0 ? d2 : 0.0));  // K in FP64
+        } else if (ktype == 1) {  // linear: x . y (L76-L78)
+        } else if (ktype == 2) {  // polynomial
+          const double z = fma(gamma, acc[i][j], coef0);
+          double v = 1.0;
+          for (int e = 0; e < degree; ++e) v *= z;
+          acc[i][j] = v;
+        } else {  // sigmoid
+          acc[i][j] = tanh(fma(gamma, acc[i][j], coef0));
+        }
       }
     }
     for (int u = 0; u < km1; ++u) {
@@ -371,7 +382,7 @@ void launch_col_norms64(const float* XT, int64_t ld, int64_t n, int d_pad, doubl
 
 void launch_dec_f64(const float* XtT, int64_t ldt, const double* nt64, int64_t m_pad, const float* SvT, int64_t lds,
                     const double* nsv64, const double* coef64, int km1, int km1_pad, const DecItem* items, int n_items,
-                    int d_pad, double gamma, double* part, cudaStream_t st) {
+                    int d_pad, double gamma, double* part, cudaStream_t st, int ktype, double coef0, int degree) {
   const size_t smem = (size_t)(2 * kF64BK * kF64Tile + 2 * kF64Tile * km1_pad) * sizeof(double);
   static bool configured = false;
   if (!configured) {
@@ -379,7 +390,7 @@ void launch_dec_f64(const float* XtT, int64_t ldt, const double* nt64, int64_t m
     configured = true;
   }
   GM_LAUNCH(dec_f64_kernel, dim3((unsigned)(m_pad / kF64Tile), (unsigned)n_items), dim3(256), smem, st, XtT, ldt, nt64,
-            SvT, lds, nsv64, coef64, km1, km1_pad, items, d_pad, gamma, m_pad, part);
+            SvT, lds, nsv64, coef64, km1, km1_pad, items, d_pad, gamma, m_pad, part, ktype, coef0, degree);
 }
 
 void launch_dec_reduce64(const double* part, int64_t m, int64_t m_pad, int k, int km1_pad, const int32_t* item_begin,

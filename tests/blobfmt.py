@@ -43,4 +43,5 @@ def make_blob(X, y, k, C, gamma, eps, alphas, b, A, B, stats_size):
     out += alpha.tobytes()
     out += struct.pack("<q", len(sv_pos)) + sv_pos.tobytes() + sv_X.tobytes()
     out += bytes(stats_size)
+    out += struct.pack("<di", 0.0, 3)  # kernel coef0, degree (the kernel type is the header's 4th int: 0 = RBF)
     return np.frombuffer(bytes(out), dtype=np.uint8), perm, sv_pos

@@ -330,3 +330,33 @@ def test_fp64_decision_path_vs_oracle(gm, tmp_path):
     dec_o, prob_o = oracle.predict(ref, X, y, Xt)
     assert np.abs(r["dec"] - dec_o).max() <= 1e-9 * max(1.0, np.abs(dec_o).max())
     assert np.abs(r["prob"] - prob_o).max() <= 1e-9
+
+
+# ------------------------------------------------------------------------------------ NEXT-4
+@pytest.mark.parametrize("name,kind,gamma,coef0,degree,C", [
+    ("blobs", "linear", 1.0, 0.0, 3, 1.0), ("blobs", "poly", 0.5, 1.0, 3, 1.0), ("blobs", "sigmoid", 0.02, 0.0, 3, 1.0),
+    ("letter", "poly", 0.3, 1.0, 2, 1.0), ("letter", "linear", 1.0, 0.0, 3, 0.5)])
+def test_other_kernels_vs_oracle(gm, name, kind, gamma, coef0, degree, C):
+    """The paper's other kernels (L76-L78; NEXT-4) through the same FULL_K tensor-core
+    contraction (uncentred rows; K = f(x.y)) and the FP64 decision path: the same fixed point
+    (alpha, SV sets, b, probabilities, KKT audit) as the oracle with that kernel.  The sigmoid
+    kernel is not positive semi-definite in general (the dual then has several KKT points, SURVEY
+    §8(c) #28); it is checked where it is close to the linear one (coef0 = 0, small gamma)."""
+    n = None if name == "blobs" else 1200
+    spec, X, y, Xt, yt = datagen.make_config(name, n_train=n, n_test=None if name == "blobs" else 200)
+    with oracle.kernel(kind, coef0, degree):
+        ref = oracle.train(X, y, spec.k, C, gamma, EPS)
+        model = gm.train(X, y, spec.k, C, gamma, EPS, kernel=kind, coef0=coef0, degree=degree)
+        _compare_models(model, ref, X, y, C)
+        _, prob_o = oracle.predict(ref, X, y, Xt, want_dec=False)
+    prob = model.predict_proba(Xt)
+    assert np.abs(prob - prob_o).max() <= 1e-4
+    # round trip keeps the kernel
+    rt = gm.Model.deserialize(model.serialize())
+    np.testing.assert_array_equal(rt.predict_proba(Xt), prob)
+
+
+def test_other_kernels_need_full_k(gm):
+    spec, X, y, Xt, yt = datagen.make_config("blobs")
+    with pytest.raises(gm.GmpsvmError):
+        gm.train(X, y, spec.k, 1.0, 1.0, 1e-3, kernel="linear", cache_bytes=1)  # ROW_CACHE: not built
