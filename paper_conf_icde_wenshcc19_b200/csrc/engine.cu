@@ -501,8 +501,10 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   static const char* dec_env = getenv("GMPSVM_DEC");
   const std::string dec_mode = dec_env ? dec_env : "";
   // the other kernels (L76-L78) predict through the FP64 path only (its epilogue has them)
-  dm->f64 = m.kernel != 0 || dec_mode == "f64" || (dec_mode.empty() && dm->cond > kDecF64Cond);
-  if (dm->f64) dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
+  dm->f64 = (m.kernel != 0 && (!krow_use_tc() || !krow_split_f16() || dm->km1_pad > 12 || dec_mode == "simt")) ||
+            dec_mode == "f64" || (dec_mode.empty() && dm->cond > kDecF64Cond);
+  // FP64 coefficients also for the other kernels' fallback (test rows outside the FP16 range)
+  if (dm->f64 || m.kernel != 0) dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
   if (dev_coef) {
     dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st);
     if (alpha_tot) GM_CUDA(cudaMemcpyAsync(dm->alpha_dev, alpha_hp, (size_t)alpha_tot * 8, cudaMemcpyDeviceToDevice, st));
@@ -516,7 +518,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
                       dm->coef, dm->coef64, st);
   } else {
     GM_CUDA(cudaMemcpyAsync(dm->coef, coef.data(), coef.size() * 4, cudaMemcpyHostToDevice, st));
-    if (dm->f64) GM_CUDA(cudaMemcpyAsync(dm->coef64, coef64.data(), coef64.size() * 8, cudaMemcpyHostToDevice, st));
+    if (dm->coef64) GM_CUDA(cudaMemcpyAsync(dm->coef64, coef64.data(), coef64.size() * 8, cudaMemcpyHostToDevice, st));
   }
   GM_CUDA(cudaMemcpyAsync(dm->items, items.data(), items.size() * sizeof(DecItem), cudaMemcpyHostToDevice, st));
   GM_CUDA(cudaMemcpyAsync(dm->item_begin, ib.data(), k * 4, cudaMemcpyHostToDevice, st));
@@ -527,7 +529,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
   HT("h2d_svt");
-  if (dm->f64) {
+  if (dm->coef64) {
     dm->nsv64 = dev_alloc<double>(dm->nsv_pad, st);
     launch_col_norms64(dm->SvT, dm->nsv_pad, dm->nsv_pad, dm->d_pad, dm->nsv64, st);
   }
@@ -544,6 +546,9 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
     if (mu_in) {
       GM_CUDA(cudaMemcpyAsync(dm->mu, mu_in, (size_t)m.d * 4, cudaMemcpyDeviceToDevice, st));
       dm->sc = sc_in;
+    } else if (m.kernel != 0) {  // dot-product kernels: uncentred rows (x . y itself)
+      GM_CUDA(cudaMemsetAsync(dm->mu, 0, (size_t)m.d * 4, st));
+      dm->sc = krow_split_scale(launch_maxabs(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, st));
     } else {
       launch_gather_col_mean(rows, m.d, d_src.get(), dm->nsv_pad, nsv, dm->mu, st);
       HT("mean");
@@ -1533,8 +1538,9 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   DevBuf<float> Xhi(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st), Xlo(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st);
   // the SIMT decision values need the feature-major copy only as the FP16-range fallback
   DevBuf<float> XtTf(dm.tc ? (size_t)dm.d_pad * mc_pad : 0, st);
-  DevBuf<float> part(dm.f64 ? 0 : (size_t)dm.n_items * mc_pad * dm.km1_pad, st);
-  DevBuf<double> part64(dm.f64 ? (size_t)dm.n_items * mc_pad * dm.km1_pad : 0, st), nt64(dm.f64 ? mc_pad : 0, st);
+  DevBuf<float> part((size_t)dm.n_items * mc_pad * dm.km1_pad, st);
+  const bool may64 = dm.f64 || mdl.kernel != 0;
+  DevBuf<double> part64(may64 ? (size_t)dm.n_items * mc_pad * dm.km1_pad : 0, st), nt64(may64 ? mc_pad : 0, st);
   DevBuf<double> dec_buf(opt.inputs_on_device ? 0 : (size_t)mc_max * P, st);
   DevBuf<double> prob_buf((opt.inputs_on_device || !prob_out) ? 0 : (size_t)mc_max * k, st);
   DevBuf<double> dec_tmp((opt.inputs_on_device && !dec_out) ? (size_t)mc_max * P : 0, st);
@@ -1555,6 +1561,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     // FP16 split: test rows far outside the SVs' range would overflow half precision -> SIMT
     const bool use_tc = !dm.f64 && dm.tc &&
                         (!krow_split_f16() || launch_maxabs(src, mc, d, nullptr, dm.mu, st) * dm.sc < 60000.f);
+    const bool f64 = dm.f64 || (mdl.kernel != 0 && !use_tc);  // the SIMT fallback is the Gaussian's only
     if (use_tc) {
       launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
       launch_split_tf32_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
@@ -1584,7 +1591,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     tm.mark(PH_STAGE);
     double* dec_d = opt.inputs_on_device ? (dec_out ? dec_out + i0 * P : dec_tmp.get()) : dec_buf.get();
     tm.mark(PH_DEC);
-    if (dm.f64) {  // ill-conditioned model: FP64 decision values
+    if (f64) {  // ill-conditioned model (or another kernel off the tensor cores): FP64 decision values
       float* xt = dm.tc ? XtTf.get() : XtT.get();
       launch_col_norms64(xt, mcp, mcp, dm.d_pad, nt64.get(), st);
       GM_CUDA(cudaMemsetAsync(part64.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 8, st));
@@ -1594,14 +1601,17 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     } else if (use_tc) {
       GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
       if (n_units > 0)
+      {
+        const KrowKernel kk{mdl.kernel, (float)mdl.gamma, (float)mdl.coef0, 0.f, mdl.degree};
         launch_dec_tc(Xhi.get(), Xlo.get(), mcp, dm.SvHi, dm.SvLo, dm.nsv_pad, dm.dpt, d_dtiles.get(), d_uoff.get(),
                       d_uitem.get(), n_units, nt.get(), dm.nsvc, dm.coef, dm.km1, dm.km1_pad, mdl.gamma, dm.sc, part.get(),
-                      st);
+                      st, mdl.kernel != 0 ? &kk : nullptr);
+      }
     } else {
       launch_dec_contract(dm.tc ? XtTf.get() : XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef,
                           dm.km1, dm.km1_pad, dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
     }
-    if (!dm.f64) launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
+    if (!f64) launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     ps.dec_launches += 1;
     tm.mark(PH_DEC);
     double* prob_d = nullptr;

@@ -68,7 +68,8 @@ int dec_tc_max_km1();
 void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* shi, const void* slo, int64_t nsv_pad,
                    int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item, int n_units,
                    const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma, float sc,
-                   float* part, cudaStream_t st);
+                   float* part, cudaStream_t st,
+                   const KrowKernel* dk = nullptr);
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
                     bool two_cta = false, const KrowKernel* dk = nullptr);

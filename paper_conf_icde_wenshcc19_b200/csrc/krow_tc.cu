@@ -731,14 +731,16 @@ struct DecTcSmem {
   uint32_t tmem_base;
 };
 
-template <int KM, bool F16>  // KM: compile-time bound of the pair columns (k - 1 <= KM, KM % 4 == 0)
+// KM: compile-time bound of the pair columns (k - 1 <= KM, KM % 4 == 0); KT: 0 the Gaussian, else
+// a dot-product kernel of L76-L78 (uncentred rows, kp), as krow_tc_kernel
+template <int KM, bool F16, int KT = 0>
 __global__ void __launch_bounds__(kTcThreads, 1)
     dec_tc_kernel(const __grid_constant__ CUtensorMap map_thi, const __grid_constant__ CUtensorMap map_tlo,
                   const __grid_constant__ CUtensorMap map_shi, const __grid_constant__ CUtensorMap map_slo,
                   const int2* __restrict__ tiles, const int32_t* __restrict__ unit_off,
                   const int32_t* __restrict__ unit_item, int n_units, const float* __restrict__ nt,
                   const float* __restrict__ nsv, const float* __restrict__ coef, int km1, int km1_pad, int nk,
-                  float scale, int64_t m_pad, float* __restrict__ part) {
+                  float scale, int64_t m_pad, float* __restrict__ part, KrowKernel kp) {
   extern __shared__ __align__(1024) uint8_t dsmem[];
   DecTcSmem<KM>& sm =
       *reinterpret_cast<DecTcSmem<KM>*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
@@ -854,9 +856,13 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         const float nr = nt[r];
 #pragma unroll
         for (int j = 0; j < kTN; ++j) {
-          const float d2 = fmaf(-2.f, dot[j], nr + __ldg(nsv + c0 + j));
           float kv;
-          asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv) : "f"(fmaxf(d2, 0.f) * scale));
+          if (KT != 0) {
+            kv = dot_kernel_value<KT>(dot[j] * kp.inv_s2, kp);
+          } else {
+            const float d2 = fmaf(-2.f, dot[j], nr + __ldg(nsv + c0 + j));
+            asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(kv) : "f"(fmaxf(d2, 0.f) * scale));
+          }
           const float4* cj = reinterpret_cast<const float4*>(cs + j * KM);
 #pragma unroll
           for (int v4 = 0; v4 < KM / 4; ++v4) {
@@ -1247,7 +1253,7 @@ int dec_tc_max_km1() { return kDecMaxKm1; }
 void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* shi, const void* slo, int64_t nsv_pad,
                    int d_pad, const int2* tiles, const int32_t* unit_off, const int32_t* unit_item, int n_units,
                    const float* nt, const float* nsv, const float* coef, int km1, int km1_pad, double gamma, float sc,
-                   float* part, cudaStream_t st) {
+                   float* part, cudaStream_t st, const KrowKernel* dk) {
   const bool f16 = krow_split_f16();
   const CUtensorMap mthi = make_map(thi, m_pad, d_pad, f16), mtlo = make_map(tlo, m_pad, d_pad, f16);
   const CUtensorMap mshi = make_map(shi, nsv_pad, d_pad, f16), mslo = make_map(slo, nsv_pad, d_pad, f16);
@@ -1255,16 +1261,26 @@ void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* 
   const int sms = num_sms();
   const int grid = n_units < sms ? n_units : sms;
   const int nk = d_pad / (f16 ? 2 * kTK : kTK);
+  KrowKernel kp{};
+  if (dk) {
+    kp = *dk;
+    kp.inv_s2 = (float)(1.0 / ((double)sc * (double)sc));
+  }
   auto go = [&](auto kern, size_t smem, bool& configured) {
     if (!configured) {
       GM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       configured = true;
     }
     GM_LAUNCH(kern, dim3(grid), dim3(kTcThreads), smem, st, mthi, mtlo, mshi, mslo, tiles, unit_off, unit_item, n_units,
-              nt, nsv, coef, km1, km1_pad, nk, scale, m_pad, part);
+              nt, nsv, coef, km1, km1_pad, nk, scale, m_pad, part, kp);
   };
-  static bool c[4] = {false, false, false, false};
-  if (km1_pad <= 12) {
+  static bool c[7] = {false, false, false, false, false, false, false};
+  if (dk) {  // the other kernels: FP16 split, k - 1 <= 12 (engine.cu routes the rest to the FP64 path)
+    if (!f16 || km1_pad > 12) throw Error(GMPSVM_ENOTIMPL, "tensor-core decision values of this kernel need k <= 13");
+    if (kp.type == 1) go(dec_tc_kernel<12, true, 1>, sizeof(DecTcSmem<12>) + 1024, c[4]);
+    else if (kp.type == 2) go(dec_tc_kernel<12, true, 2>, sizeof(DecTcSmem<12>) + 1024, c[5]);
+    else go(dec_tc_kernel<12, true, 3>, sizeof(DecTcSmem<12>) + 1024, c[6]);
+  } else if (km1_pad <= 12) {
     if (f16) go(dec_tc_kernel<12, true>, sizeof(DecTcSmem<12>) + 1024, c[0]);
     else go(dec_tc_kernel<12, false>, sizeof(DecTcSmem<12>) + 1024, c[1]);
   } else {
