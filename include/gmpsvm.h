@@ -82,7 +82,13 @@ typedef struct {
                                cores (else GMPSVM_ENOTIMPL); prediction runs in FP64         */
   double coef0;             /* polynomial / sigmoid offset (LibSVM coef0); default 0         */
   int32_t degree;           /* polynomial degree; 0 = 3                                      */
-  int32_t reserved[3];
+  int32_t prob_folds;       /* 0: sigmoids fitted on the pairs' in-sample decision values (the
+                               paper, L193-L195; reading R10).  F >= 2: LibSVM's practice
+                               (NEXT-2): F-fold cross-validated decision values -- F extra
+                               trainings on the other folds (fold of an instance = its rank
+                               within its class mod F), the sigmoid of each pair fitted on the
+                               out-of-fold values; every class needs >= F instances         */
+  int32_t reserved[2];
 } gmpsvm_options;
 
 enum { GMPSVM_KERNEL_RBF = 0,      /* exp(-gamma |x - y|^2)                 */

@@ -199,6 +199,47 @@ def train(X, labels, k, C, gamma, eps, nthreads=None):
                 gamma=float(gamma), C=float(C))
 
 
+def fold_of(labels, k, folds):
+    """Fold of each instance for cross-validated sigmoids (NEXT-2; R30): its rank
+    within its class (original order) mod folds.  Returns (fold, rank, class counts)."""
+    labels = np.asarray(labels)
+    rank = np.zeros(len(labels), dtype=np.int64)
+    cnt = np.zeros(k, dtype=np.int64)
+    for i, c in enumerate(labels):
+        rank[i] = cnt[c]
+        cnt[c] += 1
+    return rank % folds, rank, cnt
+
+
+def train_cv(X, labels, k, C, gamma, eps, folds=5, nthreads=None):
+    """LibSVM's probability training (ref [15]) with deterministic folds: for each fold, train
+    (Alg 2) on the other folds and evaluate Eq 11 on the held-out rows; each pair's sigmoid
+    (Eq 12-13) is fitted on its out-of-fold decision values; the final model is trained on all
+    rows and carries those A, B.  Also returns the out-of-fold values v[p] (pair-local order)."""
+    X, labels = _f32(X), _i32(labels)
+    fold, rank, cnt = fold_of(labels, k, folds)
+    pairs = pair_list(k)
+    v = [np.full(cnt[s] + cnt[t], np.nan) for s, t in pairs]
+    for f in range(folds):
+        tr, ho = fold != f, fold == f
+        mf = train(X[tr], labels[tr], k, C, gamma, eps, nthreads)
+        dec, _ = predict(mf, X[tr], labels[tr], X[ho], nthreads)
+        for h, i in enumerate(np.flatnonzero(ho)):
+            c, r = labels[i], rank[i]
+            for p, (s, t) in enumerate(pairs):
+                if c == s:
+                    v[p][r] = dec[h, p]
+                elif c == t:
+                    v[p][cnt[s] + r] = dec[h, p]
+    A, B = np.zeros(len(pairs)), np.zeros(len(pairs))
+    for p, (s, t) in enumerate(pairs):
+        ypm = np.concatenate([np.ones(cnt[s], np.int32), -np.ones(cnt[t], np.int32)])
+        A[p], B[p], _, _ = sigmoid_fit(v[p], ypm)
+    model = train(X, labels, k, C, gamma, eps, nthreads)
+    model["A"], model["B"], model["v_cv"] = A, B, v
+    return model
+
+
 def predict(model, X, labels, Xt, nthreads=None, want_dec=True):
     """(dec [m, P], prob [m, k]) by Eq 11, 12, 14/15 from an oracle-format model."""
     X, labels, Xt = _f32(X), _i32(labels), _f32(Xt)

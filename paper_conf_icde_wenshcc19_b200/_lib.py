@@ -30,7 +30,7 @@ class Options(ct.Structure):
                 ("cache_bytes", ct.c_int64), ("stream", ct.c_void_p), ("pair_ids", ct.POINTER(ct.c_int32)),
                 ("n_pair_ids", ct.c_int32), ("inputs_on_device", ct.c_int32), ("max_outer_iter", ct.c_int64),
                 ("inner_iter_cap", ct.c_int32), ("kernel", ct.c_int32), ("coef0", ct.c_double), ("degree", ct.c_int32),
-                ("reserved", ct.c_int32 * 3)]
+                ("prob_folds", ct.c_int32), ("reserved", ct.c_int32 * 2)]
 
 
 KERNELS = {"rbf": 0, "linear": 1, "poly": 2, "sigmoid": 3}  # GMPSVM_KERNEL_*
@@ -145,7 +145,7 @@ class _Arg:
 
 
 def _options(args, ws_size=0, q=0, pair_ids=None, stream=None, max_outer_iter=0, inner_iter_cap=0, cache_bytes=0,
-             device=None, kernel="rbf", coef0=0.0, degree=3):
+             device=None, kernel="rbf", coef0=0.0, degree=3, prob_folds=0):
     o = Options()
     lib().gmpsvm_options_init(ct.byref(o))
     dev_flags = {a.on_device for a in args if a is not None}
@@ -167,6 +167,7 @@ def _options(args, ws_size=0, q=0, pair_ids=None, stream=None, max_outer_iter=0,
     o.ws_size, o.q = int(ws_size), int(q)
     o.max_outer_iter, o.inner_iter_cap, o.cache_bytes = int(max_outer_iter), int(inner_iter_cap), int(cache_bytes)
     o.kernel, o.coef0, o.degree = KERNELS[kernel], float(coef0), int(degree)
+    o.prob_folds = int(prob_folds)
     keep = None
     if pair_ids is not None:
         keep = (ct.c_int32 * len(pair_ids))(*[int(p) for p in pair_ids])

@@ -602,8 +602,138 @@ void ensure_host_alpha(const Model& mdl) {
 }
 
 // ------------------------------------------------------------------------------------------
+static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
+                             double eps, const gmpsvm_options& opt, Model** out);
+
+// NEXT-2, LibSVM's probability training (ref [15]; the paper fits on in-sample values, R10):
+// F-fold cross-validated decision values.  Fold of instance i = (its rank within its class,
+// original order) mod F.  For each fold: train on the other folds (all pairs), decision values of
+// the held-out rows (Eq 11) scattered into the pairs' pair-local layout; then every pair's
+// sigmoid (Eq 12-13) is fitted on its out-of-fold values, and the final model (trained on all
+// rows) gets those A, B.  All steps are the library's own kernels; F + 1 trainings.
+static int engine_train_cv(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
+                           double eps, const gmpsvm_options& opt, Model** out) {
+  const auto t_start = std::chrono::steady_clock::now();
+  const int F = opt.prob_folds;
+  if (F < 2 || F > 64) throw Error(GMPSVM_EINVAL, "prob_folds must be 0 or in [2, 64]");
+  if (opt.pair_ids && opt.n_pair_ids > 0)
+    throw Error(GMPSVM_ENOTIMPL, "cross-validated sigmoids need all pairs (no pair_ids)");
+  if (!X || !y || !out) throw Error(GMPSVM_EINVAL, "null argument");
+  if (n < 2 || d < 1 || k < 2) throw Error(GMPSVM_EINVAL, "need n >= 2, d >= 1, k >= 2");
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  std::vector<int32_t> hy(n);
+  if (opt.inputs_on_device) GM_CUDA(cudaMemcpy(hy.data(), y, (size_t)n * 4, cudaMemcpyDeviceToHost));
+  else std::memcpy(hy.data(), y, (size_t)n * 4);
+  std::vector<int64_t> rank(n), cnt(k, 0);
+  for (int64_t i = 0; i < n; ++i) {
+    if (hy[i] < 0 || hy[i] >= k) throw Error(GMPSVM_EINVAL, "labels must be in [0, k)");
+    rank[i] = cnt[hy[i]]++;
+  }
+  for (int c = 0; c < k; ++c)
+    if (cnt[c] < F) throw Error(GMPSVM_EINVAL, "prob_folds: every class needs at least `prob_folds` instances");
+  DevBuf<float> bufX(opt.inputs_on_device ? 0 : (size_t)n * d, st);
+  const float* dX = X;
+  if (!opt.inputs_on_device) {
+    GM_CUDA(cudaMemcpyAsync(bufX.get(), X, (size_t)n * d * 4, cudaMemcpyHostToDevice, st));
+    dX = bufX.get();
+  }
+  gmpsvm_options o2 = opt;
+  o2.prob_folds = 0;
+  o2.inputs_on_device = 1;
+  o2.stream = st;
+  const int P = k * (k - 1) / 2;
+  std::vector<PairDesc> pdv(P);
+  int64_t tot = 0;
+  for (int p = 0; p < P; ++p) {
+    PairDesc& x = pdv[p];
+    std::memset(&x, 0, sizeof(x));
+    x.s = ps_of(p, k);
+    x.t = pt_of(p, k);
+    x.n_s = (int32_t)cnt[x.s];
+    x.n_t = (int32_t)cnt[x.t];
+    x.a_off = tot;
+    x.pid = p;
+    tot += x.n_s + x.n_t;
+  }
+  DevBuf<PairDesc> d_pairs(P, st);
+  GM_CUDA(cudaMemcpyAsync(d_pairs.get(), pdv.data(), (size_t)P * sizeof(PairDesc), cudaMemcpyHostToDevice, st));
+  DevBuf<double> d_v(tot, st);
+  GM_CUDA(cudaMemsetAsync(d_v.get(), 0, (size_t)tot * 8, st));
+  for (int f = 0; f < F; ++f) {
+    std::vector<int64_t> tr, ho;
+    std::vector<int32_t> ytr, cls;
+    std::vector<int64_t> rk;
+    for (int64_t i = 0; i < n; ++i) {
+      if (rank[i] % F != f) {
+        tr.push_back(i);
+        ytr.push_back(hy[i]);
+      } else {
+        ho.push_back(i);
+        cls.push_back(hy[i]);
+        rk.push_back(rank[i]);
+      }
+    }
+    const int64_t ntr = (int64_t)tr.size(), nho = (int64_t)ho.size();
+    DevBuf<int64_t> d_tr(ntr, st), d_ho(nho, st), d_rk(nho, st);
+    DevBuf<int32_t> d_ytr(ntr, st), d_cls(nho, st);
+    DevBuf<float> Xtr((size_t)ntr * d, st), Xho((size_t)nho * d, st);
+    DevBuf<double> dec((size_t)nho * P, st);
+    GM_CUDA(cudaMemcpyAsync(d_tr.get(), tr.data(), (size_t)ntr * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_ho.get(), ho.data(), (size_t)nho * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_rk.get(), rk.data(), (size_t)nho * 8, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_ytr.get(), ytr.data(), (size_t)ntr * 4, cudaMemcpyHostToDevice, st));
+    GM_CUDA(cudaMemcpyAsync(d_cls.get(), cls.data(), (size_t)nho * 4, cudaMemcpyHostToDevice, st));
+    launch_gather_rows(dX, d, d_tr.get(), ntr, Xtr.get(), st);
+    launch_gather_rows(dX, d, d_ho.get(), nho, Xho.get(), st);
+    Model* mf = nullptr;
+    engine_train_core(Xtr.get(), d_ytr.get(), ntr, d, k, C, gamma, eps, o2, &mf);
+    std::unique_ptr<Model> gf(mf);
+    engine_predict(*mf, Xho.get(), nho, nullptr, dec.get(), o2);
+    launch_scatter_oof(dec.get(), nho, P, d_cls.get(), d_rk.get(), d_pairs.get(), d_v.get(), st);
+    GM_CUDA(cudaStreamSynchronize(st));  // fold buffers go out of scope
+  }
+  DevBuf<double> dA(P, st), dB(P, st);
+  DevBuf<int32_t> dS(P, st);
+  launch_sigmoid_fit_on(d_pairs.get(), P, d_v.get(), dA.get(), dB.get(), dS.get(), st);
+  std::vector<double> hA(P), hB(P);
+  std::vector<int32_t> hS(P);
+  GM_CUDA(cudaMemcpyAsync(hA.data(), dA.get(), (size_t)P * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(hB.data(), dB.get(), (size_t)P * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(hS.data(), dS.get(), (size_t)P * 4, cudaMemcpyDeviceToHost, st));
+  DevBuf<int32_t> bufY(opt.inputs_on_device ? 0 : (size_t)n, st);
+  const int32_t* dy = y;
+  if (!opt.inputs_on_device) {
+    GM_CUDA(cudaMemcpyAsync(bufY.get(), hy.data(), (size_t)n * 4, cudaMemcpyHostToDevice, st));
+    dy = bufY.get();
+  }
+  Model* m = nullptr;
+  int rc = engine_train_core(dX, dy, n, d, k, C, gamma, eps, o2, &m);
+  std::unique_ptr<Model> gm(m);
+  GM_CUDA(cudaStreamSynchronize(st));
+  for (int p = 0; p < P; ++p) {  // the cross-validated sigmoids replace the in-sample ones
+    m->A[p] = hA[p];
+    m->B[p] = hB[p];
+    m->status[p] = (m->status[p] & 0xff) | (hS[p] << 8);
+    if (hS[p] == 1) rc = GMPSVM_WARN_MAXITER;
+  }
+  if (m->dev) {
+    GM_CUDA(cudaMemcpy(m->dev->A, hA.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+    GM_CUDA(cudaMemcpy(m->dev->B, hB.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  }
+  m->stats.t_total_ms = host_ms_since(t_start);
+  *out = gm.release();
+  return rc;
+}
+
 int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma, double eps,
                  const gmpsvm_options& opt, Model** out) {
+  if (opt.prob_folds != 0) return engine_train_cv(X, y, n, d, k, C, gamma, eps, opt, out);
+  return engine_train_core(X, y, n, d, k, C, gamma, eps, opt, out);
+}
+
+static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
+                             double eps, const gmpsvm_options& opt, Model** out) {
   const auto t_start = std::chrono::steady_clock::now();
   // GMPSVM_HOST_TIMING=1: host-clock checkpoints of the training call on stderr
   static const bool host_timing = getenv("GMPSVM_HOST_TIMING") != nullptr;

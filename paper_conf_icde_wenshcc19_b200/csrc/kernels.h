@@ -47,6 +47,10 @@ struct KrowKernel {
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
 bool krow_tc_2cta();
+void launch_scatter_oof(const double* dec, int64_t m, int P, const int32_t* cls, const int64_t* rnk,
+                        const PairDesc* pairs, double* v, cudaStream_t st);
+void launch_sigmoid_fit_on(const PairDesc* pairs, int P, const double* v, double* A, double* B, int32_t* status,
+                           cudaStream_t st);
 void launch_build_coef(const double* alpha, const int64_t* aoff, const int64_t* slot_g, const int64_t* off,
                        const int64_t* cc, int k, int64_t nsv_pad, int km1_pad, float* coef, double* coef64,
                        cudaStream_t st);

@@ -18,6 +18,8 @@
 #include <string>
 
 #include "gemm_simt.cuh"
+#include <cstring>
+
 #include "kernels.h"
 #include "solver_dev.cuh"
 
@@ -1631,6 +1633,42 @@ void launch_f_update_loop(const SolverArgs& a, int P, int64_t np_max, cudaGraphC
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st) {
   GM_LAUNCH(finalize_kernel, dim3(P), dim3(1024), 0, st, a);
 }
+// NEXT-2: out-of-fold decision values of held-out rows into the pairs' pair-local layout.
+// Row h (class cls[h], rank rnk[h] within its class) of a fold's held-out set feeds every pair
+// (s, t) containing its class: v[a_off(p) + (cls == s ? rnk : n_s + rnk)] = dec[h][p].
+__global__ void scatter_oof_kernel(const double* __restrict__ dec, int64_t m, int P, const int32_t* __restrict__ cls,
+                                   const int64_t* __restrict__ rnk, const PairDesc* __restrict__ pairs,
+                                   double* __restrict__ v) {
+  const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (gid >= m * P) return;
+  const int64_t h = gid / P;
+  const int p = (int)(gid % P);
+  const PairDesc pd = pairs[p];
+  const int c = cls[h];
+  if (c != pd.s && c != pd.t) return;
+  v[pd.a_off + (c == pd.s ? rnk[h] : pd.n_s + rnk[h])] = dec[gid];
+}
+
+void launch_scatter_oof(const double* dec, int64_t m, int P, const int32_t* cls, const int64_t* rnk,
+                        const PairDesc* pairs, double* v, cudaStream_t st) {
+  const int64_t tot = m * (int64_t)P;
+  if (tot > 0) GM_LAUNCH(scatter_oof_kernel, dim3((unsigned)ceil_div(tot, 256)), dim3(256), 0, st, dec, m, P, cls, rnk, pairs, v);
+}
+
+// the Platt fit (Eq 12-13) of every pair on given decision values v (pair-local layout, a_off)
+void launch_sigmoid_fit_on(const PairDesc* pairs, int P, const double* v, double* A, double* B, int32_t* status,
+                           cudaStream_t st) {
+  SolverArgs a;
+  std::memset(&a, 0, sizeof(a));
+  a.pairs = pairs;
+  a.v = const_cast<double*>(v);
+  a.A = A;
+  a.Bs = B;
+  a.sig_status = status;
+  a.pair_base = 0;
+  GM_LAUNCH(sigmoid_fit_kernel, dim3(P), dim3(512), 0, st, a);
+}
+
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st) {
   GM_LAUNCH(sigmoid_fit_kernel, dim3(P), dim3(512), 0, st, a);
 }

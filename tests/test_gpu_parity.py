@@ -360,3 +360,22 @@ def test_other_kernels_need_full_k(gm):
     spec, X, y, Xt, yt = datagen.make_config("blobs")
     with pytest.raises(gm.GmpsvmError):
         gm.train(X, y, spec.k, 1.0, 1.0, 1e-3, kernel="linear", cache_bytes=1)  # ROW_CACHE: not built
+
+
+# ------------------------------------------------------------------------------------ NEXT-2
+@pytest.mark.parametrize("name,folds", [("blobs", 5), ("mnist", 3)])
+def test_cross_validated_sigmoids_vs_oracle(gm, name, folds):
+    """prob_folds = F (LibSVM's probability training, NEXT-2): F extra trainings on the other
+    folds, each pair's sigmoid fitted on its out-of-fold decision values -- the same A, B and
+    probabilities as oracle.train_cv on the same deterministic folds (R30)."""
+    n, m = (None, None) if name == "blobs" else (1500, 200)
+    spec, X, y, Xt, yt = datagen.make_config(name, n_train=n, n_test=m)
+    ref = oracle.train_cv(X, y, spec.k, spec.C, spec.gamma, EPS, folds=folds)
+    model = gm.train(X, y, spec.k, spec.C, spec.gamma, EPS, prob_folds=folds)
+    counts = np.bincount(y, minlength=spec.k)
+    for p, (s, t) in enumerate(oracle.pair_list(spec.k)):
+        info = model.pair(s, t, counts[s], counts[t])
+        assert abs(info["A"] - ref["A"][p]) <= 1e-3 * max(1.0, abs(ref["A"][p])), (p, info["A"], ref["A"][p])
+        assert abs(info["B"] - ref["B"][p]) <= 1e-3 * max(1.0, abs(ref["B"][p])), (p, info["B"], ref["B"][p])
+    _, prob_o = oracle.predict(ref, X, y, Xt, want_dec=False)
+    assert np.abs(model.predict_proba(Xt) - prob_o).max() <= 1e-4

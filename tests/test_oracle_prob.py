@@ -143,3 +143,41 @@ def test_pipeline_in_sample_identity_and_sklearn():
     # Table-4 pattern (L423-L436): errors of the probabilistic classifier are sane
     test_err = (prob_t := oracle.predict(m, X, y, Xt, want_dec=False)[1]).argmax(1) != yt
     assert test_err.mean() < 0.2
+
+
+# ------------------------------------------------------------------------------------ NEXT-2
+def test_cross_validated_sigmoids_oracle():
+    """oracle.train_cv (LibSVM's F-fold probability training, deterministic folds R30): every
+    pair's out-of-fold decision value of an instance equals Eq 11 evaluated independently (numpy,
+    direct-difference RBF) with the model trained without that instance's fold; the sigmoid is
+    the unique minimiser on those values (zero gradient); every value is filled exactly once."""
+    import datagen
+
+    spec, X, y, _, _ = datagen.make_config("blobs")
+    folds = 3
+    m = oracle.train_cv(X, y, spec.k, spec.C, spec.gamma, 1e-6, folds=folds)
+    fold, rank, cnt = oracle.fold_of(y, spec.k, folds)
+    pairs = oracle.pair_list(spec.k)
+    assert all(np.isfinite(v).all() for v in m["v_cv"])
+    rng = np.random.default_rng(3)
+    for i in rng.choice(len(y), size=6, replace=False):
+        f = fold[i]
+        tr = fold != f
+        mf = oracle.train(X[tr], y[tr], spec.k, spec.C, spec.gamma, 1e-6)
+        Xtr, ytr = X[tr].astype(np.float64), y[tr]
+        for p, (s, t) in enumerate(pairs):
+            if y[i] not in (s, t):
+                continue
+            idx = np.concatenate([np.flatnonzero(ytr == s), np.flatnonzero(ytr == t)])
+            ypm = np.where(ytr[idx] == s, 1.0, -1.0)
+            Kx = np.exp(-spec.gamma * ((Xtr[idx] - X[i].astype(np.float64)) ** 2).sum(1))
+            dec = (mf["alpha"][p] * ypm * Kx).sum() + mf["b"][p]
+            j = rank[i] if y[i] == s else cnt[s] + rank[i]
+            np.testing.assert_allclose(m["v_cv"][p][j], dec, rtol=1e-9, atol=1e-9)
+    for p, (s, t) in enumerate(pairs):
+        ypm = np.concatenate([np.ones(cnt[s]), -np.ones(cnt[t])])
+        tgt = np.where(ypm > 0, (cnt[s] + 1) / (cnt[s] + 2), 1 / (cnt[t] + 2))
+        z = m["A"][p] * m["v_cv"][p] + m["B"][p]
+        P1 = 1 / (1 + np.exp(z))
+        gA, gB = ((tgt - P1) * m["v_cv"][p]).sum(), (tgt - P1).sum()
+        assert abs(gA) < 1e-4 and abs(gB) < 1e-4
