@@ -148,6 +148,16 @@ GMPSVM_API int gmpsvm_train_ex(const float* X, const int32_t* y, int64_t n, int3
 
 /* Probability estimation (L259-L273, L331-L363): out [m x k] FP64 row-major, caller-
  * allocated; each row sums to 1.  Requires a model with every pair trained. */
+/* CSR input (NEXT-3; the sparse format of the paper's datasets, L385): row i's nonzeros are
+ * values[indptr[i] .. indptr[i+1]) at columns indices[.] (each in [0, d), else EINVAL).  The rows
+ * are densified on the device and take the dense path (the kernel-value contraction runs on the
+ * dense rows).  indptr: n+1 int64; indices: nnz int32; values: nnz float; host or device pointers
+ * per opt->inputs_on_device.  y, model, out, errors as gmpsvm_train_ex / gmpsvm_predict_proba. */
+GMPSVM_API int gmpsvm_train_csr(const int64_t* indptr, const int32_t* indices, const float* values, const int32_t* y,
+                                int64_t n, int32_t d, int32_t k, double C, double gamma, double eps,
+                                const gmpsvm_options* opt, gmpsvm_model** out);
+GMPSVM_API int gmpsvm_predict_proba_csr(const gmpsvm_model* model, const int64_t* indptr, const int32_t* indices,
+                                        const float* values, int64_t m, double* out, const gmpsvm_options* opt);
 GMPSVM_API int gmpsvm_predict_proba(const gmpsvm_model* model, const float* Xtest, int64_t m, double* out);
 GMPSVM_API int gmpsvm_predict_proba_ex(const gmpsvm_model* model, const float* Xtest, int64_t m, double* out,
                             const gmpsvm_options* opt);

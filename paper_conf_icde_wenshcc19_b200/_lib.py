@@ -78,6 +78,9 @@ _SIGS = {
     "gmpsvm_model_serialize": (ct.c_int, [_P, _P, _P]),
     "gmpsvm_model_deserialize": (ct.c_int, [_P, ct.c_size_t, _P]),
     "gmpsvm_model_merge": (ct.c_int, [_P, ct.c_int32, _P]),
+    "gmpsvm_train_csr": (ct.c_int, [_P, _P, _P, _P, ct.c_int64, ct.c_int32, ct.c_int32, ct.c_double, ct.c_double,
+                                    ct.c_double, _P, _P]),
+    "gmpsvm_predict_proba_csr": (ct.c_int, [_P, _P, _P, _P, ct.c_int64, _P, _P]),
     "gmpsvm_model_from_alpha": (ct.c_int, [_P, _P, ct.c_int64, ct.c_int32, ct.c_int32, ct.c_double, ct.c_double, _P, _P,
                                            _P, _P, _P, _P, _P]),
     "gmpsvm_rbf_kernel": (ct.c_int, [_P, ct.c_int64, _P, ct.c_int64, ct.c_int32, ct.c_double, _P, _P]),
@@ -123,7 +126,8 @@ class _Arg:
         self.device = 0
         if _is_torch(x):
             import torch
-            tdt = {np.float32: torch.float32, np.float64: torch.float64, np.int32: torch.int32}[dtype]
+            tdt = {np.float32: torch.float32, np.float64: torch.float64, np.int32: torch.int32,
+                   np.int64: torch.int64}[dtype]
             if x.dtype != tdt:
                 raise TypeError(f"{name}: expected {tdt}, got {x.dtype}")
             if not x.is_contiguous():
@@ -221,6 +225,18 @@ class Model:
         _check(lib().gmpsvm_predict_proba_ex(self._h, a.ptr, m, _data_ptr(out), ct.byref(o)))
         return out
 
+    def predict_proba_csr(self, csr, out=None, **opts):
+        """predict_proba for CSR rows (gmpsvm_predict_proba_csr): a scipy.sparse CSR matrix, or
+        (indptr int64, indices int32, values float32, (m, d)) as numpy arrays / CUDA tensors."""
+        ip, ix, vv, (m, d) = _csr_args(csr)
+        if d != self.d:
+            raise ValueError(f"CSR rows must have {self.d} columns")
+        if out is None:
+            out = _empty((m, self.k), np.float64, ip)
+        o, keep = _options([ip, ix, vv], **opts)
+        _check(lib().gmpsvm_predict_proba_csr(self._h, ip.ptr, ix.ptr, vv.ptr, m, _data_ptr(out), ct.byref(o)))
+        return out
+
     def decision_function(self, Xt, out=None, **opts):
         """m x P FP64 decision values (Eq 11, b included), pair order p = s*k - s(s+1)/2 + t-s-1."""
         a = _Arg(Xt, np.float32, "Xtest", 2)
@@ -294,6 +310,27 @@ def train(X, y, k, C, gamma, eps, **opts) -> Model:
     h = ct.c_void_p()
     rc = _check(lib().gmpsvm_train_ex(a.ptr, b.ptr, n, d, int(k), float(C), float(gamma), float(eps), ct.byref(o),
                                       ct.byref(h)))
+    return Model(h.value, rc)
+
+
+def _csr_args(csr):
+    if isinstance(csr, tuple):
+        ip, ix, vv, shape = csr
+    else:  # scipy.sparse
+        c = csr.tocsr()
+        ip, ix, vv, shape = c.indptr.astype(np.int64), c.indices.astype(np.int32), c.data.astype(np.float32), c.shape
+    return (_Arg(ip, np.int64, "indptr", 1), _Arg(ix, np.int32, "indices", 1), _Arg(vv, np.float32, "values", 1),
+            (int(shape[0]), int(shape[1])))
+
+
+def train_csr(csr, y, k, C, gamma, eps, **opts) -> Model:
+    """gmpsvm_train_csr: CSR rows (the paper's sparse format) densified on the device, then train."""
+    ip, ix, vv, (n, d) = _csr_args(csr)
+    b = _Arg(y, np.int32, "y", 1)
+    o, keep = _options([ip, ix, vv, b], **opts)
+    h = ct.c_void_p()
+    rc = _check(lib().gmpsvm_train_csr(ip.ptr, ix.ptr, vv.ptr, b.ptr, n, d, int(k), float(C), float(gamma), float(eps),
+                                       ct.byref(o), ct.byref(h)))
     return Model(h.value, rc)
 
 

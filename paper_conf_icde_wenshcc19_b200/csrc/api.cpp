@@ -273,6 +273,29 @@ int gmpsvm_predict_proba_ex(const gmpsvm_model* model, const float* Xtest, int64
   });
 }
 
+int gmpsvm_train_csr(const int64_t* indptr, const int32_t* indices, const float* values, const int32_t* y, int64_t n,
+                     int32_t d, int32_t k, double C, double gamma, double eps, const gmpsvm_options* opt,
+                     gmpsvm_model** out) {
+  return guarded([&]() {
+    if (!out) throw Error(GMPSVM_EINVAL, "out is NULL");
+    *out = nullptr;
+    Model* m = nullptr;
+    const int rc = gmpsvm::engine_train_csr(indptr, indices, values, y, n, d, k, C, gamma, eps, resolve(opt), &m);
+    auto* h = new gmpsvm_model();
+    h->m.reset(m);
+    *out = h;
+    return rc;
+  });
+}
+
+int gmpsvm_predict_proba_csr(const gmpsvm_model* model, const int64_t* indptr, const int32_t* indices,
+                             const float* values, int64_t m, double* out, const gmpsvm_options* opt) {
+  return guarded([&]() {
+    if (!model) throw Error(GMPSVM_EINVAL, "model is NULL");
+    return gmpsvm::engine_predict_csr(*model->m, indptr, indices, values, m, out, resolve(opt));
+  });
+}
+
 int gmpsvm_predict_proba(const gmpsvm_model* model, const float* Xtest, int64_t m, double* out) {
   return gmpsvm_predict_proba_ex(model, Xtest, m, out, nullptr);
 }

@@ -1627,6 +1627,81 @@ int engine_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t
 }
 
 // ------------------------------------------------------------------------------------------
+// CSR input (NEXT-3, the format of the paper's datasets): densified on the device, then the dense
+// path (the kernel-value contraction runs on the dense rows).  indptr [n+1] int64, indices [nnz]
+// int32, values [nnz] float; host or device pointers per opt.inputs_on_device.
+struct CsrDense {
+  DevBuf<float> X;
+  CsrDense(const int64_t* indptr, const int32_t* indices, const float* values, int64_t n, int32_t d,
+           const gmpsvm_options& opt, cudaStream_t st)
+      : X((size_t)std::max<int64_t>(n, 1) * d, st) {
+    if (n < 0 || d < 1 || !indptr) throw Error(GMPSVM_EINVAL, "bad CSR arguments");
+    int64_t nnz = 0;
+    if (opt.inputs_on_device) GM_CUDA(cudaMemcpy(&nnz, indptr + n, 8, cudaMemcpyDeviceToHost));
+    else nnz = indptr[n];
+    if (nnz < 0 || (nnz > 0 && (!indices || !values))) throw Error(GMPSVM_EINVAL, "bad CSR arguments");
+    DevBuf<int64_t> ip(opt.inputs_on_device ? 0 : (size_t)n + 1, st);
+    DevBuf<int32_t> ix(opt.inputs_on_device ? 0 : (size_t)nnz, st);
+    DevBuf<float> vv(opt.inputs_on_device ? 0 : (size_t)nnz, st);
+    const int64_t* dip = indptr;
+    const int32_t* dix = indices;
+    const float* dvv = values;
+    if (!opt.inputs_on_device) {
+      GM_CUDA(cudaMemcpyAsync(ip.get(), indptr, ((size_t)n + 1) * 8, cudaMemcpyHostToDevice, st));
+      if (nnz) {
+        GM_CUDA(cudaMemcpyAsync(ix.get(), indices, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
+        GM_CUDA(cudaMemcpyAsync(vv.get(), values, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
+      }
+      dip = ip.get();
+      dix = ix.get();
+      dvv = vv.get();
+    }
+    DevBuf<int32_t> bad(1, st);
+    GM_CUDA(cudaMemsetAsync(bad.get(), 0, 4, st));
+    launch_csr_densify(dip, dix, dvv, n, d, X.get(), bad.get(), st);
+    int32_t hb = 0;
+    GM_CUDA(cudaMemcpyAsync(&hb, bad.get(), 4, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaStreamSynchronize(st));
+    if (hb) throw Error(GMPSVM_EINVAL, "CSR column index outside [0, d)");
+  }
+};
+
+int engine_train_csr(const int64_t* indptr, const int32_t* indices, const float* values, const int32_t* y, int64_t n,
+                     int32_t d, int32_t k, double C, double gamma, double eps, const gmpsvm_options& opt, Model** out) {
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  CsrDense cd(indptr, indices, values, n, d, opt, st);
+  gmpsvm_options o2 = opt;
+  DevBuf<int32_t> yb(opt.inputs_on_device ? 0 : (size_t)n, st);
+  const int32_t* dy = y;
+  if (!opt.inputs_on_device) {
+    if (!y) throw Error(GMPSVM_EINVAL, "null argument");
+    GM_CUDA(cudaMemcpyAsync(yb.get(), y, (size_t)n * 4, cudaMemcpyHostToDevice, st));
+    dy = yb.get();
+  }
+  o2.inputs_on_device = 1;
+  o2.stream = st;
+  return engine_train(cd.X.get(), dy, n, d, k, C, gamma, eps, o2, out);
+}
+
+int engine_predict_csr(const Model& mdl, const int64_t* indptr, const int32_t* indices, const float* values, int64_t m,
+                       double* prob_out, const gmpsvm_options& opt) {
+  if (m == 0) return GMPSVM_OK;
+  DeviceGuard dg(opt.device);
+  cudaStream_t st = get_stream(opt);
+  CsrDense cd(indptr, indices, values, m, mdl.d, opt, st);
+  gmpsvm_options o2 = opt;
+  o2.stream = st;
+  if (opt.inputs_on_device) return engine_predict(mdl, cd.X.get(), m, prob_out, nullptr, o2);
+  DevBuf<double> pb((size_t)m * mdl.k, st);
+  o2.inputs_on_device = 1;
+  const int rc = engine_predict(mdl, cd.X.get(), m, pb.get(), nullptr, o2);
+  GM_CUDA(cudaMemcpyAsync(prob_out, pb.get(), (size_t)m * mdl.k * 8, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaStreamSynchronize(st));
+  return rc;
+}
+
+// ------------------------------------------------------------------------------------------
 static void ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
   std::lock_guard<std::mutex> lk(mdl.mu);
   if (mdl.dev && mdl.dev->device == device) return;

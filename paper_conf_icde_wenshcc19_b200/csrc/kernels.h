@@ -47,6 +47,8 @@ struct KrowKernel {
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
 bool krow_tc_2cta();
+void launch_csr_densify(const int64_t* indptr, const int32_t* indices, const float* values, int64_t n, int d, float* X,
+                        int32_t* bad, cudaStream_t st);
 void launch_scatter_oof(const double* dec, int64_t m, int P, const int32_t* cls, const int64_t* rnk,
                         const PairDesc* pairs, double* v, cudaStream_t st);
 void launch_sigmoid_fit_on(const PairDesc* pairs, int P, const double* v, double* A, double* B, int32_t* status,

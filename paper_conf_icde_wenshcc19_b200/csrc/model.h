@@ -86,6 +86,10 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
 int engine_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
                             const double* alpha, const double* b, const double* A, const double* B,
                             const int32_t* status, const gmpsvm_options& opt, Model** out);
+int engine_train_csr(const int64_t* indptr, const int32_t* indices, const float* values, const int32_t* y, int64_t n,
+                     int32_t d, int32_t k, double C, double gamma, double eps, const gmpsvm_options& opt, Model** out);
+int engine_predict_csr(const Model& mdl, const int64_t* indptr, const int32_t* indices, const float* values, int64_t m,
+                       double* prob_out, const gmpsvm_options& opt);
 int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
                    const gmpsvm_options& opt);
 int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int32_t d, double gamma, float* K_out,

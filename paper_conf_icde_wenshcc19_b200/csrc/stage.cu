@@ -227,4 +227,31 @@ void launch_build_coef(const double* alpha, const int64_t* aoff, const int64_t* 
             nsv_pad, km1_pad, coef, coef64);
 }
 
+// CSR input (the paper's / LibSVM's sparse format, NEXT-3): row i's nonzeros
+// values[indptr[i] .. indptr[i+1]) at columns indices[.] scattered into a zeroed dense row-major
+// n x d matrix; one warp per row.  Out-of-range columns set *bad.
+__global__ void csr_densify_kernel(const int64_t* __restrict__ indptr, const int32_t* __restrict__ indices,
+                                   const float* __restrict__ values, int64_t n, int d, float* __restrict__ X,
+                                   int32_t* __restrict__ bad) {
+  const int64_t row = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= n) return;
+  const int64_t b = indptr[row], e = indptr[row + 1];
+  for (int64_t j = b + lane; j < e; j += 32) {
+    const int32_t c = indices[j];
+    if (c < 0 || c >= d) {
+      *bad = 1;
+      continue;
+    }
+    X[row * d + c] = values[j];
+  }
+}
+
+void launch_csr_densify(const int64_t* indptr, const int32_t* indices, const float* values, int64_t n, int d, float* X,
+                        int32_t* bad, cudaStream_t st) {
+  GM_CUDA(cudaMemsetAsync(X, 0, (size_t)n * d * sizeof(float), st));
+  if (n > 0)
+    GM_LAUNCH(csr_densify_kernel, dim3((unsigned)ceil_div(n, 8)), dim3(256), 0, st, indptr, indices, values, n, d, X, bad);
+}
+
 }  // namespace gmpsvm

@@ -210,3 +210,32 @@ def test_sv_index_matches_alpha(gm):
         a = m.pair(s, t, int((y == s).sum()), int((y == t).sum()))["alpha"]
         expect |= set(idx[a > 0].tolist())
     assert sv == expect
+
+
+def test_csr_input_matches_dense_bitwise(gm):
+    """CSR rows (NEXT-3: the paper's sparse format; MNIST-shaped data is ~68 % zeros) are densified
+    on the device and take the dense path: the same model and probabilities, bitwise, from host
+    scipy CSR and from CUDA tensors; a column index outside [0, d) is rejected."""
+    sp = pytest.importorskip("scipy.sparse")
+    spec, X, y, Xt, yt = datagen.make_config("mnist", n_train=1500, n_test=150)
+    dense = gm.train(X, y, spec.k, spec.C, spec.gamma, 1e-3)
+    p_dense = dense.predict_proba(Xt)
+    A, At = sp.csr_matrix(X), sp.csr_matrix(Xt)
+    assert A.nnz < 0.5 * X.size
+    m = gm.train_csr(A, y, spec.k, spec.C, spec.gamma, 1e-3)
+    np.testing.assert_array_equal(m.sv_index(), dense.sv_index())
+    np.testing.assert_array_equal(m.predict_proba_csr(At), p_dense)
+    np.testing.assert_array_equal(m.predict_proba(Xt), p_dense)
+    dev = torch.device("cuda:0")
+    tup = (torch.from_numpy(A.indptr.astype(np.int64)).to(dev), torch.from_numpy(A.indices.astype(np.int32)).to(dev),
+           torch.from_numpy(A.data.astype(np.float32)).to(dev), A.shape)
+    md = gm.train_csr(tup, torch.from_numpy(y).to(dev), spec.k, spec.C, spec.gamma, 1e-3)
+    tupt = (torch.from_numpy(At.indptr.astype(np.int64)).to(dev), torch.from_numpy(At.indices.astype(np.int32)).to(dev),
+            torch.from_numpy(At.data.astype(np.float32)).to(dev), At.shape)
+    np.testing.assert_array_equal(md.predict_proba_csr(tupt).cpu().numpy(), p_dense)
+    bad = A.copy()
+    bad.indices = bad.indices.copy()
+    bad.indices[0] = spec.d + 5
+    with pytest.raises(gm.GmpsvmError):
+        gm.train_csr((bad.indptr.astype(np.int64), bad.indices.astype(np.int32), bad.data.astype(np.float32), bad.shape),
+                     y, spec.k, spec.C, spec.gamma, 1e-3)
