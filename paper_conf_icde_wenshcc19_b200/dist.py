@@ -153,7 +153,7 @@ def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
     counts = np.bincount(yy, minlength=k)
     mine = plan_pairs(counts, world)[rank]
     part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts)
-    dev_opts = {key: opts[key] for key in ("device", "stream") if key in opts}
+    dev_opts = {key: opts[key] for key in ("device", "stream", "kernel", "coef0", "degree") if key in opts}
     model = gather_solutions(part, X, y, k, C, gamma, group, **dev_opts)
     model.part_stats = part.train_stats()  # this rank's training (the rebuilt model has no solver stats)
     m = Xt.shape[0]
