@@ -196,6 +196,11 @@ def test_model_from_alpha_and_sharded_gather_bitwise(gm):
     try:
         model, prob = gdist.train_predict(X, y, Xt, spec.k, spec.C, spec.gamma, 1e-3, ws_size=128)
         np.testing.assert_array_equal(np.asarray(prob), full.predict_proba(Xt))
+        # the rebuilt model keeps a non-Gaussian kernel (L76-L78)
+        kw = dict(ws_size=128, kernel="poly", coef0=1.0, degree=2)
+        fp = gm.train(X, y, spec.k, 1.0, 0.3, 1e-3, **kw)
+        _, pp = gdist.train_predict(X, y, Xt, spec.k, 1.0, 0.3, 1e-3, **kw)
+        np.testing.assert_array_equal(np.asarray(pp), fp.predict_proba(Xt))
     finally:
         dist.destroy_process_group()
 
