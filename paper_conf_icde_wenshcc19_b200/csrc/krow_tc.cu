@@ -977,20 +977,23 @@ __global__ void split_tf32_kernel(const float* __restrict__ X, int64_t n, int d,
   if (lane == 0) norms[j] = (float)s;
 }
 
-// max over the rows of |x - mu| (non-negative floats order as their bit patterns: atomicMax)
+// max over the rows of |x - mu| (non-negative floats order as their bit patterns: atomicMax);
+// one warp per row (grid-stride), lanes over the columns: no per-element index division
 __global__ void maxabs_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
                               const float* __restrict__ mu, unsigned* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w0 = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
   float m = 0.f;
-  const int64_t total = n * d;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t j = e / d;
-    const int c = (int)(e - j * d);
+  for (int64_t j = w0; j < n; j += nw) {
     const int64_t src = perm ? perm[j] : j;
-    if (src >= 0) m = fmaxf(m, fabsf(X[src * d + c] - mu[c]));
+    if (src < 0) continue;
+    const float* row = X + src * d;
+    for (int c = lane; c < d; c += 32) m = fmaxf(m, fabsf(row[c] - mu[c]));
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-  if ((threadIdx.x & 31) == 0) atomicMax(out, __float_as_uint(m));
+  if (lane == 0) atomicMax(out, __float_as_uint(m));
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -1052,7 +1055,7 @@ float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const
   unsigned* dm = nullptr;
   GM_CUDA(cudaMallocAsync(&dm, sizeof(unsigned), st));
   GM_CUDA(cudaMemsetAsync(dm, 0, sizeof(unsigned), st));
-  GM_LAUNCH(maxabs_kernel, dim3(592), dim3(256), 0, st, X, n, d, perm, mu, dm);
+  GM_LAUNCH(maxabs_kernel, dim3(1184), dim3(256), 0, st, X, n, d, perm, mu, dm);
   unsigned h = 0;
   GM_CUDA(cudaMemcpyAsync(&h, dm, sizeof(unsigned), cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaFreeAsync(dm, st));
