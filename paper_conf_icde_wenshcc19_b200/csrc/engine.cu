@@ -1090,8 +1090,8 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   DevBuf<int64_t> d_phase(smo_prof ? (size_t)Pl * 5 : 0, st);
   if (smo_prof) GM_CUDA(cudaMemsetAsync(d_phase.get(), 0, (size_t)Pl * 5 * 8, st));
   a.smo_phase = smo_prof ? d_phase.get() : nullptr;
-  DevBuf<int64_t> d_sphase(smo_prof ? (size_t)(Pl + 4096) * 5 : 0, st);
-  if (smo_prof) GM_CUDA(cudaMemsetAsync(d_sphase.get(), 0, (size_t)(Pl + 4096) * 5 * 8, st));
+  DevBuf<int64_t> d_sphase(smo_prof ? (size_t)(Pl + 8192) * 5 : 0, st);
+  if (smo_prof) GM_CUDA(cudaMemsetAsync(d_sphase.get(), 0, (size_t)(Pl + 8192) * 5 * 8, st));
   a.sel_phase = smo_prof ? d_sphase.get() : nullptr;
   // GMPSVM_TRACE=<pair position>: kernel timeline of that pair (entries sorted largest pair first)
   static const int trace_pos = getenv("GMPSVM_TRACE") ? atoi(getenv("GMPSVM_TRACE")) : -1;
@@ -1442,6 +1442,12 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
       for (int q = 0; q < 5; ++q) fs[q] += (double)fq[i * 5 + q];
     fprintf(stderr, "[gmpsvm] fast select cycles/launch: staging %.0f  thresholds %.0f  compact %.0f  ranks %.0f  write-out %.0f (fallbacks x1e6)\n",
             fs[0] / outer, fs[1] / outer, fs[2] / outer, fs[3] / outer, fs[4] / outer);
+    GM_CUDA(cudaMemcpy(fq.data(), d_sphase.get() + (size_t)8192 * 5, fq.size() * 8, cudaMemcpyDeviceToHost));
+    double wo[5] = {0, 0, 0, 0, 0};
+    for (int i = 0; i < Pl; ++i)
+      for (int q = 0; q < 5; ++q) wo[q] += (double)fq[i * 5 + q];
+    fprintf(stderr, "[gmpsvm] select write-out cycles/launch: bitmap %.0f  prefix %.0f  stores %.0f\n", wo[0] / outer,
+            wo[1] / outer, wo[2] / outer);
     std::string per;
     for (int i = 0; i < Pl; ++i)
       per += " (" + std::to_string(hp[i].s) + "," + std::to_string(hp[i].t) + "):" + std::to_string(h_outer[i]) + "/" +

@@ -157,13 +157,23 @@ __device__ void bitmap_prefix(const uint32_t* bm, int nwords, int32_t* wpre, int
 __device__ void ws_write_out(const SolverArgs& a, int lp, const int32_t* pick, int cnt, uint32_t* bm, int32_t* wpre,
                              int* sm) {
   const int t = threadIdx.x;
+  long long tq = clock64();
+  auto mark = [&](int k) {  // GMPSVM_SMO_PHASES: write-out sub-phase cycles (thread 0)
+    if (a.sel_phase && t == 0) {
+      const long long tc = clock64();
+      a.sel_phase[(int64_t)(lp + 8192) * 5 + k] += tc - tq;
+      tq = tc;
+    }
+  };
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t, B = a.B, nwords = (np + 31) / 32;
   for (int w = t; w < nwords; w += blockDim.x) bm[w] = 0u;
   __syncthreads();
   for (int e = t; e < cnt; e += blockDim.x) atomicOr(&bm[pick[e] >> 5], 1u << (pick[e] & 31));
   __syncthreads();
+  mark(0);
   bitmap_prefix(bm, nwords, wpre, sm);
+  mark(1);
   float* buf = a.Kws + (int64_t)lp * ws_buf_floats(B);
   double* st_al = reinterpret_cast<double*>(buf + ws_state_off(B));
   double* st_f = st_al + B;
@@ -177,6 +187,7 @@ __device__ void ws_write_out(const SolverArgs& a, int lp, const int32_t* pick, i
     st_f[rank] = a.f[pd.a_off + x];
     st_ix[rank] = x;
   }
+  mark(2);
   if (t == 0) a.ws_n[lp] = cnt;
 }
 
