@@ -17,6 +17,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import shutil
 import subprocess
 import sys
 import threading
@@ -74,17 +75,37 @@ class ClockSampler:
             pass
 
     def _run(self):
-        while not self._stop.is_set():
-            self.sample()
-            self._stop.wait(0.2)
+        # one long-running nvidia-smi (the recipe's `-lms 200` loop): NVML is initialised once, so
+        # the sampling does not stall the host's CUDA calls the way a fresh process every 0.2 s did
+        try:
+            lb = ["stdbuf", "-oL"] if shutil.which("stdbuf") else []  # a line per sample through the pipe
+            self._proc = subprocess.Popen([*lb, "nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                           "--format=csv,noheader,nounits", "-lms", "200"],
+                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self._proc = None
+            return
+        for line in self._proc.stdout:
+            f = [x.strip() for x in line.strip().split(",")]
+            if len(f) >= 7:
+                self.samples.append(f)
+            if self._stop.is_set():
+                break
 
     def __enter__(self):
+        self._proc = None
         self._th = threading.Thread(target=self._run, daemon=True)
         self._th.start()
         return self
 
     def __exit__(self, *a):
         self._stop.set()
+        if self._proc is not None:
+            self._proc.terminate()
+            try:
+                self._proc.wait(timeout=5)
+            except Exception:
+                self._proc.kill()
         if self._th:
             self._th.join(timeout=10)
 

@@ -194,10 +194,7 @@ __device__ void ws_write_out(const SolverArgs& a, int lp, const int32_t* pick, i
 // ------------------------------------------------------------------------------------------
 // a4 selection
 __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t max_outer) {
-  pdl_enter();
   const int lp = blockIdx.x + a.pair_base;
-  TraceScope ts_(a, lp, 0);
-  if (a.status[lp] != 0) return;
   extern __shared__ __align__(16) unsigned char sdyn[];
   uint64_t* keys = reinterpret_cast<uint64_t*>(sdyn);
   uint8_t* flags = sdyn + (size_t)kWMaxNp * 8;
@@ -208,7 +205,10 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
   const double C = a.C;
   const double* al = a.alpha + pd.a_off;
   const double* fl = a.f + pd.a_off;
-  const int first = a.outer_iters[lp] == 0;
+  // Before the dependency wait: the retained rows come from the previous selection's output
+  // (ws_tmp, ws_n, outer_iters), which completed before this launch's predecessor (the f-update)
+  // was released, so building their bitmap overlaps the f-update's tail.  L2 loads (.cg).
+  const int first = __ldcg(a.outer_iters + lp) == 0;
   int32_t* ws_age = a.ws_tmp + (int64_t)lp * B;  // age order (oldest first)
   long long tq = clock64();
   auto mark = [&](int k) {  // GMPSVM_SMO_PHASES: selection sub-phase cycles (thread 0)
@@ -219,16 +219,20 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
     }
   };
   // retained rows: the newest B - q of the previous working set (reading R19)
-  const int prev_n = first ? 0 : a.ws_n[lp];
+  const int prev_n = first ? 0 : __ldcg(a.ws_n + lp);
   const int keep = np <= B ? 0 : min(prev_n, B - a.q);
   for (int w = t; w < (np + 31) / 32; w += kWT) W.retained[w] = 0u;
   if (t == 0) W.overflow = 0;
   __syncthreads();
   for (int e = t; e < keep; e += kWT) {
-    const int idx = ws_age[prev_n - keep + e];
+    const int idx = __ldcg(ws_age + prev_n - keep + e);
     W.pick[e] = idx;
     atomicOr(&W.retained[idx >> 5], 1u << (idx & 31));
   }
+  pdl_enter();  // alpha (local SMO), f (f-update) and status are read after the wait
+  TraceScope ts_(a, lp, 0);
+  if (a.status[lp] != 0) return;
+  tq = clock64();
   __syncthreads();
   // stage keys / flags, stop test (Eq 9-10), per-thread minima of the candidates of both sides
   double fmin = DBL_MAX, fmax = -DBL_MAX;
@@ -475,10 +479,10 @@ constexpr int kGR = 8;  // tile rows per CTA
 
 __global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
+  const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
   pdl_enter();
   TraceScope ts_(a, lp, 1);
   if (a.status[lp] != 0) return;
-  const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t;
   if (np <= a.B && a.outer_iters[lp] != 1) return;  // working set (and tile) unchanged
   const int wn = a.ws_n[lp];
@@ -562,12 +566,12 @@ __device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
 template <int E>
 __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
+  const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
   pdl_wait();  // the f-update is released when the local solve ends (below)
   TraceScope ts_(a, lp, 2);
   if (a.status[lp] != 0) return;
   extern __shared__ __align__(16) unsigned char mdyn[];
   const int lane = threadIdx.x;
-  const PairDesc pd = a.pairs[lp];
   const int B = a.B, wn = a.ws_n[lp], ld = ws_tile_ld(B);
   uint32_t kws;  // K_ws,ws tile, row stride ld (opaque: keeps the shared window base out of the loop)
   asm volatile("mov.u32 %0, %1;" : "=r"(kws) : "r"(smem_addr(mdyn)));
@@ -803,8 +807,9 @@ struct WFup {
 };
 
 __global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraphConditionalHandle h, int set_cond) {
-  pdl_enter();
   const int lp = blockIdx.x + a.pair_base;
+  const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
+  pdl_enter();
   TraceScope ts_(a, lp, 3);
   const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
   if (blockIdx.x == 0 && blockIdx.y == 0 && t == 0) {
@@ -817,7 +822,6 @@ __global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraph
   }
   if (a.status[lp] != 0) return;
   __shared__ WFup F;
-  const PairDesc pd = a.pairs[lp];
   const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;
   const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;
   const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
