@@ -54,7 +54,9 @@ def _peaks():
 class ClockSampler:
     """nvidia-smi clocks / throttle reasons sampled during the timed region (B200_PROFILING.md)."""
 
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+    # no power.draw: reading it holds the driver long enough to stall a concurrent step's host
+    # calls (30 ms outlier steps were seen with it in the query)
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
 
@@ -69,7 +71,7 @@ class ClockSampler:
             out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
                                   "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
             f = [x.strip() for x in out.stdout.strip().split(",")]
-            if len(f) >= 7:
+            if len(f) >= 6:
                 self.samples.append(f)
         except Exception:
             pass
@@ -87,7 +89,7 @@ class ClockSampler:
             return
         for line in self._proc.stdout:
             f = [x.strip() for x in line.strip().split(",")]
-            if len(f) >= 7:
+            if len(f) >= 6:
                 self.samples.append(f)
             if self._stop.is_set():
                 break
@@ -115,7 +117,7 @@ class ClockSampler:
         sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
         mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[3 + i].lower() == "active"})
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[2 + i].lower() == "active"})
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
                 "reasons": reasons, "samples": len(self.samples)}
 
@@ -219,11 +221,12 @@ def run_gpu(args, spec):
     # the clock sampler (an nvidia-smi process every 0.2 s) starts during the warm-up, so its
     # start-up cost does not land in the first timed step
     clk = ClockSampler(gpu).__enter__()
+    t_wait = time.time()  # first sample before the warm-up: the GPU must not idle between warm-up and timing
+    while not clk.samples and clk._th.is_alive() and time.time() - t_wait < 10:
+        time.sleep(0.05)
     for _ in range(args.warmup):
         model, prob = step(Xd, yd, Xtd)
     torch.cuda.synchronize(dev)
-    while not clk.samples and clk._th.is_alive():
-        time.sleep(0.05)
     n_warm = len(clk.samples)
 
     # ---- device-resident timed region
