@@ -25,6 +25,8 @@
 #include <cstdlib>
 #include <string>
 
+#include <math_constants.h>
+
 #include "kernels.h"
 #include "solver_dev.cuh"
 
@@ -556,6 +558,24 @@ __device__ __forceinline__ void tree_max_u32(uint32_t (&k)[E], int (&q)[E]) {
       }
 }
 template <int E>
+__device__ __forceinline__ void tree_min_f64(double (&k)[E], int (&q)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w)
+      if (k[i + w] < k[i]) {
+        k[i] = k[i + w];
+        q[i] = q[i + w];
+      }
+}
+template <int E>
+__device__ __forceinline__ void tree_max_f64(double (&k)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w) k[i] = k[i + w] > k[i] ? k[i + w] : k[i];
+}
+template <int E>
 __device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
 #pragma unroll
   for (int w = 1; w < E; w <<= 1)
@@ -657,16 +677,19 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   };
   for (;;) {
     // Eq 4: u = argmin_{I_u} f; ties -> lowest position (== lowest pair-local index, R5)
-    uint64_t uk[E];
+    // the lane's minimum in FP64 compares (ties: lower row), one ord_key for the warp reduction
+    double uv[E];
     int uq[E];
 #pragma unroll
     for (int q = 0; q < E; ++q) {
-      uk[q] = ((umask >> q) & 1u) ? ord_key(f[q]) : ~0ull;
+      uv[q] = ((umask >> q) & 1u) ? f[q] : CUDART_INF;
       uq[q] = q;
     }
-    tree_min_u64<E>(uk, uq);
-    const uint32_t h = (uint32_t)(uk[0] >> 32), l = (uint32_t)uk[0];
-    const uint32_t pos = uk[0] == ~0ull ? 0xffffffffu : (uint32_t)(lane + 32 * uq[0]);
+    tree_min_f64<E>(uv, uq);
+    const bool uempty = uv[0] == CUDART_INF;  // f is finite: +inf marks "no I_u row in this lane"
+    const uint64_t uk0 = uempty ? ~0ull : ord_key(uv[0]);
+    const uint32_t h = (uint32_t)(uk0 >> 32), l = (uint32_t)uk0;
+    const uint32_t pos = uempty ? 0xffffffffu : (uint32_t)(lane + 32 * uq[0]);
     const uint32_t m0 = __reduce_min_sync(FULLMASK, h);
     const uint32_t m1 = __reduce_min_sync(FULLMASK, h == m0 ? l : 0xffffffffu);
     const uint32_t ue32 = __reduce_min_sync(FULLMASK, (h == m0 && l == m1) ? pos : 0xffffffffu);
@@ -687,7 +710,7 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
     uint32_t sb[E];
     int sq[E];
     float st[E];
-    uint64_t lk[E];
+    double lv[E];
 #pragma unroll
     for (int q = 0; q < E; ++q) {
       const bool il = (lmask >> q) & 1u;
@@ -698,12 +721,13 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
       st[q] = df * r;
       sb[q] = (il && f[q] > fu) ? __float_as_uint(df * st[q]) : 0u;  // scores >= 0: bits order as values
       sq[q] = q;
-      lk[q] = il ? ord_key(f[q]) : 0ull;
+      lv[q] = il ? f[q] : -CUDART_INF;
     }
     tree_max_u32<E>(sb, sq);
-    tree_max_u64<E>(lk);
-    const uint32_t xh = __reduce_max_sync(FULLMASK, (uint32_t)(lk[0] >> 32));
-    const uint32_t xl = __reduce_max_sync(FULLMASK, (uint32_t)(lk[0] >> 32) == xh ? (uint32_t)lk[0] : 0u);
+    tree_max_f64<E>(lv);
+    const uint64_t lk0 = lv[0] == -CUDART_INF ? 0ull : ord_key(lv[0]);  // 0: no I_l row in this lane
+    const uint32_t xh = __reduce_max_sync(FULLMASK, (uint32_t)(lk0 >> 32));
+    const uint32_t xl = __reduce_max_sync(FULLMASK, (uint32_t)(lk0 >> 32) == xh ? (uint32_t)lk0 : 0u);
     const uint32_t smax = __reduce_max_sync(FULLMASK, sb[0]);
     const uint32_t lpos = (sb[0] != 0u && sb[0] == smax) ? (uint32_t)(lane + 32 * sq[0]) : 0xffffffffu;
     const uint32_t le32 = __reduce_min_sync(FULLMASK, lpos);
