@@ -583,7 +583,7 @@ __device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
     for (int i = 0; i + w < E; i += 2 * w) k[i] = k[i + w] > k[i] ? k[i + w] : k[i];
 }
 
-template <int E>
+template <int E, bool PROF>  // PROF: GMPSVM_SMO_PHASES per-phase cycle counters (compiled out otherwise)
 __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   const int lp = blockIdx.x + a.pair_base;
   const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
@@ -666,7 +666,7 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   int it = 0;
   double delta0 = 0.0;
   const long long t_begin = clock64();
-  const bool prof = a.smo_phase != nullptr;  // GMPSVM_SMO_PHASES: per-phase SM cycles
+  constexpr bool prof = PROF;  // GMPSVM_SMO_PHASES: per-phase SM cycles (a.smo_phase != NULL)
   long long ph[4] = {0, 0, 0, 0}, tp = t_begin;
   auto markp = [&](int k) {
     if (prof) {
@@ -950,18 +950,29 @@ static void launch_pdl(void (*kern)(KArgs...), dim3 g, dim3 b, size_t smem, cuda
   g_launches.fetch_add(1, std::memory_order_relaxed);
 }
 
+template <int E>
+static void smo_configure(int smem) {
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<E, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<E, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+}
+template <int E>
+static void launch_smo(const SolverArgs& a, int P, size_t smem, cudaStream_t st) {
+  if (a.smo_phase) launch_pdl(ws_smo_kernel<E, true>, dim3(P), dim3(32), smem, st, a);
+  else launch_pdl(ws_smo_kernel<E, false>, dim3(P), dim3(32), smem, st, a);
+}
+
 static void ws_configure() {
   static bool configured = false;
   if (configured) return;
   GM_CUDA(cudaFuncSetAttribute(ws_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)((size_t)kWMaxNp * 9)));
   const int mx = (int)ws_smo_smem(kWMaxB);
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<5>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+  smo_configure<1>(mx);
+  smo_configure<2>(mx);
+  smo_configure<3>(mx);
+  smo_configure<4>(mx);
+  smo_configure<5>(mx);
+  smo_configure<6>(mx);
+  smo_configure<7>(mx);
   configured = true;
 }
 
@@ -973,13 +984,13 @@ void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphCo
   else GM_LAUNCH(ws_select_kernel, dim3(P), dim3(kWT), sel_dyn, st, a, max_outer);
   launch_pdl(ws_gather_kernel, dim3(P, (unsigned)ceil_div(a.B, kGR)), dim3(256), 0, st, a);
   switch ((a.B + 31) / 32) {
-    case 1: launch_pdl(ws_smo_kernel<1>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 2: launch_pdl(ws_smo_kernel<2>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 3: launch_pdl(ws_smo_kernel<3>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 4: launch_pdl(ws_smo_kernel<4>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 5: launch_pdl(ws_smo_kernel<5>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    case 6: launch_pdl(ws_smo_kernel<6>, dim3(P), dim3(32), smo_dyn, st, a); break;
-    default: launch_pdl(ws_smo_kernel<7>, dim3(P), dim3(32), smo_dyn, st, a); break;
+    case 1: launch_smo<1>(a, P, smo_dyn, st); break;
+    case 2: launch_smo<2>(a, P, smo_dyn, st); break;
+    case 3: launch_smo<3>(a, P, smo_dyn, st); break;
+    case 4: launch_smo<4>(a, P, smo_dyn, st); break;
+    case 5: launch_smo<5>(a, P, smo_dyn, st); break;
+    case 6: launch_smo<6>(a, P, smo_dyn, st); break;
+    default: launch_smo<7>(a, P, smo_dyn, st); break;
   }
   launch_pdl(ws_fupdate_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, 128)), dim3(kFT), 0, st, a, h, set_cond);
 }
