@@ -15,6 +15,7 @@ so higher_is_better = false.
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import os
 import shutil
@@ -224,6 +225,8 @@ def run_gpu(args, spec):
     t_wait = time.time()  # first sample before the warm-up: the GPU must not idle between warm-up and timing
     while not clk.samples and clk._th.is_alive() and time.time() - t_wait < 10:
         time.sleep(0.05)
+    gc.collect()
+    gc.disable()  # no Python collector pauses from here through the e2e timed region
     for _ in range(args.warmup):
         model, prob = step(Xd, yd, Xtd)
     torch.cuda.synchronize(dev)
@@ -277,6 +280,7 @@ def run_gpu(args, spec):
         model_h, prob_h = step(Xh, yh, Xth, host=True)
     torch.cuda.synchronize(dev)
     e2e_ms = (time.perf_counter() - t0) * 1e3 / args.steps
+    gc.enable()
     e2e_train = model_h.train_stats() if ws == 1 else getattr(model_h, "part_stats", {})
     e2e_pred = gm.last_predict_stats()
     if ws > 1:
