@@ -72,7 +72,7 @@ typedef struct {
                                row buffers exceed 85% of device memory                       */
   void* stream;             /* cudaStream_t to run on (NULL = a library-owned stream)       */
   const int32_t* pair_ids;  /* train only these pair indices (multi-GPU sharding); NULL = all */
-  int32_t n_pair_ids;
+  int32_t n_pair_ids;       /* >= 1 when pair_ids != NULL (else GMPSVM_EINVAL)               */
   int32_t inputs_on_device; /* 1: X/y/Xtest/out are device pointers on `device`             */
   int64_t max_outer_iter;   /* cap on outer (working-set) iterations per pair; 0 = 1,000,000 */
   int32_t inner_iter_cap;   /* cap on inner SMO steps per working set; 0 = 100 * B          */

@@ -2,6 +2,8 @@
 // Converts engine exceptions into status codes + a thread-local message; implements the
 // model introspection and the serialize / deserialize / merge plumbing used by the
 // multi-GPU driver (pairs sharded across ranks, blobs gathered with NCCL).
+#include <dlfcn.h>
+
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
@@ -17,9 +19,30 @@ namespace {
 
 // The solver runs every pair's outer loop as its own branch of one CUDA graph; the runtime
 // executes at most CUDA_DEVICE_MAX_CONNECTIONS (default 8, max 32) branches concurrently.
-// Raise the default to 32 when the library is loaded, before the process creates its CUDA
-// context (an explicit user setting is kept; engine.cu packs the pairs into that many branches).
-__attribute__((constructor)) void gmpsvm_default_connections() { setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0); }
+// Raise the default to 32 when the library is loaded (an explicit user setting is kept).  The
+// variable is read when a CUDA context is created: if the process already has one (e.g. torch
+// initialised CUDA before the library was loaded), the setting cannot take effect, so the
+// number of connections actually in effect is recorded here and engine.cu packs the pairs into
+// that many branches.  libcuda is only probed if it is already loaded (RTLD_NOLOAD).
+int g_conn_effective = 8;
+__attribute__((constructor)) void gmpsvm_default_connections() {
+  const char* prev = getenv("CUDA_DEVICE_MAX_CONNECTIONS");
+  const int want = prev ? atoi(prev) : 32;
+  int ctx_active = 0;
+  if (void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_NOLOAD)) {
+    using GetState = int (*)(int, unsigned*, int*);
+    if (auto fn = reinterpret_cast<GetState>(dlsym(h, "cuDevicePrimaryCtxGetState"))) {
+      unsigned flags = 0;
+      int active = 0;
+      if (fn(0, &flags, &active) == 0) ctx_active = active;
+    }
+    dlclose(h);
+  }
+  if (!prev) setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
+  // a context created before the load saw the user's value (if any) or the runtime default
+  const int eff = ctx_active ? (prev ? want : 8) : want;
+  g_conn_effective = std::max(1, std::min(32, eff));
+}
 
 
 thread_local std::string g_err;
@@ -236,6 +259,10 @@ Model* merge(const Model* const* parts, int n) {
 }
 
 }  // namespace
+
+namespace gmpsvm {
+int connections_in_effect() { return g_conn_effective; }
+}  // namespace gmpsvm
 
 extern "C" {
 

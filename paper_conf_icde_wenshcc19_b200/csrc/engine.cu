@@ -10,6 +10,7 @@
 #include <cstring>
 #include <deque>
 #include <thread>
+#include <map>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -27,16 +28,26 @@ std::atomic<uint64_t> g_launches{0};
   throw Error(GMPSVM_ECUDA, msg);
 }
 
+void set_max_dyn_smem(const void* func, size_t bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, size_t> done;
+  int dev = 0;
+  GM_CUDA(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(mu);
+  size_t& cur = done[{func, dev}];
+  if (bytes <= cur) return;
+  GM_CUDA(cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+  cur = bytes;
+}
+
 namespace {
 
 constexpr int kMaxK = 64;          // label-rank shared memory bound
 constexpr int kMaxCoupleK = 40;    // coupling shared memory bound
 constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
 constexpr int64_t kPredictChunk = 32768;
-constexpr int kMaxStreams = 48;    // concurrent pair groups in the solver
-constexpr int kDefaultStreams = 8; // default pair groups (hardware queues: CUDA_DEVICE_MAX_CONNECTIONS)
+constexpr int kMaxStreams = 2;     // solver streams: graph launch + graph capture
 constexpr int kDefaultB = 192;     // working-set rows (tuned on MNIST-shaped data; the tile of K_ws,ws stays in shared memory for B <= 224)
-constexpr int kChunk = 2;          // outer iterations per issued chunk
 
 struct DeviceGuard {
   int prev = -1;
@@ -270,12 +281,6 @@ T* pinned_scratch(size_t count, int slot = 0) {
 }
 
 enum { PH_STAGE, PH_KERNEL, PH_SELECT, PH_SUB, PH_FUP, PH_FIN, PH_DEC, PH_COUPLE, PH_D2H, PH_SOLVER, PH_N };
-
-// default solver structure (device-driven graph), i.e. neither GMPSVM_SOLVER=fused nor =streams
-static bool graph_solver_default(int B) {
-  static const bool streams = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "streams";
-  return !fused_solver_enabled(B) && !streams;
-}
 
 // timing events of the overlap mode's kernel-value waves (destroyed with the scope)
 struct TimedEvents {
@@ -555,7 +560,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
       dm->sc = krow_split_scale(launch_maxabs(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, st));
       HT("maxabs");
     }
-    launch_split_tf32_mu(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, dm->sc, dm->SvHi, dm->SvLo, dm->nsvc, dm->nsv_pad,
+    launch_split_hilo_mu(rows, dm->nsv_pad, m.d, d_src.get(), dm->mu, dm->sc, dm->SvHi, dm->SvLo, dm->nsvc, dm->nsv_pad,
                          dm->dpt, st);
     HT("split");
   }
@@ -616,7 +621,7 @@ static int engine_train_cv(const float* X, const int32_t* y, int64_t n, int32_t 
   const auto t_start = std::chrono::steady_clock::now();
   const int F = opt.prob_folds;
   if (F < 2 || F > 64) throw Error(GMPSVM_EINVAL, "prob_folds must be 0 or in [2, 64]");
-  if (opt.pair_ids && opt.n_pair_ids > 0)
+  if (opt.pair_ids)
     throw Error(GMPSVM_ENOTIMPL, "cross-validated sigmoids need all pairs (no pair_ids)");
   if (!X || !y || !out) throw Error(GMPSVM_EINVAL, "null argument");
   if (n < 2 || d < 1 || k < 2) throw Error(GMPSVM_EINVAL, "need n >= 2, d >= 1, k >= 2");
@@ -813,7 +818,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   DevBuf<uint8_t> tc_scratch(use_tc ? krow_tc_scratch_bytes(n, d) : 0, st);
   if (use_tc) {
     launch_row_norms(dX, n, d, d_perm.get(), norms.get(), n_pad, bad.get(), st);  // validation (non-finite rows)
-    ksc = launch_split_tf32(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st,
+    ksc = launch_split_hilo(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st,
                             ktype == 0);
   } else {
     launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
@@ -848,6 +853,9 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // ---------------- pairs to train
   const int P = k * (k - 1) / 2;
   std::vector<int> pids;
+  // an explicit but empty subset is an error, not "all pairs" (a multi-GPU rank with no pair
+  // must skip training; dist.train_predict does)
+  if (opt.pair_ids && opt.n_pair_ids <= 0) throw Error(GMPSVM_EINVAL, "pair_ids given with n_pair_ids <= 0");
   if (opt.pair_ids && opt.n_pair_ids > 0) {
     std::vector<uint8_t> seen(P, 0);
     for (int i = 0; i < opt.n_pair_ids; ++i) {
@@ -939,7 +947,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // predict) -- the waves' tensor/HBM load stretches the solver's latency-bound chain more than
   // the overlap saves.
   static const bool overlap_env = getenv("GMPSVM_OVERLAP") && std::string(getenv("GMPSVM_OVERLAP")) == "1";
-  const bool overlap = overlap_env && ktype == 0 && use_tc && graph_solver_default(B) && ws_solve_supported(B, np_max);
+  const bool overlap = overlap_env && ktype == 0 && use_tc && ws_solve_supported(B, np_max);
   cudaStream_t kst = krow_stream(opt.device);
   TimedEvents kev;
   cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
@@ -1122,79 +1130,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   HT("solver_alloc");
   launch_init_pairs(a, Pl, tot, st);
   const int64_t max_outer = opt.max_outer_iter > 0 ? opt.max_outer_iter : 1000000;
-  // Pairs are independent: groups of pairs run their outer loops on
-  // concurrent streams, so a long local solve of one pair overlaps the selection / f-update
-  // of the others instead of every pair waiting for the slowest one at each outer iteration.
-  // The host keeps two chunks of kChunk outer iterations in flight per group and stops
-  // issuing when the group's stop flags (copied back after each chunk) are all set; kernels
-  // of converged pairs exit at once, so over-issued iterations cost only empty launches.
-  static const int env_streams = getenv("GMPSVM_STREAMS") ? atoi(getenv("GMPSVM_STREAMS")) : 0;
-  const int G = std::max(1, std::min(Pl, env_streams > 0 ? std::min(env_streams, kMaxStreams) : kDefaultStreams));
-  std::vector<int> gb(G + 1);
-  for (int g = 0; g <= G; ++g) gb[g] = (int)((int64_t)g * Pl / G);
-  std::vector<int64_t> g_npmax(G, 0);
-  for (int g = 0; g < G; ++g)
-    for (int i = gb[g]; i < gb[g + 1]; ++i) g_npmax[g] = std::max<int64_t>(g_npmax[g], hp[i].n_s + hp[i].n_t);
   const std::vector<cudaStream_t>& pool = stream_pool(opt.device);
   EventPool evp;
   cudaEvent_t ev_ready = evp.get();
   GM_CUDA(cudaEventRecord(ev_ready, st));
   tm.mark(PH_SOLVER);
   HT("init");
-  for (int g = 0; g < G; ++g) GM_CUDA(cudaStreamWaitEvent(pool[g], ev_ready, 0));
-  struct {
-    int32_t* p;
-  } h_slot{pinned_scratch<int32_t>((size_t)2 * Pl)};  // two status snapshots per pair (alternating chunks)
-  struct Chunk {
-    cudaEvent_t ev;
-    int slot;
-  };
-  std::vector<std::deque<Chunk>> inflight(G);
-  std::vector<int64_t> issued(G, 0);
-  std::vector<int> nchunks(G, 0);
-  std::vector<char> stop(G, 0);
   int64_t rc_launches = 0;  // ROW_CACHE row-contraction launches
-  auto issue_chunk = [&](int g) {
-    cudaStream_t gs = pool[g];
-    SolverArgs ag = a;
-    ag.pair_base = gb[g];
-    const int gn = gb[g + 1] - gb[g];
-    for (int c = 0; c < kChunk && issued[g] < max_outer + 1; ++c) {
-      const int64_t it = issued[g]++;
-      if (!rc && ws_solve_supported(Bw, g_npmax[g])) {  // default kernels (wsolve.cu)
-        launch_ws_iteration(ag, gn, g_npmax[g], 0, 0, max_outer, gs, it > 0);
-        if (it >= max_outer) break;
-        continue;
-      }
-      launch_select_ws(ag, gn, (uint32_t)(it + 1), it == 0 ? 1 : 0, gs);
-      if (it >= max_outer) break;  // the last selection only evaluates the stop test
-      if (rc) {
-        launch_rows_compute(ag, gn, g_npmax[g], gs);
-        ++rc_launches;
-      }
-      launch_gather_kws(ag, gn, it == 0 ? 1 : 0, gs);
-      launch_local_smo(ag, gn, gs);
-      launch_f_update(ag, gn, g_npmax[g], gs);
-    }
-    const int slot = nchunks[g]++ & 1;
-    GM_CUDA(cudaMemcpyAsync(h_slot.p + (size_t)slot * Pl + gb[g], d_status.get() + gb[g], gn * 4,
-                            cudaMemcpyDeviceToHost, gs));
-    cudaEvent_t ev = evp.get();
-    GM_CUDA(cudaEventRecord(ev, gs));
-    inflight[g].push_back(Chunk{ev, slot});
-  };
-  const bool fused = full_k && fused_solver_enabled(Bw);
-  static const bool streams_mode = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "streams";
-  const bool graph_mode = !fused && !streams_mode;
   GraphGuard gg;
   int64_t body_launches = 0;
   std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
   int n_branches = 0, final_selects = 0;
-  if (fused) {  // the whole outer loop of every pair in one launch (clusters, no host round trips)
-    SolverArgs ag = a;
-    ag.pair_base = 0;
-    launch_pair_solver(ag, Pl, max_outer, pool[0]);
-  } else if (graph_mode) {
+  {
     // Device-driven outer loops (default): one CUDA graph holding, per pair, a conditional
     // WHILE node whose body is that pair's select -> [rows] -> gather -> local SMO -> f-update
     // chain (the f-update kernel sets the loop condition), followed by one last selection (the
@@ -1203,8 +1150,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     // The runtime runs at most CUDA_DEVICE_MAX_CONNECTIONS branches of a graph concurrently (a
     // branch beyond that waits for another to finish), so the pairs are packed into that many
     // branches: the largest pairs alone, the smallest two (or more) to a branch in lockstep.
-    const char* conn_env = getenv("CUDA_DEVICE_MAX_CONNECTIONS");
-    const int conn = std::max(1, std::min(32, conn_env ? atoi(conn_env) : 8));
+    const int conn = connections_in_effect();
     const int nbr = std::min(Pl, conn);
     std::vector<int> bb(nbr + 1, 0);
     {
@@ -1288,39 +1234,10 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     HT("graph_build");
     GM_CUDA(cudaGraphLaunch(gg.exec, pool[0]));
     destroy_parked_graphs();  // the previous calls' graphs, while this solver runs
-  } else {
-    for (int g = 0; g < G; ++g) issue_chunk(g);
-    for (int g = 0; g < G; ++g) issue_chunk(g);
   }
-  int running = (fused || graph_mode) ? 0 : G;
-  while (running > 0) {
-    bool progressed = false;
-    for (int g = 0; g < G; ++g) {
-      if (inflight[g].empty()) continue;
-      const Chunk ch = inflight[g].front();
-      const cudaError_t q = cudaEventQuery(ch.ev);
-      if (q == cudaErrorNotReady) continue;
-      GM_CUDA(q);
-      inflight[g].pop_front();
-      progressed = true;
-      if (stop[g]) {
-        if (inflight[g].empty()) --running;
-        continue;
-      }
-      bool all_done = true;
-      for (int i = gb[g]; i < gb[g + 1]; ++i) all_done = all_done && h_slot.p[(size_t)ch.slot * Pl + i] != 0;
-      if (all_done || issued[g] > max_outer) {
-        stop[g] = 1;
-        if (inflight[g].empty()) --running;
-      } else {
-        issue_chunk(g);
-      }
-    }
-    if (!progressed) std::this_thread::yield();
-  }
-  for (int g = 0; g < G; ++g) {
+  {
     cudaEvent_t ev = evp.get();
-    GM_CUDA(cudaEventRecord(ev, pool[g]));
+    GM_CUDA(cudaEventRecord(ev, pool[0]));
     GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
   }
   if (overlap) GM_CUDA(cudaStreamWaitEvent(st, ev_k1, 0));  // every kernel-value wave (K is reused by the next call)
@@ -1366,7 +1283,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
   HT("fin_d2h");
-  if (graph_mode) {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
+  {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
     int64_t ex = n_branches;  // one final selection per split-path branch
     for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_per_pair[i];  // counted at each branch's first pair
     g_launches.fetch_add((uint64_t)ex);
@@ -1519,7 +1436,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   s.t_fupdate_ms = tm.ms(PH_FUP);
   s.t_finalize_ms = tm.ms(PH_FIN);
   s.t_solver_ms = tm.ms(PH_SOLVER);
-  s.n_streams = graph_mode ? n_branches : G;
+  s.n_streams = n_branches;
   if (full_k) {
     s.kernel_values = kv_subset >= 0 ? kv_subset : (double)n * (double)(n + 1) / 2.0;
     s.krow_launches = 1;
@@ -1708,9 +1625,9 @@ int engine_predict_csr(const Model& mdl, const int64_t* indptr, const int32_t* i
 }
 
 // ------------------------------------------------------------------------------------------
-static void ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
+static std::shared_ptr<DevModel> ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
   std::lock_guard<std::mutex> lk(mdl.mu);
-  if (mdl.dev && mdl.dev->device == device) return;
+  if (mdl.dev && mdl.dev->device == device) return mdl.dev;
   if (mdl.dev) {  // moving to another device: the host copies are the source of the new one
     ensure_host_sv(mdl);
     ensure_host_alpha(mdl);
@@ -1724,6 +1641,7 @@ static void ensure_dev_model(const Model& mdl, int device, cudaStream_t st) {
   std::vector<int64_t> row_of_sv(nsv);
   for (int64_t i = 0; i < nsv; ++i) row_of_sv[i] = i;
   mdl.dev = build_dev_model(mdl, rows.get(), row_of_sv, device, st);
+  return mdl.dev;
 }
 
 int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
@@ -1738,8 +1656,8 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   DeviceGuard dg(opt.device);
   cudaStream_t st = get_stream(opt);
   const uint64_t launches0 = g_launches.load();
-  ensure_dev_model(mdl, opt.device, st);
-  const DevModel& dm = *mdl.dev;
+  const std::shared_ptr<DevModel> dm_ref = ensure_dev_model(mdl, opt.device, st);  // held for the whole call
+  const DevModel& dm = *dm_ref;
   const int k = mdl.k, d = mdl.d, P = mdl.P();
   PhaseTimer tm(st);
   const int64_t mc_max = std::min<int64_t>(m, kPredictChunk);
@@ -1775,7 +1693,7 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     const bool f64 = dm.f64 || (mdl.kernel != 0 && !use_tc);  // the SIMT fallback is the Gaussian's only
     if (use_tc) {
       launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
-      launch_split_tf32_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
+      launch_split_hilo_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
       // work units: (item, test tile), test tiles fastest; unit = the item's SV tiles for that test tile
       const int ntt = (int)(mcp / kTile);
       std::vector<int2> dt;
@@ -1882,7 +1800,7 @@ int engine_rbf_kernel(const float* X, int64_t n, const float* Y, int64_t m, int3
     const int64_t np2 = krow_tc_rows_pad(n);
     DevBuf<float> hi(krow_tc_buf_floats(np2, dp), st), lo(krow_tc_buf_floats(np2, dp), st), nx2(np2, st);
     DevBuf<uint8_t> scr(krow_tc_scratch_bytes(n, d), st);
-    const float ksc = launch_split_tf32(dX, n, d, nullptr, hi.get(), lo.get(), nx2.get(), np2, dp, scr.get(), st);
+    const float ksc = launch_split_hilo(dX, n, d, nullptr, hi.get(), lo.get(), nx2.get(), np2, dp, scr.get(), st);
     DevBuf<float> kb2(opt.inputs_on_device ? 0 : (size_t)n * m, st);
     float* dK2 = opt.inputs_on_device ? K_out : kb2.get();
     const bool two_cta = krow_tc_2cta() && (m % 4) == 0 && (reinterpret_cast<uintptr_t>(dK2) & 15) == 0;

@@ -7,6 +7,17 @@
 
 namespace gmpsvm {
 
+// CUDA_DEVICE_MAX_CONNECTIONS actually in effect for this process (api.cpp, at library load)
+int connections_in_effect();
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) for the CURRENT device (the attribute is
+// per device context): set once per (kernel, device) and raised when a launch needs more
+void set_max_dyn_smem(const void* func, size_t bytes);
+template <typename F>
+inline void set_max_dyn_smem(F* func, size_t bytes) {
+  set_max_dyn_smem(reinterpret_cast<const void*>(func), bytes);
+}
+
+
 // ---------------- a1 staging (stage.cu)
 void launch_class_sort(const int32_t* y, int64_t n, int k, int32_t* blk_counts, int32_t* blk_off,
                        int64_t* class_count, int64_t* class_off, cudaStream_t st);
@@ -36,7 +47,7 @@ float krow_split_scale(float maxabs);  // exact power-of-two scale of the FP16 s
 // hi/lo rows and compute the squared norms (scaled units); returns the scale
 size_t krow_tc_scratch_bytes(int64_t n, int d);
 const float* krow_tc_scratch_mu(const void* scratch, int64_t n, int d);
-float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
+float launch_split_hilo(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
                         int64_t n_pad, int d_pad, void* scratch, cudaStream_t st, bool center = true);
 // the paper's other kernels (L76-L78): type 1 linear, 2 polynomial, 3 sigmoid (inv_s2 set by the launch)
 struct KrowKernel {
@@ -63,7 +74,7 @@ constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
 // per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
 void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
 // split with a given centre mu[d] and scale sc (prediction: the test rows take the SVs' mu, sc)
-void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
+void launch_split_hilo_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
                           void* lo, float* norms, int64_t n_pad, int d_pad, cudaStream_t st);
 // mu[c] = mean over the rows idx[i] >= 0 (cnt of them) of X[., c]
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
@@ -142,9 +153,6 @@ void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st
 void launch_f_update_loop(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int64_t max_outer,
                           cudaStream_t st);
 void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
-// fused outer loop: one cluster per pair, whole solve in one launch (B <= 224)
-bool fused_solver_enabled(int B);
-void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStream_t st);
 // a3-a5 default kernels (wsolve.cu): fast selection, multi-CTA K_ws,ws gather into an
 // L2-resident tile, single-warp local SMO (FULL_K regime, B <= 224, n_p <= 16384;
 // GMPSVM_WSOLVE=0 selects the select_ws / gather_kws / local_smo kernels of solver.cu)

@@ -1,22 +1,23 @@
-// krow_tc.cu -- a2 on the 5th-generation tensor cores: the kernel-value contraction with a
-// 3xTF32 split (x = hi + lo, hi = x truncated to TF32, lo = x - hi exactly), so that
+// krow_tc.cu -- a2 (and the a10 decision values) on the 5th-generation tensor cores: the
+// kernel-value contraction with a hi/lo split of every operand, x = hi + lo, so that
 //   x.y ~= hi.hi + hi.lo + lo.hi   (the lo.lo term is below FP32 rounding)
-// is accumulated in FP32 in TMEM by tcgen05.mma kind::tf32, operands staged by TMA into
-// 128-byte-swizzled shared memory.  The epilogue (norm combine, clamp, ex2, K_ii = 1,
-// symmetric mirrored store) is the same arithmetic as krow.cu's SIMT kernel.
+// is accumulated in FP32 in TMEM by tcgen05.mma, operands staged by TMA into 128-byte-swizzled
+// shared memory.  The epilogue (norm combine, clamp, ex2, K_ii = 1, symmetric mirrored store) is
+// the same arithmetic as krow.cu's SIMT kernel.
 //
-// CTA tile 128 x 128, one CTA per tile (bi, bj) of the upper triangle, warp 0 = TMA producer,
-// warp 1 = MMA issuer (+ TMEM allocation), warps 2..5 = epilogue (one TMEM lane quarter each),
-// 3-stage smem ring of 64 KB (A hi/lo and B hi/lo, 128 x 32 FP32 each).  TMEM holds four
-// 128-column FP32 accumulators: hi.hi over each third of the k range, and hi.lo + lo.hi.
+// Default split: FP16 (kind::f16).  The rows are centred by the column means and scaled by an
+// exact power of two s (max |x - mu| s <= 2^12, inside FP16's range and away from its
+// subnormals); hi = half(x'), lo = half(x' - hi), both round-to-nearest: 11 significant bits
+// per part, so hi + lo carries x' to ~2^-22.  Distances are computed in scaled units and the exp
+// argument is divided by s^2 (exact).  GMPSVM_SPLIT=tf32 selects the TF32 split (kind::tf32, the
+// same precision at half the MMA rate).
+//
+// CTA tile 128 x 128, persistent CTAs walking the tiles (bi, bj) of the upper triangle; warp 0 =
+// TMA producer, warp 1 = MMA issuer (+ TMEM allocation), warps 2..5 = epilogue (one TMEM lane
+// quarter each); 3-stage smem ring of 64 KB (A hi/lo and B hi/lo, 128 rows x one 128-byte
+// swizzle atom along K each: 64 FP16 or 32 TF32 elements).  TMEM holds four 128-column FP32
+// accumulators: hi.hi over each third of the k range, and hi.lo + lo.hi.
 // Entry (r, c) is written, with its mirror (c, r), only by the tile that holds it with r <= c.
-//
-// Default split: FP16 instead of TF32 (GMPSVM_SPLIT=tf32 selects TF32).  Both carry an 11-bit
-// significand per part, so hi + lo represents x to ~2^-22 either way, but kind::f16 runs at twice
-// the kind::tf32 rate (K = 16 per MMA in the same cycles as K = 8).  FP16's narrow exponent range
-// is handled by an exact power-of-two scale s (max |x - mu| s <= 2^12, well inside FP16 and away
-// from its subnormals); distances are computed in scaled units and the exp argument is divided
-// by s^2 (exact).
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cudaTypedefs.h>
@@ -946,7 +947,7 @@ __global__ void col_mean_kernel(const double* __restrict__ part, int nchunks, in
 // nearest); FP16: hi = half(x'), lo = half(x' - hi); norms[j] = ||x'_j||^2 accumulated in FP64
 // (one warp per row); zero padding.  hi / lo rows are d_pad elements (4 or 2 bytes).
 template <bool F16>
-__global__ void split_tf32_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
+__global__ void split_hilo_kernel(const float* __restrict__ X, int64_t n, int d, const int64_t* __restrict__ perm,
                                   const float* __restrict__ mu, float sc, void* __restrict__ hi_, void* __restrict__ lo_,
                                   float* __restrict__ norms, int64_t n_pad, int d_pad) {
   const int64_t j = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -1044,7 +1045,7 @@ float krow_split_scale(float maxabs) {  // power of two with maxabs * s <= 2^12 
   return (float)std::ldexp(1.0, e);
 }
 
-const float* krow_tc_scratch_mu(const void* scratch, int64_t n, int d) {  // the column means launch_split_tf32 left
+const float* krow_tc_scratch_mu(const void* scratch, int64_t n, int d) {  // the column means launch_split_hilo left
   return reinterpret_cast<const float*>(static_cast<const double*>(scratch) + (size_t)ceil_div(n, kMeanRows) * d);
 }
 size_t krow_tc_scratch_bytes(int64_t n, int d) {
@@ -1065,17 +1066,17 @@ float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const
   return v;
 }
 
-void launch_split_tf32_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
+void launch_split_hilo_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
                           void* lo, float* norms, int64_t n_pad, int d_pad, cudaStream_t st) {
   if (krow_split_f16())
-    GM_LAUNCH(split_tf32_kernel<true>, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, sc, hi,
+    GM_LAUNCH(split_hilo_kernel<true>, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, sc, hi,
               lo, norms, n_pad, d_pad);
   else
-    GM_LAUNCH(split_tf32_kernel<false>, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, 1.f,
+    GM_LAUNCH(split_hilo_kernel<false>, dim3((unsigned)ceil_div(n_pad, 8)), dim3(256), 0, st, X, n, d, perm, mu, 1.f,
               hi, lo, norms, n_pad, d_pad);
 }
 
-float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
+float launch_split_hilo(const float* X, int64_t n, int d, const int64_t* perm, void* hi, void* lo, float* norms,
                         int64_t n_pad, int d_pad, void* scratch, cudaStream_t st, bool center) {
   const int nch = (int)ceil_div(n, kMeanRows);
   double* part = static_cast<double*>(scratch);
@@ -1087,7 +1088,7 @@ float launch_split_tf32(const float* X, int64_t n, int d, const int64_t* perm, v
     GM_CUDA(cudaMemsetAsync(mu, 0, (size_t)d * sizeof(float), st));
   }
   const float sc = krow_split_f16() ? krow_split_scale(launch_maxabs(X, n, d, nullptr, mu, st)) : 1.f;
-  launch_split_tf32_mu(X, n, d, perm, mu, sc, hi, lo, norms, n_pad, d_pad, st);
+  launch_split_hilo_mu(X, n, d, perm, mu, sc, hi, lo, norms, n_pad, d_pad, st);
   return sc;
 }
 
@@ -1186,15 +1187,11 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
   const int tma = !no_tma_env && (ldk % 4) == 0 && (reinterpret_cast<uintptr_t>(K) & 15) == 0 && n < (int64_t)INT32_MAX;
   const CUtensorMap mksw = make_kmap(K, tma ? n : 1, tma ? ldk : 4, true), mkns = make_kmap(K, tma ? n : 1, tma ? ldk : 4, false);
   const size_t smem = sizeof(TcSmem) + 1024;
-  static bool configured = false;
-  if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<false, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    GM_CUDA(cudaFuncSetAttribute(krow_tc_kernel<true, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured = true;
-  }
+  set_max_dyn_smem(krow_tc_kernel<true, 0>, smem);
+  set_max_dyn_smem(krow_tc_kernel<false, 0>, smem);
+  set_max_dyn_smem(krow_tc_kernel<true, 1>, smem);
+  set_max_dyn_smem(krow_tc_kernel<true, 2>, smem);
+  set_max_dyn_smem(krow_tc_kernel<true, 3>, smem);
   // distances are in units scaled by sc: exp(-gamma d2 / sc^2) = exp2(d2 * scale)
   const float scale = (float)(-gamma * 1.4426950408889634 / ((double)sc * (double)sc));
   const int sms = num_sms();
@@ -1202,11 +1199,7 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
   if (two_cta) {
     if (!f16 || !tma) throw Error(GMPSVM_EINVAL, "CTA-pair kernel-value launch needs the FP16 split and TMA stores");
     const size_t smem2 = sizeof(Tc2Smem) + 1024;
-    static bool configured2 = false;
-    if (!configured2) {
-      GM_CUDA(cudaFuncSetAttribute(krow_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2));
-      configured2 = true;
-    }
+    set_max_dyn_smem(krow_tc2_kernel, smem2);
     // B operand: 64-row boxes (each CTA of the pair loads its half of the 128 columns' rows)
     const CUtensorMap mbhi = make_map(hi, n_pad, d_pad, f16, kTN / 2), mblo = make_map(lo, n_pad, d_pad, f16, kTN / 2);
     const int clusters = std::min(n_tiles, sms / 2);
@@ -1269,26 +1262,22 @@ void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* 
     kp = *dk;
     kp.inv_s2 = (float)(1.0 / ((double)sc * (double)sc));
   }
-  auto go = [&](auto kern, size_t smem, bool& configured) {
-    if (!configured) {
-      GM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      configured = true;
-    }
+  auto go = [&](auto kern, size_t smem) {
+    set_max_dyn_smem(kern, smem);
     GM_LAUNCH(kern, dim3(grid), dim3(kTcThreads), smem, st, mthi, mtlo, mshi, mslo, tiles, unit_off, unit_item, n_units,
               nt, nsv, coef, km1, km1_pad, nk, scale, m_pad, part, kp);
   };
-  static bool c[7] = {false, false, false, false, false, false, false};
   if (dk) {  // the other kernels: FP16 split, k - 1 <= 12 (engine.cu routes the rest to the FP64 path)
     if (!f16 || km1_pad > 12) throw Error(GMPSVM_ENOTIMPL, "tensor-core decision values of this kernel need k <= 13");
-    if (kp.type == 1) go(dec_tc_kernel<12, true, 1>, sizeof(DecTcSmem<12>) + 1024, c[4]);
-    else if (kp.type == 2) go(dec_tc_kernel<12, true, 2>, sizeof(DecTcSmem<12>) + 1024, c[5]);
-    else go(dec_tc_kernel<12, true, 3>, sizeof(DecTcSmem<12>) + 1024, c[6]);
+    if (kp.type == 1) go(dec_tc_kernel<12, true, 1>, sizeof(DecTcSmem<12>) + 1024);
+    else if (kp.type == 2) go(dec_tc_kernel<12, true, 2>, sizeof(DecTcSmem<12>) + 1024);
+    else go(dec_tc_kernel<12, true, 3>, sizeof(DecTcSmem<12>) + 1024);
   } else if (km1_pad <= 12) {
-    if (f16) go(dec_tc_kernel<12, true>, sizeof(DecTcSmem<12>) + 1024, c[0]);
-    else go(dec_tc_kernel<12, false>, sizeof(DecTcSmem<12>) + 1024, c[1]);
+    if (f16) go(dec_tc_kernel<12, true>, sizeof(DecTcSmem<12>) + 1024);
+    else go(dec_tc_kernel<12, false>, sizeof(DecTcSmem<12>) + 1024);
   } else {
-    if (f16) go(dec_tc_kernel<kDecMaxKm1, true>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024, c[2]);
-    else go(dec_tc_kernel<kDecMaxKm1, false>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024, c[3]);
+    if (f16) go(dec_tc_kernel<kDecMaxKm1, true>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024);
+    else go(dec_tc_kernel<kDecMaxKm1, false>, sizeof(DecTcSmem<kDecMaxKm1>) + 1024);
   }
 }
 

@@ -72,7 +72,9 @@ struct Model {
   bool sv_X_ready = false;
   gmpsvm_train_stats stats{};
   mutable std::mutex mu;
-  mutable std::unique_ptr<DevModel> dev;
+  // shared: a prediction holds its own reference for the whole call, so a concurrent call that
+  // moves the model to another device (ensure_dev_model) cannot free structures still in use
+  mutable std::shared_ptr<DevModel> dev;
 
   int P() const { return k * (k - 1) / 2; }
   std::vector<int64_t> class_off() const;

@@ -233,11 +233,7 @@ void launch_dec_contract(const float* XtT, int64_t ldt, const float* nt, int64_t
                          int64_t lds, const float* nsv, const float* coef, int km1, int km1_pad, const DecItem* items,
                          int n_items, int kdim, double gamma, float* part, cudaStream_t st) {
   const size_t smem = sizeof(GemmSmem) + 2 * (size_t)kTile * km1_pad * sizeof(float);
-  static size_t configured = 0;
-  if (smem > 48 * 1024 && smem > configured) {
-    GM_CUDA(cudaFuncSetAttribute(dec_contract_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured = smem;
-  }
+  if (smem > 48 * 1024) set_max_dyn_smem(dec_contract_kernel, smem);
   const float scale = (float)(-gamma * 1.4426950408889634);
   GM_LAUNCH(dec_contract_kernel, dim3((unsigned)(m_pad / kTile), (unsigned)n_items), dim3(kGemmThreads), smem, st, XtT,
             ldt, nt, m, m_pad, SvT, lds, nsv, coef, km1, km1_pad, items, kdim, scale, part);
@@ -384,11 +380,7 @@ void launch_dec_f64(const float* XtT, int64_t ldt, const double* nt64, int64_t m
                     const double* nsv64, const double* coef64, int km1, int km1_pad, const DecItem* items, int n_items,
                     int d_pad, double gamma, double* part, cudaStream_t st, int ktype, double coef0, int degree) {
   const size_t smem = (size_t)(2 * kF64BK * kF64Tile + 2 * kF64Tile * km1_pad) * sizeof(double);
-  static bool configured = false;
-  if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(dec_f64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(96 * 1024)));
-    configured = true;
-  }
+  set_max_dyn_smem(dec_f64_kernel, 96 * 1024);
   GM_LAUNCH(dec_f64_kernel, dim3((unsigned)(m_pad / kF64Tile), (unsigned)n_items), dim3(256), smem, st, XtT, ldt, nt64,
             SvT, lds, nsv64, coef64, km1, km1_pad, items, d_pad, gamma, m_pad, part, ktype, coef0, degree);
 }
@@ -411,11 +403,7 @@ void launch_couple(const double* dec, int64_t m, int k, const double* A, const d
                    cudaStream_t st) {
   const size_t per = (size_t)k * k + (size_t)(k + 1) * (k + 2);
   const size_t smem = per * kCoupleWarps * sizeof(double);
-  static size_t configured = 0;
-  if (smem > 48 * 1024 && smem > configured) {
-    GM_CUDA(cudaFuncSetAttribute(couple_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured = smem;
-  }
+  if (smem > 48 * 1024) set_max_dyn_smem(couple_kernel, smem);
   GM_LAUNCH(couple_kernel, dim3((unsigned)ceil_div(m, kCoupleWarps)), dim3(32 * kCoupleWarps), smem, st, dec, m, k, A,
             B, prob);
 }

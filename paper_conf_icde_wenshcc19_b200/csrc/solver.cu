@@ -777,221 +777,6 @@ __global__ void __launch_bounds__(SMEM ? kSmemMaxB : 1024 / E) local_smo_kernel(
   smo_body<E, SMEM>(a, blockIdx.x + a.pair_base, blockDim.x, 0, slots, kw_smem);
 }
 
-// Single-warp local SMO (B <= kSmemMaxB): the whole working set lives in the registers of one
-// warp (lane owns rows lane, lane + 32, ...), so the two argmin/argmax reductions of every inner
-// step are warp-level (redux.sync + ballot) with no CTA barrier and no shared-memory slots; the
-// winner's f comes from its key, its K_ee from the shared K_ws,ws tile, so only alpha and the
-// row index are shuffled.  All CTA threads copy K_ws,ws into shared memory first; warps 1.. then
-// exit.  Same arithmetic and tie rules as smo_body, so the iterates are identical.
-template <int E>
-__device__ __forceinline__ void smo_warp(const SolverArgs& a, int lp, const float* Kw, long long t_entry) {
-  const int lane = threadIdx.x;
-  const PairDesc pd = a.pairs[lp];
-  const int B = a.B, wn = a.ws_n[lp];
-  const double C = a.C;
-  bool valid[E], iu[E], il[E];
-  int32_t idx[E];
-  int y[E];
-  double al[E], a0[E], fv[E];
-  float kd[E], va[E], vb[E], ku[E];
-#pragma unroll
-  for (int q = 0; q < E; ++q) {
-    const int e = lane + 32 * q;
-    valid[q] = e < wn;
-    idx[q] = valid[q] ? a.ws[(int64_t)lp * B + e] : INT_MAX;
-    y[q] = (valid[q] && idx[q] < pd.n_s) ? 1 : -1;
-    al[q] = valid[q] ? a.alpha[pd.a_off + idx[q]] : 0.0;
-    a0[q] = al[q];
-    fv[q] = valid[q] ? a.f[pd.a_off + idx[q]] : 0.0;
-    kd[q] = valid[q] ? Kw[(int64_t)e * B + e] : 1.f;
-    iu[q] = valid[q] && in_u(y[q], al[q], C);
-    il[q] = valid[q] && in_l(y[q], al[q], C);
-    va[q] = vb[q] = 0.f;
-  }
-  int ra = -1, rb = -1;
-  const int cap = a.inner_cap;
-  int it = 0;
-  double delta0 = 0.0;
-  const long long t_begin = clock64();
-  long long ph[4] = {0, 0, 0, 0}, tp = t_begin;
-  const bool prof = a.smo_phase != nullptr;
-  for (;;) {
-    // Step 1 (Eq 4): u = argmin_{I_u} f, ties -> lowest pair-local index
-    uint32_t h0 = 0xffffffffu, l0 = 0xffffffffu;
-    int32_t bi = INT_MAX;
-    int be = 0;
-    double ba = 0.0;
-#pragma unroll
-    for (int q = 0; q < E; ++q) {
-      if (iu[q]) {
-        const uint64_t key = ord_key(fv[q]);
-        const uint32_t h = (uint32_t)(key >> 32), l = (uint32_t)key;
-        if (h < h0 || (h == h0 && (l < l0 || (l == l0 && idx[q] < bi)))) {
-          h0 = h;
-          l0 = l;
-          bi = idx[q];
-          be = lane + 32 * q;
-          ba = al[q];
-        }
-      }
-    }
-    const int wu = warp_argmin(h0, l0, bi);
-    if (bi == INT_MAX) break;
-    const int ue = __shfl_sync(FULLMASK, be, wu);
-    const double au = __shfl_sync(FULLMASK, ba, wu);
-    const double fu = key_double(((uint64_t)h0 << 32) | l0);
-    const float kuu = Kw[(int64_t)ue * B + ue];
-    const int yu = bi < pd.n_s ? 1 : -1;
-    if (prof) {
-      const long long t = clock64();
-      ph[0] += t - tp;
-      tp = t;
-    }
-    if (ue == ra) {
-#pragma unroll
-      for (int q = 0; q < E; ++q) ku[q] = va[q];
-    } else if (ue == rb) {
-#pragma unroll
-      for (int q = 0; q < E; ++q) ku[q] = vb[q];
-    } else {
-      const float* row = Kw + (int64_t)ue * B;
-#pragma unroll
-      for (int q = 0; q < E; ++q) ku[q] = valid[q] ? row[lane + 32 * q] : 0.f;
-    }
-    // Eq 5: l = argmax_{t in I_l, f_t > f_u} (f_u - f_t)^2 / eta_t, and f_max over I_l (Eq 10)
-    uint32_t m0 = 0u, m1 = 0u;
-    uint32_t g0 = 0xffffffffu, g1 = 0u;
-    int32_t li = INT_MAX;
-    int le_c = 0;
-    double la = 0.0, lf = 0.0;
-#pragma unroll
-    for (int q = 0; q < E; ++q) {
-      if (il[q]) {
-        const uint64_t fk = ord_key(fv[q]);
-        const uint32_t h = (uint32_t)(fk >> 32), l = (uint32_t)fk;
-        if (h > m0 || (h == m0 && l > m1)) {
-          m0 = h;
-          m1 = l;
-        }
-        if (fv[q] > fu) {
-          const float eta = fmaxf(kuu + kd[q] - 2.f * ku[q], 1e-12f);
-          const float df = (float)(fv[q] - fu);
-          const uint32_t sk = ~__float_as_uint(df * df * __frcp_rn(eta));
-          if (sk < g0 || (sk == g0 && idx[q] < li)) {
-            g0 = sk;
-            li = idx[q];
-            le_c = lane + 32 * q;
-            la = al[q];
-            lf = fv[q];
-          }
-        }
-      }
-    }
-    const int wl = warp_argmin(g0, g1, li);
-    warp_max64(m0, m1);
-    if (prof) {
-      const long long t = clock64();
-      ph[1] += t - tp;
-      tp = t;
-    }
-    const double fmax = (m0 == 0u && m1 == 0u) ? -DBL_MAX : key_double(((uint64_t)m0 << 32) | m1);
-    const double gap = fmax - fu;
-    if (it == 0) delta0 = gap;
-    const double tol = a.eps > a.local_ratio * delta0 ? a.eps : a.local_ratio * delta0;
-    if (!(gap >= tol) || li == INT_MAX || it >= cap) break;
-    const int le = __shfl_sync(FULLMASK, le_c, wl);
-    const double alv = __shfl_sync(FULLMASK, la, wl);
-    const double fl = __shfl_sync(FULLMASK, lf, wl);
-    const float kll = Kw[(int64_t)le * B + le], kul = Kw[(int64_t)ue * B + le];
-    const int yl = li < pd.n_s ? 1 : -1;
-    // Step 2 (Eq 6-7) with explicit clipping (reading R4): common step s (FP64)
-    double eta = (double)kuu + (double)kll - 2.0 * (double)kul;
-    eta = eta > kTau ? eta : kTau;
-    double s = (fl - fu) / eta;
-    const double Uu = yu > 0 ? C - au : au;
-    const double Ll = yl > 0 ? alv : C - alv;
-    bool bu = false, bl = false;
-    if (Uu <= s) {
-      s = Uu;
-      bu = true;
-    }
-    if (Ll <= s) {
-      if (Ll < s) bu = false;
-      s = Ll;
-      bl = true;
-    }
-    double nau = au + yu * s, nal = alv - yl * s;
-    if (bu) nau = yu > 0 ? C : 0.0;
-    if (bl) nal = yl > 0 ? 0.0 : C;
-    // Step 3 (Eq 8) on the working set: f_i += s (K_ui - K_li)
-    float kl[E];
-    if (le == ra) {
-#pragma unroll
-      for (int q = 0; q < E; ++q) kl[q] = va[q];
-    } else if (le == rb) {
-#pragma unroll
-      for (int q = 0; q < E; ++q) kl[q] = vb[q];
-    } else {
-      const float* row = Kw + (int64_t)le * B;
-#pragma unroll
-      for (int q = 0; q < E; ++q) kl[q] = valid[q] ? row[lane + 32 * q] : 0.f;
-    }
-#pragma unroll
-    for (int q = 0; q < E; ++q) {
-      const int e = lane + 32 * q;
-      fv[q] += s * ((double)ku[q] - (double)kl[q]);
-      if (e == ue || e == le) {
-        al[q] = (e == ue) ? nau : nal;
-        iu[q] = in_u(y[q], al[q], C);
-        il[q] = in_l(y[q], al[q], C);
-      }
-      va[q] = ku[q];
-      vb[q] = kl[q];
-    }
-    ra = ue;
-    rb = le;
-    ++it;
-    if (prof) {
-      const long long t = clock64();
-      ph[3] += t - tp;
-      tp = t;
-    }
-  }
-#pragma unroll
-  for (int q = 0; q < E; ++q) {
-    const int e = lane + 32 * q;
-    if (valid[q]) {
-      a.alpha[pd.a_off + idx[q]] = al[q];
-      a.dcoef[(int64_t)lp * B + e] = (al[q] - a0[q]) * (double)y[q];
-    }
-  }
-  if (lane == 0) {
-    a.inner_iters[lp] += it;
-    a.smo_cycles[lp] += clock64() - t_begin;
-    if (prof) {
-      for (int k = 0; k < 4; ++k) a.smo_phase[lp * 5 + k] += ph[k];
-      a.smo_phase[lp * 5 + 4] += t_begin - t_entry;
-    }
-  }
-}
-
-template <int E>
-__global__ void __launch_bounds__(256) local_smo_warp_kernel(SolverArgs a) {
-  TraceScope ts_(a, blockIdx.x + a.pair_base, 2);
-  extern __shared__ float kw_smem[];
-  const long long t_entry = clock64();
-  const int lp = blockIdx.x + a.pair_base;
-  if (a.status[lp] != 0) return;
-  const int B = a.B;
-  const float4* src = reinterpret_cast<const float4*>(a.Kws + (int64_t)lp * kws_pair_stride(B));
-  float4* dst = reinterpret_cast<float4*>(kw_smem);
-  const int nv = (B * B) / 4;
-  for (int i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
-  __syncthreads();
-  if (threadIdx.x >= 32) return;
-  smo_warp<E>(a, lp, kw_smem, t_entry);
-}
-
 // ------------------------------------------------------------------------------------------
 // a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij for all j in the pair.
 // HBM-bound GEMV over the rows with dalpha != 0: each thread owns kFQ 16-byte column quads of
@@ -1226,98 +1011,6 @@ __global__ void __launch_bounds__(kFSThreads) f_update_kernel(SolverArgs a) {
   if (a.status[lp] != 0) return;
   __shared__ FupSplitSmem fs;
   fupdate_split(a, lp, (int64_t)blockIdx.y * 32, fs);
-}
-
-
-// ------------------------------------------------------------------------------------------
-// a3-a6 fused: one thread-block cluster of nc CTAs runs the whole outer loop of one pair
-// (Algorithm 2 lines 5-12) without returning to the host.  Per outer iteration:
-//   all CTAs   f-update of the previous local solve, columns split across the cluster
-//   CTA 0      working-set selection + stop test (all threads)
-//   all CTAs   K_ws,ws gather, rows split across the cluster
-//   CTA 0      local SMO on the first round_up(B, 32) threads (named barrier 1)
-// separated by cluster barriers (release/acquire at cluster scope also order the global
-// memory the phases exchange).  Pairs progress independently -- no lock-step with the slowest
-// pair, no host round trip per outer iteration.  Shared memory is reused by the phases.
-constexpr size_t kFusedDynBytes =
-    kSelDynBytes > (size_t)kSmemMaxB * kSmemMaxB * 4 ? kSelDynBytes : (size_t)kSmemMaxB * kSmemMaxB * 4;
-
-constexpr int kFusedThreads = 512;  // 128 registers per thread for the local SMO loop
-
-__global__ void __launch_bounds__(kFusedThreads, 1) pair_solver_kernel(SolverArgs a, int64_t max_outer) {
-  __shared__ SelSmem sm;
-  __shared__ RedSlot slots[2][32];
-  extern __shared__ __align__(16) unsigned char dyn[];
-  uint32_t nc, rank;
-  asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(nc));
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
-  const int lp = blockIdx.x / nc + a.pair_base;
-  const PairDesc pd = a.pairs[lp];
-  const int np = pd.n_s + pd.n_t;
-  const int64_t nq = (((pd.off_s + pd.n_s + 3) >> 2) - (pd.off_s >> 2)) + (((pd.off_t + pd.n_t + 3) >> 2) - (pd.off_t >> 2));
-  const int nts = (a.B + 31) / 32 * 32;
-  auto cluster_sync = []() {
-    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-  };
-  for (int64_t it = 0;; ++it) {
-    if (it > 0) {
-      const int64_t per = (nq + nc - 1) / nc;
-      fupdate_body(a, lp, rank * per, rank * per + per, *reinterpret_cast<FupSmem*>(dyn));
-      __syncthreads();
-    }
-    cluster_sync();
-    if (rank == 0) select_body(a, lp, (uint32_t)(it + 1), it == 0 ? 1 : 0, sm, dyn);
-    __syncthreads();
-    cluster_sync();
-    if (*(volatile int32_t*)(a.status + lp) != 0 || it >= max_outer) break;
-    if (np > a.B || it == 0) {
-      const int wn = *(volatile int32_t*)(a.ws_n + lp);
-      const int per = (wn + (int)nc - 1) / (int)nc;
-      gather_rows_body(a, lp, rank * per, rank * per + per, reinterpret_cast<int64_t*>(dyn));
-      __syncthreads();
-    }
-    cluster_sync();
-    if (rank == 0 && (int)threadIdx.x < nts) smo_body<1, true>(a, lp, nts, 1, slots, reinterpret_cast<float*>(dyn));
-    __syncthreads();
-    cluster_sync();
-  }
-}
-
-int fused_solver_cluster() {
-  static const int nc = getenv("GMPSVM_CLUSTER") ? atoi(getenv("GMPSVM_CLUSTER")) : 3;
-  return nc < 1 ? 1 : (nc > 8 ? 8 : nc);
-}
-
-void launch_pair_solver(const SolverArgs& a, int P, int64_t max_outer, cudaStream_t st) {
-  const int nc = fused_solver_cluster();
-  static bool configured = false;
-  if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(pair_solver_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFusedDynBytes));
-    configured = true;
-  }
-  cudaLaunchConfig_t cfg{};
-  cfg.gridDim = dim3((unsigned)(P * nc));
-  cfg.blockDim = dim3(kFusedThreads);
-  cfg.dynamicSmemBytes = kFusedDynBytes;
-  cfg.stream = st;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = nc;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  GM_CUDA(cudaLaunchKernelEx(&cfg, pair_solver_kernel, a, max_outer));
-  g_launches.fetch_add(1, std::memory_order_relaxed);
-}
-
-// Default: the stream-group solver (measured faster on MNIST-shaped data, where the hardest
-// pair's chain dominates and benefits from whole-GPU f-update / gather launches);
-// GMPSVM_SOLVER=fused selects the one-launch cluster solver.
-bool fused_solver_enabled(int B) {
-  static const bool on = getenv("GMPSVM_SOLVER") && std::string(getenv("GMPSVM_SOLVER")) == "fused";
-  return on && B <= kSmemMaxB;
 }
 
 
@@ -1562,11 +1255,7 @@ void launch_init_pairs(const SolverArgs& a, int P, int64_t tot, cudaStream_t st)
 }
 void launch_select_ws(const SolverArgs& a, int P, uint32_t stampv, int first, cudaStream_t st) {
   const size_t dyn = (size_t)kSelSmemMax * 9 + 16 + sizeof(SelLists);  // keys (8 B) + flags (1 B) + lists
-  static bool configured = false;
-  if (!configured) {
-    GM_CUDA(cudaFuncSetAttribute(select_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
-    configured = true;
-  }
+  set_max_dyn_smem(select_ws_kernel, dyn);
   GM_LAUNCH(select_ws_kernel, dim3(P), dim3(1024), dyn, st, a, stampv, first);
 }
 void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st) {
@@ -1575,51 +1264,17 @@ void launch_gather_kws(const SolverArgs& a, int P, int first, cudaStream_t st) {
 bool local_smo_uses_smem(int B) { return B <= kSmemMaxB; }
 
 void launch_local_smo(const SolverArgs& a, int P, cudaStream_t st) {
-  // default: the CTA-wide solver (2,130 cycles per inner step on B200 vs 4,350 for the
-  // single-warp variant, whose per-lane FP64 work over 7 rows is serial); GMPSVM_SMO=warp
-  // selects the single-warp one
-  static const bool warp_smo = getenv("GMPSVM_SMO") && std::string(getenv("GMPSVM_SMO")) == "warp";
-  if (local_smo_uses_smem(a.B) && warp_smo) {
-    const size_t dyn = (size_t)a.B * a.B * sizeof(float);
-    const int E = (int)ceil_div(a.B, 32);
-    static bool configured_w[8] = {};
-    auto go = [&](auto kern) {
-      if (!configured_w[E]) {
-        GM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSmemMaxB * kSmemMaxB * 4)));
-        configured_w[E] = true;
-      }
-      GM_LAUNCH(kern, dim3(P), dim3(256), dyn, st, a);
-    };
-    switch (E) {
-      case 1: go(local_smo_warp_kernel<1>); break;
-      case 2: go(local_smo_warp_kernel<2>); break;
-      case 3: go(local_smo_warp_kernel<3>); break;
-      case 4: go(local_smo_warp_kernel<4>); break;
-      case 5: go(local_smo_warp_kernel<5>); break;
-      case 6: go(local_smo_warp_kernel<6>); break;
-      default: go(local_smo_warp_kernel<7>); break;
-    }
-    return;
-  }
   if (local_smo_uses_smem(a.B)) {
     const size_t dyn = (size_t)a.B * a.B * sizeof(float);
-    static size_t configured = 0;
-    if (dyn > configured) {
-      GM_CUDA(cudaFuncSetAttribute(local_smo_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)(kSmemMaxB * kSmemMaxB * 4 + kSmemMaxB * 4)));
-      configured = (size_t)kSmemMaxB * kSmemMaxB * 4 + kSmemMaxB * 4;
-    }
+    set_max_dyn_smem(local_smo_kernel<1, true>, (size_t)kSmemMaxB * kSmemMaxB * 4 + kSmemMaxB * 4);
     GM_LAUNCH((local_smo_kernel<1, true>), dim3(P), dim3((unsigned)round_up(a.B, 32)), dyn, st, a);
     return;
   }
-  // E working-set rows per thread; GMPSVM_SMO_E overrides the default (tuning)
-  static const int e_env = getenv("GMPSVM_SMO_E") ? atoi(getenv("GMPSVM_SMO_E")) : 0;
-  int E = e_env > 0 ? e_env : (a.B > 256 ? 2 : 1);
-  if (E != 1 && E != 2 && E != 4) E = 2;
+  // E working-set rows per thread (B <= 1024 with at most 512 threads)
+  const int E = a.B > 256 ? 2 : 1;
   const int nt = (int)round_up(ceil_div(a.B, E), 32);
   if (E == 1) GM_LAUNCH((local_smo_kernel<1, false>), dim3(P), dim3(nt), 0, st, a);
-  else if (E == 2) GM_LAUNCH((local_smo_kernel<2, false>), dim3(P), dim3(nt), 0, st, a);
-  else GM_LAUNCH((local_smo_kernel<4, false>), dim3(P), dim3(nt), 0, st, a);
+  else GM_LAUNCH((local_smo_kernel<2, false>), dim3(P), dim3(nt), 0, st, a);
 }
 void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st) {
   // +8 columns: each class segment may add a partial quad at either end

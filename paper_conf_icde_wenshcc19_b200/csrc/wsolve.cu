@@ -952,8 +952,8 @@ static void launch_pdl(void (*kern)(KArgs...), dim3 g, dim3 b, size_t smem, cuda
 
 template <int E>
 static void smo_configure(int smem) {
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<E, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  GM_CUDA(cudaFuncSetAttribute(ws_smo_kernel<E, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  set_max_dyn_smem(ws_smo_kernel<E, false>, smem);
+  set_max_dyn_smem(ws_smo_kernel<E, true>, smem);
 }
 template <int E>
 static void launch_smo(const SolverArgs& a, int P, size_t smem, cudaStream_t st) {
@@ -962,9 +962,7 @@ static void launch_smo(const SolverArgs& a, int P, size_t smem, cudaStream_t st)
 }
 
 static void ws_configure() {
-  static bool configured = false;
-  if (configured) return;
-  GM_CUDA(cudaFuncSetAttribute(ws_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)((size_t)kWMaxNp * 9)));
+  set_max_dyn_smem(ws_select_kernel, (size_t)kWMaxNp * 9);
   const int mx = (int)ws_smo_smem(kWMaxB);
   smo_configure<1>(mx);
   smo_configure<2>(mx);
@@ -973,7 +971,6 @@ static void ws_configure() {
   smo_configure<5>(mx);
   smo_configure<6>(mx);
   smo_configure<7>(mx);
-  configured = true;
 }
 
 void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int set_cond,

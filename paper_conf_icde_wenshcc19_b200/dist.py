@@ -84,6 +84,8 @@ def pack_solutions(part: "gm.Model", counts):
     P = len(pairs)
     tot = int(off[-1])
     v = np.zeros(tot + 5 * P)
+    if part is None:  # a rank with no pair (more ranks than pairs): contributes zeros
+        return v
     mine = part.trained_pairs()
     for p in mine:
         s, t = pairs[p]
@@ -152,10 +154,12 @@ def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
     yy = y.cpu().numpy() if isinstance(y, torch.Tensor) else np.asarray(y)
     counts = np.bincount(yy, minlength=k)
     mine = plan_pairs(counts, world)[rank]
-    part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts)
+    # more ranks than pairs: a rank with an empty shard trains nothing and adds zeros to the
+    # all-reduce (the library rejects an empty pair_ids list rather than training every pair)
+    part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts) if mine else None
     dev_opts = {key: opts[key] for key in ("device", "stream", "kernel", "coef0", "degree") if key in opts}
     model = gather_solutions(part, X, y, k, C, gamma, group, **dev_opts)
-    model.part_stats = part.train_stats()  # this rank's training (the rebuilt model has no solver stats)
+    model.part_stats = part.train_stats() if part is not None else None  # this rank's training
     m = Xt.shape[0]
     lo, hi = row_range(m, world, rank)
     prob_local = model.predict_proba(Xt[lo:hi])

@@ -20,9 +20,9 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _problem():
+def _problem(k=4):
     rng = np.random.default_rng(0)
-    k, n, d = 4, 60, 5
+    n, d = 60, 5
     X = rng.normal(size=(n, d)).astype(np.float32)
     y = (np.arange(n) % k).astype(np.int32)
     rng.shuffle(y)
@@ -75,6 +75,64 @@ def _worker(rank, world, port, q):
     finally:
         if dist.is_initialized():
             dist.destroy_process_group()
+
+
+def _pack_worker(rank, world, port, q):
+    """pack_solutions + the all-reduce of dist.gather_solutions with more ranks than pairs
+    (k = 3: P = 3 < world = 4): the empty shard contributes zeros; the reduced vector holds every
+    pair exactly once, in the global [alpha | b | A | B | status | trained] layout."""
+    try:
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        import paper_conf_icde_wenshcc19_b200 as gm
+        from paper_conf_icde_wenshcc19_b200 import dist as gdist
+
+        X, y, k, alphas, b, A, B = _problem(k=3)
+        counts = np.bincount(y, minlength=k)
+        shards = gdist.plan_pairs(counts, world)
+        mine = shards[rank]
+        ssz = ct.sizeof(gm._lib.TrainStats)
+        part = None
+        if mine:
+            blob, _, _ = make_blob(X, y, k, 1.0, 0.5, 1e-3, {p: alphas[p] for p in mine}, b, A, B, ssz)
+            part = gm.Model.deserialize(blob)
+        v = torch.from_numpy(gdist.pack_solutions(part, counts))
+        dist.all_reduce(v, op=dist.ReduceOp.SUM)
+        v = v.numpy()
+        pairs, off = gdist.pair_layout(counts)
+        P, tot = len(pairs), int(off[-1])
+        ok = sum(1 for s in shards if not s) == world - P
+        ok &= bool(np.all(v[tot + 4 * P:] == 1.0))
+        for p in range(P):
+            ok &= bool(np.array_equal(v[off[p]:off[p + 1]], alphas[p]))
+        ok &= bool(np.array_equal(v[tot:tot + P], b) and np.array_equal(v[tot + P:tot + 2 * P], A))
+        ok &= bool(np.array_equal(v[tot + 2 * P:tot + 3 * P], B))
+        q.put((rank, bool(ok), ""))
+    except Exception as e:
+        q.put((rank, False, repr(e)))
+    finally:
+        if dist.is_initialized():
+            dist.destroy_process_group()
+
+
+def _run(target, world):
+    import __graft_entry__
+
+    __graft_entry__.build()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=target, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    assert all(ok for _, ok, _ in res), res
+
+
+def test_gloo_world4_pack_solutions_more_ranks_than_pairs():
+    _run(_pack_worker, 4)
 
 
 def test_plan_pairs_lpt_covers_all_pairs():

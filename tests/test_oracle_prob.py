@@ -181,3 +181,53 @@ def test_cross_validated_sigmoids_oracle():
         P1 = 1 / (1 + np.exp(z))
         gA, gB = ((tgt - P1) * m["v_cv"][p]).sum(), (tgt - P1).sum()
         assert abs(gA) < 1e-4 and abs(gB) < 1e-4
+
+
+# ----------------------------------------------------------------------------- predict (Eq 11, 12, 14-15)
+@pytest.mark.parametrize("name,C,gamma", [("blobs", 1.0, 0.5), ("blobs", 100.0, 0.03), ("letter", 10.0, 0.5)])
+def test_predict_pinned_by_independent_numpy(name, C, gamma):
+    """oracle.predict re-derived independently: Eq 11 by a direct-difference numpy RBF, the pair
+    sigmoid of Eq 12 with r_st = P(class s | pair) = 1/(1 + exp(A dec + B)) for s the +1 class,
+    clamped to [1e-7, 1 - 1e-7] (reading R15) and r_ts = 1 - r_st (L208), then Eq 14-15 as the
+    bordered linear system [Q e; e^T 0][p; mu] = [0; 1] solved by scipy.linalg.solve.  A swapped
+    orientation (r_st <-> r_ts), a different clamp or a wrong Q entry fails here."""
+    from scipy.linalg import solve
+
+    n = None if name == "blobs" else 1300
+    spec, X, y, Xt, yt = datagen.make_config(name, n_train=n, n_test=None if name == "blobs" else 60)
+    m = oracle.train(X, y, spec.k, C, gamma, 1e-6)
+    dec, prob = oracle.predict(m, X, y, Xt)
+    k, pairs = spec.k, m["pairs"]
+    X64, Xt64 = X.astype(np.float64), Xt.astype(np.float64)
+    dec_np = np.zeros((len(Xt), len(pairs)))
+    for p, (s, t) in enumerate(pairs):
+        idx, ypm = oracle.pair_members(y, k, s, t)
+        Kt = np.exp(-gamma * ((Xt64[:, None, :] - X64[idx][None, :, :]) ** 2).sum(-1))
+        dec_np[:, p] = Kt @ (m["alpha"][p] * ypm) + m["b"][p]
+    np.testing.assert_allclose(dec, dec_np, rtol=1e-10, atol=1e-10)
+    clamped = 0
+    for i in range(len(Xt)):
+        r = np.zeros((k, k))
+        for p, (s, t) in enumerate(pairs):
+            rst = 1.0 / (1.0 + np.exp(m["A"][p] * dec_np[i, p] + m["B"][p]))
+            clamped += int(rst < 1e-7 or rst > 1 - 1e-7)
+            rst = min(max(rst, 1e-7), 1 - 1e-7)
+            r[s, t], r[t, s] = rst, 1.0 - rst
+        Q = np.zeros((k, k))
+        for s in range(k):
+            for t in range(k):
+                Q[s, t] = sum(r[u, s] ** 2 for u in range(k) if u != s) if s == t else -r[t, s] * r[s, t]
+        M = np.zeros((k + 1, k + 1))
+        M[:k, :k], M[:k, k], M[k, :k] = Q, 1.0, 1.0
+        rhs = np.zeros(k + 1)
+        rhs[k] = 1.0
+        p_np = solve(M, rhs)[:k]
+        np.testing.assert_allclose(prob[i], p_np, atol=1e-12)
+    if name == "blobs" and C == 1.0:
+        # the argmax of p agrees with the pair votes' winner for confidently classified rows
+        votes = np.zeros((len(Xt), k))
+        for p, (s, t) in enumerate(pairs):
+            votes[:, s] += dec_np[:, p] > 0
+            votes[:, t] += dec_np[:, p] <= 0
+        sure = np.sort(prob, 1)[:, -1] > 0.9
+        assert np.all(prob.argmax(1)[sure] == votes.argmax(1)[sure])
