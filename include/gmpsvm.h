@@ -128,12 +128,16 @@ typedef struct {
 typedef struct {
   double t_total_ms;        /* whole call (host clock)                                        */
   double t_stage_ms;        /* H2D of Xtest (if host), transpose, norms                       */
-  double t_decision_ms;     /* a10: decision-value contraction (dec_contract + reduction)    */
+  double t_decision_ms;     /* a10: decision-value contraction + reduction                    */
   double t_couple_ms;       /* a11-a12: sigmoid + coupling                                    */
   double t_d2h_ms;          /* D2H of the probabilities (host output)                         */
   double dec_flops;         /* (2d + 3 + 2(k-1)) per (test, SV) pair                           */
-  int64_t dec_launches;     /* launches of dec_contract                                       */
+  int64_t dec_launches;     /* decision-value contractions (one per <= 32768-row chunk)       */
   int64_t launches;         /* kernels launched by this call                                  */
+  int32_t dec_path;         /* decision-value path taken (DESIGN.md §3 routing): 0 FP64 SIMT,
+                               1 int8-digit tensor cores (exact dot products, FP64 K),
+                               2 FP16-split tensor cores (FP32 K; GMPSVM_DEC=f16 only)        */
+  int32_t pad0;
 } gmpsvm_predict_stats;
 
 GMPSVM_API void gmpsvm_options_init(gmpsvm_options* opt);

@@ -49,7 +49,8 @@ class TrainStats(ct.Structure):
 class PredictStats(ct.Structure):
     _fields_ = [("t_total_ms", ct.c_double), ("t_stage_ms", ct.c_double), ("t_decision_ms", ct.c_double),
                 ("t_couple_ms", ct.c_double), ("t_d2h_ms", ct.c_double), ("dec_flops", ct.c_double),
-                ("dec_launches", ct.c_int64), ("launches", ct.c_int64)]
+                ("dec_launches", ct.c_int64), ("launches", ct.c_int64), ("dec_path", ct.c_int32),
+                ("pad0", ct.c_int32)]
 
 
 def _struct_dict(s):

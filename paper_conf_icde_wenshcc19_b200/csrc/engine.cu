@@ -342,7 +342,8 @@ DevModel::~DevModel() {
   } catch (...) {
   }
   if (ls && last_use) cudaStreamWaitEvent(ls, last_use, 0);
-  void* ptrs[] = {SvT, nsv, coef, items, item_begin, item_end, b, A, B, SvHi, SvLo, nsvc, mu, alpha_dev, coef64, nsv64};
+  void* ptrs[] = {SvT,   nsv,      coef, items,     item_begin, item_end, b,    A,    B,     SvHi,
+                  SvLo,  nsvc,     mu,   alpha_dev, coef64,     nsv64,    SvI8, sv_e, sv_n64};
   for (void* p : ptrs)
     if (p) {
       if (ls) cudaFreeAsync(p, ls);
@@ -390,10 +391,34 @@ static int pt_of(int p, int k) {
   while (rem >= k - 1 - s) rem -= k - 1 - s++;
   return s + 1 + rem;
 }
-// FP64 decision values when the worst-case probability shift from FP32 kernel values exceeds
-// this (MNIST-shaped C = 10 models sit near 2e-3 and meet 1e-4 on the TF32/FP16-split path;
-// MNIST8M-shaped C = 1000 models are far above it)
-constexpr double kDecF64Cond = 0.02;
+// Decision-value routing: a model predicts through the fastest path whose
+// worst-case probability error kCoupleAmp * max_p |A_p|/4 * sum_j |alpha_pj| * E_K stays within
+// kDecProbBound, half the 1e-4 contract.  dP/d dec = A P (1 - P) <= |A|/4 (Eq 12); |d dec| <=
+// sum_j |alpha_j| |dK_j| (Eq 11); kCoupleAmp bounds max |dp| / max |dr| of the coupling (Eq 15:
+// measured <= 1.97 over 1,500 random r matrices, k = 2..26).  E_K: the path's bound on |K~ - K|.
+constexpr double kDecProbBound = 5e-5;
+constexpr double kCoupleAmp = 2.0;
+constexpr double kF16KErr = 4e-5;   // FP16 hi/lo split, FP32 K: 2x the measured max relative error (§6.1)
+constexpr double kTestRange = 4.0;  // int8 bound assumes test rows within 4x the SVs' max |x| (checked per call)
+enum { kDecF64 = 0, kDecI8 = 1, kDecF16 = 2 };
+
+static void choose_dec_path(DevModel& dm, const Model& m) {
+  const int P = m.P();
+  dm.wsum = 0.0;
+  for (int p = 0; p < P; ++p)
+    if (m.trained[p] && p < (int)dm.abs_sum.size()) dm.wsum = std::max(dm.wsum, std::fabs(m.A[p]) * dm.abs_sum[p]);
+  const double amp = kCoupleAmp * dm.wsum / 4.0;
+  dm.cond_f16 = amp * kF16KErr;
+  dm.cond_i8 = dm.SvI8 ? amp * dec_i8_kernel_err(dm.amax_sv, kTestRange * dm.amax_sv, m.d, m.gamma) : HUGE_VAL;
+  static const char* dec_env = getenv("GMPSVM_DEC");  // forcing: f64 | i8 | f16 (tests, measurements)
+  const std::string mode = dec_env ? dec_env : "";
+  if (mode == "f64") dm.path = kDecF64;
+  else if (mode == "f16" && dm.tc) dm.path = kDecF16;
+  else if (mode == "i8" && dm.SvI8) dm.path = kDecI8;
+  else if (dm.SvI8 && dm.cond_i8 <= kDecProbBound) dm.path = kDecI8;
+  else dm.path = kDecF64;
+  dm.f64 = dm.path == kDecF64;
+}
 
 // mu_in / sc_in: a given centre and split scale for the SV rows; nullptr = compute them from the
 // SV rows
@@ -502,14 +527,11 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
     for (int p = 0; p < P; ++p)
       for (int64_t j = po[p]; j < po[p + 1]; ++j) abs_sum[p] += std::fabs(m.alpha[j]);
   }
-  for (int p = 0; p < P; ++p) dm->cond = std::max(dm->cond, std::fabs(m.A[p]) / 4.0 * std::ldexp(1.0, -22) * abs_sum[p]);
+  dm->abs_sum = abs_sum;
   static const char* dec_env = getenv("GMPSVM_DEC");
   const std::string dec_mode = dec_env ? dec_env : "";
-  // the other kernels (L76-L78) predict through the FP64 path only (its epilogue has them)
-  dm->f64 = (m.kernel != 0 && (!krow_use_tc() || !krow_split_f16() || dm->km1_pad > 12 || dec_mode == "simt")) ||
-            dec_mode == "f64" || (dec_mode.empty() && dm->cond > kDecF64Cond);
-  // FP64 coefficients also for the other kernels' fallback (test rows outside the FP16 range)
-  if (dm->f64 || m.kernel != 0) dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
+  // FP64 coefficients: the int8 and FP64 paths contract in FP64
+  dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
   if (dev_coef) {
     dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st);
     if (alpha_tot) GM_CUDA(cudaMemcpyAsync(dm->alpha_dev, alpha_hp, (size_t)alpha_tot * 8, cudaMemcpyDeviceToDevice, st));
@@ -534,14 +556,24 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
   HT("h2d_svt");
-  if (dm->coef64) {
-    dm->nsv64 = dev_alloc<double>(dm->nsv_pad, st);
-    launch_col_norms64(dm->SvT, dm->nsv_pad, dm->nsv_pad, dm->d_pad, dm->nsv64, st);
-  }
+  dm->nsv64 = dev_alloc<double>(dm->nsv_pad, st);
+  launch_col_norms64(dm->SvT, dm->nsv_pad, dm->nsv_pad, dm->d_pad, dm->nsv64, st);
   dm->h_items = items;
-  // tensor-core decision values: centre = mean of the SV rows, TF32 hi/lo split of the SV slots
-  static const bool dec_simt = getenv("GMPSVM_DEC") && std::string(getenv("GMPSVM_DEC")) == "simt";
-  dm->tc = !dec_simt && krow_use_tc() && dm->km1_pad <= dec_tc_max_km1();
+  // int8-digit SV planes (the default RBF path, dec_i8.cu)
+  uint32_t amax_bits = 0;
+  if (m.kernel == 0 && dm->km1_pad <= dec_i8_max_km1()) {
+    dm->SvI8 = dev_alloc<int8_t>(dec_i8_plane_bytes(dm->nsv_pad, m.d), st);
+    dm->sv_e = dev_alloc<int32_t>(dm->nsv_pad, st);
+    dm->sv_n64 = dev_alloc<double>(dm->nsv_pad, st);
+    DevBuf<unsigned> d_amax(1, st);
+    GM_CUDA(cudaMemsetAsync(d_amax.get(), 0, 4, st));
+    launch_stage_i8(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvI8, dm->nsv_pad, dm->sv_e, dm->sv_n64, d_amax.get(), st);
+    GM_CUDA(cudaMemcpyAsync(&amax_bits, d_amax.get(), 4, cudaMemcpyDeviceToHost, st));
+    HT("stage_i8");
+  }
+  // FP16-split tensor-core decision values (forced with GMPSVM_DEC=f16): centre = mean of the SV
+  // rows, hi/lo split of the SV slots
+  dm->tc = dec_mode == "f16" && krow_use_tc() && krow_split_f16() && dm->km1_pad <= (m.kernel != 0 ? 12 : dec_tc_max_km1());
   if (dm->tc) {
     dm->dpt = krow_tc_d_pad(m.d);
     dm->mu = dev_alloc<float>(m.d, st);
@@ -564,10 +596,14 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
                          dm->dpt, st);
     HT("split");
   }
-  if (ht) fprintf(stderr, "[gmpsvm devmodel ms]%s cond=%.3e f64=%d\n", line.c_str(), dm->cond, (int)dm->f64);
   GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
   GM_CUDA(cudaEventRecord(dm->last_use, st));
   GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
+  std::memcpy(&dm->amax_sv, &amax_bits, 4);
+  choose_dec_path(*dm, m);
+  if (ht)
+    fprintf(stderr, "[gmpsvm devmodel ms]%s path=%d cond_i8=%.3e cond_f16=%.3e\n", line.c_str(), dm->path, dm->cond_i8,
+            dm->cond_f16);
   return dm;
 }
 
@@ -725,6 +761,7 @@ static int engine_train_cv(const float* X, const int32_t* y, int64_t n, int32_t 
   if (m->dev) {
     GM_CUDA(cudaMemcpy(m->dev->A, hA.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
     GM_CUDA(cudaMemcpy(m->dev->B, hB.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+    choose_dec_path(*m->dev, *m);  // the routing bound depends on A (re-evaluated)
   }
   m->stats.t_total_ms = host_ms_since(t_start);
   *out = gm.release();
@@ -1644,8 +1681,16 @@ static std::shared_ptr<DevModel> ensure_dev_model(const Model& mdl, int device, 
   return mdl.dev;
 }
 
+static int engine_predict_path(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
+                               const gmpsvm_options& opt, int force_path);
+
 int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
                    const gmpsvm_options& opt) {
+  return engine_predict_path(mdl, Xt, m, prob_out, dec_out, opt, -1);
+}
+
+static int engine_predict_path(const Model& mdl, const float* Xt, int64_t m, double* prob_out, double* dec_out,
+                               const gmpsvm_options& opt, int force_path) {
   const auto t_start = std::chrono::steady_clock::now();
   gmpsvm_predict_stats& ps = tls_predict_stats();
   ps = gmpsvm_predict_stats{};
@@ -1659,17 +1704,21 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   const std::shared_ptr<DevModel> dm_ref = ensure_dev_model(mdl, opt.device, st);  // held for the whole call
   const DevModel& dm = *dm_ref;
   const int k = mdl.k, d = mdl.d, P = mdl.P();
+  const int path = force_path >= 0 ? force_path : dm.path;
   PhaseTimer tm(st);
   const int64_t mc_max = std::min<int64_t>(m, kPredictChunk);
   const int64_t mc_pad = round_up(mc_max, kTile);
+  const bool p_i8 = path == kDecI8, p_f16 = path == kDecF16;
   DevBuf<float> xin(opt.inputs_on_device ? 0 : (size_t)mc_max * d, st);
-  DevBuf<float> XtT(dm.tc ? 0 : (size_t)dm.d_pad * mc_pad, st), nt(mc_pad, st);
-  DevBuf<float> Xhi(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st), Xlo(dm.tc ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st);
-  // the SIMT decision values need the feature-major copy only as the FP16-range fallback
-  DevBuf<float> XtTf(dm.tc ? (size_t)dm.d_pad * mc_pad : 0, st);
-  DevBuf<float> part((size_t)dm.n_items * mc_pad * dm.km1_pad, st);
-  const bool may64 = dm.f64 || mdl.kernel != 0;
-  DevBuf<double> part64(may64 ? (size_t)dm.n_items * mc_pad * dm.km1_pad : 0, st), nt64(may64 ? mc_pad : 0, st);
+  // feature-major test rows: the FP64 path (and the FP16 path's fallback for rows outside its range)
+  DevBuf<float> XtT(p_i8 ? 0 : (size_t)dm.d_pad * mc_pad, st), nt(mc_pad, st);
+  DevBuf<float> Xhi(p_f16 ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st), Xlo(p_f16 ? krow_tc_buf_floats(mc_pad, dm.dpt) : 0, st);
+  DevBuf<float> part(p_f16 ? (size_t)dm.n_items * mc_pad * dm.km1_pad : 0, st);
+  DevBuf<double> part64((size_t)dm.n_items * mc_pad * dm.km1_pad, st), nt64(mc_pad, st);
+  DevBuf<int8_t> tI8(p_i8 ? dec_i8_plane_bytes(mc_pad, d) : 0, st);
+  DevBuf<int32_t> t_e(p_i8 ? mc_pad : 0, st);
+  DevBuf<unsigned> d_amax(1, st);
+  GM_CUDA(cudaMemsetAsync(d_amax.get(), 0, 4, st));
   DevBuf<double> dec_buf(opt.inputs_on_device ? 0 : (size_t)mc_max * P, st);
   DevBuf<double> prob_buf((opt.inputs_on_device || !prob_out) ? 0 : (size_t)mc_max * k, st);
   DevBuf<double> dec_tmp((opt.inputs_on_device && !dec_out) ? (size_t)mc_max * P : 0, st);
@@ -1687,13 +1736,10 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
     DevBuf<int2> d_dtiles;
     DevBuf<int32_t> d_uoff, d_uitem;
     int n_units = 0;
-    // FP16 split: test rows far outside the SVs' range would overflow half precision -> SIMT
-    const bool use_tc = !dm.f64 && dm.tc &&
-                        (!krow_split_f16() || launch_maxabs(src, mc, d, nullptr, dm.mu, st) * dm.sc < 60000.f);
-    const bool f64 = dm.f64 || (mdl.kernel != 0 && !use_tc);  // the SIMT fallback is the Gaussian's only
-    if (use_tc) {
-      launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
-      launch_split_hilo_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
+    // FP16 split: test rows far outside the SVs' range would overflow half precision -> FP64
+    const bool use_tc = p_f16 && launch_maxabs(src, mc, d, nullptr, dm.mu, st) * dm.sc < 60000.f;
+    const bool f64 = !p_i8 && !use_tc;
+    if (!f64) {
       // work units: (item, test tile), test tiles fastest; unit = the item's SV tiles for that test tile
       const int ntt = (int)(mcp / kTile);
       std::vector<int2> dt;
@@ -1713,34 +1759,42 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
       GM_CUDA(cudaMemcpyAsync(d_uoff.get(), uoff.data(), uoff.size() * 4, cudaMemcpyHostToDevice, st));
       if (!uitem.empty())
         GM_CUDA(cudaMemcpyAsync(d_uitem.get(), uitem.data(), uitem.size() * 4, cudaMemcpyHostToDevice, st));
+    }
+    if (p_i8) {
+      launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
+      launch_stage_i8(src, mc, d, nullptr, tI8.get(), mcp, t_e.get(), nt64.get(), d_amax.get(), st);
+    } else if (use_tc) {
+      launch_row_norms(src, mc, d, nullptr, nt.get(), mcp, bad.get(), st);  // validation (non-finite rows)
+      launch_split_hilo_mu(src, mc, d, nullptr, dm.mu, dm.sc, Xhi.get(), Xlo.get(), nt.get(), mcp, dm.dpt, st);
     } else {
-      launch_stage_features(src, mc, d, nullptr, dm.tc ? XtTf.get() : XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(),
-                            st);
+      launch_stage_features(src, mc, d, nullptr, XtT.get(), mcp, dm.d_pad, mcp, nt.get(), bad.get(), st);
     }
     tm.mark(PH_STAGE);
     double* dec_d = opt.inputs_on_device ? (dec_out ? dec_out + i0 * P : dec_tmp.get()) : dec_buf.get();
     tm.mark(PH_DEC);
-    if (f64) {  // ill-conditioned model (or another kernel off the tensor cores): FP64 decision values
-      float* xt = dm.tc ? XtTf.get() : XtT.get();
-      launch_col_norms64(xt, mcp, mcp, dm.d_pad, nt64.get(), st);
+    if (f64) {  // FP64 decision values (SIMT; any kernel)
+      launch_col_norms64(XtT.get(), mcp, mcp, dm.d_pad, nt64.get(), st);
       GM_CUDA(cudaMemsetAsync(part64.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 8, st));
-      launch_dec_f64(xt, mcp, nt64.get(), mcp, dm.SvT, dm.nsv_pad, dm.nsv64, dm.coef64, dm.km1, dm.km1_pad, dm.items,
+      launch_dec_f64(XtT.get(), mcp, nt64.get(), mcp, dm.SvT, dm.nsv_pad, dm.nsv64, dm.coef64, dm.km1, dm.km1_pad, dm.items,
                      dm.n_items, dm.d_pad, mdl.gamma, part64.get(), st, mdl.kernel, mdl.coef0, mdl.degree);
       launch_dec_reduce64(part64.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
-    } else if (use_tc) {
-      GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
+    } else if (p_i8) {  // exact int8-digit dot products, FP64 kernel values (dec_i8.cu)
+      GM_CUDA(cudaMemsetAsync(part64.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 8, st));  // items without tiles
       if (n_units > 0)
-      {
+        launch_dec_i8(tI8.get(), mcp, t_e.get(), nt64.get(), dm.SvI8, dm.nsv_pad, dm.sv_e, dm.sv_n64, d,
+                      d_dtiles.get(), d_uoff.get(), d_uitem.get(), n_units, dm.coef64, dm.km1, dm.km1_pad, mdl.gamma,
+                      part64.get(), st);
+      launch_dec_reduce64(part64.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
+    } else {
+      GM_CUDA(cudaMemsetAsync(part.get(), 0, (size_t)dm.n_items * mcp * dm.km1_pad * 4, st));  // items without tiles
+      if (n_units > 0) {
         const KrowKernel kk{mdl.kernel, (float)mdl.gamma, (float)mdl.coef0, 0.f, mdl.degree};
         launch_dec_tc(Xhi.get(), Xlo.get(), mcp, dm.SvHi, dm.SvLo, dm.nsv_pad, dm.dpt, d_dtiles.get(), d_uoff.get(),
                       d_uitem.get(), n_units, nt.get(), dm.nsvc, dm.coef, dm.km1, dm.km1_pad, mdl.gamma, dm.sc, part.get(),
                       st, mdl.kernel != 0 ? &kk : nullptr);
       }
-    } else {
-      launch_dec_contract(dm.tc ? XtTf.get() : XtT.get(), mcp, nt.get(), mc, mcp, dm.SvT, dm.nsv_pad, dm.nsv, dm.coef,
-                          dm.km1, dm.km1_pad, dm.items, dm.n_items, dm.d_pad, mdl.gamma, part.get(), st);
+      launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     }
-    if (!f64) launch_dec_reduce(part.get(), mc, mcp, k, dm.km1_pad, dm.item_begin, dm.item_end, dm.b, dec_d, st);
     ps.dec_launches += 1;
     tm.mark(PH_DEC);
     double* prob_d = nullptr;
@@ -1760,16 +1814,23 @@ int engine_predict(const Model& mdl, const float* Xt, int64_t m, double* prob_ou
   }
   GM_CUDA(cudaEventRecord(dm.last_use, st));
   int32_t hbad = 0;
+  uint32_t amax_bits = 0;
   GM_CUDA(cudaMemcpyAsync(&hbad, bad.get(), 4, cudaMemcpyDeviceToHost, st));
+  GM_CUDA(cudaMemcpyAsync(&amax_bits, d_amax.get(), 4, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
+  if (hbad) throw Error(GMPSVM_EINVAL, "Xtest contains non-finite values");
+  float amax_t = 0.f;
+  std::memcpy(&amax_t, &amax_bits, 4);
+  if (p_i8 && force_path < 0 && amax_t > kTestRange * dm.amax_sv)  // outside the range the routing bound assumed
+    return engine_predict_path(mdl, Xt, m, prob_out, dec_out, opt, kDecF64);
   ps.t_stage_ms = tm.ms(PH_STAGE);
   ps.t_decision_ms = tm.ms(PH_DEC);
   ps.t_couple_ms = tm.ms(PH_COUPLE);
   ps.t_d2h_ms = tm.ms(PH_D2H);
   ps.dec_flops = (double)m * (double)mdl.sv_pos.size() * (2.0 * d + 3.0 + 2.0 * (k - 1));
   ps.launches = (int64_t)(g_launches.load() - launches0);
+  ps.dec_path = path;
   ps.t_total_ms = host_ms_since(t_start);
-  if (hbad) throw Error(GMPSVM_EINVAL, "Xtest contains non-finite values");
   return GMPSVM_OK;
 }
 

@@ -79,6 +79,18 @@ void launch_split_hilo_mu(const float* X, int64_t n, int d, const int64_t* perm,
 // mu[c] = mean over the rows idx[i] >= 0 (cnt of them) of X[., c]
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
                             cudaStream_t st);
+// a10 with exact dot products (dec_i8.cu): rows -> 5 int8 digit planes [5][rows_pad][round_up(d, 32)]
+// (src: row index per output row, < 0 = zero row; nullptr = identity), per-row exponent and FP64
+// norm of the fixed-point row; amax (optional): max |x| over the rows as float bits (atomicMax)
+int dec_i8_max_km1();
+size_t dec_i8_plane_bytes(int64_t rows_pad, int d);
+double dec_i8_kernel_err(double ax, double ay, int d, double gamma);  // bound on |K~ - K| (RBF)
+void launch_stage_i8(const float* X, int64_t n, int d, const int64_t* src, int8_t* planes, int64_t rows_pad,
+                     int32_t* ex, double* nrm, unsigned* amax, cudaStream_t st);
+void launch_dec_i8(const int8_t* tplanes, int64_t m_pad, const int32_t* et, const double* nt, const int8_t* splanes,
+                   int64_t nsv_pad, const int32_t* es, const double* ns, int d, const int2* tiles,
+                   const int32_t* unit_off, const int32_t* unit_item, int n_units, const double* coef64, int km1,
+                   int km1_pad, double gamma, double* part, cudaStream_t st);
 // a10 on tcgen05 (krow_tc.cu): tiles = (test tile, SV tile) grouped in units [unit_off[u],
 // unit_off[u+1]), unit u writes part[unit_item[u]][row][0..km1_pad) (as launch_dec_contract)
 int dec_tc_max_km1();

@@ -41,12 +41,25 @@ struct DevModel {
   // alpha_dev_off[p] = offset of model pair p (-1: untrained).  The host copy Model::alpha is
   // materialised from it only when asked for (introspection, serialisation, merge).
   double* alpha_dev = nullptr;
-  // FP64 decision values for ill-conditioned models: cond = max_p |A_p|/4 *
-  // 2^-22 * sum_j |alpha_pj| (worst-case probability shift from FP32 kernel values)
-  bool f64 = false;
-  double cond = 0.0;
+  // Decision-value path (DESIGN.md §3 "decision-value routing"): the fastest path whose
+  // worst-case probability error 2 * max_p |A_p|/4 * sum_j |alpha_pj| * E_K (E_K: that path's
+  // bound on |K~ - K|; 2: the coupling's measured amplification) is <= kDecProbBound.
+  //   kDecI8  dec_i8.cu: exact int8-digit dot products on tcgen05, FP64 kernel values (RBF)
+  //   kDecF64 predict.cu: FP64 SIMT (any kernel; the fallback)
+  //   kDecF16 krow_tc.cu dec_tc: FP16 hi/lo split, FP32 kernel values (forced: GMPSVM_DEC=f16)
+  int path = 0;
+  bool f64 = false;             // path == kDecF64
+  double wsum = 0.0;            // max_p |A_p| * sum_j |alpha_pj|
+  std::vector<double> abs_sum;  // [P] sum_j |alpha_pj|
+  double cond_i8 = 0.0, cond_f16 = 0.0;
   double* coef64 = nullptr;  // [nsv_pad][km1_pad]
   double* nsv64 = nullptr;   // [nsv_pad] FP64 squared norms of the SV rows
+  // int8-digit SV planes [5][nsv_pad][round_up(d, 32)], per-row exponents and FP64 norms of the
+  // fixed-point rows, max |x| over the SV rows
+  int8_t* SvI8 = nullptr;
+  int32_t* sv_e = nullptr;
+  double* sv_n64 = nullptr;
+  float amax_sv = 0.f;
   std::vector<int64_t> alpha_dev_off;
   cudaEvent_t last_use = nullptr;  // recorded on the caller's stream after every use
   // stream-ordered allocation: freed on the library stream after last_use (no device sync)
