@@ -31,6 +31,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
 #include <string>
 
 #include "kernels.h"
@@ -48,18 +49,21 @@ constexpr uint32_t kIAPlane = kIM * kIK;  // 8 KB
 constexpr uint32_t kIBPlane = kIN * kIK;  // 4 KB
 constexpr uint32_t kIStageBytes = kND * (kIAPlane + kIBPlane);  // 60 KB
 constexpr uint32_t kITmemCols = 512;      // 6 x 64 used (power-of-two allocation)
-constexpr int kIThreads = 192;
+constexpr int kIThreads = 320;  // producer, MMA issuer, 8 epilogue warps
 constexpr int kIExp = 37;                 // max |x| 2^e in [2^37, 2^38)
 // kind::i8, D S32 (2), A S8 (1), B S8 (1), K-major, N = 64, M = 128
 constexpr uint32_t kIdescI8 =
     (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(kIN >> 3) << 17) | ((uint32_t)(kIM >> 4) << 24);
 
 template <int KM>
+constexpr int i8_stages() { return KM > 12 ? 2 : kIStages; }  // large k: the coefficient tiles need the room
+template <int KM>
 struct DecI8Smem {
-  alignas(1024) uint8_t stage[kIStages][kIStageBytes];
+  alignas(1024) uint8_t stage[i8_stages<KM>()][kIStageBytes];
   alignas(16) double coefS[2][kIN][KM];
-  alignas(8) uint64_t full[kIStages];
-  uint64_t empty[kIStages];
+  double red[kIM][KM];  // column-half reduction of the per-row sums
+  alignas(8) uint64_t full[i8_stages<KM>()];
+  uint64_t empty[i8_stages<KM>()];
   uint64_t tmem_full;
   uint64_t tmem_empty;
   uint32_t tmem_base;
@@ -76,13 +80,57 @@ __device__ __forceinline__ uint64_t umma_desc_sw64(const void* p) {
   d |= (uint64_t)4 << 61;  // SWIZZLE_64B
   return d;
 }
+// collector: 0 none, 1 fill (keep A for the next MMA), 2 use (reuse and keep), 3 lastuse
+template <int COL>
 __device__ __forceinline__ void umma_i8(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
-  asm volatile(
-      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n}\n" ::"r"(
-          tmem_d),
-      "l"(a), "l"(b), "r"(kIdescI8), "r"(accum));
+  if (COL == 1)
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::i8.collector::a::fill [%0], %1, %2, %3, "
+        "p;\n}\n" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(kIdescI8), "r"(accum));
+  else if (COL == 2)
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::i8.collector::a::use [%0], %1, %2, %3, "
+        "p;\n}\n" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(kIdescI8), "r"(accum));
+  else if (COL == 3)
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::i8.collector::a::lastuse [%0], %1, %2, "
+        "%3, p;\n}\n" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(kIdescI8), "r"(accum));
+  else
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n}\n" ::"r"(
+            tmem_d),
+        "l"(a), "l"(b), "r"(kIdescI8), "r"(accum));
 }
 __device__ __forceinline__ double pow2(int k) { return __hiloint2double((k + 1023) << 20, 0); }  // 2^k, |k| < 1023
+
+// 2^t for t <= 0 in FP64: t = n + f, n = rint(t), |f| <= 1/2; 2^f by its Taylor series in
+// f ln 2 to degree 10 (remainder <= (ln2 / 2)^11 / 11! e^(ln2 / 2) < 3.2e-13 relative) evaluated by
+// Horner in FP64; 2^n exactly.  Below 2^-1020 the result is 0 (absolute error < 1e-307).
+__device__ __forceinline__ double exp2_neg(double t) {
+  if (t < -1020.0) return 0.0;
+  const double n = rint(t);
+  const double f = t - n;  // exact
+  // c_k = ln(2)^k / k!, k = 10 .. 0
+  constexpr double c[11] = {
+    7.054911620801123e-09,
+    1.01780860092397e-07,
+    1.321548679014431e-06,
+    1.5252733804059841e-05,
+    0.0001540353039338161,
+    0.0013333558146428443,
+    0.009618129107628477,
+    0.05550410866482158,
+    0.24022650695910072,
+    0.6931471805599453,
+    1.0};
+  double p = c[0];
+#pragma unroll
+  for (int k = 1; k < 11; ++k) p = fma(p, f, c[k]);
+  return p * pow2((int)n);
+}
 
 // rows [0, n_pad) of X (row src[j], or j; < 0 / >= n: zero row) -> planes[p][j][0..d8), e[j], nrm[j];
 // amax_out (optional): max over the rows of max |x| as float bits (atomicMax, non-negative floats)
@@ -122,26 +170,27 @@ __global__ void stage_i8_kernel(const float* __restrict__ X, int64_t n, int d, c
   }
 }
 
-template <int KM>
+template <int KM, bool COLLECT>
 __global__ void __launch_bounds__(kIThreads, 1)
     dec_i8_kernel(const __grid_constant__ CUtensorMap map_t, const __grid_constant__ CUtensorMap map_s,
                   const int2* __restrict__ tiles, const int32_t* __restrict__ unit_off,
                   const int32_t* __restrict__ unit_item, int n_units, const int32_t* __restrict__ et,
                   const double* __restrict__ nt, const int32_t* __restrict__ es, const double* __restrict__ ns,
                   const double* __restrict__ coef, int km1, int km1_pad, int d8, int64_t m_pad, int64_t nsv_pad,
-                  double gamma, double* __restrict__ part) {
+                  double gamma, double* __restrict__ part, int diag) {
   extern __shared__ __align__(1024) uint8_t dsmem[];
   DecI8Smem<KM>& sm =
       *reinterpret_cast<DecI8Smem<KM>*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  constexpr int NS = i8_stages<KM>();
   const int nk = (d8 + kIK - 1) / kIK;
   if (warp == 0 && lane == 0) {
-    for (int s = 0; s < kIStages; ++s) {
+    for (int s = 0; s < NS; ++s) {
       mbar_init(&sm.full[s], 1);
       mbar_init(&sm.empty[s], 1);
     }
     mbar_init(&sm.tmem_full, 1);
-    mbar_init(&sm.tmem_empty, 4);
+    mbar_init(&sm.tmem_empty, 8);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_t)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_s)) : "memory");
@@ -167,9 +216,13 @@ __global__ void __launch_bounds__(kIThreads, 1)
           for (int h = 0; h < 2; ++h) {
             const int c0 = tile.y * 2 * kIN + h * kIN;
             for (int kb = 0; kb < nk; ++kb, ++g) {
-              const int s = g % kIStages;
-              if (g >= kIStages) mbar_wait(&sm.empty[s], ((g / kIStages) + 1) & 1);
+              const int s = g % NS;
+              if (g >= NS) mbar_wait(&sm.empty[s], ((g / NS) + 1) & 1);
               uint8_t* st = sm.stage[s];
+              if (diag & 4) {  // GMPSVM_I8_DIAG bit 2 (timing experiments): no operand loads
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.full[s])) : "memory");
+                continue;
+              }
               mbar_expect_tx(&sm.full[s], kIStageBytes);
 #pragma unroll
               for (int p = 0; p < kND; ++p) {
@@ -190,22 +243,29 @@ __global__ void __launch_bounds__(kIThreads, 1)
             if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             for (int kb = 0; kb < nk; ++kb, ++g) {
-              const int s = g % kIStages;
-              mbar_wait(&sm.full[s], (g / kIStages) & 1);
+              const int s = g % NS;
+              mbar_wait(&sm.full[s], (g / NS) & 1);
               asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
               uint8_t* st = sm.stage[s];
-              const int nsub = min(2, (d8 - kb * kIK + 31) / 32);  // valid 32-wide k steps (d8 % 32 == 0)
+              const int nsub = (diag & 2) ? 0 : min(2, (d8 - kb * kIK + 31) / 32);  // valid 32-wide k steps
               for (int kk = 0; kk < nsub; ++kk) {
                 const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+                // A plane i stays in the tensor core's collector across its products with every B
+                // plane j (i + j <= 5): the A operand is read from shared memory once per (i, kk)
 #pragma unroll
-                for (int gg = 0; gg < kNG; ++gg) {
+                for (int i = 0; i < kND; ++i) {
+                  const uint64_t ad = umma_desc_sw64(st + i * kIAPlane) + adv;
+                  const int jn = min(kND, kNG - i);  // j = 0 .. jn - 1
 #pragma unroll
-                  for (int i = 0; i < kND; ++i) {
-                    const int j = gg - i;
-                    if (j < 0 || j >= kND) continue;
+                  for (int j = 0; j < jn; ++j) {
+                    const int gg = i + j;
                     const bool first = kb == 0 && kk == 0 && i == (gg < kND ? 0 : gg - kND + 1);
-                    umma_i8(tmem + gg * kIN, umma_desc_sw64(st + i * kIAPlane) + adv,
-                            umma_desc_sw64(st + kND * kIAPlane + j * kIBPlane) + adv, first ? 0u : 1u);
+                    const uint64_t bd = umma_desc_sw64(st + kND * kIAPlane + j * kIBPlane) + adv;
+                    const uint32_t acc = first ? 0u : 1u;
+                    if (!COLLECT) umma_i8<0>(tmem + gg * kIN, ad, bd, acc);
+                    else if (j == 0) umma_i8<1>(tmem + gg * kIN, ad, bd, acc);
+                    else if (j == jn - 1) umma_i8<3>(tmem + gg * kIN, ad, bd, acc);
+                    else umma_i8<2>(tmem + gg * kIN, ad, bd, acc);
                   }
                 }
               }
@@ -214,10 +274,11 @@ __global__ void __launch_bounds__(kIThreads, 1)
             umma_commit(&sm.tmem_full);
           }
     }
-  } else {  // ---- epilogue: warps 2..5 (TMEM lane quarter warp % 4), thread = one test row
-    const int q = warp & 3, et_id = threadIdx.x - 64;  // 0..127
+  } else {  // ---- epilogue: warps 2..9; TMEM lane quarter warp % 4, column half (warp - 2) / 4;
+            //      thread = one test row x 32 of the tile's 64 SVs
+    const int q = warp & 3, half = (warp - 2) >> 2, et_id = threadIdx.x - 64;  // et_id 0..255
     int it = 0;
-    const double ng = -gamma;
+    const double tsc = -gamma * 1.4426950408889634074;  // exp(-gamma d2) = 2^(tsc d2)
     for (int u = blockIdx.x; u < n_units; u += gridDim.x) {
       double acc[KM];
 #pragma unroll
@@ -231,50 +292,69 @@ __global__ void __launch_bounds__(kIThreads, 1)
         for (int h = 0; h < 2; ++h, ++it) {
           const int64_t c0 = (int64_t)tile.y * 2 * kIN + h * kIN;
           double* cs = &sm.coefS[it & 1][0][0];  // this half-tile's coefficients (double buffer)
-          for (int idx = et_id; idx < kIN * KM; idx += 128) {
+          for (int idx = et_id; idx < kIN * KM; idx += 256) {
             const int jj = idx / KM, v = idx - jj * KM;
-            cs[idx] = v < km1_pad ? coef[(c0 + jj) * km1_pad + v] : 0.0;
+            cs[idx] = v < km1 ? coef[(c0 + jj) * km1_pad + v] : 0.0;
           }
-          asm volatile("bar.sync 1, 128;" ::: "memory");
+          asm volatile("bar.sync 1, 256;" ::: "memory");
           mbar_wait(&sm.tmem_full, it & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          double dot[kIN];  // sum_g 256^(5-g) G_g (exact integers up to rounding in the last adds)
+          // sum_g 256^(5-g) G_g by 16-column chunks: groups 0-2 and 3-5 combined exactly in int64
+          // (|G| < 2^26: |hi|, |lo| < 2^43, exact in FP64), then hi 2^24 + lo in FP64
+          const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(half * 32);
+          double dot[32];
 #pragma unroll
-          for (int ch = 0; ch < kIN / 32; ++ch) {
-            const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(ch * 32);
+          for (int ch = 0; ch < 2; ++ch) {
 #pragma unroll
-            for (int gg = 0; gg < kNG; ++gg) {
-              uint32_t v[32];
-              tmem_ld32(taddr + gg * kIN, v);
-              asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-              const double w = pow2(8 * (kNG - 1 - gg));
+            for (int part3 = 0; part3 < 2; ++part3) {
+              long long w[16];
 #pragma unroll
-              for (int jj = 0; jj < 32; ++jj) {
-                const double gv = (double)(int32_t)v[jj];
-                dot[ch * 32 + jj] = gg == 0 ? gv * w : fma(gv, w, dot[ch * 32 + jj]);
+              for (int g3 = 0; g3 < 3; ++g3) {
+                uint32_t v[16];
+                tmem_ld16(taddr + (uint32_t)((part3 * 3 + g3) * kIN + ch * 16), v);
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+                for (int jj = 0; jj < 16; ++jj) w[jj] = (g3 == 0 ? 0ll : w[jj] * 256) + (int32_t)v[jj];
               }
+#pragma unroll
+              for (int jj = 0; jj < 16; ++jj)
+                dot[ch * 16 + jj] = part3 == 0 ? (double)w[jj] : fma(dot[ch * 16 + jj], 16777216.0, (double)w[jj]);
             }
           }
           asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
           __syncwarp();
           if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
-          // x~.y~ = 2^-(e_x+e_y) 256^3 dot: the 256^3 = 2^24 folds into the exponent
+          // x~.y~ = 2^-(e_x+e_y) 256^3 (hi 2^24 + lo): the 256^3 = 2^24 folds into the exponent
+          if (diag & 1) {  // GMPSVM_I8_DIAG bit 0 (timing experiments): no epilogue arithmetic
+            acc[0] += dot[0] + dot[31];
+            continue;
+          }
 #pragma unroll
-          for (int jj = 0; jj < kIN; ++jj) {
-            const int64_t c = c0 + jj;
+          for (int jj = 0; jj < 32; ++jj) {
+            const int64_t c = c0 + half * 32 + jj;
             const double xy = dot[jj] * pow2(24 - ex_r - __ldg(es + c));
-            const double d2 = fmax(nr + __ldg(ns + c) - 2.0 * xy, 0.0);
-            const double kv = exp(ng * d2);
-            const double* cj = cs + jj * KM;
+            const double d2 = fmax(fma(-2.0, xy, nr + __ldg(ns + c)), 0.0);
+            const double kv = exp2_neg(tsc * d2);
+            const double* cj = cs + (half * 32 + jj) * KM;
 #pragma unroll
             for (int v = 0; v < KM; ++v) acc[v] = fma(kv, cj[v], acc[v]);
           }
         }
       }
-      double* out = part + ((int64_t)unit_item[u] * m_pad + r) * km1_pad;
+      // the two column halves of a row: half 1 hands its sums to half 0 through shared memory
+      double* red = &sm.red[0][0];
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      if (half == 1)
 #pragma unroll
-      for (int v = 0; v < KM; ++v)
-        if (v < km1_pad) out[v] = v < km1 ? acc[v] : 0.0;
+        for (int v = 0; v < KM; ++v) red[(q * 32 + lane) * KM + v] = acc[v];
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      if (half == 0) {
+        double* out = part + ((int64_t)unit_item[u] * m_pad + r) * km1_pad;
+#pragma unroll
+        for (int v = 0; v < KM; ++v)
+          if (v < km1) out[v] = acc[v] + red[(q * 32 + lane) * KM + v];
+        for (int v = km1; v < km1_pad; ++v) out[v] = 0.0;
+      }
     }
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -311,14 +391,15 @@ int dec_i8_max_km1() { return 32; }
 // representation error Delta = ||dx|| + ||dy|| <= sqrt(d) 2^-38 (ax + ay) moves d2 by at most
 // 2 r Delta + Delta^2 (r = ||x - y||), and K e^(-gamma r^2) 2 gamma r Delta peaks at
 // Delta sqrt(2 gamma) e^(-1/2); the dropped digit groups add <= 2 (3 d 2^-44 ax ay), FP64 rounding
-// of the norm combine <= 2^-49 (||x||^2 + ||y||^2) <= 2^-49 d (ax^2 + ay^2), exp and the products
-// a few ulps.  (DESIGN.md §3 "decision-value routing".)
+// of the norm combine <= 2^-49 (||x||^2 + ||y||^2) <= 2^-49 d (ax^2 + ay^2), the exp series
+// remainder 3.2e-13 and rounding.  (DESIGN.md §3 "decision-value routing".)
 double dec_i8_kernel_err(double ax, double ay, int d, double gamma) {
   const double sd = std::sqrt((double)d);
   const double delta = sd * std::ldexp(1.0, -38) * (ax + ay);
   const double ed2 = delta * delta + 6.0 * d * std::ldexp(1.0, -44) * ax * ay +
                      std::ldexp(1.0, -49) * d * (ax * ax + ay * ay);
-  return delta * std::sqrt(2.0 * gamma) * std::exp(-0.5) + gamma * ed2 + std::ldexp(1.0, -48);
+  // + exp2_neg's series remainder (< 3.2e-13 relative, K <= 1) and rounding
+  return delta * std::sqrt(2.0 * gamma) * std::exp(-0.5) + gamma * ed2 + 5e-13;
 }
 
 void launch_stage_i8(const float* X, int64_t n, int d, const int64_t* src, int8_t* planes, int64_t rows_pad,
@@ -338,14 +419,21 @@ void launch_dec_i8(const int8_t* tplanes, int64_t m_pad, const int32_t* et, cons
   GM_CUDA(cudaGetDevice(&dev));
   GM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
   const int grid = n_units < sms ? n_units : sms;
+  static const int diag = getenv("GMPSVM_I8_DIAG") ? atoi(getenv("GMPSVM_I8_DIAG")) : 0;
   auto go = [&](auto kern, size_t smem) {
     set_max_dyn_smem(kern, smem);
     GM_LAUNCH(kern, dim3(grid), dim3(kIThreads), smem, st, mt, ms, tiles, unit_off, unit_item, n_units, et, nt, es, ns,
-              coef64, km1, km1_pad, d8, m_pad, nsv_pad, gamma, part);
+              coef64, km1, km1_pad, d8, m_pad, nsv_pad, gamma, part, diag);
   };
-  if (km1_pad <= 4) go(dec_i8_kernel<4>, sizeof(DecI8Smem<4>) + 1024);
-  else if (km1_pad <= 12) go(dec_i8_kernel<12>, sizeof(DecI8Smem<12>) + 1024);
-  else if (km1_pad <= 32) go(dec_i8_kernel<32>, sizeof(DecI8Smem<32>) + 1024);
+  // GMPSVM_I8_COLLECT=0: no A-operand collector reuse (measurement)
+  static const bool collect = !(getenv("GMPSVM_I8_COLLECT") && std::string(getenv("GMPSVM_I8_COLLECT")) == "0");
+  // KM: pair columns contracted per SV, the smallest instantiation >= k - 1
+  if (km1 <= 2) collect ? go(dec_i8_kernel<2, true>, sizeof(DecI8Smem<2>) + 1024) : go(dec_i8_kernel<2, false>, sizeof(DecI8Smem<2>) + 1024);
+  else if (km1 <= 4) collect ? go(dec_i8_kernel<4, true>, sizeof(DecI8Smem<4>) + 1024) : go(dec_i8_kernel<4, false>, sizeof(DecI8Smem<4>) + 1024);
+  else if (km1 <= 9) collect ? go(dec_i8_kernel<9, true>, sizeof(DecI8Smem<9>) + 1024) : go(dec_i8_kernel<9, false>, sizeof(DecI8Smem<9>) + 1024);
+  else if (km1 <= 12) collect ? go(dec_i8_kernel<12, true>, sizeof(DecI8Smem<12>) + 1024) : go(dec_i8_kernel<12, false>, sizeof(DecI8Smem<12>) + 1024);
+  else if (km1 <= 25) collect ? go(dec_i8_kernel<25, true>, sizeof(DecI8Smem<25>) + 1024) : go(dec_i8_kernel<25, false>, sizeof(DecI8Smem<25>) + 1024);
+  else if (km1 <= 32) collect ? go(dec_i8_kernel<32, true>, sizeof(DecI8Smem<32>) + 1024) : go(dec_i8_kernel<32, false>, sizeof(DecI8Smem<32>) + 1024);
   else throw Error(GMPSVM_ENOTIMPL, "int8 decision values support k <= 33");
 }
 

@@ -1,0 +1,87 @@
+// tcgen05.mma kind::i8 / kind::f16 issue-rate microbenchmark: one CTA per SM, one thread issues
+// `iters` MMAs (M = 128, N = 64 / 128 / 256) from shared memory into TMEM back to back; time per
+// MMA from clock64 around the loop + the final commit's mbarrier.
+#include <cstdint>
+#include <cstdio>
+#include <cuda_runtime.h>
+__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint64_t desc(const void* p, int sw) {  // sw: 2 = 128B, 4 = 64B
+  uint64_t d = (su32(p) >> 4) & 0x3FFF;
+  d |= 1ull << 16;
+  d |= (uint64_t)((sw == 2 ? 1024 : 512) >> 4) << 32;
+  d |= 1ull << 46;
+  d |= (uint64_t)sw << 61;
+  return d;
+}
+template <int KIND, int N>  // KIND 0: i8 (K = 32), 1: f16 (K = 16)
+__global__ void k(int iters, long long* out) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  __shared__ uint32_t tbase;
+  __shared__ __align__(8) uint64_t bar;
+  const int warp = threadIdx.x >> 5;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(&tbase)), "r"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (threadIdx.x == 32) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar)));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  if (threadIdx.x == 32) {
+    const uint32_t tm = tbase;
+    const int sw = 2;
+    const uint64_t a = desc(sm, sw), b = desc(sm + 32768, sw);
+    constexpr uint32_t idesc = KIND == 0 ? ((2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (8u << 24))
+                                         : ((1u << 4) | ((uint32_t)(N >> 3) << 17) | (8u << 24));
+    const long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+      const uint32_t d = tm + (uint32_t)((i & 1) * N) % 512;
+      if (KIND == 0)
+        asm volatile("{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+                     "l"(a + (uint64_t)((i & 3) * 2)), "l"(b + (uint64_t)((i & 3) * 2)), "r"(idesc), "r"(1));
+      else
+        asm volatile("{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+                     "l"(a + (uint64_t)((i & 3) * 2)), "l"(b + (uint64_t)((i & 3) * 2)), "r"(idesc), "r"(1));
+    }
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(&bar)) : "memory");
+    uint32_t done = 0;
+    do {
+      asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n selp.u32 %0, 1, 0, p;\n}\n"
+                   : "=r"(done) : "r"(su32(&bar)) : "memory");
+    } while (!done);
+    const long long t1 = clock64();
+    if (blockIdx.x == 0) out[0] = t1 - t0;
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 0) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase), "r"(512));
+  }
+}
+int main() {
+  long long* out;
+  cudaMalloc(&out, 8);
+  const int iters = 20000;
+  auto run = [&](const char* name, auto kern, double macs) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 98304);
+    kern<<<148, 64, 98304>>>(100, out);
+    cudaDeviceSynchronize();
+    kern<<<148, 64, 98304>>>(iters, out);
+    cudaError_t e = cudaDeviceSynchronize();
+    long long cyc = 0;
+    cudaMemcpy(&cyc, out, 8, cudaMemcpyDeviceToHost);
+    printf("{\"mma\": \"%s\", \"err\": \"%s\", \"cycles_per_mma\": %.2f, \"macs_per_cycle_per_sm\": %.0f}\n", name,
+           cudaGetErrorString(e), (double)cyc / iters, macs / ((double)cyc / iters));
+  };
+  run("i8 M128 N64 K32", k<0, 64>, 128.0 * 64 * 32);
+  run("i8 M128 N128 K32", k<0, 128>, 128.0 * 128 * 32);
+  run("i8 M128 N256 K32", k<0, 256>, 128.0 * 256 * 32);
+  run("f16 M128 N64 K16", k<1, 64>, 128.0 * 64 * 16);
+  run("f16 M128 N128 K16", k<1, 128>, 128.0 * 128 * 16);
+  run("f16 M128 N256 K16", k<1, 256>, 128.0 * 256 * 16);
+  return 0;
+}
