@@ -121,7 +121,7 @@ typedef struct {
   int64_t smo_cycles_sum;   /* SM clock cycles spent in the local SMO, summed over pairs      */
   double t_solver_ms;       /* a3-a6 as a whole: pairs run on concurrent streams, so select,  */
                             /* subproblem and f-update overlap (their own fields then stay 0)  */
-  int32_t n_streams;        /* concurrent pair groups (streams) used by the solver             */
+  int32_t n_streams;        /* concurrent branches of the solver graph (pairs packed into them) */
   int32_t pad0;
 } gmpsvm_train_stats;
 

@@ -1263,7 +1263,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         ++final_selects;
       }
     }
-    n_branches = final_selects;
+    n_branches = nbr;
     g_launches.fetch_sub(g_launches.load() - l0);  // captured, not executed: counted after the run
     GM_CUDA(cudaEventRecord(ev_ready, st));
     GM_CUDA(cudaStreamWaitEvent(pool[0], ev_ready, 0));
@@ -1321,7 +1321,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   GM_CUDA(cudaStreamSynchronize(st));
   HT("fin_d2h");
   {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
-    int64_t ex = n_branches;  // one final selection per split-path branch
+    int64_t ex = final_selects;  // one final selection per split-path branch
     for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_per_pair[i];  // counted at each branch's first pair
     g_launches.fetch_add((uint64_t)ex);
     if (rc) {
