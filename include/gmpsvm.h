@@ -204,6 +204,46 @@ GMPSVM_API int gmpsvm_model_from_alpha(const float* X, const int32_t* y, int64_t
                                        const double* B, const int32_t* status, const gmpsvm_options* opt,
                                        gmpsvm_model** out);
 
+/* ---- NEXT-1: one pair's binary SVM trained by several ranks, its instances sharded ----------
+ * (the paper's instance-level parallelism; kernel rows
+ * as a product of the working-set rows with the rest, L299; Algorithm 2 lines 5-13.)  Each rank
+ * holds X (replicated) and owns the slice [lo, hi) of the pair's instances (pair-local order:
+ * class s, then class t).  Per outer iteration the caller runs, on every rank, with its own
+ * collectives (torch.distributed; paper_conf_icde_wenshcc19_b200/dist.py train_pair_sharded):
+ *   gmpsvm_shard_candidates(sh, c)          c: this rank's block of gmpsvm_shard_cand_doubles
+ *   all_gather(c) -> all [world x cand_doubles], rank order
+ *   gmpsvm_shard_select(sh, all, &stop)     identical merge on every rank; stop = 1: converged
+ *                                           (Eq 9 with tolerance eps) or the outer cap
+ *   gmpsvm_shard_fws(sh, fws)               fws: B doubles, f of the members this rank owns
+ *   all_reduce_sum(fws)
+ *   gmpsvm_shard_step(sh, fws)              local SMO (same on every rank) + f update of the slice
+ * then gathers every rank's f slice (gmpsvm_shard_f, rank order) and calls gmpsvm_shard_finish
+ * for alpha (n_p, pair-local order), b, A, B and the status word of gmpsvm_model_pair.  All
+ * buffers are host pointers.  world = 1 is a complete single-rank solver; any world gives
+ * bitwise the same alpha.  RBF kernel only (else ENOTIMPL); opt: ws_size, q, device, stream,
+ * max_outer_iter, inputs_on_device (X, y device pointers). */
+typedef struct gmpsvm_shard gmpsvm_shard;
+GMPSVM_API int gmpsvm_shard_create(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, int32_t s,
+                                   int32_t t, double C, double gamma, double eps, int32_t rank, int32_t world,
+                                   const gmpsvm_options* opt, gmpsvm_shard** out);
+GMPSVM_API int32_t gmpsvm_shard_cand_doubles(const gmpsvm_shard* sh);
+GMPSVM_API int gmpsvm_shard_slice(const gmpsvm_shard* sh, int64_t* lo, int64_t* hi, int64_t* n_p, int32_t* ws_size);
+GMPSVM_API int gmpsvm_shard_candidates(gmpsvm_shard* sh, double* out);
+GMPSVM_API int gmpsvm_shard_select(gmpsvm_shard* sh, const double* all, int32_t* stop);
+GMPSVM_API int gmpsvm_shard_fws(gmpsvm_shard* sh, double* fws);
+GMPSVM_API int gmpsvm_shard_step(gmpsvm_shard* sh, const double* fws_sum);
+GMPSVM_API int gmpsvm_shard_f(gmpsvm_shard* sh, double* f_slice);
+GMPSVM_API int gmpsvm_shard_finish(gmpsvm_shard* sh, const double* f_full, double* alpha, double* b, double* A,
+                                   double* B, int32_t* status, int64_t* outer_iters, int64_t* inner_iters);
+GMPSVM_API void gmpsvm_shard_free(gmpsvm_shard* sh);
+/* The candidate merge alone (host arithmetic, no GPU): all = world blocks of cand_doubles
+ * [fmin, fmax, nU, nL, U keys (order-preserving bits of f, as doubles) x m, U indices x m, L keys
+ * (~bits) x m, L indices x m], m = (cand_doubles - 4) / 4; need picks, need_u of them from I_u
+ * first (R19).  picks_out: need int32 (selection order), *n_picks; *gap = max_{I_l} f - min_{I_u} f
+ * (-DBL_MAX if a side is empty). */
+GMPSVM_API int gmpsvm_shard_merge(const double* all, int32_t world, int32_t cand_doubles, int32_t need, int32_t need_u,
+                                  int32_t* picks_out, int32_t* n_picks, double* gap);
+
 /* ---- component entry points (steps of the path, exposed for parity tests and bench) ---- */
 /* a2 alone (K1, L287-L299, RBF L75): K_out[i*m + j] = exp(-gamma ||X_i - Y_j||^2) in FP32 via
  * the norm expansion ||x||^2 + ||y||^2 - 2 x.y (distance clamped at 0).  K_out [n x m].

@@ -86,6 +86,18 @@ _SIGS = {
                                            _P, _P, _P, _P, _P]),
     "gmpsvm_rbf_kernel": (ct.c_int, [_P, ct.c_int64, _P, ct.c_int64, ct.c_int32, ct.c_double, _P, _P]),
     "gmpsvm_couple": (ct.c_int, [_P, ct.c_int64, ct.c_int32, _P, _P, _P, _P]),
+    "gmpsvm_shard_create": (ct.c_int, [_P, _P, ct.c_int64, ct.c_int32, ct.c_int32, ct.c_int32, ct.c_int32, ct.c_double,
+                                       ct.c_double, ct.c_double, ct.c_int32, ct.c_int32, _P, _P]),
+    "gmpsvm_shard_cand_doubles": (ct.c_int32, [_P]),
+    "gmpsvm_shard_slice": (ct.c_int, [_P, _P, _P, _P, _P]),
+    "gmpsvm_shard_candidates": (ct.c_int, [_P, _P]),
+    "gmpsvm_shard_select": (ct.c_int, [_P, _P, _P]),
+    "gmpsvm_shard_fws": (ct.c_int, [_P, _P]),
+    "gmpsvm_shard_step": (ct.c_int, [_P, _P]),
+    "gmpsvm_shard_f": (ct.c_int, [_P, _P]),
+    "gmpsvm_shard_finish": (ct.c_int, [_P, _P, _P, _P, _P, _P, _P, _P, _P]),
+    "gmpsvm_shard_free": (None, [_P]),
+    "gmpsvm_shard_merge": (ct.c_int, [_P, ct.c_int32, ct.c_int32, ct.c_int32, ct.c_int32, _P, _P, _P]),
     "gmpsvm_launch_count": (ct.c_uint64, []),
     "gmpsvm_abi_version": (ct.c_int32, []),
 }
@@ -379,6 +391,77 @@ def couple(dec, k, A, B, out=None, **opts):
     o, keep = _options([a, aA, aB], **opts)
     _check(lib().gmpsvm_couple(a.ptr, a.shape[0], int(k), aA.ptr, aB.ptr, _data_ptr(out), ct.byref(o)))
     return out
+
+
+class Shard:
+    """NEXT-1: this rank's part of one pair's solver, the pair's instances sharded over `world`
+    ranks (gmpsvm_shard_*; the collectives between the calls are the caller's, see
+    dist.train_pair_sharded).  Host numpy buffers throughout."""
+
+    def __init__(self, X, y, k, s, t, C, gamma, eps, rank=0, world=1, **opts):
+        a = _Arg(X, np.float32, "X", 2)
+        b = _Arg(y, np.int32, "y", 1)
+        n, d = a.shape
+        o, keep = _options([a, b], **opts)
+        h = ct.c_void_p()
+        _check(lib().gmpsvm_shard_create(a.ptr, b.ptr, n, d, int(k), int(s), int(t), float(C), float(gamma), float(eps),
+                                         int(rank), int(world), ct.byref(o), ct.byref(h)))
+        self.h = h.value
+        self.cand_doubles = int(lib().gmpsvm_shard_cand_doubles(self.h))
+        lo, hi, npp, wsz = ct.c_int64(), ct.c_int64(), ct.c_int64(), ct.c_int32()
+        _check(lib().gmpsvm_shard_slice(self.h, ct.byref(lo), ct.byref(hi), ct.byref(npp), ct.byref(wsz)))
+        self.lo, self.hi, self.n_p, self.ws_size = lo.value, hi.value, npp.value, wsz.value
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().gmpsvm_shard_free(self.h)
+            self.h = None
+
+    def candidates(self):
+        out = np.zeros(self.cand_doubles)
+        _check(lib().gmpsvm_shard_candidates(self.h, out.ctypes.data))
+        return out
+
+    def select(self, all_cands):
+        a = np.ascontiguousarray(all_cands, dtype=np.float64)
+        stop = ct.c_int32()
+        _check(lib().gmpsvm_shard_select(self.h, a.ctypes.data, ct.byref(stop)))
+        return bool(stop.value)
+
+    def fws(self):
+        out = np.zeros(self.ws_size)
+        _check(lib().gmpsvm_shard_fws(self.h, out.ctypes.data))
+        return out
+
+    def step(self, fws_sum):
+        a = np.ascontiguousarray(fws_sum, dtype=np.float64)
+        _check(lib().gmpsvm_shard_step(self.h, a.ctypes.data))
+
+    def f_slice(self):
+        out = np.zeros(self.hi - self.lo)
+        if out.size:
+            _check(lib().gmpsvm_shard_f(self.h, out.ctypes.data))
+        return out
+
+    def finish(self, f_full):
+        f = np.ascontiguousarray(f_full, dtype=np.float64)
+        alpha = np.zeros(self.n_p)
+        b, A, B = ct.c_double(), ct.c_double(), ct.c_double()
+        st, outer, inner = ct.c_int32(), ct.c_int64(), ct.c_int64()
+        rc = _check(lib().gmpsvm_shard_finish(self.h, f.ctypes.data, alpha.ctypes.data, ct.byref(b), ct.byref(A),
+                                              ct.byref(B), ct.byref(st), ct.byref(outer), ct.byref(inner)))
+        return dict(alpha=alpha, b=b.value, A=A.value, B=B.value, status=st.value, outer_iters=outer.value,
+                    inner_iters=inner.value, rc=rc)
+
+
+def shard_merge(all_cands, world, cand_doubles, need, need_u):
+    """gmpsvm_shard_merge: the exact candidate merge of the sharded solver (host arithmetic)."""
+    a = np.ascontiguousarray(all_cands, dtype=np.float64)
+    picks = np.zeros(max(int(need), 1), dtype=np.int32)
+    n, gap = ct.c_int32(), ct.c_double()
+    _check(lib().gmpsvm_shard_merge(a.ctypes.data, int(world), int(cand_doubles), int(need), int(need_u),
+                                    picks.ctypes.data, ct.byref(n), ct.byref(gap)))
+    return picks[: n.value], gap.value
 
 
 def launch_count() -> int:

@@ -464,6 +464,89 @@ int gmpsvm_couple(const double* dec, int64_t m, int32_t k, const double* A, cons
   return guarded([&]() { return gmpsvm::engine_couple(dec, m, k, A, B, prob_out, resolve(opt)); });
 }
 
+struct gmpsvm_shard {
+  gmpsvm::Shard* s = nullptr;
+};
+
+int gmpsvm_shard_create(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, int32_t s, int32_t t,
+                        double C, double gamma, double eps, int32_t rank, int32_t world, const gmpsvm_options* opt,
+                        gmpsvm_shard** out) {
+  return guarded([&]() {
+    if (!out) throw Error(GMPSVM_EINVAL, "out is NULL");
+    *out = nullptr;
+    gmpsvm::Shard* sh = gmpsvm::shard_create(X, y, n, d, k, s, t, C, gamma, eps, rank, world, resolve(opt));
+    *out = new gmpsvm_shard{sh};
+    return GMPSVM_OK;
+  });
+}
+int32_t gmpsvm_shard_cand_doubles(const gmpsvm_shard* sh) { return sh ? gmpsvm::shard_cand_doubles(sh->s) : 0; }
+int gmpsvm_shard_slice(const gmpsvm_shard* sh, int64_t* lo, int64_t* hi, int64_t* n_p, int32_t* ws_size) {
+  return guarded([&]() {
+    if (!sh) throw Error(GMPSVM_EINVAL, "shard is NULL");
+    gmpsvm::shard_slice(sh->s, lo, hi, n_p, ws_size);
+    return GMPSVM_OK;
+  });
+}
+int gmpsvm_shard_candidates(gmpsvm_shard* sh, double* out) {
+  return guarded([&]() {
+    if (!sh || !out) throw Error(GMPSVM_EINVAL, "null argument");
+    gmpsvm::shard_candidates(sh->s, out);
+    return GMPSVM_OK;
+  });
+}
+int gmpsvm_shard_select(gmpsvm_shard* sh, const double* all, int32_t* stop) {
+  return guarded([&]() {
+    if (!sh || !all || !stop) throw Error(GMPSVM_EINVAL, "null argument");
+    return gmpsvm::shard_select(sh->s, all, stop);
+  });
+}
+int gmpsvm_shard_fws(gmpsvm_shard* sh, double* fws) {
+  return guarded([&]() {
+    if (!sh || !fws) throw Error(GMPSVM_EINVAL, "null argument");
+    gmpsvm::shard_fws(sh->s, fws);
+    return GMPSVM_OK;
+  });
+}
+int gmpsvm_shard_step(gmpsvm_shard* sh, const double* fws_sum) {
+  return guarded([&]() {
+    if (!sh || !fws_sum) throw Error(GMPSVM_EINVAL, "null argument");
+    gmpsvm::shard_step(sh->s, fws_sum);
+    return GMPSVM_OK;
+  });
+}
+int gmpsvm_shard_f(gmpsvm_shard* sh, double* f_slice) {
+  return guarded([&]() {
+    if (!sh || !f_slice) throw Error(GMPSVM_EINVAL, "null argument");
+    gmpsvm::shard_f(sh->s, f_slice);
+    return GMPSVM_OK;
+  });
+}
+int gmpsvm_shard_finish(gmpsvm_shard* sh, const double* f_full, double* alpha, double* b, double* A, double* B,
+                        int32_t* status, int64_t* outer_iters, int64_t* inner_iters) {
+  return guarded([&]() {
+    if (!sh || !f_full || !alpha || !b || !A || !B) throw Error(GMPSVM_EINVAL, "null argument");
+    return gmpsvm::shard_finish(sh->s, f_full, alpha, b, A, B, status, outer_iters, inner_iters);
+  });
+}
+void gmpsvm_shard_free(gmpsvm_shard* sh) {
+  if (!sh) return;
+  gmpsvm::shard_free(sh->s);
+  delete sh;
+}
+int gmpsvm_shard_merge(const double* all, int32_t world, int32_t cand_doubles, int32_t need, int32_t need_u,
+                       int32_t* picks_out, int32_t* n_picks, double* gap) {
+  return guarded([&]() {
+    if (!all || world < 1 || cand_doubles < 4 || need < 0 || need_u < 0 || need_u > need || !n_picks || !gap ||
+        (need > 0 && !picks_out))
+      throw Error(GMPSVM_EINVAL, "bad merge arguments");
+    std::vector<int32_t> picks;
+    *gap = gmpsvm::shard_merge(all, world, cand_doubles, need, need_u, picks);
+    *n_picks = (int32_t)picks.size();
+    for (size_t i = 0; i < picks.size(); ++i) picks_out[i] = picks[i];
+    return GMPSVM_OK;
+  });
+}
+
 uint64_t gmpsvm_launch_count(void) { return gmpsvm::g_launches.load(); }
 
 int32_t gmpsvm_abi_version(void) { return GMPSVM_ABI_VERSION; }

@@ -38,6 +38,23 @@ extern std::atomic<uint64_t> g_launches;  // kernels launched by this library
     GM_CHECK_LAUNCH();                                                     \
   } while (0)
 
+// Stream-ordered device buffer (cudaMallocAsync / cudaFreeAsync on the owning stream).
+template <class T>
+struct DevBuf {
+  T* p = nullptr;
+  cudaStream_t st = nullptr;
+  DevBuf() = default;
+  DevBuf(size_t count, cudaStream_t s) : st(s) {
+    if (count) GM_CUDA(cudaMallocAsync((void**)&p, count * sizeof(T), s));
+  }
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  ~DevBuf() {
+    if (p) cudaFreeAsync(p, st);
+  }
+  T* get() const { return p; }
+};
+
 inline int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 

@@ -138,22 +138,6 @@ struct EventPool {
   }
 };
 
-template <class T>
-struct DevBuf {
-  T* p = nullptr;
-  cudaStream_t st = nullptr;
-  DevBuf() = default;
-  DevBuf(size_t count, cudaStream_t s) : st(s) {
-    if (count) GM_CUDA(cudaMallocAsync((void**)&p, count * sizeof(T), s));
-  }
-  DevBuf(const DevBuf&) = delete;
-  DevBuf& operator=(const DevBuf&) = delete;
-  ~DevBuf() {
-    if (p) cudaFreeAsync(p, st);
-  }
-  T* get() const { return p; }
-};
-
 // Kernel-matrix workspace cache (FULL_K regime): the n^2 x 4 B buffer is the largest
 // allocation of a training run; growing a stream-ordered pool by 14.4 GB costs 0.1-0.5 s, so
 // the buffer is kept per device and reused by later runs.  A buffer is handed out to one run

@@ -115,6 +115,22 @@ void ensure_host_sv(const Model& mdl);     // materialise sv_X on the host
 void ensure_host_alpha(const Model& mdl);  // materialise alpha on the host
 gmpsvm_predict_stats& tls_predict_stats();
 
+// shard.cu (NEXT-1)
+struct Shard;
+Shard* shard_create(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, int32_t s, int32_t t, double C,
+                    double gamma, double eps, int32_t rank, int32_t world, const gmpsvm_options& opt);
+void shard_free(Shard* S);
+int shard_cand_doubles(const Shard* S);
+void shard_slice(const Shard* S, int64_t* lo, int64_t* hi, int64_t* np, int32_t* ws_size);
+void shard_candidates(Shard* S, double* out);
+int shard_select(Shard* S, const double* all, int32_t* stop);
+void shard_fws(Shard* S, double* out);
+void shard_step(Shard* S, const double* fws_sum);
+void shard_f(Shard* S, double* out);
+int shard_finish(Shard* S, const double* f_full, double* alpha_out, double* b, double* A, double* Bsig, int32_t* status,
+                 int64_t* outer, int64_t* inner);
+double shard_merge(const double* all, int world, int cand_doubles, int need, int need_u, std::vector<int32_t>& picks);
+
 }  // namespace gmpsvm
 
 struct gmpsvm_model {

@@ -8,6 +8,12 @@ no collective inside the solver loop.  The ranks then combine the disjoint per-p
 complete model from its own replicated X (gmpsvm_model_from_alpha); serializing and merging
 whole partial models (gather_models) remains available.  Prediction shards the test rows
 (instances are independent, L273) and all-gathers the m x k probabilities.
+
+NEXT-1 (intra-pair sharding): a pair too costly for one rank -- on MNIST-shaped data one pair
+runs 232 outer iterations and bounds pair sharding at ~1.5x on 8 GPUs -- is
+trained by every rank at once, its instances split into slices (train_pair_sharded over the
+gmpsvm_shard_* calls: per outer iteration one all_gather of the ranks' candidate blocks and one
+all-reduce of the working set's f values, O(world * B) doubles).
 """
 from __future__ import annotations
 
@@ -20,11 +26,15 @@ def pair_list(k):
     return [(s, t) for s in range(k) for t in range(s + 1, k)]
 
 
-def plan_pairs(class_counts, world, exponent=1.5):
-    """LPT (longest processing time first) assignment of pair indices to `world` ranks."""
+def plan_pairs(class_counts, world, exponent=1.5, only=None):
+    """LPT (longest processing time first) assignment of pair indices (all, or `only`) to `world`
+    ranks."""
     k = len(class_counts)
     sizes = np.array([class_counts[s] + class_counts[t] for s, t in pair_list(k)], dtype=np.float64)
     order = np.argsort(-(sizes ** exponent), kind="stable")
+    if only is not None:
+        keep = set(int(p) for p in only)
+        order = [p for p in order if int(p) in keep]
     load = np.zeros(world)
     shards = [[] for _ in range(world)]
     for p in order:
@@ -77,13 +87,19 @@ def pair_layout(counts):
     return pairs, np.concatenate([[0], np.cumsum(sizes)]).astype(np.int64)
 
 
-def pack_solutions(part: "gm.Model", counts):
+def pack_solutions(part: "gm.Model", counts, extra=None):
     """This rank's trained pairs as one flat FP64 vector [alpha | b | A | B | status | trained]
-    in the global layout (zeros for pairs other ranks train) -- disjoint across ranks."""
+    in the global layout (zeros for pairs other ranks train) -- disjoint across ranks.
+    extra: {pair index: train_pair_sharded result} solved outside `part` (rank 0 passes them)."""
     pairs, off = pair_layout(counts)
     P = len(pairs)
     tot = int(off[-1])
     v = np.zeros(tot + 5 * P)
+    for p, r in (extra or {}).items():
+        v[off[p]:off[p + 1]] = r["alpha"]
+        v[tot + p], v[tot + P + p], v[tot + 2 * P + p] = r["b"], r["A"], r["B"]
+        v[tot + 3 * P + p] = float(r["status"])
+        v[tot + 4 * P + p] = 1.0
     if part is None:  # a rank with no pair (more ranks than pairs): contributes zeros
         return v
     mine = part.trained_pairs()
@@ -97,15 +113,17 @@ def pack_solutions(part: "gm.Model", counts):
     return v
 
 
-def gather_solutions(part: "gm.Model", X, y, k, C, gamma, group=None, **opts) -> "gm.Model":
+def gather_solutions(part: "gm.Model", X, y, k, C, gamma, group=None, extra=None, **opts) -> "gm.Model":
     """All-reduce (sum) of the disjoint per-pair solutions, then the complete model rebuilt from
-    the local X on every rank (identical on all ranks)."""
+    the local X on every rank (identical on all ranks).  extra: pairs solved by
+    train_pair_sharded (identical on every rank: rank 0 contributes them)."""
     import torch
     import torch.distributed as dist
 
     yy = y.cpu().numpy() if isinstance(y, torch.Tensor) else np.asarray(y)
     counts = np.bincount(yy, minlength=k)
-    v = torch.from_numpy(pack_solutions(part, counts)).to(_backend_device(group))
+    ex = extra if dist.get_rank(group) == 0 else None
+    v = torch.from_numpy(pack_solutions(part, counts, ex)).to(_backend_device(group))
     dist.all_reduce(v, op=dist.ReduceOp.SUM, group=group)
     v = v.cpu().numpy()
     pairs, off = pair_layout(counts)
@@ -144,8 +162,51 @@ def all_gather_rows(local, m_total, group=None):
     return torch.cat(pieces, 0)
 
 
-def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
-    """Sharded train (pairs) + sharded predict (rows) on every rank; returns (model, prob)."""
+def _all_gather_f64(x: np.ndarray, group=None):
+    """All-gather variable-length FP64 vectors (rank order)."""
+    parts = all_gather_bytes(np.frombuffer(np.ascontiguousarray(x, dtype=np.float64).tobytes(), dtype=np.uint8), group)
+    return [np.frombuffer(p.tobytes(), dtype=np.float64) for p in parts]
+
+
+def train_pair_sharded(X, y, k, s, t, C, gamma, eps, group=None, **opts):
+    """NEXT-1: pair (s, t) trained by every rank of `group`, its instances sharded (PAPER.md
+    L250, L299).  Per outer iteration: candidates -> all_gather -> the same exact selection on
+    every rank -> f of the working set all-reduced -> the same local SMO everywhere, f updated
+    on each rank's slice.  Returns the pair's alpha (pair-local order), b, A, B, status and
+    iteration counts, identical on every rank (and bitwise those of world = 1)."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    dev = _backend_device(group)
+    sh = gm.Shard(X, y, k, s, t, C, gamma, eps, rank, world, **opts)
+    while True:
+        c = torch.from_numpy(sh.candidates()).to(dev)
+        outs = [torch.empty_like(c) for _ in range(world)]
+        dist.all_gather(outs, c, group=group)
+        if sh.select(torch.stack(outs).cpu().numpy()):
+            break
+        fw = torch.from_numpy(sh.fws()).to(dev)
+        dist.all_reduce(fw, op=dist.ReduceOp.SUM, group=group)
+        sh.step(fw.cpu().numpy())
+    f_full = np.concatenate(_all_gather_f64(sh.f_slice(), group))
+    return sh.finish(f_full)
+
+
+def plan_intra(counts, world, exponent=1.5):
+    """Pairs to shard across every rank (NEXT-1): those whose estimated cost (n_p^exponent)
+    alone exceeds a rank's even share of the total."""
+    k = len(counts)
+    sizes = np.array([counts[s] + counts[t] for s, t in pair_list(k)], dtype=np.float64)
+    cost = sizes ** exponent
+    return [int(p) for p in np.flatnonzero(cost > cost.sum() / world)] if world > 1 else []
+
+
+def train_predict(X, y, Xt, k, C, gamma, eps, group=None, intra_pairs=None, **opts):
+    """Sharded train (pairs) + sharded predict (rows) on every rank; returns (model, prob).
+    intra_pairs: pair indices trained by all ranks at once (NEXT-1, train_pair_sharded);
+    "auto" = plan_intra; None = none (every pair on one rank)."""
     import torch
     import torch.distributed as dist
 
@@ -153,12 +214,22 @@ def train_predict(X, y, Xt, k, C, gamma, eps, group=None, **opts):
     rank = dist.get_rank(group)
     yy = y.cpu().numpy() if isinstance(y, torch.Tensor) else np.asarray(y)
     counts = np.bincount(yy, minlength=k)
-    mine = plan_pairs(counts, world)[rank]
+    if isinstance(intra_pairs, str):
+        intra_pairs = plan_intra(counts, world)
+    intra = sorted(int(p) for p in (intra_pairs or []))
+    extra = {}
+    if intra:
+        sopts = {key: opts[key] for key in ("device", "stream", "ws_size", "q", "max_outer_iter") if key in opts}
+        pairs = pair_list(k)
+        for p in intra:
+            extra[p] = train_pair_sharded(X, y, k, pairs[p][0], pairs[p][1], C, gamma, eps, group, **sopts)
+    rest = [p for p in range(len(pair_list(k))) if p not in extra]
+    mine = plan_pairs(counts, world, only=rest)[rank] if rest else []
     # more ranks than pairs: a rank with an empty shard trains nothing and adds zeros to the
     # all-reduce (the library rejects an empty pair_ids list rather than training every pair)
     part = gm.train(X, y, k, C, gamma, eps, pair_ids=mine, **opts) if mine else None
     dev_opts = {key: opts[key] for key in ("device", "stream", "kernel", "coef0", "degree") if key in opts}
-    model = gather_solutions(part, X, y, k, C, gamma, group, **dev_opts)
+    model = gather_solutions(part, X, y, k, C, gamma, group, extra=extra, **dev_opts)
     model.part_stats = part.train_stats() if part is not None else None  # this rank's training
     m = Xt.shape[0]
     lo, hi = row_range(m, world, rank)

@@ -161,3 +161,99 @@ def test_gloo_world2_gather_merge():
     for p in procs:
         p.join(timeout=60)
     assert all(ok for _, ok, _ in res), res
+
+
+# ------------------------------------------------------------------------------------ NEXT-1
+def _ord_key(f):
+    """Order-preserving uint64 key of FP64 values (negative: all bits flipped; else sign set)."""
+    u = np.asarray(f, dtype=np.float64).view(np.uint64)
+    neg = (u >> np.uint64(63)) == 1
+    return np.where(neg, ~u, u | np.uint64(1 << 63))
+
+
+def _cand_block(f, a, y, C, ret, lo, hi, need, m):
+    """A rank's candidate block (layout of gmpsvm_shard_merge) from its slice [lo, hi), numpy."""
+    blk = np.zeros(4 + 4 * m)
+    idx = np.arange(lo, hi)
+    iu = ((y[idx] > 0) & (a[idx] < C)) | ((y[idx] < 0) & (a[idx] > 0))
+    il = ((y[idx] > 0) & (a[idx] > 0)) | ((y[idx] < 0) & (a[idx] < C))
+    blk[0] = f[idx][iu].min() if iu.any() else np.finfo(np.float64).max
+    blk[1] = f[idx][il].max() if il.any() else -np.finfo(np.float64).max
+    cu = idx[iu & ~ret[idx]]
+    cl = idx[il & ~ret[idx]]
+    cu = cu[np.lexsort((cu, f[cu]))][:need]       # smallest f, lowest index on ties
+    cl = cl[np.lexsort((cl, -f[cl]))][:need]      # largest f, lowest index on ties
+    blk[2], blk[3] = len(cu), len(cl)
+    blk[4:4 + len(cu)] = _ord_key(f[cu]).view(np.float64)
+    blk[4 + m:4 + m + len(cu)] = cu
+    blk[4 + 2 * m:4 + 2 * m + len(cl)] = (~_ord_key(f[cl])).view(np.float64)
+    blk[4 + 3 * m:4 + 3 * m + len(cl)] = cl
+    return blk
+
+
+def _reference_selection(f, a, y, C, ret, need, need_u):
+    """Reading R19 on the whole vector: need_u smallest f in I_u \\ retained, then the largest f in
+    I_l \\ retained not taken, then I_u again if I_l ran short (ties: lowest index)."""
+    n = len(f)
+    idx = np.arange(n)
+    iu = (((y > 0) & (a < C)) | ((y < 0) & (a > 0))) & ~ret
+    il = (((y > 0) & (a > 0)) | ((y < 0) & (a < C))) & ~ret
+    U = idx[iu][np.lexsort((idx[iu], f[iu]))]
+    L = idx[il][np.lexsort((idx[il], -f[il]))]
+    picks = list(U[:need_u])
+    for j in L:
+        if len(picks) >= need:
+            break
+        if j not in picks:
+            picks.append(j)
+    for j in U[need_u:]:
+        if len(picks) >= need:
+            break
+        if j not in picks:
+            picks.append(j)
+    gap = f[(((y > 0) & (a > 0)) | ((y < 0) & (a < C)))].max() - f[(((y > 0) & (a < C)) | ((y < 0) & (a > 0)))].min()
+    return np.array(picks, dtype=np.int32), gap
+
+
+def _merge_worker(rank, world, port, q):
+    try:
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        import paper_conf_icde_wenshcc19_b200 as gm
+
+        ok = True
+        for seed in range(6):
+            rng = np.random.default_rng(seed)
+            n, C, B = 1500, 1.0, 96
+            y = np.where(np.arange(n) < 700, 1, -1)
+            a = np.where(rng.random(n) < 0.4, 0.0, np.where(rng.random(n) < 0.5, C, rng.uniform(0, C, n)))
+            f = np.round(rng.normal(0, 1, n), 2 if seed % 2 else 9)  # seed odd: many exact ties
+            ret = np.zeros(n, dtype=bool)
+            ret[rng.choice(n, size=B // 2, replace=False)] = True
+            need = B - int(ret.sum())
+            if seed == 5:  # I_l almost empty: the selection takes I_u again
+                a[:700] = 0.0
+                a[700:] = C
+                a[700:705] = 0.5
+            per = -(-n // world)
+            lo, hi = min(n, rank * per), min(n, rank * per + per)
+            blk = torch.from_numpy(_cand_block(f, a, y, C, ret, lo, hi, need, B))
+            outs = [torch.empty_like(blk) for _ in range(world)]
+            dist.all_gather(outs, blk)
+            picks, gap = gm.shard_merge(torch.stack(outs).numpy(), world, 4 + 4 * B, need, need // 2)
+            ref, gref = _reference_selection(f, a, y, C, ret, need, need // 2)
+            ok &= bool(np.array_equal(picks, ref)) and abs(gap - gref) < 1e-15
+        q.put((rank, bool(ok), ""))
+    except Exception as e:
+        q.put((rank, False, repr(e)))
+    finally:
+        if dist.is_initialized():
+            dist.destroy_process_group()
+
+
+def test_gloo_world2_intra_pair_candidate_merge():
+    """NEXT-1's exchange: every rank's candidate block of its slice, all_gather over gloo, and the
+    library's merge (gmpsvm_shard_merge) reproduces reading R19's selection on the whole vector
+    (ties to the lowest index, I_u taken again when I_l runs short) and the global gap."""
+    _run(_merge_worker, 2)
+    _run(_merge_worker, 3)

@@ -1,0 +1,131 @@
+"""NEXT-1 intra-pair sharding on the GPU (shard.cu through gmpsvm_shard_*, dist.py).
+
+* world 2 (two processes, gloo, both on cuda:0) trains one pair with its instances split and gets
+  alpha, b, A, B BITWISE equal to world 1;
+* the sharded solver reaches the oracle's fixed point (alpha within 1e-3 C, SV sets up to
+  documented ties, b within 1e-3, FP64 KKT audit of the GPU alpha);
+* dist.train_predict with that pair sharded and the others pair-sharded gives probabilities
+  within 1e-4 of the oracle's.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+EPS = 1e-5
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, job, q):
+    try:
+        import sys
+
+        sys.path.insert(0, ROOT)
+        import torch.distributed as dist
+
+        import datagen
+        from paper_conf_icde_wenshcc19_b200 import dist as gdist
+
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        name, n, m, s, t, ws = job
+        spec, X, y, Xt, yt = datagen.make_config(name, n_train=n, n_test=m)
+        if s is not None:
+            r = gdist.train_pair_sharded(X, y, spec.k, s, t, spec.C, spec.gamma, EPS, ws_size=ws)
+            q.put((rank, r, ""))
+        else:
+            _, prob = gdist.train_predict(X, y, Xt, spec.k, spec.C, spec.gamma, EPS, intra_pairs=[t], ws_size=ws)
+            q.put((rank, prob.cpu().numpy(), ""))
+    except Exception as e:  # report instead of hanging the parent
+        import traceback
+
+        q.put((rank, None, traceback.format_exc()))
+    finally:
+        import torch.distributed as dist
+
+        if dist.is_initialized():
+            dist.destroy_process_group()
+
+
+def _spawn(world, job):
+    import torch.multiprocessing as mp
+
+    ctx = mp.get_context("spawn")
+    qu = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, job, qu)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([qu.get(timeout=900) for _ in procs], key=lambda r: r[0])
+    for p in procs:
+        p.join(timeout=60)
+    assert all(r[2] == "" for r in res), [r[2] for r in res]
+    return [r[1] for r in res]
+
+
+@pytest.fixture(scope="module")
+def gm():
+    import __graft_entry__
+
+    __graft_entry__.build()
+    import paper_conf_icde_wenshcc19_b200 as m
+
+    return m
+
+
+def _single_rank(gm, X, y, k, s, t, C, gamma, ws):
+    sh = gm.Shard(X, y, k, s, t, C, gamma, EPS, 0, 1, ws_size=ws)
+    while True:
+        if sh.select(sh.candidates()[None, :]):
+            break
+        sh.step(sh.fws())
+    return sh.finish(sh.f_slice())
+
+
+@pytest.mark.parametrize("name,n,s,t,ws", [("mnist", 2500, 0, 8, 64), ("letter", 4000, 4, 17, 32), ("blobs", None, 0, 1, 96)])
+def test_sharded_pair_world2_bitwise_and_oracle(gm, name, n, s, t, ws):
+    spec, X, y, Xt, yt = datagen.make_config(name, n_train=n, n_test=None if n is None else 50)
+    one = _single_rank(gm, X, y, spec.k, s, t, spec.C, spec.gamma, ws)
+    assert one["outer_iters"] > 3 and one["rc"] == 0
+    two = _spawn(2, (name, n, 50, s, t, ws))
+    for r in two:
+        np.testing.assert_array_equal(r["alpha"], one["alpha"])
+        assert (r["b"], r["A"], r["B"], r["outer_iters"]) == (one["b"], one["A"], one["B"], one["outer_iters"])
+    # the oracle's fixed point (SURVEY §8(c) contract)
+    idx, ypm = oracle.pair_members(y, spec.k, s, t)
+    ref = oracle.smo(X[idx], ypm, spec.C, spec.gamma, EPS)
+    a, C = one["alpha"], spec.C
+    assert np.abs(a - ref["alpha"]).max() <= 1e-3 * C
+    diff = (a > 0) != (ref["alpha"] > 0)
+    assert np.all(np.maximum(a, ref["alpha"])[diff] < 1e-4 * C)
+    f = oracle.exact_f(X[idx], ypm, a, spec.gamma)
+    rho = oracle.rho(ref["alpha"], oracle.exact_f(X[idx], ypm, ref["alpha"], spec.gamma), ypm, C)
+    assert abs(one["b"] + rho) <= 1e-3 * max(1.0, abs(rho))
+    iu = ((ypm > 0) & (a < C)) | ((ypm < 0) & (a > 0))
+    il = ((ypm > 0) & (a > 0)) | ((ypm < 0) & (a < C))
+    assert f[il].max() - f[iu].min() <= EPS + 2 * 1e-4 * a.sum()
+    assert abs((ypm * a).sum()) <= 1e-9 * C * len(a)
+
+
+def test_train_predict_with_an_intra_sharded_pair_vs_oracle(gm):
+    spec, X, y, Xt, yt = datagen.make_config("mnist", n_train=2000, n_test=200)
+    prob = _spawn(2, ("mnist", 2000, 200, None, 7, 64))  # pair 7 = (0, 8) sharded, the rest by pairs
+    ref = oracle.train(X, y, spec.k, spec.C, spec.gamma, EPS)
+    _, prob_o = oracle.predict(ref, X, y, Xt, want_dec=False)
+    for p in prob:
+        assert np.abs(p - prob_o).max() <= 1e-4
+    np.testing.assert_array_equal(prob[0], prob[1])
