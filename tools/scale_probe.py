@@ -37,5 +37,8 @@ st = model.train_stats()
 out = {"config": name, "n_train": n, "n_test": m, "d": spec.d, "k": spec.k, "C": spec.C, "gamma": spec.gamma,
        "train_s": t1 - t0, "predict_s": t2 - t1, "test_acc": acc,
        "stats": {k: (round(v, 3) if isinstance(v, float) else v) for k, v in st.items()},
-       "kernel_tflops": st["kernel_flops"] / max(1e-9, st["t_kernel_ms"] * 1e-3) / 1e12 if st["t_kernel_ms"] else None}
+       # FULL_K only: ROW_CACHE rows run inside the solver graph, t_kernel_ms does not time them
+       # (their time comes from the ncu launch list, profiles/r02)
+       "kernel_tflops": (st["kernel_flops"] / (st["t_kernel_ms"] * 1e-3) / 1e12
+                         if st["cache_regime"] == 0 and st["t_kernel_ms"] > 0 else None)}
 print(json.dumps(out), flush=True)
