@@ -181,6 +181,12 @@ GMPSVM_API int gmpsvm_model_dims(const gmpsvm_model* model, int32_t* k, int32_t*
 GMPSVM_API int gmpsvm_model_pair(const gmpsvm_model* model, int32_t s, int32_t t, double* b, double* A, double* B,
                       double* alpha_out);
 /* Original training indices of the SV union, ascending in (class, original index). */
+/* Telemetry of pair (s, t) from its training run (SURVEY §8(d) "report outer/inner iterations
+ * and rows computed"): outer iterations (Alg 2 l.5-12), inner SMO steps, kernel rows computed
+ * (ROW_CACHE regime; 0 in FULL_K, where every row is computed once for all pairs).  0 for models
+ * rebuilt from alpha or deserialised.  Any pointer may be NULL. */
+GMPSVM_API int gmpsvm_model_pair_iters(const gmpsvm_model* model, int32_t s, int32_t t, int64_t* outer, int64_t* inner,
+                                       int64_t* rows);
 GMPSVM_API int gmpsvm_model_sv_index(const gmpsvm_model* model, int64_t* idx_out);
 GMPSVM_API int gmpsvm_model_train_stats(const gmpsvm_model* model, gmpsvm_train_stats* stats);
 GMPSVM_API void gmpsvm_last_predict_stats(gmpsvm_predict_stats* stats); /* thread-local, last predict call */

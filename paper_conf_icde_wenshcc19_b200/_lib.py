@@ -74,6 +74,7 @@ _SIGS = {
     "gmpsvm_model_dims": (ct.c_int, [_P, _P, _P, _P, _P]),
     "gmpsvm_model_pair": (ct.c_int, [_P, ct.c_int32, ct.c_int32, _P, _P, _P, _P]),
     "gmpsvm_model_sv_index": (ct.c_int, [_P, _P]),
+    "gmpsvm_model_pair_iters": (ct.c_int, [_P, ct.c_int32, ct.c_int32, _P, _P, _P]),
     "gmpsvm_model_train_stats": (ct.c_int, [_P, _P]),
     "gmpsvm_last_predict_stats": (None, [_P]),
     "gmpsvm_model_serialize": (ct.c_int, [_P, _P, _P]),
@@ -270,6 +271,12 @@ class Model:
         rc = _check(lib().gmpsvm_model_pair(self._h, s, t, ct.byref(b), ct.byref(A), ct.byref(B),
                                             alpha.ctypes.data if alpha is not None else None))
         return dict(b=b.value, A=A.value, B=B.value, alpha=alpha, status=rc)
+
+    def pair_iters(self, s, t):
+        """(outer iterations, inner SMO steps, kernel rows computed) of pair (s, t)'s training."""
+        o, i, r = ct.c_int64(), ct.c_int64(), ct.c_int64()
+        _check(lib().gmpsvm_model_pair_iters(self._h, int(s), int(t), ct.byref(o), ct.byref(i), ct.byref(r)))
+        return o.value, i.value, r.value
 
     def trained_pairs(self):
         """Indices of the pairs this model holds (all of them unless trained with pair_ids)."""

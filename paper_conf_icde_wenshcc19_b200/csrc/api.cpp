@@ -355,6 +355,21 @@ int gmpsvm_model_dims(const gmpsvm_model* model, int32_t* k, int32_t* d, int64_t
   });
 }
 
+int gmpsvm_model_pair_iters(const gmpsvm_model* model, int32_t s, int32_t t, int64_t* outer, int64_t* inner,
+                            int64_t* rows) {
+  return guarded([&]() {
+    if (!model) throw Error(GMPSVM_EINVAL, "model is NULL");
+    const Model& m = *model->m;
+    if (s < 0 || t <= s || t >= m.k) throw Error(GMPSVM_EINVAL, "need 0 <= s < t < k");
+    const int p = gmpsvm::pair_index(s, t, m.k);
+    auto at = [&](const std::vector<int64_t>& v) { return p < (int)v.size() ? v[p] : (int64_t)0; };
+    if (outer) *outer = at(m.pair_outer);
+    if (inner) *inner = at(m.pair_inner);
+    if (rows) *rows = at(m.pair_rows);
+    return GMPSVM_OK;
+  });
+}
+
 int gmpsvm_model_pair(const gmpsvm_model* model, int32_t s, int32_t t, double* b, double* A, double* B,
                       double* alpha_out) {
   return guarded([&]() {

@@ -1410,6 +1410,9 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   mdl->A.assign(P, 0.0);
   mdl->B.assign(P, 0.0);
   mdl->status.assign(P, 0);
+  mdl->pair_outer.assign(P, 0);
+  mdl->pair_inner.assign(P, 0);
+  mdl->pair_rows.assign(P, 0);
   const auto po = mdl->pair_offsets();
   mdl->alpha_ready = false;
   std::vector<int64_t> alpha_off(P, -1);  // model pair -> offset into the solver's device alpha
@@ -1425,6 +1428,8 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
       cap_hit = true;
     }
     mdl->status[p] = (h_st[i] == 1 ? 0 : h_st[i]) | (h_sig[i] << 8);
+    mdl->pair_outer[p] = h_outer[i];
+    mdl->pair_inner[p] = h_inner[i];
     alpha_off[p] = hp[i].a_off;
     outer_max = std::max<int64_t>(outer_max, h_outer[i]);
     outer_sum += h_outer[i];
@@ -1464,6 +1469,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   } else {
     std::vector<int64_t> rows(Pl);
     GM_CUDA(cudaMemcpy(rows.data(), d_rows.get(), Pl * 8, cudaMemcpyDeviceToHost));
+    for (int i = 0; i < Pl; ++i) mdl->pair_rows[hp[i].pid] = rows[i];
     s.kernel_values = 0;
     for (int i = 0; i < Pl; ++i) s.kernel_values += (double)rows[i] * (double)(hp[i].n_s + hp[i].n_t);
     s.krow_launches = rc_launches;
@@ -1544,6 +1550,9 @@ int engine_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t
   mdl->A.assign(A, A + P);
   mdl->B.assign(B, B + P);
   mdl->status.assign(P, 0);
+  mdl->pair_outer.assign(P, 0);
+  mdl->pair_inner.assign(P, 0);
+  mdl->pair_rows.assign(P, 0);
   if (status) mdl->status.assign(status, status + P);
   mdl->alpha.assign(alpha, alpha + po[P]);
   for (int64_t j = 0; j < po[P]; ++j)

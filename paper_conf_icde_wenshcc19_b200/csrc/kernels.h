@@ -169,6 +169,9 @@ void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_
 // L2-resident tile, single-warp local SMO (FULL_K regime, B <= 224, n_p <= 16384;
 // GMPSVM_WSOLVE=0 selects the select_ws / gather_kws / local_smo kernels of solver.cu)
 bool ws_solve_supported(int B, int64_t np_max);
+void launch_ws_smo(const SolverArgs& a, int P, cudaStream_t st);  // single-warp local SMO alone (B <= ws_smo_max_b)
+int ws_smo_max_b();
+int ws_tile_ld_of(int B);  // row stride of the K_ws,ws tile of the single-warp solver
 size_t ws_tile_floats(int B);  // per-pair floats of the Kws buffer (tile + SMO state)
 // Per-pair stride (floats) of the Kws buffer, the same for both solver paths: one graph may run
 // wsolve.cu pairs (tile with row stride round_up(B, 4) + alpha/f/index state) next to solver.cu

@@ -78,6 +78,9 @@ struct Model {
   std::vector<uint8_t> trained;      // [P]
   std::vector<double> b, A, B;       // [P]
   std::vector<int32_t> status;       // [P] solver status (0 ok, 2 outer cap) | sigmoid status << 8
+  // [P] telemetry of the training run (0 for models built from alpha / deserialised): outer
+  // iterations, inner SMO steps, kernel rows computed (ROW_CACHE regime; 0 in FULL_K)
+  std::vector<int64_t> pair_outer, pair_inner, pair_rows;
   std::vector<double> alpha;         // [sum_p n_p] pair-local order, all pairs (0 for untrained)
   bool alpha_ready = true;           // false: alpha still only on the device (ensure_host_alpha)
   std::vector<int64_t> sv_pos;       // class-sorted positions of the SV union, ascending

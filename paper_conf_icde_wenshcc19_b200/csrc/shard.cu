@@ -35,6 +35,8 @@ namespace gmpsvm {
 
 namespace {
 
+constexpr int kCandChunk = 16384;  // slice elements per candidate CTA
+
 // candidate source over the slice [lo, lo + len) of the pair (alpha / f full pair-local vectors)
 struct SliceSrc {
   const double* al;
@@ -60,11 +62,20 @@ struct SliceSrc {
 };
 
 // out (doubles): [fmin, fmax, nU, nL, U key bits x need, U index x need, L key bits x need, L index x need]
-__global__ void __launch_bounds__(1024) shard_cand_kernel(const double* al, const double* fl, const uint8_t* ret,
-                                                          uint32_t* st, uint32_t stamp0, int64_t lo, int len, int n_s,
-                                                          double C, int need, int stride, int32_t* tmp, double* out) {
+// grid: one CTA per chunk of the slice (chunk elements each), CTA c writing sub-block c
+__global__ void __launch_bounds__(1024) shard_cand_kernel(const double* al, const double* fl, const uint8_t* ret_all,
+                                                          uint32_t* st_all, uint32_t stamp0, int64_t lo_all, int len_all,
+                                                          int chunk, int n_s, double C, int need, int stride,
+                                                          int32_t* tmp_all, double* out_all) {
   __shared__ SelSmem sm;
   __shared__ double red[32];
+  const int c0 = blockIdx.x * chunk;
+  const int len = max(0, min(chunk, len_all - c0));
+  const int64_t lo = lo_all + c0;
+  const uint8_t* ret = ret_all + c0;
+  uint32_t* st = st_all + c0;
+  int32_t* tmp = tmp_all + (int64_t)blockIdx.x * 2 * need;
+  double* out = out_all + (int64_t)blockIdx.x * (4 + 4 * stride);
   double fmin = DBL_MAX, fmax = -DBL_MAX;
   for (int i = threadIdx.x; i < len; i += blockDim.x) {
     const int64_t j = lo + i;
@@ -125,21 +136,28 @@ __global__ void shard_place_rows_kernel(const float* tmp, int64_t ldt, const int
     dst[j] = src[j];
 }
 
-// f_j += sum_{e : dcoef_e != 0} dcoef_e R[slot_e][j - lo] over the slice, FP64, rows in position order
-__global__ void shard_fupdate_kernel(const double* dcoef, const int32_t* slot, int wn, const float* R, int64_t ldr,
-                                     int64_t lo, int64_t len, double* f) {
-  __shared__ double cf[1024];
-  __shared__ int32_t sl[1024];
-  __shared__ int nz;
+// the rows with dalpha != 0, in position order: nzl = [count, (coef, slot) ...]
+__global__ void shard_nz_kernel(const double* dcoef, const int32_t* slot, int wn, double* nzc, int32_t* nzs, int* nzn) {
   if (threadIdx.x == 0) {
     int c = 0;
     for (int e = 0; e < wn; ++e)
       if (dcoef[e] != 0.0) {
-        cf[c] = dcoef[e];
-        sl[c] = slot[e];
+        nzc[c] = dcoef[e];
+        nzs[c] = slot[e];
         ++c;
       }
-    nz = c;
+    *nzn = c;
+  }
+}
+// f_j += sum_{e : dcoef_e != 0} dcoef_e R[slot_e][j - lo] over the slice, FP64, rows in position order
+__global__ void shard_fupdate_kernel(const double* nzc, const int32_t* nzs, const int* nzn, const float* R, int64_t ldr,
+                                     int64_t lo, int64_t len, double* f) {
+  __shared__ double cf[1024];
+  __shared__ int32_t sl[1024];
+  const int nz = *nzn;
+  for (int r = threadIdx.x; r < nz; r += blockDim.x) {
+    cf[r] = nzc[r];
+    sl[r] = nzs[r];
   }
   __syncthreads();
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -158,6 +176,18 @@ __global__ void shard_fws_kernel(const double* f, const int32_t* ws, int wn, int
 __global__ void shard_scatter_fws_kernel(const double* fws, const int32_t* ws, int wn, double* f) {
   const int e = blockIdx.x * blockDim.x + threadIdx.x;
   if (e < wn) f[ws[e]] = fws[e];
+}
+// the single-warp solver's state behind the tile: alpha, f, index of the working set (sorted order)
+__global__ void shard_state_kernel(const double* alpha, const double* fws, const int32_t* ws, int wn, float* buf,
+                                   size_t state_off, int B) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= wn) return;
+  double* st_al = reinterpret_cast<double*>(buf + state_off);
+  double* st_f = st_al + B;
+  int32_t* st_ix = reinterpret_cast<int32_t*>(st_f + B);
+  st_al[e] = alpha[ws[e]];
+  st_f[e] = fws[e];
+  st_ix[e] = ws[e];
 }
 __global__ void shard_init_kernel(double* alpha, double* f, int64_t np, int n_s) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -190,11 +220,15 @@ struct Shard {
   DevBuf<double> alpha, f, cand, v, dcoef, fws, bb, AA, BB, gapv;
   DevBuf<uint8_t> ret;
   DevBuf<uint32_t> stamp;
-  DevBuf<int32_t> tmp, d_ws, d_slot, d_status, d_wsn, d_inner, d_outer, d_sig;
+  DevBuf<int32_t> tmp, d_ws, d_slot, d_status, d_wsn, d_inner, d_outer, d_sig, nzs, nzn;
+  DevBuf<double> nzc;
   DevBuf<int64_t> d_inner64, d_cyc;
   DevBuf<PairDesc> d_pair;
   uint32_t stampv = 1;
-  int cand_doubles() const { return 4 + 4 * need_max; }
+  int chunks = 1;  // candidate CTAs (sub-blocks) per rank: the same count on every rank
+  bool warp_smo() const { return B <= ws_smo_max_b(); }  // wsolve.cu's single-warp solver, tile in smem
+  int tile_ld() const { return warp_smo() ? ws_tile_ld_of(B) : B; }
+  int cand_doubles() const { return chunks * (4 + 4 * need_max); }
 };
 
 static SolverArgs shard_args(Shard& S) {
@@ -275,6 +309,7 @@ Shard* shard_create(const float* X, const int32_t* y, int64_t n, int32_t d, int3
   S->lo = std::min(S->np, per * rank);
   S->hi = std::min(S->np, S->lo + per);
   S->len = S->hi - S->lo;
+  S->chunks = (int)std::max<int64_t>(1, ceil_div(per, kCandChunk));
   S->ldr = round_up(std::max<int64_t>(S->len, 1), 4);
   S->d_pad = (int)round_up(d, kBK);
   S->ldx = round_up(S->np, kTile) + kTile;  // + a tile: column tiles starting at lo stay in bounds
@@ -310,7 +345,10 @@ Shard* shard_create(const float* X, const int32_t* y, int64_t n, int32_t d, int3
   new (&S->gapv) DevBuf<double>(1, st);
   new (&S->ret) DevBuf<uint8_t>(std::max<int64_t>(S->len, 1), st);
   new (&S->stamp) DevBuf<uint32_t>(std::max<int64_t>(S->len, 1), st);
-  new (&S->tmp) DevBuf<int32_t>(2 * S->B, st);
+  new (&S->tmp) DevBuf<int32_t>((size_t)2 * S->B * S->chunks, st);
+  new (&S->nzs) DevBuf<int32_t>(S->B, st);
+  new (&S->nzn) DevBuf<int32_t>(1, st);
+  new (&S->nzc) DevBuf<double>(S->B, st);
   new (&S->d_ws) DevBuf<int32_t>(S->B, st);
   new (&S->d_slot) DevBuf<int32_t>(S->B, st);
   new (&S->d_status) DevBuf<int32_t>(1, st);
@@ -371,8 +409,9 @@ void shard_candidates(Shard* S, double* out) {
   GM_CUDA(cudaMemcpyAsync(S->ret.get(), r.data(), r.size(), cudaMemcpyHostToDevice, st));
   const int need = S->np <= S->B ? 0 : S->B - (int)kept.size();
   GM_CUDA(cudaMemsetAsync(S->cand.get(), 0, (size_t)S->cand_doubles() * 8, st));
-  GM_LAUNCH(shard_cand_kernel, dim3(1), dim3(1024), 0, st, S->alpha.get(), S->f.get(), S->ret.get(), S->stamp.get(),
-            S->stampv, S->lo, (int)S->len, (int)S->n_s, S->C, need, S->need_max, S->tmp.get(), S->cand.get());
+  GM_LAUNCH(shard_cand_kernel, dim3((unsigned)S->chunks), dim3(1024), 0, st, S->alpha.get(), S->f.get(), S->ret.get(),
+            S->stamp.get(), S->stampv, S->lo, (int)S->len, kCandChunk, (int)S->n_s, S->C, need, S->need_max,
+            S->tmp.get(), S->cand.get());
   S->stampv += 2;
   GM_CUDA(cudaMemcpyAsync(out, S->cand.get(), (size_t)S->cand_doubles() * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
@@ -440,7 +479,7 @@ int shard_select(Shard* S, const double* all, int32_t* stop) {
   const std::vector<int32_t> kept = retained(*S);
   const int need = S->np <= S->B ? 0 : S->B - (int)kept.size();
   std::vector<int32_t> picks;
-  const double gap = shard_merge(all, S->world, S->cand_doubles(), need, need / 2, picks);
+  const double gap = shard_merge(all, S->world * S->chunks, 4 + 4 * S->need_max, need, need / 2, picks);
   S->gap = gap;
   if (!(gap >= S->eps)) {
     S->status = 1;
@@ -512,7 +551,7 @@ int shard_select(Shard* S, const double* all, int32_t* stop) {
   GM_LAUNCH(shard_gather_kernel, dim3((unsigned)ceil_div(ldat, 128), 64), dim3(128), 0, st, S->XT.get(), S->ldx,
             S->nx.get(), S->d_ws.get(), wn, S->d_pad, S->AT.get(), (int64_t)ldat, S->na.get());
   launch_krow_rect(S->AT.get(), ldat, S->na.get(), wn, S->AT.get(), ldat, S->na.get(), wn, S->d_pad, S->gamma,
-                   S->Kws.get(), S->B, st);
+                   S->Kws.get(), S->tile_ld(), st);
   GM_CUDA(cudaMemcpyAsync(S->d_slot.get(), slot.data(), (size_t)wn * 4, cudaMemcpyHostToDevice, st));
   GM_CUDA(cudaStreamSynchronize(st));
   return GMPSVM_OK;
@@ -536,10 +575,20 @@ void shard_step(Shard* S, const double* fws_sum) {
   GM_LAUNCH(shard_scatter_fws_kernel, dim3((unsigned)ceil_div(std::max(wn, 1), 256)), dim3(256), 0, st, S->fws.get(),
             S->d_ws.get(), wn, S->f.get());
   SolverArgs a = shard_args(*S);
-  launch_local_smo(a, 1, st);  // the same local solve on every rank (alpha stays replicated)
-  if (S->len > 0)
-    GM_LAUNCH(shard_fupdate_kernel, dim3((unsigned)ceil_div(S->len, 256)), dim3(256), 0, st, S->dcoef.get(),
-              S->d_slot.get(), wn, S->R.get(), S->ldr, S->lo, S->len, S->f.get());
+  // the same local solve on every rank (alpha stays replicated)
+  if (S->warp_smo()) {
+    GM_LAUNCH(shard_state_kernel, dim3((unsigned)ceil_div(std::max(wn, 1), 256)), dim3(256), 0, st, S->alpha.get(),
+              S->fws.get(), S->d_ws.get(), wn, S->Kws.get(), (size_t)S->B * S->tile_ld(), S->B);
+    launch_ws_smo(a, 1, st);
+  } else {
+    launch_local_smo(a, 1, st);
+  }
+  if (S->len > 0) {
+    GM_LAUNCH(shard_nz_kernel, dim3(1), dim3(32), 0, st, S->dcoef.get(), S->d_slot.get(), wn, S->nzc.get(), S->nzs.get(),
+              S->nzn.get());
+    GM_LAUNCH(shard_fupdate_kernel, dim3((unsigned)ceil_div(S->len, 256)), dim3(256), 0, st, S->nzc.get(), S->nzs.get(),
+              S->nzn.get(), S->R.get(), S->ldr, S->lo, S->len, S->f.get());
+  }
   GM_CUDA(cudaStreamSynchronize(st));
 }
 

@@ -973,6 +973,24 @@ static void ws_configure() {
   smo_configure<7>(mx);
 }
 
+// The single-warp local SMO alone (the sharded pair solver, shard.cu): each pair's K_ws,ws tile
+// (row stride ws_tile_ld(B)) and state (alpha, f, index; sorted order) in the ws_write_out layout.
+void launch_ws_smo(const SolverArgs& a, int P, cudaStream_t st) {
+  ws_configure();
+  const size_t smo_dyn = ws_smo_smem(a.B);
+  switch ((a.B + 31) / 32) {
+    case 1: launch_smo<1>(a, P, smo_dyn, st); break;
+    case 2: launch_smo<2>(a, P, smo_dyn, st); break;
+    case 3: launch_smo<3>(a, P, smo_dyn, st); break;
+    case 4: launch_smo<4>(a, P, smo_dyn, st); break;
+    case 5: launch_smo<5>(a, P, smo_dyn, st); break;
+    case 6: launch_smo<6>(a, P, smo_dyn, st); break;
+    default: launch_smo<7>(a, P, smo_dyn, st); break;
+  }
+}
+int ws_smo_max_b() { return kWMaxB; }
+int ws_tile_ld_of(int B) { return ws_tile_ld(B); }
+
 void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int set_cond,
                          int64_t max_outer, cudaStream_t st, bool chained) {
   ws_configure();
