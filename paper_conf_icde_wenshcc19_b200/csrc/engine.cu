@@ -151,6 +151,15 @@ struct KCacheEntry {
 std::mutex g_kcache_mu;
 std::vector<KCacheEntry> g_kcache[64];
 
+// bytes of the cached kernel-matrix workspaces of a device (reusable by the next run)
+size_t kcache_bytes(int dev) {
+  std::lock_guard<std::mutex> lk(g_kcache_mu);
+  size_t b = 0;
+  for (const auto& e : g_kcache[dev])
+    if (!e.busy) b += e.bytes;
+  return b;
+}
+
 struct KWorkspace {
   int dev;
   size_t slot = (size_t)-1;
@@ -927,11 +936,24 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // solver.cu kernels, where the paper's B = 1024, q = 512 (L377) cuts the outer iterations 4-40x
   // (measured: covtype-shaped 581k 0.41 -> 0.20 s, MNIST8M-shaped 1M 15.9 -> 5.1 s): the largest
   // of 1024 / 512 / 256 whose ROW_CACHE row buffers fit the budget (else 192).
+  // ROW_CACHE: the row buffers must fit next to what is already allocated (X, its staged copy):
+  // the free device memory now (+ a cached kernel-matrix workspace this call may reuse), less a
+  // 4 GB margin for the solver's other buffers
+  double rc_avail = 0.0;
+  if (!full_k) {
+    size_t fr = 0, tt = 0;
+    cudaMemPool_t pool;  // memory the stream-ordered pool holds but does not use goes back first
+    GM_CUDA(cudaStreamSynchronize(st));
+    GM_CUDA(cudaDeviceGetDefaultMemPool(&pool, opt.device));
+    GM_CUDA(cudaMemPoolTrimTo(pool, 0));
+    GM_CUDA(cudaMemGetInfo(&fr, &tt));
+    rc_avail = std::min((double)fr + (double)kcache_bytes(opt.device) - 4e9, 0.85 * (double)device_total_mem(opt.device));
+  }
   if (!opt.ws_size && np_max > kWsMaxNp) {
-    for (int cand : {1024, 512, 256}) {
+    for (int cand : {1024, 512, 256, 128}) {
       double r = 0;
       for (const auto& x : hp) r += (double)cand * round_up(x.n_s + x.n_t, 4) * 4.0;
-      if (full_k || r + (double)Pl * d_pad * round_up(cand, kTile) * 4.0 <= 0.85 * (double)device_total_mem(opt.device)) {
+      if (full_k || r + (double)Pl * d_pad * round_up(cand, kTile) * 4.0 <= rc_avail) {
         B = cand;
         break;
       }
@@ -949,7 +971,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   }
   if (!full_k) {
     const double rc_total = bytes_R + (double)Pl * d_pad * ldat * 4.0;
-    if (rc_total > 0.85 * (double)device_total_mem(opt.device))
+    if (rc_total > rc_avail)
       throw Error(GMPSVM_ENOTIMPL, "ROW_CACHE buffers (" + std::to_string(rc_total / 1e9) +
                                        " GB) exceed the device memory; train the pairs in parts (pair_ids) and merge");
   }

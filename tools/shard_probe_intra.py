@@ -65,8 +65,8 @@ def shard_run(world, max_iters=None):
     blk = sh.cand_doubles
     empty = np.zeros(blk)
     sub = 4 + 4 * sh.ws_size
-    for c in range(blk // sub):  # an empty sub-block: no candidates, neutral min / max
-        empty[c * sub], empty[c * sub + 1] = np.finfo(np.float64).max, -np.finfo(np.float64).max
+    for c in range(blk // sub):  # a peer sub-block without candidates whose I_l keeps the gap open
+        empty[c * sub], empty[c * sub + 1] = np.finfo(np.float64).max, 1e300
     it, t_iter = 0, []
     while max_iters is None or it < max_iters:
         ta = time.perf_counter()
@@ -82,9 +82,25 @@ def shard_run(world, max_iters=None):
 
 sh1, O, t1 = shard_run(1)
 res1 = sh1.finish(sh1.f_slice())
+# the same pair's kernel rows on their own: q rows x the pair's n_p columns (rectangular SIMT
+# contraction, as rows_contract / the sharded solver run it), timed on the device
+idx = np.concatenate([np.flatnonzero(y == s), np.flatnonzero(y == t)])
+Xp = torch.from_numpy(X[idx]).to(dev)
+rows = Xp[:ws // 2].contiguous()
+gm.rbf_kernel(rows, Xp, spec.gamma)
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record()
+for _ in range(5):
+    gm.rbf_kernel(rows, Xp, spec.gamma)
+e1.record()
+torch.cuda.synchronize()
+rows_ms = e0.elapsed_time(e1) / 5
+rows_tflops = (ws // 2) * len(idx) * (2 * spec.d + 3) / (rows_ms * 1e-3) / 1e12
 out = {"config": name, "n_train": n, "ws_size": ws, "coll_us_assumed": coll_us, "T1_s": T1,
        "hard_pair": list(pairs[hard]), "hard_pair_main_solver": iters[hard],
-       "hard_pair_sharded_world1": {"outer": O, "s": sum(t1), "per_iter_ms": 1e3 * float(np.median(t1))},
+       "hard_pair_sharded_world1": {"outer": O, "inner": res1["inner_iters"], "s": sum(t1),
+                                    "per_iter_ms": 1e3 * float(np.median(t1))},
+       "rows_contract_isolated": {"rows": ws // 2, "cols": int(len(idx)), "ms": rows_ms, "tflops": rows_tflops},
        "estimates": {}}
 print(f"sharded solver world 1: {O} outer iterations, {sum(t1):.3f} s", flush=True)
 for N in (2, 4, 8):
