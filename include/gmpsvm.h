@@ -216,13 +216,16 @@ GMPSVM_API int gmpsvm_model_from_alpha(const float* X, const int32_t* y, int64_t
  * holds X (replicated) and owns the slice [lo, hi) of the pair's instances (pair-local order:
  * class s, then class t).  Per outer iteration the caller runs, on every rank, with its own
  * collectives (torch.distributed; paper_conf_icde_wenshcc19_b200/dist.py train_pair_sharded):
- *   gmpsvm_shard_candidates(sh, c)          c: this rank's block of gmpsvm_shard_cand_doubles
+ *   gmpsvm_shard_candidates(sh, c)          once before the loop; c: this rank's block of
+ *                                           gmpsvm_shard_cand_doubles
  *   all_gather(c) -> all [world x cand_doubles], rank order
- *   gmpsvm_shard_select(sh, all, &stop)     identical merge on every rank; stop = 1: converged
- *                                           (Eq 9 with tolerance eps) or the outer cap
- *   gmpsvm_shard_fws(sh, fws)               fws: B doubles, f of the members this rank owns
+ *   gmpsvm_shard_select(sh, all, &stop, fws)  identical merge on every rank; stop = 1: converged
+ *                                           (Eq 9 with tolerance eps) or the outer cap; fws (B
+ *                                           doubles, may be NULL): f of the members this rank owns
  *   all_reduce_sum(fws)
- *   gmpsvm_shard_step(sh, fws)              local SMO (same on every rank) + f update of the slice
+ *   gmpsvm_shard_step(sh, fws, c)           local SMO (same on every rank) + f update of the slice;
+ *                                           c (may be NULL): the next iteration's candidates
+ * (one device round trip per collective; gmpsvm_shard_fws gives fws separately.)
  * then gathers every rank's f slice (gmpsvm_shard_f, rank order) and calls gmpsvm_shard_finish
  * for alpha (n_p, pair-local order), b, A, B and the status word of gmpsvm_model_pair.  All
  * buffers are host pointers.  world = 1 is a complete single-rank solver; any world gives
@@ -235,9 +238,9 @@ GMPSVM_API int gmpsvm_shard_create(const float* X, const int32_t* y, int64_t n, 
 GMPSVM_API int32_t gmpsvm_shard_cand_doubles(const gmpsvm_shard* sh);
 GMPSVM_API int gmpsvm_shard_slice(const gmpsvm_shard* sh, int64_t* lo, int64_t* hi, int64_t* n_p, int32_t* ws_size);
 GMPSVM_API int gmpsvm_shard_candidates(gmpsvm_shard* sh, double* out);
-GMPSVM_API int gmpsvm_shard_select(gmpsvm_shard* sh, const double* all, int32_t* stop);
+GMPSVM_API int gmpsvm_shard_select(gmpsvm_shard* sh, const double* all, int32_t* stop, double* fws_out);
 GMPSVM_API int gmpsvm_shard_fws(gmpsvm_shard* sh, double* fws);
-GMPSVM_API int gmpsvm_shard_step(gmpsvm_shard* sh, const double* fws_sum);
+GMPSVM_API int gmpsvm_shard_step(gmpsvm_shard* sh, const double* fws_sum, double* cand_out);
 GMPSVM_API int gmpsvm_shard_f(gmpsvm_shard* sh, double* f_slice);
 GMPSVM_API int gmpsvm_shard_finish(gmpsvm_shard* sh, const double* f_full, double* alpha, double* b, double* A,
                                    double* B, int32_t* status, int64_t* outer_iters, int64_t* inner_iters);

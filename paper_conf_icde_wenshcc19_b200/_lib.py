@@ -92,9 +92,9 @@ _SIGS = {
     "gmpsvm_shard_cand_doubles": (ct.c_int32, [_P]),
     "gmpsvm_shard_slice": (ct.c_int, [_P, _P, _P, _P, _P]),
     "gmpsvm_shard_candidates": (ct.c_int, [_P, _P]),
-    "gmpsvm_shard_select": (ct.c_int, [_P, _P, _P]),
+    "gmpsvm_shard_select": (ct.c_int, [_P, _P, _P, _P]),
     "gmpsvm_shard_fws": (ct.c_int, [_P, _P]),
-    "gmpsvm_shard_step": (ct.c_int, [_P, _P]),
+    "gmpsvm_shard_step": (ct.c_int, [_P, _P, _P]),
     "gmpsvm_shard_f": (ct.c_int, [_P, _P]),
     "gmpsvm_shard_finish": (ct.c_int, [_P, _P, _P, _P, _P, _P, _P, _P, _P]),
     "gmpsvm_shard_free": (None, [_P]),
@@ -429,20 +429,25 @@ class Shard:
         _check(lib().gmpsvm_shard_candidates(self.h, out.ctypes.data))
         return out
 
-    def select(self, all_cands):
+    def select(self, all_cands, want_fws=False):
+        """The merge; returns stop, or (stop, this rank's f of the new working set) with want_fws."""
         a = np.ascontiguousarray(all_cands, dtype=np.float64)
         stop = ct.c_int32()
-        _check(lib().gmpsvm_shard_select(self.h, a.ctypes.data, ct.byref(stop)))
-        return bool(stop.value)
+        fw = np.zeros(self.ws_size) if want_fws else None
+        _check(lib().gmpsvm_shard_select(self.h, a.ctypes.data, ct.byref(stop), fw.ctypes.data if want_fws else None))
+        return (bool(stop.value), fw) if want_fws else bool(stop.value)
 
     def fws(self):
         out = np.zeros(self.ws_size)
         _check(lib().gmpsvm_shard_fws(self.h, out.ctypes.data))
         return out
 
-    def step(self, fws_sum):
+    def step(self, fws_sum, want_cands=False):
+        """Local SMO + f update; with want_cands the next iteration's candidate block."""
         a = np.ascontiguousarray(fws_sum, dtype=np.float64)
-        _check(lib().gmpsvm_shard_step(self.h, a.ctypes.data))
+        c = np.zeros(self.cand_doubles) if want_cands else None
+        _check(lib().gmpsvm_shard_step(self.h, a.ctypes.data, c.ctypes.data if want_cands else None))
+        return c
 
     def f_slice(self):
         out = np.zeros(self.hi - self.lo)

@@ -509,10 +509,10 @@ int gmpsvm_shard_candidates(gmpsvm_shard* sh, double* out) {
     return GMPSVM_OK;
   });
 }
-int gmpsvm_shard_select(gmpsvm_shard* sh, const double* all, int32_t* stop) {
+int gmpsvm_shard_select(gmpsvm_shard* sh, const double* all, int32_t* stop, double* fws_out) {
   return guarded([&]() {
     if (!sh || !all || !stop) throw Error(GMPSVM_EINVAL, "null argument");
-    return gmpsvm::shard_select(sh->s, all, stop);
+    return gmpsvm::shard_select(sh->s, all, stop, fws_out);
   });
 }
 int gmpsvm_shard_fws(gmpsvm_shard* sh, double* fws) {
@@ -522,10 +522,10 @@ int gmpsvm_shard_fws(gmpsvm_shard* sh, double* fws) {
     return GMPSVM_OK;
   });
 }
-int gmpsvm_shard_step(gmpsvm_shard* sh, const double* fws_sum) {
+int gmpsvm_shard_step(gmpsvm_shard* sh, const double* fws_sum, double* cand_out) {
   return guarded([&]() {
     if (!sh || !fws_sum) throw Error(GMPSVM_EINVAL, "null argument");
-    gmpsvm::shard_step(sh->s, fws_sum);
+    gmpsvm::shard_step(sh->s, fws_sum, cand_out);
     return GMPSVM_OK;
   });
 }

@@ -126,9 +126,9 @@ void shard_free(Shard* S);
 int shard_cand_doubles(const Shard* S);
 void shard_slice(const Shard* S, int64_t* lo, int64_t* hi, int64_t* np, int32_t* ws_size);
 void shard_candidates(Shard* S, double* out);
-int shard_select(Shard* S, const double* all, int32_t* stop);
+int shard_select(Shard* S, const double* all, int32_t* stop, double* fws_out);
 void shard_fws(Shard* S, double* out);
-void shard_step(Shard* S, const double* fws_sum);
+void shard_step(Shard* S, const double* fws_sum, double* cand_out);
 void shard_f(Shard* S, double* out);
 int shard_finish(Shard* S, const double* f_full, double* alpha_out, double* b, double* A, double* Bsig, int32_t* status,
                  int64_t* outer, int64_t* inner);

@@ -399,8 +399,7 @@ static std::vector<int32_t> retained(const Shard& S) {
   return std::vector<int32_t>(S.ws_age.end() - keep, S.ws_age.end());
 }
 
-void shard_candidates(Shard* S, double* out) {
-  GM_CUDA(cudaSetDevice(S->device));
+static void cand_launch(Shard* S, double* out) {
   cudaStream_t st = S->st;
   const std::vector<int32_t> kept = retained(*S);
   std::vector<uint8_t> r(std::max<int64_t>(S->len, 1), 0);
@@ -414,7 +413,12 @@ void shard_candidates(Shard* S, double* out) {
             S->tmp.get(), S->cand.get());
   S->stampv += 2;
   GM_CUDA(cudaMemcpyAsync(out, S->cand.get(), (size_t)S->cand_doubles() * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaStreamSynchronize(st));
+}
+
+void shard_candidates(Shard* S, double* out) {
+  GM_CUDA(cudaSetDevice(S->device));
+  cand_launch(S, out);
+  GM_CUDA(cudaStreamSynchronize(S->st));
 }
 
 // The exact merge of every rank's candidate block (host, deterministic).  need / need_u: picks
@@ -473,7 +477,9 @@ double shard_merge(const double* all, int world, int cand_doubles, int need, int
   return fmax - fmin;
 }
 
-int shard_select(Shard* S, const double* all, int32_t* stop) {
+static void fws_launch(Shard* S, double* out);
+
+int shard_select(Shard* S, const double* all, int32_t* stop, double* fws_out) {
   GM_CUDA(cudaSetDevice(S->device));
   cudaStream_t st = S->st;
   const std::vector<int32_t> kept = retained(*S);
@@ -553,21 +559,26 @@ int shard_select(Shard* S, const double* all, int32_t* stop) {
   launch_krow_rect(S->AT.get(), ldat, S->na.get(), wn, S->AT.get(), ldat, S->na.get(), wn, S->d_pad, S->gamma,
                    S->Kws.get(), S->tile_ld(), st);
   GM_CUDA(cudaMemcpyAsync(S->d_slot.get(), slot.data(), (size_t)wn * 4, cudaMemcpyHostToDevice, st));
+  if (fws_out) fws_launch(S, fws_out);  // this rank's f of the new working set, same round trip
   GM_CUDA(cudaStreamSynchronize(st));
   return GMPSVM_OK;
 }
 
-void shard_fws(Shard* S, double* out) {
-  GM_CUDA(cudaSetDevice(S->device));
+static void fws_launch(Shard* S, double* out) {
   const int wn = (int)S->ws.size();
   GM_LAUNCH(shard_fws_kernel, dim3((unsigned)ceil_div(std::max(wn, 1), 256)), dim3(256), 0, S->st, S->f.get(),
             S->d_ws.get(), wn, S->lo, S->hi, S->fws.get());
   std::memset(out, 0, (size_t)S->B * 8);
   if (wn) GM_CUDA(cudaMemcpyAsync(out, S->fws.get(), (size_t)wn * 8, cudaMemcpyDeviceToHost, S->st));
+}
+
+void shard_fws(Shard* S, double* out) {
+  GM_CUDA(cudaSetDevice(S->device));
+  fws_launch(S, out);
   GM_CUDA(cudaStreamSynchronize(S->st));
 }
 
-void shard_step(Shard* S, const double* fws_sum) {
+void shard_step(Shard* S, const double* fws_sum, double* cand_out) {
   GM_CUDA(cudaSetDevice(S->device));
   cudaStream_t st = S->st;
   const int wn = (int)S->ws.size();
@@ -589,6 +600,7 @@ void shard_step(Shard* S, const double* fws_sum) {
     GM_LAUNCH(shard_fupdate_kernel, dim3((unsigned)ceil_div(S->len, 256)), dim3(256), 0, st, S->nzc.get(), S->nzs.get(),
               S->nzn.get(), S->R.get(), S->ldr, S->lo, S->len, S->f.get());
   }
+  if (cand_out) cand_launch(S, cand_out);  // the next iteration's candidates, same round trip
   GM_CUDA(cudaStreamSynchronize(st));
 }
 

@@ -181,15 +181,17 @@ def train_pair_sharded(X, y, k, s, t, C, gamma, eps, group=None, **opts):
     rank = dist.get_rank(group)
     dev = _backend_device(group)
     sh = gm.Shard(X, y, k, s, t, C, gamma, eps, rank, world, **opts)
-    while True:
-        c = torch.from_numpy(sh.candidates()).to(dev)
+    cand = sh.candidates()
+    while True:  # one device round trip per collective
+        c = torch.from_numpy(cand).to(dev)
         outs = [torch.empty_like(c) for _ in range(world)]
         dist.all_gather(outs, c, group=group)
-        if sh.select(torch.stack(outs).cpu().numpy()):
+        stop, fws = sh.select(torch.stack(outs).cpu().numpy(), want_fws=True)
+        if stop:
             break
-        fw = torch.from_numpy(sh.fws()).to(dev)
+        fw = torch.from_numpy(fws).to(dev)
         dist.all_reduce(fw, op=dist.ReduceOp.SUM, group=group)
-        sh.step(fw.cpu().numpy())
+        cand = sh.step(fw.cpu().numpy(), want_cands=True)
     f_full = np.concatenate(_all_gather_f64(sh.f_slice(), group))
     return sh.finish(f_full)
 

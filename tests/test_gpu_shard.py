@@ -89,7 +89,7 @@ def gm():
 
 def _single_rank(gm, X, y, k, s, t, C, gamma, ws):
     sh = gm.Shard(X, y, k, s, t, C, gamma, EPS, 0, 1, ws_size=ws)
-    while True:
+    while True:  # the separate calls (candidates / select / fws / step) give the same iterates
         if sh.select(sh.candidates()[None, :]):
             break
         sh.step(sh.fws())

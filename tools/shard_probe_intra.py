@@ -68,13 +68,13 @@ def shard_run(world, max_iters=None):
     for c in range(blk // sub):  # a peer sub-block without candidates whose I_l keeps the gap open
         empty[c * sub], empty[c * sub + 1] = np.finfo(np.float64).max, 1e300
     it, t_iter = 0, []
+    c = sh.candidates()
     while max_iters is None or it < max_iters:
         ta = time.perf_counter()
-        c = sh.candidates()
-        allc = np.concatenate([c] + [empty] * (world - 1))
-        if sh.select(allc):
+        stop, fw = sh.select(np.concatenate([c] + [empty] * (world - 1)), want_fws=True)
+        if stop:
             break
-        sh.step(sh.fws())
+        c = sh.step(fw, want_cands=True)
         t_iter.append(time.perf_counter() - ta)
         it += 1
     return sh, it, t_iter
