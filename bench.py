@@ -354,11 +354,31 @@ def run_gpu(args, spec):
                     "train_total_ms": e2e_train.get("t_total_ms"), "train_stage_ms": e2e_train.get("t_stage_ms"),
                     "predict_total_ms": e2e_pred["t_total_ms"], "predict_stage_ms": e2e_pred["t_stage_ms"]},
         }
+        # the int8-digit decision-value contraction (dec_i8.cu): executed int8 tensor-core work =
+        # 19 digit products x 2 d ops per (test row, SV); peak = int8 dense = 2 x the measured bf16
+        if ps.get("dec_path", -1) == 1 and ps["t_decision_ms"] > 0:
+            i8_ops = X.shape[1] * 2.0 * 19 * Xt.shape[0] * s["n_sv"]
+            i8_peak = 2.0 * bf16
+            line["dec_roofline"] = {"kernel": "dec_i8_kernel (tcgen05 kind::i8, 5 int8 digit planes, 19 products)",
+                                    "bound": "tensor", "achieved": i8_ops / (ps["t_decision_ms"] * 1e-3) / 1e12,
+                                    "peak": i8_peak, "unit": "TOP/s (int8)",
+                                    "frac": i8_ops / (ps["t_decision_ms"] * 1e-3) / 1e12 / i8_peak,
+                                    "decision_ms": ps["t_decision_ms"],
+                                    "algorithmic_tflops": ps["dec_flops"] / (ps["t_decision_ms"] * 1e-3) / 1e12}
         if not args.no_cpu_baseline and ws == 1:
             v, tt, tp, cores = cpu_sample(spec, args.eps)
             line["cpu_baseline"] = {"value": v, "unit": "s (sample)", "cores": cores, "kind": "oracle",
                                     "sample": f"6000 train / 1000 test MNIST-shaped rows (10% of the workload), "
                                               f"eps={args.eps:g}: train {tt:.1f} s + predict {tp:.1f} s"}
+        full_ref = os.path.join(ROOT, "profiles", "r02", "cpu_full_mnist_r02.json")
+        if os.path.exists(full_ref) and spec.name == "mnist":
+            # the oracle once on the FULL workload on a GPU box's host (tools/cpu_full.py, committed:
+            # ~2 minutes on 16 threads, too long to repeat in every bench run)
+            fr = json.load(open(full_ref))
+            line["cpu_baseline_full"] = {"value": fr["total_s"], "unit": "s", "train_s": fr["train_s"],
+                                         "predict_s": fr["predict_s"], "cores": fr["threads"],
+                                         "cpu_model": fr["cpu_model"], "kind": "oracle",
+                                         "source": "profiles/r02/cpu_full_mnist_r02.json (tools/cpu_full.py)"}
         print(json.dumps(line), flush=True)
     if ws > 1:
         dist.destroy_process_group()

@@ -833,14 +833,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // tens of milliseconds, so it is not queried per call)
   const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)device_total_mem(opt.device);
   const bool full_k = bytes_K <= budget;
-  const bool use_tc = full_k && krow_use_tc();
+  // tensor cores for the kernel values: FULL_K always; ROW_CACHE rows for the Gaussian with the
+  // FP16 split (rows_tc_kernel); the SIMT contraction otherwise (GMPSVM_KROW=simt)
+  const bool use_tc = krow_use_tc() && (full_k || (ktype == 0 && krow_split_f16()));
   if (ktype != 0 && !(use_tc && krow_split_f16()))
     throw Error(GMPSVM_ENOTIMPL, "the linear / polynomial / sigmoid kernels need the FULL_K regime on the tensor cores");
   const int d_pad = use_tc ? krow_tc_d_pad(d) : (int)round_up(d, kBK);
   // ROW_CACHE column tiles start at 4-aligned segment starts and may run 127 columns past n
   const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile) + (full_k ? 0 : kTile);
-  // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split
-  DevBuf<float> XT(use_tc ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad, st);
+  // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split.
+  // norms: + one tile of zeros (ROW_CACHE column tiles run up to 127 columns past n)
+  DevBuf<float> XT(use_tc ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad + kTile, st);
+  GM_CUDA(cudaMemsetAsync(norms.get() + n_pad, 0, kTile * sizeof(float), st));
   DevBuf<float> Xhi(use_tc ? krow_tc_buf_floats(n_pad, d_pad) : 0, st), Xlo(use_tc ? krow_tc_buf_floats(n_pad, d_pad) : 0, st);
   float ksc = 1.f;  // scale of the split (FP16: exact power of two)
   DevBuf<int32_t> bad(1, st);
@@ -1104,8 +1108,11 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
   DevBuf<float> d_Kws((size_t)Pl * kws_pair_stride(Bw), st);
   const bool rc = !full_k;
+  const bool rc_tc = rc && use_tc;  // ROW_CACHE rows on tcgen05
+  DevBuf<float> d_Ahi(rc_tc ? krow_tc_buf_floats((int64_t)Pl * ldat, d_pad) : 0, st),
+      d_Alo(rc_tc ? krow_tc_buf_floats((int64_t)Pl * ldat, d_pad) : 0, st);
   DevBuf<int32_t> d_slot(rc ? (size_t)Pl * Bw : 0, st), d_slot_tmp(rc ? (size_t)Pl * Bw : 0, st), d_keep(rc ? Pl : 0, st);
-  DevBuf<float> d_ATnew(rc ? (size_t)Pl * d_pad * ldat : 0, st);
+  DevBuf<float> d_ATnew(rc && !rc_tc ? (size_t)Pl * d_pad * ldat : 0, st);
   DevBuf<int64_t> d_rows(rc ? Pl : 0, st);
   if (rc) GM_CUDA(cudaMemsetAsync(d_rows.get(), 0, Pl * 8, st));
   SolverArgs a{};
@@ -1123,6 +1130,15 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   a.ATnew = d_ATnew.get();
   a.d_pad = d_pad;
   a.ldat = ldat;
+  if (rc_tc) {
+    a.Xhi = Xhi.get();
+    a.Xlo = Xlo.get();
+    a.Ahi = d_Ahi.get();
+    a.Alo = d_Alo.get();
+    a.dpt = d_pad;
+    a.n_pad = n_pad;
+    a.kscale = (float)(-gamma * 1.4426950408889634 / ((double)ksc * (double)ksc));
+  }
   a.gamma = gamma;
   a.alpha = d_alpha.get();
   a.f = d_f.get();
@@ -1181,6 +1197,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   HT("init");
   int64_t rc_launches = 0;  // ROW_CACHE row-contraction launches
   GraphGuard gg;
+  DevBuf<int4> d_rtiles;  // ROW_CACHE tcgen05 row tiles of every branch (outlives the graph run)
   int64_t body_launches = 0;
   std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
   int n_branches = 0, final_selects = 0;
@@ -1200,6 +1217,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
       const int m = Pl / nbr, r = Pl % nbr;  // the last r branches take m + 1 pairs
       for (int b = 0; b < nbr; ++b) bb[b + 1] = bb[b] + m + (b >= nbr - r ? 1 : 0);
     }
+    // ROW_CACHE rows on tcgen05: each branch's static tile list (its pairs x row tiles x column tiles)
+    std::vector<int> rtile_off(nbr + 1, 0);
+    std::vector<int4> rtiles;
+    if (rc_tc)
+      for (int br = 0; br < nbr; ++br) {
+        const std::vector<int4> t = rows_tc_tiles(hp, bb[br], bb[br + 1] - bb[br], Bw);
+        rtiles.insert(rtiles.end(), t.begin(), t.end());
+        rtile_off[br + 1] = (int)rtiles.size();
+      }
+    new (&d_rtiles) DevBuf<int4>(std::max<size_t>(rtiles.size(), 1), st);
+    if (!rtiles.empty())
+      GM_CUDA(cudaMemcpyAsync(d_rtiles.get(), rtiles.data(), rtiles.size() * sizeof(int4), cudaMemcpyHostToDevice, st));
     std::vector<cudaEvent_t> ev_wave(Pl, nullptr);
     if (overlap) {  // kernel-value waves on the low-priority stream, one event per wave
       cudaEvent_t ev_staged = evp.get();
@@ -1254,7 +1283,10 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         for (int u = 0; u < unroll; ++u) launch_ws_iteration(ag, gn, npi, h, u == unroll - 1, max_outer, cs, u > 0);
       } else {
         launch_select_ws(ag, gn, 0, -1, cs);
-        if (rc) launch_rows_compute(ag, gn, npi, cs);
+        if (rc_tc)
+          launch_rows_compute_tc(ag, gn, d_rtiles.get() + rtile_off[br], rtile_off[br + 1] - rtile_off[br], Pl, cs);
+        else if (rc)
+          launch_rows_compute(ag, gn, npi, cs);
         launch_gather_kws(ag, gn, -1, cs);
         launch_local_smo(ag, gn, cs);
         launch_f_update_loop(ag, gn, npi, h, max_outer, cs);

@@ -152,6 +152,16 @@ struct SolverArgs {
   int64_t* rows_done;  // [P] kernel rows computed (ROW_CACHE statistics)
   int ldat;            // leading dimension of ATnew (round_up(B, 128))
   double gamma;
+  // ---- ROW_CACHE rows on tcgen05 (krow_tc.cu rows_tc_kernel): the class-sorted FP16 hi/lo split
+  // of X (row-major, dpt halfs per row; norms above are then its centred, scaled norms) and the
+  // gathered new rows of every pair [P][ldat][dpt]; exp2 scale of the split (-gamma log2 e / s^2)
+  const void* Xhi;
+  const void* Xlo;
+  void* Ahi;
+  void* Alo;
+  int dpt;
+  int64_t n_pad;
+  float kscale;
 };
 constexpr int kWsMaxNp = 16384;  // pair size limit of the default path (keys + flags in shared memory)
 
@@ -165,6 +175,11 @@ void launch_f_update(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st
 void launch_f_update_loop(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int64_t max_outer,
                           cudaStream_t st);
 void launch_rows_compute(const SolverArgs& a, int P, int64_t np_max, cudaStream_t st);
+// the same rows on tcgen05: tiles = (local pair, 128-row tile of its new rows, column tile of its
+// two class segments) for the pairs of the launch (krow_tc.cu); n_pairs_all = Pl (rows of A)
+std::vector<int4> rows_tc_tiles(const std::vector<PairDesc>& pairs, int first, int count, int B);
+void launch_rows_compute_tc(const SolverArgs& a, int P, const int4* tiles, int n_tiles, int n_pairs_all,
+                            cudaStream_t st);
 // a3-a5 default kernels (wsolve.cu): fast selection, multi-CTA K_ws,ws gather into an
 // L2-resident tile, single-warp local SMO (FULL_K regime, B <= 224, n_p <= 16384;
 // GMPSVM_WSOLVE=0 selects the select_ws / gather_kws / local_smo kernels of solver.cu)

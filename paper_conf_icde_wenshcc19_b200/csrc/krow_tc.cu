@@ -32,6 +32,7 @@
 #include <vector>
 
 #include "kernels.h"
+#include "solver_dev.cuh"
 #include "tc_util.cuh"
 
 namespace gmpsvm {
@@ -797,6 +798,227 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   }
 }
 
+
+// ------------------------------------------------------------------------------------------
+// ROW_CACHE rows on tcgen05 (a2 + a3 when K does not fit): per outer
+// iteration, the kernel rows of every pair's NEW working-set entries against the pair's
+// instances, K(x_new, x_pair) with the same FP16 hi/lo split and split accumulators as the FULL_K
+// contraction.  A = the new rows gathered per pair ([pair][ldat] rows of the Ahi / Alo buffers,
+// rows_gather_tc_kernel), B = the class-sorted split X; column tiles walk the pair's two class
+// segments; the epilogue writes row r's values at R[r_off + slot * ldr + pair-local column]
+// (per-thread stores, K_ii = 1).  Tiles whose rows do not exist this iteration (fewer new rows,
+// pair converged) are skipped by all three roles from the same global state.
+struct RowsTcArgs {
+  const PairDesc* pairs;
+  const int32_t* status;
+  const int32_t* ws;
+  const int32_t* ws_n;
+  const int32_t* ws_keep;
+  const int32_t* ws_slot;
+  const float* norms;
+  float* R;
+  int B, ldat;
+  float scale;
+};
+
+__device__ __forceinline__ bool rows_tile_live(const RowsTcArgs& ra, const int4 tl, int& nnew) {
+  const int lp = tl.x;
+  if (ra.status[lp] != 0) return false;
+  nnew = ra.ws_n[lp] - ra.ws_keep[lp];
+  return tl.y * kTM < nnew;
+}
+
+__global__ void __launch_bounds__(kTcThreads, 1)
+    rows_tc_kernel(const __grid_constant__ CUtensorMap map_ahi, const __grid_constant__ CUtensorMap map_alo,
+                   const __grid_constant__ CUtensorMap map_xhi, const __grid_constant__ CUtensorMap map_xlo,
+                   const int4* __restrict__ tiles, int n_tiles, int nk, RowsTcArgs ra) {
+  extern __shared__ __align__(1024) uint8_t dsmem[];
+  TcSmem& sm = *reinterpret_cast<TcSmem*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < kTcStages; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], 1);
+    }
+    mbar_init(&sm.tmem_full, 1);
+    mbar_init(&sm.tmem_empty, 4);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&sm.tmem_base)),
+                 "r"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = sm.tmem_base;
+  const int jn = nk < kMainAcc ? nk : kMainAcc;
+  auto col0 = [&](const int4 tl, int64_t& c0, int64_t& hi, int64_t& loc0) {
+    const PairDesc pd = ra.pairs[tl.x];
+    const int ts = (pd.n_s + kTN - 1) / kTN;
+    const bool seg_s = tl.z < ts;
+    c0 = seg_s ? pd.off_s + (int64_t)tl.z * kTN : pd.off_t + (int64_t)(tl.z - ts) * kTN;
+    hi = seg_s ? pd.off_s + pd.n_s : pd.off_t + pd.n_t;
+    loc0 = seg_s ? -pd.off_s : pd.n_s - pd.off_t;  // pair-local column = g + loc0
+  };
+  if (warp == 0) {
+    if (lane == 0) {  // ---- TMA producer
+      int g = 0, nnew = 0;
+      const uint64_t pol = policy_evict_last();
+      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+        const int4 tl = tiles[t];
+        if (!rows_tile_live(ra, tl, nnew)) continue;
+        int64_t c0, hi, loc0;
+        col0(tl, c0, hi, loc0);
+        const int r0 = tl.x * ra.ldat + tl.y * kTM;
+        for (int kb = 0; kb < nk; ++kb, ++g) {
+          const int s = g % kTcStages;
+          if (g >= kTcStages) mbar_wait(&sm.empty[s], ((g / kTcStages) + 1) & 1);
+          uint8_t* st = sm.stage[s];
+          mbar_expect_tx(&sm.full[s], kStageBytes);
+          const int kx = kb * 2 * kTK;
+          tma_load_2d(st, &map_ahi, kx, r0, &sm.full[s], pol);
+          tma_load_2d(st + kABytes, &map_alo, kx, r0, &sm.full[s], pol);
+          tma_load_2d(st + 2 * kABytes, &map_xhi, kx, (int)c0, &sm.full[s], pol);
+          tma_load_2d(st + 2 * kABytes + kBBytes, &map_xlo, kx, (int)c0, &sm.full[s], pol);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---- MMA issuer
+      int g = 0, it = 0, nnew = 0;
+      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+        const int4 tl = tiles[t];
+        if (!rows_tile_live(ra, tl, nnew)) continue;
+        if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        for (int kb = 0; kb < nk; ++kb, ++g) {
+          const int s = g % kTcStages;
+          mbar_wait(&sm.full[s], (g / kTcStages) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          uint8_t* st = sm.stage[s];
+          const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
+          const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
+          const int j = (kb * jn) / nk;
+          const int kb_first = (j * nk + jn - 1) / jn;
+#pragma unroll
+          for (int kk = 0; kk < kTK / 8; ++kk) {
+            const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+            umma_tf32<true>(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
+            umma_tf32<true>(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
+            umma_tf32<true>(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+          }
+          umma_commit(&sm.empty[s]);
+        }
+        umma_commit(&sm.tmem_full);
+        ++it;
+      }
+    }
+  } else {  // ---- epilogue: warps 2..5 (TMEM lane quarter warp % 4), thread = one new row
+    const int q = warp & 3;
+    int it = 0, nnew = 0;
+    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+      const int4 tl = tiles[t];
+      if (!rows_tile_live(ra, tl, nnew)) continue;
+      const PairDesc pd = ra.pairs[tl.x];
+      int64_t c0, hi, loc0;
+      col0(tl, c0, hi, loc0);
+      const int r = tl.y * kTM + q * 32 + lane;  // index among the pair's new rows
+      const bool live = r < nnew;
+      const int keep = ra.ws_keep[tl.x];
+      const int64_t gr = live ? gpos(pd, ra.ws[(int64_t)tl.x * ra.B + keep + r]) : -1;
+      const float nr = live ? ra.norms[gr] : 0.f;
+      const int64_t ldr = (pd.n_s + pd.n_t + 3) & ~3;
+      float* dst = live ? ra.R + pd.r_off + (int64_t)ra.ws_slot[(int64_t)tl.x * ra.B + keep + r] * ldr : nullptr;
+      float cnv[kTN / 32];
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) cnv[ch] = ra.norms[c0 + ch * 32 + lane];  // norms zero-padded past n
+      mbar_wait(&sm.tmem_full, it & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      float dot[kTN];
+      const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) {
+        uint32_t v0[32], w[32];
+        tmem_ld32(trow + (uint32_t)(ch * 32), v0);
+        tmem_ld32(trow + (uint32_t)(ch * 32) + kMainAcc * kTN, w);
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+        for (int j = 0; j < 32; ++j) dot[ch * 32 + j] = __uint_as_float(v0[j]) + __uint_as_float(w[j]);
+        if (nk > 1) {
+          tmem_ld32(trow + (uint32_t)(ch * 32) + kTN, v0);
+          tmem_ld32(trow + (uint32_t)(ch * 32) + 2 * kTN, w);
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            float x = dot[ch * 32 + j] + __uint_as_float(v0[j]);
+            if (nk > 2) x += __uint_as_float(w[j]);
+            dot[ch * 32 + j] = x;
+          }
+        }
+      }
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+      ++it;
+#pragma unroll
+      for (int ch = 0; ch < kTN / 32; ++ch) {
+        const int64_t cb = c0 + ch * 32;
+        float kv[32];
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const float d2 = fmaf(-2.f, dot[ch * 32 + j], nr + __shfl_sync(0xffffffffu, cnv[ch], j));
+          float val;
+          asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(val) : "f"(fmaxf(d2, 0.f) * ra.scale));
+          kv[j] = (cb + j == gr) ? 1.f : val;
+        }
+        if (!live || cb >= hi) continue;
+        float* o = dst + cb + loc0;
+        if (cb + 31 < hi && (reinterpret_cast<uintptr_t>(o) & 15) == 0) {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4) *reinterpret_cast<float4*>(o + j) = make_float4(kv[j], kv[j + 1], kv[j + 2], kv[j + 3]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; ++j)
+            if (cb + j < hi) o[j] = kv[j];
+        }
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
+  }
+}
+
+// the new rows' hi / lo split rows into A (row lp * ldat + r), FP16 halfs, dpt per row
+__global__ void rows_gather_tc_kernel(const PairDesc* pairs, const int32_t* status, const int32_t* ws,
+                                      const int32_t* ws_n, const int32_t* ws_keep, int B, int ldat, int pair_base,
+                                      const __half* xhi, const __half* xlo, __half* ahi, __half* alo, int dpt,
+                                      int64_t* rows_done) {
+  const int lp = blockIdx.x + pair_base;
+  if (status[lp] != 0) return;
+  const PairDesc pd = pairs[lp];
+  const int keep = ws_keep[lp], nnew = ws_n[lp] - keep;
+  if (nnew <= 0) return;
+  if (blockIdx.y == 0 && threadIdx.x == 0) rows_done[lp] += nnew;
+  const int vq = dpt / 8;  // 16-byte vectors per row
+  for (int r = blockIdx.y; r < nnew; r += gridDim.y) {
+    const int64_t g = gpos(pd, ws[(int64_t)lp * B + keep + r]);
+    const uint4* sh = reinterpret_cast<const uint4*>(xhi + g * dpt);
+    const uint4* sl = reinterpret_cast<const uint4*>(xlo + g * dpt);
+    uint4* dh = reinterpret_cast<uint4*>(ahi + ((int64_t)lp * ldat + r) * dpt);
+    uint4* dl = reinterpret_cast<uint4*>(alo + ((int64_t)lp * ldat + r) * dpt);
+    for (int v = threadIdx.x; v < vq; v += blockDim.x) {
+      dh[v] = sh[v];
+      dl[v] = sl[v];
+    }
+  }
+}
+
 // column means of the rows idx[0..n) of X (idx < 0: skipped): per-chunk FP64 partials, then a
 // fixed-order sum over the chunks (deterministic)
 constexpr int kGatherMeanRows = 256;  // rows per partial
@@ -1125,6 +1347,34 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
     GM_LAUNCH((krow_tc_kernel<false, 0>), dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles,
               n_tiles, norms, n, nk, scale, K, ldk, tma, kp);
   }
+}
+
+std::vector<int4> rows_tc_tiles(const std::vector<PairDesc>& pairs, int first, int count, int B) {
+  std::vector<int4> t;
+  const int at = (int)ceil_div(B, kTM);
+  for (int lp = first; lp < first + count; ++lp) {
+    const PairDesc& pd = pairs[lp];
+    const int ct = (int)(ceil_div(pd.n_s, kTN) + ceil_div(pd.n_t, kTN));
+    for (int a = 0; a < at; ++a)
+      for (int c = 0; c < ct; ++c) t.push_back(make_int4(lp, a, c, 0));
+  }
+  return t;
+}
+
+void launch_rows_compute_tc(const SolverArgs& a, int P, const int4* tiles, int n_tiles, int n_pairs_all,
+                            cudaStream_t st) {
+  GM_LAUNCH(rows_gather_tc_kernel, dim3(P, 64), dim3(128), 0, st, a.pairs, a.status, a.ws, a.ws_n, a.ws_keep, a.B,
+            a.ldat, a.pair_base, static_cast<const __half*>(a.Xhi), static_cast<const __half*>(a.Xlo),
+            static_cast<__half*>(a.Ahi), static_cast<__half*>(a.Alo), a.dpt, a.rows_done);
+  const CUtensorMap mahi = make_map(a.Ahi, (int64_t)n_pairs_all * a.ldat, a.dpt, true);
+  const CUtensorMap malo = make_map(a.Alo, (int64_t)n_pairs_all * a.ldat, a.dpt, true);
+  const CUtensorMap mxhi = make_map(a.Xhi, a.n_pad, a.dpt, true), mxlo = make_map(a.Xlo, a.n_pad, a.dpt, true);
+  const size_t smem = sizeof(TcSmem) + 1024;
+  set_max_dyn_smem(rows_tc_kernel, smem);
+  RowsTcArgs ra{a.pairs, a.status, a.ws, a.ws_n, a.ws_keep, a.ws_slot, a.norms, a.R, a.B, a.ldat, a.kscale};
+  const int grid = std::min(n_tiles, num_sms());
+  GM_LAUNCH(rows_tc_kernel, dim3(grid), dim3(kTcThreads), smem, st, mahi, malo, mxhi, mxlo, tiles, n_tiles,
+            a.dpt / (2 * kTK), ra);
 }
 
 void launch_gather_col_mean(const float* X, int d, const int64_t* idx, int64_t n, int64_t cnt, float* mu,
