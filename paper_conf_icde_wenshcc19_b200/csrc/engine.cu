@@ -994,15 +994,16 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // predict) -- the waves' tensor/HBM load stretches the solver's latency-bound chain more than
   // the overlap saves.
   static const bool overlap_env = getenv("GMPSVM_OVERLAP") && std::string(getenv("GMPSVM_OVERLAP")) == "1";
-  const bool overlap = overlap_env && ktype == 0 && use_tc && ws_solve_supported(B, np_max);
+  const bool fk_tc = full_k && use_tc;  // the FULL_K contraction on tcgen05
+  const bool overlap = overlap_env && ktype == 0 && fk_tc && ws_solve_supported(B, np_max);
   cudaStream_t kst = krow_stream(opt.device);
   TimedEvents kev;
   cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
   std::vector<int> wave_off;     // tile range of wave w: [wave_off[w], wave_off[w + 1])
   std::vector<int> ready_wave;   // per pair position: the wave after which its kernel values are complete
-  const bool two_cta = use_tc && !overlap && ktype == 0 && krow_tc_2cta();  // overlap waves: single-CTA tiles
+  const bool two_cta = fk_tc && !overlap && ktype == 0 && krow_tc_2cta();  // overlap waves: single-CTA tiles
   double kv_subset = -1;  // >= 0: kernel values computed for a pair subset (tiles skipped)
-  if (use_tc) {
+  if (fk_tc) {
     tiles = krow_tc_tiles(n, two_cta);
     if (!overlap && !two_cta && Pl < P) {
       // pair subset (multi-GPU shard, pair_ids): only the tiles overlapping a class block
@@ -1085,7 +1086,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     GM_CUDA(cudaMemcpyAsync(d_tiles.get(), tiles.data(), tiles.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
   }
   tm.mark(PH_KERNEL);
-  if (use_tc && !overlap)
+  if (fk_tc && !overlap)
   {
     const KrowKernel kk{ktype, (float)gamma, (float)kcoef0, 0.f, kdegree};
     launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, ksc, K.get(),
