@@ -308,14 +308,14 @@ __global__ void __launch_bounds__(kIThreads, 1)
 #pragma unroll
             for (int part3 = 0; part3 < 2; ++part3) {
               long long w[16];
+              uint32_t v0[16], v1[16], v2[16];  // the three groups' loads in flight together, one wait
+              tmem_ld16(taddr + (uint32_t)((part3 * 3 + 0) * kIN + ch * 16), v0);
+              tmem_ld16(taddr + (uint32_t)((part3 * 3 + 1) * kIN + ch * 16), v1);
+              tmem_ld16(taddr + (uint32_t)((part3 * 3 + 2) * kIN + ch * 16), v2);
+              asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 #pragma unroll
-              for (int g3 = 0; g3 < 3; ++g3) {
-                uint32_t v[16];
-                tmem_ld16(taddr + (uint32_t)((part3 * 3 + g3) * kIN + ch * 16), v);
-                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-                for (int jj = 0; jj < 16; ++jj) w[jj] = (g3 == 0 ? 0ll : w[jj] * 256) + (int32_t)v[jj];
-              }
+              for (int jj = 0; jj < 16; ++jj)
+                w[jj] = ((long long)(int32_t)v0[jj] * 65536 + (long long)(int32_t)v1[jj] * 256) + (int32_t)v2[jj];
 #pragma unroll
               for (int jj = 0; jj < 16; ++jj)
                 dot[ch * 16 + jj] = part3 == 0 ? (double)w[jj] : fma(dot[ch * 16 + jj], 16777216.0, (double)w[jj]);

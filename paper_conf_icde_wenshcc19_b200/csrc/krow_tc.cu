@@ -68,9 +68,22 @@ struct TcSmem {
 constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(kTN >> 3) << 17) | ((uint32_t)(kTM >> 4) << 24);
 constexpr uint32_t kIdescF16 = (1u << 4) | ((uint32_t)(kTN >> 3) << 17) | ((uint32_t)(kTM >> 4) << 24);
 
-template <bool F16>
+// COL: A-operand collector (kind::f16 only): 0 none, 1 fill (keep A for the next MMA), 3 lastuse.
+// hi.hi and hi.lo share the A tile (hi): issued back to back, the second reuses the collector and
+// the tensor core reads A from shared memory once for both
+template <bool F16, int COL = 0>
 __device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
-  if (F16)
+  if (F16 && COL == 1)
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::f16.collector::a::fill [%0], %1, %2, "
+        "%3, p;\n}\n" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(kIdescF16), "r"(accum));
+  else if (F16 && COL == 3)
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::f16.collector::a::lastuse [%0], %1, "
+        "%2, %3, p;\n}\n" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(kIdescF16), "r"(accum));
+  else if (F16)
     asm volatile(
         "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(
             tmem_d),
@@ -80,6 +93,19 @@ __device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t a, uint64_t 
         "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(
             tmem_d),
         "l"(a), "l"(b), "r"(kIdesc), "r"(accum));
+}
+// the three products of one k step: hi.hi into accumulator j, hi.lo + lo.hi into the corrections
+template <bool F16, bool COLLECT>
+__device__ __forceinline__ void umma_split3(uint32_t dj, uint32_t dc, uint64_t ahi, uint64_t alo, uint64_t bhi,
+                                            uint64_t blo, uint32_t acc_j, uint32_t acc_c) {
+  if (F16 && COLLECT) {
+    umma_tf32<true, 1>(dj, ahi, bhi, acc_j);
+    umma_tf32<true, 3>(dc, ahi, blo, acc_c);
+  } else {
+    umma_tf32<F16>(dj, ahi, bhi, acc_j);
+    umma_tf32<F16>(dc, ahi, blo, acc_c);
+  }
+  umma_tf32<F16>(dc, alo, bhi, 1u);
 }
 // The paper's other kernels (L76-L78, NEXT-4) on the same contraction: with uncentred rows the
 // tensor cores deliver s^2 x . y; K = x.y, (gamma x.y + coef0)^degree or tanh(gamma x.y + coef0).
@@ -183,9 +209,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 TF32 = 32 bytes along K inside the atom
-            umma_tf32<F16>(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
-            umma_tf32<F16>(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
-            umma_tf32<F16>(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+            umma_split3<F16, true>(tmem + j * kTN, tmem + kMainAcc * kTN, ahi + adv, alo + adv, bhi + adv, blo + adv,
+                                   (kb == kb_first && kk == 0) ? 0u : 1u, (kb | kk) ? 1u : 0u);
           }
           umma_commit(&sm.empty[s]);
         }
@@ -713,9 +738,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
             for (int kk = 0; kk < kTK / 8; ++kk) {
               const uint64_t adv = (uint64_t)(kk * 32) >> 4;
-              umma_tf32<F16>(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
-              umma_tf32<F16>(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
-              umma_tf32<F16>(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+              umma_split3<F16, true>(tmem + j * kTN, tmem + kMainAcc * kTN, ahi + adv, alo + adv, bhi + adv, blo + adv,
+                                     (kb == kb_first && kk == 0) ? 0u : 1u, (kb | kk) ? 1u : 0u);
             }
             umma_commit(&sm.empty[s]);
           }
@@ -905,9 +929,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;
-            umma_tf32<true>(tmem + j * kTN, ahi + adv, bhi + adv, (kb == kb_first && kk == 0) ? 0u : 1u);
-            umma_tf32<true>(tmem + kMainAcc * kTN, ahi + adv, blo + adv, (kb | kk) ? 1u : 0u);
-            umma_tf32<true>(tmem + kMainAcc * kTN, alo + adv, bhi + adv, 1u);
+            umma_split3<true, true>(tmem + j * kTN, tmem + kMainAcc * kTN, ahi + adv, alo + adv, bhi + adv, blo + adv,
+                                    (kb == kb_first && kk == 0) ? 0u : 1u, (kb | kk) ? 1u : 0u);
           }
           umma_commit(&sm.empty[s]);
         }
