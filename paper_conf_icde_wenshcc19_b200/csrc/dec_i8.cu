@@ -5,7 +5,7 @@
 // and a decision value sums sum_j |alpha_j| K_j of kernel values (Eq 11).  Any path that holds K
 // in FP32 has a worst-case error of sum_j |alpha_j| * 2^-24 and more -- MNIST-shaped C = 10 models
 // (sum |alpha| ~ 10^3, |A| ~ 6) then cannot be bounded below the 1e-4 probability contract.
-// Here the dot products are EXACT integers and K is formed in FP64 (DESIGN.md §3, §6.4):
+// Here the dot products are EXACT integers and K is formed in FP64 (DESIGN.md §3, §6.5):
 //
 //   staging (one warp per row): e_r = 37 - ilogb(max_c |x_rc|), X_int = rint(x * 2^e_r) with
 //     |X_int| < 2^38 (exact for every element >= max|x| 2^-14, else off by <= max|x| 2^-38), written

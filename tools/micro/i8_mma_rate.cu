@@ -67,11 +67,12 @@ __global__ void k(int iters, long long* out) {
 // (i = 0..4) times B planes j with i + j <= 5 into accumulator i + j (N = 64 each, 6 x 64 TMEM
 // columns), optionally with the A-operand collector (fill / use / lastuse), one commit per
 // 64-wide k block.  Cycles per MMA for the whole sequence.
-template <bool COLLECT, int NN>
+template <bool COLLECT, int NN, bool SYNC = false>
 __global__ void pattern_k(int kblocks, long long* out) {
   extern __shared__ __align__(1024) uint8_t sm[];
   __shared__ uint32_t tbase;
   __shared__ __align__(8) uint64_t bar;
+  __shared__ __align__(8) uint64_t bar2;
   const int warp = threadIdx.x >> 5;
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(&tbase)), "r"(512));
@@ -79,6 +80,7 @@ __global__ void pattern_k(int kblocks, long long* out) {
   }
   if (threadIdx.x == 32) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar)));
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar2)));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -89,6 +91,14 @@ __global__ void pattern_k(int kblocks, long long* out) {
     constexpr uint32_t idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(NN >> 3) << 17) | (8u << 24);
     const long long t0 = clock64();
     for (int kb = 0; kb < kblocks; ++kb) {
+      if (SYNC) {  // as in the kernel: wait on a (completed) stage barrier, fence, ..., commit
+        uint32_t done = 0;
+        do {
+          asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 1;\n selp.u32 %0, 1, 0, p;\n}\n"
+                       : "=r"(done) : "r"(su32(&bar)) : "memory");
+        } while (!done);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      }
       for (int kk = 0; kk < 2; ++kk) {
         for (int i = 0; i < 5; ++i) {
           const uint64_t a = desc(sm + i * 8192, 4) + (uint64_t)(kk * 2);
@@ -107,6 +117,7 @@ __global__ void pattern_k(int kblocks, long long* out) {
           }
         }
       }
+      if (SYNC) asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(&bar2)) : "memory");
     }
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(&bar)) : "memory");
     uint32_t done = 0;
@@ -162,5 +173,6 @@ int main() {
   runp("dec_i8 19-product pattern N64, collector", pattern_k<true, 64>, 64);
   runp("dec_i8 19-product pattern N64, no collector", pattern_k<false, 64>, 64);
   runp("dec_i8 19-product pattern N80, collector", pattern_k<true, 80>, 80);
+  runp("dec_i8 19-product pattern N64, collector, per-k-block wait+fence+commit", pattern_k<true, 64, true>, 64);
   return 0;
 }
