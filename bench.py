@@ -211,12 +211,17 @@ def run_gpu(args, spec):
     stream = torch.cuda.current_stream(dev)
     opts = dict(ws_size=args.ws_size)
 
+    host_ms = []  # host-clock duration of each step's calls (diagnostic: stalls outside the GPU)
+
     def step(Xa, ya, Xta, host=False):
+        t0 = time.perf_counter()
         if ws > 1:
             model, prob = gdist.train_predict(Xa, ya, Xta, spec.k, spec.C, spec.gamma, args.eps, **opts)
         else:
             model = gm.train(Xa, ya, spec.k, spec.C, spec.gamma, args.eps, **opts)
+            t1 = time.perf_counter()
             prob = model.predict_proba(Xta)
+            host_ms.append((round((t1 - t0) * 1e3, 2), round((time.perf_counter() - t1) * 1e3, 2)))
         return model, prob
 
     # the clock sampler (an nvidia-smi process every 0.2 s) starts during the warm-up, so its
@@ -342,6 +347,7 @@ def run_gpu(args, spec):
                           "predict_stage": ps["t_stage_ms"], "decision_values": ps["t_decision_ms"],
                           "couple": ps["t_couple_ms"], "predict_total": ps["t_total_ms"]},
             "step_ms": step_ms,
+            "host_ms_train_predict": host_ms[args.warmup:args.warmup + args.steps],
             "counters": {"outer_iters_max": s["outer_iters_max"], "inner_iters_sum": s["inner_iters_sum"],
                          "smo_cycles_per_step": s["smo_cycles_sum"] / max(1, s["inner_iters_sum"]),
                          "n_sv": s["n_sv"], "dec_tflops": ps["dec_flops"] / (ps["t_decision_ms"] * 1e-3) / 1e12
