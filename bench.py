@@ -78,6 +78,8 @@ class ClockSampler:
             pass
 
     def _run(self):
+        if os.environ.get("GMPSVM_BENCH_CLOCKS") == "off":  # diagnostics only: no sampler process
+            return
         # one long-running nvidia-smi (the recipe's `-lms 200` loop): NVML is initialised once, so
         # the sampling does not stall the host's CUDA calls the way a fresh process every 0.2 s did
         try:

@@ -43,14 +43,12 @@ namespace {
 
 constexpr int kND = 5;                     // digit planes per operand (40-bit fixed point)
 constexpr int kNG = 6;                     // digit-product groups kept: g = i + j <= 5
-constexpr int kIM = 128, kIN = 80, kIK = 64;  // test rows, SVs per sub-tile, int8 per k-block (64 B atom)
-constexpr int kIHalf = kIN / 2;                // SV columns per epilogue warp
-constexpr int kTileSv = 128;                   // the model's class-pure SV slot tiles
+constexpr int kIM = 128, kIN = 64, kIK = 64;  // test rows, SVs per tile, int8 per k-block (64 B atom)
 constexpr int kIStages = 3;
 constexpr uint32_t kIAPlane = kIM * kIK;  // 8 KB
-constexpr uint32_t kIBPlane = kIN * kIK;  // 5 KB
-constexpr uint32_t kIStageBytes = kND * (kIAPlane + kIBPlane);  // 65 KB (1024-byte multiple)
-constexpr uint32_t kITmemCols = 512;      // 6 x 80 used (power-of-two allocation)
+constexpr uint32_t kIBPlane = kIN * kIK;  // 4 KB
+constexpr uint32_t kIStageBytes = kND * (kIAPlane + kIBPlane);  // 60 KB
+constexpr uint32_t kITmemCols = 512;      // 6 x 64 used (power-of-two allocation)
 constexpr int kIThreads = 320;  // producer, MMA issuer, 8 epilogue warps
 constexpr int kIExp = 37;                 // max |x| 2^e in [2^37, 2^38)
 // kind::i8, D S32 (2), A S8 (1), B S8 (1), K-major, N = 64, M = 128
@@ -208,16 +206,15 @@ __global__ void __launch_bounds__(kIThreads, 1)
   const uint32_t tmem = sm.tmem_base;
 
   if (warp == 0) {
-    if (lane == 0) {  // ---- TMA producer: per (unit, 80-SV sub-tile, k-block) the 5 + 5 digit planes
+    if (lane == 0) {  // ---- TMA producer: per (tile, half, k-block) the 5 + 5 digit planes
       int g = 0;
       const uint64_t pol = policy_evict_last();
-      for (int u = blockIdx.x; u < n_units; u += gridDim.x) {
-        const int t0 = unit_off[u], t1 = unit_off[u + 1];
-        if (t1 <= t0) continue;
-        const int r0 = tiles[t0].x * kIM;
-        const int s_end = (tiles[t1 - 1].y + 1) * kTileSv;
-        for (int c0 = tiles[t0].y * kTileSv; c0 < s_end; c0 += kIN) {
-          {
+      for (int u = blockIdx.x; u < n_units; u += gridDim.x)
+        for (int t = unit_off[u]; t < unit_off[u + 1]; ++t) {
+          const int2 tile = tiles[t];
+          const int r0 = tile.x * kIM;
+          for (int h = 0; h < 2; ++h) {
+            const int c0 = tile.y * 2 * kIN + h * kIN;
             for (int kb = 0; kb < nk; ++kb, ++g) {
               const int s = g % NS;
               if (g >= NS) mbar_wait(&sm.empty[s], ((g / NS) + 1) & 1);
@@ -236,16 +233,13 @@ __global__ void __launch_bounds__(kIThreads, 1)
             }
           }
         }
-      }
     }
   } else if (warp == 1) {
     if (lane == 0) {  // ---- MMA issuer: group g = i + j of the digit products into accumulator g
       int g = 0, it = 0;
-      for (int u = blockIdx.x; u < n_units; u += gridDim.x) {
-        const int t0 = unit_off[u], t1 = unit_off[u + 1];
-        if (t1 <= t0) continue;
-        const int s_end = (tiles[t1 - 1].y + 1) * kTileSv;
-        for (int c0 = tiles[t0].y * kTileSv; c0 < s_end; c0 += kIN, ++it) {
+      for (int u = blockIdx.x; u < n_units; u += gridDim.x)
+        for (int t = unit_off[u]; t < unit_off[u + 1]; ++t)
+          for (int h = 0; h < 2; ++h, ++it) {
             if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             for (int kb = 0; kb < nk; ++kb, ++g) {
@@ -279,71 +273,69 @@ __global__ void __launch_bounds__(kIThreads, 1)
             }
             umma_commit(&sm.tmem_full);
           }
-      }
     }
   } else {  // ---- epilogue: warps 2..9; TMEM lane quarter warp % 4, column half (warp - 2) / 4;
-            //      thread = one test row x 40 of the sub-tile's 80 SVs
+            //      thread = one test row x 32 of the tile's 64 SVs
     const int q = warp & 3, half = (warp - 2) >> 2, et_id = threadIdx.x - 64;  // et_id 0..255
     int it = 0;
     const double tsc = -gamma * 1.4426950408889634074;  // exp(-gamma d2) = 2^(tsc d2)
     for (int u = blockIdx.x; u < n_units; u += gridDim.x) {
-      const int t0 = unit_off[u], t1 = unit_off[u + 1];
-      if (t1 <= t0) continue;
       double acc[KM];
 #pragma unroll
       for (int v = 0; v < KM; ++v) acc[v] = 0.0;
-      const int64_t r = (int64_t)tiles[t0].x * kIM + q * 32 + lane;
-      const int ex_r = et[r];
-      const double nr = nt[r];
-      const int64_t s_end = (int64_t)(tiles[t1 - 1].y + 1) * kTileSv;
-      for (int64_t c0 = (int64_t)tiles[t0].y * kTileSv; c0 < s_end; c0 += kIN, ++it) {
-        // this sub-tile's coefficients (double buffer); slots past the unit (the sub-tile's tail
-        // runs into the next class or past the SVs) get 0 and are skipped below
-        double* cs = &sm.coefS[it & 1][0][0];
-        for (int idx = et_id; idx < kIN * KM; idx += 256) {
-          const int jj = idx / KM, v = idx - jj * KM;
-          cs[idx] = (v < km1 && c0 + jj < s_end) ? coef[(c0 + jj) * km1_pad + v] : 0.0;
-        }
-        asm volatile("bar.sync 1, 256;" ::: "memory");
-        mbar_wait(&sm.tmem_full, it & 1);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        // sum_g 256^(5-g) G_g by 8-column chunks: groups 0-2 and 3-5 combined exactly in int64
-        // (|G| < 2^26: |hi|, |lo| < 2^43, exact in FP64), then hi 2^24 + lo in FP64
-        const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(half * kIHalf);
-        double dot[kIHalf];
-#pragma unroll
-        for (int ch = 0; ch < kIHalf / 8; ++ch) {
-          uint32_t v0[8], v1[8], v2[8], v3[8], v4[8], v5[8];  // the six groups' loads in flight, one wait
-          tmem_ld8(taddr + (uint32_t)(0 * kIN + ch * 8), v0);
-          tmem_ld8(taddr + (uint32_t)(1 * kIN + ch * 8), v1);
-          tmem_ld8(taddr + (uint32_t)(2 * kIN + ch * 8), v2);
-          tmem_ld8(taddr + (uint32_t)(3 * kIN + ch * 8), v3);
-          tmem_ld8(taddr + (uint32_t)(4 * kIN + ch * 8), v4);
-          tmem_ld8(taddr + (uint32_t)(5 * kIN + ch * 8), v5);
-          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-          for (int jj = 0; jj < 8; ++jj) {
-            const long long hi = ((long long)(int32_t)v0[jj] * 65536 + (long long)(int32_t)v1[jj] * 256) + (int32_t)v2[jj];
-            const long long lo = ((long long)(int32_t)v3[jj] * 65536 + (long long)(int32_t)v4[jj] * 256) + (int32_t)v5[jj];
-            dot[ch * 8 + jj] = fma((double)hi, 16777216.0, (double)lo);
+      int64_t r = 0;
+      for (int t = unit_off[u]; t < unit_off[u + 1]; ++t) {
+        const int2 tile = tiles[t];
+        r = (int64_t)tile.x * kIM + q * 32 + lane;
+        const int ex_r = et[r];
+        const double nr = nt[r];
+        for (int h = 0; h < 2; ++h, ++it) {
+          const int64_t c0 = (int64_t)tile.y * 2 * kIN + h * kIN;
+          double* cs = &sm.coefS[it & 1][0][0];  // this half-tile's coefficients (double buffer)
+          for (int idx = et_id; idx < kIN * KM; idx += 256) {
+            const int jj = idx / KM, v = idx - jj * KM;
+            cs[idx] = v < km1 ? coef[(c0 + jj) * km1_pad + v] : 0.0;
           }
-        }
-        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncwarp();
-        if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
-        // x~.y~ = 2^-(e_x+e_y) 256^3 (hi 2^24 + lo): the 256^3 = 2^24 folds into the exponent
-        if (diag & 1) {  // GMPSVM_I8_DIAG bit 0 (timing experiments): no epilogue arithmetic
-          acc[0] += dot[0] + dot[kIHalf - 1];
-          continue;
-        }
+          asm volatile("bar.sync 1, 256;" ::: "memory");
+          mbar_wait(&sm.tmem_full, it & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          // sum_g 256^(5-g) G_g by 16-column chunks: groups 0-2 and 3-5 combined exactly in int64
+          // (|G| < 2^26: |hi|, |lo| < 2^43, exact in FP64), then hi 2^24 + lo in FP64
+          const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(half * 32);
+          double dot[32];
 #pragma unroll
-        for (int jj = 0; jj < kIHalf; ++jj) {
-          const int64_t c = c0 + half * kIHalf + jj;
-          if (c < s_end) {
+          for (int ch = 0; ch < 2; ++ch) {
+#pragma unroll
+            for (int part3 = 0; part3 < 2; ++part3) {
+              long long w[16];
+              uint32_t v0[16], v1[16], v2[16];  // the three groups' loads in flight together, one wait
+              tmem_ld16(taddr + (uint32_t)((part3 * 3 + 0) * kIN + ch * 16), v0);
+              tmem_ld16(taddr + (uint32_t)((part3 * 3 + 1) * kIN + ch * 16), v1);
+              tmem_ld16(taddr + (uint32_t)((part3 * 3 + 2) * kIN + ch * 16), v2);
+              asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+              for (int jj = 0; jj < 16; ++jj)
+                w[jj] = ((long long)(int32_t)v0[jj] * 65536 + (long long)(int32_t)v1[jj] * 256) + (int32_t)v2[jj];
+#pragma unroll
+              for (int jj = 0; jj < 16; ++jj)
+                dot[ch * 16 + jj] = part3 == 0 ? (double)w[jj] : fma(dot[ch * 16 + jj], 16777216.0, (double)w[jj]);
+            }
+          }
+          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+          // x~.y~ = 2^-(e_x+e_y) 256^3 (hi 2^24 + lo): the 256^3 = 2^24 folds into the exponent
+          if (diag & 1) {  // GMPSVM_I8_DIAG bit 0 (timing experiments): no epilogue arithmetic
+            acc[0] += dot[0] + dot[31];
+            continue;
+          }
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj) {
+            const int64_t c = c0 + half * 32 + jj;
             const double xy = dot[jj] * pow2(24 - ex_r - __ldg(es + c));
             const double d2 = fmax(fma(-2.0, xy, nr + __ldg(ns + c)), 0.0);
             const double kv = exp2_neg(tsc * d2);
-            const double* cj = cs + (half * kIHalf + jj) * KM;
+            const double* cj = cs + (half * 32 + jj) * KM;
 #pragma unroll
             for (int v = 0; v < KM; ++v) acc[v] = fma(kv, cj[v], acc[v]);
           }
