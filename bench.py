@@ -396,7 +396,7 @@ def run_gpu(args, spec):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gmpsvm", choices=["gmpsvm", "reference"])
     ap.add_argument("--config", default="mnist")

@@ -5,6 +5,9 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <stdexcept>
 #include <string>
 
@@ -20,10 +23,23 @@ struct Error : std::runtime_error {
 
 [[noreturn]] void throw_cuda(cudaError_t e, const char* what, const char* file, int line);
 
-#define GM_CUDA(call)                                                      \
-  do {                                                                     \
-    cudaError_t e_ = (call);                                               \
-    if (e_ != cudaSuccess) ::gmpsvm::throw_cuda(e_, #call, __FILE__, __LINE__); \
+// GMPSVM_SLOW_API=<ms> (diagnostics): report every CUDA runtime call of the library that blocks
+// the host longer than that
+inline double slow_api_ms() {
+  static const double v = getenv("GMPSVM_SLOW_API") ? atof(getenv("GMPSVM_SLOW_API")) : 0.0;
+  return v;
+}
+
+#define GM_CUDA(call)                                                                                     \
+  do {                                                                                                    \
+    const double thr_ = ::gmpsvm::slow_api_ms();                                                          \
+    const auto t0_ = thr_ > 0 ? std::chrono::steady_clock::now() : std::chrono::steady_clock::time_point(); \
+    cudaError_t e_ = (call);                                                                              \
+    if (thr_ > 0) {                                                                                       \
+      const double ms_ = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0_).count(); \
+      if (ms_ > thr_) fprintf(stderr, "[gmpsvm slow api] %.2f ms %s (%s:%d)\n", ms_, #call, __FILE__, __LINE__); \
+    }                                                                                                     \
+    if (e_ != cudaSuccess) ::gmpsvm::throw_cuda(e_, #call, __FILE__, __LINE__);                           \
   } while (0)
 
 #define GM_CHECK_LAUNCH() GM_CUDA(cudaGetLastError())

@@ -9,7 +9,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <deque>
-#include <thread>
+#include <functional>
 #include <map>
 #include <mutex>
 #include <string>
@@ -46,7 +46,7 @@ constexpr int kMaxK = 64;          // label-rank shared memory bound
 constexpr int kMaxCoupleK = 40;    // coupling shared memory bound
 constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
 constexpr int64_t kPredictChunk = 32768;
-constexpr int kMaxStreams = 2;     // solver streams: graph launch + graph capture
+constexpr int kMaxStreams = 3;     // solver streams: graph launches (rest, lead) + graph capture
 constexpr int kDefaultB = 192;     // working-set rows (tuned on MNIST-shaped data; the tile of K_ws,ws stays in shared memory for B <= 224)
 
 struct DeviceGuard {
@@ -97,7 +97,7 @@ size_t device_total_mem(int dev) {
 std::mutex g_pool_mu;
 std::vector<cudaStream_t> g_pools[64];
 // The solver's streams have the highest priority: when the kernel-value waves share the GPU with
-// the solver (overlap mode), the block scheduler dispatches solver CTAs first.
+// the lead pairs' solver (lead mode), the block scheduler dispatches solver CTAs first.
 const std::vector<cudaStream_t>& stream_pool(int dev) {
   std::lock_guard<std::mutex> lk(g_pool_mu);
   auto& v = g_pools[dev];
@@ -111,7 +111,7 @@ const std::vector<cudaStream_t>& stream_pool(int dev) {
   return v;
 }
 
-// Low-priority stream for the kernel-value waves of the overlap mode.
+// Low-priority stream for the kernel-value waves of lead mode.
 cudaStream_t krow_stream(int dev) {
   static std::mutex mu;
   static cudaStream_t s[64] = {};
@@ -236,6 +236,96 @@ struct GraphGuard {
   }
 };
 
+// Solver-state arena: pointers carved from one allocation at fixed offsets (same sizes -> same
+// pointers, so a cached graph's kernel arguments stay valid).
+template <class T>
+struct ArenaPtr {
+  T* p = nullptr;
+  T* get() const { return p; }
+};
+struct ArenaLayout {
+  size_t bytes = 0;
+  std::vector<std::function<void(char*)>> set;
+  template <class T>
+  void add(ArenaPtr<T>& a, size_t count) {
+    bytes = (bytes + 255) & ~(size_t)255;
+    const size_t off = bytes;
+    set.push_back([&a, off](char* base) { a.p = reinterpret_cast<T*>(base + off); });
+    bytes += std::max<size_t>(count, 1) * sizeof(T);
+  }
+  void place(void* base) {
+    for (auto& f : set) f(static_cast<char*>(base));
+  }
+};
+
+// Per-device solver workspace kept across training calls: the arena and the instantiated solver
+// graphs (lead graph + the rest) with the signature of what they were captured with.
+struct SolverWs {
+  void* base = nullptr;
+  size_t cap = 0;
+  bool busy = false;
+  cudaEvent_t done = nullptr;  // end of the last call's use of the arena
+  std::vector<uint8_t> sig;
+  cudaGraph_t graph[2] = {nullptr, nullptr};
+  cudaGraphExec_t exec[2] = {nullptr, nullptr};
+  std::vector<int64_t> body_per_pair;
+  int final_selects = 0;
+  // kernel-value tile list of the last call (FULL_K on tcgen05): key, device copy, wave split
+  std::vector<int64_t> tkey;
+  int2* tiles = nullptr;
+  size_t n_tiles = 0, n_wave0 = 0;
+  double kv_subset = -1;
+  void park_graphs() {  // destroyed later by destroy_parked_graphs (it blocks until the device idles)
+    std::lock_guard<std::mutex> lk(g_parked_mu);
+    for (int i = 0; i < 2; ++i) {
+      if (exec[i] || graph[i]) g_parked.emplace_back(exec[i], graph[i]);
+      exec[i] = nullptr;
+      graph[i] = nullptr;
+    }
+    sig.clear();
+  }
+};
+std::mutex g_sws_mu;
+SolverWs g_sws[64];
+
+// A training call's hold on its device's SolverWs (ws == nullptr: not cacheable, or in use by a
+// concurrent call -- the caller then allocates its own arena and tiles and builds its own graphs).
+struct SolverCacheLease {
+  SolverWs* ws = nullptr;
+  cudaStream_t st = nullptr;
+  SolverCacheLease(int dev, cudaStream_t s) : st(s) {
+    if (dev < 0 || dev >= 64) return;
+    std::lock_guard<std::mutex> lk(g_sws_mu);
+    SolverWs& w = g_sws[dev];
+    if (w.busy) return;
+    if (w.done) GM_CUDA(cudaStreamWaitEvent(st, w.done, 0));  // the previous call is done with it
+    w.busy = true;
+    ws = &w;
+  }
+  // the cached arena, (re)allocated for `bytes` (same size as before: same base)
+  void* arena(size_t bytes) {
+    SolverWs& w = *ws;
+    if (w.cap < bytes || w.cap > 2 * bytes + ((size_t)64 << 20)) {
+      w.park_graphs();  // their kernel arguments point into the old arena
+      if (w.base) cudaFreeAsync(w.base, st);
+      w.base = nullptr;
+      w.cap = 0;
+      GM_CUDA(cudaMallocAsync(&w.base, bytes, st));
+      w.cap = bytes;
+    }
+    return w.base;
+  }
+  ~SolverCacheLease() {
+    if (!ws) return;
+    std::lock_guard<std::mutex> lk(g_sws_mu);
+    if (!ws->done) cudaEventCreateWithFlags(&ws->done, cudaEventDisableTiming);
+    if (ws->done) cudaEventRecord(ws->done, st);
+    ws->busy = false;
+  }
+  SolverCacheLease(const SolverCacheLease&) = delete;
+  SolverCacheLease& operator=(const SolverCacheLease&) = delete;
+};
+
 template <class T>
 struct PinnedBuf {
   T* p = nullptr;
@@ -247,11 +337,82 @@ struct PinnedBuf {
   }
 };
 
-template <class T>
-T* dev_alloc(size_t count, cudaStream_t st) {
-  T* p = nullptr;
-  if (count) GM_CUDA(cudaMallocAsync((void**)&p, count * sizeof(T), st));
+// Device buffers of a model (DevModel).  A model is freed on the library stream while the next
+// one is typically allocated on the caller's stream; the stream-ordered pool then cannot hand the
+// freed blocks straight to the new allocation, and a cudaMallocAsync of the ~90 MB int8 SV planes
+// was measured blocking the host for 2-28 ms per training call (GMPSVM_SLOW_API).  So a freed
+// model's buffers go to a small per-device cache instead, each with an event marking the end of
+// its last use; an allocation of a size within 25 % of a cached block takes it and makes its
+// stream wait on that event (no host block).  Bounded: beyond kModelCacheBytes the oldest cached
+// blocks are released to the pool.
+constexpr size_t kModelCacheBytes = (size_t)2 << 30;
+struct CachedBlock {
+  void* p;
+  size_t bytes;
+  cudaEvent_t ev;
+};
+std::mutex g_mcache_mu;
+std::deque<CachedBlock> g_mcache[64];
+std::map<void*, size_t> g_msize[64];  // live and cached model blocks: bytes
+
+void* model_alloc(size_t bytes, cudaStream_t st, int dev) {
+  if (!bytes) return nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_mcache_mu);
+    auto& c = g_mcache[dev];
+    int best = -1;
+    for (int i = 0; i < (int)c.size(); ++i)
+      if (c[i].bytes >= bytes && c[i].bytes - bytes <= bytes / 4 && (best < 0 || c[i].bytes < c[best].bytes)) best = i;
+    if (best >= 0) {
+      const CachedBlock b = c[best];
+      c.erase(c.begin() + best);
+      GM_CUDA(cudaStreamWaitEvent(st, b.ev, 0));
+      cudaEventDestroy(b.ev);
+      return b.p;
+    }
+  }
+  void* p = nullptr;
+  GM_CUDA(cudaMallocAsync(&p, bytes, st));
+  std::lock_guard<std::mutex> lk(g_mcache_mu);
+  g_msize[dev][p] = bytes;
   return p;
+}
+
+// ls: a stream ordered after the block's last use
+void model_free(void* p, cudaStream_t ls, int dev) {
+  if (!p) return;
+  std::lock_guard<std::mutex> lk(g_mcache_mu);
+  auto it = g_msize[dev].find(p);
+  if (!ls || it == g_msize[dev].end()) {  // no stream (device gone?) or not ours: plain free
+    if (it != g_msize[dev].end()) g_msize[dev].erase(it);
+    cudaFree(p);
+    return;
+  }
+  cudaEvent_t ev = nullptr;
+  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess || cudaEventRecord(ev, ls) != cudaSuccess) {
+    if (ev) cudaEventDestroy(ev);
+    g_msize[dev].erase(it);
+    cudaFreeAsync(p, ls);
+    return;
+  }
+  auto& c = g_mcache[dev];
+  c.push_back(CachedBlock{p, it->second, ev});
+  size_t tot = 0;
+  for (const auto& b : c) tot += b.bytes;
+  while (tot > kModelCacheBytes && !c.empty()) {  // release the oldest
+    const CachedBlock b = c.front();
+    c.pop_front();
+    tot -= b.bytes;
+    cudaStreamWaitEvent(ls, b.ev, 0);
+    cudaEventDestroy(b.ev);
+    g_msize[dev].erase(b.p);
+    cudaFreeAsync(b.p, ls);
+  }
+}
+
+template <class T>
+T* dev_alloc(size_t count, cudaStream_t st, int dev) {
+  return static_cast<T*>(model_alloc(count * sizeof(T), st, dev));
 }
 
 // Per-thread cached pinned host staging (cudaMallocHost / cudaFreeHost are slow and the
@@ -275,7 +436,7 @@ T* pinned_scratch(size_t count, int slot = 0) {
 
 enum { PH_STAGE, PH_KERNEL, PH_SELECT, PH_SUB, PH_FUP, PH_FIN, PH_DEC, PH_COUPLE, PH_D2H, PH_SOLVER, PH_N };
 
-// timing events of the overlap mode's kernel-value waves (destroyed with the scope)
+// timing events of lead mode's kernel-value waves (destroyed with the scope)
 struct TimedEvents {
   cudaEvent_t a = nullptr, b = nullptr;
   TimedEvents() {
@@ -337,11 +498,7 @@ DevModel::~DevModel() {
   if (ls && last_use) cudaStreamWaitEvent(ls, last_use, 0);
   void* ptrs[] = {SvT,   nsv,      coef, items,     item_begin, item_end, b,    A,    B,     SvHi,
                   SvLo,  nsvc,     mu,   alpha_dev, coef64,     nsv64,    SvI8, sv_e, sv_n64};
-  for (void* p : ptrs)
-    if (p) {
-      if (ls) cudaFreeAsync(p, ls);
-      else cudaFree(p);
-    }
+  for (void* p : ptrs) model_free(p, ls, device >= 0 && device < 64 ? device : 0);
   if (last_use) cudaEventDestroy(last_use);
   if (prev >= 0) cudaSetDevice(prev);
 }
@@ -493,15 +650,15 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   if (items.empty()) items.push_back(DecItem{0, 0, 0, 0});  // no SV at all: zero contribution
   dm->n_items = (int)items.size();
   HT("host_coef");
-  dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad, st);
-  dm->nsv = dev_alloc<float>(dm->nsv_pad, st);
-  dm->coef = dev_alloc<float>((size_t)dm->nsv_pad * dm->km1_pad, st);
-  dm->items = dev_alloc<DecItem>(items.size(), st);
-  dm->item_begin = dev_alloc<int32_t>(k, st);
-  dm->item_end = dev_alloc<int32_t>(k, st);
-  dm->b = dev_alloc<double>(P, st);
-  dm->A = dev_alloc<double>(P, st);
-  dm->B = dev_alloc<double>(P, st);
+  dm->SvT = dev_alloc<float>((size_t)dm->d_pad * dm->nsv_pad, st, device);
+  dm->nsv = dev_alloc<float>(dm->nsv_pad, st, device);
+  dm->coef = dev_alloc<float>((size_t)dm->nsv_pad * dm->km1_pad, st, device);
+  dm->items = dev_alloc<DecItem>(items.size(), st, device);
+  dm->item_begin = dev_alloc<int32_t>(k, st, device);
+  dm->item_end = dev_alloc<int32_t>(k, st, device);
+  dm->b = dev_alloc<double>(P, st, device);
+  dm->A = dev_alloc<double>(P, st, device);
+  dm->B = dev_alloc<double>(P, st, device);
   DevBuf<int64_t> d_src(slot_src.size(), st);
   GM_CUDA(cudaMemcpyAsync(d_src.get(), slot_src.data(), slot_src.size() * 8, cudaMemcpyHostToDevice, st));
   // conditioning of the decision values: sum_j |alpha_pj| per trained pair
@@ -524,9 +681,9 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   static const char* dec_env = getenv("GMPSVM_DEC");
   const std::string dec_mode = dec_env ? dec_env : "";
   // FP64 coefficients: the int8 and FP64 paths contract in FP64
-  dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st);
+  dm->coef64 = dev_alloc<double>((size_t)dm->nsv_pad * dm->km1_pad, st, device);
   if (dev_coef) {
-    dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st);
+    dm->alpha_dev = dev_alloc<double>(std::max<int64_t>(alpha_tot, 1), st, device);
     if (alpha_tot) GM_CUDA(cudaMemcpyAsync(dm->alpha_dev, alpha_hp, (size_t)alpha_tot * 8, cudaMemcpyDeviceToDevice, st));
     dm->alpha_dev_off = *alpha_off;
     DevBuf<int64_t> d_g(slot_g.size(), st), d_aoff(P, st), d_off(k + 1, st), d_cc(k, st);
@@ -549,15 +706,15 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   launch_stage_features(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvT, dm->nsv_pad, dm->d_pad, dm->nsv_pad, dm->nsv,
                         nullptr, st);
   HT("h2d_svt");
-  dm->nsv64 = dev_alloc<double>(dm->nsv_pad, st);
+  dm->nsv64 = dev_alloc<double>(dm->nsv_pad, st, device);
   launch_col_norms64(dm->SvT, dm->nsv_pad, dm->nsv_pad, dm->d_pad, dm->nsv64, st);
   dm->h_items = items;
   // int8-digit SV planes (the default RBF path, dec_i8.cu)
   uint32_t amax_bits = 0;
   if (m.kernel == 0 && dm->km1_pad <= dec_i8_max_km1()) {
-    dm->SvI8 = dev_alloc<int8_t>(dec_i8_plane_bytes(dm->nsv_pad, m.d), st);
-    dm->sv_e = dev_alloc<int32_t>(dm->nsv_pad, st);
-    dm->sv_n64 = dev_alloc<double>(dm->nsv_pad, st);
+    dm->SvI8 = dev_alloc<int8_t>(dec_i8_plane_bytes(dm->nsv_pad, m.d), st, device);
+    dm->sv_e = dev_alloc<int32_t>(dm->nsv_pad, st, device);
+    dm->sv_n64 = dev_alloc<double>(dm->nsv_pad, st, device);
     DevBuf<unsigned> d_amax(1, st);
     GM_CUDA(cudaMemsetAsync(d_amax.get(), 0, 4, st));
     launch_stage_i8(rows, dm->nsv_pad, m.d, d_src.get(), dm->SvI8, dm->nsv_pad, dm->sv_e, dm->sv_n64, d_amax.get(), st);
@@ -569,10 +726,10 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   dm->tc = dec_mode == "f16" && krow_use_tc() && krow_split_f16() && dm->km1_pad <= (m.kernel != 0 ? 12 : dec_tc_max_km1());
   if (dm->tc) {
     dm->dpt = krow_tc_d_pad(m.d);
-    dm->mu = dev_alloc<float>(m.d, st);
-    dm->SvHi = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st);
-    dm->SvLo = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st);
-    dm->nsvc = dev_alloc<float>(dm->nsv_pad, st);
+    dm->mu = dev_alloc<float>(m.d, st, device);
+    dm->SvHi = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st, device);
+    dm->SvLo = dev_alloc<float>(krow_tc_buf_floats(dm->nsv_pad, dm->dpt), st, device);
+    dm->nsvc = dev_alloc<float>(dm->nsv_pad, st, device);
     if (mu_in) {
       GM_CUDA(cudaMemcpyAsync(dm->mu, mu_in, (size_t)m.d * 4, cudaMemcpyDeviceToDevice, st));
       dm->sc = sc_in;
@@ -799,6 +956,9 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   cudaStream_t st = get_stream(opt);
   const uint64_t launches0 = g_launches.load();
   PhaseTimer tm(st);
+  static const bool lead_dbg = getenv("GMPSVM_LEAD_DEBUG") != nullptr;  // diagnostics: device timeline
+  TimedEvents dbg0, dbg1;  // call entry (a), solver done on st (b); finalize done (dbg1.a)
+  if (lead_dbg) GM_CUDA(cudaEventRecord(dbg0.a, st));
 
   // ---------------- a1 staging
   HT("stage0");
@@ -863,16 +1023,26 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   if (hbad) throw Error(GMPSVM_EINVAL, "X contains non-finite values");
   tm.mark(PH_STAGE);
   HT("stage1");
-  // class means of the staged rows: pairs of the closest classes are expected to need the most
-  // solver work, so they get their kernel values first (overlap mode) and their own branches
-  std::vector<double> cdist;  // squared distance of the class means, per pair index (tc path)
+  // class means and spreads of the staged rows: the pairs whose classes overlap most -- smallest
+  // Fisher ratio |mu_s - mu_t|^2 / (tr S_s + tr S_t) -- are expected to need the most solver work
+  // (measured, MNIST-shaped: Spearman 0.85 against the pairs' inner SMO steps, the hardest pair
+  // (0,8) ranked first; tools/pair_difficulty.py), so they come first: their own graph branches
+  // and, in lead mode below, their kernel values first
+  std::vector<double> fisher;  // per pair index (tc path)
   if (use_tc) {
-    DevBuf<float> d_mu((size_t)k * d_pad, st);
-    launch_class_means(Xhi.get(), d_pad, d_off.get(), k, d_mu.get(), st);
-    std::vector<float> mu((size_t)k * d_pad);
+    DevBuf<float> d_mu((size_t)k * d_pad, st), d_m2((size_t)k * d_pad, st);
+    launch_class_means(Xhi.get(), d_pad, d_off.get(), k, d_mu.get(), d_m2.get(), st);
+    std::vector<float> mu((size_t)k * d_pad), m2((size_t)k * d_pad);
     GM_CUDA(cudaMemcpyAsync(mu.data(), d_mu.get(), mu.size() * 4, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaMemcpyAsync(m2.data(), d_m2.get(), m2.size() * 4, cudaMemcpyDeviceToHost, st));
     GM_CUDA(cudaStreamSynchronize(st));
-    cdist.assign((size_t)k * (k - 1) / 2, 0.0);
+    std::vector<double> var(k, 0.0);
+    for (int c = 0; c < k; ++c)
+      for (int f = 0; f < d_pad; ++f) {
+        const double m = mu[(size_t)c * d_pad + f];
+        var[c] += std::max(0.0, (double)m2[(size_t)c * d_pad + f] - m * m);
+      }
+    fisher.assign((size_t)k * (k - 1) / 2, 0.0);
     for (int s0 = 0; s0 < k; ++s0)
       for (int t0 = s0 + 1; t0 < k; ++t0) {
         double acc = 0.0;
@@ -880,7 +1050,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
           const double df = (double)mu[(size_t)s0 * d_pad + f] - mu[(size_t)t0 * d_pad + f];
           acc += df * df;
         }
-        cdist[pair_index(s0, t0, k)] = acc;
+        fisher[pair_index(s0, t0, k)] = acc / std::max(var[s0] + var[t0], 1e-30);
       }
   }
 
@@ -910,10 +1080,10 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
       ps[pair_index(s, t, k)] = s;
       pt[pair_index(s, t, k)] = t;
     }
-  // largest pairs first (closest class means first on the tensor-core path, see above): they
+  // largest pairs first (smallest Fisher ratio first on the tensor-core path, see above): they
   // start first and share streams with pairs of similar cost
-  if (!cdist.empty())
-    std::stable_sort(pids.begin(), pids.end(), [&](int x, int y) { return cdist[x] < cdist[y]; });
+  if (!fisher.empty())
+    std::stable_sort(pids.begin(), pids.end(), [&](int x, int y) { return fisher[x] < fisher[y]; });
   else
     std::stable_sort(pids.begin(), pids.end(),
                      [&](int x, int y) { return cc[ps[x]] + cc[pt[x]] > cc[ps[y]] + cc[pt[y]]; });
@@ -982,132 +1152,206 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // FULL_K: the n x ldk matrix; ROW_CACHE: the per-pair B x round_up(n_p, 4) row buffers
   KWorkspace K(opt.device, full_k ? (size_t)n * ldk * sizeof(float) : (size_t)bytes_R, st);
   HT("k_alloc");
-  std::vector<int2> tiles;
-  DevBuf<int2> d_tiles;
-  // Overlap mode (tensor-core FULL_K path with the device-driven default solver): the kernel
-  // matrix is computed in waves on a low-priority stream, wave w holding the tiles first needed
-  // by the w-th pair (pair order above); each pair's solver branch starts as soon as the waves
-  // covering its class blocks (s,s), (s,t), (t,t) are done, so the solver of the first pairs runs
-  // while the kernel values of the others are still being computed.  Tiles no trained pair needs
-  // (pair subsets, multi-GPU shards) are skipped.
-  // Opt-in (GMPSVM_OVERLAP=1): measured slower on MNIST-shaped data (B200: 62 vs 57 ms train +
-  // predict) -- the waves' tensor/HBM load stretches the solver's latency-bound chain more than
-  // the overlap saves.
-  static const bool overlap_env = getenv("GMPSVM_OVERLAP") && std::string(getenv("GMPSVM_OVERLAP")) == "1";
+  // The solver's state, its graphs and the kernel-value tile list are kept per device and reused by
+  // the next call of the same shape in the default regime (FULL_K, every pair on the wsolve.cu
+  // kernels, no diagnostics); see the arena below.
+  static const bool smo_prof = getenv("GMPSVM_SMO_PHASES") != nullptr;
+  // GMPSVM_TRACE=<pair position>: kernel timeline of that pair (entries sorted largest pair first)
+  static const int trace_pos = getenv("GMPSVM_TRACE") ? atoi(getenv("GMPSVM_TRACE")) : -1;
+  static const bool no_reuse = getenv("GMPSVM_GRAPH_REUSE") && std::string(getenv("GMPSVM_GRAPH_REUSE")) == "0";
+  const bool cacheable = !no_reuse && full_k && !smo_prof && trace_pos < 0 && ws_solve_supported(B, np_max);
+  SolverCacheLease lease(cacheable ? opt.device : -1, st);  // cached arena, graphs, tiles -- or none
+  DevBuf<int2> d_tiles_own;
+  const int2* d_tiles = nullptr;
+  size_t n_tiles = 0;
+  // Lead mode (default on the tensor-core FULL_K path with the device-driven solver): the first
+  // pairs -- the predicted hardest, above -- form a graph of their own (one branch each) that starts
+  // as soon as the kernel values of their class blocks (s,s), (s,t), (t,t) are done (wave 0, on
+  // every SM); the rest of the kernel matrix (wave 1) is then computed on all but `reserve` SMs,
+  // where the lead chains run, and the other pairs -- a second graph -- wait for all of it.  The
+  // solver's critical path, the hardest pair's chain of outer iterations, so overlaps the
+  // kernel-value contraction instead of following it.  GMPSVM_LEAD=<pairs> (0: off),
+  // GMPSVM_LEAD_RESERVE=<SMs>.
   const bool fk_tc = full_k && use_tc;  // the FULL_K contraction on tcgen05
-  const bool overlap = overlap_env && ktype == 0 && fk_tc && ws_solve_supported(B, np_max);
+  static const int lead_env = getenv("GMPSVM_LEAD") ? std::max(0, atoi(getenv("GMPSVM_LEAD"))) : 1;
+  static const int reserve_env = getenv("GMPSVM_LEAD_RESERVE") ? std::max(0, atoi(getenv("GMPSVM_LEAD_RESERVE"))) : 8;
+  // Solver graph branches (below): the runtime runs at most CUDA_DEVICE_MAX_CONNECTIONS branches
+  // concurrently -- a branch beyond that shares a hardware queue with another and waits for it --
+  // so the pairs are packed into that many branches: the first pairs alone, the last two (or more)
+  // to a branch in lockstep.  Lead mode keeps two queues more free (the lead graph's and the
+  // kernel-value stream's): measured, a rest branch otherwise queued behind the lead chain.
+  const int conn = connections_in_effect();
+  const int n_lead = (fk_tc && lead_env > 0 && Pl > lead_env && conn - lead_env - 2 >= 1 && ws_solve_supported(B, np_max))
+                         ? lead_env
+                         : 0;
+  const bool lead = n_lead > 0;
+  const int nb_lead = n_lead;  // lead graph: branches [0, nb_lead), one pair each
+  const int nb_rest = std::min(Pl - n_lead, lead ? conn - n_lead - 2 : conn);
+  const int nbr = nb_lead + nb_rest;
+  std::vector<int> bb(nbr + 1, 0);
+  {
+    for (int b = 0; b < nb_lead; ++b) bb[b + 1] = b + 1;
+    const int m = (Pl - n_lead) / nb_rest, r = (Pl - n_lead) % nb_rest;  // the last r branches take m + 1 pairs
+    for (int b = 0; b < nb_rest; ++b) bb[nb_lead + b + 1] = bb[nb_lead + b] + m + (b >= nb_rest - r ? 1 : 0);
+  }
   cudaStream_t kst = krow_stream(opt.device);
   TimedEvents kev;
   cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
-  std::vector<int> wave_off;     // tile range of wave w: [wave_off[w], wave_off[w + 1])
-  std::vector<int> ready_wave;   // per pair position: the wave after which its kernel values are complete
-  const bool two_cta = fk_tc && !overlap && ktype == 0 && krow_tc_2cta();  // overlap waves: single-CTA tiles
+  EventPool evk;
+  TimedEvents kev_w, kev_g, kev_s;  // lead mode: wave 0 done (a); lead / rest graph start (kev_s), done (kev_g)
+  cudaEvent_t ev_w0 = nullptr;
+  size_t n_wave0 = 0;
+  const bool two_cta = fk_tc && !lead && ktype == 0 && krow_tc_2cta();  // lead waves: single-CTA tiles
   double kv_subset = -1;  // >= 0: kernel values computed for a pair subset (tiles skipped)
   if (fk_tc) {
-    tiles = krow_tc_tiles(n, two_cta);
-    if (!overlap && !two_cta && Pl < P) {
-      // pair subset (multi-GPU shard, pair_ids): only the tiles overlapping a class block
-      // (s,s), (s,t), (t,t) of a trained pair are computed (PAPER.md L313-L325 sharing, per rank)
-      std::vector<uint8_t> need((size_t)k * k, 0);
-      for (int i = 0; i < Pl; ++i) {
-        need[(size_t)hp[i].s * k + hp[i].s] = need[(size_t)hp[i].t * k + hp[i].t] = 1;
-        need[(size_t)std::min(hp[i].s, hp[i].t) * k + std::max(hp[i].s, hp[i].t)] = 1;
-      }
-      auto cls = [&](int64_t r) { return (int)(std::upper_bound(coff.begin(), coff.end(), r) - coff.begin()) - 1; };
-      std::vector<int2> kept;
-      for (const int2 tl : tiles) {
-        const int64_t r0 = (int64_t)tl.x * kKrowTileRows, c0 = (int64_t)tl.y * kKrowTileRows;
-        const int ra = cls(r0), rb = cls(std::min<int64_t>(n, r0 + kKrowTileRows) - 1);
-        const int ca = cls(c0), cb = cls(std::min<int64_t>(n, c0 + kKrowTileRows) - 1);
-        bool any = false;
-        for (int a0 = ra; a0 <= rb && !any; ++a0)
-          for (int b0 = ca; b0 <= cb && !any; ++b0) any = need[(size_t)std::min(a0, b0) * k + std::max(a0, b0)] != 0;
-        if (any) kept.push_back(tl);
-      }
-      tiles.swap(kept);
-      kv_subset = 0;  // kernel values (r <= c) the kept tiles compute
-      for (const int2 tl : tiles) {
-        const int64_t r0 = (int64_t)tl.x * kKrowTileRows, c0 = (int64_t)tl.y * kKrowTileRows;
-        const int64_t nr = std::min<int64_t>(n, r0 + kKrowTileRows) - r0, nc = std::min<int64_t>(n, c0 + kKrowTileRows) - c0;
-        kv_subset += tl.x == tl.y ? (double)nr * (double)(nr + 1) / 2.0 : (double)nr * (double)nc;
-      }
+    // class range [cr[2i], cr[2i+1]] of the rows of tile row / column i
+    const int nti = (int)ceil_div(n, kKrowTileRows);
+    std::vector<int> cr(2 * (size_t)nti);
+    for (int i = 0, c = 0; i < nti; ++i) {
+      const int64_t r0 = (int64_t)i * kKrowTileRows, r1 = std::min<int64_t>(n, r0 + kKrowTileRows) - 1;
+      while (coff[c + 1] <= r0) ++c;
+      int e = c;
+      while (coff[e + 1] <= r1) ++e;
+      cr[2 * i] = c;
+      cr[2 * i + 1] = e;
     }
-    if (overlap) {
-      const int INF = INT_MAX;
-      std::vector<int> minpos(k, INF);  // first position of a pair containing class c
-      std::vector<int> pos((size_t)k * k, INF);
-      for (int i = 0; i < Pl; ++i) {
-        minpos[hp[i].s] = std::min(minpos[hp[i].s], i);
-        minpos[hp[i].t] = std::min(minpos[hp[i].t], i);
-        pos[(size_t)hp[i].s * k + hp[i].t] = i;
+    // does tile tl overlap a class block marked in blk (k x k, upper triangle)?
+    auto touches = [&](const int2 tl, const std::vector<uint8_t>& blk) {
+      for (int a0 = cr[2 * tl.x]; a0 <= cr[2 * tl.x + 1]; ++a0)
+        for (int b0 = cr[2 * tl.y]; b0 <= cr[2 * tl.y + 1]; ++b0)
+          if (blk[(size_t)std::min(a0, b0) * k + std::max(a0, b0)]) return true;
+      return false;
+    };
+    auto blocks_of = [&](int i0, int i1) {  // class blocks of the pairs at positions [i0, i1)
+      std::vector<uint8_t> blk((size_t)k * k, 0);
+      for (int i = i0; i < i1; ++i) {
+        blk[(size_t)hp[i].s * k + hp[i].s] = blk[(size_t)hp[i].t * k + hp[i].t] = 1;
+        blk[(size_t)std::min(hp[i].s, hp[i].t) * k + std::max(hp[i].s, hp[i].t)] = 1;
       }
-      auto cls = [&](int64_t r) { return (int)(std::upper_bound(coff.begin(), coff.end(), r) - coff.begin()) - 1; };
-      std::vector<int> tw(tiles.size());
-      std::vector<int> blockmax((size_t)k * k, -1);
-      for (size_t ti = 0; ti < tiles.size(); ++ti) {
-        const int64_t r0 = (int64_t)tiles[ti].x * kKrowTileRows, c0 = (int64_t)tiles[ti].y * kKrowTileRows;
-        const int ra = cls(r0), rb = cls(std::min<int64_t>(n, r0 + kKrowTileRows) - 1);
-        const int ca = cls(c0), cb = cls(std::min<int64_t>(n, c0 + kKrowTileRows) - 1);
-        int w = INF;
-        for (int a0 = ra; a0 <= rb; ++a0)
-          for (int b0 = ca; b0 <= cb; ++b0) {
-            const int lo = std::min(a0, b0), hi = std::max(a0, b0);
-            w = std::min(w, lo == hi ? minpos[lo] : pos[(size_t)lo * k + hi]);
-          }
-        tw[ti] = w;
-        if (w == INF) continue;
-        for (int a0 = ra; a0 <= rb; ++a0)
-          for (int b0 = ca; b0 <= cb; ++b0) {
-            int& m = blockmax[(size_t)std::min(a0, b0) * k + std::max(a0, b0)];
-            m = std::max(m, w);
-          }
+      return blk;
+    };
+    const bool subset = !two_cta && Pl < P;
+    const std::vector<uint8_t> need = subset ? blocks_of(0, Pl) : std::vector<uint8_t>();
+    const std::vector<uint8_t> lb = lead ? blocks_of(0, n_lead) : std::vector<uint8_t>();
+    std::vector<int64_t> tkey = {n, two_cta ? 1 : 0, k};  // what the tile list depends on
+    tkey.insert(tkey.end(), coff.begin(), coff.end());
+    for (const uint8_t v : need) tkey.push_back(v);
+    tkey.push_back(-1);
+    for (const uint8_t v : lb) tkey.push_back(v);
+    SolverWs* ws = lease.ws;
+    if (ws && ws->tiles && ws->tkey == tkey) {  // the last call's list
+      d_tiles = ws->tiles;
+      n_tiles = ws->n_tiles;
+      n_wave0 = ws->n_wave0;
+      kv_subset = ws->kv_subset;
+    } else {
+      std::vector<int2> tiles = krow_tc_tiles(n, two_cta);
+      if (subset) {
+        // pair subset (multi-GPU shard, pair_ids): only the tiles overlapping a class block
+        // (s,s), (s,t), (t,t) of a trained pair are computed (PAPER.md L313-L325 sharing, per rank)
+        std::vector<int2> kept;
+        for (const int2 tl : tiles)
+          if (touches(tl, need)) kept.push_back(tl);
+        tiles.swap(kept);
+        kv_subset = 0;  // kernel values (r <= c) the kept tiles compute
+        for (const int2 tl : tiles) {
+          const int64_t r0 = (int64_t)tl.x * kKrowTileRows, c0 = (int64_t)tl.y * kKrowTileRows;
+          const int64_t nr = std::min<int64_t>(n, r0 + kKrowTileRows) - r0, nc = std::min<int64_t>(n, c0 + kKrowTileRows) - c0;
+          kv_subset += tl.x == tl.y ? (double)nr * (double)(nr + 1) / 2.0 : (double)nr * (double)nc;
+        }
       }
-      std::vector<int> order(tiles.size());
-      for (size_t ti = 0; ti < tiles.size(); ++ti) order[ti] = (int)ti;
-      std::stable_sort(order.begin(), order.end(), [&](int x, int y) { return tw[x] < tw[y]; });
-      std::vector<int2> sorted;
-      sorted.reserve(tiles.size());
-      wave_off.assign(Pl + 1, 0);
-      for (int ti : order) {
-        if (tw[ti] == INF) break;
-        sorted.push_back(tiles[ti]);
-        wave_off[tw[ti] + 1] += 1;
+      if (lead) {  // wave 0: the tiles of the lead pairs' class blocks (blocked order kept), then the rest
+        std::vector<int2> w0, w1;
+        for (const int2 tl : tiles) (touches(tl, lb) ? w0 : w1).push_back(tl);
+        n_wave0 = w0.size();
+        w0.insert(w0.end(), w1.begin(), w1.end());
+        tiles.swap(w0);
       }
-      for (int w = 0; w < Pl; ++w) wave_off[w + 1] += wave_off[w];
-      tiles.swap(sorted);
-      ready_wave.assign(Pl, -1);
-      for (int i = 0; i < Pl; ++i) {
-        const int s0 = hp[i].s, t0 = hp[i].t;
-        ready_wave[i] = std::max(std::max(blockmax[(size_t)s0 * k + s0], blockmax[(size_t)s0 * k + t0]),
-                                 blockmax[(size_t)t0 * k + t0]);
+      n_tiles = tiles.size();
+      int2* dt = nullptr;
+      if (ws) {
+        if (ws->tiles) cudaFreeAsync(ws->tiles, st);
+        ws->tiles = nullptr;
+        ws->tkey.clear();
+        GM_CUDA(cudaMallocAsync((void**)&ws->tiles, std::max<size_t>(n_tiles, 1) * sizeof(int2), st));
+        dt = ws->tiles;
+        ws->tkey = tkey;
+        ws->n_tiles = n_tiles;
+        ws->n_wave0 = n_wave0;
+        ws->kv_subset = kv_subset;
+      } else {
+        new (&d_tiles_own) DevBuf<int2>(n_tiles, st);
+        dt = d_tiles_own.get();
       }
+      GM_CUDA(cudaMemcpyAsync(dt, tiles.data(), n_tiles * sizeof(int2), cudaMemcpyHostToDevice, st));
+      d_tiles = dt;
     }
-    new (&d_tiles) DevBuf<int2>(tiles.size(), st);
-    GM_CUDA(cudaMemcpyAsync(d_tiles.get(), tiles.data(), tiles.size() * sizeof(int2), cudaMemcpyHostToDevice, st));
   }
   tm.mark(PH_KERNEL);
-  if (fk_tc && !overlap)
-  {
-    const KrowKernel kk{ktype, (float)gamma, (float)kcoef0, 0.f, kdegree};
-    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get(), (int)tiles.size(), norms.get(), n, gamma, ksc, K.get(),
-                   ldk, st, two_cta, ktype != 0 ? &kk : nullptr);
-  }
-  else if (full_k && !use_tc)
+  const KrowKernel kk{ktype, (float)gamma, (float)kcoef0, 0.f, kdegree};
+  const KrowKernel* kkp = ktype != 0 ? &kk : nullptr;
+  if (fk_tc && !lead) {
+    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles, (int)n_tiles, norms.get(), n, gamma, ksc, K.get(), ldk, st,
+                   two_cta, kkp);
+  } else if (fk_tc) {  // the waves on the low-priority stream: the solver's CTAs are dispatched first
+    cudaEvent_t ev_staged = evk.get();
+    GM_CUDA(cudaEventRecord(ev_staged, st));
+    GM_CUDA(cudaStreamWaitEvent(kst, ev_staged, 0));
+    GM_CUDA(cudaEventRecord(ev_k0, kst));
+    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles, (int)n_wave0, norms.get(), n, gamma, ksc, K.get(), ldk, kst,
+                   false, kkp);
+    ev_w0 = kev_w.a;
+    GM_CUDA(cudaEventRecord(ev_w0, kst));
+    if (n_tiles > n_wave0)
+      launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles + n_wave0, (int)(n_tiles - n_wave0), norms.get(), n, gamma,
+                     ksc, K.get(), ldk, kst, false, kkp, reserve_env);
+    GM_CUDA(cudaEventRecord(ev_k1, kst));
+  } else if (full_k && !use_tc) {
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
+  }
   tm.mark(PH_KERNEL);
   HT("krow_launched");
 
   // ---------------- a4-a6 batched working-set solver, all pairs concurrently
   const int Bw = B;
-  DevBuf<PairDesc> d_pairs(Pl, st);
+  // The solver's state lives in one arena.  In the default regime (FULL_K, every pair on the
+  // wsolve.cu kernels, no diagnostics) the arena and the instantiated solver graphs are kept per
+  // device and reused by the next call of the same shape: same buffers, same kernel arguments,
+  // so the graphs are relaunched as they are -- no per-call capture / instantiation (~4.7 ms of
+  // host time) and no graph destruction, which blocks the host until the device is idle and then
+  // takes another ~3.4 ms (measured, GMPSVM_HOST_TIMING / GMPSVM_LEAD_DEBUG).  The per-call state
+  // is re-initialised by launch_init_pairs as before; the kernels never read state they have not
+  // written in this call (the same holds for fresh pool memory).
+  ArenaPtr<PairDesc> d_pairs;
+  ArenaPtr<double> d_alpha, d_f, d_v, d_dcoef, d_gap, d_b, d_A, d_B;
+  ArenaPtr<uint32_t> d_stamp;
+  ArenaPtr<int32_t> d_ws, d_wsn, d_wst, d_status, d_outer, d_sig;
+  ArenaPtr<int64_t> d_inner, d_cyc, d_body;
+  ArenaPtr<float> d_Kws;
+  ArenaLayout lay;
+  lay.add(d_pairs, Pl);
+  lay.add(d_alpha, tot);
+  lay.add(d_f, tot);
+  lay.add(d_v, tot);
+  lay.add(d_dcoef, (size_t)Pl * Bw);
+  lay.add(d_gap, Pl);
+  lay.add(d_b, Pl);
+  lay.add(d_A, Pl);
+  lay.add(d_B, Pl);
+  lay.add(d_stamp, tot);
+  lay.add(d_ws, (size_t)Pl * Bw);
+  lay.add(d_wsn, Pl);
+  lay.add(d_wst, (size_t)Pl * Bw);
+  lay.add(d_status, Pl);
+  lay.add(d_outer, Pl);
+  lay.add(d_sig, Pl);
+  lay.add(d_inner, Pl);
+  lay.add(d_cyc, Pl);
+  lay.add(d_body, Pl);
+  lay.add(d_Kws, (size_t)Pl * kws_pair_stride(Bw));
+  DevBuf<uint8_t> arena_own(lease.ws ? 0 : lay.bytes, st);
+  lay.place(lease.ws ? lease.arena(lay.bytes) : arena_own.get());
   GM_CUDA(cudaMemcpyAsync(d_pairs.get(), hp.data(), Pl * sizeof(PairDesc), cudaMemcpyHostToDevice, st));
-  DevBuf<double> d_alpha(tot, st), d_f(tot, st), d_v(tot, st), d_dcoef((size_t)Pl * Bw, st), d_gap(Pl, st),
-      d_b(Pl, st), d_A(Pl, st), d_B(Pl, st);
-  DevBuf<uint32_t> d_stamp(tot, st);
-  DevBuf<int32_t> d_ws((size_t)Pl * Bw, st), d_wsn(Pl, st), d_wst((size_t)Pl * Bw, st), d_status(Pl, st),
-      d_outer(Pl, st), d_sig(Pl, st);
-  DevBuf<int64_t> d_inner(Pl, st), d_cyc(Pl, st);
-  DevBuf<float> d_Kws((size_t)Pl * kws_pair_stride(Bw), st);
   const bool rc = !full_k;
   const bool rc_tc = rc && use_tc;  // ROW_CACHE rows on tcgen05
   DevBuf<float> d_Ahi(rc_tc ? krow_tc_buf_floats((int64_t)Pl * ldat, d_pad) : 0, st),
@@ -1117,6 +1361,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   DevBuf<int64_t> d_rows(rc ? Pl : 0, st);
   if (rc) GM_CUDA(cudaMemsetAsync(d_rows.get(), 0, Pl * 8, st));
   SolverArgs a{};
+  std::memset(&a, 0, sizeof a);  // padding included: the bytes are the cached graphs' signature
   a.pairs = d_pairs.get();
   a.K = full_k ? K.get() : nullptr;
   a.ldk = ldk;
@@ -1125,9 +1370,9 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   a.ws_slot_tmp = d_slot_tmp.get();
   a.ws_keep = d_keep.get();
   a.rows_done = d_rows.get();
-  a.XT = XT.get();
+  a.XT = rc ? XT.get() : nullptr;  // ROW_CACHE operands only (FULL_K: no per-call pointers in the graph)
   a.ldx = n_pad;
-  a.norms = norms.get();
+  a.norms = rc ? norms.get() : nullptr;
   a.ATnew = d_ATnew.get();
   a.d_pad = d_pad;
   a.ldat = ldat;
@@ -1154,21 +1399,17 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   a.gap = d_gap.get();
   a.inner_iters = d_inner.get();
   a.smo_cycles = d_cyc.get();
-  static const bool smo_prof = getenv("GMPSVM_SMO_PHASES") != nullptr;
   DevBuf<int64_t> d_phase(smo_prof ? (size_t)Pl * 5 : 0, st);
   if (smo_prof) GM_CUDA(cudaMemsetAsync(d_phase.get(), 0, (size_t)Pl * 5 * 8, st));
   a.smo_phase = smo_prof ? d_phase.get() : nullptr;
   DevBuf<int64_t> d_sphase(smo_prof ? (size_t)(Pl + 8192) * 5 : 0, st);
   if (smo_prof) GM_CUDA(cudaMemsetAsync(d_sphase.get(), 0, (size_t)(Pl + 8192) * 5 * 8, st));
   a.sel_phase = smo_prof ? d_sphase.get() : nullptr;
-  // GMPSVM_TRACE=<pair position>: kernel timeline of that pair (entries sorted largest pair first)
-  static const int trace_pos = getenv("GMPSVM_TRACE") ? atoi(getenv("GMPSVM_TRACE")) : -1;
   const int trace_cap = 1 << 16;
   DevBuf<int64_t> d_trace(trace_pos >= 0 ? (size_t)trace_cap * 3 + 2 * (size_t)Pl : 0, st);
   if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace.get(), 0, ((size_t)trace_cap * 3 + 2 * (size_t)Pl) * 8, st));
   DevBuf<int32_t> d_trace_n(trace_pos >= 0 ? 1 : 0, st);
   if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace_n.get(), 0, 4, st));
-  DevBuf<int64_t> d_body(Pl, st);
   GM_CUDA(cudaMemsetAsync(d_body.get(), 0, Pl * 8, st));
   a.body_iters = d_body.get();
   a.trace = d_trace.get();
@@ -1197,27 +1438,17 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   tm.mark(PH_SOLVER);
   HT("init");
   int64_t rc_launches = 0;  // ROW_CACHE row-contraction launches
-  GraphGuard gg;
+  GraphGuard gg, gl;  // the solver graph (lead mode: the other branches) and the lead graph
   DevBuf<int4> d_rtiles;  // ROW_CACHE tcgen05 row tiles of every branch (outlives the graph run)
   int64_t body_launches = 0;
   std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
   int n_branches = 0, final_selects = 0;
   {
-    // Device-driven outer loops (default): one CUDA graph holding, per pair, a conditional
-    // WHILE node whose body is that pair's select -> [rows] -> gather -> local SMO -> f-update
-    // chain (the f-update kernel sets the loop condition), followed by one last selection (the
-    // stop test on the final alpha).  The pairs are independent branches of the graph, so no
+    // Device-driven outer loops (default): one CUDA graph holding, per branch (packing above), a
+    // conditional WHILE node whose body is that branch's select -> [rows] -> gather -> local SMO ->
+    // f-update chain (the f-update kernel sets the loop condition), followed by one last selection
+    // (the stop test on the final alpha) on the split path.  The branches are independent, so no
     // pair waits for another at a kernel boundary and the host is not involved until the end.
-    // The runtime runs at most CUDA_DEVICE_MAX_CONNECTIONS branches of a graph concurrently (a
-    // branch beyond that waits for another to finish), so the pairs are packed into that many
-    // branches: the largest pairs alone, the smallest two (or more) to a branch in lockstep.
-    const int conn = connections_in_effect();
-    const int nbr = std::min(Pl, conn);
-    std::vector<int> bb(nbr + 1, 0);
-    {
-      const int m = Pl / nbr, r = Pl % nbr;  // the last r branches take m + 1 pairs
-      for (int b = 0; b < nbr; ++b) bb[b + 1] = bb[b] + m + (b >= nbr - r ? 1 : 0);
-    }
     // ROW_CACHE rows on tcgen05: each branch's static tile list (its pairs x row tiles x column tiles)
     std::vector<int> rtile_off(nbr + 1, 0);
     std::vector<int4> rtiles;
@@ -1230,93 +1461,135 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     new (&d_rtiles) DevBuf<int4>(std::max<size_t>(rtiles.size(), 1), st);
     if (!rtiles.empty())
       GM_CUDA(cudaMemcpyAsync(d_rtiles.get(), rtiles.data(), rtiles.size() * sizeof(int4), cudaMemcpyHostToDevice, st));
-    std::vector<cudaEvent_t> ev_wave(Pl, nullptr);
-    if (overlap) {  // kernel-value waves on the low-priority stream, one event per wave
-      cudaEvent_t ev_staged = evp.get();
-      GM_CUDA(cudaEventRecord(ev_staged, st));
-      GM_CUDA(cudaStreamWaitEvent(kst, ev_staged, 0));
-      GM_CUDA(cudaEventRecord(ev_k0, kst));
-      for (int w = 0; w < Pl; ++w) {
-        const int cnt = wave_off[w + 1] - wave_off[w];
-        if (cnt > 0)
-          launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles.get() + wave_off[w], cnt, norms.get(), n, gamma, ksc,
-                         K.get(), ldk, kst);
-        ev_wave[w] = evp.get();
-        GM_CUDA(cudaEventRecord(ev_wave[w], kst));
-      }
-      GM_CUDA(cudaEventRecord(ev_k1, kst));
-    }
-    const uint64_t l0 = g_launches.load();
-    GM_CUDA(cudaGraphCreate(&gg.graph, 0));
-    cudaStream_t cs = pool.back();
-    for (int br = 0; br < nbr; ++br) {
-      const int i = bb[br], gn = bb[br + 1] - bb[br];
-      int64_t npi = 0;
-      int rw = -1;
-      for (int j = bb[br]; j < bb[br + 1]; ++j) {
-        npi = std::max<int64_t>(npi, hp[j].n_s + hp[j].n_t);
-        if (overlap) rw = std::max(rw, ready_wave[j]);
-      }
-      cudaGraphConditionalHandle h;
-      GM_CUDA(cudaGraphConditionalHandleCreate(&h, gg.graph, 1, cudaGraphCondAssignDefault));
-      cudaGraphNodeParams cp = {};
-      cp.type = cudaGraphNodeTypeConditional;
-      cp.conditional.handle = h;
-      cp.conditional.type = cudaGraphCondTypeWhile;
-      cp.conditional.size = 1;
-      cudaGraphNode_t wnode, wait_node;
-      if (rw >= 0) {  // the branch starts when the waves covering its pairs' class blocks are done
-        GM_CUDA(cudaGraphAddEventWaitNode(&wait_node, gg.graph, nullptr, 0, ev_wave[rw]));
-        GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, &wait_node, 1, &cp));
-      } else {
-        GM_CUDA(cudaGraphAddNode(&wnode, gg.graph, nullptr, 0, &cp));
-      }
-      SolverArgs ag = a;
-      ag.pair_base = i;
-      const bool wsp = !rc && ws_solve_supported(Bw, npi);
-      const uint64_t b0 = g_launches.load();
-      cudaGraph_t cap;
-      GM_CUDA(cudaStreamBeginCaptureToGraph(cs, cp.conditional.phGraph_out[0], nullptr, nullptr, 0,
-                                            cudaStreamCaptureModeRelaxed));
-      if (wsp) {  // default kernels (wsolve.cu): selection -> gather -> local SMO -> f-update, unrolled:
-                  // the conditional node's re-launch (~10 us) is paid every `unroll` iterations
-        static const int unroll = getenv("GMPSVM_UNROLL") ? std::max(1, atoi(getenv("GMPSVM_UNROLL"))) : 4;
-        for (int u = 0; u < unroll; ++u) launch_ws_iteration(ag, gn, npi, h, u == unroll - 1, max_outer, cs, u > 0);
-      } else {
-        launch_select_ws(ag, gn, 0, -1, cs);
-        if (rc_tc)
-          launch_rows_compute_tc(ag, gn, d_rtiles.get() + rtile_off[br], rtile_off[br + 1] - rtile_off[br], Pl, cs);
-        else if (rc)
-          launch_rows_compute(ag, gn, npi, cs);
-        launch_gather_kws(ag, gn, -1, cs);
-        launch_local_smo(ag, gn, cs);
-        launch_f_update_loop(ag, gn, npi, h, max_outer, cs);
-      }
-      GM_CUDA(cudaStreamEndCapture(cs, &cap));
-      body_launches = (int64_t)(g_launches.load() - b0);
-      body_per_pair[i] = body_launches;
-      if (!wsp) {  // the stop test on the final alpha (the default path tests in every f-update)
-        GM_CUDA(cudaStreamBeginCaptureToGraph(cs, gg.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
-        launch_select_ws(ag, gn, 0, -1, cs);
-        GM_CUDA(cudaStreamEndCapture(cs, &cap));
-        ++final_selects;
-      }
-    }
-    n_branches = nbr;
-    g_launches.fetch_sub(g_launches.load() - l0);  // captured, not executed: counted after the run
     GM_CUDA(cudaEventRecord(ev_ready, st));
-    GM_CUDA(cudaStreamWaitEvent(pool[0], ev_ready, 0));
-    GM_CUDA(cudaGraphInstantiate(&gg.exec, gg.graph, 0));
+    cudaStream_t cs = pool[2];  // capture stream
+    static const int unroll = getenv("GMPSVM_UNROLL") ? std::max(1, atoi(getenv("GMPSVM_UNROLL"))) : 4;
+    auto build = [&](int br0, int br1, GraphGuard& g) {  // branches [br0, br1), instantiated
+      const uint64_t l0 = g_launches.load();
+      GM_CUDA(cudaGraphCreate(&g.graph, 0));
+      for (int br = br0; br < br1; ++br) {
+        const int i = bb[br], gn = bb[br + 1] - bb[br];
+        int64_t npi = 0;
+        for (int j = bb[br]; j < bb[br + 1]; ++j) npi = std::max<int64_t>(npi, hp[j].n_s + hp[j].n_t);
+        cudaGraphConditionalHandle h;
+        GM_CUDA(cudaGraphConditionalHandleCreate(&h, g.graph, 1, cudaGraphCondAssignDefault));
+        cudaGraphNodeParams cp = {};
+        cp.type = cudaGraphNodeTypeConditional;
+        cp.conditional.handle = h;
+        cp.conditional.type = cudaGraphCondTypeWhile;
+        cp.conditional.size = 1;
+        cudaGraphNode_t wnode;
+        GM_CUDA(cudaGraphAddNode(&wnode, g.graph, nullptr, 0, &cp));
+        SolverArgs ag = a;
+        ag.pair_base = i;
+        const bool wsp = !rc && ws_solve_supported(Bw, npi);
+        const uint64_t b0 = g_launches.load();
+        cudaGraph_t cap;
+        GM_CUDA(cudaStreamBeginCaptureToGraph(cs, cp.conditional.phGraph_out[0], nullptr, nullptr, 0,
+                                              cudaStreamCaptureModeRelaxed));
+        if (wsp) {  // default kernels (wsolve.cu): selection -> gather -> local SMO -> f-update, unrolled:
+                    // the conditional node's re-launch (~10 us) is paid every `unroll` iterations
+          for (int u = 0; u < unroll; ++u) launch_ws_iteration(ag, gn, npi, h, u == unroll - 1, max_outer, cs, u > 0);
+        } else {
+          launch_select_ws(ag, gn, 0, -1, cs);
+          if (rc_tc)
+            launch_rows_compute_tc(ag, gn, d_rtiles.get() + rtile_off[br], rtile_off[br + 1] - rtile_off[br], Pl, cs);
+          else if (rc)
+            launch_rows_compute(ag, gn, npi, cs);
+          launch_gather_kws(ag, gn, -1, cs);
+          launch_local_smo(ag, gn, cs);
+          launch_f_update_loop(ag, gn, npi, h, max_outer, cs);
+        }
+        GM_CUDA(cudaStreamEndCapture(cs, &cap));
+        body_launches = (int64_t)(g_launches.load() - b0);
+        body_per_pair[i] = body_launches;
+        if (!wsp) {  // the stop test on the final alpha (the default path tests in every f-update)
+          GM_CUDA(cudaStreamBeginCaptureToGraph(cs, g.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
+          launch_select_ws(ag, gn, 0, -1, cs);
+          GM_CUDA(cudaStreamEndCapture(cs, &cap));
+          ++final_selects;
+        }
+      }
+      g_launches.fetch_sub(g_launches.load() - l0);  // captured, not executed: counted after the run
+      GM_CUDA(cudaGraphInstantiate(&g.exec, g.graph, 0));
+    };
+    auto launch_after = [&](cudaGraphExec_t ex, cudaStream_t ls, cudaEvent_t extra, cudaEvent_t done, cudaEvent_t start) {
+      GM_CUDA(cudaStreamWaitEvent(ls, ev_ready, 0));
+      if (extra) GM_CUDA(cudaStreamWaitEvent(ls, extra, 0));
+      if (start) GM_CUDA(cudaEventRecord(start, ls));
+      GM_CUDA(cudaGraphLaunch(ex, ls));
+      cudaEvent_t ev = done ? done : evp.get();
+      GM_CUDA(cudaEventRecord(ev, ls));
+      GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
+    };
+    // the cached graphs fit this call if they were captured with the same kernel arguments,
+    // branch packing and per-branch launch shapes
+    std::vector<uint8_t> sig;
+    SolverWs* ws = lease.ws;
+    if (ws) {
+      auto put = [&](const void* p, size_t nb) {
+        sig.insert(sig.end(), static_cast<const uint8_t*>(p), static_cast<const uint8_t*>(p) + nb);
+      };
+      put(&a, sizeof a);
+      put(bb.data(), bb.size() * sizeof(int));
+      put(&nb_lead, sizeof nb_lead);
+      put(&max_outer, sizeof max_outer);
+      put(&unroll, sizeof unroll);
+      for (int br = 0; br < nbr; ++br) {
+        int64_t npi = 0;
+        for (int j = bb[br]; j < bb[br + 1]; ++j) npi = std::max<int64_t>(npi, hp[j].n_s + hp[j].n_t);
+        put(&npi, sizeof npi);
+      }
+    }
+    const bool reuse = ws && ws->exec[1] && ws->sig == sig;
+    cudaGraphExec_t ex_lead = nullptr, ex_rest = nullptr;
+    if (reuse) {
+      ex_lead = ws->exec[0];
+      ex_rest = ws->exec[1];
+      body_per_pair = ws->body_per_pair;
+      final_selects = ws->final_selects;
+    }
+    auto keep = [&]() {  // the freshly built graphs become the device's cached ones
+      if (!ws) return;
+      ws->park_graphs();
+      ws->graph[0] = gl.graph;
+      ws->exec[0] = gl.exec;
+      ws->graph[1] = gg.graph;
+      ws->exec[1] = gg.exec;
+      gl.graph = gg.graph = nullptr;
+      gl.exec = gg.exec = nullptr;
+      ws->sig = sig;
+      ws->body_per_pair = body_per_pair;
+      ws->final_selects = final_selects;
+    };
+    if (lead) {  // the lead graph first (small: built in well under wave 0's time), then the rest
+      if (!reuse) {
+        build(0, nb_lead, gl);
+        ex_lead = gl.exec;
+      }
+      launch_after(ex_lead, pool[1], ev_w0, kev_g.a, kev_s.a);
+      if (!reuse) {
+        build(nb_lead, nbr, gg);
+        ex_rest = gg.exec;
+        keep();
+      }
+      launch_after(ex_rest, pool[0], ev_k1, kev_g.b, kev_s.b);
+    } else {
+      if (!reuse) {
+        build(0, nbr, gg);
+        ex_rest = gg.exec;
+        keep();
+      }
+      launch_after(ex_rest, pool[0], nullptr, nullptr, nullptr);
+    }
     HT("graph_build");
-    GM_CUDA(cudaGraphLaunch(gg.exec, pool[0]));
-    destroy_parked_graphs();  // the previous calls' graphs, while this solver runs
+    n_branches = nbr;
+    // graphs no call will launch again (uncached calls, replaced cached ones): destroying one
+    // blocks the host until the device is idle, so it is done here, behind the running solver
+    destroy_parked_graphs();
+    HT("destroy");
   }
-  {
-    cudaEvent_t ev = evp.get();
-    GM_CUDA(cudaEventRecord(ev, pool[0]));
-    GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
-  }
-  if (overlap) GM_CUDA(cudaStreamWaitEvent(st, ev_k1, 0));  // every kernel-value wave (K is reused by the next call)
+  if (lead_dbg) GM_CUDA(cudaEventRecord(dbg0.b, st));
   tm.mark(PH_SOLVER);
   HT("solver_loop");
   bool cap_hit = false;
@@ -1501,14 +1774,32 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st, nullptr, 0.f, d_alpha.get(), tot, &alpha_off);
   tm.mark(PH_FIN);
   HT("devmodel");
+  if (lead_dbg) GM_CUDA(cudaEventRecord(dbg1.a, st));
   GM_CUDA(cudaStreamSynchronize(st));
+  if (lead_dbg) {
+    float sv = 0.f, en = 0.f, k0 = -1.f;
+    GM_CUDA(cudaEventElapsedTime(&sv, dbg0.a, dbg0.b));
+    GM_CUDA(cudaEventElapsedTime(&en, dbg0.a, dbg1.a));
+    if (lead) GM_CUDA(cudaEventElapsedTime(&k0, dbg0.a, ev_k0));
+    fprintf(stderr, "[gmpsvm timeline ms] from the call: first wave %.3f  solver done (st) %.3f  end %.3f\n", k0, sv, en);
+  }
 
   gmpsvm_train_stats& s = mdl->stats;
   s.t_stage_ms = tm.ms(PH_STAGE);
-  if (overlap) {  // span of the kernel-value waves (they share the GPU with the solver)
+  if (lead) {  // span of the kernel-value waves (they share the GPU with the lead pairs' solver)
     float x = 0.f;
     GM_CUDA(cudaEventElapsedTime(&x, ev_k0, ev_k1));
     s.t_kernel_ms = x;
+    if (lead_dbg) {
+      float w0 = 0.f, gl_end = 0.f, gr_end = 0.f, gl_st = 0.f, gr_st = 0.f;
+      GM_CUDA(cudaEventElapsedTime(&w0, ev_k0, ev_w0));
+      GM_CUDA(cudaEventElapsedTime(&gl_st, ev_k0, kev_s.a));
+      GM_CUDA(cudaEventElapsedTime(&gr_st, ev_k0, kev_s.b));
+      GM_CUDA(cudaEventElapsedTime(&gl_end, ev_k0, kev_g.a));
+      GM_CUDA(cudaEventElapsedTime(&gr_end, ev_k0, kev_g.b));
+      fprintf(stderr, "[gmpsvm lead ms] from the first wave: wave0 %.3f  waves %.3f  lead graph %.3f-%.3f  rest graph %.3f-%.3f (lead pairs %d, tiles %zu of %zu)\n",
+              w0, x, gl_st, gl_end, gr_st, gr_end, n_lead, n_wave0, n_tiles);
+    }
   } else {
     s.t_kernel_ms = tm.ms(PH_KERNEL);
   }

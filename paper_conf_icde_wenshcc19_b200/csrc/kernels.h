@@ -72,7 +72,7 @@ void launch_alpha_abs_sum(const double* alpha, const int64_t* aoff, const int64_
 std::vector<int2> krow_tc_tiles(int64_t n, bool two_cta);
 constexpr int kKrowTileRows = 128;  // krow_tc tile edge (rows = columns)
 // per-class means of the staged hi rows (class c = rows [coff[c], coff[c+1])): mu[k][d_pad]
-void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st);
+void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, float* m2, cudaStream_t st);
 // split with a given centre mu[d] and scale sc (prediction: the test rows take the SVs' mu, sc)
 void launch_split_hilo_mu(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, float sc, void* hi,
                           void* lo, float* norms, int64_t n_pad, int d_pad, cudaStream_t st);
@@ -101,7 +101,7 @@ void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* 
                    const KrowKernel* dk = nullptr);
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
-                    bool two_cta = false, const KrowKernel* dk = nullptr);
+                    bool two_cta = false, const KrowKernel* dk = nullptr, int reserve_sms = 0);
 void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
                       cudaStream_t st);
 bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel

@@ -1231,33 +1231,43 @@ float launch_split_hilo(const float* X, int64_t n, int d, const int64_t* perm, v
   return sc;
 }
 
-// Per-class means of the staged (centred, class-sorted) rows, from the hi part: used only to
-// order the pairs (engine.cu).
+// Per-class means and second moments (per feature) of the staged (centred, class-sorted) rows,
+// from the hi part: used only to order the pairs (engine.cu).
 template <typename T>
-__global__ void class_means_kernel(const T* hi, int d_pad, const int64_t* coff, float* mu) {
+__global__ void class_means_kernel(const T* hi, int d_pad, const int64_t* coff, float* mu, float* m2) {
   const int c = blockIdx.y, f = blockIdx.x * 32 + threadIdx.x;
   const int64_t r0 = coff[c], r1 = coff[c + 1];
-  float s = 0.f;
+  float s = 0.f, s2 = 0.f;
   if (f < d_pad)
-    for (int64_t r = r0 + threadIdx.y; r < r1; r += 8) s += (float)hi[r * d_pad + f];
-  __shared__ float red[8][33];
-  red[threadIdx.y][threadIdx.x] = s;
+    for (int64_t r = r0 + threadIdx.y; r < r1; r += 8) {
+      const float v = (float)hi[r * d_pad + f];
+      s += v;
+      s2 = fmaf(v, v, s2);
+    }
+  __shared__ float red[2][8][33];
+  red[0][threadIdx.y][threadIdx.x] = s;
+  red[1][threadIdx.y][threadIdx.x] = s2;
   __syncthreads();
   if (threadIdx.y == 0 && f < d_pad) {
-    float t = 0.f;
+    float t = 0.f, t2 = 0.f;
 #pragma unroll
-    for (int y = 0; y < 8; ++y) t += red[y][threadIdx.x];
-    mu[(int64_t)c * d_pad + f] = r1 > r0 ? t / (float)(r1 - r0) : 0.f;
+    for (int y = 0; y < 8; ++y) {
+      t += red[0][y][threadIdx.x];
+      t2 += red[1][y][threadIdx.x];
+    }
+    const float inv = r1 > r0 ? 1.f / (float)(r1 - r0) : 0.f;
+    mu[(int64_t)c * d_pad + f] = t * inv;
+    m2[(int64_t)c * d_pad + f] = t2 * inv;
   }
 }
 
-void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, cudaStream_t st) {
+void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, float* m2, cudaStream_t st) {
   if (krow_split_f16())
     GM_LAUNCH(class_means_kernel<__half>, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st,
-              static_cast<const __half*>(hi), d_pad, coff, mu);
+              static_cast<const __half*>(hi), d_pad, coff, mu, m2);
   else
     GM_LAUNCH(class_means_kernel<float>, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st,
-              static_cast<const float*>(hi), d_pad, coff, mu);
+              static_cast<const float*>(hi), d_pad, coff, mu, m2);
 }
 
 // Tiles (bi, bj) of 128 x 128 with at least one entry r <= c, in blocked order (16 x 16 tiles)
@@ -1317,7 +1327,7 @@ CUtensorMap make_kmap(float* K, int64_t n, int64_t ldk, bool swizzle) {
 
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
-                    bool two_cta, const KrowKernel* dk) {
+                    bool two_cta, const KrowKernel* dk, int reserve_sms) {
   const bool f16 = krow_split_f16();
   const CUtensorMap mhi = make_map(hi, n_pad, d_pad, f16), mlo = make_map(lo, n_pad, d_pad, f16);
   // TMA stores need a 16-byte aligned base and row stride; otherwise every tile takes the
@@ -1347,9 +1357,8 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
               n_tiles, norms, n, nk, scale, K, ldk, diag);
     return;
   }
-  // GMPSVM_KROW_RESERVE: SMs left free (the overlap mode's solver chains run beside the waves)
-  static const int reserve = getenv("GMPSVM_KROW_RESERVE") ? std::max(0, atoi(getenv("GMPSVM_KROW_RESERVE"))) : 0;
-  const int cap = std::max(1, sms - reserve);
+  // reserve_sms: SMs left free (the lead pairs' solver chains run beside the kernel values, engine.cu)
+  const int cap = std::max(1, sms - std::max(0, reserve_sms));
   const int grid = n_tiles < cap ? n_tiles : cap;
   KrowKernel kp{};
   if (dk) {
