@@ -46,7 +46,8 @@ constexpr int kMaxK = 64;          // label-rank shared memory bound
 constexpr int kMaxCoupleK = 40;    // coupling shared memory bound
 constexpr int kItemTiles = 4;      // SV tiles per dec_contract work item
 constexpr int64_t kPredictChunk = 32768;
-constexpr int kMaxStreams = 3;     // solver streams: graph launches (rest, lead) + graph capture
+constexpr int kMaxGroups = 4;      // solver graphs per call (lead mode: the lead pairs + up to 3 groups)
+constexpr int kMaxStreams = kMaxGroups + 1;  // solver streams: one graph launch per group + graph capture
 constexpr int kDefaultB = 192;     // working-set rows (tuned on MNIST-shaped data; the tile of K_ws,ws stays in shared memory for B <= 224)
 
 struct DeviceGuard {
@@ -103,6 +104,7 @@ const std::vector<cudaStream_t>& stream_pool(int dev) {
   auto& v = g_pools[dev];
   int least = 0, greatest = 0;
   if (v.size() < (size_t)kMaxStreams) GM_CUDA(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+  // pool[g]: the graph of pair group g (lead mode; else pool[0] alone), pool.back(): capture
   while ((int)v.size() < kMaxStreams) {
     cudaStream_t s;
     GM_CUDA(cudaStreamCreateWithPriority(&s, cudaStreamNonBlocking, greatest));
@@ -124,12 +126,12 @@ cudaStream_t krow_stream(int dev) {
   return s[dev];
 }
 
-// Timing-free events created on demand and destroyed with the pool.
+// Events created on demand and destroyed with the pool (timing-free unless asked).
 struct EventPool {
   std::vector<cudaEvent_t> evs;
-  cudaEvent_t get() {
+  cudaEvent_t get(bool timing = false) {
     cudaEvent_t e;
-    GM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    GM_CUDA(cudaEventCreateWithFlags(&e, timing ? cudaEventDefault : cudaEventDisableTiming));
     evs.push_back(e);
     return e;
   }
@@ -266,22 +268,22 @@ struct SolverWs {
   bool busy = false;
   cudaEvent_t done = nullptr;  // end of the last call's use of the arena
   std::vector<uint8_t> sig;
-  cudaGraph_t graph[2] = {nullptr, nullptr};
-  cudaGraphExec_t exec[2] = {nullptr, nullptr};
+  std::vector<cudaGraph_t> graph;  // one per pair group
+  std::vector<cudaGraphExec_t> exec;
   std::vector<int64_t> body_per_pair;
   int final_selects = 0;
   // kernel-value tile list of the last call (FULL_K on tcgen05): key, device copy, wave split
   std::vector<int64_t> tkey;
   int2* tiles = nullptr;
-  size_t n_tiles = 0, n_wave0 = 0;
+  size_t n_tiles = 0;
+  std::vector<size_t> wave_off;
   double kv_subset = -1;
   void park_graphs() {  // destroyed later by destroy_parked_graphs (it blocks until the device idles)
     std::lock_guard<std::mutex> lk(g_parked_mu);
-    for (int i = 0; i < 2; ++i) {
+    for (size_t i = 0; i < exec.size(); ++i)
       if (exec[i] || graph[i]) g_parked.emplace_back(exec[i], graph[i]);
-      exec[i] = nullptr;
-      graph[i] = nullptr;
-    }
+    exec.clear();
+    graph.clear();
     sig.clear();
   }
 };
@@ -1164,43 +1166,68 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   DevBuf<int2> d_tiles_own;
   const int2* d_tiles = nullptr;
   size_t n_tiles = 0;
-  // Lead mode (default on the tensor-core FULL_K path with the device-driven solver): the first
-  // pairs -- the predicted hardest, above -- form a graph of their own (one branch each) that starts
-  // as soon as the kernel values of their class blocks (s,s), (s,t), (t,t) are done (wave 0, on
-  // every SM); the rest of the kernel matrix (wave 1) is then computed on all but `reserve` SMs,
-  // where the lead chains run, and the other pairs -- a second graph -- wait for all of it.  The
-  // solver's critical path, the hardest pair's chain of outer iterations, so overlaps the
-  // kernel-value contraction instead of following it.  GMPSVM_LEAD=<pairs> (0: off),
-  // GMPSVM_LEAD_RESERVE=<SMs>.
+  // Lead mode (default on the tensor-core FULL_K path with the device-driven solver): the pairs
+  // are split into groups in their order (the predicted hardest first, above) -- the lead pairs,
+  // one graph branch each, then GMPSVM_GROUPS groups of the rest -- and each group is a graph of
+  // its own that starts as soon as the kernel values of its pairs' class blocks (s,s), (s,t), (t,t)
+  // are done.  The kernel matrix is computed in that order, one wave per group: wave 0 (the lead
+  // blocks) on every SM, the later waves on all but `reserve` SMs, where the started groups' solver
+  // chains run.  The solver's critical path -- the hardest pairs' chains of outer iterations --
+  // so overlaps the kernel-value contraction instead of following it.  GMPSVM_LEAD=<pairs>
+  // (0: off), GMPSVM_LEAD_RESERVE=<SMs>, GMPSVM_GROUPS=<groups of the rest> (measured on
+  // MNIST-shaped data: 1 group best -- more groups start more chains beside the lead chain and
+  // slow it down: 33.3 / 34.4 / 34.8 ms per bench step for 1 / 2 / 3 groups; 1 / 2 / 4 lead pairs
+  // and 4 / 8 / 12 / 16 reserved SMs within 0.3 ms of each other).
   const bool fk_tc = full_k && use_tc;  // the FULL_K contraction on tcgen05
   static const int lead_env = getenv("GMPSVM_LEAD") ? std::max(0, atoi(getenv("GMPSVM_LEAD"))) : 1;
   static const int reserve_env = getenv("GMPSVM_LEAD_RESERVE") ? std::max(0, atoi(getenv("GMPSVM_LEAD_RESERVE"))) : 8;
+  static const int groups_env =
+      std::max(1, std::min(kMaxGroups - 1, getenv("GMPSVM_GROUPS") ? atoi(getenv("GMPSVM_GROUPS")) : 1));
   // Solver graph branches (below): the runtime runs at most CUDA_DEVICE_MAX_CONNECTIONS branches
   // concurrently -- a branch beyond that shares a hardware queue with another and waits for it --
   // so the pairs are packed into that many branches: the first pairs alone, the last two (or more)
-  // to a branch in lockstep.  Lead mode keeps two queues more free (the lead graph's and the
-  // kernel-value stream's): measured, a rest branch otherwise queued behind the lead chain.
+  // to a branch in lockstep.  Lead mode keeps a queue free per graph launch stream and one for the
+  // kernel-value stream: measured, a branch otherwise queued behind the lead chain.
   const int conn = connections_in_effect();
-  const int n_lead = (fk_tc && lead_env > 0 && Pl > lead_env && conn - lead_env - 2 >= 1 && ws_solve_supported(B, np_max))
-                         ? lead_env
-                         : 0;
-  const bool lead = n_lead > 0;
-  const int nb_lead = n_lead;  // lead graph: branches [0, nb_lead), one pair each
-  const int nb_rest = std::min(Pl - n_lead, lead ? conn - n_lead - 2 : conn);
-  const int nbr = nb_lead + nb_rest;
-  std::vector<int> bb(nbr + 1, 0);
-  {
-    for (int b = 0; b < nb_lead; ++b) bb[b + 1] = b + 1;
-    const int m = (Pl - n_lead) / nb_rest, r = (Pl - n_lead) % nb_rest;  // the last r branches take m + 1 pairs
-    for (int b = 0; b < nb_rest; ++b) bb[nb_lead + b + 1] = bb[nb_lead + b] + m + (b >= nb_rest - r ? 1 : 0);
+  int n_lead = (fk_tc && lead_env > 0 && Pl > lead_env && ws_solve_supported(B, np_max)) ? lead_env : 0;
+  int ng = 1;  // pair groups (graphs)
+  if (n_lead) {
+    ng = 1 + std::min(groups_env, Pl - n_lead);
+    if (conn - n_lead - ng - 1 < ng - 1) n_lead = 0, ng = 1;  // not enough queues
   }
+  const bool lead = n_lead > 0;
+  std::vector<int> gpos(ng + 1, 0), gbr(ng + 1, 0);  // per group: pair positions, branches
+  std::vector<int> bb(1, 0);                          // per branch: pair positions [bb[b], bb[b+1])
+  auto pack = [&](int p0, int cnt, int nb) {          // cnt pairs from position p0 into nb branches
+    const int m = cnt / nb, r = cnt % nb;             // the last r branches take m + 1 pairs
+    for (int b = 0; b < nb; ++b) bb.push_back(bb.back() + m + (b >= nb - r ? 1 : 0));
+    (void)p0;
+  };
+  if (!lead) {
+    gpos[1] = Pl;
+    pack(0, Pl, std::min(Pl, conn));
+    gbr[1] = (int)bb.size() - 1;
+  } else {
+    gpos[1] = n_lead;
+    pack(0, n_lead, n_lead);
+    gbr[1] = n_lead;
+    const int rest = Pl - n_lead, ngr = ng - 1, budget = conn - n_lead - ng - 1;
+    for (int g = 1; g < ng; ++g) {
+      const int cnt = rest / ngr + (g - 1 < rest % ngr ? 1 : 0);
+      gpos[g + 1] = gpos[g] + cnt;
+      const int nb = std::max(1, std::min(cnt, (int)((double)budget * cnt / rest)));
+      pack(gpos[g], cnt, nb);
+      gbr[g + 1] = (int)bb.size() - 1;
+    }
+  }
+  const int nbr = (int)bb.size() - 1;
   cudaStream_t kst = krow_stream(opt.device);
   TimedEvents kev;
   cudaEvent_t ev_k0 = kev.a, ev_k1 = kev.b;
   EventPool evk;
-  TimedEvents kev_w, kev_g, kev_s;  // lead mode: wave 0 done (a); lead / rest graph start (kev_s), done (kev_g)
-  cudaEvent_t ev_w0 = nullptr;
-  size_t n_wave0 = 0;
+  static const bool lead_dbg_t = getenv("GMPSVM_LEAD_DEBUG") != nullptr;
+  std::vector<cudaEvent_t> ev_wave(ng, nullptr), ev_gst(ng, nullptr), ev_gend(ng, nullptr);  // per group
+  std::vector<size_t> wave_off(ng + 1, 0);  // lead mode: tile range of wave g
   const bool two_cta = fk_tc && !lead && ktype == 0 && krow_tc_2cta();  // lead waves: single-CTA tiles
   double kv_subset = -1;  // >= 0: kernel values computed for a pair subset (tiles skipped)
   if (fk_tc) {
@@ -1232,17 +1259,21 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     };
     const bool subset = !two_cta && Pl < P;
     const std::vector<uint8_t> need = subset ? blocks_of(0, Pl) : std::vector<uint8_t>();
-    const std::vector<uint8_t> lb = lead ? blocks_of(0, n_lead) : std::vector<uint8_t>();
+    std::vector<std::vector<uint8_t>> gmask;  // lead mode: class blocks per group
+    if (lead)
+      for (int g = 0; g < ng; ++g) gmask.push_back(blocks_of(gpos[g], gpos[g + 1]));
     std::vector<int64_t> tkey = {n, two_cta ? 1 : 0, k};  // what the tile list depends on
     tkey.insert(tkey.end(), coff.begin(), coff.end());
     for (const uint8_t v : need) tkey.push_back(v);
-    tkey.push_back(-1);
-    for (const uint8_t v : lb) tkey.push_back(v);
+    for (const auto& gm : gmask) {
+      tkey.push_back(-1);
+      for (const uint8_t v : gm) tkey.push_back(v);
+    }
     SolverWs* ws = lease.ws;
     if (ws && ws->tiles && ws->tkey == tkey) {  // the last call's list
       d_tiles = ws->tiles;
       n_tiles = ws->n_tiles;
-      n_wave0 = ws->n_wave0;
+      wave_off = ws->wave_off;
       kv_subset = ws->kv_subset;
     } else {
       std::vector<int2> tiles = krow_tc_tiles(n, two_cta);
@@ -1260,12 +1291,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
           kv_subset += tl.x == tl.y ? (double)nr * (double)(nr + 1) / 2.0 : (double)nr * (double)nc;
         }
       }
-      if (lead) {  // wave 0: the tiles of the lead pairs' class blocks (blocked order kept), then the rest
-        std::vector<int2> w0, w1;
-        for (const int2 tl : tiles) (touches(tl, lb) ? w0 : w1).push_back(tl);
-        n_wave0 = w0.size();
-        w0.insert(w0.end(), w1.begin(), w1.end());
-        tiles.swap(w0);
+      if (lead) {  // wave g: the tiles first needed by group g (blocked order kept within a wave)
+        std::vector<std::vector<int2>> w(ng);
+        for (const int2 tl : tiles) {
+          int g = 0;
+          while (g < ng - 1 && !touches(tl, gmask[g])) ++g;
+          w[g].push_back(tl);
+        }
+        tiles.clear();
+        for (int g = 0; g < ng; ++g) {
+          tiles.insert(tiles.end(), w[g].begin(), w[g].end());
+          wave_off[g + 1] = tiles.size();
+        }
       }
       n_tiles = tiles.size();
       int2* dt = nullptr;
@@ -1277,7 +1314,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         dt = ws->tiles;
         ws->tkey = tkey;
         ws->n_tiles = n_tiles;
-        ws->n_wave0 = n_wave0;
+        ws->wave_off = wave_off;
         ws->kv_subset = kv_subset;
       } else {
         new (&d_tiles_own) DevBuf<int2>(n_tiles, st);
@@ -1298,13 +1335,14 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     GM_CUDA(cudaEventRecord(ev_staged, st));
     GM_CUDA(cudaStreamWaitEvent(kst, ev_staged, 0));
     GM_CUDA(cudaEventRecord(ev_k0, kst));
-    launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles, (int)n_wave0, norms.get(), n, gamma, ksc, K.get(), ldk, kst,
-                   false, kkp);
-    ev_w0 = kev_w.a;
-    GM_CUDA(cudaEventRecord(ev_w0, kst));
-    if (n_tiles > n_wave0)
-      launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles + n_wave0, (int)(n_tiles - n_wave0), norms.get(), n, gamma,
-                     ksc, K.get(), ldk, kst, false, kkp, reserve_env);
+    for (int g = 0; g < ng; ++g) {
+      const size_t cnt = wave_off[g + 1] - wave_off[g];
+      if (cnt)
+        launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles + wave_off[g], (int)cnt, norms.get(), n, gamma, ksc,
+                       K.get(), ldk, kst, false, kkp, g == 0 ? 0 : reserve_env);
+      ev_wave[g] = evk.get(lead_dbg_t);
+      GM_CUDA(cudaEventRecord(ev_wave[g], kst));
+    }
     GM_CUDA(cudaEventRecord(ev_k1, kst));
   } else if (full_k && !use_tc) {
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
@@ -1438,7 +1476,6 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   tm.mark(PH_SOLVER);
   HT("init");
   int64_t rc_launches = 0;  // ROW_CACHE row-contraction launches
-  GraphGuard gg, gl;  // the solver graph (lead mode: the other branches) and the lead graph
   DevBuf<int4> d_rtiles;  // ROW_CACHE tcgen05 row tiles of every branch (outlives the graph run)
   int64_t body_launches = 0;
   std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
@@ -1462,7 +1499,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     if (!rtiles.empty())
       GM_CUDA(cudaMemcpyAsync(d_rtiles.get(), rtiles.data(), rtiles.size() * sizeof(int4), cudaMemcpyHostToDevice, st));
     GM_CUDA(cudaEventRecord(ev_ready, st));
-    cudaStream_t cs = pool[2];  // capture stream
+    cudaStream_t cs = pool.back();  // capture stream
     static const int unroll = getenv("GMPSVM_UNROLL") ? std::max(1, atoi(getenv("GMPSVM_UNROLL"))) : 4;
     auto build = [&](int br0, int br1, GraphGuard& g) {  // branches [br0, br1), instantiated
       const uint64_t l0 = g_launches.load();
@@ -1532,7 +1569,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
       };
       put(&a, sizeof a);
       put(bb.data(), bb.size() * sizeof(int));
-      put(&nb_lead, sizeof nb_lead);
+      put(gbr.data(), gbr.size() * sizeof(int));
       put(&max_outer, sizeof max_outer);
       put(&unroll, sizeof unroll);
       for (int br = 0; br < nbr; ++br) {
@@ -1541,46 +1578,38 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         put(&npi, sizeof npi);
       }
     }
-    const bool reuse = ws && ws->exec[1] && ws->sig == sig;
-    cudaGraphExec_t ex_lead = nullptr, ex_rest = nullptr;
+    const bool reuse = ws && (int)ws->exec.size() == ng && ws->sig == sig;
+    std::vector<GraphGuard> gg(ng);  // this call's graphs (uncached, or to be kept)
+    std::vector<cudaGraphExec_t> ex(ng, nullptr);
     if (reuse) {
-      ex_lead = ws->exec[0];
-      ex_rest = ws->exec[1];
+      ex = ws->exec;
       body_per_pair = ws->body_per_pair;
       final_selects = ws->final_selects;
     }
-    auto keep = [&]() {  // the freshly built graphs become the device's cached ones
-      if (!ws) return;
+    // group g's graph on pool[g]; lead mode: after its wave (the lead graph is small and built in
+    // well under wave 0's time; the others are built while their waves run)
+    for (int g = 0; g < ng; ++g) {
+      if (!reuse) {
+        build(gbr[g], gbr[g + 1], gg[g]);
+        ex[g] = gg[g].exec;
+      }
+      if (lead_dbg_t) {
+        ev_gst[g] = evk.get(true);
+        ev_gend[g] = evk.get(true);
+      }
+      launch_after(ex[g], pool[g], lead ? ev_wave[g] : nullptr, ev_gend[g], ev_gst[g]);
+    }
+    if (ws && !reuse) {  // the freshly built graphs become the device's cached ones
       ws->park_graphs();
-      ws->graph[0] = gl.graph;
-      ws->exec[0] = gl.exec;
-      ws->graph[1] = gg.graph;
-      ws->exec[1] = gg.exec;
-      gl.graph = gg.graph = nullptr;
-      gl.exec = gg.exec = nullptr;
+      for (int g = 0; g < ng; ++g) {
+        ws->graph.push_back(gg[g].graph);
+        ws->exec.push_back(gg[g].exec);
+        gg[g].graph = nullptr;
+        gg[g].exec = nullptr;
+      }
       ws->sig = sig;
       ws->body_per_pair = body_per_pair;
       ws->final_selects = final_selects;
-    };
-    if (lead) {  // the lead graph first (small: built in well under wave 0's time), then the rest
-      if (!reuse) {
-        build(0, nb_lead, gl);
-        ex_lead = gl.exec;
-      }
-      launch_after(ex_lead, pool[1], ev_w0, kev_g.a, kev_s.a);
-      if (!reuse) {
-        build(nb_lead, nbr, gg);
-        ex_rest = gg.exec;
-        keep();
-      }
-      launch_after(ex_rest, pool[0], ev_k1, kev_g.b, kev_s.b);
-    } else {
-      if (!reuse) {
-        build(0, nbr, gg);
-        ex_rest = gg.exec;
-        keep();
-      }
-      launch_after(ex_rest, pool[0], nullptr, nullptr, nullptr);
     }
     HT("graph_build");
     n_branches = nbr;
@@ -1791,14 +1820,17 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     GM_CUDA(cudaEventElapsedTime(&x, ev_k0, ev_k1));
     s.t_kernel_ms = x;
     if (lead_dbg) {
-      float w0 = 0.f, gl_end = 0.f, gr_end = 0.f, gl_st = 0.f, gr_st = 0.f;
-      GM_CUDA(cudaEventElapsedTime(&w0, ev_k0, ev_w0));
-      GM_CUDA(cudaEventElapsedTime(&gl_st, ev_k0, kev_s.a));
-      GM_CUDA(cudaEventElapsedTime(&gr_st, ev_k0, kev_s.b));
-      GM_CUDA(cudaEventElapsedTime(&gl_end, ev_k0, kev_g.a));
-      GM_CUDA(cudaEventElapsedTime(&gr_end, ev_k0, kev_g.b));
-      fprintf(stderr, "[gmpsvm lead ms] from the first wave: wave0 %.3f  waves %.3f  lead graph %.3f-%.3f  rest graph %.3f-%.3f (lead pairs %d, tiles %zu of %zu)\n",
-              w0, x, gl_st, gl_end, gr_st, gr_end, n_lead, n_wave0, n_tiles);
+      std::string line;
+      for (int g = 0; g < ng; ++g) {
+        float w = 0.f, g0 = 0.f, g1 = 0.f;
+        GM_CUDA(cudaEventElapsedTime(&w, ev_k0, ev_wave[g]));
+        GM_CUDA(cudaEventElapsedTime(&g0, ev_k0, ev_gst[g]));
+        GM_CUDA(cudaEventElapsedTime(&g1, ev_k0, ev_gend[g]));
+        char buf[160];
+        snprintf(buf, sizeof buf, "  g%d[%d pairs] wave %.3f graph %.3f-%.3f", g, gpos[g + 1] - gpos[g], w, g0, g1);
+        line += buf;
+      }
+      fprintf(stderr, "[gmpsvm lead ms] from the first wave:%s (tiles %zu)\n", line.c_str(), n_tiles);
     }
   } else {
     s.t_kernel_ms = tm.ms(PH_KERNEL);
