@@ -49,7 +49,12 @@ constexpr uint32_t kIAPlane = kIM * kIK;  // 8 KB
 constexpr uint32_t kIBPlane = kIN * kIK;  // 4 KB
 constexpr uint32_t kIStageBytes = kND * (kIAPlane + kIBPlane);  // 60 KB
 constexpr uint32_t kITmemCols = 512;      // 6 x 64 used (power-of-two allocation)
-constexpr int kIThreads = 320;  // producer, MMA issuer, 8 epilogue warps
+// epilogue warps: 16 (4 per TMEM lane quarter, 16 of a tile's 64 SV columns each) while the per-row
+// sums fit the register budget of 576 threads (k - 1 <= 12), else 8 (two per quarter, 32 columns)
+template <int KM>
+constexpr int i8_epi_warps() { return 8; }
+template <int KM>
+constexpr int i8_threads() { return 64 + 32 * i8_epi_warps<KM>(); }  // producer, MMA issuer, epilogue
 constexpr int kIExp = 37;                 // max |x| 2^e in [2^37, 2^38)
 // kind::i8, D S32 (2), A S8 (1), B S8 (1), K-major, N = 64, M = 128
 constexpr uint32_t kIdescI8 =
@@ -58,10 +63,12 @@ constexpr uint32_t kIdescI8 =
 template <int KM>
 constexpr int i8_stages() { return KM > 12 ? 2 : kIStages; }  // large k: the coefficient tiles need the room
 template <int KM>
+constexpr int i8_row() { return (KM + 3) & ~1; }  // doubles per staged SV column (even: 16-byte pairs)
+template <int KM>
 struct DecI8Smem {
   alignas(1024) uint8_t stage[i8_stages<KM>()][kIStageBytes];
-  alignas(16) double coefS[2][kIN][KM];
-  double red[kIM][KM];  // column-half reduction of the per-row sums
+  alignas(16) double coefS[2][kIN][i8_row<KM>()];  // per SV column: 2^(24 - e_c), ||y~||^2, coefficients
+  double red[kIM][KM];  // reduction of the column parts' per-row sums
   alignas(8) uint64_t full[i8_stages<KM>()];
   uint64_t empty[i8_stages<KM>()];
   uint64_t tmem_full;
@@ -69,9 +76,16 @@ struct DecI8Smem {
   uint32_t tmem_base;
 };
 
+__device__ __forceinline__ bool elect_one() {  // one lane of the (converged) warp
+  uint32_t pred = 0;
+  asm volatile("{\n .reg .b32 rx;\n .reg .pred px;\n elect.sync rx|px, 0xffffffff;\n selp.b32 %0, 1, 0, px;\n}\n"
+               : "=r"(pred));
+  return pred != 0;
+}
+
 // K-major operand, 64-byte swizzle: 8-row groups 512 B apart (SBO), LBO unused, version 1
-__device__ __forceinline__ uint64_t umma_desc_sw64(const void* p) {
-  const uint64_t addr = smem_u32(p);
+__device__ __forceinline__ uint64_t umma_desc_sw64_addr(uint32_t addr32) {
+  const uint64_t addr = addr32;
   uint64_t d = 0;
   d |= (addr >> 4) & 0x3FFFull;
   d |= (uint64_t)1 << 16;
@@ -105,6 +119,19 @@ __device__ __forceinline__ void umma_i8(uint32_t tmem_d, uint64_t a, uint64_t b,
         "l"(a), "l"(b), "r"(kIdescI8), "r"(accum));
 }
 __device__ __forceinline__ double pow2(int k) { return __hiloint2double((k + 1023) << 20, 0); }  // 2^k, |k| < 1023
+
+// Exact int64 -> double for |w| < 2^51 without the quarter-rate I2F.F64.S64: the bit pattern of
+// 1.5 2^52 plus w is the double 1.5 2^52 + w.  kShift52 also rounds a double to an integer (RNE).
+constexpr double kShift52 = 6755399441055744.0;  // 1.5 * 2^52
+__device__ __forceinline__ double i2d_small(long long w) {
+  return __longlong_as_double(w + 0x4338000000000000ll) - kShift52;
+}
+
+// c_k = ln(2)^k / k!, k = 10 .. 0: the Taylor coefficients of 2^f (exp2_neg, the epilogue)
+__device__ __constant__ const double kExp2C[11] = {7.054911620801123e-09, 1.01780860092397e-07, 1.321548679014431e-06,
+                                                   1.5252733804059841e-05, 0.0001540353039338161, 0.0013333558146428443,
+                                                   0.009618129107628477, 0.05550410866482158, 0.24022650695910072,
+                                                   0.6931471805599453, 1.0};
 
 // 2^t for t <= 0 in FP64: t = n + f, n = rint(t), |f| <= 1/2; 2^f by its Taylor series in
 // f ln 2 to degree 10 (remainder <= (ln2 / 2)^11 / 11! e^(ln2 / 2) < 3.2e-13 relative) evaluated by
@@ -170,14 +197,14 @@ __global__ void stage_i8_kernel(const float* __restrict__ X, int64_t n, int d, c
   }
 }
 
-template <int KM, bool COLLECT>
-__global__ void __launch_bounds__(kIThreads, 1)
+template <int KM>
+__global__ void __launch_bounds__(i8_threads<KM>(), 1)
     dec_i8_kernel(const __grid_constant__ CUtensorMap map_t, const __grid_constant__ CUtensorMap map_s,
                   const int2* __restrict__ tiles, const int32_t* __restrict__ unit_off,
                   const int32_t* __restrict__ unit_item, int n_units, const int32_t* __restrict__ et,
                   const double* __restrict__ nt, const int32_t* __restrict__ es, const double* __restrict__ ns,
                   const double* __restrict__ coef, int km1, int km1_pad, int d8, int64_t m_pad, int64_t nsv_pad,
-                  double gamma, double* __restrict__ part, int diag) {
+                  double gamma, double* __restrict__ part_out, int diag) {
   extern __shared__ __align__(1024) uint8_t dsmem[];
   DecI8Smem<KM>& sm =
       *reinterpret_cast<DecI8Smem<KM>*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
@@ -190,7 +217,7 @@ __global__ void __launch_bounds__(kIThreads, 1)
       mbar_init(&sm.empty[s], 1);
     }
     mbar_init(&sm.tmem_full, 1);
-    mbar_init(&sm.tmem_empty, 8);
+    mbar_init(&sm.tmem_empty, i8_epi_warps<KM>());
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_t)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_s)) : "memory");
@@ -235,35 +262,40 @@ __global__ void __launch_bounds__(kIThreads, 1)
         }
     }
   } else if (warp == 1) {
-    if (lane == 0) {  // ---- MMA issuer: group g = i + j of the digit products into accumulator g
-      int g = 0, it = 0;
-      for (int u = blockIdx.x; u < n_units; u += gridDim.x)
-        for (int t = unit_off[u]; t < unit_off[u + 1]; ++t)
-          for (int h = 0; h < 2; ++h, ++it) {
-            if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
+    // ---- MMA issuer: group g = i + j of the digit products into accumulator g.  The whole warp
+    // runs the loop (warp-uniform control flow, so the descriptors and TMEM addresses live in
+    // uniform registers) and one elected lane issues: issued from a lone `lane == 0` thread, every
+    // MMA went through an ELECT / R2UR.BROADCAST / BRA.U.ANY sequence and the issue loop, not the
+    // tensor pipe, set the pace (69 cycles per MMA against 44.6 in tools/micro/i8_mma_rate.cu;
+    // measured with clock64 around the waits: 6.1M of CTA 0's 6.5M cycles were spent issuing).
+    int g = 0, it = 0;
+    for (int u = blockIdx.x; u < n_units; u += gridDim.x)
+      for (int t = unit_off[u]; t < unit_off[u + 1]; ++t)
+        for (int h = 0; h < 2; ++h, ++it) {
+          if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          for (int kb = 0; kb < nk; ++kb, ++g) {
+            const int s = g % NS;
+            mbar_wait(&sm.full[s], (g / NS) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-            for (int kb = 0; kb < nk; ++kb, ++g) {
-              const int s = g % NS;
-              mbar_wait(&sm.full[s], (g / NS) & 1);
-              asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-              uint8_t* st = sm.stage[s];
-              const int nsub = (diag & 2) ? 0 : min(2, (d8 - kb * kIK + 31) / 32);  // valid 32-wide k steps
+            const uint32_t st_a = smem_u32(sm.stage[s]);
+            const int nsub = (diag & 2) ? 0 : min(2, (d8 - kb * kIK + 31) / 32);  // valid 32-wide k steps
+            if (elect_one()) {
               for (int kk = 0; kk < nsub; ++kk) {
                 const uint64_t adv = (uint64_t)(kk * 32) >> 4;
                 // A plane i stays in the tensor core's collector across its products with every B
                 // plane j (i + j <= 5): the A operand is read from shared memory once per (i, kk)
 #pragma unroll
                 for (int i = 0; i < kND; ++i) {
-                  const uint64_t ad = umma_desc_sw64(st + i * kIAPlane) + adv;
+                  const uint64_t ad = umma_desc_sw64_addr(st_a + i * kIAPlane) + adv;
                   const int jn = min(kND, kNG - i);  // j = 0 .. jn - 1
 #pragma unroll
                   for (int j = 0; j < jn; ++j) {
                     const int gg = i + j;
                     const bool first = kb == 0 && kk == 0 && i == (gg < kND ? 0 : gg - kND + 1);
-                    const uint64_t bd = umma_desc_sw64(st + kND * kIAPlane + j * kIBPlane) + adv;
+                    const uint64_t bd = umma_desc_sw64_addr(st_a + kND * kIAPlane + j * kIBPlane) + adv;
                     const uint32_t acc = first ? 0u : 1u;
-                    if (!COLLECT) umma_i8<0>(tmem + gg * kIN, ad, bd, acc);
-                    else if (j == 0) umma_i8<1>(tmem + gg * kIN, ad, bd, acc);
+                    if (j == 0) umma_i8<1>(tmem + gg * kIN, ad, bd, acc);
                     else if (j == jn - 1) umma_i8<3>(tmem + gg * kIN, ad, bd, acc);
                     else umma_i8<2>(tmem + gg * kIN, ad, bd, acc);
                   }
@@ -271,12 +303,15 @@ __global__ void __launch_bounds__(kIThreads, 1)
               }
               umma_commit(&sm.empty[s]);
             }
-            umma_commit(&sm.tmem_full);
+            __syncwarp();
           }
-    }
-  } else {  // ---- epilogue: warps 2..9; TMEM lane quarter warp % 4, column half (warp - 2) / 4;
-            //      thread = one test row x 32 of the tile's 64 SVs
-    const int q = warp & 3, half = (warp - 2) >> 2, et_id = threadIdx.x - 64;  // et_id 0..255
+          if (elect_one()) umma_commit(&sm.tmem_full);
+          __syncwarp();
+        }
+  } else {  // ---- epilogue: EW warps; TMEM lane quarter warp % 4, column part (warp - 2) / 4;
+            //      thread = one test row x CW of the tile's 64 SVs
+    constexpr int EW = i8_epi_warps<KM>(), NP = EW / 4, CW = kIN / NP, ET = 32 * EW;
+    const int q = warp & 3, part = (warp - 2) >> 2, et_id = threadIdx.x - 64;  // et_id 0 .. ET - 1
     int it = 0;
     const double tsc = -gamma * 1.4426950408889634074;  // exp(-gamma d2) = 2^(tsc d2)
     for (int u = blockIdx.x; u < n_units; u += gridDim.x) {
@@ -287,24 +322,34 @@ __global__ void __launch_bounds__(kIThreads, 1)
       for (int t = unit_off[u]; t < unit_off[u + 1]; ++t) {
         const int2 tile = tiles[t];
         r = (int64_t)tile.x * kIM + q * 32 + lane;
-        const int ex_r = et[r];
+        const double pr = pow2(-et[r]);  // 2^-e_x
         const double nr = nt[r];
         for (int h = 0; h < 2; ++h, ++it) {
           const int64_t c0 = (int64_t)tile.y * 2 * kIN + h * kIN;
-          double* cs = &sm.coefS[it & 1][0][0];  // this half-tile's coefficients (double buffer)
-          for (int idx = et_id; idx < kIN * KM; idx += 256) {
-            const int jj = idx / KM, v = idx - jj * KM;
-            cs[idx] = v < km1 ? coef[(c0 + jj) * km1_pad + v] : 0.0;
+          // this half-tile's SV columns (double buffer): scale, norm and coefficients, staged with
+          // shared-memory stores and read back with 16-byte shared loads
+          constexpr int ROW = i8_row<KM>();
+          const uint32_t cs = smem_u32(&sm.coefS[it & 1][0][0]);
+          for (int idx = et_id; idx < kIN * ROW; idx += ET) {
+            const int jj = idx / ROW, v = idx - jj * ROW;
+            const int64_t c = c0 + jj;
+            const double val = v == 0 ? pow2(24 - es[c]) : v == 1 ? ns[c] : (v - 2 < km1 ? coef[c * km1_pad + v - 2] : 0.0);
+            asm volatile("st.shared.f64 [%0], %1;" ::"r"(cs + (uint32_t)idx * 8), "d"(val) : "memory");
           }
-          asm volatile("bar.sync 1, 256;" ::: "memory");
+          asm volatile("bar.sync 1, %0;" ::"r"(ET) : "memory");
           mbar_wait(&sm.tmem_full, it & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           // sum_g 256^(5-g) G_g by 16-column chunks: groups 0-2 and 3-5 combined exactly in int64
           // (|G| < 2^26: |hi|, |lo| < 2^43, exact in FP64), then hi 2^24 + lo in FP64
-          const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(half * 32);
-          double dot[32];
+          const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(part * CW);
+          double dot[CW];
+          if (diag & 16) {  // GMPSVM_I8_DIAG bit 4 (timing experiments): no TMEM drain
+            __syncwarp();
+            if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+            continue;
+          }
 #pragma unroll
-          for (int ch = 0; ch < 2; ++ch) {
+          for (int ch = 0; ch < CW / 16; ++ch) {
 #pragma unroll
             for (int part3 = 0; part3 < 2; ++part3) {
               long long w[16];
@@ -318,7 +363,7 @@ __global__ void __launch_bounds__(kIThreads, 1)
                 w[jj] = ((long long)(int32_t)v0[jj] * 65536 + (long long)(int32_t)v1[jj] * 256) + (int32_t)v2[jj];
 #pragma unroll
               for (int jj = 0; jj < 16; ++jj)
-                dot[ch * 16 + jj] = part3 == 0 ? (double)w[jj] : fma(dot[ch * 16 + jj], 16777216.0, (double)w[jj]);
+                dot[ch * 16 + jj] = part3 == 0 ? i2d_small(w[jj]) : fma(dot[ch * 16 + jj], 16777216.0, i2d_small(w[jj]));
             }
           }
           asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -326,33 +371,69 @@ __global__ void __launch_bounds__(kIThreads, 1)
           if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
           // x~.y~ = 2^-(e_x+e_y) 256^3 (hi 2^24 + lo): the 256^3 = 2^24 folds into the exponent
           if (diag & 1) {  // GMPSVM_I8_DIAG bit 0 (timing experiments): no epilogue arithmetic
-            acc[0] += dot[0] + dot[31];
+            acc[0] += dot[0] + dot[CW - 1];
             continue;
           }
+          // blocks of BE columns, each step over the BE independent elements (BE chains in flight;
+          // 4 when the per-row sums take the registers)
+          constexpr int BE = KM > 12 ? 4 : 8;
 #pragma unroll
-          for (int jj = 0; jj < 32; ++jj) {
-            const int64_t c = c0 + half * 32 + jj;
-            const double xy = dot[jj] * pow2(24 - ex_r - __ldg(es + c));
-            const double d2 = fmax(fma(-2.0, xy, nr + __ldg(ns + c)), 0.0);
-            const double kv = exp2_neg(tsc * d2);
-            const double* cj = cs + (half * 32 + jj) * KM;
+          for (int jb = 0; jb < CW; jb += BE) {
+            double tt[BE], ff[BE], pp[BE];
+            int nn[BE];
 #pragma unroll
-            for (int v = 0; v < KM; ++v) acc[v] = fma(kv, cj[v], acc[v]);
+            for (int e = 0; e < BE; ++e) {
+              double sc, nc;
+              asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(sc), "=d"(nc)
+                           : "r"(cs + (uint32_t)((part * CW + jb + e) * ROW) * 8));
+              const double xy = (dot[jb + e] * pr) * sc;  // powers of two: exact
+              const double d2 = fmax(fma(-2.0, xy, nr + nc), 0.0);
+              tt[e] = fmax(tsc * d2, -1020.0);  // below 2^-1020 the kernel value is < 1e-307 (not 0)
+            }
+#pragma unroll
+            for (int e = 0; e < BE; ++e) {  // n = rint(t) (round to nearest even) by the 1.5 2^52 shift
+              const double big = tt[e] + kShift52;
+              const double n = big - kShift52;
+              ff[e] = tt[e] - n;  // exact, |f| <= 1/2
+              nn[e] = __double2loint(big);
+              pp[e] = kExp2C[0];
+            }
+#pragma unroll
+            for (int k = 1; k < 11; ++k)
+#pragma unroll
+              for (int e = 0; e < BE; ++e) pp[e] = fma(pp[e], ff[e], kExp2C[k]);
+#pragma unroll
+            for (int e = 0; e < BE; ++e) {
+              const double kv = pp[e] * pow2(nn[e]);
+              const uint32_t cj = cs + (uint32_t)((part * CW + jb + e) * ROW + 2) * 8;
+#pragma unroll
+              for (int v = 0; v < KM; v += 2) {
+                double c0v, c1v;
+                asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(c0v), "=d"(c1v) : "r"(cj + (uint32_t)v * 8));
+                acc[v] = fma(kv, c0v, acc[v]);
+                if (v + 1 < KM) acc[v + 1] = fma(kv, c1v, acc[v + 1]);
+              }
+            }
           }
         }
       }
-      // the two column halves of a row: half 1 hands its sums to half 0 through shared memory
+      // the column parts of a row: parts 1 .. NP-1 hand their sums to part 0 in turn (fixed order)
       double* red = &sm.red[0][0];
-      asm volatile("bar.sync 1, 256;" ::: "memory");
-      if (half == 1)
+      for (int p = 1; p < NP; ++p) {
+        asm volatile("bar.sync 1, %0;" ::"r"(ET) : "memory");
+        if (part == p)
 #pragma unroll
-        for (int v = 0; v < KM; ++v) red[(q * 32 + lane) * KM + v] = acc[v];
-      asm volatile("bar.sync 1, 256;" ::: "memory");
-      if (half == 0) {
-        double* out = part + ((int64_t)unit_item[u] * m_pad + r) * km1_pad;
+          for (int v = 0; v < KM; ++v) red[(q * 32 + lane) * KM + v] = acc[v];
+        asm volatile("bar.sync 1, %0;" ::"r"(ET) : "memory");
+        if (part == 0)
+#pragma unroll
+          for (int v = 0; v < KM; ++v) acc[v] += red[(q * 32 + lane) * KM + v];
+      }
+      if (part == 0) {
+        double* out = part_out + ((int64_t)unit_item[u] * m_pad + r) * km1_pad;
 #pragma unroll
         for (int v = 0; v < KM; ++v)
-          if (v < km1) out[v] = acc[v] + red[(q * 32 + lane) * KM + v];
+          if (v < km1) out[v] = acc[v];
         for (int v = km1; v < km1_pad; ++v) out[v] = 0.0;
       }
     }
@@ -420,20 +501,18 @@ void launch_dec_i8(const int8_t* tplanes, int64_t m_pad, const int32_t* et, cons
   GM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
   const int grid = n_units < sms ? n_units : sms;
   static const int diag = getenv("GMPSVM_I8_DIAG") ? atoi(getenv("GMPSVM_I8_DIAG")) : 0;
-  auto go = [&](auto kern, size_t smem) {
+  auto go = [&](auto kern, size_t smem, int threads) {
     set_max_dyn_smem(kern, smem);
-    GM_LAUNCH(kern, dim3(grid), dim3(kIThreads), smem, st, mt, ms, tiles, unit_off, unit_item, n_units, et, nt, es, ns,
+    GM_LAUNCH(kern, dim3(grid), dim3(threads), smem, st, mt, ms, tiles, unit_off, unit_item, n_units, et, nt, es, ns,
               coef64, km1, km1_pad, d8, m_pad, nsv_pad, gamma, part, diag);
   };
-  // GMPSVM_I8_COLLECT=0: no A-operand collector reuse (measurement)
-  static const bool collect = !(getenv("GMPSVM_I8_COLLECT") && std::string(getenv("GMPSVM_I8_COLLECT")) == "0");
   // KM: pair columns contracted per SV, the smallest instantiation >= k - 1
-  if (km1 <= 2) collect ? go(dec_i8_kernel<2, true>, sizeof(DecI8Smem<2>) + 1024) : go(dec_i8_kernel<2, false>, sizeof(DecI8Smem<2>) + 1024);
-  else if (km1 <= 4) collect ? go(dec_i8_kernel<4, true>, sizeof(DecI8Smem<4>) + 1024) : go(dec_i8_kernel<4, false>, sizeof(DecI8Smem<4>) + 1024);
-  else if (km1 <= 9) collect ? go(dec_i8_kernel<9, true>, sizeof(DecI8Smem<9>) + 1024) : go(dec_i8_kernel<9, false>, sizeof(DecI8Smem<9>) + 1024);
-  else if (km1 <= 12) collect ? go(dec_i8_kernel<12, true>, sizeof(DecI8Smem<12>) + 1024) : go(dec_i8_kernel<12, false>, sizeof(DecI8Smem<12>) + 1024);
-  else if (km1 <= 25) collect ? go(dec_i8_kernel<25, true>, sizeof(DecI8Smem<25>) + 1024) : go(dec_i8_kernel<25, false>, sizeof(DecI8Smem<25>) + 1024);
-  else if (km1 <= 32) collect ? go(dec_i8_kernel<32, true>, sizeof(DecI8Smem<32>) + 1024) : go(dec_i8_kernel<32, false>, sizeof(DecI8Smem<32>) + 1024);
+  if (km1 <= 2) go(dec_i8_kernel<2>, sizeof(DecI8Smem<2>) + 1024, i8_threads<2>());
+  else if (km1 <= 4) go(dec_i8_kernel<4>, sizeof(DecI8Smem<4>) + 1024, i8_threads<4>());
+  else if (km1 <= 9) go(dec_i8_kernel<9>, sizeof(DecI8Smem<9>) + 1024, i8_threads<9>());
+  else if (km1 <= 12) go(dec_i8_kernel<12>, sizeof(DecI8Smem<12>) + 1024, i8_threads<12>());
+  else if (km1 <= 25) go(dec_i8_kernel<25>, sizeof(DecI8Smem<25>) + 1024, i8_threads<25>());
+  else if (km1 <= 32) go(dec_i8_kernel<32>, sizeof(DecI8Smem<32>) + 1024, i8_threads<32>());
   else throw Error(GMPSVM_ENOTIMPL, "int8 decision values support k <= 33");
 }
 
