@@ -76,13 +76,6 @@ struct DecI8Smem {
   uint32_t tmem_base;
 };
 
-__device__ __forceinline__ bool elect_one() {  // one lane of the (converged) warp
-  uint32_t pred = 0;
-  asm volatile("{\n .reg .b32 rx;\n .reg .pred px;\n elect.sync rx|px, 0xffffffff;\n selp.b32 %0, 1, 0, px;\n}\n"
-               : "=r"(pred));
-  return pred != 0;
-}
-
 // K-major operand, 64-byte swizzle: 8-row groups 512 B apart (SBO), LBO unused, version 1
 __device__ __forceinline__ uint64_t umma_desc_sw64_addr(uint32_t addr32) {
   const uint64_t addr = addr32;

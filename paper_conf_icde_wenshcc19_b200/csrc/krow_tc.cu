@@ -183,29 +183,32 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {  // ---- MMA issuer
-      int g = 0, it = 0;
-      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
-        if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);  // epilogue drained the previous tile
+    // ---- MMA issuer: the whole warp runs the loop (warp-uniform: descriptors and TMEM addresses
+    // in uniform registers) and one elected lane issues -- from a lone lane-0 thread every MMA went
+    // through an ELECT / R2UR.BROADCAST / BRA.U.ANY sequence (dec_i8.cu)
+    int g = 0, it = 0;
+    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+      if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);  // epilogue drained the previous tile
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      for (int kb = 0; kb < nk; ++kb, ++g) {
+        const int s = g % kTcStages;
+        mbar_wait(&sm.full[s], (g / kTcStages) & 1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        for (int kb = 0; kb < nk; ++kb, ++g) {
-          const int s = g % kTcStages;
-          mbar_wait(&sm.full[s], (g / kTcStages) & 1);
+        uint8_t* st = sm.stage[s];
+        const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
+        const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
+        // the FP32 accumulation error of the tensor-core adds grows with the number of MMAs into
+        // an accumulator times its magnitude: the hi.hi
+        // products of each k third and the small corrections get accumulators of their own
+        const int j = (kb * jn) / nk;
+        const int kb_first = (j * nk + jn - 1) / jn;
+        // the epilogue releases accumulators 0 + 3 first (the next tile starts with them) and 1 + 2
+        // after: the second half of its drain overlaps this tile's first k third
+        if (it > 0 && j == 1 && kb == kb_first) {
+          mbar_wait(&sm.tmem_empty2, (it - 1) & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          uint8_t* st = sm.stage[s];
-          const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
-          const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
-          // the FP32 accumulation error of the tensor-core adds grows with the number of MMAs into
-          // an accumulator times its magnitude: the hi.hi
-          // products of each k third and the small corrections get accumulators of their own
-          const int j = (kb * jn) / nk;
-          const int kb_first = (j * nk + jn - 1) / jn;
-          // the epilogue releases accumulators 0 + 3 first (the next tile starts with them) and 1 + 2
-          // after: the second half of its drain overlaps this tile's first k third
-          if (it > 0 && j == 1 && kb == kb_first) {
-            mbar_wait(&sm.tmem_empty2, (it - 1) & 1);
-            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          }
+        }
+        if (elect_one()) {
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 TF32 = 32 bytes along K inside the atom
@@ -214,8 +217,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           }
           umma_commit(&sm.empty[s]);
         }
-        umma_commit(&sm.tmem_full);
+        __syncwarp();
       }
+      if (elect_one()) umma_commit(&sm.tmem_full);
+      __syncwarp();
     }
   } else {  // ---- epilogue: warps 2..5, TMEM lane quarter (warp % 4)
     const int q = warp & 3;
@@ -909,23 +914,23 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
       }
     }
-  } else if (warp == 1) {
-    if (lane == 0) {  // ---- MMA issuer
-      int g = 0, it = 0, nnew = 0;
-      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
-        const int4 tl = tiles[t];
-        if (!rows_tile_live(ra, tl, nnew)) continue;
-        if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
+  } else if (warp == 1) {  // ---- MMA issuer (whole warp, one elected lane issues; see krow_tc_kernel)
+    int g = 0, it = 0, nnew = 0;
+    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+      const int4 tl = tiles[t];
+      if (!rows_tile_live(ra, tl, nnew)) continue;
+      if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      for (int kb = 0; kb < nk; ++kb, ++g) {
+        const int s = g % kTcStages;
+        mbar_wait(&sm.full[s], (g / kTcStages) & 1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        for (int kb = 0; kb < nk; ++kb, ++g) {
-          const int s = g % kTcStages;
-          mbar_wait(&sm.full[s], (g / kTcStages) & 1);
-          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          uint8_t* st = sm.stage[s];
-          const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
-          const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
-          const int j = (kb * jn) / nk;
-          const int kb_first = (j * nk + jn - 1) / jn;
+        uint8_t* st = sm.stage[s];
+        const uint64_t ahi = umma_desc_sw128(st), alo = umma_desc_sw128(st + kABytes);
+        const uint64_t bhi = umma_desc_sw128(st + 2 * kABytes), blo = umma_desc_sw128(st + 2 * kABytes + kBBytes);
+        const int j = (kb * jn) / nk;
+        const int kb_first = (j * nk + jn - 1) / jn;
+        if (elect_one()) {
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;
@@ -934,9 +939,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           }
           umma_commit(&sm.empty[s]);
         }
-        umma_commit(&sm.tmem_full);
-        ++it;
+        __syncwarp();
       }
+      if (elect_one()) umma_commit(&sm.tmem_full);
+      __syncwarp();
+      ++it;
     }
   } else {  // ---- epilogue: warps 2..5 (TMEM lane quarter warp % 4), thread = one new row
     const int q = warp & 3;
