@@ -342,7 +342,11 @@ def run_gpu(args, spec):
                          "frac_of_fp32_simt_peak": achieved / _fp32_peak(),
                          "fp32_simt_peak": _fp32_peak(),
                          "flops_per_launch": s["kernel_flops"], "launch_ms": krow_ms,
-                         "algorithmic": "n(n+1)/2 kernel values x (2d+3) flop"},
+                         "algorithmic": "n(n+1)/2 kernel values x (2d+3) flop",
+                         "schedule": ("lead mode (engine.cu): launch_ms spans the contraction's two launches, wave 0 "
+                                      "(the hardest pair's class blocks) on every SM and wave 1 on 140 of 148 SMs while "
+                                      "that pair's solver runs on the rest; GMPSVM_LEAD=0 times it alone"
+                                      if os.environ.get("GMPSVM_LEAD", "1") != "0" else "alone (GMPSVM_LEAD=0)")},
             "phases_ms": {"stage": s["t_stage_ms"], "kernel_values": s["t_kernel_ms"], "select": s["t_select_ms"],
                           "subproblem": s["t_subproblem_ms"], "f_update": s["t_fupdate_ms"],
                           "finalize": s["t_finalize_ms"], "train_total": s["t_total_ms"],
