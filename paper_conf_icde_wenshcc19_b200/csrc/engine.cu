@@ -1230,6 +1230,8 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   std::vector<size_t> wave_off(ng + 1, 0);  // lead mode: tile range of wave g
   const bool two_cta = fk_tc && !lead && ktype == 0 && krow_tc_2cta();  // lead waves: single-CTA tiles
   double kv_subset = -1;  // >= 0: kernel values computed for a pair subset (tiles skipped)
+  // 2-CTA clusters sharing the row operand by TMA multicast (the Gaussian kernel, FP16 split)
+  const bool kmc = fk_tc && !two_cta && ktype == 0 && krow_tc_mc();
   if (fk_tc) {
     // class range [cr[2i], cr[2i+1]] of the rows of tile row / column i
     const int nti = (int)ceil_div(n, kKrowTileRows);
@@ -1262,7 +1264,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     std::vector<std::vector<uint8_t>> gmask;  // lead mode: class blocks per group
     if (lead)
       for (int g = 0; g < ng; ++g) gmask.push_back(blocks_of(gpos[g], gpos[g + 1]));
-    std::vector<int64_t> tkey = {n, two_cta ? 1 : 0, k};  // what the tile list depends on
+    std::vector<int64_t> tkey = {n, two_cta ? 1 : 0, k, kmc ? 1 : 0};  // what the tile list depends on
     tkey.insert(tkey.end(), coff.begin(), coff.end());
     for (const uint8_t v : need) tkey.push_back(v);
     for (const auto& gm : gmask) {
@@ -1300,9 +1302,12 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         }
         tiles.clear();
         for (int g = 0; g < ng; ++g) {
+          if (kmc) w[g] = krow_tc_mc_pairs(w[g]);
           tiles.insert(tiles.end(), w[g].begin(), w[g].end());
           wave_off[g + 1] = tiles.size();
         }
+      } else if (kmc) {
+        tiles = krow_tc_mc_pairs(tiles);
       }
       n_tiles = tiles.size();
       int2* dt = nullptr;
@@ -1325,21 +1330,28 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     }
   }
   tm.mark(PH_KERNEL);
-  const KrowKernel kk{ktype, (float)gamma, (float)kcoef0, 0.f, kdegree};
+  // lead mode: CTAs of the kernel-value wave beside the lead group that have started (the
+  // persistent lead group's workers launch only once they all hold their SMs)
+  DevBuf<unsigned long long> d_kres(fk_tc && lead ? 1 : 0, st);
+  int kres_wait = 0;
+  const KrowKernel kk{ktype, (float)gamma, (float)kcoef0, 0.f, kdegree, nullptr};
   const KrowKernel* kkp = ktype != 0 ? &kk : nullptr;
   if (fk_tc && !lead) {
     launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles, (int)n_tiles, norms.get(), n, gamma, ksc, K.get(), ldk, st,
-                   two_cta, kkp);
+                   two_cta, kkp, 0, nullptr, kmc, (int)d);
   } else if (fk_tc) {  // the waves on the low-priority stream: the solver's CTAs are dispatched first
+    GM_CUDA(cudaMemsetAsync(d_kres.get(), 0, sizeof(unsigned long long), st));
     cudaEvent_t ev_staged = evk.get();
     GM_CUDA(cudaEventRecord(ev_staged, st));
     GM_CUDA(cudaStreamWaitEvent(kst, ev_staged, 0));
     GM_CUDA(cudaEventRecord(ev_k0, kst));
     for (int g = 0; g < ng; ++g) {
       const size_t cnt = wave_off[g + 1] - wave_off[g];
+      if (cnt && g == 1) kres_wait = krow_tc_grid((int)cnt, reserve_env, kmc);  // the wave beside the lead group
       if (cnt)
         launch_krow_tc(Xhi.get(), Xlo.get(), n_pad, d_pad, d_tiles + wave_off[g], (int)cnt, norms.get(), n, gamma, ksc,
-                       K.get(), ldk, kst, false, kkp, g == 0 ? 0 : reserve_env);
+                       K.get(), ldk, kst, false, kkp, g == 0 ? 0 : reserve_env, g == 1 ? d_kres.get() : nullptr, kmc,
+                       (int)d);
       ev_wave[g] = evk.get(lead_dbg_t);
       GM_CUDA(cudaEventRecord(ev_wave[g], kst));
     }
@@ -1446,14 +1458,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   const int trace_cap = 1 << 16;
   DevBuf<int64_t> d_trace(trace_pos >= 0 ? (size_t)trace_cap * 3 + 2 * (size_t)Pl : 0, st);
   if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace.get(), 0, ((size_t)trace_cap * 3 + 2 * (size_t)Pl) * 8, st));
-  DevBuf<int32_t> d_trace_n(trace_pos >= 0 ? 1 : 0, st);
-  if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace_n.get(), 0, 4, st));
+  DevBuf<int32_t> d_trace_n(trace_pos >= 0 ? 4 : 0, st);
+  if (trace_pos >= 0) GM_CUDA(cudaMemsetAsync(d_trace_n.get(), 0, 16, st));
   GM_CUDA(cudaMemsetAsync(d_body.get(), 0, Pl * 8, st));
   a.body_iters = d_body.get();
   a.trace = d_trace.get();
   a.trace_n = d_trace_n.get();
   a.trace_pair = trace_pos;
   a.trace_cap = trace_cap;
+  static const int fu_chunks = getenv("GMPSVM_FU_CHUNKS") ? std::max(1, atoi(getenv("GMPSVM_FU_CHUNKS"))) : 1;
+  a.fu_chunks = fu_chunks;
+  static const bool smo_f64_env = getenv("GMPSVM_SMO_F32") && std::string(getenv("GMPSVM_SMO_F32")) == "0";
+  a.smo_f32 = (!smo_f64_env && ktype == 0) ? 1 : 0;  // the Gaussian kernel's QP is convex: FP32 local f
   a.outer_iters = d_outer.get();
   a.b = d_b.get();
   a.A = d_A.get();
@@ -1480,8 +1496,55 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   int64_t body_launches = 0;
   std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
   int n_branches = 0, final_selects = 0;
-  {
-    // Device-driven outer loops (default): one CUDA graph holding, per branch (packing above), a
+  // Persistent solver (default where it applies: FULL_K, every pair on the wsolve.cu kernels, at
+  // most two pair groups): one launch per group -- its pairs' leaders plus workers on the SMs the
+  // group may use (lead mode: the lead group on the `reserve` SMs beside the kernel-value waves,
+  // the rest on the others) -- instead of the graphs of per-step kernels below.
+  int n_sm = 0;
+  GM_CUDA(cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, opt.device));
+  bool persist = !rc && ng <= 2 && !smo_prof && ws_persist_supported(Bw, np_max);
+  std::vector<int> pgrid(ng, 0);
+  std::vector<size_t> pq_off(ng + 1, 0);
+  if (persist) {
+    const int wps = ws_persist_workers_per_sm();
+    for (int g = 0; g < ng; ++g) {
+      const int pg = gpos[g + 1] - gpos[g];
+      // the group's SMs: lead mode -- the lead group beside the last kernel-value wave on the
+      // `reserve` SMs, the rest on the others; workers fill the SMs around the leaders
+      const int sms = !lead ? n_sm : (g == 0 ? std::max(2, std::min(reserve_env, n_sm / 2)) : n_sm - std::max(2, std::min(reserve_env, n_sm / 2)));
+      pgrid[g] = std::max(0, sms - pg) * wps + pg;  // workers
+      if (pg >= sms || wps < 1) persist = false;
+      pq_off[g + 1] = pq_off[g] + ws_persist_ring_bytes() + ws_persist_ctr_words(pg) * 8;
+    }
+  }
+  DevBuf<uint8_t> d_pq(persist ? pq_off[ng] : 0, st);
+  if (persist) GM_CUDA(cudaMemsetAsync(d_pq.get(), 0, pq_off[ng], st));
+  auto pq_ctr = [&](int g) {
+    return reinterpret_cast<unsigned long long*>(d_pq.get() + pq_off[g] + ws_persist_ring_bytes());
+  };
+  if (persist) {
+    GM_CUDA(cudaEventRecord(ev_ready, st));
+    for (int g = 0; g < ng; ++g) {
+      cudaStream_t ls = pool[g];
+      GM_CUDA(cudaStreamWaitEvent(ls, ev_ready, 0));
+      if (lead) GM_CUDA(cudaStreamWaitEvent(ls, ev_wave[g], 0));
+      if (lead_dbg_t) {
+        ev_gst[g] = evk.get(true);
+        ev_gend[g] = evk.get(true);
+        GM_CUDA(cudaEventRecord(ev_gst[g], ls));
+      }
+      SolverArgs ag = a;
+      ag.pair_base = gpos[g];
+      launch_ws_persist(ag, gpos[g + 1] - gpos[g], pgrid[g], max_outer, d_pq.get() + pq_off[g], pq_ctr(g), ls,
+                        lead && g == 0 ? d_kres.get() : nullptr, lead && g == 0 ? kres_wait : 0);
+      cudaEvent_t ev = ev_gend[g] ? ev_gend[g] : evp.get();
+      GM_CUDA(cudaEventRecord(ev, ls));
+      GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
+    }
+    n_branches = ng;
+    destroy_parked_graphs();
+  } else {
+    // Device-driven outer loops: one CUDA graph holding, per branch (packing above), a
     // conditional WHILE node whose body is that branch's select -> [rows] -> gather -> local SMO ->
     // f-update chain (the f-update kernel sets the loop condition), followed by one last selection
     // (the stop test on the final alpha) on the split path.  The branches are independent, so no
@@ -1661,6 +1724,11 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
   HT("fin_d2h");
+  for (int g = 0; persist && g < ng; ++g) {
+    unsigned long long perr = 0;
+    GM_CUDA(cudaMemcpy(&perr, pq_ctr(g) + 3, 8, cudaMemcpyDeviceToHost));
+    if (perr) throw Error(GMPSVM_ECUDA, "persistent solver: a wait timed out (group " + std::to_string(g) + ")");
+  }
   {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
     int64_t ex = final_selects;  // one final selection per split-path branch
     for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_per_pair[i];  // counted at each branch's first pair
@@ -1680,18 +1748,28 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     std::vector<int> order(nt);
     for (int i = 0; i < nt; ++i) order[i] = i;
     std::sort(order.begin(), order.end(), [&](int x, int y) { return tr[3 * x + 1] < tr[3 * y + 1]; });
-    const char* names[7] = {"select", "gather", "smo", "fupdate", "rows_gather", "rows_contract", "ws_solve"};
-    double dur[7] = {0}, cnt[7] = {0}, gap_before[7] = {0};
+    const char* names[11] = {"select", "gather", "smo", "fupdate", "rows_gather", "rows_contract", "ws_solve",
+                             "fu_end_to_select", "select_resident_wait", "gather_task", "fupdate_task"};
+    double dur[11] = {0}, cnt[11] = {0}, gap_before[11] = {0};
+    int prev = -1;
     for (int j = 0; j < nt; ++j) {
       const int i = order[j];
       const int kd = (int)tr[3 * i];
       dur[kd] += (double)(tr[3 * i + 2] - tr[3 * i + 1]);
       cnt[kd] += 1;
-      if (j > 0) gap_before[kd] += (double)(tr[3 * i + 1] - tr[3 * order[j - 1] + 2]);
+      if (kd >= 7) continue;  // handoff records: not part of the kernel chain
+      if (prev >= 0) gap_before[kd] += (double)(tr[3 * i + 1] - tr[3 * prev + 2]);
+      prev = i;
     }
-    const double span = nt ? (double)(tr[3 * order[nt - 1] + 2] - tr[3 * order[0] + 1]) : 0.0;
+    int64_t s_lo = INT64_MAX, s_hi = 0;  // span of the kernel chain (kinds 0-6)
+    for (int i = 0; i < nt; ++i)
+      if (tr[3 * i] < 7) {
+        s_lo = std::min(s_lo, tr[3 * i + 1]);
+        s_hi = std::max(s_hi, tr[3 * i + 2]);
+      }
+    const double span = s_hi > 0 ? (double)(s_hi - s_lo) : 0.0;
     std::string line;
-    for (int kd = 0; kd < 7; ++kd)
+    for (int kd = 0; kd < 11; ++kd)
       if (cnt[kd] > 0)
         line += std::string(" ") + names[kd] + " n=" + std::to_string((int)cnt[kd]) +
                 " mean_us=" + std::to_string(dur[kd] / cnt[kd] / 1e3).substr(0, 6) +

@@ -54,6 +54,7 @@ struct KrowKernel {
   int type;
   float gamma, coef0, inv_s2;
   int degree;
+  unsigned long long* resident;  // optional: each CTA adds 1 when it starts (persistent solver's lead group)
 };
 // max over the rows (perm[j] >= 0, or all) of |x - mu| (synchronises the stream)
 float launch_maxabs(const float* X, int64_t n, int d, const int64_t* perm, const float* mu, cudaStream_t st);
@@ -101,7 +102,13 @@ void launch_dec_tc(const void* thi, const void* tlo, int64_t m_pad, const void* 
                    const KrowKernel* dk = nullptr);
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
-                    bool two_cta = false, const KrowKernel* dk = nullptr, int reserve_sms = 0);
+                    bool two_cta = false, const KrowKernel* dk = nullptr, int reserve_sms = 0,
+                    unsigned long long* resident = nullptr, bool mc = false, int d_real = 0);
+int krow_tc_grid(int n_tiles, int reserve_sms, bool mc = false);  // CTAs of that launch
+// 2-CTA clusters with the shared row operand multicast (default; GMPSVM_KROW_MC=0 off): the tile
+// list must be cluster pairs (krow_tc_mc_pairs) and the launch passes mc = true
+bool krow_tc_mc();
+std::vector<int2> krow_tc_mc_pairs(const std::vector<int2>& tiles);
 void launch_row_norms(const float* X, int64_t n, int d, const int64_t* perm, float* norms, int64_t n_pad, int32_t* bad,
                       cudaStream_t st);
 bool krow_use_tc();  // GMPSVM_KROW=simt selects the FP32 SIMT kernel
@@ -129,6 +136,8 @@ struct SolverArgs {
   int64_t* trace;       // optional kernel timeline of one pair (GMPSVM_TRACE=<pair position>): [cap][3]
   int32_t* trace_n;
   int32_t trace_pair, trace_cap;
+  int32_t fu_chunks = 1;  // 128-column chunks per f-update CTA (ws_fupdate_kernel)
+  int32_t smo_f32 = 0;    // local SMO with FP32 working-set f (wsolve.cu ws_smo_body)
   int64_t* sel_phase;   // [P][5] optional select_ws phase cycles (GMPSVM_SMO_PHASES=1), else NULL
   int32_t* outer_iters; // [P]
   double* b;            // [P]
@@ -200,6 +209,19 @@ __host__ __device__ inline size_t kws_pair_stride(int B) {
 // iteration, and across iterations when chained (the previous iteration is in the same stream)
 void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphConditionalHandle h, int set_cond,
                          int64_t max_outer, cudaStream_t st, bool chained = false);
+// Persistent solver (wsolve.cu): the outer loops of pairs [pair_base, pair_base + P) as P leader
+// CTAs (one per SM) and `nworkers` worker CTAs (ws_persist_workers_per_sm() per SM beside them),
+// launched together on st; ring: ws_persist_ring_bytes(), ctr: ws_persist_ctr_words(P) words,
+// both zeroed before the launch; ctr[3] != 0 after the run: a wait timed out (the solve is invalid).
+bool ws_persist_supported(int B, int64_t np_max);
+size_t ws_persist_smem(int B);
+size_t ws_persist_ctr_words(int P);
+size_t ws_persist_ring_bytes();
+int ws_persist_workers_per_sm();
+// wait_resident > 0: the leaders trigger the workers only once *res_ctr (the kernel-value launch's
+// started-CTA count, KrowKernel::resident) reaches it, so the workers land beside that launch.
+void launch_ws_persist(const SolverArgs& a, int P, int nworkers, int64_t max_outer, void* ring, unsigned long long* ctr,
+                       cudaStream_t st, const unsigned long long* res_ctr = nullptr, int wait_resident = 0);
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st);

@@ -129,20 +129,35 @@ __device__ __forceinline__ float dot_kernel_value(float xy, const KrowKernel& kp
 // producer runs ahead across tile boundaries through the smem ring; the epilogue drains the four
 // TMEM accumulators into registers and releases TMEM at once (tmem_empty), so the MMAs of the
 // next tile overlap the exp + stores of the current one.
-template <bool F16, int KT>  // KT: 0 the Gaussian, else a dot-product kernel (kp): 1 linear, 2 poly, 3 sigmoid
+//
+// MC (2-CTA cluster, krow_tc_mc): the tile list holds pairs of tiles of the same row block --
+// entries 2p and 2p + 1 go to cluster p's CTA 0 and 1 (a second entry with y < 0 is a dummy: its
+// CTA runs the pipeline on valid rows and stores nothing).  Each CTA loads half of the shared A
+// rows (hi and lo) and multicasts it to both CTAs, and its own B rows: 48 instead of 64 KB per
+// k-step leave L2 for each SM.  The MMA commits free a ring stage in both CTAs (empty barriers
+// count two arrivals), so neither producer overwrites a stage its peer still reads.
+// kk_last: MMAs (K = 16) of the last k-step that touch real columns -- the rest multiply the zero
+// padding of d (784 -> 832 for MNIST-shaped rows) and are skipped (same sums, bit for bit).
+template <bool F16, int KT, bool MC = false>  // KT: 0 the Gaussian, else a dot-product kernel (kp): 1 linear, 2 poly, 3 sigmoid
 __global__ void __launch_bounds__(kTcThreads, 1)
     krow_tc_kernel(const __grid_constant__ CUtensorMap map_hi, const __grid_constant__ CUtensorMap map_lo,
                    const __grid_constant__ CUtensorMap map_ksw, const __grid_constant__ CUtensorMap map_kns,
                    const int2* __restrict__ tiles, int n_tiles, const float* __restrict__ norms, int64_t n, int nk,
-                   float scale, float* __restrict__ K, int64_t ldk, int tma_store, KrowKernel kp) {
+                   float scale, float* __restrict__ K, int64_t ldk, int tma_store, KrowKernel kp,
+                   const __grid_constant__ CUtensorMap map_hi64, const __grid_constant__ CUtensorMap map_lo64, int kk_last) {
   extern __shared__ __align__(1024) uint8_t dsmem[];
   TcSmem& sm = *reinterpret_cast<TcSmem*>((reinterpret_cast<uintptr_t>(dsmem) + 1023) & ~uintptr_t(1023));
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // the CTA's tiles: entry t0, t0 + tstep, ... of the list
+  const int crank = MC ? (int)cluster_ctarank() : 0;
+  const int t0 = MC ? 2 * (int)(blockIdx.x >> 1) + crank : (int)blockIdx.x;
+  const int tstep = (int)gridDim.x;  // MC: gridDim.x / 2 clusters x 2 entries
 
   if (warp == 0 && lane == 0) {
+    if (kp.resident) atomicAdd(kp.resident, 1ull);  // this CTA holds its SM (engine.cu lead mode)
     for (int s = 0; s < kTcStages; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], 1);
+      mbar_init(&sm.empty[s], MC ? 2 : 1);
     }
     mbar_init(&sm.tmem_full, 1);
     mbar_init(&sm.tmem_empty, 4);   // one arrive per epilogue warp: accumulators 0 and 3 drained
@@ -159,6 +174,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  if (MC) cluster_sync();  // both CTAs' barriers initialised before any multicast or remote arrive
   const uint32_t tmem = sm.tmem_base;
   const int jn = nk < kMainAcc ? nk : kMainAcc;  // hi.hi accumulators in use (short k ranges)
 
@@ -166,17 +182,23 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     if (lane == 0) {  // ---- TMA producer (runs ahead across tiles)
       int g = 0;
       const uint64_t pol = policy_evict_last();
-      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+      for (int t = t0; t < n_tiles; t += tstep) {
         const int2 tile = tiles[t];
-        const int r0 = tile.x * kTM, c0 = tile.y * kTN;
+        const int r0 = tile.x * kTM, c0 = (tile.y < 0 ? tile.x : tile.y) * kTN;  // dummy: valid rows, no stores
         for (int kb = 0; kb < nk; ++kb, ++g) {
           const int s = g % kTcStages;
           if (g >= kTcStages) mbar_wait(&sm.empty[s], ((g / kTcStages) + 1) & 1);
           uint8_t* st = sm.stage[s];
           mbar_expect_tx(&sm.full[s], kStageBytes);
           const int kx = kb * (F16 ? 2 * kTK : kTK);
-          tma_load_2d(st, &map_hi, kx, r0, &sm.full[s], pol);
-          tma_load_2d(st + kABytes, &map_lo, kx, r0, &sm.full[s], pol);
+          if (MC) {  // half of the A rows from each CTA, to both
+            const uint32_t ho = (uint32_t)crank * (kABytes / 2);
+            tma_load_2d_mc(st + ho, &map_hi64, kx, r0 + crank * (kTM / 2), &sm.full[s], (uint16_t)3, pol);
+            tma_load_2d_mc(st + kABytes + ho, &map_lo64, kx, r0 + crank * (kTM / 2), &sm.full[s], (uint16_t)3, pol);
+          } else {
+            tma_load_2d(st, &map_hi, kx, r0, &sm.full[s], pol);
+            tma_load_2d(st + kABytes, &map_lo, kx, r0, &sm.full[s], pol);
+          }
           tma_load_2d(st + 2 * kABytes, &map_hi, kx, c0, &sm.full[s], pol);
           tma_load_2d(st + 2 * kABytes + kBBytes, &map_lo, kx, c0, &sm.full[s], pol);
         }
@@ -187,7 +209,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     // in uniform registers) and one elected lane issues -- from a lone lane-0 thread every MMA went
     // through an ELECT / R2UR.BROADCAST / BRA.U.ANY sequence (dec_i8.cu)
     int g = 0, it = 0;
-    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+    for (int t = t0; t < n_tiles; t += tstep, ++it) {
       if (it > 0) mbar_wait(&sm.tmem_empty, (it - 1) & 1);  // epilogue drained the previous tile
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       for (int kb = 0; kb < nk; ++kb, ++g) {
@@ -209,13 +231,16 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         }
         if (elect_one()) {
+          const int nkk = kb == nk - 1 ? kk_last : kTK / 8;
 #pragma unroll
           for (int kk = 0; kk < kTK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 TF32 = 32 bytes along K inside the atom
-            umma_split3<F16, true>(tmem + j * kTN, tmem + kMainAcc * kTN, ahi + adv, alo + adv, bhi + adv, blo + adv,
-                                   (kb == kb_first && kk == 0) ? 0u : 1u, (kb | kk) ? 1u : 0u);
+            if (kk < nkk)
+              umma_split3<F16, true>(tmem + j * kTN, tmem + kMainAcc * kTN, ahi + adv, alo + adv, bhi + adv,
+                                     blo + adv, (kb == kb_first && kk == 0) ? 0u : 1u, (kb | kk) ? 1u : 0u);
           }
-          umma_commit(&sm.empty[s]);
+          if (MC) umma_commit_mc(&sm.empty[s], (uint16_t)3);  // the stage is free in both CTAs
+          else umma_commit(&sm.empty[s]);
         }
         __syncwarp();
       }
@@ -226,8 +251,18 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const int q = warp & 3;
     const uint64_t spol = policy_evict_first();
     int it = 0;
-    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+    for (int t = t0; t < n_tiles; t += tstep, ++it) {
       const int2 tile = tiles[t];
+      if (MC && tile.y < 0) {  // dummy partner tile: release the accumulators, store nothing
+        mbar_wait(&sm.tmem_full, it & 1);
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) {
+          asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty)) : "memory");
+          asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tmem_empty2)) : "memory");
+        }
+        continue;
+      }
       const int64_t r0 = (int64_t)tile.x * kTM, c0 = (int64_t)tile.y * kTN;
       const int64_t r = r0 + q * 32 + lane;
       const float nr = (r < n) ? norms[r] : 0.f;
@@ -348,6 +383,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
+  if (MC) cluster_sync();  // the peer's multicasts and commit arrivals into this CTA are done
   if (warp == 1) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
@@ -1332,9 +1368,16 @@ CUtensorMap make_kmap(float* K, int64_t n, int64_t ldk, bool swizzle) {
   return m;
 }
 
+int krow_tc_grid(int n_tiles, int reserve_sms, bool mc) {
+  const int cap = std::max(1, num_sms() - std::max(0, reserve_sms));
+  if (mc) return 2 * std::min(n_tiles / 2, cap / 2);  // clusters of two CTAs, one tile pair each
+  return n_tiles < cap ? n_tiles : cap;
+}
+
 void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, const int2* tiles, int n_tiles,
                     const float* norms, int64_t n, double gamma, float sc, float* K, int64_t ldk, cudaStream_t st,
-                    bool two_cta, const KrowKernel* dk, int reserve_sms) {
+                    bool two_cta, const KrowKernel* dk, int reserve_sms, unsigned long long* resident, bool mc,
+                    int d_real) {
   const bool f16 = krow_split_f16();
   const CUtensorMap mhi = make_map(hi, n_pad, d_pad, f16), mlo = make_map(lo, n_pad, d_pad, f16);
   // TMA stores need a 16-byte aligned base and row stride; otherwise every tile takes the
@@ -1365,27 +1408,85 @@ void launch_krow_tc(const void* hi, const void* lo, int64_t n_pad, int d_pad, co
     return;
   }
   // reserve_sms: SMs left free (the lead pairs' solver chains run beside the kernel values, engine.cu)
-  const int cap = std::max(1, sms - std::max(0, reserve_sms));
-  const int grid = n_tiles < cap ? n_tiles : cap;
+  const int grid = krow_tc_grid(n_tiles, reserve_sms, mc);
+  // MMAs of the last k-step over real columns (K = 16 FP16 / 8 TF32 per MMA)
+  const int kper = f16 ? 16 : 8, kblk = f16 ? 2 * kTK : kTK;
+  const int dr = d_real > 0 ? std::min(d_real, d_pad) : d_pad;
+  const int kk_last = std::max(1, (int)ceil_div(dr - (nk - 1) * kblk, kper));
+  const CUtensorMap mhi64 = mc ? make_map(hi, n_pad, d_pad, f16, kTM / 2) : mhi;
+  const CUtensorMap mlo64 = mc ? make_map(lo, n_pad, d_pad, f16, kTM / 2) : mlo;
   KrowKernel kp{};
   if (dk) {
     if (!f16 || two_cta) throw Error(GMPSVM_ENOTIMPL, "dot-product kernels need the FP16-split single-CTA launch");
+    if (mc) throw Error(GMPSVM_EINVAL, "cluster tile pairs are built for the Gaussian kernel only");
     kp = *dk;
+    kp.resident = nullptr;
     kp.inv_s2 = (float)(1.0 / ((double)sc * (double)sc));
     auto go = [&](auto kern) {
       GM_LAUNCH(kern, dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles, n_tiles, norms, n, nk, scale,
-                K, ldk, tma, kp);
+                K, ldk, tma, kp, mhi, mlo, kk_last);
     };
     if (kp.type == 1) go(krow_tc_kernel<true, 1>);
     else if (kp.type == 2) go(krow_tc_kernel<true, 2>);
     else go(krow_tc_kernel<true, 3>);
+    return;
+  }
+  kp.resident = resident;
+  if (mc) {
+    if (!f16 || (n_tiles & 1)) throw Error(GMPSVM_EINVAL, "cluster launch: FP16 split and tile pairs required");
+    set_max_dyn_smem(krow_tc_kernel<true, 0, true>, smem);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kTcThreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    GM_CUDA(cudaLaunchKernelEx(&cfg, krow_tc_kernel<true, 0, true>, mhi, mlo, mksw, mkns, tiles, n_tiles, norms, n, nk,
+                               scale, K, ldk, tma, kp, mhi64, mlo64, kk_last));
+    g_launches.fetch_add(1, std::memory_order_relaxed);
   } else if (f16) {
     GM_LAUNCH((krow_tc_kernel<true, 0>), dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles,
-              n_tiles, norms, n, nk, scale, K, ldk, tma, kp);
+              n_tiles, norms, n, nk, scale, K, ldk, tma, kp, mhi, mlo, kk_last);
   } else {
     GM_LAUNCH((krow_tc_kernel<false, 0>), dim3(grid), dim3(kTcThreads), smem, st, mhi, mlo, mksw, mkns, tiles,
-              n_tiles, norms, n, nk, scale, K, ldk, tma, kp);
+              n_tiles, norms, n, nk, scale, K, ldk, tma, kp, mhi, mlo, kk_last);
   }
+}
+
+bool krow_tc_mc() {
+  static const bool off = getenv("GMPSVM_KROW_MC") && std::string(getenv("GMPSVM_KROW_MC")) == "0";
+  return !off && krow_split_f16();
+}
+
+// Cluster tile pairs (krow_tc_kernel MC): tiles of the same row block, in list order as far as the
+// pairing allows (a tile waits for the next one of its row); an unmatched tile gets a dummy partner.
+std::vector<int2> krow_tc_mc_pairs(const std::vector<int2>& t) {
+  std::vector<int2> out;
+  out.reserve(t.size() + 64);
+  std::vector<int> pend;  // per row block: index into t of the unpaired tile, or -1
+  for (size_t i = 0; i < t.size(); ++i) {
+    const int r = t[i].x;
+    if ((int)pend.size() <= r) pend.resize(r + 1, -1);
+    if (pend[r] < 0) {
+      pend[r] = (int)i;
+    } else {
+      out.push_back(t[pend[r]]);
+      out.push_back(t[i]);
+      pend[r] = -1;
+    }
+  }
+  for (size_t r = 0; r < pend.size(); ++r)
+    if (pend[r] >= 0) {
+      out.push_back(t[pend[r]]);
+      out.push_back(make_int2((int)r, -1));
+    }
+  return out;
 }
 
 std::vector<int4> rows_tc_tiles(const std::vector<PairDesc>& pairs, int first, int count, int B) {

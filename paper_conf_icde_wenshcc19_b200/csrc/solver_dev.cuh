@@ -97,6 +97,19 @@ __device__ __forceinline__ uint64_t gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// one extra record (kind, t0, t1) of the traced pair
+__device__ __forceinline__ void trace_rec(const SolverArgs& a, int kid, int64_t t0, int64_t t1) {
+  const int s = atomicAdd(a.trace_n, 1);
+  if (s < a.trace_cap) {
+    a.trace[3 * s] = kid;
+    a.trace[3 * s + 1] = t0;
+    a.trace[3 * s + 2] = t1;
+  }
+}
+// latest exit of any f-update CTA of the traced pair (trace_n[2..3], 8-byte aligned)
+__device__ __forceinline__ unsigned long long* trace_fu_end(const SolverArgs& a) {
+  return reinterpret_cast<unsigned long long*>(a.trace_n + 2);
+}
 struct TraceScope {
   int64_t* buf;
   int32_t* n;

@@ -185,8 +185,8 @@ __device__ void ws_write_out(const SolverArgs& a, int lp, const int32_t* pick, i
     const int rank = wpre[x >> 5] + __popc(bm[x >> 5] & ((1u << (x & 31)) - 1u));
     a.ws_tmp[(int64_t)lp * B + e] = x;
     a.ws[(int64_t)lp * B + rank] = x;
-    st_al[rank] = a.alpha[pd.a_off + x];
-    st_f[rank] = a.f[pd.a_off + x];
+    st_al[rank] = __ldcg(a.alpha + pd.a_off + x);  // L2 loads: written by other CTAs of a persistent solver
+    st_f[rank] = __ldcg(a.f + pd.a_off + x);
     st_ix[rank] = x;
   }
   mark(2);
@@ -195,12 +195,13 @@ __device__ void ws_write_out(const SolverArgs& a, int lp, const int32_t* pick, i
 
 // ------------------------------------------------------------------------------------------
 // a4 selection
-__global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t max_outer) {
-  const int lp = blockIdx.x + a.pair_base;
-  extern __shared__ __align__(16) unsigned char sdyn[];
+// The selection of pair lp by the whole (kWT-thread) CTA: sdyn holds kWMaxNp * 9 bytes (keys,
+// flags), W the rest.  pdl: called from ws_select_kernel (programmatic dependent launch); the
+// persistent solver (ws_persist_kernel) calls it with its own ordering.
+__device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp, const int64_t max_outer,
+                                               unsigned char* sdyn, WSelSmall& W, const bool pdl) {
   uint64_t* keys = reinterpret_cast<uint64_t*>(sdyn);
   uint8_t* flags = sdyn + (size_t)kWMaxNp * 8;
-  __shared__ WSelSmall W;
   const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
   const PairDesc pd = a.pairs[lp];
   const int np = pd.n_s + pd.n_t, B = a.B;
@@ -231,7 +232,14 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
     W.pick[e] = idx;
     atomicOr(&W.retained[idx >> 5], 1u << (idx & 31));
   }
-  pdl_enter();  // alpha (local SMO), f (f-update) and status are read after the wait
+  const int64_t t_res = (a.trace && lp == a.trace_pair && t == 0) ? (int64_t)gtimer() : 0;
+  if (pdl) pdl_enter();  // alpha (local SMO), f (f-update) and status are read after the wait
+  if (t_res) {  // GMPSVM_TRACE: f-update grid end -> selection released; selection resident -> released
+    const int64_t t_go = (int64_t)gtimer();
+    const int64_t fe = (int64_t)*trace_fu_end(a);
+    if (fe) trace_rec(a, 7, fe, t_go);
+    trace_rec(a, 8, t_res, t_go);
+  }
   TraceScope ts_(a, lp, 0);
   if (a.status[lp] != 0) return;
   tq = clock64();
@@ -245,8 +253,8 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
 #pragma unroll
     for (int m = 0; m < kStageUnroll; ++m) {
       const int i = base + m * kWT + t;
-      av[m] = i < np ? al[i] : 0.0;
-      fv[m] = i < np ? fl[i] : 0.0;
+      av[m] = i < np ? __ldcg(al + i) : 0.0;  // L2 loads (see ws_write_out)
+      fv[m] = i < np ? __ldcg(fl + i) : 0.0;
     }
 #pragma unroll
     for (int m = 0; m < kStageUnroll; ++m) {
@@ -475,24 +483,25 @@ __global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t
   mark(4);
 }
 
+__global__ void __launch_bounds__(kWT, 1) ws_select_kernel(SolverArgs a, int64_t max_outer) {
+  extern __shared__ __align__(16) unsigned char sdyn[];
+  __shared__ WSelSmall W;
+  ws_select_body(a, blockIdx.x + a.pair_base, max_outer, sdyn, W, true);
+}
+
 // ------------------------------------------------------------------------------------------
 // a3: K_ws,ws tile (row stride ws_tile_ld(B)) from the resident kernel matrix
 constexpr int kGR = 8;  // tile rows per CTA
 
-__global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
-  const int lp = blockIdx.x + a.pair_base;
-  const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
-  pdl_enter();
-  TraceScope ts_(a, lp, 1);
-  if (a.status[lp] != 0) return;
-  const int np = pd.n_s + pd.n_t;
-  if (np <= a.B && a.outer_iters[lp] != 1) return;  // working set (and tile) unchanged
-  const int wn = a.ws_n[lp];
-  const int r0 = blockIdx.y * kGR;
+// rows [by * kGR, +kGR) of pair lp's tile by one 256-thread CTA (g: kWMaxB shared slots).  The
+// working set is read from L2: the persistent solver's workers run beside the selection's CTA.
+__device__ __forceinline__ void ws_gather_body(const SolverArgs& a, const int lp, const int by, int64_t* g) {
+  const PairDesc pd = a.pairs[lp];
+  const int wn = __ldcg(a.ws_n + lp);
+  const int r0 = by * kGR;
   if (r0 >= wn) return;
-  __shared__ int64_t g[kWMaxB];
   const int32_t* ws = a.ws + (int64_t)lp * a.B;
-  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, ws[e]);
+  for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, __ldcg(ws + e));
   __syncthreads();
   const int ld = ws_tile_ld(a.B);
   float* tile = a.Kws + (int64_t)lp * ws_buf_floats(a.B);
@@ -511,6 +520,18 @@ __global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
     const int r = r0 + q / wn, c = q % wn;
     if (r < r1) tile[(int64_t)r * ld + c] = v[m];
   }
+}
+
+__global__ void __launch_bounds__(256) ws_gather_kernel(SolverArgs a) {
+  const int lp = blockIdx.x + a.pair_base;
+  const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
+  pdl_enter();
+  TraceScope ts_(a, lp, 1);
+  if (a.status[lp] != 0) return;
+  const int np = pd.n_s + pd.n_t;
+  if (np <= a.B && a.outer_iters[lp] != 1) return;  // working set (and tile) unchanged
+  __shared__ int64_t g[kWMaxB];
+  ws_gather_body(a, lp, blockIdx.y, g);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -576,6 +597,31 @@ __device__ __forceinline__ void tree_max_f64(double (&k)[E]) {
     for (int i = 0; i + w < E; i += 2 * w) k[i] = k[i + w] > k[i] ? k[i + w] : k[i];
 }
 template <int E>
+__device__ __forceinline__ void tree_min_f32(float (&k)[E], int (&q)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w)
+      if (k[i + w] < k[i]) {
+        k[i] = k[i + w];
+        q[i] = q[i + w];
+      }
+}
+template <int E>
+__device__ __forceinline__ void tree_max_f32(float (&k)[E]) {
+#pragma unroll
+  for (int w = 1; w < E; w <<= 1)
+#pragma unroll
+    for (int i = 0; i + w < E; i += 2 * w) k[i] = k[i + w] > k[i] ? k[i + w] : k[i];
+}
+__device__ __forceinline__ uint32_t ord_key_f32(float x) {  // order-preserving bits of a finite float
+  const uint32_t u = __float_as_uint(x);
+  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
+__device__ __forceinline__ float key_f32(uint32_t k) {
+  return __uint_as_float((k & 0x80000000u) ? (k & 0x7fffffffu) : ~k);
+}
+template <int E>
 __device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
 #pragma unroll
   for (int w = 1; w < E; w <<= 1)
@@ -583,14 +629,22 @@ __device__ __forceinline__ void tree_max_u64(uint64_t (&k)[E]) {
     for (int i = 0; i + w < E; i += 2 * w) k[i] = k[i + w] > k[i] ? k[i + w] : k[i];
 }
 
-template <int E, bool PROF>  // PROF: GMPSVM_SMO_PHASES per-phase cycle counters (compiled out otherwise)
-__global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
-  const int lp = blockIdx.x + a.pair_base;
+// The local solve of pair lp by one warp (threadIdx.x < 32); mdyn: ws_smo_smem(B) bytes.
+// FT: the working set's f in the local solve -- float (a.smo_f32: the Gaussian kernel, default) or
+// double.  In FP32 the lane minima / maxima are 32-bit keys (u: two reductions instead of three,
+// f_max: one instead of two) and the f update of the working set is an FFMA; the step s was FP32
+// already (reading R29), and the global f, alpha and the clipping stay FP64, so the local solve
+// is the same heuristic subproblem solver with a rounding of f that the next outer iteration's
+// exact f replaces.  The dot-product kernels keep FP64 (the sigmoid kernel is not positive
+// semi-definite: its QP has several solutions and the iterate path decides which one is reached).
+// GMPSVM_SMO_F32=0 forces FP64 everywhere.
+template <int E, bool PROF, typename FT = double>  // PROF: GMPSVM_SMO_PHASES per-phase cycle counters
+__device__ __forceinline__ void ws_smo_body(const SolverArgs& a, const int lp, unsigned char* mdyn, const bool pdl) {
+  constexpr bool F32 = sizeof(FT) == 4;
   const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
-  pdl_wait();  // the f-update is released when the local solve ends (below)
+  if (pdl) pdl_wait();  // the f-update is released when the local solve ends (below)
   TraceScope ts_(a, lp, 2);
   if (a.status[lp] != 0) return;
-  extern __shared__ __align__(16) unsigned char mdyn[];
   const int lane = threadIdx.x;
   const int B = a.B, wn = a.ws_n[lp], ld = ws_tile_ld(B);
   uint32_t kws;  // K_ws,ws tile, row stride ld (opaque: keeps the shared window base out of the loop)
@@ -635,7 +689,7 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   const long long t_state = clock64();
   // per-row state: lane owns positions lane + 32 q (the working set sorted by index)
   int32_t idx[E];
-  double f[E];
+  FT f[E];
   uint32_t umask = 0u, lmask = 0u, ypos = 0u, vmask = 0u;
 #pragma unroll
   for (int q = 0; q < E; ++q) {
@@ -646,7 +700,7 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
     idx[q] = ix;
     const int y = (valid && ix < pd.n_s) ? 1 : -1;
     const double al = valid ? lds_f64(als + e * 8) : 0.0;
-    f[q] = valid ? lds_f64(fst + e * 8) : 0.0;
+    f[q] = valid ? (FT)lds_f64(fst + e * 8) : (FT)0;
     if (valid) {
       sts_f64(a0s + e * 8, al);
       vmask |= 1u << q;
@@ -678,26 +732,38 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   for (;;) {
     // Eq 4: u = argmin_{I_u} f; ties -> lowest position (== lowest pair-local index, R5)
     // the lane's minimum in FP64 compares (ties: lower row), one ord_key for the warp reduction
-    double uv[E];
+    FT uv[E];
     int uq[E];
 #pragma unroll
     for (int q = 0; q < E; ++q) {
-      uv[q] = ((umask >> q) & 1u) ? f[q] : CUDART_INF;
+      uv[q] = ((umask >> q) & 1u) ? f[q] : (FT)CUDART_INF;
       uq[q] = q;
     }
-    tree_min_f64<E>(uv, uq);
-    const bool uempty = uv[0] == CUDART_INF;  // f is finite: +inf marks "no I_u row in this lane"
-    const uint64_t uk0 = uempty ? ~0ull : ord_key(uv[0]);
-    const uint32_t h = (uint32_t)(uk0 >> 32), l = (uint32_t)uk0;
-    const uint32_t pos = uempty ? 0xffffffffu : (uint32_t)(lane + 32 * uq[0]);
-    const uint32_t m0 = __reduce_min_sync(FULLMASK, h);
-    const uint32_t m1 = __reduce_min_sync(FULLMASK, h == m0 ? l : 0xffffffffu);
-    const uint32_t ue32 = __reduce_min_sync(FULLMASK, (h == m0 && l == m1) ? pos : 0xffffffffu);
+    uint32_t ue32;
+    FT fu;
+    if constexpr (F32) {
+      tree_min_f32<E>(uv, uq);
+      const bool uempty = uv[0] == CUDART_INF_F;
+      const uint32_t k32 = uempty ? 0xffffffffu : ord_key_f32(uv[0]);
+      const uint32_t pos = uempty ? 0xffffffffu : (uint32_t)(lane + 32 * uq[0]);
+      const uint32_t m0 = __reduce_min_sync(FULLMASK, k32);
+      ue32 = __reduce_min_sync(FULLMASK, k32 == m0 ? pos : 0xffffffffu);
+      fu = key_f32(m0);
+    } else {
+      tree_min_f64<E>(uv, uq);
+      const bool uempty = uv[0] == CUDART_INF;  // f is finite: +inf marks "no I_u row in this lane"
+      const uint64_t uk0 = uempty ? ~0ull : ord_key(uv[0]);
+      const uint32_t h = (uint32_t)(uk0 >> 32), l = (uint32_t)uk0;
+      const uint32_t pos = uempty ? 0xffffffffu : (uint32_t)(lane + 32 * uq[0]);
+      const uint32_t m0 = __reduce_min_sync(FULLMASK, h);
+      const uint32_t m1 = __reduce_min_sync(FULLMASK, h == m0 ? l : 0xffffffffu);
+      ue32 = __reduce_min_sync(FULLMASK, (h == m0 && l == m1) ? pos : 0xffffffffu);
+      fu = (FT)key_double(((uint64_t)m0 << 32) | m1);
+    }
     if (ue32 == 0xffffffffu) break;  // I_u empty
     const int ue = (int)ue32;
     const int uq0 = ue >> 5, ul = ue & 31;
     const int yu = ((__shfl_sync(FULLMASK, ypos, ul) >> uq0) & 1u) ? 1 : -1;
-    const double fu = key_double(((uint64_t)m0 << 32) | m1);
     const uint32_t urow = kws + (uint32_t)(ue * ld) * 4;
     const double au = lds_f64(als + ue * 8);
     const float kuu = lds_f32(urow + ue * 4);
@@ -710,7 +776,7 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
     uint32_t sb[E];
     int sq[E];
     float st[E];
-    double lv[E];
+    FT lv[E];
 #pragma unroll
     for (int q = 0; q < E; ++q) {
       const bool il = (lmask >> q) & 1u;
@@ -721,19 +787,31 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
       st[q] = df * r;
       sb[q] = (il && f[q] > fu) ? __float_as_uint(df * st[q]) : 0u;  // scores >= 0: bits order as values
       sq[q] = q;
-      lv[q] = il ? f[q] : -CUDART_INF;
+      lv[q] = il ? f[q] : (FT)-CUDART_INF;
     }
     tree_max_u32<E>(sb, sq);
-    tree_max_f64<E>(lv);
-    const uint64_t lk0 = lv[0] == -CUDART_INF ? 0ull : ord_key(lv[0]);  // 0: no I_l row in this lane
-    const uint32_t xh = __reduce_max_sync(FULLMASK, (uint32_t)(lk0 >> 32));
-    const uint32_t xl = __reduce_max_sync(FULLMASK, (uint32_t)(lk0 >> 32) == xh ? (uint32_t)lk0 : 0u);
-    const uint32_t smax = __reduce_max_sync(FULLMASK, sb[0]);
-    const uint32_t lpos = (sb[0] != 0u && sb[0] == smax) ? (uint32_t)(lane + 32 * sq[0]) : 0xffffffffu;
-    const uint32_t le32 = __reduce_min_sync(FULLMASK, lpos);
+    double fmax;
+    uint32_t smax, le32;
+    if constexpr (F32) {
+      tree_max_f32<E>(lv);
+      const uint32_t lk = lv[0] == -CUDART_INF_F ? 0u : ord_key_f32(lv[0]);  // 0: no I_l row in this lane
+      const uint32_t xm = __reduce_max_sync(FULLMASK, lk);
+      smax = __reduce_max_sync(FULLMASK, sb[0]);
+      const uint32_t lpos = (sb[0] != 0u && sb[0] == smax) ? (uint32_t)(lane + 32 * sq[0]) : 0xffffffffu;
+      le32 = __reduce_min_sync(FULLMASK, lpos);
+      fmax = xm == 0u ? -DBL_MAX : (double)key_f32(xm);
+    } else {
+      tree_max_f64<E>(lv);
+      const uint64_t lk0 = lv[0] == -CUDART_INF ? 0ull : ord_key(lv[0]);  // 0: no I_l row in this lane
+      const uint32_t xh = __reduce_max_sync(FULLMASK, (uint32_t)(lk0 >> 32));
+      const uint32_t xl = __reduce_max_sync(FULLMASK, (uint32_t)(lk0 >> 32) == xh ? (uint32_t)lk0 : 0u);
+      smax = __reduce_max_sync(FULLMASK, sb[0]);
+      const uint32_t lpos = (sb[0] != 0u && sb[0] == smax) ? (uint32_t)(lane + 32 * sq[0]) : 0xffffffffu;
+      le32 = __reduce_min_sync(FULLMASK, lpos);
+      fmax = (xh == 0u && xl == 0u) ? -DBL_MAX : key_double(((uint64_t)xh << 32) | xl);
+    }
     markp(1);
-    const double fmax = (xh == 0u && xl == 0u) ? -DBL_MAX : key_double(((uint64_t)xh << 32) | xl);
-    const double gap = fmax - fu;
+    const double gap = fmax - (double)fu;
     if (it == 0) delta0 = gap;
     const double tol = eps > ratio * delta0 ? eps : ratio * delta0;
     if (!(gap >= tol) || le32 == 0xffffffffu || it >= cap) break;
@@ -768,7 +846,10 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
     const double nal = bnl ? (yl > 0 ? 0.0 : C) : alv - yl * s;
     // Eq 8 on the working set: f_i += s (K_ui - K_li)
 #pragma unroll
-    for (int q = 0; q < E; ++q) f[q] = fma(s, (double)(ku[q] - kl[q]), f[q]);
+    for (int q = 0; q < E; ++q) {
+      if constexpr (F32) f[q] = fmaf((float)s, ku[q] - kl[q], f[q]);
+      else f[q] = fma(s, (double)(ku[q] - kl[q]), f[q]);
+    }
     // membership of u and l after the step (owners update their bits; alpha in shared memory)
     const uint32_t uin = in_u(yu, nau, C) ? 1u : 0u, uil = in_l(yu, nau, C) ? 1u : 0u;
     const uint32_t lin = in_u(yl, nal, C) ? 1u : 0u, lil = in_l(yl, nal, C) ? 1u : 0u;
@@ -790,7 +871,7 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
     markp(3);
   }
   __syncwarp();
-  pdl_trigger();
+  if (pdl) pdl_trigger();
 #pragma unroll
   for (int q = 0; q < E; ++q) {
     const int e = lane + 32 * q;
@@ -813,6 +894,12 @@ __global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
   }
 }
 
+template <int E, bool PROF, typename FT = double>
+__global__ void __launch_bounds__(32, 1) ws_smo_kernel(SolverArgs a) {
+  extern __shared__ __align__(16) unsigned char mdyn[];
+  ws_smo_body<E, PROF, FT>(a, blockIdx.x + a.pair_base, mdyn, true);
+}
+
 // ------------------------------------------------------------------------------------------
 // a6: f update, f_j += sum_{i in ws, dalpha_i != 0} dalpha_i y_i K_ij over the pair (Alg 2 line 11,
 // Eq 8).  HBM-bound GEMV over the kernel-matrix rows of the working set: a CTA owns 32 column
@@ -830,39 +917,29 @@ struct WFup {
   int scan[33];
 };
 
-__global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraphConditionalHandle h, int set_cond) {
-  const int lp = blockIdx.x + a.pair_base;
-  const PairDesc pd = a.pairs[lp];  // constant for the solve: loaded before the dependency wait
-  pdl_enter();
-  TraceScope ts_(a, lp, 3);
+// columns [by * 128, +128) of pair lp's f-update by one kFT-thread CTA.  The working set, its
+// coefficients and f are read through L2 (the persistent solver's workers run beside the CTA that
+// wrote them); f of a column is updated by exactly one CTA.
+__device__ __forceinline__ void ws_fupdate_body(const SolverArgs& a, const int lp, const int by, WFup& F) {
+  const PairDesc pd = a.pairs[lp];
   const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
-  if (blockIdx.x == 0 && blockIdx.y == 0 && t == 0) {
-    bool more = false;
-    for (int i = 0; i < (int)gridDim.x; ++i) more = more || a.status[a.pair_base + i] == 0;
-    if (set_cond) {
-      cudaGraphSetConditional(h, more ? 1u : 0u);
-      a.body_iters[a.pair_base] += 1;
-    }
-  }
-  if (a.status[lp] != 0) return;
-  __shared__ WFup F;
   const int64_t q1b = pd.off_s >> 2, q1e = (pd.off_s + pd.n_s + 3) >> 2;
   const int64_t q2b = pd.off_t >> 2, q2e = (pd.off_t + pd.n_t + 3) >> 2;
   const int64_t nq1 = q1e - q1b, nq = nq1 + (q2e - q2b);
-  const int64_t q0 = (int64_t)blockIdx.y * 32;
+  const int64_t q0 = (int64_t)by * 32;
   if (q0 >= nq) return;
-  const int B = a.B, wn = a.ws_n[lp];
+  const int B = a.B, wn = __ldcg(a.ws_n + lp);
   const int32_t* ws = a.ws + (int64_t)lp * B;
   const double* dc = a.dcoef + (int64_t)lp * B;
   int nnz = 0;
   {
-    const double c = t < wn ? dc[t] : 0.0;
+    const double c = t < wn ? __ldcg(dc + t) : 0.0;
     const bool nz = c != 0.0;
     int tot = 0;
     const int pos = block_excl_scan(nz, tot, F.scan);
     if (nz) {
       F.coef[pos] = c;
-      F.rowp[pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, ws[t]) * a.ldk);
+      F.rowp[pos] = reinterpret_cast<const float4*>(a.K + gpos(pd, __ldcg(ws + t)) * a.ldk);
     }
     nnz = tot;
   }
@@ -910,10 +987,263 @@ __global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraph
         double sum = 0.0;
 #pragma unroll
         for (int w = 0; w < kFW; ++w) sum += F.red[w][l][c];
-        a.f[pd.a_off + j] += sum;
+        double* fp = a.f + pd.a_off + j;
+        __stcg(fp, __ldcg(fp) + sum);
       }
     }
   }
+}
+
+__global__ void __launch_bounds__(kFT) ws_fupdate_kernel(SolverArgs a, cudaGraphConditionalHandle h, int set_cond) {
+  const int lp = blockIdx.x + a.pair_base;
+  pdl_enter();
+  TraceScope ts_(a, lp, 3);
+  const int t = threadIdx.x;
+  if (blockIdx.x == 0 && blockIdx.y == 0 && t == 0) {
+    bool more = false;
+    for (int i = 0; i < (int)gridDim.x; ++i) more = more || a.status[a.pair_base + i] == 0;
+    if (set_cond) {
+      cudaGraphSetConditional(h, more ? 1u : 0u);
+      a.body_iters[a.pair_base] += 1;
+    }
+  }
+  if (a.status[lp] != 0) return;
+  __shared__ WFup F;
+  for (int ch = 0; ch < a.fu_chunks; ++ch) {  // GMPSVM_FU_CHUNKS (measured: 1 best)
+    if (ch > 0) __syncthreads();
+    ws_fupdate_body(a, lp, blockIdx.y * a.fu_chunks + ch, F);
+  }
+  if (a.trace && lp == a.trace_pair && t == 0) {  // GMPSVM_TRACE: latest CTA exit of the f-update
+    __threadfence();
+    atomicMax(trace_fu_end(a), (unsigned long long)gtimer());
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// Persistent solver: the outer loops of a group of pairs in two concurrent launches (Alg 2 lines
+// 6-11, the same four steps).  ws_lead_kernel: one CTA per pair runs the selection (whole CTA) and
+// the local SMO (warp 0) in its shared memory.  ws_work_kernel: small CTAs that take the gather
+// rows and f-update columns of every leader's iterations from a device task queue -- each task is
+// exactly one ws_gather_kernel / ws_fupdate_kernel CTA (same bodies, same summation order), so both
+// paths give bitwise the same alpha.  A leader publishes a phase's tasks and waits on its pair's
+// completion counter: each handoff is an L2 flag round trip instead of a kernel-grid completion
+// (~5 us each, four per outer iteration, measured with GMPSVM_TRACE fu_end_to_select).
+//
+// Residency: the worker grid is a programmatic dependent of the leader grid and every leader CTA
+// triggers it first thing, so the workers launch only once every leader is resident (one per SM
+// by its shared memory) and fill the SMs around them.  Every wait is bounded (kPTimeoutNs): a
+// stuck solve sets ctr[3] and the call fails with GMPSVM_ECUDA instead of hanging the GPU.
+struct PTask {  // one queue entry
+  int32_t kind, lp, chunk, pad;
+  unsigned long long seq;  // slot index + 1 once the entry is published
+  unsigned long long pad2;
+};
+enum { kTaskExit = 0, kTaskGather = 1, kTaskFup = 2 };
+constexpr int kPQueueCap = 1 << 15;
+constexpr unsigned long long kPTimeoutNs = 20000000000ull;  // 20 s per wait
+// ctr words: [0] head (next slot a worker takes), [1] tail (next slot a leader fills),
+// [2] leaders finished, [3] error, [8 + i] tasks completed for leader i
+constexpr int kPCtrPairs = 8;
+
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+
+// thread 0 of a leader: n tasks of one kind for leader slot li
+__device__ void p_push(PTask* ring, unsigned long long* ctr, int kind, int li, int n) {
+  const unsigned long long base = atomicAdd(&ctr[1], (unsigned long long)n);
+  for (int i = 0; i < n; ++i) {
+    PTask* e = ring + ((base + i) & (kPQueueCap - 1));
+    e->kind = kind;
+    e->lp = li;
+    e->chunk = i;
+    st_release_u64(&e->seq, base + i + 1);  // orders the fields before the sequence number
+  }
+}
+
+// whole leader CTA: publish n tasks, wait until the workers completed them (target: running count)
+__device__ bool p_run(const SolverArgs& a, int lp, PTask* ring, unsigned long long* ctr, int kind, int li, int n,
+                      unsigned long long& target, int* s_ok) {
+  __syncthreads();  // the CTA's global writes (selection output, local-solve result) precede the publish
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long t0 = gtimer();
+    target += (unsigned long long)n;
+    p_push(ring, ctr, kind, li, n);
+    int ok = 1;
+    while (ld_acquire_u64(&ctr[kPCtrPairs + li]) < target) {
+      if (gtimer() - t0 > kPTimeoutNs || ld_acquire_u64(&ctr[3]) != 0) {
+        atomicExch(&ctr[3], 1ull);
+        ok = 0;
+        break;
+      }
+    }
+    __threadfence();
+    fence_proxy_async();  // the workers' tile rows are read by the local solve's bulk copy
+    *s_ok = ok;
+    if (a.trace && lp == a.trace_pair)  // GMPSVM_TRACE: the phase from publish to completion
+      trace_rec(a, kind == kTaskGather ? 1 : 3, (int64_t)t0, (int64_t)gtimer());
+  }
+  __syncthreads();
+  return *s_ok != 0;
+}
+
+__host__ __device__ inline size_t ws_lead_w_off(int B) {
+  const size_t sel = (size_t)kWMaxNp * 9, smo = ws_buf_floats(B) * 4 + (size_t)B * 8 + 256;
+  return ((sel > smo ? sel : smo) + 127) & ~(size_t)127;
+}
+
+template <int E>
+__global__ void __launch_bounds__(kWT, 1)
+    ws_lead_kernel(SolverArgs a, int P, int nworkers, int64_t max_outer, PTask* ring, unsigned long long* ctr,
+                   const unsigned long long* res_ctr, int wait_resident) {
+  if (wait_resident > 0 && threadIdx.x == 0) {  // the kernel-value launch beside us holds its SMs first
+    const unsigned long long t0 = gtimer();
+    while (ld_acquire_u64(res_ctr) < (unsigned long long)wait_resident && gtimer() - t0 < kPTimeoutNs) __nanosleep(256);
+  }
+  __syncthreads();
+  pdl_trigger();  // the worker grid launches once every leader is resident
+  extern __shared__ __align__(128) unsigned char pdyn[];
+  WSelSmall& W = *reinterpret_cast<WSelSmall*>(pdyn + ws_lead_w_off(a.B));
+  __shared__ int s_ok;
+  const int t = threadIdx.x;
+  const int li = blockIdx.x, lp = a.pair_base + li;
+  const PairDesc pd = a.pairs[lp];
+  const int np = pd.n_s + pd.n_t;
+  const int64_t nq = ((pd.off_s + pd.n_s + 3) >> 2) - (pd.off_s >> 2) + ((pd.off_t + pd.n_t + 3) >> 2) - (pd.off_t >> 2);
+  const int n_fup = (int)((nq + 31) / 32);  // ws_fupdate_kernel CTAs with columns
+  unsigned long long target = 0;
+  for (;;) {
+    ws_select_body(a, lp, max_outer, pdyn, W, false);
+    fence_proxy_async();  // the working set's state is read by the local solve's bulk copy
+    __syncthreads();
+    if (a.status[lp] != 0) break;
+    if (!(np <= a.B && a.outer_iters[lp] != 1)) {  // the tile changed (ws_gather_kernel's test)
+      const int n_g = (a.ws_n[lp] + kGR - 1) / kGR;
+      if (!p_run(a, lp, ring, ctr, kTaskGather, li, n_g, target, &s_ok)) break;
+    }
+    if (t < 32) {
+      if (a.smo_f32) ws_smo_body<E, false, float>(a, lp, pdyn, false);
+      else ws_smo_body<E, false>(a, lp, pdyn, false);
+    }
+    if (!p_run(a, lp, ring, ctr, kTaskFup, li, n_fup, target, &s_ok)) break;
+  }
+  if (t == 0) {
+    __threadfence();
+    if (atomicAdd(&ctr[2], 1ull) == (unsigned long long)(P - 1)) p_push(ring, ctr, kTaskExit, 0, nworkers);
+  }
+}
+
+union PWork {  // worker shared memory
+  WFup F;
+  int64_t g[kWMaxB];
+};
+
+__global__ void __launch_bounds__(kFT) ws_work_kernel(SolverArgs a, PTask* ring, unsigned long long* ctr) {
+  __shared__ PWork w;
+  __shared__ int task[3];
+  const int t = threadIdx.x;
+  for (;;) {
+    if (t == 0) {
+      const unsigned long long idx = atomicAdd(&ctr[0], 1ull);
+      PTask* e = ring + (idx & (kPQueueCap - 1));
+      const unsigned long long t0 = gtimer();
+      int kind = kTaskExit, li = 0, ch = 0;
+      for (;;) {
+        if (ld_acquire_u64(&e->seq) == idx + 1) {
+          kind = e->kind;
+          li = e->lp;
+          ch = e->chunk;
+          break;
+        }
+        if (gtimer() - t0 > kPTimeoutNs) {
+          atomicExch(&ctr[3], 1ull);
+          break;
+        }
+        __nanosleep(32);
+      }
+      task[0] = kind;
+      task[1] = li;
+      task[2] = ch;
+    }
+    __syncthreads();
+    const int kind = task[0], li = task[1], ch = task[2];
+    if (kind == kTaskExit) return;
+    const bool tr = a.trace && a.pair_base + li == a.trace_pair && t == 0;
+    const int64_t tt0 = tr ? (int64_t)gtimer() : 0;
+    if (kind == kTaskGather) {
+      ws_gather_body(a, a.pair_base + li, ch, w.g);
+      fence_proxy_async();  // read by the leader's bulk copy (async proxy)
+    } else {
+      ws_fupdate_body(a, a.pair_base + li, ch, w.F);
+    }
+    __syncthreads();
+    if (t == 0) {
+      __threadfence();
+      atomicAdd(&ctr[kPCtrPairs + li], 1ull);
+    }
+    if (tr) trace_rec(a, kind == kTaskGather ? 9 : 10, tt0, (int64_t)gtimer());  // GMPSVM_TRACE: one task
+  }
+}
+
+size_t ws_persist_smem(int B) { return ws_lead_w_off(B) + sizeof(WSelSmall); }
+size_t ws_persist_ctr_words(int P) { return (size_t)kPCtrPairs + P; }
+size_t ws_persist_ring_bytes() { return sizeof(PTask) * kPQueueCap; }
+
+bool ws_persist_supported(int B, int64_t np_max) {
+  // opt-in (GMPSVM_PERSIST=1): measured slower on MNIST-shaped data
+  static const bool off = !(getenv("GMPSVM_PERSIST") && std::string(getenv("GMPSVM_PERSIST")) == "1");
+  int dev = 0, optin = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  return !off && ws_solve_supported(B, np_max) && ws_persist_smem(B) <= (size_t)optin;
+}
+
+int ws_persist_workers_per_sm() {
+  int nb = 0;
+  GM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, ws_work_kernel, kFT, 0));
+  return nb;
+}
+
+template <int E>
+static void launch_lead(const SolverArgs& a, int P, int nworkers, int64_t max_outer, PTask* ring,
+                        unsigned long long* ctr, cudaStream_t st, const unsigned long long* res_ctr, int wait_resident) {
+  const size_t smem = ws_persist_smem(a.B);
+  set_max_dyn_smem(ws_lead_kernel<E>, smem);
+  GM_LAUNCH(ws_lead_kernel<E>, dim3(P), dim3(kWT), smem, st, a, P, nworkers, max_outer, ring, ctr, res_ctr,
+            wait_resident);
+}
+
+void launch_ws_persist(const SolverArgs& a, int P, int nworkers, int64_t max_outer, void* ring_v,
+                       unsigned long long* ctr, cudaStream_t st, const unsigned long long* res_ctr, int wait_resident) {
+  PTask* ring = static_cast<PTask*>(ring_v);
+  switch ((a.B + 31) / 32) {
+    case 1: launch_lead<1>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+    case 2: launch_lead<2>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+    case 3: launch_lead<3>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+    case 4: launch_lead<4>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+    case 5: launch_lead<5>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+    case 6: launch_lead<6>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+    default: launch_lead<7>(a, P, nworkers, max_outer, ring, ctr, st, res_ctr, wait_resident); break;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(nworkers);
+  cfg.blockDim = dim3(kFT);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  GM_CUDA(cudaLaunchKernelEx(&cfg, ws_work_kernel, a, ring, ctr));
+  g_launches.fetch_add(1, std::memory_order_relaxed);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -954,11 +1284,18 @@ template <int E>
 static void smo_configure(int smem) {
   set_max_dyn_smem(ws_smo_kernel<E, false>, smem);
   set_max_dyn_smem(ws_smo_kernel<E, true>, smem);
+  set_max_dyn_smem(ws_smo_kernel<E, false, float>, smem);
+  set_max_dyn_smem(ws_smo_kernel<E, true, float>, smem);
 }
 template <int E>
 static void launch_smo(const SolverArgs& a, int P, size_t smem, cudaStream_t st) {
-  if (a.smo_phase) launch_pdl(ws_smo_kernel<E, true>, dim3(P), dim3(32), smem, st, a);
-  else launch_pdl(ws_smo_kernel<E, false>, dim3(P), dim3(32), smem, st, a);
+  if (a.smo_f32) {
+    if (a.smo_phase) launch_pdl(ws_smo_kernel<E, true, float>, dim3(P), dim3(32), smem, st, a);
+    else launch_pdl(ws_smo_kernel<E, false, float>, dim3(P), dim3(32), smem, st, a);
+  } else {
+    if (a.smo_phase) launch_pdl(ws_smo_kernel<E, true>, dim3(P), dim3(32), smem, st, a);
+    else launch_pdl(ws_smo_kernel<E, false>, dim3(P), dim3(32), smem, st, a);
+  }
 }
 
 static void ws_configure() {
@@ -1007,7 +1344,8 @@ void launch_ws_iteration(const SolverArgs& a, int P, int64_t np_max, cudaGraphCo
     case 6: launch_smo<6>(a, P, smo_dyn, st); break;
     default: launch_smo<7>(a, P, smo_dyn, st); break;
   }
-  launch_pdl(ws_fupdate_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, 128)), dim3(kFT), 0, st, a, h, set_cond);
+  launch_pdl(ws_fupdate_kernel, dim3(P, (unsigned)ceil_div(np_max + 8, 128 * a.fu_chunks)), dim3(kFT), 0, st, a, h,
+             set_cond);
 }
 
 }  // namespace gmpsvm

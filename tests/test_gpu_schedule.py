@@ -1,8 +1,9 @@
 """Scheduling of the training call must not change its result (engine.cu lead mode, cached solver
 graphs / arena / tile list).  Every pair's solve is a deterministic chain of kernels whatever the
 order the pairs run in, so the model is bitwise the same with lead mode off, with more lead pairs
-and groups, with the graph cache disabled, and when the cached graphs are reused or rebuilt after
-a call of another shape.  The default configuration itself is parity-tested against the oracle
+and groups, with the graph cache disabled, when the cached graphs are reused or rebuilt after
+a call of another shape, on the per-kernel graphs (default) or the persistent solver (opt-in), and
+with the kernel values from 2-CTA clusters (default) or single CTAs.  The default configuration itself is parity-tested against the oracle
 (test_gpu_parity.py, test_gpu_full.py).
 """
 import os
@@ -60,7 +61,10 @@ def test_schedule_does_not_change_the_model(tmp_path):
             np.testing.assert_array_equal(base[i + j], base[j])
     for tag, env in [("nolead", {"GMPSVM_LEAD": "0"}),
                      ("lead2_groups2", {"GMPSVM_LEAD": "2", "GMPSVM_GROUPS": "2", "GMPSVM_LEAD_RESERVE": "16"}),
-                     ("noreuse", {"GMPSVM_GRAPH_REUSE": "0"})]:
+                     ("noreuse", {"GMPSVM_GRAPH_REUSE": "0"}),
+                     ("krow_no_cluster", {"GMPSVM_KROW_MC": "0"}),
+                     ("persistent", {"GMPSVM_PERSIST": "1"}),
+                     ("persistent_nolead", {"GMPSVM_PERSIST": "1", "GMPSVM_LEAD": "0"})]:
         other = _run(tmp_path, tag, env)
         for a, b in zip(other, base):
             np.testing.assert_array_equal(a, b, err_msg=tag)
