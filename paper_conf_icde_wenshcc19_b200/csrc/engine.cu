@@ -1522,7 +1522,25 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   auto pq_ctr = [&](int g) {
     return reinterpret_cast<unsigned long long*>(d_pq.get() + pq_off[g] + ws_persist_ring_bytes());
   };
-  if (persist) {
+  // GMPSVM_NOGRAPH=1 (profiling only: ncu does not see the kernels of the conditional graphs): the
+  // same per-iteration kernels launched from the host on `st`, all pairs per launch, the host
+  // polling the pairs' status every 8 iterations -- the same arithmetic, far slower
+  static const bool nograph = getenv("GMPSVM_NOGRAPH") && std::string(getenv("GMPSVM_NOGRAPH")) == "1";
+  if (nograph && !persist && !rc && ws_solve_supported(Bw, np_max)) {
+    std::vector<int32_t> hst(Pl);
+    for (int g = 0; lead && g < ng; ++g) GM_CUDA(cudaStreamWaitEvent(st, ev_wave[g], 0));
+    for (int64_t it = 0;; ++it) {
+      launch_ws_iteration(a, Pl, np_max, cudaGraphConditionalHandle{}, 0, max_outer, st, false);
+      if (it % 8 == 7) {
+        GM_CUDA(cudaMemcpyAsync(hst.data(), d_status.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
+        GM_CUDA(cudaStreamSynchronize(st));
+        bool more = false;
+        for (int i = 0; i < Pl; ++i) more = more || hst[i] == 0;
+        if (!more) break;
+      }
+    }
+    n_branches = 1;
+  } else if (persist) {
     GM_CUDA(cudaEventRecord(ev_ready, st));
     for (int g = 0; g < ng; ++g) {
       cudaStream_t ls = pool[g];

@@ -506,19 +506,24 @@ __device__ __forceinline__ void ws_gather_body(const SolverArgs& a, const int lp
   const int ld = ws_tile_ld(a.B);
   float* tile = a.Kws + (int64_t)lp * ws_buf_floats(a.B);
   const int r1 = min(wn, r0 + kGR);
+  // K is stored symmetric (both triangles, the same values): the tile's upper triangle is loaded
+  // and written to both positions -- half the scattered loads (each one a DRAM burst of its own)
   constexpr int M = (kGR * kWMaxB + 255) / 256;  // loads per thread, all in flight
   float v[M];
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int q = threadIdx.x + m * 256;
     const int r = r0 + q / wn, c = q % wn;
-    v[m] = r < r1 ? __ldg(a.K + g[r] * a.ldk + g[c]) : 0.f;
+    v[m] = (r < r1 && c >= r) ? __ldg(a.K + g[r] * a.ldk + g[c]) : 0.f;
   }
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int q = threadIdx.x + m * 256;
     const int r = r0 + q / wn, c = q % wn;
-    if (r < r1) tile[(int64_t)r * ld + c] = v[m];
+    if (r < r1 && c >= r) {
+      tile[(int64_t)r * ld + c] = v[m];
+      tile[(int64_t)c * ld + r] = v[m];
+    }
   }
 }
 
