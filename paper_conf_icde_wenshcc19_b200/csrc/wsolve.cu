@@ -58,38 +58,52 @@ __device__ __forceinline__ void pdl_enter() {
 struct WSelSmall {
   uint32_t retained[kWMaxNp / 32];  // retained rows; then the write-out bitmap
   double red[2][32];
-  uint64_t sk[2][kWRank];  // the warps' 4 smallest per-thread minima
-  int32_t si[2][kWRank];
+  uint64_t sk[2][kWRank];  // the warps' 4 smallest per-thread minima (candidate keys, below)
   uint64_t bk[2][32][kBufW];  // per-warp candidates <= threshold
-  int32_t bi[2][32][kBufW];
   int32_t bcnt[2][32];
   int32_t boff[2][33];
   uint64_t fk[2][kFlat];  // flattened candidate lists
-  int32_t fi[2][kFlat];
   int32_t pick[1024];  // new working set in age order
   int32_t wpre[kWMaxNp / 32];  // prefix popcounts of the picked-index bitmap
   uint64_t thr_k[2];
-  int32_t thr_i[2];
   int32_t overflow;
   SelSmem sel;  // radix_pick fallback
 };
 
-__device__ __forceinline__ bool kless(uint64_t ka, int32_t ia, uint64_t kb, int32_t ib) {
-  return ka < kb || (ka == kb && ia < ib);
-}
+// Candidate keys: the order-preserving key of f (I_u side) or of -f (I_l side) with its low 14 bits
+// replaced by the pair-local index (n_p <= kWMaxNp = 2^14), so one 64-bit compare orders the
+// candidates by value and then by index (R19 / R5: smallest f first, lowest index on ties).
+// Values closer than 2^-38 relative count as equal and go by index.
+constexpr uint64_t kIdxBits = 14, kIdxMask = (1ull << kIdxBits) - 1;
+static_assert(kWMaxNp <= (1 << kIdxBits), "the index must fit the key's low bits");
+__device__ __forceinline__ uint64_t ckey_u(double f, int i) { return (ord_key(f) & ~kIdxMask) | (uint64_t)i; }
+__device__ __forceinline__ uint64_t ckey_l_of_u(uint64_t ku) { return (~ku & ~kIdxMask) | (ku & kIdxMask); }
+__device__ __forceinline__ int ckey_idx(uint64_t k) { return (int)(k & kIdxMask); }
 
-// lexicographic warp min of (key64, idx); all lanes get the winner's (k, i); returns its lane
-__device__ __forceinline__ int warp_min_ki(uint64_t& k, int32_t& i) {
+// warp min of distinct keys (~0: none); all lanes get it; returns the winner's lane (-1: none)
+__device__ __forceinline__ int warp_min_k(uint64_t& k) {
   const uint32_t h = (uint32_t)(k >> 32), l = (uint32_t)k;
   const uint32_t m0 = __reduce_min_sync(FULLMASK, h);
   const uint32_t m1 = __reduce_min_sync(FULLMASK, h == m0 ? l : 0xffffffffu);
-  const bool tie = h == m0 && l == m1;
-  const uint32_t m2 = __reduce_min_sync(FULLMASK, tie ? (uint32_t)i : 0xffffffffu);
-  const unsigned b = __ballot_sync(FULLMASK, tie && (uint32_t)i == m2);
-  k = ((uint64_t)m0 << 32) | m1;
-  i = (int32_t)m2;
+  const uint64_t m = ((uint64_t)m0 << 32) | m1;
+  const unsigned b = __ballot_sync(FULLMASK, k == m && m != ~0ull);
+  k = m;
   return __ffs(b) - 1;
 }
+
+// radix_pick's view of the combined keys (its `~key` for the I_l side inverts only the value bits)
+struct SmemSrcCK {
+  const uint64_t* keys;
+  uint8_t* flags;  // bit0 in I_u, bit1 in I_l, bit2 taken / retained
+  template <bool SIDE_U>
+  __device__ __forceinline__ bool cand(int i, uint64_t& key) const {
+    const uint8_t fl = flags[i];
+    if (!(fl & (SIDE_U ? 1 : 2)) || (fl & 4)) return false;
+    key = SIDE_U ? keys[i] : ckey_l_of_u(keys[i]);
+    return true;
+  }
+  __device__ __forceinline__ void take(int i) const { flags[i] |= 4; }
+};
 
 // Threads per list entry for a rank count over n entries by the whole CTA: the largest power of
 // two g <= 32 with n * g <= kWT (g lanes of one warp share an entry and split its comparisons).
@@ -247,7 +261,6 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
   // stage keys / flags, stop test (Eq 9-10), per-thread minima of the candidates of both sides
   double fmin = DBL_MAX, fmax = -DBL_MAX;
   uint64_t mk[2] = {~0ull, ~0ull};
-  int32_t mi[2] = {INT_MAX, INT_MAX};
   for (int base = 0; base < np; base += kStageUnroll * kWT) {
     double av[kStageUnroll], fv[kStageUnroll];
 #pragma unroll
@@ -265,17 +278,11 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
         const bool ret = (W.retained[i >> 5] >> (i & 31)) & 1u;
         if (u) fmin = fmin < fv[m] ? fmin : fv[m];
         if (l) fmax = fmax > fv[m] ? fmax : fv[m];
-        const uint64_t key = ord_key(fv[m]);
+        const uint64_t key = ckey_u(fv[m], i), lkey = ckey_l_of_u(key);
         keys[i] = key;
         flags[i] = (uint8_t)((u ? 1 : 0) | (l ? 2 : 0) | (ret ? 4 : 0));
-        if (u && !ret && key < mk[0]) {  // ascending i: strict < keeps the lowest index
-          mk[0] = key;
-          mi[0] = i;
-        }
-        if (l && !ret && ~key < mk[1]) {
-          mk[1] = ~key;
-          mi[1] = i;
-        }
+        if (u && !ret && key < mk[0]) mk[0] = key;
+        if (l && !ret && lkey < mk[1]) mk[1] = lkey;
       }
     }
   }
@@ -320,22 +327,12 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
 #pragma unroll
     for (int s = 0; s < 2; ++s) {
       uint64_t k = mk[s];
-      int32_t x = mi[s];
-      const int wl = warp_min_ki(k, x);
-      if (lane == 0) {
-        W.sk[s][warp * 4 + j] = k;
-        W.si[s][warp * 4 + j] = x;
-      }
-      if (lane == wl) {
-        mk[s] = ~0ull;
-        mi[s] = INT_MAX;
-      }
+      const int wl = warp_min_k(k);
+      if (lane == 0) W.sk[s][warp * 4 + j] = k;
+      if (lane == wl) mk[s] = ~0ull;
     }
   }
-  if (t < 2) {
-    W.thr_k[t] = ~0ull;  // fewer samples than the rank: every candidate qualifies
-    W.thr_i[t] = INT_MAX;
-  }
+  if (t < 2) W.thr_k[t] = ~0ull;  // fewer samples than the rank: every candidate qualifies
   __syncthreads();
   // thresholds by counting ranks: U at rank need_u - 1, L at rank need - 1 (so the L list
   // still holds need - (U picks) candidates after removing the U picks it shares); 4 threads per
@@ -346,19 +343,12 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
     const int s = e / kWRank, j = e % kWRank;
     const int r = s == 0 ? need_u : need;
     const uint64_t k = W.sk[s][j];
-    const int32_t x = W.si[s][j];
     int rank = 0;
-    for (int q = sub; q < kWRank; q += G) rank += kless(W.sk[s][q], W.si[s][q], k, x) ? 1 : 0;
+    for (int q = sub; q < kWRank; q += G) rank += W.sk[s][q] < k ? 1 : 0;
     rank = group_sum(rank, G);
     if (sub == 0) {
-      if (x != INT_MAX && r >= 1 && r <= kWRank && rank == r - 1) {
-        W.thr_k[s] = k;
-        W.thr_i[s] = x;
-      }
-      if (s == 0 && j == 0 && r == 0) {  // nothing wanted from U
-        W.thr_k[0] = 0ull;
-        W.thr_i[0] = -1;
-      }
+      if (k != ~0ull && r >= 1 && r <= kWRank && rank == r - 1) W.thr_k[s] = k;
+      if (s == 0 && j == 0 && r == 0) W.thr_k[0] = 0ull;  // nothing wanted from U (no key is 0)
     }
   }
   __syncthreads();
@@ -366,28 +356,22 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
   // compaction of the candidates at or below the thresholds into per-warp buffers
   {
     const uint64_t tk0 = W.thr_k[0], tk1 = W.thr_k[1];
-    const int32_t ti0 = W.thr_i[0], ti1 = W.thr_i[1];
     int c0 = 0, c1 = 0;
     for (int base = 0; base < np; base += kWT) {
       const int i = base + t;
       bool cu = false, cl = false;
-      uint64_t kk = 0;
+      uint64_t kk = 0, lk = 0;
       if (i < np) {
         const uint8_t fg = flags[i];
         kk = keys[i];
-        cu = (fg & 5) == 1 && !kless(tk0, ti0, kk, i);
-        cl = (fg & 6) == 2 && !kless(tk1, ti1, ~kk, i);
+        lk = ckey_l_of_u(kk);
+        cu = (fg & 5) == 1 && kk <= tk0;
+        cl = (fg & 6) == 2 && lk <= tk1;
       }
       const unsigned bu = __ballot_sync(FULLMASK, cu), bl = __ballot_sync(FULLMASK, cl);
       const int ou = c0 + __popc(bu & ((1u << lane) - 1u)), ol = c1 + __popc(bl & ((1u << lane) - 1u));
-      if (cu && ou < kBufW) {
-        W.bk[0][warp][ou] = kk;
-        W.bi[0][warp][ou] = i;
-      }
-      if (cl && ol < kBufW) {
-        W.bk[1][warp][ol] = ~kk;
-        W.bi[1][warp][ol] = i;
-      }
+      if (cu && ou < kBufW) W.bk[0][warp][ou] = kk;
+      if (cl && ol < kBufW) W.bk[1][warp][ol] = lk;
       c0 += __popc(bu);
       c1 += __popc(bl);
     }
@@ -418,11 +402,7 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
   if (!W.overflow) {
     {  // flatten: thread (warp w, lane j) copies slot j of warp w's U (j < 16) or L (j >= 16) buffer
       const int s = lane >> 4, j = lane & 15;
-      if (j < W.bcnt[s][warp]) {
-        const int o = W.boff[s][warp] + j;
-        W.fk[s][o] = W.bk[s][warp][j];
-        W.fi[s][o] = W.bi[s][warp][j];
-      }
+      if (j < W.bcnt[s][warp]) W.fk[s][W.boff[s][warp] + j] = W.bk[s][warp][j];
     }
     __syncthreads();
     const int nu = W.boff[0][32], nl = W.boff[1][32];
@@ -431,15 +411,14 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
     {
       const int g = rank_group(nu), e = t / g, sub = t % g;
       uint64_t k = 0;
-      int32_t x = 0;
       int rank = 0;
       if (e < nu) {
         k = W.fk[0][e];
-        x = W.fi[0][e];
-        for (int q = sub; q < nu; q += g) rank += kless(W.fk[0][q], W.fi[0][q], k, x) ? 1 : 0;
+        for (int q = sub; q < nu; q += g) rank += W.fk[0][q] < k ? 1 : 0;
       }
       rank = group_sum(rank, g);
       if (e < nu && sub == 0 && rank < got_u) {
+        const int x = ckey_idx(k);
         W.pick[keep + rank] = x;
         flags[x] |= 4;
       }
@@ -454,12 +433,12 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
       int32_t x = 0;
       if (e < nl) {
         const uint64_t k = W.fk[1][e];
-        x = W.fi[1][e];
+        x = ckey_idx(k);
         free_l = !(flags[x] & 4);
         if (free_l)
           for (int q = sub; q < nl; q += g) {
-            const int32_t xq = W.fi[1][q];
-            rank += (!(flags[xq] & 4) && kless(W.fk[1][q], xq, k, x)) ? 1 : 0;
+            const uint64_t kq = W.fk[1][q];
+            rank += (kq < k && !(flags[ckey_idx(kq)] & 4)) ? 1 : 0;
           }
       }
       rank = group_sum(rank, g);
@@ -471,9 +450,9 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
     for (int e = keep + got_u + t; e < keep + got; e += kWT) flags[W.pick[e]] |= 4;
     __syncthreads();
     // L ran short (every L candidate is in the list): U again, as select_sides does
-    if (got < need) got += radix_pick<true>(SmemSrc{keys, flags}, np, need - got, W.pick + keep + got, W.sel);
+    if (got < need) got += radix_pick<true>(SmemSrcCK{keys, flags}, np, need - got, W.pick + keep + got, W.sel);
   } else {  // a buffer overflowed (heavily tied or clustered keys): exact radix selection
-    got = select_sides(SmemSrc{keys, flags}, np, need, W.pick + keep, W.sel);
+    got = select_sides(SmemSrcCK{keys, flags}, np, need, W.pick + keep, W.sel);
     if (a.sel_phase && t == 0) a.sel_phase[(int64_t)(lp + 4096) * 5 + 4] += 1000000;  // fallbacks (diagnostic)
   }
   __syncthreads();
