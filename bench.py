@@ -321,6 +321,11 @@ def run_gpu(args, spec):
         split = "tf32" if os.environ.get("GMPSVM_SPLIT", "") == "tf32" else "f16"
         mma_peak = bf16 * (0.5 if split == "tf32" else 1.0)
         peak = mma_peak / 3.0
+        # lead mode: the contraction's main wave runs on all but the reserved SMs (the hardest pair's
+        # solver holds those); frac_of_launch_sms scales the peak to the SMs the launch was given
+        n_sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        lead_on = os.environ.get("GMPSVM_LEAD", "1") != "0"
+        launch_sms = n_sms - (int(os.environ.get("GMPSVM_LEAD_RESERVE", "8")) if lead_on else 0)
         traffic = None
         tr_path = os.path.join(ROOT, "profiles", "krow_traffic.json")
         if os.path.exists(tr_path):
@@ -338,6 +343,8 @@ def run_gpu(args, spec):
                                        f"{' x 0.5' if split == 'tf32' else ''} = {mma_peak:.1f} TFLOP/s"
                                        f"{'' if 'bf16_tflops' in peaks else ' (fallback)'}; the hi/lo split needs 3 MMAs "
                                        "per FP32-accurate product, so peak = that / 3"),
+                         "frac_of_launch_sms": achieved / (peak * launch_sms / n_sms),
+                         "launch_sms": launch_sms,
                          "frac_of_mma_peak": achieved / mma_peak,
                          "frac_of_fp32_simt_peak": achieved / _fp32_peak(),
                          "fp32_simt_peak": _fp32_peak(),
