@@ -1496,6 +1496,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   int64_t body_launches = 0;
   std::vector<int64_t> body_per_pair(Pl, 0);  // kernels per loop-body run of the pair's branch
   int n_branches = 0, final_selects = 0;
+  bool fin_in_graph = false;  // finalize + sigmoid fit captured at the end of each graph branch
   // Persistent solver (default where it applies: FULL_K, every pair on the wsolve.cu kernels, at
   // most two pair groups): one launch per group -- its pairs' leaders plus workers on the SMs the
   // group may use (lead mode: the lead group on the `reserve` SMs beside the kernel-value waves,
@@ -1622,12 +1623,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         GM_CUDA(cudaStreamEndCapture(cs, &cap));
         body_launches = (int64_t)(g_launches.load() - b0);
         body_per_pair[i] = body_launches;
-        if (!wsp) {  // the stop test on the final alpha (the default path tests in every f-update)
-          GM_CUDA(cudaStreamBeginCaptureToGraph(cs, g.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
+        // after the loop, in the branch: the stop test on the final alpha (split path; the default
+        // path tests in every f-update), then the branch's bias / in-sample values (a7) and sigmoid
+        // fits (a8) -- they overlap the pairs still iterating instead of following the last one
+        GM_CUDA(cudaStreamBeginCaptureToGraph(cs, g.graph, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
+        if (!wsp) {
           launch_select_ws(ag, gn, 0, -1, cs);
-          GM_CUDA(cudaStreamEndCapture(cs, &cap));
           ++final_selects;
         }
+        launch_finalize(ag, gn, cs);
+        launch_sigmoid_fit(ag, gn, cs);
+        final_selects += 2;  // counted with the final selections: one run per graph launch
+        GM_CUDA(cudaStreamEndCapture(cs, &cap));
       }
       g_launches.fetch_sub(g_launches.load() - l0);  // captured, not executed: counted after the run
       GM_CUDA(cudaGraphInstantiate(&g.exec, g.graph, 0));
@@ -1695,6 +1702,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     }
     HT("graph_build");
     n_branches = nbr;
+    fin_in_graph = true;
     // graphs no call will launch again (uncached calls, replaced cached ones): destroying one
     // blocks the host until the device is idle, so it is done here, behind the running solver
     destroy_parked_graphs();
@@ -1712,8 +1720,10 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     GM_CUDA(cudaStreamSynchronize(st));
     HT("solver_wait");
   }
-  launch_finalize(a, Pl, st);
-  launch_sigmoid_fit(a, Pl, st);
+  if (!fin_in_graph) {  // the graph path ran them per branch
+    launch_finalize(a, Pl, st);
+    launch_sigmoid_fit(a, Pl, st);
+  }
   DevBuf<uint8_t> d_flags(n, st);
   GM_CUDA(cudaMemsetAsync(d_flags.get(), 0, n, st));
   launch_sv_flags(a, Pl, np_max, d_flags.get(), st);
