@@ -185,7 +185,7 @@ def _config(spec, args):
     return {"workload": f"{spec.name}-shaped {spec.n_train} train / {spec.n_test} test x {spec.d}, k={spec.k}, "
                         f"C={spec.C:g}, gamma={spec.gamma:g}, eps={args.eps:g}",
             "n_train": spec.n_train, "n_test": spec.n_test, "d": spec.d, "k": spec.k, "C": spec.C,
-            "gamma": spec.gamma, "eps": args.eps, "ws_size": args.ws_size, "q": args.ws_size // 2,
+            "gamma": spec.gamma, "eps": args.eps, "ws_size": args.ws_size, "q": args.q or args.ws_size // 2,
             "parallelism": f"pairs+test-rows x{args.gpus}",
             "l2": "inputs larger than L2 (X 188 MB, kernel matrix 14.4 GB > 126 MB L2); no flush needed"}
 
@@ -211,7 +211,7 @@ def run_gpu(args, spec):
     Xp, yp, Xtp = (torch.from_numpy(X).pin_memory(), torch.from_numpy(y).pin_memory(),
                    torch.from_numpy(Xt).pin_memory())
     stream = torch.cuda.current_stream(dev)
-    opts = dict(ws_size=args.ws_size)
+    opts = dict(ws_size=args.ws_size, q=args.q)
 
     host_ms = []  # host-clock duration of each step's calls (diagnostic: stalls outside the GPU)
 
@@ -413,6 +413,7 @@ def main():
     ap.add_argument("--config", default="mnist")
     ap.add_argument("--eps", type=float, default=1e-3)
     ap.add_argument("--ws-size", dest="ws_size", type=int, default=192)
+    ap.add_argument("--q", type=int, default=0, help="new working-set rows per outer iteration (0: ws_size / 2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
