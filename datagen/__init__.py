@@ -12,6 +12,8 @@ PAPER.md Table 2 (L381-L387) and BASELINE.json `configs`:
   mnist    10 classes, 60k/10k x 784, gamma=0.125, C=10 (config 3, Table 2)
   covtype  7 classes, 581,012 x 54, gamma=1, C=3    (config 4)
   mnist8m  10 classes, 8.1M x 784, gamma=0.006, C=1000 (config 5, Table 2)
+  news20   4 classes, 3k/600 x 5000 sparse text-like rows (~1.2 % non-zero), gamma=0.5, C=10
+           (NEXT-3: the CSR path; shaped like the paper's News20 / RCV1 sparse inputs, L479, L513)
 
 Every array is float32 features (row-major n x d) and int32 labels in [0, k).
 """
@@ -44,6 +46,7 @@ CONFIGS = {
     "mnist": ConfigSpec("mnist", 10, 784, 60_000, 10_000, 0.125, 10.0, 1234, 1, 2),
     "covtype": ConfigSpec("covtype", 7, 54, 581_012, 58_101, 1.0, 3.0, 4242, 1, 2),
     "mnist8m": ConfigSpec("mnist8m", 10, 784, 8_100_000, 10_000, 0.006, 1000.0, 1234, 3, 2),
+    "news20": ConfigSpec("news20", 4, 5000, 3_000, 600, 0.5, 10.0, 2020, 1, 2),
 }
 
 _CHUNK = 100_000  # rows generated per child stream for the big configs
@@ -165,7 +168,31 @@ def _covtype(spec: ConfigSpec, split: str, n: int):
     return X, y.astype(np.int32)
 
 
-_GEN = {"blobs": _blobs, "letter": _letter, "mnist": _mnist, "mnist8m": _mnist, "covtype": _covtype}
+# ----------------------------------------------------------------------------------------
+# news20 (sparse, text-like): a Zipf word distribution over d words; each class prefers its own
+# 250 topic words.  A document has 30 + Poisson(30) word draws, half from its class's topic words,
+# half from the Zipf distribution; value = log(1 + count), rows scaled to unit L2 norm.
+# ----------------------------------------------------------------------------------------
+def _news20(spec: ConfigSpec, split: str, n: int):
+    srng = np.random.default_rng(spec.structure_seed)
+    zipf = 1.0 / np.arange(1, spec.d + 1) ** 1.1
+    zipf /= zipf.sum()
+    topics = np.stack([srng.choice(spec.d, size=250, replace=False) for _ in range(spec.k)])
+    rng = np.random.default_rng(spec.train_seed if split == "train" else spec.test_seed)
+    y = rng.integers(0, spec.k, size=n)
+    X = np.zeros((n, spec.d), dtype=np.float32)
+    for i in range(n):
+        m = 30 + rng.poisson(30)
+        h = m // 2
+        words = np.concatenate([topics[y[i]][rng.integers(0, 250, size=h)], rng.choice(spec.d, size=m - h, p=zipf)])
+        idx, cnt = np.unique(words, return_counts=True)
+        v = np.log1p(cnt.astype(np.float64))
+        X[i, idx] = (v / np.linalg.norm(v)).astype(np.float32)
+    return X, y.astype(np.int32)
+
+
+_GEN = {"blobs": _blobs, "letter": _letter, "mnist": _mnist, "mnist8m": _mnist, "covtype": _covtype,
+        "news20": _news20}
 
 
 def make_split(name: str, split: str, n: int | None = None):

@@ -122,7 +122,8 @@ typedef struct {
   double t_solver_ms;       /* a3-a6 as a whole: pairs run on concurrent streams, so select,  */
                             /* subproblem and f-update overlap (their own fields then stay 0)  */
   int32_t n_streams;        /* concurrent branches of the solver graph (pairs packed into them) */
-  int32_t pad0;
+  int32_t kernel_path;      /* kernel values from: 0 dense rows on tcgen05, 1 dense rows on the FP32
+                               SIMT contraction, 2 CSR rows (sparse x dense, NEXT-3, L299 / L513) */
 } gmpsvm_train_stats;
 
 typedef struct {

@@ -43,7 +43,7 @@ class TrainStats(ct.Structure):
                 ("krow_launches", ct.c_int64), ("outer_iters_max", ct.c_int64), ("outer_iters_sum", ct.c_int64),
                 ("inner_iters_sum", ct.c_int64), ("n_sv", ct.c_int64), ("cache_regime", ct.c_int32),
                 ("n_pairs_trained", ct.c_int32), ("launches", ct.c_int64), ("smo_cycles_sum", ct.c_int64),
-                ("t_solver_ms", ct.c_double), ("n_streams", ct.c_int32), ("pad0", ct.c_int32)]
+                ("t_solver_ms", ct.c_double), ("n_streams", ct.c_int32), ("kernel_path", ct.c_int32)]
 
 
 class PredictStats(ct.Structure):

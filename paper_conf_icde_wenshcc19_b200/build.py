@@ -21,7 +21,8 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
          "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC]
 FLAGS += os.environ.get("GMPSVM_NVCC_EXTRA", "").split()  # experiments only (e.g. -DGMPSVM_STAGE_UNROLL=8)
-SOURCES = ["stage.cu", "krow.cu", "krow_tc.cu", "solver.cu", "wsolve.cu", "predict.cu", "dec_i8.cu", "shard.cu", "engine.cu", "api.cpp"]
+SOURCES = ["stage.cu", "krow.cu", "krow_tc.cu", "solver.cu", "wsolve.cu", "predict.cu", "dec_i8.cu", "shard.cu", "csr.cu",
+           "engine.cu", "api.cpp"]
 
 
 def _newest_input():

@@ -796,7 +796,7 @@ void ensure_host_alpha(const Model& mdl) {
 
 // ------------------------------------------------------------------------------------------
 static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
-                             double eps, const gmpsvm_options& opt, Model** out);
+                             double eps, const gmpsvm_options& opt, Model** out, const CsrSrc* csr = nullptr);
 
 // NEXT-2, LibSVM's probability training (ref [15]; the paper fits on in-sample values, R10):
 // F-fold cross-validated decision values.  Fold of instance i = (its rank within its class,
@@ -927,7 +927,7 @@ int engine_train(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t
 }
 
 static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_t d, int32_t k, double C, double gamma,
-                             double eps, const gmpsvm_options& opt, Model** out) {
+                             double eps, const gmpsvm_options& opt, Model** out, const CsrSrc* csr) {
   const auto t_start = std::chrono::steady_clock::now();
   // GMPSVM_HOST_TIMING=1: host-clock checkpoints of the training call on stderr
   static const bool host_timing = getenv("GMPSVM_HOST_TIMING") != nullptr;
@@ -940,7 +940,9 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
                std::to_string(std::chrono::duration<double, std::milli>(now - t_last).count()).substr(0, 6);
     t_last = now;
   };
-  if (!X || !y || !out) throw Error(GMPSVM_EINVAL, "null argument");
+  if ((!X && !csr) || !y || !out) throw Error(GMPSVM_EINVAL, "null argument");
+  if (csr && (!opt.inputs_on_device || opt.kernel != 0 || opt.prob_folds != 0))
+    throw Error(GMPSVM_ENOTIMPL, "sparse kernel values: device CSR rows, the Gaussian kernel, no CV sigmoids");
   if (n < 2 || d < 1 || k < 2) throw Error(GMPSVM_EINVAL, "need n >= 2, d >= 1, k >= 2");
   if (k > kMaxK) throw Error(GMPSVM_ENOTIMPL, "k > 64 classes not supported by this build");
   if (n >= (int64_t)1 << 31) throw Error(GMPSVM_ENOTIMPL, "n >= 2^31 not supported");
@@ -995,9 +997,10 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   // tens of milliseconds, so it is not queried per call)
   const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * (double)device_total_mem(opt.device);
   const bool full_k = bytes_K <= budget;
+  if (csr && !full_k) throw Error(GMPSVM_ENOTIMPL, "sparse kernel values: the n x n kernel matrix must fit (FULL_K)");
   // tensor cores for the kernel values: FULL_K always; ROW_CACHE rows for the Gaussian with the
   // FP16 split (rows_tc_kernel); the SIMT contraction otherwise (GMPSVM_KROW=simt)
-  const bool use_tc = krow_use_tc() && (full_k || (ktype == 0 && krow_split_f16()));
+  const bool use_tc = !csr && krow_use_tc() && (full_k || (ktype == 0 && krow_split_f16()));
   if (ktype != 0 && !(use_tc && krow_split_f16()))
     throw Error(GMPSVM_ENOTIMPL, "the linear / polynomial / sigmoid kernels need the FULL_K regime on the tensor cores");
   const int d_pad = use_tc ? krow_tc_d_pad(d) : (int)round_up(d, kBK);
@@ -1005,7 +1008,11 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile) + (full_k ? 0 : kTile);
   // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split.
   // norms: + one tile of zeros (ROW_CACHE column tiles run up to 127 columns past n)
-  DevBuf<float> XT(use_tc ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad + kTile, st);
+  DevBuf<float> XT(use_tc || csr ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad + kTile, st);
+  // NEXT-3: class-sorted CSR rows (sptr on the host from the input row pointers and the order)
+  DevBuf<int64_t> c_ptr(csr ? (size_t)n + 1 : 0, st);
+  DevBuf<int32_t> c_idx(csr ? (size_t)std::max<int64_t>(csr->nnz, 1) : 0, st);
+  DevBuf<float> c_val(csr ? (size_t)std::max<int64_t>(csr->nnz, 1) : 0, st);
   GM_CUDA(cudaMemsetAsync(norms.get() + n_pad, 0, kTile * sizeof(float), st));
   DevBuf<float> Xhi(use_tc ? krow_tc_buf_floats(n_pad, d_pad) : 0, st), Xlo(use_tc ? krow_tc_buf_floats(n_pad, d_pad) : 0, st);
   float ksc = 1.f;  // scale of the split (FP16: exact power of two)
@@ -1016,6 +1023,20 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     launch_row_norms(dX, n, d, d_perm.get(), norms.get(), n_pad, bad.get(), st);  // validation (non-finite rows)
     ksc = launch_split_hilo(dX, n, d, d_perm.get(), Xhi.get(), Xlo.get(), norms.get(), n_pad, d_pad, tc_scratch.get(), st,
                             ktype == 0);
+  } else if (csr) {
+    std::vector<int64_t> hptr((size_t)n + 1), hperm(n), sptr((size_t)n + 1, 0);
+    GM_CUDA(cudaMemcpyAsync(hptr.data(), csr->indptr, ((size_t)n + 1) * 8, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaMemcpyAsync(hperm.data(), d_perm.get(), (size_t)n * 8, cudaMemcpyDeviceToHost, st));
+    GM_CUDA(cudaStreamSynchronize(st));
+    for (int64_t i = 0; i < n; ++i) {
+      const int64_t len = hptr[hperm[i] + 1] - hptr[hperm[i]];
+      if (len < 0) throw Error(GMPSVM_EINVAL, "CSR row pointers must be non-decreasing");
+      sptr[i + 1] = sptr[i] + len;
+    }
+    if (sptr[n] != csr->nnz) throw Error(GMPSVM_EINVAL, "CSR row pointers do not match nnz");
+    GM_CUDA(cudaMemcpyAsync(c_ptr.get(), sptr.data(), ((size_t)n + 1) * 8, cudaMemcpyHostToDevice, st));
+    launch_csr_stage(csr->indptr, csr->indices, csr->values, d_perm.get(), n, d, c_ptr.get(), c_idx.get(), c_val.get(),
+                     norms.get(), bad.get(), st);
   } else {
     launch_stage_features(dX, n, d, d_perm.get(), XT.get(), n_pad, d_pad, n_pad, norms.get(), bad.get(), st);
   }
@@ -1356,6 +1377,8 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
       GM_CUDA(cudaEventRecord(ev_wave[g], kst));
     }
     GM_CUDA(cudaEventRecord(ev_k1, kst));
+  } else if (full_k && csr) {  // NEXT-3: sparse x dense from the class-sorted CSR rows
+    launch_krow_csr(c_ptr.get(), c_idx.get(), c_val.get(), norms.get(), n, d, gamma, K.get(), ldk, st);
   } else if (full_k && !use_tc) {
     launch_krow_full_sym(XT.get(), n_pad, norms.get(), n, d_pad, gamma, K.get(), ldk, st);
   }
@@ -1907,7 +1930,18 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   HT("assembled");
   // the SV-row centre and scale are recomputed from the SV rows (not the training call's), so a
   // model merged from partial trainings predicts bitwise like the single-call model
-  mdl->dev = build_dev_model(*mdl, dX, row_of_sv, opt.device, st, nullptr, 0.f, d_alpha.get(), tot, &alpha_off);
+  DevBuf<float> sv_dense(csr ? (size_t)std::max<size_t>(row_of_sv.size(), 1) * d : 0, st);
+  if (csr) {  // the model's support-vector rows, densified (prediction contracts dense SV tiles)
+    DevBuf<int64_t> d_rows(std::max<size_t>(row_of_sv.size(), 1), st);
+    if (!row_of_sv.empty())
+      GM_CUDA(cudaMemcpyAsync(d_rows.get(), row_of_sv.data(), row_of_sv.size() * 8, cudaMemcpyHostToDevice, st));
+    launch_csr_densify_rows(csr->indptr, csr->indices, csr->values, d_rows.get(), (int64_t)row_of_sv.size(), d,
+                            sv_dense.get(), st);
+    for (size_t i = 0; i < row_of_sv.size(); ++i) row_of_sv[i] = (int64_t)i;
+    GM_CUDA(cudaStreamSynchronize(st));  // d_rows goes out of scope
+  }
+  mdl->dev = build_dev_model(*mdl, csr ? sv_dense.get() : dX, row_of_sv, opt.device, st, nullptr, 0.f, d_alpha.get(),
+                             tot, &alpha_off);
   tm.mark(PH_FIN);
   HT("devmodel");
   if (lead_dbg) GM_CUDA(cudaEventRecord(dbg1.a, st));
@@ -1966,6 +2000,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   s.smo_cycles_sum = cyc_sum;
   s.n_sv = (int64_t)mdl->sv_pos.size();
   s.cache_regime = full_k ? 0 : 1;
+  s.kernel_path = csr ? 2 : (use_tc ? 0 : 1);
   s.n_pairs_trained = Pl;
   s.launches = (int64_t)(g_launches.load() - launches0);
   s.t_total_ms = host_ms_since(t_start);
@@ -2068,35 +2103,39 @@ int engine_model_from_alpha(const float* X, const int32_t* y, int64_t n, int32_t
 // CSR input (NEXT-3, the format of the paper's datasets): densified on the device, then the dense
 // path (the kernel-value contraction runs on the dense rows).  indptr [n+1] int64, indices [nnz]
 // int32, values [nnz] float; host or device pointers per opt.inputs_on_device.
-struct CsrDense {
-  DevBuf<float> X;
-  CsrDense(const int64_t* indptr, const int32_t* indices, const float* values, int64_t n, int32_t d,
-           const gmpsvm_options& opt, cudaStream_t st)
-      : X((size_t)std::max<int64_t>(n, 1) * d, st) {
+struct CsrDev {  // the CSR arrays on the device (uploaded, or the caller's device pointers)
+  DevBuf<int64_t> ip;
+  DevBuf<int32_t> ix;
+  DevBuf<float> vv;
+  CsrSrc src{};
+  CsrDev(const int64_t* indptr, const int32_t* indices, const float* values, int64_t n, int32_t d,
+         const gmpsvm_options& opt, cudaStream_t st) {
     if (n < 0 || d < 1 || !indptr) throw Error(GMPSVM_EINVAL, "bad CSR arguments");
     int64_t nnz = 0;
     if (opt.inputs_on_device) GM_CUDA(cudaMemcpy(&nnz, indptr + n, 8, cudaMemcpyDeviceToHost));
     else nnz = indptr[n];
     if (nnz < 0 || (nnz > 0 && (!indices || !values))) throw Error(GMPSVM_EINVAL, "bad CSR arguments");
-    DevBuf<int64_t> ip(opt.inputs_on_device ? 0 : (size_t)n + 1, st);
-    DevBuf<int32_t> ix(opt.inputs_on_device ? 0 : (size_t)nnz, st);
-    DevBuf<float> vv(opt.inputs_on_device ? 0 : (size_t)nnz, st);
-    const int64_t* dip = indptr;
-    const int32_t* dix = indices;
-    const float* dvv = values;
+    src = CsrSrc{indptr, indices, values, nnz};
     if (!opt.inputs_on_device) {
+      new (&ip) DevBuf<int64_t>((size_t)n + 1, st);
+      new (&ix) DevBuf<int32_t>((size_t)std::max<int64_t>(nnz, 1), st);
+      new (&vv) DevBuf<float>((size_t)std::max<int64_t>(nnz, 1), st);
       GM_CUDA(cudaMemcpyAsync(ip.get(), indptr, ((size_t)n + 1) * 8, cudaMemcpyHostToDevice, st));
       if (nnz) {
         GM_CUDA(cudaMemcpyAsync(ix.get(), indices, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
         GM_CUDA(cudaMemcpyAsync(vv.get(), values, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
       }
-      dip = ip.get();
-      dix = ix.get();
-      dvv = vv.get();
+      src = CsrSrc{ip.get(), ix.get(), vv.get(), nnz};
     }
+  }
+};
+
+struct CsrDense {  // densified on the device (the dense path's input)
+  DevBuf<float> X;
+  CsrDense(const CsrSrc& c, int64_t n, int32_t d, cudaStream_t st) : X((size_t)std::max<int64_t>(n, 1) * d, st) {
     DevBuf<int32_t> bad(1, st);
     GM_CUDA(cudaMemsetAsync(bad.get(), 0, 4, st));
-    launch_csr_densify(dip, dix, dvv, n, d, X.get(), bad.get(), st);
+    launch_csr_densify(c.indptr, c.indices, c.values, n, d, X.get(), bad.get(), st);
     int32_t hb = 0;
     GM_CUDA(cudaMemcpyAsync(&hb, bad.get(), 4, cudaMemcpyDeviceToHost, st));
     GM_CUDA(cudaStreamSynchronize(st));
@@ -2104,11 +2143,32 @@ struct CsrDense {
   }
 };
 
+// Sparse kernel values (NEXT-3, csr.cu): GMPSVM_CSR=sparse forces them (read per call), =dense
+// the densified path.  By default the rows are densified -- on the news20-shaped data the dense
+// tcgen05 contraction is faster (n = 20k, d = 5000, 1 % non-zero: 4.4 vs 8.1 ms) --
+// unless the dense copy would take more than a quarter of the device memory.  The sparse path
+// needs the Gaussian kernel, FULL_K, no CV sigmoids and one dense row in shared memory (d <= 56k).
+static bool csr_sparse_path(const CsrSrc& c, int64_t n, int32_t d, const gmpsvm_options& opt) {
+  const char* env = getenv("GMPSVM_CSR");
+  const std::string mode = env ? env : "";
+  if (mode == "dense") return false;
+  const double mem = (double)device_total_mem(opt.device);
+  const double budget = opt.cache_bytes > 0 ? (double)opt.cache_bytes : 0.85 * mem;
+  const bool ok = opt.kernel == 0 && opt.prob_folds == 0 && krow_csr_rows_per_cta(d) >= 1 &&
+                  (double)n * round_up(n, 4) * 4.0 <= budget;
+  if (mode == "sparse") {
+    if (!ok) throw Error(GMPSVM_ENOTIMPL, "GMPSVM_CSR=sparse: needs the Gaussian kernel, FULL_K, no CV sigmoids, d <= 56k");
+    return true;
+  }
+  (void)c;
+  return ok && (double)n * (double)d * 4.0 > 0.25 * mem;
+}
+
 int engine_train_csr(const int64_t* indptr, const int32_t* indices, const float* values, const int32_t* y, int64_t n,
                      int32_t d, int32_t k, double C, double gamma, double eps, const gmpsvm_options& opt, Model** out) {
   DeviceGuard dg(opt.device);
   cudaStream_t st = get_stream(opt);
-  CsrDense cd(indptr, indices, values, n, d, opt, st);
+  CsrDev cdev(indptr, indices, values, n, d, opt, st);
   gmpsvm_options o2 = opt;
   DevBuf<int32_t> yb(opt.inputs_on_device ? 0 : (size_t)n, st);
   const int32_t* dy = y;
@@ -2119,6 +2179,8 @@ int engine_train_csr(const int64_t* indptr, const int32_t* indices, const float*
   }
   o2.inputs_on_device = 1;
   o2.stream = st;
+  if (csr_sparse_path(cdev.src, n, d, opt)) return engine_train_core(nullptr, dy, n, d, k, C, gamma, eps, o2, out, &cdev.src);
+  CsrDense cd(cdev.src, n, d, st);
   return engine_train(cd.X.get(), dy, n, d, k, C, gamma, eps, o2, out);
 }
 
@@ -2127,7 +2189,8 @@ int engine_predict_csr(const Model& mdl, const int64_t* indptr, const int32_t* i
   if (m == 0) return GMPSVM_OK;
   DeviceGuard dg(opt.device);
   cudaStream_t st = get_stream(opt);
-  CsrDense cd(indptr, indices, values, m, mdl.d, opt, st);
+  CsrDev cdev(indptr, indices, values, m, mdl.d, opt, st);
+  CsrDense cd(cdev.src, m, mdl.d, st);
   gmpsvm_options o2 = opt;
   o2.stream = st;
   if (opt.inputs_on_device) return engine_predict(mdl, cd.X.get(), m, prob_out, nullptr, o2);

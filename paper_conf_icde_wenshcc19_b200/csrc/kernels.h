@@ -222,6 +222,25 @@ int ws_persist_workers_per_sm();
 // started-CTA count, KrowKernel::resident) reaches it, so the workers land beside that launch.
 void launch_ws_persist(const SolverArgs& a, int P, int nworkers, int64_t max_outer, void* ring, unsigned long long* ctr,
                        cudaStream_t st, const unsigned long long* res_ctr = nullptr, int wait_resident = 0);
+// ---------------- NEXT-3: CSR kernel values (csr.cu)
+// device CSR rows of X: indptr [n+1], indices [nnz] (columns in [0, d)), values [nnz]
+struct CsrSrc {
+  const int64_t* indptr;
+  const int32_t* indices;
+  const float* values;
+  int64_t nnz;
+};
+// class-sorted copy: row i of the sorted order = input row perm[i], sptr its row pointers;
+// norms[i] = |x_i|^2 (FP64-accumulated); *bad = 1 on a column outside [0, d) or a non-finite value
+void launch_csr_stage(const int64_t* indptr, const int32_t* indices, const float* values, const int64_t* perm, int64_t n,
+                      int32_t d, const int64_t* sptr, int32_t* sidx, float* sval, float* norms, int32_t* bad,
+                      cudaStream_t st);
+int krow_csr_rows_per_cta(int32_t d);  // dense rows per CTA in shared memory (0: d too large)
+// FULL_K (n x ldk, symmetric, K_ii = 1) from the sorted CSR rows: sparse x dense, one warp per column row
+void launch_krow_csr(const int64_t* sptr, const int32_t* sidx, const float* sval, const float* norms, int64_t n,
+                     int32_t d, double gamma, float* K, int64_t ldk, cudaStream_t st);
+void launch_csr_densify_rows(const int64_t* indptr, const int32_t* indices, const float* values, const int64_t* rows,
+                             int64_t nr, int32_t d, float* out, cudaStream_t st);
 void launch_finalize(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sigmoid_fit(const SolverArgs& a, int P, cudaStream_t st);
 void launch_sv_flags(const SolverArgs& a, int P, int64_t np_max, uint8_t* flags, cudaStream_t st);
