@@ -24,4 +24,13 @@ m = gm.train(X, y, spec.k, spec.C, spec.gamma, 1e-3, ws_size=96)
 p = m.predict_proba(Xt)
 K = gm.rbf_kernel(X[:300], X[:200], spec.gamma)
 K2 = gm.rbf_kernel(X[:257], X[:257], spec.gamma)
+if os.environ.get("SANITIZE_SPARSE", "1") == "1":  # NEXT-3: sparse kernel values from CSR rows (csr.cu)
+    import scipy.sparse as sps
+    os.environ["GMPSVM_CSR"] = "sparse"
+    specn, Xn, yn, Xnt, ynt = datagen.make_config("news20", n_train=400, n_test=50)
+    ms = gm.train_csr(sps.csr_matrix(Xn), yn, specn.k, specn.C, specn.gamma, 1e-3)
+    assert ms.train_stats()["kernel_path"] == 2
+    ps = ms.predict_proba(Xnt)
+    del os.environ["GMPSVM_CSR"]
+    print("sparse ok", ms.n_sv, float(ps.sum()))
 print("sanitize workload ok", m.n_sv, float(p.sum()), float(K.sum()), float(K2.sum()))
