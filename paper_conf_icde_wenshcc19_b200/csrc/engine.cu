@@ -1398,6 +1398,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   ArenaPtr<PairDesc> d_pairs;
   ArenaPtr<double> d_alpha, d_f, d_v, d_dcoef, d_gap, d_b, d_A, d_B;
   ArenaPtr<uint32_t> d_stamp;
+  ArenaPtr<uint8_t> d_ulf;
   ArenaPtr<int32_t> d_ws, d_wsn, d_wst, d_status, d_outer, d_sig;
   ArenaPtr<int64_t> d_inner, d_cyc, d_body;
   ArenaPtr<float> d_Kws;
@@ -1412,6 +1413,7 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   lay.add(d_A, Pl);
   lay.add(d_B, Pl);
   lay.add(d_stamp, tot);
+  lay.add(d_ulf, tot);
   lay.add(d_ws, (size_t)Pl * Bw);
   lay.add(d_wsn, Pl);
   lay.add(d_wst, (size_t)Pl * Bw);
@@ -1491,6 +1493,8 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   a.trace_cap = trace_cap;
   static const int fu_chunks = getenv("GMPSVM_FU_CHUNKS") ? std::max(1, atoi(getenv("GMPSVM_FU_CHUNKS"))) : 1;
   a.fu_chunks = fu_chunks;
+  static const bool ulf_off = getenv("GMPSVM_ULF") && std::string(getenv("GMPSVM_ULF")) == "0";
+  a.ulf = ulf_off ? nullptr : d_ulf.get();  // selection reads membership bits instead of alpha
   static const bool smo_f64_env = getenv("GMPSVM_SMO_F32") && std::string(getenv("GMPSVM_SMO_F32")) == "0";
   a.smo_f32 = (!smo_f64_env && ktype == 0) ? 1 : 0;  // the Gaussian kernel's QP is convex: FP32 local f
   a.outer_iters = d_outer.get();

@@ -138,6 +138,8 @@ struct SolverArgs {
   int32_t trace_pair, trace_cap;
   int32_t fu_chunks = 1;  // 128-column chunks per f-update CTA (ws_fupdate_kernel)
   int32_t smo_f32 = 0;    // local SMO with FP32 working-set f (wsolve.cu ws_smo_body)
+  uint8_t* ulf = nullptr;  // per instance: bit0 in I_u, bit1 in I_l (wsolve.cu: written by the local SMO,
+                           // read by the selection instead of alpha; null: alpha is read)
   int64_t* sel_phase;   // [P][5] optional select_ws phase cycles (GMPSVM_SMO_PHASES=1), else NULL
   int32_t* outer_iters; // [P]
   double* b;            // [P]

@@ -41,6 +41,7 @@ __global__ void init_pairs_kernel(SolverArgs a, const int64_t tot, int P) {
     a.alpha[i] = 0.0;
     a.f[i] = (j < pd.n_s) ? -1.0 : 1.0;
     a.stamp[i] = 0u;
+    if (a.ulf) a.ulf[i] = (j < pd.n_s) ? 1 : 2;  // alpha = 0: y = +1 in I_u only, y = -1 in I_l only
   }
   if (i < P) {
     a.status[i] = 0;

@@ -222,6 +222,7 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
   const double C = a.C;
   const double* al = a.alpha + pd.a_off;
   const double* fl = a.f + pd.a_off;
+  const uint8_t* ulf = a.ulf ? a.ulf + pd.a_off : nullptr;
   // Before the dependency wait: the retained rows come from the previous selection's output
   // (ws_tmp, ws_n, outer_iters), which completed before this launch's predecessor (the f-update)
   // was released, so building their bitmap overlaps the f-update's tail.  L2 loads (.cg).
@@ -263,10 +264,12 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
   uint64_t mk[2] = {~0ull, ~0ull};
   for (int base = 0; base < np; base += kStageUnroll * kWT) {
     double av[kStageUnroll], fv[kStageUnroll];
+    uint8_t uf[kStageUnroll];
 #pragma unroll
     for (int m = 0; m < kStageUnroll; ++m) {
       const int i = base + m * kWT + t;
-      av[m] = i < np ? __ldcg(al + i) : 0.0;  // L2 loads (see ws_write_out)
+      if (ulf) uf[m] = i < np ? __ldcg(ulf + i) : (uint8_t)0;  // membership bits (1 B) instead of alpha (8 B)
+      else av[m] = i < np ? __ldcg(al + i) : 0.0;  // L2 loads (see ws_write_out)
       fv[m] = i < np ? __ldcg(fl + i) : 0.0;
     }
 #pragma unroll
@@ -274,7 +277,7 @@ __device__ __forceinline__ void ws_select_body(const SolverArgs& a, const int lp
       const int i = base + m * kWT + t;
       if (i < np) {
         const int y = i < pd.n_s ? 1 : -1;
-        const bool u = in_u(y, av[m], C), l = in_l(y, av[m], C);
+        const bool u = ulf ? (uf[m] & 1) != 0 : in_u(y, av[m], C), l = ulf ? (uf[m] & 2) != 0 : in_l(y, av[m], C);
         const bool ret = (W.retained[i >> 5] >> (i & 31)) & 1u;
         if (u) fmin = fmin < fv[m] ? fmin : fv[m];
         if (l) fmax = fmax > fv[m] ? fmax : fv[m];
@@ -862,8 +865,10 @@ __device__ __forceinline__ void ws_smo_body(const SolverArgs& a, const int lp, u
     if ((vmask >> q) & 1u) {
       const double al = lds_f64(als + e * 8);
       const double a0 = lds_f64(a0s + e * 8);
-      a.dcoef[(int64_t)lp * B + e] = (al - a0) * (((ypos >> q) & 1u) ? 1.0 : -1.0);
+      const int y = ((ypos >> q) & 1u) ? 1 : -1;
+      a.dcoef[(int64_t)lp * B + e] = (al - a0) * (double)y;
       a.alpha[pd.a_off + idx[q]] = al;
+      if (a.ulf) a.ulf[pd.a_off + idx[q]] = (uint8_t)((in_u(y, al, C) ? 1 : 0) | (in_l(y, al, C) ? 2 : 0));
     }
   }
   if (lane == 0) {
