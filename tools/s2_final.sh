@@ -12,6 +12,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
 python tools/launch_sum.py $out/launches.csv > $out/launches_sum.txt 2>&1; head -14 $out/launches_sum.txt
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:krow_tc_kernel -s 1 -c 1 -f -o $out/krow_tc python tools/prof_step.py --ws-size 192 > $out/ncu_krow.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:dec_i8_kernel -c 1 -f -o $out/dec_i8 python tools/prof_dec.py --reps 1 > $out/ncu_dec.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:krow_csr_kernel -c 1 -f -o $out/krow_csr python tools/sparse_probe.py --n 20000 --reps 1 > $out/ncu_csr.log 2>&1
 for k in ws_select_kernel ws_smo_kernel ws_fupdate_kernel ws_gather_kernel; do
 GMPSVM_NOGRAPH=1 timeout 900 ncu --set full --clock-control none --import-source on -k regex:$k -s 100 -c 1 -f -o $out/$k python tools/prof_step.py --ws-size 192 > $out/ncu_$k.log 2>&1
 done
