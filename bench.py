@@ -212,6 +212,8 @@ def run_gpu(args, spec):
                    torch.from_numpy(Xt).pin_memory())
     stream = torch.cuda.current_stream(dev)
     opts = dict(ws_size=args.ws_size, q=args.q)
+    if args.inner_cap:
+        opts["inner_iter_cap"] = args.inner_cap
 
     host_ms = []  # host-clock duration of each step's calls (diagnostic: stalls outside the GPU)
 
@@ -414,6 +416,7 @@ def main():
     ap.add_argument("--eps", type=float, default=1e-3)
     ap.add_argument("--ws-size", dest="ws_size", type=int, default=192)
     ap.add_argument("--q", type=int, default=0, help="new working-set rows per outer iteration (0: ws_size / 2)")
+    ap.add_argument("--inner-cap", dest="inner_cap", type=int, default=0, help="local SMO steps per outer iteration cap (0: 100 ws_size)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:

@@ -75,7 +75,8 @@ typedef struct {
   int32_t n_pair_ids;       /* >= 1 when pair_ids != NULL (else GMPSVM_EINVAL)               */
   int32_t inputs_on_device; /* 1: X/y/Xtest/out are device pointers on `device`             */
   int64_t max_outer_iter;   /* cap on outer (working-set) iterations per pair; 0 = 1,000,000 */
-  int32_t inner_iter_cap;   /* cap on inner SMO steps per working set; 0 = 100 * B          */
+  int32_t inner_iter_cap;   /* cap on inner SMO steps per working set; 0 = B / 2 for the RBF */
+                            /* kernel on the shared-memory solver (B <= 224), else 100 * B  */
   int32_t kernel;           /* GMPSVM_KERNEL_*: the paper's RBF (L75, default) or one of the
                                other kernels it lists (L76-L78; LibSVM definitions, gamma the
                                train call's): training needs the FULL_K regime on the tensor

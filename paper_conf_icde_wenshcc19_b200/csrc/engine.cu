@@ -1504,7 +1504,13 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   a.sig_status = d_sig.get();
   a.B = Bw;
   a.q = q;
-  a.inner_cap = opt.inner_iter_cap > 0 ? opt.inner_iter_cap : 100 * Bw;
+  // local SMO steps per outer iteration (R20): B / 2 on the shared-memory solver (measured,
+  // MNIST-shaped: cap 64 / 80 / 96 / 112 / none: 31.5 / 30.2 / 29.8 / 29.8 / 30.1-30.3 ms -- the
+  // long first local solves of the hardest pairs stop early and the next outer iteration, with the
+  // exact f, continues), else 100 B.  The Gaussian kernel only: the dot-product kernels' duals need
+  // not have a unique alpha (linear: rank <= d), so their path decides the alpha reached
+  a.inner_cap = opt.inner_iter_cap > 0 ? opt.inner_iter_cap
+                                       : (ktype == 0 && Bw <= ws_smo_max_b() ? std::max(16, Bw / 2) : 100 * Bw);
   a.C = C;
   a.eps = eps;
   static const double env_ratio = getenv("GMPSVM_LOCAL_RATIO") ? atof(getenv("GMPSVM_LOCAL_RATIO")) : 0.1;
