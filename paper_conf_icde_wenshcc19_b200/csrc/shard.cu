@@ -252,7 +252,10 @@ static SolverArgs shard_args(Shard& S) {
   a.sig_status = S.d_sig.get();
   a.B = S.B;
   a.q = S.q;
-  a.inner_cap = 100 * S.B;
+  // the single-GPU defaults of the shared-memory solver for the Gaussian kernel (engine.cu, R20,
+  // R29): FP32 working-set f in the local solve, at most B / 2 steps per outer iteration
+  a.inner_cap = S.B <= ws_smo_max_b() ? std::max(16, S.B / 2) : 100 * S.B;
+  a.smo_f32 = 1;
   a.pair_base = 0;
   a.C = S.C;
   a.eps = S.eps;
