@@ -480,14 +480,24 @@ constexpr int kGR = 8;  // tile rows per CTA
 __device__ __forceinline__ void ws_gather_body(const SolverArgs& a, const int lp, const int by, int64_t* g) {
   const PairDesc pd = a.pairs[lp];
   const int wn = __ldcg(a.ws_n + lp);
-  const int r0 = by * kGR;
-  if (r0 >= wn) return;
+  // rows of the CTA: kGR / 2 from the top of the triangle and their mirrors from the bottom
+  // (row r has wn - r entries c >= r, so each pair of rows has wn + 1: every CTA the same work)
+  constexpr int kH = kGR / 2;
+  const int half = (wn + 1) / 2;
+  const int t0 = by * kH;
+  if (t0 >= half) return;
   const int32_t* ws = a.ws + (int64_t)lp * a.B;
   for (int e = threadIdx.x; e < wn; e += blockDim.x) g[e] = gpos(pd, __ldcg(ws + e));
   __syncthreads();
   const int ld = ws_tile_ld(a.B);
   float* tile = a.Kws + (int64_t)lp * ws_buf_floats(a.B);
-  const int r1 = min(wn, r0 + kGR);
+  auto row_of = [&](int k) -> int {  // CTA row k in [0, kGR): -1 if none
+    const int tt = t0 + (k < kH ? k : k - kH);
+    if (tt >= half) return -1;
+    if (k < kH) return tt;
+    const int rb = wn - 1 - tt;
+    return rb > tt ? rb : -1;  // the middle row of an odd wn belongs to the top half only
+  };
   // K is stored symmetric (both triangles, the same values): the tile's upper triangle is loaded
   // and written to both positions -- half the scattered loads (each one a DRAM burst of its own)
   constexpr int M = (kGR * kWMaxB + 255) / 256;  // loads per thread, all in flight
@@ -495,14 +505,16 @@ __device__ __forceinline__ void ws_gather_body(const SolverArgs& a, const int lp
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int q = threadIdx.x + m * 256;
-    const int r = r0 + q / wn, c = q % wn;
-    v[m] = (r < r1 && c >= r) ? __ldg(a.K + g[r] * a.ldk + g[c]) : 0.f;
+    const int k = q / wn, c = q % wn;
+    const int r = k < kGR ? row_of(k) : -1;
+    v[m] = (r >= 0 && c >= r) ? __ldg(a.K + g[r] * a.ldk + g[c]) : 0.f;
   }
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int q = threadIdx.x + m * 256;
-    const int r = r0 + q / wn, c = q % wn;
-    if (r < r1 && c >= r) {
+    const int k = q / wn, c = q % wn;
+    const int r = k < kGR ? row_of(k) : -1;
+    if (r >= 0 && c >= r) {
       tile[(int64_t)r * ld + c] = v[m];
       tile[(int64_t)c * ld + r] = v[m];
     }
