@@ -1304,11 +1304,62 @@ __global__ void class_means_kernel(const T* hi, int d_pad, const int64_t* coff, 
   }
 }
 
+// FP16 split: the rows of a class in kCmChunks slices (more loads in flight than one CTA per 32
+// features and class; the sequential loop of class_means_kernel took ~170 us for MNIST-shaped X,
+// on the path to the first kernel-value wave), each thread two features (half2), partial sums
+// reduced over the slices in a fixed order (deterministic).
+constexpr int kCmChunks = 16;
+__global__ void class_means_part_kernel(const __half* hi, int d_pad, const int64_t* coff, float* part) {
+  const int c = blockIdx.y, ch = blockIdx.z, f = blockIdx.x * 64 + 2 * threadIdx.x;
+  const int64_t r0 = coff[c], r1 = coff[c + 1], len = r1 - r0;
+  const int64_t a = r0 + len * ch / kCmChunks, b = r0 + len * (ch + 1) / kCmChunks;
+  float s0 = 0.f, s1 = 0.f, q0 = 0.f, q1 = 0.f;
+  if (f < d_pad)
+    for (int64_t r = a + threadIdx.y; r < b; r += 8) {
+      const float2 v = __half22float2(*reinterpret_cast<const __half2*>(hi + r * d_pad + f));
+      s0 += v.x;
+      s1 += v.y;
+      q0 = fmaf(v.x, v.x, q0);
+      q1 = fmaf(v.y, v.y, q1);
+    }
+  __shared__ float red[4][8][33];
+  red[0][threadIdx.y][threadIdx.x] = s0;
+  red[1][threadIdx.y][threadIdx.x] = s1;
+  red[2][threadIdx.y][threadIdx.x] = q0;
+  red[3][threadIdx.y][threadIdx.x] = q1;
+  __syncthreads();
+  if (threadIdx.y < 4) {  // y = 0, 1: sums of features f, f + 1; y = 2, 3: their squares
+    float t = 0.f;
+#pragma unroll
+    for (int y = 0; y < 8; ++y) t += red[threadIdx.y][y][threadIdx.x];
+    const int ff = f + (threadIdx.y & 1);
+    if (ff < d_pad) part[(((int64_t)ch * 2 + (threadIdx.y >> 1)) * gridDim.y + c) * d_pad + ff] = t;
+  }
+}
+__global__ void class_means_reduce_kernel(const float* part, int d_pad, int k, const int64_t* coff, float* mu,
+                                          float* m2) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;  // c * d_pad + f
+  if (i >= (int64_t)k * d_pad) return;
+  const int c = (int)(i / d_pad);
+  float t = 0.f, t2 = 0.f;
+  for (int ch = 0; ch < kCmChunks; ++ch) {
+    t += part[((int64_t)ch * 2 + 0) * k * d_pad + i];
+    t2 += part[((int64_t)ch * 2 + 1) * k * d_pad + i];
+  }
+  const int64_t cnt = coff[c + 1] - coff[c];
+  const float inv = cnt > 0 ? 1.f / (float)cnt : 0.f;
+  mu[i] = t * inv;
+  m2[i] = t2 * inv;
+}
+
 void launch_class_means(const void* hi, int d_pad, const int64_t* coff, int k, float* mu, float* m2, cudaStream_t st) {
-  if (krow_split_f16())
-    GM_LAUNCH(class_means_kernel<__half>, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st,
-              static_cast<const __half*>(hi), d_pad, coff, mu, m2);
-  else
+  if (krow_split_f16()) {  // d_pad is a multiple of 64 (krow_tc_d_pad): half2 loads stay aligned
+    DevBuf<float> part((size_t)kCmChunks * 2 * k * d_pad, st);
+    GM_LAUNCH(class_means_part_kernel, dim3((unsigned)ceil_div(d_pad, 64), (unsigned)k, kCmChunks), dim3(32, 8), 0, st,
+              static_cast<const __half*>(hi), d_pad, coff, part.get());
+    GM_LAUNCH(class_means_reduce_kernel, dim3((unsigned)ceil_div((int64_t)k * d_pad, 256)), dim3(256), 0, st, part.get(),
+              d_pad, k, coff, mu, m2);
+  } else
     GM_LAUNCH(class_means_kernel<float>, dim3((unsigned)ceil_div(d_pad, 32), (unsigned)k), dim3(32, 8), 0, st,
               static_cast<const float*>(hi), d_pad, coff, mu, m2);
 }
