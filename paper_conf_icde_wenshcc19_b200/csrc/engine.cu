@@ -1537,22 +1537,30 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   int n_sm = 0;
   GM_CUDA(cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, opt.device));
   bool persist = !rc && ng <= 2 && !smo_prof && ws_persist_supported(Bw, np_max);
+  // GMPSVM_PERSIST=lead: only the lead group persistent (its handoffs are flag round trips, its
+  // workers on its reserved SMs); the other groups run the graphs below
+  static const bool persist_lead_env = getenv("GMPSVM_PERSIST") && std::string(getenv("GMPSVM_PERSIST")) == "lead";
+  bool plead = persist && persist_lead_env && lead && ng >= 2;
+  if (plead) persist = false;
+  int npg = plead ? 1 : (persist ? ng : 0);  // groups on the persistent solver: [0, npg)
   std::vector<int> pgrid(ng, 0);
   std::vector<size_t> pq_off(ng + 1, 0);
-  if (persist) {
+  if (npg > 0) {
     const int wps = ws_persist_workers_per_sm();
-    for (int g = 0; g < ng; ++g) {
+    for (int g = 0; g < npg; ++g) {
       const int pg = gpos[g + 1] - gpos[g];
       // the group's SMs: lead mode -- the lead group beside the last kernel-value wave on the
       // `reserve` SMs, the rest on the others; workers fill the SMs around the leaders
       const int sms = !lead ? n_sm : (g == 0 ? std::max(2, std::min(reserve_env, n_sm / 2)) : n_sm - std::max(2, std::min(reserve_env, n_sm / 2)));
       pgrid[g] = std::max(0, sms - pg) * wps + pg;  // workers
-      if (pg >= sms || wps < 1) persist = false;
+      if (pg >= sms || wps < 1) persist = plead = false;
       pq_off[g + 1] = pq_off[g] + ws_persist_ring_bytes() + ws_persist_ctr_words(pg) * 8;
     }
+    if (!persist && !plead) npg = 0;
   }
-  DevBuf<uint8_t> d_pq(persist ? pq_off[ng] : 0, st);
-  if (persist) GM_CUDA(cudaMemsetAsync(d_pq.get(), 0, pq_off[ng], st));
+  const bool pq_on = persist || plead;
+  DevBuf<uint8_t> d_pq(pq_on ? pq_off[npg] : 0, st);
+  if (pq_on) GM_CUDA(cudaMemsetAsync(d_pq.get(), 0, pq_off[npg], st));
   auto pq_ctr = [&](int g) {
     return reinterpret_cast<unsigned long long*>(d_pq.get() + pq_off[g] + ws_persist_ring_bytes());
   };
@@ -1719,6 +1727,22 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
         ev_gst[g] = evk.get(true);
         ev_gend[g] = evk.get(true);
       }
+      if (plead && g == 0) {  // the lead group's graph stays unlaunched (cached with the others)
+        cudaStream_t ls = pool[0];
+        GM_CUDA(cudaStreamWaitEvent(ls, ev_ready, 0));
+        GM_CUDA(cudaStreamWaitEvent(ls, ev_wave[0], 0));
+        if (ev_gst[0]) GM_CUDA(cudaEventRecord(ev_gst[0], ls));
+        SolverArgs ag = a;
+        ag.pair_base = gpos[0];
+        const int pg = gpos[1] - gpos[0];
+        launch_ws_persist(ag, pg, pgrid[0], max_outer, d_pq.get(), pq_ctr(0), ls, d_kres.get(), kres_wait);
+        launch_finalize(ag, pg, ls);
+        launch_sigmoid_fit(ag, pg, ls);
+        cudaEvent_t ev = ev_gend[0] ? ev_gend[0] : evp.get();
+        GM_CUDA(cudaEventRecord(ev, ls));
+        GM_CUDA(cudaStreamWaitEvent(st, ev, 0));
+        continue;
+      }
       launch_after(ex[g], pool[g], lead ? ev_wave[g] : nullptr, ev_gend[g], ev_gst[g]);
     }
     if (ws && !reuse) {  // the freshly built graphs become the device's cached ones
@@ -1786,13 +1810,17 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
   HT("fin_d2h");
-  for (int g = 0; persist && g < ng; ++g) {
+  for (int g = 0; g < npg; ++g) {
     unsigned long long perr = 0;
     GM_CUDA(cudaMemcpy(&perr, pq_ctr(g) + 3, 8, cudaMemcpyDeviceToHost));
     if (perr) throw Error(GMPSVM_ECUDA, "persistent solver: a wait timed out (group " + std::to_string(g) + ")");
   }
   {  // kernels the graph executed: every body run launches body_launches kernels, + final selects
     int64_t ex = final_selects;  // one final selection per split-path branch
+    if (plead) {  // the lead group ran persistent: its launches were counted at launch
+      ex -= 2 * (gbr[1] - gbr[0]);
+      for (int i = gpos[0]; i < gpos[1]; ++i) body_per_pair[i] = 0;
+    }
     for (int i = 0; i < Pl; ++i) ex += h_body[i] * body_per_pair[i];  // counted at each branch's first pair
     g_launches.fetch_add((uint64_t)ex);
     if (rc) {

@@ -1198,8 +1198,10 @@ size_t ws_persist_ctr_words(int P) { return (size_t)kPCtrPairs + P; }
 size_t ws_persist_ring_bytes() { return sizeof(PTask) * kPQueueCap; }
 
 bool ws_persist_supported(int B, int64_t np_max) {
-  // opt-in (GMPSVM_PERSIST=1): measured slower on MNIST-shaped data
-  static const bool off = !(getenv("GMPSVM_PERSIST") && std::string(getenv("GMPSVM_PERSIST")) == "1");
+  // opt-in (GMPSVM_PERSIST=1: every group; =lead: the lead group only, the others on the graphs):
+  // measured slower on MNIST-shaped data
+  static const char* e = getenv("GMPSVM_PERSIST");
+  static const bool off = !(e && (std::string(e) == "1" || std::string(e) == "lead"));
   int dev = 0, optin = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);

@@ -64,7 +64,8 @@ def test_schedule_does_not_change_the_model(tmp_path):
                      ("noreuse", {"GMPSVM_GRAPH_REUSE": "0"}),
                      ("krow_no_cluster", {"GMPSVM_KROW_MC": "0"}),
                      ("persistent", {"GMPSVM_PERSIST": "1"}),
-                     ("persistent_nolead", {"GMPSVM_PERSIST": "1", "GMPSVM_LEAD": "0"})]:
+                     ("persistent_nolead", {"GMPSVM_PERSIST": "1", "GMPSVM_LEAD": "0"}),
+                     ("persistent_lead_only", {"GMPSVM_PERSIST": "lead"})]:
         other = _run(tmp_path, tag, env)
         for a, b in zip(other, base):
             np.testing.assert_array_equal(a, b, err_msg=tag)
