@@ -421,8 +421,8 @@ T* dev_alloc(size_t count, cudaStream_t st, int dev) {
 // latter synchronises the device, so they are not called per training run).
 template <class T>
 T* pinned_scratch(size_t count, int slot = 0) {
-  static thread_local void* bufs[2] = {nullptr, nullptr};
-  static thread_local size_t caps[2] = {0, 0};
+  static thread_local void* bufs[3] = {nullptr, nullptr, nullptr};
+  static thread_local size_t caps[3] = {0, 0, 0};
   void*& buf = bufs[slot];
   size_t& cap = caps[slot];
   const size_t bytes = count * sizeof(T);
@@ -665,6 +665,7 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   GM_CUDA(cudaMemcpyAsync(d_src.get(), slot_src.data(), slot_src.size() * 8, cudaMemcpyHostToDevice, st));
   // conditioning of the decision values: sum_j |alpha_pj| per trained pair
   std::vector<double> abs_sum(P, 0.0);
+  double* abs_pin = nullptr;  // device path: read after the call's last synchronisation
   if (dev_coef) {
     std::vector<int64_t> npv(P, 0);
     for (int p = 0; p < P; ++p) npv[p] = m.class_count[ps_of(p, k)] + m.class_count[pt_of(p, k)];
@@ -673,13 +674,12 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
     GM_CUDA(cudaMemcpyAsync(d_ao.get(), alpha_off->data(), (size_t)P * 8, cudaMemcpyHostToDevice, st));
     GM_CUDA(cudaMemcpyAsync(d_np.get(), npv.data(), (size_t)P * 8, cudaMemcpyHostToDevice, st));
     launch_alpha_abs_sum(alpha_hp, d_ao.get(), d_np.get(), P, d_sum.get(), st);
-    GM_CUDA(cudaMemcpyAsync(abs_sum.data(), d_sum.get(), (size_t)P * 8, cudaMemcpyDeviceToHost, st));
-    GM_CUDA(cudaStreamSynchronize(st));
+    abs_pin = pinned_scratch<double>((size_t)P, 2);
+    GM_CUDA(cudaMemcpyAsync(abs_pin, d_sum.get(), (size_t)P * 8, cudaMemcpyDeviceToHost, st));
   } else {
     for (int p = 0; p < P; ++p)
       for (int64_t j = po[p]; j < po[p + 1]; ++j) abs_sum[p] += std::fabs(m.alpha[j]);
   }
-  dm->abs_sum = abs_sum;
   static const char* dec_env = getenv("GMPSVM_DEC");
   const std::string dec_mode = dec_env ? dec_env : "";
   // FP64 coefficients: the int8 and FP64 paths contract in FP64
@@ -751,6 +751,8 @@ static std::unique_ptr<DevModel> build_dev_model(const Model& m, const float* ro
   GM_CUDA(cudaEventCreateWithFlags(&dm->last_use, cudaEventDisableTiming));
   GM_CUDA(cudaEventRecord(dm->last_use, st));
   GM_CUDA(cudaStreamSynchronize(st));  // host vectors above go out of scope
+  if (abs_pin) std::copy(abs_pin, abs_pin + P, abs_sum.begin());
+  dm->abs_sum = abs_sum;
   std::memcpy(&dm->amax_sv, &amax_bits, 4);
   choose_dec_path(*dm, m);
   if (ht)
@@ -1961,8 +1963,19 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
     inner_sum += h_inner[i];
     cyc_sum += h_cyc[i];
   }
-  for (int64_t g = 0; g < n; ++g)
-    if (h_flags[g]) mdl->sv_pos.push_back(g);
+  {  // the SV positions: count, then a branchless compaction (~1/3 of the flags are set, at random)
+    int64_t cnt = 0;
+    for (int64_t g = 0; g < n; ++g) cnt += h_flags[g] != 0;
+    mdl->sv_pos.resize((size_t)cnt + 1);
+    int64_t* o = mdl->sv_pos.data();
+    int64_t j = 0;
+    for (int64_t g = 0; g < n; ++g) {
+      o[j] = g;
+      j += h_flags[g] != 0;
+    }
+    mdl->sv_pos.resize((size_t)cnt);
+  }
+  HT("asm_svpos");
   std::vector<int64_t> row_of_sv(mdl->sv_pos.size());
   for (size_t i = 0; i < row_of_sv.size(); ++i) row_of_sv[i] = mdl->perm[mdl->sv_pos[i]];
   HT("assembled");
