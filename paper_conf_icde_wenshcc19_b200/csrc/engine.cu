@@ -1008,7 +1008,8 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   const int d_pad = use_tc ? krow_tc_d_pad(d) : (int)round_up(d, kBK);
   // ROW_CACHE column tiles start at 4-aligned segment starts and may run 127 columns past n
   const int64_t n_pad = use_tc ? krow_tc_rows_pad(n) : round_up(n, kTile) + (full_k ? 0 : kTile);
-  // SIMT path: class-sorted feature-major copy; tensor-core path: row-major TF32 hi/lo split.
+  // SIMT path: class-sorted feature-major copy; tensor-core path: row-major FP16 hi/lo split
+  // (TF32 with GMPSVM_SPLIT=tf32).
   // norms: + one tile of zeros (ROW_CACHE column tiles run up to 127 columns past n)
   DevBuf<float> XT(use_tc || csr ? 0 : (size_t)d_pad * n_pad, st), norms(n_pad + kTile, st);
   // NEXT-3: class-sorted CSR rows (sptr on the host from the input row pointers and the order)

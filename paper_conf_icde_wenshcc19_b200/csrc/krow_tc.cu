@@ -72,7 +72,7 @@ constexpr uint32_t kIdescF16 = (1u << 4) | ((uint32_t)(kTN >> 3) << 17) | ((uint
 // hi.hi and hi.lo share the A tile (hi): issued back to back, the second reuses the collector and
 // the tensor core reads A from shared memory once for both
 template <bool F16, int COL = 0>
-__device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
+__device__ __forceinline__ void umma_hilo(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t accum) {
   if (F16 && COL == 1)
     asm volatile(
         "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n tcgen05.mma.cta_group::1.kind::f16.collector::a::fill [%0], %1, %2, "
@@ -99,13 +99,13 @@ template <bool F16, bool COLLECT>
 __device__ __forceinline__ void umma_split3(uint32_t dj, uint32_t dc, uint64_t ahi, uint64_t alo, uint64_t bhi,
                                             uint64_t blo, uint32_t acc_j, uint32_t acc_c) {
   if (F16 && COLLECT) {
-    umma_tf32<true, 1>(dj, ahi, bhi, acc_j);
-    umma_tf32<true, 3>(dc, ahi, blo, acc_c);
+    umma_hilo<true, 1>(dj, ahi, bhi, acc_j);
+    umma_hilo<true, 3>(dc, ahi, blo, acc_c);
   } else {
-    umma_tf32<F16>(dj, ahi, bhi, acc_j);
-    umma_tf32<F16>(dc, ahi, blo, acc_c);
+    umma_hilo<F16>(dj, ahi, bhi, acc_j);
+    umma_hilo<F16>(dc, ahi, blo, acc_c);
   }
-  umma_tf32<F16>(dc, alo, bhi, 1u);
+  umma_hilo<F16>(dc, alo, bhi, 1u);
 }
 // The paper's other kernels (L76-L78, NEXT-4) on the same contraction: with uncentred rows the
 // tensor cores deliver s^2 x . y; K = x.y, (gamma x.y + coef0)^degree or tanh(gamma x.y + coef0).
