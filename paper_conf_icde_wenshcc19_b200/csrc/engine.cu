@@ -1793,25 +1793,43 @@ static int engine_train_core(const float* X, const int32_t* y, int64_t n, int32_
   }
   std::vector<double> hb(Pl), hA(Pl), hB(Pl);
   std::vector<int32_t> h_sig(Pl), h_st(Pl), h_outer(Pl);
-  std::vector<int64_t> h_inner(Pl), h_cyc(Pl);
-  // the large read-backs (alpha, permutation, SV flags) land in pinned memory (async DMA)
-  // alpha stays on the device (the model's host copy is materialised on demand, ensure_host_alpha)
-  uint8_t* pin = pinned_scratch<uint8_t>((size_t)n * 8 + (size_t)n + 64, 1);
+  std::vector<int64_t> h_inner(Pl), h_cyc(Pl), h_body(Pl);
+  // every read-back lands in pinned memory (async DMA, one synchronisation; a copy into pageable
+  // memory would wait for the stream each time): the permutation, the SV flags and the per-pair
+  // results; alpha stays on the device (the model's host copy is materialised on demand,
+  // ensure_host_alpha)
+  const size_t o_flags = (size_t)n * 8, o_small = round_up((int64_t)(o_flags + (size_t)n), 8);
+  uint8_t* pin = pinned_scratch<uint8_t>(o_small + (size_t)Pl * (6 * 8 + 3 * 4) + 64, 1);
   int64_t* h_permp = reinterpret_cast<int64_t*>(pin);
-  uint8_t* h_flags = pin + (size_t)n * 8;
-  GM_CUDA(cudaMemcpyAsync(hb.data(), d_b.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(hA.data(), d_A.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(hB.data(), d_B.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_sig.data(), d_sig.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_st.data(), d_status.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_outer.data(), d_outer.get(), Pl * 4, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_inner.data(), d_inner.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
-  GM_CUDA(cudaMemcpyAsync(h_cyc.data(), d_cyc.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
+  uint8_t* h_flags = pin + o_flags;
+  uint8_t* sp = pin + o_small;
+  struct Rb {
+    void* host;
+    const void* dev;
+    size_t bytes;
+  };
+  const Rb rb[] = {{hb.data(), d_b.get(), (size_t)Pl * 8},         {hA.data(), d_A.get(), (size_t)Pl * 8},
+                   {hB.data(), d_B.get(), (size_t)Pl * 8},         {h_inner.data(), d_inner.get(), (size_t)Pl * 8},
+                   {h_cyc.data(), d_cyc.get(), (size_t)Pl * 8},    {h_body.data(), d_body.get(), (size_t)Pl * 8},
+                   {h_sig.data(), d_sig.get(), (size_t)Pl * 4},    {h_st.data(), d_status.get(), (size_t)Pl * 4},
+                   {h_outer.data(), d_outer.get(), (size_t)Pl * 4}};
+  {
+    size_t o = 0;
+    for (const Rb& r : rb) {
+      GM_CUDA(cudaMemcpyAsync(sp + o, r.dev, r.bytes, cudaMemcpyDeviceToHost, st));
+      o += r.bytes;
+    }
+  }
   GM_CUDA(cudaMemcpyAsync(h_permp, d_perm.get(), n * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaMemcpyAsync(h_flags, d_flags.get(), n, cudaMemcpyDeviceToHost, st));
-  std::vector<int64_t> h_body(Pl);
-  GM_CUDA(cudaMemcpyAsync(h_body.data(), d_body.get(), Pl * 8, cudaMemcpyDeviceToHost, st));
   GM_CUDA(cudaStreamSynchronize(st));
+  {
+    size_t o = 0;
+    for (const Rb& r : rb) {
+      std::memcpy(r.host, sp + o, r.bytes);
+      o += r.bytes;
+    }
+  }
   HT("fin_d2h");
   for (int g = 0; g < npg; ++g) {
     unsigned long long perr = 0;
